@@ -9,7 +9,7 @@ CPP_SRCS := $(wildcard $(CSRC)/*.cpp)
 HDRS     := $(wildcard $(CSRC)/*.cuh) $(wildcard $(CSRC)/*.h) include/bmr.h
 OBJS     := $(patsubst $(CSRC)/%.cu,build/%.o,$(CU_SRCS)) $(patsubst $(CSRC)/%.cpp,build/%.cpp.o,$(CPP_SRCS))
 
-all: gen/libbmrgen.so oracle/liboracle.so gen/libbmrgen_cuda.so
+all: gen/libbmrgen.so oracle/liboracle.so gen/libbmrgen_cuda.so $(PKG)/libbmr.so
 
 gen/libbmrgen.so: gen/gen_host.c gen/bmr_gen.h
 	gcc -O2 -fPIC -shared -Wall -Wextra -o $@ gen/gen_host.c -lpthread -lm
@@ -29,7 +29,7 @@ build/%.cpp.o: $(CSRC)/%.cpp $(HDRS)
 	$(NVCC) -O2 -std=c++17 -Xcompiler -fPIC -Iinclude -c -o $@ $<
 
 $(PKG)/libbmr.so: $(OBJS)
-	$(NVCC) $(ARCH) -shared -o $@ $(OBJS) -lcudart
+	$(NVCC) $(ARCH) -shared --cudart static -o $@ $(OBJS)
 
 clean:
 	rm -rf build gen/*.so oracle/*.so $(PKG)/*.so

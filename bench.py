@@ -1,0 +1,379 @@
+#!/usr/bin/env python
+"""bench.py — libbmr hot-path benchmark (BASELINE.json metric: Map+Group+Reduce input GB/s and
+% HBM roofline, vs the CPU oracle).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C5|C4|C3|C2|C1] [--impl reference]
+
+One step = one pass of the whole hot path (tile scheduling, stage-in,
+user map, emit, flush, digit histogram, onesweep passes, segment boundaries, reduce + output
+assembly) over one shard of synthetic input already resident in HBM.  Default workload = C5
+(WordCount, Zipf V=1M, 8 GiB per GPU, weak scaling): the configuration the metric's
+"1/2/4/8 B200" is quoted on that exercises every row (C2 StringMatch is Map-only).
+Prints ONE JSON line on rank 0.  Timing: W warm-up steps, then K steps bracketed by barrier +
+cuda.synchronize, CUDA events on the job stream, max over ranks.  Inputs (8 GiB) exceed L2
+(126 MB), so no extra flush is needed.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+WORKLOADS = {
+    # name: (workload, description, pages-or-points per GPU)
+    "C1": ("wc", "WordCount 1 MiB Zipf text, V=10k", 1),
+    "C2": ("sm", "StringMatch 4 GiB text, 16-byte pattern", 4096),
+    "C3": ("km", "KMeans one Lloyd step, 64M x 8 fp32, k=32", 64 << 20),
+    "C4": ("ii", "InvertedIndex 8 GiB HTML-like", 8192),
+    "C5": ("wc", "WordCount 8 GiB/GPU Zipf text, V=1M (weak)", 8192),
+}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+def spec_for(cfg):
+    from gen import pygen
+    if cfg == "C1":
+        return pygen.spec_wc(10_000, 1)
+    if cfg == "C2":
+        return pygen.spec_sm(1000, 2)
+    if cfg == "C4":
+        return pygen.spec_ii(4)
+    if cfg == "C5":
+        return pygen.spec_wc(1_000_000, 5)
+    return pygen.KMSpec()
+
+
+# ------------------------------------------------------------------ clocks (NVML, during timing)
+class ClockSampler:
+    REASONS = {0x4: "sw_power_cap", 0x8: "hw_slowdown", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown", 0x2: "applications_clocks_setting"}
+
+    def __init__(self, dev):
+        self.samples, self.reasons, self.stop_ev = [], set(), threading.Event()
+        self.max_mhz = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(dev)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+        self.t = threading.Thread(target=self._run, daemon=True)
+
+    def _run(self):
+        while not self.stop_ev.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.05)
+
+    def __enter__(self):
+        if self.nv:
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self.stop_ev.set()
+        if self.nv:
+            self.t.join()
+
+    def summary(self):
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------ inputs
+def make_input(cfg, rank, dev):
+    """Device-resident synthetic shard of rank `rank` (weak scaling: global units r*P..)."""
+    from gen import pygen
+    wl, _, units = WORKLOADS[cfg]
+    spec = spec_for(cfg)
+    if wl == "km":
+        pts = pygen.device_km(spec, units, i0=rank * units, device=dev)
+        _, init = pygen.km_centres(spec)
+        return {"wl": wl, "data": pts.view(-1).view(__import__("torch").uint8), "offsets": None, "n": units,
+                "nbytes": units * 32, "centroids": init, "spec": spec, "page0": rank * units}
+    g = pygen.device_text(spec, units, page0=rank * units, device=dev)
+    return {"wl": wl, "data": g["data"], "offsets": g["offsets"], "n": g["n"], "nbytes": units * spec.page_bytes,
+            "spec": spec, "page0": rank * units, "base": g["base"]}
+
+
+def job_kwargs(inp, flags=0, device=0):
+    kw = {"device": device, "flags": flags}
+    if inp["wl"] == "sm":
+        kw["pattern"] = inp["spec"].pattern
+    if inp["wl"] == "km":
+        kw["centroids"] = inp["centroids"]
+    if inp["wl"] in ("sm", "ii"):
+        kw["input_base"] = inp.get("base", 0)
+    return kw
+
+
+# ------------------------------------------------------------------ CPU oracle (baseline / reference arm)
+def oracle_sample(cfg, sample_units, page0=0):
+    """Time the oracle (as it stands) on the first `sample_units` pages/points of rank 0's shard."""
+    from gen import pygen
+    from oracle import oracle
+    wl = WORKLOADS[cfg][0]
+    spec = spec_for(cfg)
+    if wl == "km":
+        pts = pygen.host_km(spec, sample_units, i0=page0)
+        _, init = pygen.km_centres(spec)
+        data = pts.view(np.uint8).reshape(-1)
+        t0 = time.perf_counter()
+        oracle.run("km", [(data, None, sample_units, 32, 0)], centroids=init)
+        dt = time.perf_counter() - t0
+        return data.size, dt, f"first {sample_units} points ({data.size / 2**20:.0f} MiB) of the shard"
+    g = pygen.host_text(spec, sample_units, page0=page0)
+    kw = {"pattern": spec.pattern} if wl == "sm" else {}
+    t0 = time.perf_counter()
+    oracle.run(wl, [(g["data"], g["offsets"], g["n"], 0, g["base"])], **kw)
+    dt = time.perf_counter() - t0
+    return g["data"].size, dt, f"first {sample_units} pages ({sample_units} MiB) of the shard"
+
+
+ORACLE_SAMPLE = {"C1": 1, "C2": 48, "C3": 4 << 20, "C4": 96, "C5": 96}   # ~10-30 s of CPU work
+REF_STEP_SAMPLE = {"C1": 1, "C2": 4, "C3": 1 << 19, "C4": 8, "C5": 8}     # per reference-arm step
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    cfg = args.workload
+    su = REF_STEP_SAMPLE[cfg]
+    for _ in range(args.warmup):
+        oracle_sample(cfg, su)
+    times = []
+    nb = 0
+    desc = ""
+    for _ in range(args.steps):
+        nb, dt, desc = oracle_sample(cfg, su)
+        times.append(dt)
+    ms = 1000.0 * sum(times) / len(times)
+    val = nb / (ms / 1000.0) / 1e9
+    line = {"impl": "reference", "metric": "Map+Group+Reduce input GB/s (CPU oracle)", "value": round(val, 6),
+            "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(ms, 3), "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "u8" if WORKLOADS[cfg][0] != "km" else "f32", "data": "synthetic",
+            "config": {"workload": cfg, "description": WORKLOADS[cfg][1], "sample": desc},
+            "cpu_baseline": {"value": round(val, 6), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": desc},
+            "e2e": {"value": round(val, 6), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ GPU arm
+def algorithmic(inp, st, steps):
+    """Algorithmic bytes per step of each phase."""
+    wl = inp["wl"]
+    m = st["pairs"] / steps
+    n = inp["n"]
+    pair_bytes = {"wc": 20, "sm": 8, "km": 40, "ii": 24}[wl]
+    map_b = inp["nbytes"] + (8 * (n + 1) if inp["offsets"] is not None else 0) + m * pair_bytes
+    passes = st["sort_passes"] / steps
+    sort_b = (passes * 24 - 4) * m if passes else 0.0   # first pass reads no payload
+    return {"map": map_b, "hist": 8 * m, "sort": sort_b, "passes": passes, "pairs": m}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default="C5", choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="bmr", choices=["bmr", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ipps_jim11_b200 as bmr
+
+    torch.cuda.set_device(local)
+    dev = f"cuda:{local}"
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device(dev))
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    inp = make_input(args.workload, rank, dev)
+    torch.cuda.synchronize()
+    job = bmr.Job(inp["wl"], **job_kwargs(inp, bmr.FLAG_PROFILE, local))
+    stream = torch.cuda.current_stream()
+
+    def step():
+        job.reset()
+        job.map(inp["data"], inp["offsets"], inp["n"])
+        job.group()
+        job.reduce()
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    job.fetch()
+    barrier()
+    job.reset()
+    # timed region: K steps, per-phase device times from the job's CUDA events
+    acc = {k: 0.0 for k in ("map_ms", "hist_ms", "sort_ms", "seg_ms")}
+    tot = {"pairs": 0, "sort_passes": 0, "kernel_launches": 0, "flushes": 0, "n_keys": 0}
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        barrier()
+        t0 = time.perf_counter()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            step()
+            s = job.stats()  # map/hist/sort/seg events are collected at mr_group's synchronisation
+            for k in tot:
+                tot[k] += s[k]
+            for k in acc:
+                acc[k] += s[k]
+        ev1.record(stream)
+        ev1.synchronize()
+        wall = time.perf_counter() - t0
+        barrier()
+    ms = ev0.elapsed_time(ev1) / args.steps
+    t = torch.tensor([ms], device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max = float(t.item())
+    # reduce-phase events are collected at mr_fetch: one extra (untimed) pass of K steps
+    red = 0.0
+    for _ in range(args.steps):
+        step()
+        job.fetch()
+        red += job.stats()["reduce_ms"]
+    per = {k: v / args.steps for k, v in acc.items()}
+    per["reduce_ms"] = red / args.steps
+    alg = algorithmic(inp, tot, args.steps)
+    hbm, peak_kind = load_peaks()
+    sort_launch_ms = per["sort_ms"] / max(alg["passes"], 1)
+    sort_launch_bytes = alg["sort"] / max(alg["passes"], 1)
+    roof = None
+    if alg["passes"]:
+        ach = sort_launch_bytes / (sort_launch_ms / 1e3) / 1e9
+        roof = {"kernel": "k_onesweep (LSD pass)", "bound": "hbm", "achieved": round(ach, 1), "peak": hbm,
+                "peak_kind": peak_kind, "unit": "GB/s", "frac": round(ach / hbm, 4), "traffic": None,
+                "bytes_per_launch": int(sort_launch_bytes), "ms_per_launch": round(sort_launch_ms, 4)}
+    map_ach = alg["map"] / (per["map_ms"] / 1e3) / 1e9 if per["map_ms"] else 0.0
+    traffic_p = os.path.join(ROOT, "profiles", "traffic.json")
+    if roof and os.path.exists(traffic_p):
+        tr = json.load(open(traffic_p)).get(args.workload, {}).get("k_onesweep")
+        if tr:
+            roof["traffic"] = tr
+    if roof is None:   # Map-only (SM) or single-digit sort: the Map kernel dominates
+        roof = {"kernel": "k_map", "bound": "hbm", "achieved": round(map_ach, 1), "peak": hbm,
+                "peak_kind": peak_kind, "unit": "GB/s", "frac": round(map_ach / hbm, 4), "traffic": None,
+                "bytes_per_launch": int(alg["map"]), "ms_per_launch": round(per["map_ms"], 4)}
+
+    nbytes_all = inp["nbytes"] * world
+    value = nbytes_all / (ms_max / 1e3) / 1e9
+
+    # ---- end to end: host buffers through mr_map_host, H2D + D2H inside the timed region
+    e2e = None
+    if args.e2e_steps > 0:
+        h_data = torch.empty(inp["data"].numel(), dtype=torch.uint8, pin_memory=True)
+        h_data.copy_(inp["data"])
+        h_off = None
+        if inp["offsets"] is not None:
+            h_off = torch.empty(inp["offsets"].numel(), dtype=torch.int64, pin_memory=True)
+            h_off.copy_(inp["offsets"])
+        torch.cuda.synchronize()
+        job_e = bmr.Job(inp["wl"], **job_kwargs(inp, 0, local))
+        d2h = 0
+
+        def estep():
+            job_e.reset()
+            job_e.map_host(h_data.numpy(), None if h_off is None else h_off.numpy().view(np.uint64), inp["n"])
+            job_e.group()
+            job_e.reduce()
+            r = job_e.fetch()
+            return r["keys"].nbytes + r["vals"].nbytes + r["key_offsets"].nbytes + r["val_offsets"].nbytes
+
+        estep()
+        barrier()
+        t0 = time.perf_counter()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.e2e_steps):
+            d2h = estep()
+        e1.record(stream)
+        e1.synchronize()
+        ems = max(e0.elapsed_time(e1), (time.perf_counter() - t0) * 1e3) / args.e2e_steps
+        te = torch.tensor([ems], device=dev)
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        ems = float(te.item())
+        h2d = inp["nbytes"] + (8 * (inp["n"] + 1) if h_off is not None else 0)
+        e2e = {"value": round(nbytes_all / (ems / 1e3) / 1e9, 3), "unit": "GB/s", "ms_per_step": round(ems, 3),
+               "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h), "api": "mr_map_host+mr_fetch"}
+        job_e.close()
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        su = ORACLE_SAMPLE[args.workload]
+        nb, dt, desc = oracle_sample(args.workload, su)
+        cpu = {"value": round(nb / dt / 1e9, 6), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": desc,
+               "seconds": round(dt, 2)}
+
+    if rank == 0:
+        wl = inp["wl"]
+        line = {
+            "metric": "Map+Group+Reduce input GB/s", "value": round(value, 3), "unit": "GB/s",
+            "n_gpus": world, "steps": args.steps, "warmup": max(3, args.warmup), "ms_per_step": round(ms_max, 3),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "f32" if wl == "km" else "u8", "data": "synthetic",
+            "config": {"workload": args.workload, "description": WORKLOADS[args.workload][1],
+                       "input_bytes_per_gpu": inp["nbytes"], "records_per_gpu": inp["n"],
+                       "l2": "inputs larger than L2 (no flush needed)", "parallelism": f"dp{world}"},
+            "records_per_s": round(inp["n"] * world / (ms_max / 1e3), 1),
+            "hbm_frac_end_to_end": round((alg["map"] + alg["hist"] + alg["sort"]) / (ms_max / 1e3) / 1e9 / hbm, 4),
+            "phases_ms": {k[:-3]: round(v, 3) for k, v in per.items()},
+            "map": {"achieved_gbs": round(map_ach, 1), "frac": round(map_ach / hbm, 4),
+                    "bytes_per_step": int(alg["map"])},
+            "pairs_per_step": int(alg["pairs"]), "sort_passes": alg["passes"],
+            "distinct_keys": int(tot["n_keys"] / args.steps),
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+            "gpu_launches": int(tot["kernel_launches"]),
+            "clocks": clk.summary(), "wall_s_timed": round(wall, 3),
+        }
+        print(json.dumps(line), flush=True)
+    job.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,153 @@
+/* bmr.h — C ABI of libbmr, a B200-native (sm_100a) implementation of the data-parallel hot
+ * path of Ji & Ma, "Using Shared Memory to Accelerate MapReduce on GPUs" (IPDPS 2011):
+ * Map (stage-in -> user map -> emit -> flush) -> group-by-key (hash + LSD radix sort + segment
+ * boundaries) -> Reduce.
+ *
+ * Citations: "L<n>" = line n of the paper text (reference PAPER.md); "§8(x)" = SURVEY.md.
+ *
+ * Data model (L51-52 "Input, intermediate, and output are all in the format of <key, value>
+ * pairs"; L85 key/value index arrays; L36 "no assumption on input/output data sizes, size
+ * variations, or record counts"): an input batch is `records` (bytes) + `offsets` (n+1 u64;
+ * record i is records[offsets[i], offsets[i+1])) or fixed-stride records.  The record index is
+ * the implicit input value (Table II, 4-byte input value).
+ *
+ * Threading: a job is used by one host thread at a time; distinct jobs are independent.
+ * Errors: every call returns an mr_status; nothing aborts, exits or throws across the ABI.
+ * Asynchronous device faults surface as MR_ERR_CUDA at the next synchronising call
+ * (mr_map for text batches, mr_group, mr_fetch); mr_last_error() gives the detail.
+ */
+#ifndef BMR_H
+#define BMR_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MR_ABI_VERSION 1
+
+typedef struct mr_job mr_job; /* opaque; owned by the library */
+
+typedef enum {
+  MR_OK = 0,
+  MR_ERR_INVALID = 1,     /* bad argument (NULL, abi_version, k, dim, alignment, ...) */
+  MR_ERR_STATE = 2,       /* call out of order (see state machine below) */
+  MR_ERR_OOM = 3,         /* device cannot hold the demanded intermediate / output */
+  MR_ERR_OVERFLOW = 4,    /* an emitted key exceeds 65535 bytes; the batch is rejected */
+  MR_ERR_CUDA = 5,        /* CUDA runtime / kernel error (detail in mr_last_error) */
+  MR_ERR_NCCL = 6,        /* collective failure (multi-GPU) */
+  MR_ERR_UNSUPPORTED = 7  /* e.g. >= 2^32 intermediate pairs in one group */
+} mr_status;
+
+/* Workloads (L125): compiled-in device functors. */
+typedef enum { MR_WORDCOUNT = 1, MR_STRINGMATCH = 2, MR_KMEANS = 3, MR_INVINDEX = 4 } mr_workload;
+
+/* Flags */
+#define MR_FLAG_NO_SMEM_IN      0x01u /* reserved: SO ablation (L134) */
+#define MR_FLAG_NO_SMEM_OUT     0x02u /* reserved: SI ablation (L135) */
+#define MR_FLAG_FORCE_TINY_OUT  0x04u /* output half = one warp result: every warp result overflows (L113) */
+#define MR_FLAG_WEAK_HASH_DEBUG 0x08u /* 4-bit key hash: forces collisions, exercises verification */
+#define MR_FLAG_VALIDATE        0x10u /* host-side argument validation of offsets (reads them back) */
+#define MR_FLAG_NO_COMBINE      0x20u /* multi-GPU: exchange raw pairs (no combiner) */
+#define MR_FLAG_PROFILE         0x40u /* record CUDA events per phase on the job stream (mr_stats *_ms) */
+
+typedef struct { uint8_t pattern[16]; } mr_sm_params;                      /* StringMatch */
+typedef struct { uint32_t k, dim; const float* centroids; } mr_km_params;  /* KMeans: host ptr, k x dim fp32, dim == 8, 1 <= k <= 1024 */
+
+typedef struct {
+  uint32_t abi_version;      /* must equal MR_ABI_VERSION */
+  mr_workload workload;
+  int device;                /* CUDA ordinal; made current on every call */
+  void* stream;              /* cudaStream_t to enqueue on; NULL = job-owned stream */
+  uint32_t record_stride;    /* 0: variable-size records (offsets required); KM: 32 */
+  const void* params;        /* mr_sm_params* / mr_km_params* / NULL; copied at create */
+  uint64_t input_base;       /* global byte offset of this rank's first record (SM/II offsets are global) */
+  int rank, nranks;          /* nranks == 1: single GPU */
+  void* nccl_comm;           /* ncclComm_t (multi-GPU; reserved in ABI v1) */
+  uint64_t max_pairs_hint;   /* initial intermediate capacity in pairs (0: heuristic) */
+  uint64_t heap_bytes_hint;  /* reserved */
+  uint32_t flags;            /* MR_FLAG_* */
+} mr_config;
+
+/* Job-owned host memory, valid until the next mr_* call on the job or mr_job_destroy.
+ *   WC: key = word bytes,        val = u64 count                       (L125 "number of occurrences")
+ *   SM: key = u64 global offset, val = empty    (Map-only; one entry per match, overlaps counted)
+ *   KM: key = u32 cluster id,    val = 8 x fp32 new centroid || u64 count (all k clusters)
+ *   II: key = URL bytes,         val = u64[] global offsets of the URL (L125 "link's position")
+ * Key order is unspecified (hash order); callers canonicalise. */
+typedef struct {
+  uint64_t n_keys;
+  const uint8_t* keys; const uint64_t* key_offsets; /* n_keys + 1 */
+  const uint8_t* vals; const uint64_t* val_offsets; /* n_keys + 1 */
+} mr_result;
+
+typedef struct {
+  uint64_t pairs;          /* intermediate pairs emitted by Map (M) */
+  uint64_t flushes;        /* SMEM output-half flushes (one global atomic each, L113) */
+  uint64_t replays;        /* batches replayed after capacity growth */
+  uint64_t n_keys;         /* distinct keys (S) */
+  uint64_t collisions;     /* hashed-key mismatches found by verification (then re-sorted) */
+  uint64_t sort_passes;    /* LSD passes executed (constant digits skipped) */
+  uint64_t map_tiles;      /* input tiles staged by the producer warps */
+  uint64_t input_bytes;    /* record bytes mapped */
+  uint64_t capacity_pairs; /* current intermediate capacity */
+  uint64_t kernel_launches;/* libbmr kernels launched since create / reset */
+  /* MR_FLAG_PROFILE: device time per phase (CUDA events on the job stream), ms */
+  double map_ms, hist_ms, sort_ms, seg_ms, reduce_ms;
+} mr_stats;
+
+/* State machine: CREATED -> mr_map x k (batches append) -> mr_group -> mr_reduce -> mr_fetch
+ * (-> mr_job_reset -> CREATED, keeping device buffers).  Out of order -> MR_ERR_STATE.
+ * SM (Map-only): mr_group and mr_reduce are valid no-ops. */
+
+/* Create a job.  Copies cfg and params.  Allocates nothing large until the first mr_map. */
+mr_status mr_job_create(const mr_config* cfg, mr_job** out);
+
+/* Map one batch of DEVICE-resident records (§8(a) a1-a5).
+ *   records: device bytes.  Keys are emitted BY REFERENCE into records (L110 "addressable
+ *            place"), so every mapped batch must stay alive and unmodified until mr_reduce has
+ *            completed.  KM (record_stride 32) requires 16-byte aligned records.
+ *   offsets: device, n+1 u64, offsets[0] == 0, non-decreasing, offsets[n] = batch length;
+ *            NULL iff record_stride > 0 (then record i = records[i*stride, (i+1)*stride)).
+ *   n:       number of records (0 allowed).
+ * Text batches read offsets[n] back to the host (8 bytes, synchronising the stream) to size
+ * the launch; fixed-stride batches are fully asynchronous.  Global byte offsets emitted by
+ * SM/II are input_base + (sum of earlier batch lengths) + in-batch offset. */
+mr_status mr_map(mr_job* job, const uint8_t* records, const uint64_t* offsets, uint64_t n);
+
+/* Same as mr_map for HOST buffers: the library copies records/offsets into job-owned device
+ * memory on the job stream (the end-to-end path of bench.py). */
+mr_status mr_map_host(mr_job* job, const uint8_t* records, const uint64_t* offsets, uint64_t n);
+
+/* Group by key (§8(a) a6-a8): capacity check (grow + replay on overflow), digit histogram,
+ * onesweep LSD passes over non-constant digits, segment boundaries with byte verification of
+ * hashed keys (re-sort with a fresh hash on collision).  Synchronises the stream. */
+mr_status mr_group(mr_job* job);
+
+/* Reduce (§8(a) a9) and device-side output assembly.  Asynchronous. */
+mr_status mr_reduce(mr_job* job);
+
+/* Copy the output to job-owned pinned host memory; synchronises.  *out valid until the next
+ * call on the job. */
+mr_status mr_fetch(mr_job* job, mr_result* out);
+
+/* Back to CREATED, keeping every device buffer (repeated runs without reallocation). */
+mr_status mr_job_reset(mr_job* job);
+
+/* Fill min(bytes, sizeof(mr_stats)) bytes of an mr_stats. */
+mr_status mr_get_stats(const mr_job* job, void* stats, size_t bytes);
+
+mr_status mr_job_destroy(mr_job* job); /* NULL-safe */
+const char* mr_status_string(mr_status s);
+const char* mr_last_error(const mr_job* job);
+
+/* Group-by primitive exposed for testing (§8(a) a7): stable LSD radix sort of n u64 device
+ * keys; writes the sorted keys and the u32 permutation (perm[i] = source index of the i-th
+ * key).  Synchronises `stream`. n < 2^32. */
+mr_status mr_sort_u64(const uint64_t* keys, uint64_t* keys_out, uint32_t* perm_out, uint64_t n, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BMR_H */

@@ -1,0 +1,229 @@
+"""paper_conf_ipps_jim11_b200 — thin Python binding of libbmr (include/bmr.h).
+
+Argument marshalling only: every step of Map -> group-by-key -> Reduce runs in the CUDA
+kernels of ``libbmr.so`` (sm_100a).  PyTorch is used by callers for device memory and streams;
+this module accepts torch CUDA tensors (or raw device pointers) and numpy arrays for the host
+entry point.  There is no CPU fallback: if ``libbmr.so`` is missing or no CUDA device is
+present, calls raise.
+
+Names follow the C ABI: ``Job.map`` = ``mr_map``, ``Job.group`` = ``mr_group``, ...
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libbmr.so")
+
+MR_ABI_VERSION = 1
+WORDCOUNT, STRINGMATCH, KMEANS, INVINDEX = 1, 2, 3, 4
+WORKLOADS = {"wc": WORDCOUNT, "sm": STRINGMATCH, "km": KMEANS, "ii": INVINDEX}
+FLAG_NO_SMEM_IN, FLAG_NO_SMEM_OUT, FLAG_FORCE_TINY_OUT = 0x01, 0x02, 0x04
+FLAG_WEAK_HASH_DEBUG, FLAG_VALIDATE, FLAG_NO_COMBINE = 0x08, 0x10, 0x20
+FLAG_PROFILE = 0x40
+
+STATUS = {0: "MR_OK", 1: "MR_ERR_INVALID", 2: "MR_ERR_STATE", 3: "MR_ERR_OOM", 4: "MR_ERR_OVERFLOW",
+          5: "MR_ERR_CUDA", 6: "MR_ERR_NCCL", 7: "MR_ERR_UNSUPPORTED"}
+
+EXPORTS = ("mr_job_create", "mr_map", "mr_map_host", "mr_group", "mr_reduce", "mr_fetch", "mr_job_reset",
+           "mr_get_stats", "mr_job_destroy", "mr_status_string", "mr_last_error", "mr_sort_u64")
+
+
+class MRError(RuntimeError):
+    def __init__(self, status: int, detail: str = ""):
+        self.status = status
+        super().__init__(f"{STATUS.get(status, status)}: {detail}")
+
+
+class Config(C.Structure):
+    _fields_ = [("abi_version", C.c_uint32), ("workload", C.c_int), ("device", C.c_int), ("stream", C.c_void_p),
+                ("record_stride", C.c_uint32), ("params", C.c_void_p), ("input_base", C.c_uint64),
+                ("rank", C.c_int), ("nranks", C.c_int), ("nccl_comm", C.c_void_p),
+                ("max_pairs_hint", C.c_uint64), ("heap_bytes_hint", C.c_uint64), ("flags", C.c_uint32)]
+
+
+class SMParams(C.Structure):
+    _fields_ = [("pattern", C.c_uint8 * 16)]
+
+
+class KMParams(C.Structure):
+    _fields_ = [("k", C.c_uint32), ("dim", C.c_uint32), ("centroids", C.c_void_p)]
+
+
+class Result(C.Structure):
+    _fields_ = [("n_keys", C.c_uint64), ("keys", C.c_void_p), ("key_offsets", C.c_void_p),
+                ("vals", C.c_void_p), ("val_offsets", C.c_void_p)]
+
+
+class Stats(C.Structure):
+    _fields_ = [(n, C.c_uint64) for n in ("pairs", "flushes", "replays", "n_keys", "collisions", "sort_passes",
+                                          "map_tiles", "input_bytes", "capacity_pairs", "kernel_launches")] + \
+               [(n, C.c_double) for n in ("map_ms", "hist_ms", "sort_ms", "seg_ms", "reduce_ms")]
+
+
+_LIB = None
+
+
+def lib() -> C.CDLL:
+    """Load libbmr.so (fails loudly if it was not built)."""
+    global _LIB
+    if _LIB is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} not built: run __graft_entry__.build()")
+        L = C.CDLL(LIB_PATH)
+        vp, u64 = C.c_void_p, C.c_uint64
+        L.mr_job_create.argtypes = [C.POINTER(Config), C.POINTER(vp)]
+        L.mr_map.argtypes = [vp, vp, vp, u64]
+        L.mr_map_host.argtypes = [vp, vp, vp, u64]
+        for f in ("mr_group", "mr_reduce", "mr_job_reset", "mr_job_destroy"):
+            getattr(L, f).argtypes = [vp]
+        L.mr_fetch.argtypes = [vp, C.POINTER(Result)]
+        L.mr_get_stats.argtypes = [vp, vp, C.c_size_t]
+        L.mr_status_string.argtypes = [C.c_int]
+        L.mr_status_string.restype = C.c_char_p
+        L.mr_last_error.argtypes = [vp]
+        L.mr_last_error.restype = C.c_char_p
+        L.mr_sort_u64.argtypes = [vp, vp, vp, u64, vp]
+        for f in EXPORTS:
+            if f not in ("mr_status_string", "mr_last_error"):
+                getattr(L, f).restype = C.c_int
+        _LIB = L
+    return _LIB
+
+
+def _ptr(x) -> int:
+    if x is None:
+        return 0
+    if isinstance(x, int):
+        return x
+    if hasattr(x, "data_ptr"):
+        return int(x.data_ptr())
+    if isinstance(x, np.ndarray):
+        return int(x.ctypes.data)
+    raise TypeError(type(x))
+
+
+def _copy(addr, nbytes, dtype=np.uint8):
+    if nbytes == 0:
+        return np.zeros(0, dtype)
+    return np.frombuffer((C.c_uint8 * nbytes).from_address(addr), np.uint8).copy().view(dtype)
+
+
+class Job:
+    """One MapReduce job (mr_job).  ``workload`` in {"wc", "sm", "km", "ii"}."""
+
+    def __init__(self, workload: str, device: int = 0, stream=None, pattern: bytes | None = None,
+                 centroids: np.ndarray | None = None, input_base: int = 0, flags: int = 0,
+                 max_pairs_hint: int = 0):
+        L = lib()
+        self.workload = workload
+        cfg = Config()
+        cfg.abi_version = MR_ABI_VERSION
+        cfg.workload = WORKLOADS[workload]
+        cfg.device = device
+        if stream is None:
+            import torch
+            stream = torch.cuda.current_stream(device).cuda_stream
+        cfg.stream = stream
+        cfg.input_base = input_base
+        cfg.rank, cfg.nranks = 0, 1
+        cfg.max_pairs_hint = max_pairs_hint
+        cfg.flags = flags
+        self._keep = []
+        if workload == "sm":
+            p = SMParams()
+            for i, b in enumerate(pattern[:16]):
+                p.pattern[i] = b
+            cfg.params = C.addressof(p)
+            self._keep.append(p)
+        elif workload == "km":
+            cen = np.ascontiguousarray(centroids, np.float32)
+            p = KMParams(cen.shape[0], cen.shape[1], cen.ctypes.data)
+            cfg.params = C.addressof(p)
+            cfg.record_stride = 32
+            self._keep += [p, cen]
+        h = C.c_void_p()
+        self._check(L.mr_job_create(C.byref(cfg), C.byref(h)), None)
+        self.h = h
+
+    def _check(self, rc, h=-1):
+        if rc != 0:
+            hh = self.h if h == -1 else h
+            detail = lib().mr_last_error(hh).decode() if hh else ""
+            raise MRError(rc, detail)
+
+    def map(self, records, offsets=None, n: int | None = None):
+        """mr_map over device records (torch uint8 CUDA tensor or pointer); offsets: int64 tensor
+        holding the n+1 u64 offsets (None for KM)."""
+        if n is None:
+            n = (offsets.numel() - 1) if offsets is not None else records.numel() // 32
+        self._check(lib().mr_map(self.h, _ptr(records), _ptr(offsets), n))
+
+    def map_host(self, records: np.ndarray, offsets: np.ndarray | None = None, n: int | None = None):
+        if n is None:
+            n = (len(offsets) - 1) if offsets is not None else records.size // 32
+        self._check(lib().mr_map_host(self.h, _ptr(records), _ptr(offsets), n))
+
+    def group(self):
+        self._check(lib().mr_group(self.h))
+
+    def reduce(self):
+        self._check(lib().mr_reduce(self.h))
+
+    def fetch(self) -> dict:
+        r = Result()
+        self._check(lib().mr_fetch(self.h, C.byref(r)))
+        n = int(r.n_keys)
+        ko = _copy(r.key_offsets, 8 * (n + 1), np.uint64)
+        vo = _copy(r.val_offsets, 8 * (n + 1), np.uint64)
+        return {"n_keys": n, "keys": _copy(r.keys, int(ko[-1])), "key_offsets": ko,
+                "vals": _copy(r.vals, int(vo[-1])), "val_offsets": vo}
+
+    def run(self, *batches) -> dict:
+        for b in batches:
+            self.map(*b)
+        self.group()
+        self.reduce()
+        return self.fetch()
+
+    def reset(self):
+        self._check(lib().mr_job_reset(self.h))
+
+    def stats(self) -> dict:
+        s = Stats()
+        self._check(lib().mr_get_stats(self.h, C.byref(s), C.sizeof(s)))
+        return {n: (float(getattr(s, n)) if t is C.c_double else int(getattr(s, n))) for n, t in Stats._fields_}
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().mr_job_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+
+def sort_u64(keys, stream=None):
+    """mr_sort_u64 on an int64 CUDA tensor (u64 bit patterns): returns (sorted keys, perm int32)."""
+    import torch
+    n = keys.numel()
+    out = torch.empty_like(keys)
+    perm = torch.empty(n, dtype=torch.int32, device=keys.device)
+    if stream is None:
+        stream = torch.cuda.current_stream(keys.device).cuda_stream
+    rc = lib().mr_sort_u64(_ptr(keys), _ptr(out), _ptr(perm), n, stream)
+    if rc:
+        raise MRError(rc, "mr_sort_u64")
+    return out, perm

@@ -1,0 +1,695 @@
+// api.cpp — the libbmr C ABI (include/bmr.h) and the host job runtime: state machine, buffer
+// sizing, overflow detection + replay, sort-pass planning, output assembly and fetch.
+// Every computational step runs in the CUDA kernels of map.cu / sort.cu / reduce.cu; this file
+// only orchestrates launches on the job stream.  There is no CPU fallback: without a CUDA
+// device every call that needs one fails with MR_ERR_CUDA.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "bmr.h"
+#include "kernels.h"
+
+using namespace bmr;
+
+std::atomic<unsigned long long> bmr::g_kernel_launches{0};
+
+namespace {
+
+enum State { kCreated = 0, kMapped = 1, kGrouped = 2, kReduced = 3 };
+
+template <typename T>
+struct DBuf {
+  T* p = nullptr;
+  uint64_t n = 0;
+  cudaError_t ensure(uint64_t need) {
+    if (need <= n && p) return cudaSuccess;
+    release();
+    const uint64_t cnt = std::max<uint64_t>(need, 1);
+    cudaError_t e = cudaMalloc(reinterpret_cast<void**>(&p), cnt * sizeof(T));
+    if (e != cudaSuccess) { p = nullptr; n = 0; cudaGetLastError(); return e; }
+    n = cnt;
+    return cudaSuccess;
+  }
+  void release() { if (p) cudaFree(p); p = nullptr; n = 0; }
+};
+
+template <typename T>
+struct HBuf {  // pinned host
+  T* p = nullptr;
+  uint64_t n = 0;
+  cudaError_t ensure(uint64_t need) {
+    if (need <= n && p) return cudaSuccess;
+    release();
+    const uint64_t cnt = std::max<uint64_t>(need, 1);
+    cudaError_t e = cudaMallocHost(reinterpret_cast<void**>(&p), cnt * sizeof(T));
+    if (e != cudaSuccess) { p = nullptr; n = 0; cudaGetLastError(); return e; }
+    n = cnt;
+    return cudaSuccess;
+  }
+  void release() { if (p) cudaFreeHost(p); p = nullptr; n = 0; }
+};
+
+// MR_FLAG_PROFILE: CUDA events around each phase on the job stream; elapsed times are
+// collected at the next synchronisation point.
+struct Prof {
+  struct Span { cudaEvent_t a, b; double* acc; };
+  std::vector<cudaEvent_t> pool;
+  std::vector<Span> open;
+  size_t used = 0;
+  bool on = false;
+  cudaEvent_t get() {
+    if (used == pool.size()) {
+      cudaEvent_t e;
+      cudaEventCreate(&e);
+      pool.push_back(e);
+    }
+    return pool[used++];
+  }
+  void begin(cudaStream_t s, Span& sp) { sp.a = get(); cudaEventRecord(sp.a, s); }
+  void end(cudaStream_t s, Span& sp, double* acc) {
+    sp.b = get();
+    cudaEventRecord(sp.b, s);
+    sp.acc = acc;
+    open.push_back(sp);
+  }
+  void collect() {  // call after the stream was synchronised
+    for (auto& sp : open) {
+      float ms = 0;
+      if (cudaEventElapsedTime(&ms, sp.a, sp.b) == cudaSuccess) *sp.acc += ms;
+    }
+    cudaGetLastError();
+    open.clear();
+    used = 0;
+  }
+  void release() { for (auto e : pool) cudaEventDestroy(e); pool.clear(); open.clear(); used = 0; }
+};
+
+struct Batch {
+  const uint8_t* rec;
+  const uint64_t* off;
+  uint64_t n, nbytes, gbase;
+};
+
+// Sort workspace shared by mr_group and mr_sort_u64.
+struct SortWork {
+  DBuf<uint64_t> ka, kb, status;
+  DBuf<uint32_t> ia, ib, hist, bases;
+  HBuf<uint32_t> hist_h, bases_h;
+  uint32_t epoch = 1;
+  uint64_t passes = 0;
+  void release() { ka.release(); kb.release(); status.release(); ia.release(); ib.release(); hist.release(); bases.release(); hist_h.release(); bases_h.release(); }
+};
+
+__global__ void k_iota_u32(uint32_t* p, uint64_t n) {
+  const uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (i < n) p[i] = static_cast<uint32_t>(i);
+}
+
+int sm_count(int dev) {
+  int v = 148;
+  if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) { cudaGetLastError(); v = 148; }
+  return v;
+}
+
+// Radix sort of m keys: writes *out_keys / *out_perm pointing into the workspace (or to
+// `keys` + an identity permutation when every digit is constant).
+cudaError_t run_sort(SortWork& W, const uint64_t* keys, uint64_t m, const uint64_t** out_keys,
+                     const uint32_t** out_perm, DevState* st, int nsm, cudaStream_t s, Prof* prof = nullptr,
+                     double* hist_ms = nullptr, double* pass_ms = nullptr) {
+  cudaError_t e;
+  if ((e = W.ka.ensure(m)) || (e = W.kb.ensure(m)) || (e = W.ia.ensure(m)) || (e = W.ib.ensure(m))) return e;
+  const uint64_t tiles = (m + kSortTile - 1) / kSortTile;
+  const uint64_t need_status = std::max<uint64_t>(tiles * 256, 3 * ((m + 2047) / 2048) + 3);
+  if (W.status.n < need_status) {
+    if ((e = W.status.ensure(need_status))) return e;
+    if ((e = cudaMemsetAsync(W.status.p, 0, W.status.n * sizeof(uint64_t), s))) return e;
+  }
+  if ((e = W.hist.ensure(8 * 256)) || (e = W.bases.ensure(8 * 256))) return e;
+  if ((e = W.hist_h.ensure(8 * 256)) || (e = W.bases_h.ensure(8 * 256))) return e;
+  Prof::Span sp{};
+  if (prof && prof->on) prof->begin(s, sp);
+  if ((e = launch_hist(keys, m, W.hist.p, nsm, s))) return e;
+  if (prof && prof->on) prof->end(s, sp, hist_ms);
+  if ((e = cudaMemcpyAsync(W.hist_h.p, W.hist.p, 8 * 256 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s))) return e;
+  if ((e = cudaStreamSynchronize(s))) return e;
+  int digits[8];
+  int nd = 0;
+  for (int d = 0; d < 8; ++d) {
+    uint32_t run = 0;
+    int nonzero = 0;
+    for (int b = 0; b < 256; ++b) {
+      const uint32_t c = W.hist_h.p[d * 256 + b];
+      W.bases_h.p[d * 256 + b] = run;
+      run += c;
+      nonzero += c ? 1 : 0;
+    }
+    if (nonzero > 1) digits[nd++] = d;  // constant digits are skipped
+  }
+  W.passes = nd;
+  if (nd == 0) {
+    k_iota_u32<<<static_cast<unsigned>((m + 255) / 256 + 1), 256, 0, s>>>(W.ia.p, m);
+    *out_keys = keys;
+    *out_perm = W.ia.p;
+    return cudaGetLastError();
+  }
+  if ((e = cudaMemcpyAsync(W.bases.p, W.bases_h.p, 8 * 256 * sizeof(uint32_t), cudaMemcpyHostToDevice, s))) return e;
+  const uint64_t* kin = keys;
+  const uint32_t* iin = nullptr;
+  Prof::Span sp2{};
+  if (prof && prof->on) prof->begin(s, sp2);
+  for (int p = 0; p < nd; ++p) {
+    uint64_t* kout = (p & 1) ? W.kb.p : W.ka.p;
+    uint32_t* iout = (p & 1) ? W.ib.p : W.ia.p;
+    if ((e = launch_onesweep(kin, iin, kout, iout, m, digits[p], W.bases.p, W.status.p, W.epoch++,
+                             &st->tile_counter[0], s)))
+      return e;
+    kin = kout;
+    iin = iout;
+  }
+  if (prof && prof->on) prof->end(s, sp2, pass_ms);
+  *out_keys = kin;
+  *out_perm = iin;
+  return cudaSuccess;
+}
+
+}  // namespace
+
+struct mr_job {
+  mr_config cfg{};
+  mr_sm_params sm{};
+  uint32_t k = 0;
+  std::vector<float> cent_h;
+  int state = kCreated;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  int nsm = 148;
+  std::string err;
+  DevState* st = nullptr;
+  HBuf<DevState> st_h;
+  HBuf<uint64_t> tmp_h;
+  DBuf<float> cent;
+  DBuf<uint64_t> h, kref, tb;
+  DBuf<uint8_t> v;
+  uint64_t cap = 0;
+  std::vector<Batch> batches;
+  uint64_t next_base = 0;
+  std::vector<void*> owned;       // reserved
+  std::vector<DBuf<uint8_t>> host_rec;   // device copies made by mr_map_host (reused after reset)
+  std::vector<DBuf<uint64_t>> host_off;
+  size_t host_batches = 0;
+  Prof prof;
+  unsigned long long launches0 = 0;
+  SortWork sw;
+  const uint64_t* skeys = nullptr;
+  const uint32_t* perm = nullptr;
+  uint64_t m = 0, nseg = 0, key_bytes = 0;
+  DBuf<uint32_t> seg_counts;
+  DBuf<uint64_t> tile_base, seg_start, key_off, val_off, counts, worklist, gathered;
+  DBuf<uint8_t> keys_out, vals_out;
+  DBuf<double> sums;
+  DBuf<unsigned long long> cnts;
+  // fetched result
+  HBuf<uint8_t> keys_h, vals_h;
+  HBuf<uint64_t> key_off_h, val_off_h;
+  uint64_t out_keys_bytes = 0, out_vals_bytes = 0, out_n = 0;
+  mr_stats stats{};
+};
+
+namespace {
+
+mr_status fail(mr_job* j, mr_status s, const std::string& msg) {
+  if (j) j->err = msg;
+  return s;
+}
+mr_status cuda_fail(mr_job* j, cudaError_t e, const char* where) {
+  std::string m = std::string(where) + ": " + cudaGetErrorString(e);
+  cudaGetLastError();
+  return fail(j, e == cudaErrorMemoryAllocation ? MR_ERR_OOM : MR_ERR_CUDA, m);
+}
+#define CK(expr, where)                                  \
+  do {                                                   \
+    cudaError_t e_ = (expr);                             \
+    if (e_ != cudaSuccess) return cuda_fail(job, e_, where); \
+  } while (0)
+
+uint64_t initial_cap(const mr_job* job, uint64_t nbytes, uint64_t n) {
+  if (job->cfg.max_pairs_hint) return job->cfg.max_pairs_hint;
+  switch (job->cfg.workload) {
+    case MR_WORDCOUNT: return nbytes / 4 + 4096;
+    case MR_STRINGMATCH: return nbytes / 256 + 4096;
+    case MR_KMEANS: return n + 4096;
+    default: return nbytes / 32 + 4096;
+  }
+}
+
+cudaError_t ensure_pairs(mr_job* job, uint64_t cap) {
+  cudaError_t e;
+  if ((e = job->h.ensure(cap))) return e;
+  if (has_kref(job->cfg.workload) && (e = job->kref.ensure(cap))) return e;
+  const int vb = vbytes_of(job->cfg.workload);
+  if (vb && (e = job->v.ensure(cap * vb))) return e;
+  job->cap = cap;
+  return cudaSuccess;
+}
+
+cudaError_t launch_batch(mr_job* job, const Batch& b) {
+  MapArgs a;
+  a.workload = job->cfg.workload;
+  a.flags = job->cfg.flags;
+  a.records = b.rec;
+  a.offsets = b.off;
+  a.n = b.n;
+  a.nbytes = b.nbytes;
+  a.stride = job->cfg.record_stride;
+  a.gbase = b.gbase;
+  std::memcpy(a.pattern, job->sm.pattern, 16);
+  a.centroids = job->cent.p;
+  a.k = job->k;
+  a.out.h = job->h.p;
+  a.out.kref = job->kref.p;
+  a.out.v = job->v.p;
+  a.out.cap = job->cap;
+  a.st = job->st;
+  a.hash_seed = 0x5EEDB200ULL;
+  const uint64_t nt = map_tiles(a);
+  if (a.workload != kKM) {
+    cudaError_t e = job->tb.ensure(2 * nt + 2);
+    if (e) return e;
+  }
+  a.tile_bounds = job->tb.p;
+  job->stats.map_tiles += nt;
+  return launch_map(a, job->nsm, job->stream);
+}
+
+cudaError_t read_state(mr_job* job) {
+  cudaError_t e = cudaMemcpyAsync(job->st_h.p, job->st, sizeof(DevState), cudaMemcpyDeviceToHost, job->stream);
+  if (e) return e;
+  return cudaStreamSynchronize(job->stream);
+}
+
+mr_status do_segments(mr_job* job) {
+  const uint64_t m = job->m;
+  const uint64_t tiles = (m + 4095) / 4096;
+  CK(job->seg_counts.ensure(tiles + 1), "alloc seg counts");
+  CK(job->tile_base.ensure(tiles + 1), "alloc tile base");
+  CK(cudaMemsetAsync(&job->st->collisions, 0, sizeof(unsigned int), job->stream), "memset");
+  const uint64_t* kref = has_kref(job->cfg.workload) ? job->kref.p : nullptr;
+  CK(launch_seg_count(job->skeys, job->perm, kref, m, job->seg_counts.p, job->st, job->stream), "seg_count");
+  CK(launch_scan_u32to64(job->seg_counts.p, job->tile_base.p, tiles, &job->st->seg_total, job->sw.status.p,
+                         job->sw.epoch++, &job->st->tile_counter[1], job->stream),
+     "scan tiles");
+  CK(read_state(job), "sync segments");
+  job->nseg = m ? job->st_h.p->seg_total : 0;
+  CK(job->seg_start.ensure(job->nseg + 1), "alloc seg_start");
+  CK(launch_seg_write(job->skeys, m, job->tile_base.p, job->seg_start.p, job->stream), "seg_write");
+  return MR_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* mr_status_string(mr_status s) {
+  switch (s) {
+    case MR_OK: return "MR_OK";
+    case MR_ERR_INVALID: return "MR_ERR_INVALID";
+    case MR_ERR_STATE: return "MR_ERR_STATE";
+    case MR_ERR_OOM: return "MR_ERR_OOM";
+    case MR_ERR_OVERFLOW: return "MR_ERR_OVERFLOW";
+    case MR_ERR_CUDA: return "MR_ERR_CUDA";
+    case MR_ERR_NCCL: return "MR_ERR_NCCL";
+    case MR_ERR_UNSUPPORTED: return "MR_ERR_UNSUPPORTED";
+  }
+  return "MR_ERR_UNKNOWN";
+}
+
+const char* mr_last_error(const mr_job* job) { return job ? job->err.c_str() : "null job"; }
+
+mr_status mr_job_create(const mr_config* cfg, mr_job** out) {
+  if (!cfg || !out) return MR_ERR_INVALID;
+  *out = nullptr;
+  if (cfg->abi_version != MR_ABI_VERSION) return MR_ERR_INVALID;
+  if (cfg->workload < MR_WORDCOUNT || cfg->workload > MR_INVINDEX) return MR_ERR_INVALID;
+  if (cfg->nranks > 1) return MR_ERR_UNSUPPORTED;
+  if (cfg->workload == MR_KMEANS) {
+    const mr_km_params* p = static_cast<const mr_km_params*>(cfg->params);
+    if (!p || !p->centroids || p->dim != 8 || p->k < 1 || p->k > 1024 || cfg->record_stride != 32)
+      return MR_ERR_INVALID;
+  } else if (cfg->record_stride != 0) {
+    return MR_ERR_INVALID;
+  }
+  if (cfg->workload == MR_STRINGMATCH && !cfg->params) return MR_ERR_INVALID;
+  mr_job* job = new (std::nothrow) mr_job();
+  if (!job) return MR_ERR_OOM;
+  job->cfg = *cfg;
+  job->cfg.params = nullptr;
+  if (cfg->workload == MR_STRINGMATCH) job->sm = *static_cast<const mr_sm_params*>(cfg->params);
+  cudaError_t e = cudaSetDevice(cfg->device);
+  if (e == cudaSuccess && cfg->workload == MR_KMEANS) {
+    const mr_km_params* p = static_cast<const mr_km_params*>(cfg->params);
+    job->k = p->k;
+    job->cent_h.assign(p->centroids, p->centroids + static_cast<size_t>(p->k) * 8);
+  }
+  if (e == cudaSuccess) {
+    if (cfg->stream) {
+      job->stream = static_cast<cudaStream_t>(cfg->stream);
+    } else {
+      e = cudaStreamCreateWithFlags(&job->stream, cudaStreamNonBlocking);
+      job->own_stream = (e == cudaSuccess);
+    }
+  }
+  if (e == cudaSuccess) e = cudaMalloc(reinterpret_cast<void**>(&job->st), sizeof(DevState));
+  if (e == cudaSuccess) e = job->st_h.ensure(1);
+  if (e == cudaSuccess) e = job->tmp_h.ensure(16);
+  if (e == cudaSuccess) e = cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream);
+  if (e == cudaSuccess && job->k) {
+    e = job->cent.ensure(job->k * 8);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(job->cent.p, job->cent_h.data(), job->k * 32, cudaMemcpyHostToDevice, job->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(job->stream);
+  }
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    mr_job_destroy(job);
+    return e == cudaErrorMemoryAllocation ? MR_ERR_OOM : MR_ERR_CUDA;
+  }
+  job->nsm = sm_count(cfg->device);
+  job->prof.on = (cfg->flags & MR_FLAG_PROFILE) != 0;
+  job->launches0 = g_kernel_launches.load();
+  *out = job;
+  return MR_OK;
+}
+
+mr_status mr_job_reset(mr_job* job) {
+  if (!job) return MR_ERR_INVALID;
+  CK(cudaSetDevice(job->cfg.device), "set device");
+  CK(cudaStreamSynchronize(job->stream), "sync");
+  for (void* p : job->owned) cudaFree(p);
+  job->owned.clear();
+  job->host_batches = 0;
+  job->prof.collect();
+  job->batches.clear();
+  job->next_base = 0;
+  job->m = job->nseg = job->key_bytes = 0;
+  job->skeys = nullptr;
+  job->perm = nullptr;
+  const uint64_t cap = job->stats.capacity_pairs;
+  job->stats = mr_stats{};
+  job->stats.capacity_pairs = cap;
+  job->launches0 = g_kernel_launches.load();
+  CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset state");
+  job->state = kCreated;
+  return MR_OK;
+}
+
+static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t* offsets, uint64_t n) {
+  if (job->state != kCreated && job->state != kMapped) return fail(job, MR_ERR_STATE, "mr_map after mr_group");
+  const bool fixed = job->cfg.record_stride > 0;
+  if (fixed != (offsets == nullptr)) return fail(job, MR_ERR_INVALID, "offsets must be NULL iff record_stride > 0");
+  if (fixed && (reinterpret_cast<uintptr_t>(records) & 15u))
+    return fail(job, MR_ERR_INVALID, "fixed-stride records must be 16-byte aligned");
+  if ((reinterpret_cast<uintptr_t>(records) >> 48) != 0) return fail(job, MR_ERR_INVALID, "records address >= 2^48");
+  uint64_t nbytes = 0;
+  if (fixed) {
+    nbytes = n * job->cfg.record_stride;
+  } else {
+    CK(cudaMemcpyAsync(job->tmp_h.p, offsets + n, sizeof(uint64_t), cudaMemcpyDeviceToHost, job->stream), "read offsets[n]");
+    if (job->cfg.flags & MR_FLAG_VALIDATE) {
+      std::vector<uint64_t> o(n + 1);
+      CK(cudaMemcpyAsync(o.data(), offsets, (n + 1) * 8, cudaMemcpyDeviceToHost, job->stream), "read offsets");
+      CK(cudaStreamSynchronize(job->stream), "sync");
+      if (o[0] != 0) return fail(job, MR_ERR_INVALID, "offsets[0] != 0");
+      for (uint64_t i = 0; i < n; ++i)
+        if (o[i + 1] < o[i]) return fail(job, MR_ERR_INVALID, "offsets not non-decreasing");
+    }
+    CK(cudaStreamSynchronize(job->stream), "sync offsets[n]");
+    nbytes = job->tmp_h.p[0];
+  }
+  if (nbytes && !records) return fail(job, MR_ERR_INVALID, "records is NULL");
+  if (job->cap == 0) {
+    CK(ensure_pairs(job, initial_cap(job, nbytes, n)), "alloc intermediate");
+    job->stats.capacity_pairs = job->cap;
+  }
+  Batch b{records, offsets, n, nbytes, job->cfg.input_base + job->next_base};
+  job->next_base += nbytes;
+  job->batches.push_back(b);
+  job->stats.input_bytes += nbytes;
+  Prof::Span sp{};
+  if (job->prof.on) job->prof.begin(job->stream, sp);
+  CK(launch_batch(job, b), "map kernel launch");
+  if (job->prof.on) job->prof.end(job->stream, sp, &job->stats.map_ms);
+  job->state = kMapped;
+  return MR_OK;
+}
+
+mr_status mr_map(mr_job* job, const uint8_t* records, const uint64_t* offsets, uint64_t n) {
+  if (!job) return MR_ERR_INVALID;
+  CK(cudaSetDevice(job->cfg.device), "set device");
+  return map_common(job, records, offsets, n);
+}
+
+mr_status mr_map_host(mr_job* job, const uint8_t* records, const uint64_t* offsets, uint64_t n) {
+  if (!job) return MR_ERR_INVALID;
+  CK(cudaSetDevice(job->cfg.device), "set device");
+  const bool fixed = job->cfg.record_stride > 0;
+  if (fixed != (offsets == nullptr)) return fail(job, MR_ERR_INVALID, "offsets must be NULL iff record_stride > 0");
+  const uint64_t nbytes = fixed ? n * job->cfg.record_stride : offsets[n];
+  if (nbytes && !records) return fail(job, MR_ERR_INVALID, "records is NULL");
+  const size_t i = job->host_batches++;
+  if (job->host_rec.size() <= i) { job->host_rec.resize(i + 1); job->host_off.resize(i + 1); }
+  CK(job->host_rec[i].ensure(std::max<uint64_t>(nbytes, 16)), "alloc device records");
+  if (nbytes) CK(cudaMemcpyAsync(job->host_rec[i].p, records, nbytes, cudaMemcpyHostToDevice, job->stream), "H2D records");
+  const uint64_t* doff = nullptr;
+  if (!fixed) {
+    CK(job->host_off[i].ensure(n + 1), "alloc device offsets");
+    CK(cudaMemcpyAsync(job->host_off[i].p, offsets, (n + 1) * 8, cudaMemcpyHostToDevice, job->stream), "H2D offsets");
+    doff = job->host_off[i].p;
+  }
+  return map_common(job, job->host_rec[i].p, doff, n);
+}
+
+mr_status mr_group(mr_job* job) {
+  if (!job) return MR_ERR_INVALID;
+  if (job->state != kMapped && job->state != kCreated) return fail(job, MR_ERR_STATE, "mr_group out of order");
+  CK(cudaSetDevice(job->cfg.device), "set device");
+  CK(read_state(job), "map (async)");
+  DevState* hs = job->st_h.p;
+  if (hs->err & kErrKeyTooLong) return fail(job, MR_ERR_OVERFLOW, "an emitted key exceeds 65535 bytes");
+  uint64_t m = hs->pair_cursor;
+  if (m > job->cap) {
+    // D7: the cursor counted demand past capacity -> grow and replay every batch
+    const uint64_t ncap = m + m / 8 + 4096;
+    job->h.release(); job->kref.release(); job->v.release(); job->cap = 0;
+    CK(ensure_pairs(job, ncap), "grow intermediate");
+    job->stats.capacity_pairs = job->cap;
+    CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
+    for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
+    job->stats.replays += job->batches.size();
+    CK(read_state(job), "replay (async)");
+    m = hs->pair_cursor;
+    if (m > job->cap) return fail(job, MR_ERR_OOM, "replay still overflows");
+  }
+  job->m = m;
+  job->stats.pairs = m;
+  job->stats.flushes = hs->flushes;
+  if (m >= (1ULL << 32) - 1) return fail(job, MR_ERR_UNSUPPORTED, ">= 2^32 intermediate pairs in one group");
+  if (job->cfg.workload == MR_STRINGMATCH) {  // Map-only
+    job->nseg = m;
+    job->state = kGrouped;
+    return MR_OK;
+  }
+  for (int attempt = 0;; ++attempt) {
+    CK(run_sort(job->sw, job->h.p, m, &job->skeys, &job->perm, job->st, job->nsm, job->stream, &job->prof,
+                &job->stats.hist_ms, &job->stats.sort_ms),
+       "radix sort");
+    job->stats.sort_passes += job->sw.passes;
+    Prof::Span sp2{};
+    if (job->prof.on) job->prof.begin(job->stream, sp2);
+    mr_status s = do_segments(job);
+    if (s != MR_OK) return s;
+    if (job->prof.on) job->prof.end(job->stream, sp2, &job->stats.seg_ms);
+    const uint32_t coll = hs->collisions;
+    if (coll == 0) break;
+    job->stats.collisions += coll;
+    if (attempt >= 3) return fail(job, MR_ERR_UNSUPPORTED, "unresolvable 64-bit hash collision");
+    // slow path: recompute every hashed key with a fresh full-width hash, then sort again
+    CK(launch_rehash(job->h.p, job->kref.p, m, 0xC0111DE5ULL + attempt, job->stream), "rehash");
+  }
+  job->stats.n_keys = job->nseg;
+  Prof::Span sp3{};
+  if (job->prof.on) job->prof.begin(job->stream, sp3);
+  if (job->cfg.workload == MR_WORDCOUNT || job->cfg.workload == MR_INVINDEX) {
+    CK(job->key_off.ensure(job->nseg + 1), "alloc key offsets");
+    CK(launch_key_lengths(job->seg_start.p, job->nseg, job->perm, job->kref.p, job->key_off.p, job->stream), "key lengths");
+    CK(launch_scan_u64(job->key_off.p, job->key_off.p, job->nseg,
+                       reinterpret_cast<unsigned long long*>(job->key_off.p + job->nseg), job->sw.status.p,
+                       job->sw.epoch++, &job->st->tile_counter[2], job->stream),
+       "scan key lengths");
+    CK(cudaMemcpyAsync(job->tmp_h.p, job->key_off.p + job->nseg, 8, cudaMemcpyDeviceToHost, job->stream), "read key bytes");
+    CK(cudaStreamSynchronize(job->stream), "sync key bytes");
+    job->key_bytes = job->tmp_h.p[0];
+  }
+  if (job->prof.on) { job->prof.end(job->stream, sp3, &job->stats.seg_ms); CK(cudaStreamSynchronize(job->stream), "sync"); job->prof.collect(); }
+  job->state = kGrouped;
+  return MR_OK;
+}
+
+mr_status mr_reduce(mr_job* job) {
+  if (!job) return MR_ERR_INVALID;
+  if (job->state != kGrouped) return fail(job, MR_ERR_STATE, "mr_reduce before mr_group");
+  CK(cudaSetDevice(job->cfg.device), "set device");
+  const uint64_t S = job->nseg, m = job->m;
+  cudaStream_t s = job->stream;
+  Prof::Span sp{};
+  if (job->prof.on) job->prof.begin(s, sp);
+  switch (job->cfg.workload) {
+    case MR_WORDCOUNT: {
+      CK(job->counts.ensure(S + 1), "alloc counts");
+      CK(job->worklist.ensure(m / 1024 + 64), "alloc worklist");
+      CK(launch_reduce_wc(job->seg_start.p, S, job->perm, job->v.p, job->counts.p, job->worklist.p, job->st, job->nsm, s),
+         "reduce wc");
+      CK(job->val_off.ensure(S + 1), "alloc val offsets");
+      CK(launch_iota_scaled(S, 8, job->val_off.p, s), "val offsets");
+      CK(job->keys_out.ensure(job->key_bytes + 1), "alloc keys");
+      CK(launch_key_copy(job->seg_start.p, S, job->perm, job->kref.p, job->key_off.p, job->keys_out.p, s), "key copy");
+      job->out_n = S;
+      job->out_keys_bytes = job->key_bytes;
+      job->out_vals_bytes = S * 8;
+      break;
+    }
+    case MR_INVINDEX: {
+      CK(job->gathered.ensure(m + 1), "alloc values");
+      CK(launch_gather_u64(job->perm, job->v.p, m, job->gathered.p, s), "gather values");
+      CK(job->val_off.ensure(S + 1), "alloc val offsets");
+      CK(launch_offsets_scaled(job->seg_start.p, S, 8, job->val_off.p, s), "val offsets");
+      CK(job->keys_out.ensure(job->key_bytes + 1), "alloc keys");
+      CK(launch_key_copy(job->seg_start.p, S, job->perm, job->kref.p, job->key_off.p, job->keys_out.p, s), "key copy");
+      job->out_n = S;
+      job->out_keys_bytes = job->key_bytes;
+      job->out_vals_bytes = m * 8;
+      break;
+    }
+    case MR_KMEANS: {
+      const uint32_t k = job->k;
+      CK(job->sums.ensure(8ULL * k), "alloc sums");
+      CK(job->cnts.ensure(k), "alloc counts");
+      CK(job->worklist.ensure(m / 1024 + 64), "alloc worklist");
+      CK(launch_reduce_km(job->seg_start.p, S, job->skeys, job->perm, job->v.p, job->sums.p, job->cnts.p, k,
+                          job->worklist.p, job->st, job->nsm, s),
+         "reduce km");
+      CK(job->keys_out.ensure(4ULL * k), "alloc keys");
+      CK(job->vals_out.ensure(40ULL * k), "alloc vals");
+      CK(job->key_off.ensure(k + 1), "alloc key offsets");
+      CK(job->val_off.ensure(k + 1), "alloc val offsets");
+      CK(launch_km_finalize(job->sums.p, job->cnts.p, job->cent.p, k, job->vals_out.p, job->val_off.p, job->keys_out.p,
+                            job->key_off.p, s),
+         "km finalize");
+      job->out_n = k;
+      job->out_keys_bytes = 4ULL * k;
+      job->out_vals_bytes = 40ULL * k;
+      break;
+    }
+    case MR_STRINGMATCH: {
+      CK(job->key_off.ensure(m + 1), "alloc key offsets");
+      CK(job->val_off.ensure(m + 1), "alloc val offsets");
+      CK(launch_iota_scaled(m, 8, job->key_off.p, s), "key offsets");
+      CK(cudaMemsetAsync(job->val_off.p, 0, (m + 1) * 8, s), "val offsets");
+      job->out_n = m;
+      job->out_keys_bytes = m * 8;
+      job->out_vals_bytes = 0;
+      break;
+    }
+  }
+  if (job->prof.on) job->prof.end(s, sp, &job->stats.reduce_ms);
+  job->state = kReduced;
+  return MR_OK;
+}
+
+mr_status mr_fetch(mr_job* job, mr_result* out) {
+  if (!job || !out) return MR_ERR_INVALID;
+  if (job->state != kReduced) return fail(job, MR_ERR_STATE, "mr_fetch before mr_reduce");
+  CK(cudaSetDevice(job->cfg.device), "set device");
+  cudaStream_t s = job->stream;
+  const uint64_t n = job->out_n;
+  CK(job->keys_h.ensure(job->out_keys_bytes + 1), "alloc host keys");
+  CK(job->vals_h.ensure(job->out_vals_bytes + 1), "alloc host vals");
+  CK(job->key_off_h.ensure(n + 1), "alloc host key offsets");
+  CK(job->val_off_h.ensure(n + 1), "alloc host val offsets");
+  const uint8_t* dkeys = job->cfg.workload == MR_STRINGMATCH ? reinterpret_cast<const uint8_t*>(job->h.p) : job->keys_out.p;
+  const uint8_t* dvals = job->cfg.workload == MR_WORDCOUNT ? reinterpret_cast<const uint8_t*>(job->counts.p)
+                         : job->cfg.workload == MR_INVINDEX ? reinterpret_cast<const uint8_t*>(job->gathered.p)
+                                                            : job->vals_out.p;
+  if (job->out_keys_bytes) CK(cudaMemcpyAsync(job->keys_h.p, dkeys, job->out_keys_bytes, cudaMemcpyDeviceToHost, s), "D2H keys");
+  if (job->out_vals_bytes) CK(cudaMemcpyAsync(job->vals_h.p, dvals, job->out_vals_bytes, cudaMemcpyDeviceToHost, s), "D2H vals");
+  CK(cudaMemcpyAsync(job->key_off_h.p, job->key_off.p, (n + 1) * 8, cudaMemcpyDeviceToHost, s), "D2H key offsets");
+  CK(cudaMemcpyAsync(job->val_off_h.p, job->val_off.p, (n + 1) * 8, cudaMemcpyDeviceToHost, s), "D2H val offsets");
+  CK(cudaStreamSynchronize(s), "fetch");
+  if (job->prof.on) job->prof.collect();
+  out->n_keys = n;
+  out->keys = job->keys_h.p;
+  out->key_offsets = job->key_off_h.p;
+  out->vals = job->vals_h.p;
+  out->val_offsets = job->val_off_h.p;
+  return MR_OK;
+}
+
+mr_status mr_get_stats(const mr_job* job, void* stats, size_t bytes) {
+  if (!job || !stats) return MR_ERR_INVALID;
+  mr_stats st = job->stats;
+  st.kernel_launches = g_kernel_launches.load() - job->launches0;
+  std::memcpy(stats, &st, std::min(bytes, sizeof(mr_stats)));
+  return MR_OK;
+}
+
+mr_status mr_job_destroy(mr_job* job) {
+  if (!job) return MR_OK;
+  cudaSetDevice(job->cfg.device);
+  if (job->stream) cudaStreamSynchronize(job->stream);
+  for (void* p : job->owned) cudaFree(p);
+  for (auto& b : job->host_rec) b.release();
+  for (auto& b : job->host_off) b.release();
+  job->prof.release();
+  job->cent.release(); job->h.release(); job->kref.release(); job->tb.release(); job->v.release();
+  job->sw.release();
+  job->seg_counts.release(); job->tile_base.release(); job->seg_start.release(); job->key_off.release();
+  job->val_off.release(); job->counts.release(); job->worklist.release(); job->gathered.release();
+  job->keys_out.release(); job->vals_out.release(); job->sums.release(); job->cnts.release();
+  job->keys_h.release(); job->vals_h.release(); job->key_off_h.release(); job->val_off_h.release();
+  job->st_h.release(); job->tmp_h.release();
+  if (job->st) cudaFree(job->st);
+  if (job->own_stream && job->stream) cudaStreamDestroy(job->stream);
+  cudaGetLastError();
+  delete job;
+  return MR_OK;
+}
+
+mr_status mr_sort_u64(const uint64_t* keys, uint64_t* keys_out, uint32_t* perm_out, uint64_t n, void* stream) {
+  if ((n && (!keys || !keys_out || !perm_out)) || n >= (1ULL << 32) - 1) return MR_ERR_INVALID;
+  if (n == 0) return MR_OK;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  SortWork W;
+  DevState* st = nullptr;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  cudaError_t e = cudaMalloc(reinterpret_cast<void**>(&st), sizeof(DevState));
+  if (e == cudaSuccess) e = cudaMemsetAsync(st, 0, sizeof(DevState), s);
+  const uint64_t* ko = nullptr;
+  const uint32_t* po = nullptr;
+  if (e == cudaSuccess) e = run_sort(W, keys, n, &ko, &po, st, sm_count(dev), s);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(keys_out, ko, n * 8, cudaMemcpyDeviceToDevice, s);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(perm_out, po, n * 4, cudaMemcpyDeviceToDevice, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  W.release();
+  if (st) cudaFree(st);
+  if (e != cudaSuccess) { cudaGetLastError(); return e == cudaErrorMemoryAllocation ? MR_ERR_OOM : MR_ERR_CUDA; }
+  return MR_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,138 @@
+// common.cuh — device-side building blocks shared by the libbmr kernels (sm_100a only).
+//   * PTX wrappers: mbarrier (init / arrive / expect_tx / try_wait.parity) and the 1-D TMA
+//     bulk copy cp.async.bulk (global -> shared, completion through an mbarrier).
+//   * Key encoding used by the emit step: keys of <= 7 bytes are packed
+//     injectively into the 64-bit sort key (length in the top byte, 1..7); longer keys are
+//     hashed to 64 bits with the top bit forced to 1, so the two classes never collide.
+//     Hashed keys are verified byte-for-byte at segment-boundary time (a8).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+#include "kernels.h"
+
+namespace bmr {
+
+// ---------------------------------------------------------------- PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  while (!mbar_try_wait(bar, parity)) {
+  }
+}
+// TMA 1-D bulk copy global -> shared; dst, src and bytes must be multiples of 16.
+__device__ __forceinline__ void tma_load_1d(void* smem_dst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(smem_dst)),
+      "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_shared() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+__device__ __forceinline__ uint64_t ld_volatile_u64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.volatile.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_volatile_u64(uint64_t* p, uint64_t v) {
+  asm volatile("st.volatile.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_volatile_u32(uint32_t* p, uint32_t v) {
+  asm volatile("st.volatile.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// ---------------------------------------------------------------- key encoding
+__host__ __device__ __forceinline__ uint64_t mix64(uint64_t z) {  // murmur3 finaliser
+  z ^= z >> 33;
+  z *= 0xff51afd7ed558ccdULL;
+  z ^= z >> 33;
+  z *= 0xc4ceb9fe1a85ec53ULL;
+  z ^= z >> 33;
+  return z;
+}
+constexpr uint64_t kHashedBit = 1ULL << 63;
+
+// Hash of len >= 8 key bytes read through a generic pointer (shared or global).
+__device__ __forceinline__ uint64_t hash_bytes(const uint8_t* p, uint32_t len, uint64_t seed) {
+  uint64_t h = seed ^ (static_cast<uint64_t>(len) * 0x9E3779B97F4A7C15ULL);
+  uint32_t i = 0;
+  for (; i + 8 <= len; i += 8) {
+    uint64_t b = 0;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) b |= static_cast<uint64_t>(p[i + k]) << (8 * k);
+    h = mix64(h ^ b) + 0x632BE59BD9B4E019ULL;
+  }
+  if (i < len) {
+    uint64_t b = 0;
+    for (int k = 0; i + k < len; ++k) b |= static_cast<uint64_t>(p[i + k]) << (8 * k);
+    h = mix64(h ^ b ^ 0xA5A5A5A5ULL);
+  }
+  return mix64(h);
+}
+// Final sort key of a hashed key; weak_hash (MR_FLAG_WEAK_HASH_DEBUG) keeps only 4 bits so
+// that almost every segment collides (tests the verification + re-sort slow path).
+__device__ __forceinline__ uint64_t hashed_key(uint64_t h, bool weak) {
+  return (weak ? (h & 0xFULL) : (h & ~kHashedBit)) | kHashedBit;
+}
+// <= 7 bytes packed little-endian, length in bits 56..63 (1..7): injective, top bit clear.
+__device__ __forceinline__ uint64_t inline_key(uint64_t bytes_le, uint32_t len) {
+  return (bytes_le & ((1ULL << (8 * len)) - 1ULL)) | (static_cast<uint64_t>(len) << 56);
+}
+
+// ---------------------------------------------------------------- small scans
+__device__ __forceinline__ uint32_t warp_inclusive_add(uint32_t v) {
+  const uint32_t lane = threadIdx.x & 31;
+#pragma unroll
+  for (int s = 1; s < 32; s <<= 1) {
+    uint32_t t = __shfl_up_sync(0xffffffffu, v, s);
+    if (lane >= static_cast<uint32_t>(s)) v += t;
+  }
+  return v;
+}
+__device__ __forceinline__ uint64_t warp_inclusive_add64(uint64_t v) {
+  const uint32_t lane = threadIdx.x & 31;
+#pragma unroll
+  for (int s = 1; s < 32; s <<= 1) {
+    uint64_t t = __shfl_up_sync(0xffffffffu, v, s);
+    if (lane >= static_cast<uint32_t>(s)) v += t;
+  }
+  return v;
+}
+
+}  // namespace bmr

@@ -1,0 +1,113 @@
+// kernels.h — host-visible launchers of the libbmr device kernels (internal to libbmr.so;
+// the public C ABI is include/bmr.h).  No torch types anywhere.
+#pragma once
+#include <atomic>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace bmr {
+
+// process-wide count of libbmr kernel launches (reported through mr_stats::kernel_launches)
+extern std::atomic<unsigned long long> g_kernel_launches;
+inline void count_launch(unsigned n = 1) { g_kernel_launches.fetch_add(n, std::memory_order_relaxed); }
+
+enum Workload : int { kWC = 1, kSM = 2, kKM = 3, kII = 4 };
+
+// Device-resident job state (one per job).
+struct DevState {
+  unsigned long long pair_cursor;  // D7: demand in pairs (counts past capacity -> replay)
+  unsigned long long flushes;      // number of output-half flushes (one global atomic each)
+  unsigned int err;                // kErr* bits
+  unsigned int collisions;         // hashed-key mismatches inside equal-hash runs
+  unsigned long long seg_total;    // S
+  unsigned long long key_bytes;    // total output key bytes
+  unsigned long long large_items;  // reduce work list length (large segments x tiles)
+  unsigned long long large_done;   // work-list cursor for the persistent large-segment kernel
+  unsigned int tile_counter[32];   // dynamic tile ids of the look-back kernels (one per launch slot)
+};
+constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u;
+
+// Intermediate pairs, SoA in HBM (SURVEY §8(a) layout): sort key, key reference, value.
+struct PairBufs {
+  uint64_t* h = nullptr;     // 64-bit sort key (inline key / hash / SM offset / KM id)
+  uint64_t* kref = nullptr;  // (device address of key bytes << 16) | key length
+  uint8_t* v = nullptr;      // value bytes (vbytes per pair)
+  uint64_t cap = 0;          // capacity in pairs
+};
+
+struct MapArgs {
+  int workload = 0;
+  uint32_t flags = 0;
+  const uint8_t* records = nullptr;
+  const uint64_t* offsets = nullptr;  // n+1 (text) or nullptr (fixed stride)
+  uint64_t n = 0;                     // records
+  uint64_t nbytes = 0;                // records bytes (offsets[n] or n*stride)
+  uint32_t stride = 0;
+  uint64_t gbase = 0;                 // global byte offset of records[0]
+  uint8_t pattern[16] = {0};          // SM
+  const float* centroids = nullptr;   // KM, device, k x 8
+  uint32_t k = 0;
+  PairBufs out;
+  DevState* st = nullptr;
+  uint64_t* tile_bounds = nullptr;    // scratch: 2 u64 per tile
+  uint64_t hash_seed = 0;
+  int grid = 0;                       // persistent CTAs (0 = one per SM)
+};
+
+int vbytes_of(int workload);                 // value bytes per pair
+bool has_kref(int workload);
+uint64_t map_tiles(const MapArgs& a);        // number of tiles of a batch
+cudaError_t launch_map(const MapArgs& a, int num_sms, cudaStream_t s);
+
+// ---- group-by-key (hash radix sort + segment boundaries) ----
+struct SortBufs {
+  uint64_t* keys_a = nullptr; uint64_t* keys_b = nullptr;
+  uint32_t* idx_a = nullptr;  uint32_t* idx_b = nullptr;
+  uint64_t* status = nullptr; uint64_t status_cap = 0;  // look-back words (tiles x 256)
+  uint32_t* hist = nullptr;    // 8 x 256 digit histograms
+  uint32_t* bases = nullptr;   // 8 x 256 exclusive digit bases
+  uint64_t cap = 0;
+};
+constexpr int kSortThreads = 256, kSortIPT = 16, kSortTile = kSortThreads * kSortIPT;
+cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int num_sms, cudaStream_t s);
+// one LSD pass on digit `digit`; idx_in == nullptr means the identity permutation
+cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
+                            uint32_t* idx_out, uint64_t m, int digit, const uint32_t* bases,
+                            uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s);
+
+// ---- segments ----
+// heads per sort tile + byte verification of hashed keys; counts[t] = heads in tile t
+cudaError_t launch_seg_count(const uint64_t* skeys, const uint32_t* perm, const uint64_t* kref, uint64_t m,
+                             uint32_t* counts, DevState* st, cudaStream_t s);
+// exclusive scan of u64 (in-place allowed); writes total to *total if non-null
+cudaError_t launch_scan_u64(const uint64_t* in, uint64_t* out, uint64_t n, unsigned long long* total,
+                            uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s);
+cudaError_t launch_scan_u32to64(const uint32_t* in, uint64_t* out, uint64_t n, unsigned long long* total,
+                                uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s);
+cudaError_t launch_seg_write(const uint64_t* skeys, uint64_t m, const uint64_t* tile_base, uint64_t* seg_start,
+                             cudaStream_t s);
+
+// ---- reduce + output assembly ----
+struct OutBufs {
+  uint8_t* keys = nullptr; uint64_t* key_off = nullptr;
+  uint8_t* vals = nullptr; uint64_t* val_off = nullptr;
+};
+cudaError_t launch_key_lengths(const uint64_t* seg_start, uint64_t nseg, const uint32_t* perm,
+                               const uint64_t* kref, uint64_t* lens, cudaStream_t s);
+cudaError_t launch_key_copy(const uint64_t* seg_start, uint64_t nseg, const uint32_t* perm, const uint64_t* kref,
+                            const uint64_t* key_off, uint8_t* keys, cudaStream_t s);
+cudaError_t launch_reduce_wc(const uint64_t* seg_start, uint64_t nseg, const uint32_t* perm, const uint8_t* v,
+                             uint64_t* counts, uint64_t* worklist, DevState* st, int num_sms, cudaStream_t s);
+cudaError_t launch_reduce_km(const uint64_t* seg_start, uint64_t nseg, const uint64_t* skeys, const uint32_t* perm,
+                             const uint8_t* v, double* sums, unsigned long long* cnts, uint32_t k,
+                             uint64_t* worklist, DevState* st, int num_sms, cudaStream_t s);
+cudaError_t launch_km_finalize(const double* sums, const unsigned long long* cnts, const float* centroids,
+                               uint32_t k, uint8_t* vals, uint64_t* val_off, uint8_t* keys, uint64_t* key_off,
+                               cudaStream_t s);
+cudaError_t launch_gather_u64(const uint32_t* perm, const uint8_t* v, uint64_t m, uint64_t* out, cudaStream_t s);
+cudaError_t launch_offsets_scaled(const uint64_t* seg_start, uint64_t nseg, uint64_t scale, uint64_t* out,
+                                  cudaStream_t s);
+cudaError_t launch_iota_scaled(uint64_t n, uint64_t scale, uint64_t* out, cudaStream_t s);
+cudaError_t launch_rehash(uint64_t* h, const uint64_t* kref, uint64_t m, uint64_t seed, cudaStream_t s);
+
+}  // namespace bmr

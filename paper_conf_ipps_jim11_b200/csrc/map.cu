@@ -1,0 +1,758 @@
+// map.cu — the Map phase: persistent, warp-specialised CTAs.
+//
+// PAPER.md §III (L66-113) stages input into shared memory, runs the user Map per record,
+// collects results in a shared-memory output area and flushes it to global memory with one
+// global atomic per flush.  Its GT200 mechanics (16 KB SMEM, all threads alternating between
+// stage-in / compute / stage-out, software wait-signal flags, yield by dummy global reads) are
+// prior art; the B200 re-derivation here:
+//   * producer warp (A1/A2): one elected lane issues TMA bulk copies (cp.async.bulk) of the
+//     tile bytes and of the tile's record-offset slice into a 3-stage SMEM ring guarded by
+//     mbarrier full/empty pairs (replaces the barrier-separated staging loop, L68/L85);
+//   * 16 map warps (A3): byte-parallel, record-agnostic scanning — each lane owns a 16-byte
+//     chunk, record boundaries come from a per-stage bitmap built from the staged offsets; the
+//     per-record imbalance the paper blames for SO overhead (L273) disappears;
+//   * emit allocator (A11/A12, D3/D4): a warp result is reserved with ONE shared 64-bit
+//     atomicAdd on a packed [generation | count] cursor of the active output half;
+//   * overflow (A13, L113): the unique warp whose reservation crosses the half's capacity seals
+//     the half, switches generation (double-buffered halves) and hands the half to the flush
+//     warp through an mbarrier (replaces the wait/signal flag protocol, L96-100);
+//   * flush warp (A4): one global atomicAdd per flush reserves [base, base+k) of the
+//     intermediate SoA arrays, then coalesced stores.  The global cursor counts demand even
+//     past capacity (D7), so the host can grow the buffers and replay the batch.
+#include <cstdio>
+
+#include "common.cuh"
+
+namespace bmr {
+namespace {
+
+constexpr int kNMap = 16;
+constexpr int kProdWarp = kNMap;
+constexpr int kFlushWarp = kNMap + 1;
+constexpr int kThreads = (kNMap + 2) * 32;
+constexpr int kStages = 3;
+constexpr int kT = 16384;        // owned bytes per tile (text) / bytes per tile (KM)
+constexpr int kLead = 16;        // bytes staged before the tile (previous-byte context)
+constexpr int kHalo = 256;       // bytes staged after the tile (words / matches / URLs crossing it)
+constexpr int kWin = 512;        // bytes per warp window = 32 lanes x 16 B
+constexpr int kNWin = kT / kWin;
+constexpr int kStageBytes = 16768;             // >= kLead + kT + kHalo + 32, multiple of 128
+constexpr int kOffCap = 1024;                  // record offsets staged per tile
+constexpr int kOffBytes = 8320;                // (kOffCap + 2) * 8 rounded up
+constexpr int kBitWords = kStageBytes / 32 + 4;
+constexpr int kBitBytes = 2176;                // >= kBitWords * 4, multiple of 128
+constexpr int kOutHalf = 40960;
+constexpr int kKmPts = kT / 32;                // 512 points per KM tile
+
+static_assert(kLead + kT + kHalo + 32 <= kStageBytes, "stage too small");
+static_assert(kBitWords * 4 <= kBitBytes, "bitmap too small");
+static_assert(kKmPts == kNMap * 32, "one KM point per map lane");
+
+struct StageHdr {
+  long long t;                   // tile id (-1: end of work)
+  long long sbase;               // input position of stage byte 0
+  long long chunk0;              // first (possibly negative) position of the tile's chunk grid
+  long long lo, hi;              // owned positions [lo, hi) clipped to [0, N); KM: points
+  long long stg_hi;              // staged bytes cover positions < stg_hi
+  unsigned long long ra, rb;     // record starts staged: offsets[ra..rb)
+  unsigned int off_shift;        // byte offset of offsets[ra] inside the offsets region
+  unsigned int off_staged;       // offsets slice is in SMEM
+};
+
+struct OutCtl {
+  unsigned long long cur;        // [generation:32 | count:32]; half = generation & 1
+  unsigned int committed[2];     // entries fully written into each half (current generation)
+  unsigned int fcount[2];        // sealed entry count of each half
+  unsigned int final_gen, is_final;
+  uint64_t req[2];               // mbarrier: half sealed -> flush warp
+  uint64_t done[2];              // mbarrier: half flushed -> free
+};
+
+struct Layout {
+  static constexpr int ctl = 0;                                   // OutCtl
+  static constexpr int hdr = 128;                                 // kStages x 128
+  static constexpr int full = hdr + kStages * 128;                // kStages x 8
+  static constexpr int empty = full + kStages * 8;
+  static constexpr int bytes = 1024;                              // kStages x kStageBytes
+  static constexpr int offs = bytes + kStages * kStageBytes;      // kStages x kOffBytes
+  static constexpr int bits = offs + kStages * kOffBytes;         // kStages x kBitBytes
+  static constexpr int out = bits + kStages * kBitBytes;          // 2 x kOutHalf
+  static constexpr int cent = out + 2 * kOutHalf;                 // KM centroids
+};
+static_assert(Layout::empty + kStages * 8 <= Layout::bytes, "header region overflow");
+
+template <int W>
+struct PairFmt {
+  static constexpr bool kKref = (W == kWC || W == kII);
+  static constexpr int kV = (W == kWC) ? 4 : (W == kSM) ? 0 : (W == kKM) ? 32 : 8;
+  static constexpr int kPairBytes = 8 + (kKref ? 8 : 0) + kV;
+  static constexpr uint32_t kCap = (kOutHalf / kPairBytes) & ~3u;
+  // largest single warp reservation: WC 8 words / 16 B, SM 16 matches / 16 B, II 2, KM 1 per lane
+  static constexpr uint32_t kMaxReserve = (W == kWC) ? 256 : (W == kSM) ? 512 : 32 * ((W == kII) ? 2 : 1);
+  static_assert(kCap >= kMaxReserve, "output half smaller than one warp result");
+};
+
+struct Params {
+  const uint8_t* rec;
+  const uint64_t* off;
+  uint64_t n, nbytes;
+  long long a0;            // rec & 15 (text chunk alignment)
+  uint64_t ntiles;
+  uint64_t gbase;
+  uint32_t pat[4];
+  const float* cent;
+  uint32_t k;
+  uint64_t* oh;
+  uint64_t* okref;
+  uint8_t* ov;
+  uint64_t cap_pairs;
+  uint32_t out_cap;        // per-half capacity actually used (FORCE_TINY_OUT shrinks it)
+  uint32_t flags;
+  DevState* st;
+  const uint64_t* tb;      // tile bounds
+  uint64_t hash_seed;
+};
+
+constexpr uint32_t kFull = 0xffffffffu;
+
+// ---------------------------------------------------------------- byte-class helpers
+__device__ __forceinline__ uint32_t movemask4(uint32_t m) {  // 0xFF/0x00 bytes -> 4 bits
+  return ((((m >> 7) & 0x01010101u) * 0x01020408u) >> 24) & 0xFu;
+}
+__device__ __forceinline__ uint32_t word_mask4(uint32_t x) {  // [0-9A-Za-z] (C-3 #1)
+  uint32_t dig = __vcmpltu4(__vsub4(x, 0x30303030u), 0x0a0a0a0au);
+  uint32_t alp = __vcmpltu4(__vsub4(x | 0x20202020u, 0x61616161u), 0x1a1a1a1au);
+  return movemask4(dig | alp);
+}
+__device__ __forceinline__ uint32_t eq_mask4(uint32_t x, uint32_t b4) { return movemask4(__vcmpeq4(x, b4)); }
+__device__ __forceinline__ bool is_word_byte(uint32_t c) {
+  return (c - '0' < 10u) || ((c | 0x20u) - 'a' < 26u);
+}
+// bits j (0..31) with lo <= p0 + j < hi
+__device__ __forceinline__ uint32_t range_mask32(long long p0, long long lo, long long hi) {
+  long long a = lo - p0, b = hi - p0;
+  uint32_t mb = b >= 32 ? kFull : (b <= 0 ? 0u : ((1u << b) - 1u));
+  uint32_t ma = a <= 0 ? kFull : (a >= 32 ? 0u : ~((1u << a) - 1u));
+  return ma & mb;
+}
+__device__ __forceinline__ uint32_t bits32(const uint32_t* bm, long long i0) {  // i0 % 16 == 0
+  uint32_t wi = static_cast<uint32_t>(i0 >> 5), sh = static_cast<uint32_t>(i0 & 31);
+  return sh ? ((bm[wi] >> 16) | (bm[wi + 1] << 16)) : bm[wi];
+}
+// select 3 consecutive words x[wi..wi+2] of an 8-word window (wi in 0..3, no local memory)
+__device__ __forceinline__ uint64_t window8(const uint32_t (&x)[8], uint32_t j) {
+  uint32_t wi = j >> 2, sh = (j & 3) * 8, a, b, c;
+  switch (wi) {
+    case 0: a = x[0]; b = x[1]; c = x[2]; break;
+    case 1: a = x[1]; b = x[2]; c = x[3]; break;
+    case 2: a = x[2]; b = x[3]; c = x[4]; break;
+    default: a = x[3]; b = x[4]; c = x[5]; break;
+  }
+  return (static_cast<uint64_t>(__funnelshift_r(b, c, sh)) << 32) | __funnelshift_r(a, b, sh);
+}
+// 16 bytes starting at j (0..15) of the 8-word window, as 4 words
+__device__ __forceinline__ void window16(const uint32_t (&x)[8], uint32_t j, uint32_t (&o)[4]) {
+  uint32_t wi = j >> 2, sh = (j & 3) * 8, y0, y1, y2, y3, y4;
+  switch (wi) {
+    case 0: y0 = x[0]; y1 = x[1]; y2 = x[2]; y3 = x[3]; y4 = x[4]; break;
+    case 1: y0 = x[1]; y1 = x[2]; y2 = x[3]; y3 = x[4]; y4 = x[5]; break;
+    case 2: y0 = x[2]; y1 = x[3]; y2 = x[4]; y3 = x[5]; y4 = x[6]; break;
+    default: y0 = x[3]; y1 = x[4]; y2 = x[5]; y3 = x[6]; y4 = x[7]; break;
+  }
+  o[0] = __funnelshift_r(y0, y1, sh); o[1] = __funnelshift_r(y1, y2, sh);
+  o[2] = __funnelshift_r(y2, y3, sh); o[3] = __funnelshift_r(y3, y4, sh);
+}
+
+// smallest record start > p (global binary search over offsets[0..n]; rare slow path)
+__device__ uint64_t next_start_after(const uint64_t* off, uint64_t n, uint64_t p) {
+  uint64_t lo = 0, hi = n + 1;  // first index with off[i] > p
+  while (lo < hi) {
+    uint64_t mid = (lo + hi) >> 1;
+    if (off[mid] > p) hi = mid; else lo = mid + 1;
+  }
+  return lo <= n ? off[lo] : ~0ULL;
+}
+
+struct TileView {
+  const uint8_t* sb;       // stage bytes
+  const uint32_t* bm;      // record-start bitmap
+  long long sbase, stg_hi;
+  __device__ bool is_start(long long q) const {
+    long long i = q - sbase;
+    return (bm[i >> 5] >> (i & 31)) & 1u;
+  }
+};
+
+// Word length for a word at position p whose end lies beyond the 32-byte window [p0, p0+32).
+__device__ uint32_t slow_word_len(const Params& P, const TileView& tv, long long p, long long from) {
+  long long q = from;
+  uint64_t rec_end = ~0ULL;
+  bool have_end = false;
+  const long long N = static_cast<long long>(P.nbytes);
+  for (;; ++q) {
+    if (q >= N) break;
+    uint32_t c;
+    if (q < tv.stg_hi) {
+      if (tv.is_start(q)) break;
+      c = tv.sb[q - tv.sbase];
+    } else {
+      if (!have_end) { rec_end = next_start_after(P.off, P.n, static_cast<uint64_t>(p)); have_end = true; }
+      if (static_cast<uint64_t>(q) >= rec_end) break;
+      c = P.rec[q];
+    }
+    if (!is_word_byte(c)) break;
+  }
+  return static_cast<uint32_t>(q - p);
+}
+
+// Position of the closing '"' of a URL starting at q0, or -1 if the record (or input) ends
+// first.  Scans the stage 16 bytes at a time, then global memory (slow path).
+__device__ long long find_quote(const Params& P, const TileView& tv, long long q0, long long p_marker) {
+  const long long N = static_cast<long long>(P.nbytes);
+  long long q = q0;
+  while (q < tv.stg_hi && q < N) {
+    if (tv.is_start(q)) return -1;
+    if (tv.sb[q - tv.sbase] == '"') return q;
+    ++q;
+  }
+  if (q >= N) return -1;
+  uint64_t rec_end = next_start_after(P.off, P.n, static_cast<uint64_t>(p_marker));
+  for (; q < N && static_cast<uint64_t>(q) < rec_end; ++q)
+    if (P.rec[q] == '"') return q;
+  return -1;
+}
+
+__device__ __forceinline__ uint64_t key_of(const uint8_t* kp, uint32_t len, const Params& P) {
+  if (len <= 7) {
+    uint64_t b = 0;
+    for (uint32_t i = 0; i < len; ++i) b |= static_cast<uint64_t>(kp[i]) << (8 * i);
+    return inline_key(b, len);
+  }
+  return hashed_key(hash_bytes(kp, len, P.hash_seed), (P.flags & 8u) != 0);
+}
+
+// ---------------------------------------------------------------- emit allocator
+struct Slot { uint32_t half, base; };
+
+__device__ __forceinline__ Slot reserve(OutCtl* oc, uint32_t cnt, uint32_t cap) {
+  const uint32_t lane = threadIdx.x & 31;
+  for (;;) {
+    unsigned long long old = 0;
+    if (lane == 0) old = atomicAdd(&oc->cur, static_cast<unsigned long long>(cnt));
+    old = __shfl_sync(kFull, old, 0);
+    const uint32_t gen = static_cast<uint32_t>(old >> 32), base = static_cast<uint32_t>(old);
+    const uint32_t h = gen & 1u;
+    if (base + cnt <= cap) return {h, base};
+    if (lane == 0) {
+      if (base <= cap) {
+        // This warp crossed the capacity first: it seals half h (L113 "overflow handling").
+        volatile unsigned int* cm = &oc->committed[h];
+        while (*cm != base) __nanosleep(20);
+        if (gen >= 1) mbar_wait(&oc->done[(gen - 1) & 1u], ((gen - 1) >> 1) & 1u);  // other half free
+        oc->committed[h ^ 1u] = 0;
+        oc->fcount[h] = base;
+        __threadfence_block();
+        atomicExch(&oc->cur, static_cast<unsigned long long>(gen + 1) << 32);
+        mbar_arrive(&oc->req[h]);
+      } else {
+        volatile unsigned long long* c = &oc->cur;
+        while (static_cast<uint32_t>(*c >> 32) == gen) __nanosleep(32);
+      }
+    }
+    __syncwarp();
+  }
+}
+__device__ __forceinline__ void commit(OutCtl* oc, Slot s, uint32_t cnt) {
+  __syncwarp();
+  if ((threadIdx.x & 31) == 0) {
+    __threadfence_block();
+    atomicAdd(&oc->committed[s.half], cnt);
+  }
+}
+
+// ---------------------------------------------------------------- flush warp
+template <int W>
+__device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
+  using F = PairFmt<W>;
+  const uint32_t lane = threadIdx.x & 31;
+  for (uint32_t f = 0;; ++f) {
+    const uint32_t h = f & 1u;
+    mbar_wait(&oc->req[h], (f >> 1) & 1u);
+    const uint32_t cnt = *reinterpret_cast<volatile unsigned int*>(&oc->fcount[h]);
+    const bool fin = *reinterpret_cast<volatile unsigned int*>(&oc->is_final) &&
+                     *reinterpret_cast<volatile unsigned int*>(&oc->final_gen) == f;
+    if (cnt) {
+      unsigned long long gb = 0;
+      if (lane == 0) {
+        gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(cnt));  // ONE global atomic
+        atomicAdd(&P.st->flushes, 1ULL);
+      }
+      gb = __shfl_sync(kFull, gb, 0);
+      if (gb + cnt <= P.cap_pairs) {
+        const uint8_t* half = smem + Layout::out + h * kOutHalf;
+        const uint64_t* sh = reinterpret_cast<const uint64_t*>(half);
+        for (uint32_t i = lane; i < cnt; i += 32) P.oh[gb + i] = sh[i];
+        if constexpr (F::kKref) {
+          const uint64_t* sk = sh + F::kCap;
+          for (uint32_t i = lane; i < cnt; i += 32) P.okref[gb + i] = sk[i];
+        }
+        const uint8_t* sv = half + F::kCap * (F::kKref ? 16 : 8);
+        if constexpr (F::kV == 4) {
+          const uint32_t* s4 = reinterpret_cast<const uint32_t*>(sv);
+          uint32_t* g4 = reinterpret_cast<uint32_t*>(P.ov) + gb;
+          for (uint32_t i = lane; i < cnt; i += 32) g4[i] = s4[i];
+        } else if constexpr (F::kV == 8) {
+          const uint64_t* s8 = reinterpret_cast<const uint64_t*>(sv);
+          uint64_t* g8 = reinterpret_cast<uint64_t*>(P.ov) + gb;
+          for (uint32_t i = lane; i < cnt; i += 32) g8[i] = s8[i];
+        } else if constexpr (F::kV == 32) {
+          const uint4* s16 = reinterpret_cast<const uint4*>(sv);
+          uint4* g16 = reinterpret_cast<uint4*>(P.ov) + gb * 2;
+          for (uint32_t i = lane; i < 2 * cnt; i += 32) g16[i] = s16[i];
+        }
+      }
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&oc->done[h]);
+    if (fin) break;
+  }
+}
+
+// ---------------------------------------------------------------- producer warp
+__device__ void stage_copy_edges(uint8_t* d, const uint8_t* g, uint64_t len, uint32_t lane, uint32_t& body_off,
+                                 uint32_t& body_len) {
+  const uint32_t head = static_cast<uint32_t>(
+      min(static_cast<uint64_t>((16u - (reinterpret_cast<uintptr_t>(g) & 15u)) & 15u), len));
+  const uint32_t body = static_cast<uint32_t>((len - head) & ~15ULL);
+  const uint32_t tail = static_cast<uint32_t>(len - head - body);
+  for (uint32_t i = lane; i < head; i += 32) d[i] = g[i];
+  for (uint32_t i = lane; i < tail; i += 32) d[head + body + i] = g[head + body + i];
+  body_off = head;
+  body_len = body;
+}
+
+template <int W>
+__device__ void producer_loop(const Params& P, uint8_t* smem) {
+  const uint32_t lane = threadIdx.x & 31;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout::full);
+  uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout::empty);
+  uint32_t it = 0;
+  const long long N = static_cast<long long>(P.nbytes);
+  for (uint64_t t0 = blockIdx.x; t0 < P.ntiles; t0 += 32ULL * gridDim.x) {
+    // lanes prefetch the bounds of the next 32 tiles of this CTA (one latency per 32 tiles)
+    uint64_t my_t = t0 + static_cast<uint64_t>(lane) * gridDim.x, my_ra = 0, my_rb = 0;
+    if constexpr (W != kKM) {
+      if (my_t < P.ntiles) { my_ra = P.tb[2 * my_t]; my_rb = P.tb[2 * my_t + 1]; }
+    }
+    for (uint32_t j = 0; j < 32; ++j) {
+      const uint64_t t = t0 + static_cast<uint64_t>(j) * gridDim.x;
+      if (t >= P.ntiles) break;
+      const uint64_t ra = __shfl_sync(kFull, my_ra, j), rb = __shfl_sync(kFull, my_rb, j);
+      const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
+      mbar_wait(&empty[s], ph ^ 1u);
+      StageHdr* hd = reinterpret_cast<StageHdr*>(smem + Layout::hdr + s * 128);
+      uint8_t* sb = smem + Layout::bytes + s * kStageBytes;
+      uint32_t b_off = 0, b_len = 0, o_off = 0, o_len = 0;
+      uint8_t* so = smem + Layout::offs + s * kOffBytes;
+      if constexpr (W == kKM) {
+        const uint64_t p_lo = t * kKmPts, p_hi = min(P.n, p_lo + kKmPts);
+        const uint8_t* g = P.rec + p_lo * 32;
+        uint8_t* d = sb + (reinterpret_cast<uintptr_t>(g) & 15u);   // same 16-B phase as the source
+        stage_copy_edges(d, g, (p_hi - p_lo) * 32, lane, b_off, b_len);
+        if (lane == 0) {
+          hd->t = static_cast<long long>(t);
+          hd->lo = static_cast<long long>(p_lo);
+          hd->hi = static_cast<long long>(p_hi);
+        }
+        __syncwarp();
+        if (lane == 0) {
+          mbar_arrive_expect_tx(&full[s], b_len);
+          if (b_len) tma_load_1d(d + b_off, g + b_off, b_len, &full[s]);
+        }
+      } else {
+        const long long chunk0 = static_cast<long long>(t) * kT - P.a0;
+        const long long sbase = chunk0 - kLead;
+        const long long w_lo = max(0LL, sbase);
+        const long long w_hi = chunk0 + kT + kHalo;
+        const long long stg_hi = min(w_hi, N);
+        // stage bytes [w_lo, stg_hi) at sb + (w_lo - sbase); (rec + sbase) is 16-B aligned
+        uint8_t* d = sb + (w_lo - sbase);
+        const uint8_t* g = P.rec + w_lo;
+        stage_copy_edges(d, g, static_cast<uint64_t>(max(0LL, stg_hi - w_lo)), lane, b_off, b_len);
+        // clear the record-start bitmap (map warps set bits after the full barrier)
+        uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout::bits + s * kBitBytes);
+        for (uint32_t i = lane; i < kBitBytes / 16; i += 32) reinterpret_cast<uint4*>(bm)[i] = make_uint4(0, 0, 0, 0);
+        // offsets slice offsets[ra..rb) (record starts in the staged window)
+        const uint64_t cnt = rb - ra;
+        const bool staged = cnt <= kOffCap;
+        uint32_t shift = 0;
+        const uint8_t* og = reinterpret_cast<const uint8_t*>(P.off + ra);
+        if (staged && cnt) {
+          shift = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(og) & 15u);
+          stage_copy_edges(so + shift, og, cnt * 8, lane, o_off, o_len);
+        }
+        if (lane == 0) {
+          hd->t = static_cast<long long>(t);
+          hd->sbase = sbase;
+          hd->chunk0 = chunk0;
+          hd->lo = max(0LL, chunk0);
+          hd->hi = min(N, chunk0 + kT);
+          hd->stg_hi = stg_hi;
+          hd->ra = ra;
+          hd->rb = rb;
+          hd->off_shift = shift;
+          hd->off_staged = staged ? 1u : 0u;
+        }
+        __syncwarp();
+        if (lane == 0) {
+          mbar_arrive_expect_tx(&full[s], b_len + o_len);
+          if (b_len) tma_load_1d(d + b_off, g + b_off, b_len, &full[s]);
+          if (o_len) tma_load_1d(so + shift + o_off, og + o_off, o_len, &full[s]);
+        }
+      }
+      ++it;
+    }
+  }
+  // end-of-work marker
+  const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
+  mbar_wait(&empty[s], ph ^ 1u);
+  if (lane == 0) {
+    reinterpret_cast<StageHdr*>(smem + Layout::hdr + s * 128)->t = -1;
+    mbar_arrive(&full[s]);
+  }
+}
+
+// ---------------------------------------------------------------- map warps
+template <int W>
+__device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, const TileView& tv,
+                                long long p0, long long i0, bool live) {
+  using F = PairFmt<W>;
+  const long long N = static_cast<long long>(P.nbytes);
+  uint32_t x[8];
+  uint32_t vm = 0, R = 0;
+  if (live) {
+    const uint4 c0 = *reinterpret_cast<const uint4*>(tv.sb + i0);
+    const uint4 c1 = *reinterpret_cast<const uint4*>(tv.sb + i0 + 16);
+    x[0] = c0.x; x[1] = c0.y; x[2] = c0.z; x[3] = c0.w;
+    x[4] = c1.x; x[5] = c1.y; x[6] = c1.z; x[7] = c1.w;
+    vm = range_mask32(p0, 0, N);
+    R = bits32(tv.bm, i0);
+  } else {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) x[i] = 0;
+  }
+  uint32_t emit_mask = 0;       // bit j: an emission anchored at p0 + j
+  uint32_t aux[2] = {0, 0};     // II: closing-quote distance for up to two markers
+  uint32_t wm = 0, nb = 0;
+  if constexpr (W == kWC) {
+    if (live) {
+#pragma unroll
+      for (int i = 0; i < 8; ++i) wm |= word_mask4(x[i]) << (4 * i);
+      wm &= vm;
+      uint32_t prevw = 0;
+      if (p0 - 1 >= 0 && p0 - 1 < N) prevw = is_word_byte(tv.sb[i0 - 1]) ? 1u : 0u;
+      nb = ~wm | R;                                            // a word cannot continue here
+      emit_mask = wm & 0xFFFFu & ~(((wm << 1) | prevw) & ~R);  // word starts (C-2 WC)
+    }
+  } else if constexpr (W == kSM) {
+    if (live) {
+      const uint32_t b0 = (P.pat[0] & 0xFFu) * 0x01010101u;
+      uint32_t cand = 0;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) cand |= eq_mask4(x[i], b0) << (4 * i);
+      cand &= vm & 0xFFFFu;
+      while (cand) {
+        const uint32_t j = __ffs(cand) - 1;
+        cand &= cand - 1;
+        if (p0 + j + 16 > N) continue;
+        if ((R >> (j + 1)) & 0x7FFFu) continue;             // match must lie inside one record
+        uint32_t w[4];
+        window16(x, j, w);
+        if (w[0] == P.pat[0] && w[1] == P.pat[1] && w[2] == P.pat[2] && w[3] == P.pat[3]) emit_mask |= 1u << j;
+      }
+    }
+  } else if constexpr (W == kII) {
+    if (live) {
+      uint32_t cand = 0;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) cand |= eq_mask4(x[i], 0x3C3C3C3Cu) << (4 * i);  // '<'
+      cand &= vm & 0xFFFFu;
+      int nm = 0;
+      while (cand) {
+        const uint32_t j = __ffs(cand) - 1;
+        cand &= cand - 1;
+        if (p0 + j + 9 > N) continue;
+        if ((R >> (j + 1)) & 0xFFu) continue;               // marker inside one record
+        uint32_t w[4];
+        window16(x, j, w);
+        // "<a href=\"" little-endian: 3C 61 20 68 | 72 65 66 3D | 22
+        if (w[0] != 0x6820613Cu || w[1] != 0x3D666572u || (w[2] & 0xFFu) != 0x22u) continue;
+        const long long q0 = p0 + j + 9;
+        const long long q = find_quote(P, tv, q0, p0 + j);
+        if (q > q0 && nm < 2) {
+          aux[nm++] = static_cast<uint32_t>(q - q0);
+          emit_mask |= 1u << j;
+        }
+      }
+    }
+  }
+  // ---- reserve one warp result, then lane-major emission rounds
+  const uint32_t cnt = __popc(emit_mask);
+  const uint32_t total = __reduce_add_sync(kFull, cnt);
+  if (total == 0) return;
+  const Slot slot = reserve(oc, total, P.out_cap);
+  uint8_t* half = outh + slot.half * kOutHalf;
+  uint64_t* sh = reinterpret_cast<uint64_t*>(half);
+  uint64_t* sk = sh + F::kCap;
+  uint8_t* sv = half + F::kCap * (F::kKref ? 16 : 8);
+  uint32_t k = slot.base;
+  uint32_t m_left = emit_mask;
+  int nth = 0;
+  while (__any_sync(kFull, m_left != 0)) {
+    const bool act = m_left != 0;
+    const uint32_t m = __ballot_sync(kFull, act);
+    if (act) {
+      const uint32_t j = __ffs(m_left) - 1;
+      m_left &= m_left - 1;
+      const uint32_t idx = k + __popc(m & lanemask_lt());
+      const long long p = p0 + j;
+      if constexpr (W == kWC) {
+        const uint32_t rest = nb >> (j + 1);
+        uint32_t len = rest ? static_cast<uint32_t>(__ffs(rest)) : slow_word_len(P, tv, p, p0 + 32);
+        uint64_t key;
+        if (len <= 7) {
+          key = inline_key(window8(x, j), len);
+        } else {
+          const uint8_t* kp = (p + len <= tv.stg_hi) ? tv.sb + (p - tv.sbase) : P.rec + p;
+          key = hashed_key(hash_bytes(kp, len, P.hash_seed), (P.flags & 8u) != 0);
+        }
+        if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
+        sh[idx] = key;
+        sk[idx] = (reinterpret_cast<uint64_t>(P.rec + p) << 16) | len;
+        reinterpret_cast<uint32_t*>(sv)[idx] = 1u;
+      } else if constexpr (W == kSM) {
+        sh[idx] = P.gbase + static_cast<uint64_t>(p);
+      } else if constexpr (W == kII) {
+        uint32_t len = nth == 0 ? aux[0] : aux[1];
+        ++nth;
+        const long long q0 = p + 9;
+        const uint8_t* kp = (q0 + len <= tv.stg_hi) ? tv.sb + (q0 - tv.sbase) : P.rec + q0;
+        if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
+        sh[idx] = key_of(kp, len, P);
+        sk[idx] = (reinterpret_cast<uint64_t>(P.rec + q0) << 16) | len;
+        reinterpret_cast<uint64_t*>(sv)[idx] = P.gbase + static_cast<uint64_t>(q0);
+      }
+    }
+    k += __popc(m);
+  }
+  commit(oc, slot, total);
+}
+
+template <int W>
+__device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
+  using F = PairFmt<W>;
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t tid = threadIdx.x;  // 0 .. kNMap*32-1
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout::full);
+  uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout::empty);
+  uint8_t* outh = smem + Layout::out;
+  const float* cent = reinterpret_cast<const float*>(smem + Layout::cent);
+  for (uint32_t it = 0;; ++it) {
+    const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
+    mbar_wait(&full[s], ph);
+    const StageHdr hd = *reinterpret_cast<const StageHdr*>(smem + Layout::hdr + s * 128);
+    if (hd.t < 0) break;
+    const uint8_t* sb = smem + Layout::bytes + s * kStageBytes;
+    if constexpr (W == kKM) {
+      const uint64_t i = static_cast<uint64_t>(hd.lo) + tid;
+      const bool valid = i < static_cast<uint64_t>(hd.hi);
+      // stage byte offset of the first point: same 16-B phase as the source
+      const uint8_t* pt = sb + ((reinterpret_cast<uintptr_t>(P.rec) + static_cast<uint64_t>(hd.lo) * 32) & 15u) +
+                          static_cast<uint64_t>(tid) * 32;
+      float x[8];
+      uint32_t best = 0;
+      if (valid) {
+        const float4 a = reinterpret_cast<const float4*>(pt)[0];
+        const float4 b = reinterpret_cast<const float4*>(pt)[1];
+        x[0] = a.x; x[1] = a.y; x[2] = a.z; x[3] = a.w; x[4] = b.x; x[5] = b.y; x[6] = b.z; x[7] = b.w;
+        float bd = 0.0f;
+        for (uint32_t j = 0; j < P.k; ++j) {   // C-2 KM: fp32 RN, explicit fmaf chain, ties -> lowest j
+          const float4 c0 = reinterpret_cast<const float4*>(cent + j * 8)[0];
+          const float4 c1 = reinterpret_cast<const float4*>(cent + j * 8)[1];
+          float d = 0.0f, e;
+          e = __fsub_rn(x[0], c0.x); d = __fmaf_rn(e, e, d);
+          e = __fsub_rn(x[1], c0.y); d = __fmaf_rn(e, e, d);
+          e = __fsub_rn(x[2], c0.z); d = __fmaf_rn(e, e, d);
+          e = __fsub_rn(x[3], c0.w); d = __fmaf_rn(e, e, d);
+          e = __fsub_rn(x[4], c1.x); d = __fmaf_rn(e, e, d);
+          e = __fsub_rn(x[5], c1.y); d = __fmaf_rn(e, e, d);
+          e = __fsub_rn(x[6], c1.z); d = __fmaf_rn(e, e, d);
+          e = __fsub_rn(x[7], c1.w); d = __fmaf_rn(e, e, d);
+          if (j == 0 || d < bd) { bd = d; best = j; }
+        }
+      }
+      const uint32_t m = __ballot_sync(kFull, valid);
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[s]);   // stage no longer read by this warp
+      if (m) {
+        const uint32_t total = __popc(m);
+        const Slot slot = reserve(oc, total, P.out_cap);
+        if (valid) {
+          const uint32_t idx = slot.base + __popc(m & lanemask_lt());
+          uint8_t* half = outh + slot.half * kOutHalf;
+          reinterpret_cast<uint64_t*>(half)[idx] = best;
+          float4* sv = reinterpret_cast<float4*>(half + F::kCap * 8 + static_cast<size_t>(idx) * 32);
+          sv[0] = make_float4(x[0], x[1], x[2], x[3]);
+          sv[1] = make_float4(x[4], x[5], x[6], x[7]);
+        }
+        commit(oc, slot, total);
+      }
+    } else {
+      // record-start bitmap from the staged (or global) offsets slice
+      uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout::bits + s * kBitBytes);
+      const uint64_t* soff = reinterpret_cast<const uint64_t*>(smem + Layout::offs + s * kOffBytes + hd.off_shift);
+      const uint64_t cnt = hd.rb - hd.ra;
+      for (uint64_t r = tid; r < cnt; r += kNMap * 32) {
+        const uint64_t pos = hd.off_staged ? soff[r] : P.off[hd.ra + r];
+        const long long i = static_cast<long long>(pos) - hd.sbase;
+        atomicOr(&bm[i >> 5], 1u << (i & 31));
+      }
+      named_bar_sync(1, kNMap * 32);
+      TileView tv{sb, bm, hd.sbase, hd.stg_hi};
+      for (uint32_t w = warp; w < kNWin; w += kNMap) {
+        const long long wp = hd.chunk0 + static_cast<long long>(w) * kWin;
+        if (wp >= hd.hi) break;                       // warp-uniform
+        const long long p0 = wp + lane * 16;
+        const bool live = (p0 + 16 > 0) && (p0 < static_cast<long long>(P.nbytes));
+        emit_text_chunk<W>(P, oc, outh, tv, p0, p0 - hd.sbase, live);
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[s]);
+    }
+  }
+  // final flush of the partially filled half (all map warps done)
+  named_bar_sync(2, kNMap * 32);
+  if (threadIdx.x == 0) {
+    const unsigned long long cur = *reinterpret_cast<volatile unsigned long long*>(&oc->cur);
+    const uint32_t gen = static_cast<uint32_t>(cur >> 32), cnt = static_cast<uint32_t>(cur);
+    const uint32_t h = gen & 1u;
+    oc->fcount[h] = cnt;
+    oc->final_gen = gen;
+    oc->is_final = 1;
+    __threadfence_block();
+    mbar_arrive(&oc->req[h]);
+  }
+}
+
+template <int W>
+__global__ void __launch_bounds__(kThreads, 1) k_map(Params P) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  OutCtl* oc = reinterpret_cast<OutCtl*>(smem + Layout::ctl);
+  if (threadIdx.x == 0) {
+    oc->cur = 0;
+    oc->committed[0] = oc->committed[1] = 0;
+    oc->fcount[0] = oc->fcount[1] = 0;
+    oc->final_gen = 0;
+    oc->is_final = 0;
+    mbar_init(&oc->req[0], 1); mbar_init(&oc->req[1], 1);
+    mbar_init(&oc->done[0], 1); mbar_init(&oc->done[1], 1);
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout::full);
+    uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout::empty);
+    for (int s = 0; s < kStages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], kNMap); }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if constexpr (W == kKM) {
+    float* cent = reinterpret_cast<float*>(smem + Layout::cent);
+    for (uint32_t i = threadIdx.x; i < P.k * 8; i += blockDim.x) cent[i] = P.cent[i];
+  }
+  __syncthreads();
+  const uint32_t warp = threadIdx.x >> 5;
+  if (warp == kProdWarp) producer_loop<W>(P, smem);
+  else if (warp == kFlushWarp) flush_loop<W>(P, smem, oc);
+  else map_loop<W>(P, smem, oc);
+}
+
+// tile bounds: record starts inside the staged window [w_lo, w_hi) of each text tile
+__global__ void k_tile_bounds(const uint64_t* off, uint64_t n, uint64_t ntiles, long long a0, uint64_t* tb) {
+  const uint64_t t = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (t >= ntiles) return;
+  const long long chunk0 = static_cast<long long>(t) * kT - a0;
+  const long long w_lo = max(0LL, chunk0 - kLead), w_hi = chunk0 + kT + kHalo;
+  uint64_t res[2];
+  const long long qs[2] = {w_lo, w_hi};
+  for (int k = 0; k < 2; ++k) {  // lower_bound over offsets[0..n]
+    uint64_t lo = 0, hi = n + 1;
+    const uint64_t q = static_cast<uint64_t>(qs[k]);
+    while (lo < hi) {
+      const uint64_t mid = (lo + hi) >> 1;
+      if (off[mid] < q) lo = mid + 1; else hi = mid;
+    }
+    res[k] = lo;
+  }
+  tb[2 * t] = res[0];
+  tb[2 * t + 1] = res[1];
+}
+
+template <int W>
+cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
+  using F = PairFmt<W>;
+  Params P{};
+  P.rec = a.records;
+  P.off = a.offsets;
+  P.n = a.n;
+  P.nbytes = a.nbytes;
+  P.a0 = static_cast<long long>(reinterpret_cast<uintptr_t>(a.records) & 15u);
+  P.ntiles = map_tiles(a);
+  P.gbase = a.gbase;
+  for (int i = 0; i < 4; ++i)
+    P.pat[i] = a.pattern[4 * i] | (a.pattern[4 * i + 1] << 8) | (a.pattern[4 * i + 2] << 16) |
+               (static_cast<uint32_t>(a.pattern[4 * i + 3]) << 24);
+  P.cent = a.centroids;
+  P.k = a.k;
+  P.oh = a.out.h;
+  P.okref = a.out.kref;
+  P.ov = a.out.v;
+  P.cap_pairs = a.out.cap;
+  P.out_cap = (a.flags & 4u) ? F::kMaxReserve : F::kCap;   // MR_FLAG_FORCE_TINY_OUT
+  P.flags = a.flags;
+  P.st = a.st;
+  P.tb = a.tile_bounds;
+  P.hash_seed = a.hash_seed;
+  if (P.ntiles == 0) return cudaSuccess;
+  if constexpr (W != kKM) {
+    const unsigned blocks = static_cast<unsigned>((P.ntiles + 255) / 256);
+    k_tile_bounds<<<blocks, 256, 0, s>>>(a.offsets, a.n, P.ntiles, P.a0, a.tile_bounds);
+    count_launch();
+  }
+  const size_t smem = Layout::cent + (W == kKM ? static_cast<size_t>(a.k) * 32 : 0);
+  cudaError_t e = cudaFuncSetAttribute(k_map<W>, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
+  if (e != cudaSuccess) return e;
+  int grid = a.grid > 0 ? a.grid : num_sms;
+  if (static_cast<uint64_t>(grid) > P.ntiles) grid = static_cast<int>(P.ntiles);
+  k_map<W><<<grid, kThreads, smem, s>>>(P);
+  count_launch();
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+int vbytes_of(int w) { return w == kWC ? 4 : w == kSM ? 0 : w == kKM ? 32 : 8; }
+bool has_kref(int w) { return w == kWC || w == kII; }
+
+uint64_t map_tiles(const MapArgs& a) {
+  if (a.workload == kKM) return (a.n + kKmPts - 1) / kKmPts;
+  const uint64_t a0 = reinterpret_cast<uintptr_t>(a.records) & 15u;
+  return a.nbytes ? (a.nbytes + a0 + kT - 1) / kT : 0;
+}
+
+cudaError_t launch_map(const MapArgs& a, int num_sms, cudaStream_t s) {
+  switch (a.workload) {
+    case kWC: return launch_w<kWC>(a, num_sms, s);
+    case kSM: return launch_w<kSM>(a, num_sms, s);
+    case kKM: return launch_w<kKM>(a, num_sms, s);
+    case kII: return launch_w<kII>(a, num_sms, s);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+}  // namespace bmr

@@ -1,0 +1,388 @@
+// reduce.cu — group-by-key, part 2 (segment boundaries) and the Reduce phase
+// with output assembly (a9).
+//
+// Segments: after the radix sort equal sort keys are adjacent.  head[i] = (i == 0) ||
+// key[i] != key[i-1].  For hashed keys (top bit set) equal hashes are verified byte-for-byte
+// against the neighbouring pair (C-3 #13: distinct keys must never merge); a mismatch is
+// counted in DevState::collisions and the host re-sorts with a fresh hash (slow path).
+//
+// Reduce (§IV-C, §IV-E): TR = one thread per key set, BR = a block per key
+// set; the paper found TR better for WC's 10,000s of small key sets and BR better for KM's
+// dozens of large ones.  B200 re-derivation, segment-size aware:
+//   * small segments (<= kSmall pairs): one warp per segment, lanes stride the segment and the
+//     warp reduces with shuffles (TR's parallelism across key sets, without per-thread serial
+//     loops over Zipf-heavy sets);
+//   * large segments: split into kLargeTile-pair work items appended to a work list; persistent
+//     blocks reduce one item each and combine with one global atomic per item (BR).
+// KM partial sums are fp32 over <= 32 values per lane, combined in fp64 (north_star: "fp32 on
+// GPU"; tolerance derivation in DESIGN.md).
+#include <algorithm>
+
+#include "common.cuh"
+
+namespace bmr {
+namespace {
+
+constexpr int kSegThreads = 256, kSegIPT = 16, kSegTile = kSegThreads * kSegIPT;
+constexpr uint64_t kSmallWC = 4096, kSmallKM = 1024;
+constexpr uint64_t kLargeTile = 8192;
+
+__device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+__device__ bool key_bytes_equal(uint64_t ka, uint64_t kb) {
+  const uint32_t la = static_cast<uint32_t>(ka & 0xFFFF), lb = static_cast<uint32_t>(kb & 0xFFFF);
+  if (la != lb) return false;
+  const uint8_t* pa = reinterpret_cast<const uint8_t*>(ka >> 16);
+  const uint8_t* pb = reinterpret_cast<const uint8_t*>(kb >> 16);
+  for (uint32_t i = 0; i < la; ++i)
+    if (pa[i] != pb[i]) return false;
+  return true;
+}
+
+__global__ void __launch_bounds__(kSegThreads) k_seg_count(const uint64_t* __restrict__ sk,
+                                                         const uint32_t* __restrict__ perm,
+                                                         const uint64_t* __restrict__ kref, uint64_t m,
+                                                         uint32_t* counts, DevState* st) {
+  __shared__ uint32_t red[kSegThreads / 32];
+  const uint64_t base = static_cast<uint64_t>(blockIdx.x) * kSegTile + static_cast<uint64_t>(threadIdx.x) * kSegIPT;
+  uint32_t heads = 0, coll = 0;
+  uint64_t prev = (base > 0 && base - 1 < m) ? sk[base - 1] : 0;
+  for (int j = 0; j < kSegIPT; ++j) {
+    const uint64_t i = base + j;
+    if (i >= m) break;
+    const uint64_t k = sk[i];
+    if (i == 0 || k != prev) {
+      ++heads;
+    } else if ((k & kHashedBit) && kref) {
+      if (!key_bytes_equal(kref[perm[i]], kref[perm[i - 1]])) ++coll;
+    }
+    prev = k;
+  }
+  if (coll) atomicAdd(&st->collisions, coll);
+  uint32_t w = __reduce_add_sync(0xffffffffu, heads);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = w;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t t = 0;
+    for (int i = 0; i < kSegThreads / 32; ++i) t += red[i];
+    counts[blockIdx.x] = t;
+  }
+}
+
+__global__ void __launch_bounds__(kSegThreads) k_seg_write(const uint64_t* __restrict__ sk, uint64_t m,
+                                                         const uint64_t* __restrict__ tile_base,
+                                                         uint64_t* seg_start) {
+  __shared__ uint32_t wsum[kSegThreads / 32];
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint64_t base = static_cast<uint64_t>(blockIdx.x) * kSegTile + static_cast<uint64_t>(tid) * kSegIPT;
+  uint32_t hm = 0;
+  uint64_t prev = (base > 0 && base - 1 < m) ? sk[base - 1] : 0;
+  for (int j = 0; j < kSegIPT; ++j) {
+    const uint64_t i = base + j;
+    if (i >= m) break;
+    const uint64_t k = sk[i];
+    if (i == 0 || k != prev) hm |= 1u << j;
+    prev = k;
+  }
+  const uint32_t c = __popc(hm);
+  const uint32_t inc = warp_inclusive_add(c);
+  if (lane == 31) wsum[warp] = inc;
+  __syncthreads();
+  uint32_t wpre = 0, tot = 0;
+  for (int w = 0; w < kSegThreads / 32; ++w) {
+    wpre += (w < static_cast<int>(warp)) ? wsum[w] : 0u;
+    tot += wsum[w];
+  }
+  uint64_t r = tile_base[blockIdx.x] + wpre + inc - c;
+  while (hm) {
+    const int j = __ffs(hm) - 1;
+    hm &= hm - 1;
+    seg_start[r++] = base + j;
+  }
+  const uint64_t tile_end = static_cast<uint64_t>(blockIdx.x + 1) * kSegTile;
+  if (tid == 0 && tile_end >= m) seg_start[tile_base[blockIdx.x] + tot] = m;  // sentinel S -> m
+}
+
+// ---------------------------------------------------------------- WordCount reduce (u64 sums)
+__global__ void k_reduce_wc_small(const uint64_t* __restrict__ seg, uint64_t nseg, const uint32_t* __restrict__ perm,
+                                  const uint32_t* __restrict__ v, uint64_t* counts, uint64_t* worklist,
+                                  DevState* st) {
+  const uint64_t gw = (blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x) >> 5;
+  const uint64_t nw = (static_cast<uint64_t>(gridDim.x) * blockDim.x) >> 5;
+  const uint32_t lane = threadIdx.x & 31;
+  for (uint64_t s = gw; s < nseg; s += nw) {
+    const uint64_t a = seg[s], b = seg[s + 1], size = b - a;
+    if (size <= kSmallWC) {
+      uint64_t sum = 0;
+      for (uint64_t i = a + lane; i < b; i += 32) sum += v[perm[i]];
+      sum = warp_sum_u64(sum);
+      if (lane == 0) counts[s] = sum;
+    } else if (lane == 0) {
+      counts[s] = 0;
+      const uint64_t nt = (size + kLargeTile - 1) / kLargeTile;
+      const uint64_t at = atomicAdd(&st->large_items, static_cast<unsigned long long>(nt));
+      for (uint64_t t = 0; t < nt; ++t) worklist[at + t] = (s << 24) | t;
+    }
+  }
+}
+
+__global__ void __launch_bounds__(256) k_reduce_wc_large(const uint64_t* __restrict__ seg,
+                                                       const uint32_t* __restrict__ perm,
+                                                       const uint32_t* __restrict__ v, uint64_t* counts,
+                                                       const uint64_t* __restrict__ worklist, DevState* st) {
+  __shared__ unsigned long long item;
+  __shared__ uint64_t red[8];
+  const unsigned long long nitems = st->large_items;
+  for (;;) {
+    if (threadIdx.x == 0) item = atomicAdd(&st->large_done, 1ULL);
+    __syncthreads();
+    const unsigned long long it = item;
+    if (it >= nitems) break;
+    const uint64_t w = worklist[it], s = w >> 24, t = w & 0xFFFFFF;
+    const uint64_t a = seg[s] + t * kLargeTile, b = min(seg[s + 1], a + kLargeTile);
+    uint64_t sum = 0;
+    for (uint64_t i = a + threadIdx.x; i < b; i += blockDim.x) sum += v[perm[i]];
+    sum = warp_sum_u64(sum);
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = sum;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      uint64_t tot = 0;
+      for (int i = 0; i < 8; ++i) tot += red[i];
+      atomicAdd(reinterpret_cast<unsigned long long*>(&counts[s]), static_cast<unsigned long long>(tot));
+    }
+    __syncthreads();
+  }
+}
+
+// ---------------------------------------------------------------- KMeans reduce
+__device__ __forceinline__ void load_point(const uint8_t* v, uint32_t p, float (&x)[8]) {
+  const float4* q = reinterpret_cast<const float4*>(v + static_cast<uint64_t>(p) * 32);
+  const float4 a = q[0], b = q[1];
+  x[0] = a.x; x[1] = a.y; x[2] = a.z; x[3] = a.w; x[4] = b.x; x[5] = b.y; x[6] = b.z; x[7] = b.w;
+}
+
+__global__ void k_reduce_km_small(const uint64_t* __restrict__ seg, uint64_t nseg, const uint64_t* __restrict__ sk,
+                                  const uint32_t* __restrict__ perm, const uint8_t* __restrict__ v, double* sums,
+                                  unsigned long long* cnts, uint32_t k, uint64_t* worklist, DevState* st) {
+  const uint64_t gw = (blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x) >> 5;
+  const uint64_t nw = (static_cast<uint64_t>(gridDim.x) * blockDim.x) >> 5;
+  const uint32_t lane = threadIdx.x & 31;
+  for (uint64_t s = gw; s < nseg; s += nw) {
+    const uint64_t a = seg[s], b = seg[s + 1], size = b - a;
+    const uint64_t cid = sk[a];
+    if (cid >= k) continue;
+    if (size <= kSmallKM) {
+      float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+      for (uint64_t i = a + lane; i < b; i += 32) {   // <= 32 fp32 adds per lane
+        float x[8];
+        load_point(v, perm[i], x);
+#pragma unroll
+        for (int t = 0; t < 8; ++t) acc[t] = __fadd_rn(acc[t], x[t]);
+      }
+#pragma unroll
+      for (int t = 0; t < 8; ++t) {
+        double d = static_cast<double>(acc[t]);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(0xffffffffu, d, o);
+        if (lane == 0) atomicAdd(&sums[cid * 8 + t], d);
+      }
+      if (lane == 0) atomicAdd(&cnts[cid], static_cast<unsigned long long>(size));
+    } else if (lane == 0) {
+      atomicAdd(&cnts[cid], static_cast<unsigned long long>(size));
+      const uint64_t nt = (size + kLargeTile - 1) / kLargeTile;
+      const uint64_t at = atomicAdd(&st->large_items, static_cast<unsigned long long>(nt));
+      for (uint64_t t = 0; t < nt; ++t) worklist[at + t] = (s << 24) | t;
+    }
+  }
+}
+
+__global__ void __launch_bounds__(256) k_reduce_km_large(const uint64_t* __restrict__ seg,
+                                                       const uint64_t* __restrict__ sk,
+                                                       const uint32_t* __restrict__ perm,
+                                                       const uint8_t* __restrict__ v, double* sums,
+                                                       const uint64_t* __restrict__ worklist, DevState* st) {
+  __shared__ unsigned long long item;
+  __shared__ double red[8][8];
+  const unsigned long long nitems = st->large_items;
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (;;) {
+    if (threadIdx.x == 0) item = atomicAdd(&st->large_done, 1ULL);
+    __syncthreads();
+    const unsigned long long it = item;
+    if (it >= nitems) break;
+    const uint64_t w = worklist[it], s = w >> 24, t = w & 0xFFFFFF;
+    const uint64_t a = seg[s] + t * kLargeTile, b = min(seg[s + 1], a + kLargeTile);
+    const uint64_t cid = sk[seg[s]];
+    float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};           // kLargeTile / 256 = 32 fp32 adds per thread
+    for (uint64_t i = a + threadIdx.x; i < b; i += blockDim.x) {
+      float x[8];
+      load_point(v, perm[i], x);
+#pragma unroll
+      for (int q = 0; q < 8; ++q) acc[q] = __fadd_rn(acc[q], x[q]);
+    }
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      double d = static_cast<double>(acc[q]);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(0xffffffffu, d, o);
+      if (lane == 0) red[warp][q] = d;
+    }
+    __syncthreads();
+    if (threadIdx.x < 8) {
+      double d = 0;
+      for (int ww = 0; ww < 8; ++ww) d += red[ww][threadIdx.x];
+      atomicAdd(&sums[cid * 8 + threadIdx.x], d);
+    }
+    __syncthreads();
+  }
+}
+
+__global__ void k_km_finalize(const double* sums, const unsigned long long* cnts, const float* cent, uint32_t k,
+                              uint8_t* vals, uint64_t* val_off, uint8_t* keys, uint64_t* key_off) {
+  const uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
+  if (j > k) return;
+  if (j == k) { val_off[k] = 40ULL * k; key_off[k] = 4ULL * k; return; }
+  const unsigned long long c = cnts[j];
+  float* o = reinterpret_cast<float*>(vals + 40ULL * j);
+  for (int t = 0; t < 8; ++t)
+    o[t] = c ? static_cast<float>(__ddiv_rn(sums[j * 8 + t], static_cast<double>(c))) : cent[j * 8 + t];
+  *reinterpret_cast<unsigned long long*>(vals + 40ULL * j + 32) = c;
+  *reinterpret_cast<uint32_t*>(keys + 4ULL * j) = j;
+  val_off[j] = 40ULL * j;
+  key_off[j] = 4ULL * j;
+}
+
+// ---------------------------------------------------------------- output assembly
+__global__ void k_key_lengths(const uint64_t* seg, uint64_t nseg, const uint32_t* perm, const uint64_t* kref,
+                              uint64_t* lens) {
+  const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (s < nseg) lens[s] = kref[perm[seg[s]]] & 0xFFFF;
+}
+__global__ void k_key_copy(const uint64_t* seg, uint64_t nseg, const uint32_t* perm, const uint64_t* kref,
+                           const uint64_t* key_off, uint8_t* keys) {
+  // one warp per key: lanes copy bytes
+  const uint64_t s = (blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x) >> 5;
+  const uint32_t lane = threadIdx.x & 31;
+  if (s >= nseg) return;
+  const uint64_t kr = kref[perm[seg[s]]];
+  const uint8_t* src = reinterpret_cast<const uint8_t*>(kr >> 16);
+  const uint32_t len = static_cast<uint32_t>(kr & 0xFFFF);
+  uint8_t* dst = keys + key_off[s];
+  for (uint32_t i = lane; i < len; i += 32) dst[i] = src[i];
+}
+__global__ void k_gather_u64(const uint32_t* perm, const uint64_t* v, uint64_t m, uint64_t* out) {
+  const uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (i < m) out[i] = v[perm[i]];
+}
+__global__ void k_offsets_scaled(const uint64_t* seg, uint64_t nseg, uint64_t scale, uint64_t* out) {
+  const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (s <= nseg) out[s] = seg[s] * scale;
+}
+__global__ void k_iota_scaled(uint64_t n, uint64_t scale, uint64_t* out) {
+  const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (s <= n) out[s] = s * scale;
+}
+__global__ void k_rehash(uint64_t* h, const uint64_t* kref, uint64_t m, uint64_t seed) {
+  const uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (i >= m) return;
+  const uint64_t kr = kref[i];
+  const uint32_t len = static_cast<uint32_t>(kr & 0xFFFF);
+  if (len <= 7) return;  // inline keys are exact already
+  h[i] = hashed_key(hash_bytes(reinterpret_cast<const uint8_t*>(kr >> 16), len, seed), false);
+}
+
+inline unsigned blocks_for(uint64_t n, unsigned t) { return static_cast<unsigned>((n + t - 1) / t); }
+
+}  // namespace
+
+cudaError_t launch_seg_count(const uint64_t* skeys, const uint32_t* perm, const uint64_t* kref, uint64_t m,
+                             uint32_t* counts, DevState* st, cudaStream_t s) {
+  if (m == 0) return cudaSuccess;
+  k_seg_count<<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, perm, kref, m, counts, st);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_seg_write(const uint64_t* skeys, uint64_t m, const uint64_t* tile_base, uint64_t* seg_start,
+                             cudaStream_t s) {
+  if (m == 0) return cudaMemsetAsync(seg_start, 0, sizeof(uint64_t), s);
+  k_seg_write<<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, m, tile_base, seg_start);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_key_lengths(const uint64_t* seg_start, uint64_t nseg, const uint32_t* perm, const uint64_t* kref,
+                               uint64_t* lens, cudaStream_t s) {
+  if (nseg == 0) return cudaSuccess;
+  k_key_lengths<<<blocks_for(nseg, 256), 256, 0, s>>>(seg_start, nseg, perm, kref, lens);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_key_copy(const uint64_t* seg_start, uint64_t nseg, const uint32_t* perm, const uint64_t* kref,
+                            const uint64_t* key_off, uint8_t* keys, cudaStream_t s) {
+  if (nseg == 0) return cudaSuccess;
+  k_key_copy<<<blocks_for(nseg * 32, 256), 256, 0, s>>>(seg_start, nseg, perm, kref, key_off, keys);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_reduce_wc(const uint64_t* seg_start, uint64_t nseg, const uint32_t* perm, const uint8_t* v,
+                             uint64_t* counts, uint64_t* worklist, DevState* st, int num_sms, cudaStream_t s) {
+  if (nseg == 0) return cudaSuccess;
+  cudaError_t e = cudaMemsetAsync(&st->large_items, 0, 2 * sizeof(unsigned long long), s);
+  if (e != cudaSuccess) return e;
+  const unsigned g1 = static_cast<unsigned>(std::min<uint64_t>(blocks_for(nseg * 32, 256), 148ULL * 64));
+  k_reduce_wc_small<<<g1, 256, 0, s>>>(seg_start, nseg, perm, reinterpret_cast<const uint32_t*>(v), counts, worklist,
+                                       st);
+  count_launch();
+  k_reduce_wc_large<<<num_sms * 4, 256, 0, s>>>(seg_start, perm, reinterpret_cast<const uint32_t*>(v), counts,
+                                                worklist, st);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_reduce_km(const uint64_t* seg_start, uint64_t nseg, const uint64_t* skeys, const uint32_t* perm,
+                             const uint8_t* v, double* sums, unsigned long long* cnts, uint32_t k,
+                             uint64_t* worklist, DevState* st, int num_sms, cudaStream_t s) {
+  cudaError_t e = cudaMemsetAsync(&st->large_items, 0, 2 * sizeof(unsigned long long), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(sums, 0, sizeof(double) * 8 * k, s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(cnts, 0, sizeof(unsigned long long) * k, s);
+  if (e != cudaSuccess || nseg == 0) return e;
+  const unsigned g1 = static_cast<unsigned>(std::min<uint64_t>(blocks_for(nseg * 32, 256), 148ULL * 64));
+  k_reduce_km_small<<<g1, 256, 0, s>>>(seg_start, nseg, skeys, perm, v, sums, cnts, k, worklist, st);
+  count_launch();
+  k_reduce_km_large<<<num_sms * 4, 256, 0, s>>>(seg_start, skeys, perm, v, sums, worklist, st);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_km_finalize(const double* sums, const unsigned long long* cnts, const float* centroids, uint32_t k,
+                               uint8_t* vals, uint64_t* val_off, uint8_t* keys, uint64_t* key_off, cudaStream_t s) {
+  k_km_finalize<<<blocks_for(k + 1, 128), 128, 0, s>>>(sums, cnts, centroids, k, vals, val_off, keys, key_off);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_gather_u64(const uint32_t* perm, const uint8_t* v, uint64_t m, uint64_t* out, cudaStream_t s) {
+  if (m == 0) return cudaSuccess;
+  k_gather_u64<<<blocks_for(m, 256), 256, 0, s>>>(perm, reinterpret_cast<const uint64_t*>(v), m, out);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_offsets_scaled(const uint64_t* seg_start, uint64_t nseg, uint64_t scale, uint64_t* out,
+                                  cudaStream_t s) {
+  k_offsets_scaled<<<blocks_for(nseg + 1, 256), 256, 0, s>>>(seg_start, nseg, scale, out);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_iota_scaled(uint64_t n, uint64_t scale, uint64_t* out, cudaStream_t s) {
+  k_iota_scaled<<<blocks_for(n + 1, 256), 256, 0, s>>>(n, scale, out);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_rehash(uint64_t* h, const uint64_t* kref, uint64_t m, uint64_t seed, cudaStream_t s) {
+  if (m == 0) return cudaSuccess;
+  k_rehash<<<blocks_for(m, 256), 256, 0, s>>>(h, kref, m, seed);
+  count_launch();
+  return cudaGetLastError();
+}
+
+}  // namespace bmr

@@ -1,0 +1,281 @@
+// sort.cu — group-by-key, part 1: a hand-written onesweep-style LSD radix
+// sort of the 64-bit intermediate sort keys with a u32 permutation payload, plus the generic
+// single-pass (decoupled look-back) exclusive scan used by the segment and output steps.
+//
+// The paper reuses Mars's shuffle unchanged and does not describe it (PAPER.md L295, L305:
+// "Word Count is an example where there is a large shuffle phase").  B200 design:
+//   * one histogram pass computes all eight 8-bit digit histograms (k_hist); digits whose
+//     histogram has a single non-empty bin are skipped by the host (constant-digit skip);
+//   * each remaining digit is one pass of k_onesweep: a 4096-key tile is ranked with
+//     warp-private counters + match.any (stable: warp-striped order == element order), the tile
+//     count of every digit is published and the exclusive prefix over earlier tiles is obtained
+//     by decoupled look-back on per-(tile, digit) status words; keys and payload are then
+//     scattered through SMEM so that global writes are contiguous runs per digit.
+// Look-back status words: [epoch:30 | kind:2 | value:32]; every launch uses a fresh epoch so
+// the status buffer never needs clearing.
+#include "common.cuh"
+
+namespace bmr {
+namespace {
+
+constexpr uint32_t kAgg = 1u, kPrefix = 2u;
+constexpr int kWarps = kSortThreads / 32;
+
+__device__ __forceinline__ uint64_t pack_status(uint32_t epoch, uint32_t kind, uint32_t v) {
+  return (static_cast<uint64_t>(epoch) << 34) | (static_cast<uint64_t>(kind) << 32) | v;
+}
+
+__global__ void __launch_bounds__(256) k_hist(const uint64_t* __restrict__ keys, uint64_t m, uint32_t* hist) {
+  __shared__ uint32_t sh[8 * 256];
+  for (int i = threadIdx.x; i < 8 * 256; i += blockDim.x) sh[i] = 0;
+  __syncthreads();
+  const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
+  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i < m; i += stride) {
+    const uint64_t k = __ldcs(keys + i);
+#pragma unroll
+    for (int d = 0; d < 8; ++d) atomicAdd(&sh[d * 256 + ((k >> (8 * d)) & 255u)], 1u);
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < 8 * 256; i += blockDim.x)
+    if (sh[i]) atomicAdd(&hist[i], sh[i]);
+}
+
+struct SortSmem {
+  uint64_t keys[kSortTile];
+  uint32_t idx[kSortTile];
+  uint32_t wcnt[kWarps][256];
+  uint32_t dstart[256];
+  uint32_t goff[256];
+  uint32_t wsum[kWarps];
+  uint32_t tile;
+};
+
+template <bool kFirst>
+__global__ void __launch_bounds__(kSortThreads) k_onesweep(const uint64_t* __restrict__ keys_in,
+                                                         const uint32_t* __restrict__ idx_in,
+                                                         uint64_t* __restrict__ keys_out,
+                                                         uint32_t* __restrict__ idx_out, uint64_t m,
+                                                         uint32_t shift, const uint32_t* __restrict__ bases,
+                                                         uint64_t* status, uint32_t epoch,
+                                                         unsigned int* tile_counter) {
+  extern __shared__ __align__(16) uint8_t raw[];
+  SortSmem& S = *reinterpret_cast<SortSmem*>(raw);
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tid == 0) S.tile = atomicAdd(tile_counter, 1u);
+  for (uint32_t i = tid; i < kWarps * 256; i += kSortThreads) (&S.wcnt[0][0])[i] = 0;
+  __syncthreads();
+  const uint32_t tile = S.tile;
+  const uint64_t tbase = static_cast<uint64_t>(tile) * kSortTile;
+  const uint64_t wbase = tbase + static_cast<uint64_t>(warp) * 32 * kSortIPT;
+  uint64_t key[kSortIPT];
+  uint32_t idx[kSortIPT];
+  uint32_t rank[kSortIPT];
+#pragma unroll
+  for (int j = 0; j < kSortIPT; ++j) {
+    const uint64_t e = wbase + j * 32 + lane;
+    const bool v = e < m;
+    key[j] = v ? keys_in[e] : ~0ULL;  // padding sorts last (digit 255, after every real key)
+    idx[j] = kFirst ? static_cast<uint32_t>(e) : (v ? idx_in[e] : 0u);
+  }
+  // stable warp-level ranking (element order == (j, lane) order inside the warp)
+#pragma unroll
+  for (int j = 0; j < kSortIPT; ++j) {
+    const uint32_t d = static_cast<uint32_t>(key[j] >> shift) & 255u;
+    const uint32_t peers = __match_any_sync(0xffffffffu, d);
+    const uint32_t leader = __ffs(peers) - 1;
+    uint32_t before = 0;
+    if (lane == leader) {
+      before = S.wcnt[warp][d];
+      S.wcnt[warp][d] = before + __popc(peers);
+    }
+    before = __shfl_sync(0xffffffffu, before, leader);
+    rank[j] = before + __popc(peers & lanemask_lt());
+  }
+  __syncthreads();
+  // per digit: warp-exclusive offsets, tile count, tile-local digit start, global offset
+  uint32_t tcount = 0;
+  {
+    const uint32_t d = tid;  // kSortThreads == 256
+    uint32_t run = 0;
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) {
+      const uint32_t c = S.wcnt[w][d];
+      S.wcnt[w][d] = run;
+      run += c;
+    }
+    tcount = run;
+    // block exclusive scan of tcount over digits
+    const uint32_t inc = warp_inclusive_add(tcount);
+    if (lane == 31) S.wsum[warp] = inc;
+    __syncthreads();
+    uint32_t wpre = 0;
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) wpre += (w < static_cast<int>(warp)) ? S.wsum[w] : 0u;
+    S.dstart[d] = wpre + inc - tcount;
+    // decoupled look-back for digit d
+    uint64_t* my = status + static_cast<uint64_t>(tile) * 256 + d;
+    uint32_t excl = 0;
+    if (tile == 0) {
+      st_volatile_u64(my, pack_status(epoch, kPrefix, tcount));
+    } else {
+      st_volatile_u64(my, pack_status(epoch, kAgg, tcount));
+      long long p = static_cast<long long>(tile) - 1;
+      while (p >= 0) {
+        const uint64_t s = ld_volatile_u64(status + static_cast<uint64_t>(p) * 256 + d);
+        const uint32_t ep = static_cast<uint32_t>(s >> 34), kind = static_cast<uint32_t>(s >> 32) & 3u;
+        if (ep != epoch || kind == 0) continue;
+        excl += static_cast<uint32_t>(s);
+        if (kind == kPrefix) break;
+        --p;
+      }
+      st_volatile_u64(my, pack_status(epoch, kPrefix, excl + tcount));
+    }
+    S.goff[d] = bases[d] + excl;
+  }
+  __syncthreads();
+  // scatter into SMEM in tile-sorted order
+#pragma unroll
+  for (int j = 0; j < kSortIPT; ++j) {
+    const uint32_t d = static_cast<uint32_t>(key[j] >> shift) & 255u;
+    const uint32_t lp = S.dstart[d] + S.wcnt[warp][d] + rank[j];
+    S.keys[lp] = key[j];
+    S.idx[lp] = idx[j];
+  }
+  __syncthreads();
+  const uint32_t nvalid = static_cast<uint32_t>(min(static_cast<uint64_t>(kSortTile), m - tbase));
+  for (uint32_t i = tid; i < nvalid; i += kSortThreads) {
+    const uint64_t k = S.keys[i];
+    const uint32_t d = static_cast<uint32_t>(k >> shift) & 255u;
+    const uint32_t pos = S.goff[d] + (i - S.dstart[d]);
+    keys_out[pos] = k;
+    idx_out[pos] = S.idx[i];
+  }
+}
+
+// ---- single-pass exclusive scan (u32 or u64 input -> u64 output), decoupled look-back ----
+constexpr int kScanThreads = 256, kScanIPT = 8, kScanTile = kScanThreads * kScanIPT;
+
+template <typename T>
+__global__ void __launch_bounds__(kScanThreads) k_scan(const T* __restrict__ in, uint64_t* out, uint64_t n,
+                                                     unsigned long long* total, uint64_t* status, uint32_t epoch,
+                                                     unsigned int* tile_counter) {
+  __shared__ uint64_t wsum[kScanThreads / 32];
+  __shared__ uint64_t s_excl;
+  __shared__ uint32_t s_tile;
+  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tid == 0) s_tile = atomicAdd(tile_counter, 1u);
+  __syncthreads();
+  const uint32_t tile = s_tile;
+  const uint64_t base = static_cast<uint64_t>(tile) * kScanTile + static_cast<uint64_t>(tid) * kScanIPT;
+  uint64_t v[kScanIPT];
+  uint64_t tsum = 0;
+#pragma unroll
+  for (int j = 0; j < kScanIPT; ++j) {
+    v[j] = (base + j < n) ? static_cast<uint64_t>(in[base + j]) : 0ULL;
+    tsum += v[j];
+  }
+  const uint64_t inc = warp_inclusive_add64(tsum);
+  if (lane == 31) wsum[warp] = inc;
+  __syncthreads();
+  uint64_t wpre = 0, tile_sum = 0;
+#pragma unroll
+  for (int w = 0; w < kScanThreads / 32; ++w) {
+    wpre += (w < static_cast<int>(warp)) ? wsum[w] : 0ULL;
+    tile_sum += wsum[w];
+  }
+  if (tid == 0) {
+    // status layout per tile: [flag, aggregate, inclusive prefix]
+    uint64_t* my = status + 3ULL * tile;
+    uint64_t excl = 0;
+    if (tile == 0) {
+      st_volatile_u64(my + 2, tile_sum);
+      __threadfence();
+      st_volatile_u64(my, pack_status(epoch, kPrefix, 0));
+    } else {
+      st_volatile_u64(my + 1, tile_sum);
+      __threadfence();
+      st_volatile_u64(my, pack_status(epoch, kAgg, 0));
+      long long p = static_cast<long long>(tile) - 1;
+      while (p >= 0) {
+        const uint64_t f = ld_volatile_u64(status + 3ULL * p);
+        const uint32_t ep = static_cast<uint32_t>(f >> 34), kind = static_cast<uint32_t>(f >> 32) & 3u;
+        if (ep != epoch || kind == 0) continue;
+        __threadfence();
+        if (kind == kPrefix) { excl += ld_volatile_u64(status + 3ULL * p + 2); break; }
+        excl += ld_volatile_u64(status + 3ULL * p + 1);
+        --p;
+      }
+      st_volatile_u64(my + 2, excl + tile_sum);
+      __threadfence();
+      st_volatile_u64(my, pack_status(epoch, kPrefix, 0));
+    }
+    s_excl = excl;
+    if (total && (static_cast<uint64_t>(tile) + 1) * kScanTile >= n) *total = excl + tile_sum;
+  }
+  __syncthreads();
+  uint64_t run = s_excl + wpre + inc - tsum;
+#pragma unroll
+  for (int j = 0; j < kScanIPT; ++j) {
+    if (base + j < n) out[base + j] = run;
+    run += v[j];
+  }
+}
+
+}  // namespace
+
+cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int num_sms, cudaStream_t s) {
+  cudaError_t e = cudaMemsetAsync(hist, 0, 8 * 256 * sizeof(uint32_t), s);
+  if (e != cudaSuccess || m == 0) return e;
+  uint64_t blocks = min(static_cast<uint64_t>(num_sms) * 4, (m + 255) / 256);
+  k_hist<<<static_cast<unsigned>(blocks), 256, 0, s>>>(keys, m, hist);
+  count_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out, uint32_t* idx_out,
+                            uint64_t m, int digit, const uint32_t* bases, uint64_t* status, uint32_t epoch,
+                            unsigned int* tile_counter, cudaStream_t s) {
+  if (m == 0) return cudaSuccess;
+  const uint64_t tiles = (m + kSortTile - 1) / kSortTile;
+  const size_t smem = sizeof(SortSmem);
+  cudaError_t e = cudaMemsetAsync(tile_counter, 0, sizeof(unsigned int), s);
+  if (e != cudaSuccess) return e;
+  if (idx_in == nullptr) {
+    cudaFuncSetAttribute(k_onesweep<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
+    k_onesweep<true><<<static_cast<unsigned>(tiles), kSortThreads, smem, s>>>(
+        keys_in, nullptr, keys_out, idx_out, m, 8u * digit, bases + 256 * digit, status, epoch, tile_counter);
+    count_launch();
+  } else {
+    cudaFuncSetAttribute(k_onesweep<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
+    k_onesweep<false><<<static_cast<unsigned>(tiles), kSortThreads, smem, s>>>(
+        keys_in, idx_in, keys_out, idx_out, m, 8u * digit, bases + 256 * digit, status, epoch, tile_counter);
+    count_launch();
+  }
+  return cudaGetLastError();
+}
+
+template <typename T>
+static cudaError_t scan_impl(const T* in, uint64_t* out, uint64_t n, unsigned long long* total, uint64_t* status,
+                             uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
+  if (n == 0) {
+    if (total) return cudaMemsetAsync(total, 0, sizeof(unsigned long long), s);
+    return cudaSuccess;
+  }
+  cudaError_t e = cudaMemsetAsync(tile_counter, 0, sizeof(unsigned int), s);
+  if (e != cudaSuccess) return e;
+  const uint64_t tiles = (n + kScanTile - 1) / kScanTile;
+  k_scan<T><<<static_cast<unsigned>(tiles), kScanThreads, 0, s>>>(in, out, n, total, status, epoch, tile_counter);
+  count_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t launch_scan_u64(const uint64_t* in, uint64_t* out, uint64_t n, unsigned long long* total,
+                            uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
+  return scan_impl<uint64_t>(in, out, n, total, status, epoch, tile_counter, s);
+}
+cudaError_t launch_scan_u32to64(const uint32_t* in, uint64_t* out, uint64_t n, unsigned long long* total,
+                                uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
+  return scan_impl<uint32_t>(in, out, n, total, status, epoch, tile_counter, s);
+}
+
+}  // namespace bmr
