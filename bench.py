@@ -120,8 +120,8 @@ def make_input(cfg, rank, dev):
             "spec": spec, "page0": rank * units, "base": g["base"]}
 
 
-def job_kwargs(inp, flags=0, device=0):
-    kw = {"device": device, "flags": flags}
+def job_kwargs(inp, flags=0, device=0, rank=0, world=1):
+    kw = {"device": device, "flags": flags, "rank": rank, "nranks": world}
     if inp["wl"] == "sm":
         kw["pattern"] = inp["spec"].pattern
     if inp["wl"] == "km":
@@ -154,7 +154,7 @@ def oracle_sample(cfg, sample_units, page0=0):
     return g["data"].size, dt, f"first {sample_units} pages ({sample_units} MiB) of the shard"
 
 
-ORACLE_SAMPLE = {"C1": 1, "C2": 48, "C3": 4 << 20, "C4": 96, "C5": 96}   # ~10-30 s of CPU work
+ORACLE_SAMPLE = {"C1": 1, "C2": 2048, "C3": 16 << 20, "C4": 2048, "C5": 96}   # ~10-30 s of CPU work
 REF_STEP_SAMPLE = {"C1": 1, "C2": 4, "C3": 1 << 19, "C4": 8, "C5": 8}     # per reference-arm step
 
 
@@ -205,6 +205,7 @@ def main():
     ap.add_argument("--impl", default="bmr", choices=["bmr", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--units", type=int, default=0, help="override pages (text) / points (KM) per GPU")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -228,14 +229,21 @@ def main():
             dist.barrier()
         torch.cuda.synchronize()
 
+    if args.units:
+        w = WORKLOADS[args.workload]
+        WORKLOADS[args.workload] = (w[0], w[1] + f" [reduced: {args.units} units]", args.units)
     inp = make_input(args.workload, rank, dev)
     torch.cuda.synchronize()
-    job = bmr.Job(inp["wl"], **job_kwargs(inp, bmr.FLAG_PROFILE, local))
+    job = bmr.Job(inp["wl"], **job_kwargs(inp, bmr.FLAG_PROFILE, local, rank, world))
     stream = torch.cuda.current_stream()
+    exchange = world > 1 and inp["wl"] != "sm"      # SM is Map-only: no exchange
+    xbytes = [0]
 
     def step():
         job.reset()
         job.map(inp["data"], inp["offsets"], inp["n"])
+        if exchange:  # one hash all-to-all over NCCL
+            xbytes[0] = job.shuffle()
         job.group()
         job.reduce()
 
@@ -310,12 +318,14 @@ def main():
             h_off = torch.empty(inp["offsets"].numel(), dtype=torch.int64, pin_memory=True)
             h_off.copy_(inp["offsets"])
         torch.cuda.synchronize()
-        job_e = bmr.Job(inp["wl"], **job_kwargs(inp, 0, local))
+        job_e = bmr.Job(inp["wl"], **job_kwargs(inp, 0, local, rank, world))
         d2h = 0
 
         def estep():
             job_e.reset()
             job_e.map_host(h_data.numpy(), None if h_off is None else h_off.numpy().view(np.uint64), inp["n"])
+            if exchange:
+                job_e.shuffle()
             job_e.group()
             job_e.reduce()
             r = job_e.fetch()
@@ -366,6 +376,8 @@ def main():
             "pairs_per_step": int(alg["pairs"]), "sort_passes": alg["passes"],
             "distinct_keys": int(tot["n_keys"] / args.steps),
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+            "exchange": ({"kind": "hash all-to-all over NCCL (torch.distributed)", "send_bytes_per_rank": xbytes[0],
+                          "combiner": inp["wl"] in ("wc", "km")} if exchange else None),
             "gpu_launches": int(tot["kernel_launches"]),
             "clocks": clk.summary(), "wall_s_timed": round(wall, 3),
         }

@@ -51,6 +51,7 @@ typedef enum { MR_WORDCOUNT = 1, MR_STRINGMATCH = 2, MR_KMEANS = 3, MR_INVINDEX 
 #define MR_FLAG_VALIDATE        0x10u /* host-side argument validation of offsets (reads them back) */
 #define MR_FLAG_NO_COMBINE      0x20u /* multi-GPU: exchange raw pairs (no combiner) */
 #define MR_FLAG_PROFILE         0x40u /* record CUDA events per phase on the job stream (mr_stats *_ms) */
+#define MR_FLAG_OWN_STREAM      0x80u /* ignore cfg.stream: the job creates a private non-blocking stream */
 
 typedef struct { uint8_t pattern[16]; } mr_sm_params;                      /* StringMatch */
 typedef struct { uint32_t k, dim; const float* centroids; } mr_km_params;  /* KMeans: host ptr, k x dim fp32, dim == 8, 1 <= k <= 1024 */
@@ -64,7 +65,7 @@ typedef struct {
   const void* params;        /* mr_sm_params* / mr_km_params* / NULL; copied at create */
   uint64_t input_base;       /* global byte offset of this rank's first record (SM/II offsets are global) */
   int rank, nranks;          /* nranks == 1: single GPU */
-  void* nccl_comm;           /* ncclComm_t (multi-GPU; reserved in ABI v1) */
+  void* nccl_comm;           /* reserved (the exchange is moved by the caller, see mr_ingest) */
   uint64_t max_pairs_hint;   /* initial intermediate capacity in pairs (0: heuristic) */
   uint64_t heap_bytes_hint;  /* reserved */
   uint32_t flags;            /* MR_FLAG_* */
@@ -141,6 +142,26 @@ mr_status mr_get_stats(const mr_job* job, void* stats, size_t bytes);
 mr_status mr_job_destroy(mr_job* job); /* NULL-safe */
 const char* mr_status_string(mr_status s);
 const char* mr_last_error(const mr_job* job);
+
+/* ---- Multi-GPU exchange: one all-to-all between Map and group-by ----
+ * Input is sharded by byte range (no communication in Map; input_base keeps SM/II offsets
+ * global).  Records are routed to rank mix64(hash of the key bytes) mod nranks.  WC and KM first
+ * run the local group + reduce as a combiner (the original MapReduce combiner; the paper uses
+ * none) unless MR_FLAG_NO_COMBINE (WC only); II exchanges raw pairs.  StringMatch
+ * is Map-only and has no exchange (MR_ERR_UNSUPPORTED).  The caller moves the bytes (e.g.
+ * torch.distributed all_to_all_single over NCCL):
+ *   1. mr_partition_count(job, counts, &entry_bytes): counts[2r] = entries for rank r,
+ *      counts[2r+1] = heap bytes for rank r (host array of 2*nranks u64); synchronises.
+ *   2. caller allocates device buffers of sum(entries)*entry_bytes and sum(heap) bytes;
+ *      mr_partition_write(job, entries, heap) fills them, slices in rank order (asynchronous).
+ *   3. all-to-all; then mr_ingest(job, recv_entries, recv_heap, recv_counts) with the received
+ *      buffers concatenated in source-rank order and recv_counts[2r], [2r+1] from source r.
+ *      The received heap holds the key bytes, referenced until mr_reduce completes (caller-owned).
+ *   4. mr_group / mr_reduce / mr_fetch as usual; each rank outputs the keys it owns.
+ * State: MAPPED -> partition_count -> partition_write -> ingest -> MAPPED (ingested). */
+mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_bytes);
+mr_status mr_partition_write(mr_job* job, void* entries, void* heap);
+mr_status mr_ingest(mr_job* job, const void* entries, const void* heap, const uint64_t* recv_counts);
 
 /* Group-by primitive exposed for testing (§8(a) a7): stable LSD radix sort of n u64 device
  * keys; writes the sorted keys and the u32 permutation (perm[i] = source index of the i-th

@@ -23,13 +23,14 @@ WORDCOUNT, STRINGMATCH, KMEANS, INVINDEX = 1, 2, 3, 4
 WORKLOADS = {"wc": WORDCOUNT, "sm": STRINGMATCH, "km": KMEANS, "ii": INVINDEX}
 FLAG_NO_SMEM_IN, FLAG_NO_SMEM_OUT, FLAG_FORCE_TINY_OUT = 0x01, 0x02, 0x04
 FLAG_WEAK_HASH_DEBUG, FLAG_VALIDATE, FLAG_NO_COMBINE = 0x08, 0x10, 0x20
-FLAG_PROFILE = 0x40
+FLAG_PROFILE, FLAG_OWN_STREAM = 0x40, 0x80
 
 STATUS = {0: "MR_OK", 1: "MR_ERR_INVALID", 2: "MR_ERR_STATE", 3: "MR_ERR_OOM", 4: "MR_ERR_OVERFLOW",
           5: "MR_ERR_CUDA", 6: "MR_ERR_NCCL", 7: "MR_ERR_UNSUPPORTED"}
 
 EXPORTS = ("mr_job_create", "mr_map", "mr_map_host", "mr_group", "mr_reduce", "mr_fetch", "mr_job_reset",
-           "mr_get_stats", "mr_job_destroy", "mr_status_string", "mr_last_error", "mr_sort_u64")
+           "mr_get_stats", "mr_job_destroy", "mr_status_string", "mr_last_error", "mr_sort_u64",
+           "mr_partition_count", "mr_partition_write", "mr_ingest")
 
 
 class MRError(RuntimeError):
@@ -87,6 +88,9 @@ def lib() -> C.CDLL:
         L.mr_last_error.argtypes = [vp]
         L.mr_last_error.restype = C.c_char_p
         L.mr_sort_u64.argtypes = [vp, vp, vp, u64, vp]
+        L.mr_partition_count.argtypes = [vp, vp, C.POINTER(u64)]
+        L.mr_partition_write.argtypes = [vp, vp, vp]
+        L.mr_ingest.argtypes = [vp, vp, vp, vp]
         for f in EXPORTS:
             if f not in ("mr_status_string", "mr_last_error"):
                 getattr(L, f).restype = C.c_int
@@ -117,7 +121,7 @@ class Job:
 
     def __init__(self, workload: str, device: int = 0, stream=None, pattern: bytes | None = None,
                  centroids: np.ndarray | None = None, input_base: int = 0, flags: int = 0,
-                 max_pairs_hint: int = 0):
+                 max_pairs_hint: int = 0, rank: int = 0, nranks: int = 1):
         L = lib()
         self.workload = workload
         cfg = Config()
@@ -129,7 +133,8 @@ class Job:
             stream = torch.cuda.current_stream(device).cuda_stream
         cfg.stream = stream
         cfg.input_base = input_base
-        cfg.rank, cfg.nranks = 0, 1
+        cfg.rank, cfg.nranks = rank, nranks
+        self.rank, self.nranks = rank, nranks
         cfg.max_pairs_hint = max_pairs_hint
         cfg.flags = flags
         self._keep = []
@@ -188,6 +193,39 @@ class Job:
         self.group()
         self.reduce()
         return self.fetch()
+
+    # ---- multi-GPU exchange (mr_partition_count / mr_partition_write / mr_ingest) ----
+    def partition(self):
+        """Partition this rank's records by destination; returns (entries u8 tensor, heap u8
+        tensor, counts int64 array [nranks, 2] = (entries, heap bytes) per destination, entry_bytes)."""
+        import torch
+        counts = np.zeros(2 * self.nranks, np.uint64)
+        eb = C.c_uint64(0)
+        self._check(lib().mr_partition_count(self.h, _ptr(counts), C.byref(eb)))
+        counts = counts.astype(np.int64).reshape(self.nranks, 2)
+        dev = torch.device("cuda", torch.cuda.current_device())
+        ent = torch.empty(int(counts[:, 0].sum()) * eb.value, dtype=torch.uint8, device=dev)
+        heap = torch.empty(int(counts[:, 1].sum()), dtype=torch.uint8, device=dev)
+        self._check(lib().mr_partition_write(self.h, _ptr(ent), _ptr(heap)))
+        return ent, heap, counts, int(eb.value)
+
+    def ingest(self, entries, heap, recv_counts):
+        """mr_ingest of the buffers received from every source rank (concatenated in rank order);
+        recv_counts int64 [nranks, 2].  The buffers must stay alive until reduce completes."""
+        rc = np.ascontiguousarray(recv_counts, np.int64).astype(np.uint64).reshape(-1)
+        self._recv = (entries, heap, rc)
+        self._check(lib().mr_ingest(self.h, _ptr(entries), _ptr(heap), _ptr(rc)))
+
+    def shuffle(self, group=None):
+        """One all-to-all exchange over torch.distributed (NCCL on GPUs): partition -> exchange
+        -> ingest."""
+        from . import dist as D
+        ent, heap, counts, eb = self.partition()
+        recv_counts = D.exchange_counts(counts, group)
+        r_ent = D.alltoallv(ent, counts[:, 0] * eb, recv_counts[:, 0] * eb, group)
+        r_heap = D.alltoallv(heap, counts[:, 1], recv_counts[:, 1], group)
+        self.ingest(r_ent, r_heap, recv_counts)
+        return int(counts[:, 0].sum()) * eb + int(counts[:, 1].sum())
 
     def reset(self):
         self._check(lib().mr_job_reset(self.h))

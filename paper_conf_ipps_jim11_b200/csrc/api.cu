@@ -22,7 +22,7 @@ std::atomic<unsigned long long> bmr::g_kernel_launches{0};
 
 namespace {
 
-enum State { kCreated = 0, kMapped = 1, kGrouped = 2, kReduced = 3 };
+enum State { kCreated = 0, kMapped = 1, kGrouped = 2, kReduced = 3, kPartitioned = 4 };
 
 template <typename T>
 struct DBuf {
@@ -218,6 +218,16 @@ struct mr_job {
   // fetched result
   HBuf<uint8_t> keys_h, vals_h;
   HBuf<uint64_t> key_off_h, val_off_h;
+  // multi-GPU exchange (§8(e))
+  XSource xs;
+  bool ingested = false;          // pairs come from mr_ingest (WC values are u64 partial counts)
+  bool km_partial = false;        // KM: sums/cnts hold ingested partials; finalise owned clusters
+  int vb_cur = 0;                 // value bytes of the current pairs
+  DBuf<unsigned long long> xcounts, xcursors, xheapbase;
+  HBuf<unsigned long long> xcounts_h;
+  DBuf<uint64_t> src_e, src_h;
+  DBuf<uint32_t> km_list;
+  uint32_t km_nlist = 0;
   uint64_t out_keys_bytes = 0, out_vals_bytes = 0, out_n = 0;
   mr_stats stats{};
 };
@@ -337,7 +347,7 @@ mr_status mr_job_create(const mr_config* cfg, mr_job** out) {
   *out = nullptr;
   if (cfg->abi_version != MR_ABI_VERSION) return MR_ERR_INVALID;
   if (cfg->workload < MR_WORDCOUNT || cfg->workload > MR_INVINDEX) return MR_ERR_INVALID;
-  if (cfg->nranks > 1) return MR_ERR_UNSUPPORTED;
+  if (cfg->nranks < 1 || cfg->nranks > kMaxRanks || cfg->rank < 0 || cfg->rank >= cfg->nranks) return MR_ERR_INVALID;
   if (cfg->workload == MR_KMEANS) {
     const mr_km_params* p = static_cast<const mr_km_params*>(cfg->params);
     if (!p || !p->centroids || p->dim != 8 || p->k < 1 || p->k > 1024 || cfg->record_stride != 32)
@@ -357,12 +367,14 @@ mr_status mr_job_create(const mr_config* cfg, mr_job** out) {
     job->k = p->k;
     job->cent_h.assign(p->centroids, p->centroids + static_cast<size_t>(p->k) * 8);
   }
+  // cfg->stream == NULL is CUDA's default stream (what torch's default stream handle is), so a
+  // job always orders with the caller's stream; MR_FLAG_OWN_STREAM asks for a private stream.
   if (e == cudaSuccess) {
-    if (cfg->stream) {
-      job->stream = static_cast<cudaStream_t>(cfg->stream);
-    } else {
+    if (cfg->flags & MR_FLAG_OWN_STREAM) {
       e = cudaStreamCreateWithFlags(&job->stream, cudaStreamNonBlocking);
       job->own_stream = (e == cudaSuccess);
+    } else {
+      job->stream = static_cast<cudaStream_t>(cfg->stream);
     }
   }
   if (e == cudaSuccess) e = cudaMalloc(reinterpret_cast<void**>(&job->st), sizeof(DevState));
@@ -394,6 +406,8 @@ mr_status mr_job_reset(mr_job* job) {
   for (void* p : job->owned) cudaFree(p);
   job->owned.clear();
   job->host_batches = 0;
+  job->ingested = false;
+  job->km_partial = false;
   job->prof.collect();
   job->batches.clear();
   job->next_base = 0;
@@ -479,6 +493,10 @@ mr_status mr_group(mr_job* job) {
   if (!job) return MR_ERR_INVALID;
   if (job->state != kMapped && job->state != kCreated) return fail(job, MR_ERR_STATE, "mr_group out of order");
   CK(cudaSetDevice(job->cfg.device), "set device");
+  if (job->km_partial) {           // ingested KM partials: grouping happened at the owner (atomics)
+    job->state = kGrouped;
+    return MR_OK;
+  }
   CK(read_state(job), "map (async)");
   DevState* hs = job->st_h.p;
   if (hs->err & kErrKeyTooLong) return fail(job, MR_ERR_OVERFLOW, "an emitted key exceeds 65535 bytes");
@@ -496,17 +514,20 @@ mr_status mr_group(mr_job* job) {
     m = hs->pair_cursor;
     if (m > job->cap) return fail(job, MR_ERR_OOM, "replay still overflows");
   }
+  const uint64_t m_total = m;            // includes the flush filler pairs (sentinel keys)
+  m -= hs->pads;
   job->m = m;
   job->stats.pairs = m;
   job->stats.flushes = hs->flushes;
-  if (m >= (1ULL << 32) - 1) return fail(job, MR_ERR_UNSUPPORTED, ">= 2^32 intermediate pairs in one group");
+  if (m_total >= (1ULL << 32) - 1) return fail(job, MR_ERR_UNSUPPORTED, ">= 2^32 intermediate pairs in one group");
   if (job->cfg.workload == MR_STRINGMATCH) {  // Map-only
     job->nseg = m;
     job->state = kGrouped;
     return MR_OK;
   }
   for (int attempt = 0;; ++attempt) {
-    CK(run_sort(job->sw, job->h.p, m, &job->skeys, &job->perm, job->st, job->nsm, job->stream, &job->prof,
+    // sentinel keys sort after every real key: the first m sorted positions are the real pairs
+    CK(run_sort(job->sw, job->h.p, m_total, &job->skeys, &job->perm, job->st, job->nsm, job->stream, &job->prof,
                 &job->stats.hist_ms, &job->stats.sort_ms),
        "radix sort");
     job->stats.sort_passes += job->sw.passes;
@@ -520,7 +541,7 @@ mr_status mr_group(mr_job* job) {
     job->stats.collisions += coll;
     if (attempt >= 3) return fail(job, MR_ERR_UNSUPPORTED, "unresolvable 64-bit hash collision");
     // slow path: recompute every hashed key with a fresh full-width hash, then sort again
-    CK(launch_rehash(job->h.p, job->kref.p, m, 0xC0111DE5ULL + attempt, job->stream), "rehash");
+    CK(launch_rehash(job->h.p, job->kref.p, m_total, 0xC0111DE5ULL + attempt, job->stream), "rehash");
   }
   job->stats.n_keys = job->nseg;
   Prof::Span sp3{};
@@ -553,7 +574,8 @@ mr_status mr_reduce(mr_job* job) {
     case MR_WORDCOUNT: {
       CK(job->counts.ensure(S + 1), "alloc counts");
       CK(job->worklist.ensure(m / 1024 + 64), "alloc worklist");
-      CK(launch_reduce_wc(job->seg_start.p, S, job->perm, job->v.p, job->counts.p, job->worklist.p, job->st, job->nsm, s),
+      CK(launch_reduce_wc(job->seg_start.p, S, job->perm, job->v.p, job->ingested ? 8 : 4, job->counts.p,
+                          job->worklist.p, job->st, job->nsm, s),
          "reduce wc");
       CK(job->val_off.ensure(S + 1), "alloc val offsets");
       CK(launch_iota_scaled(S, 8, job->val_off.p, s), "val offsets");
@@ -580,20 +602,24 @@ mr_status mr_reduce(mr_job* job) {
       const uint32_t k = job->k;
       CK(job->sums.ensure(8ULL * k), "alloc sums");
       CK(job->cnts.ensure(k), "alloc counts");
-      CK(job->worklist.ensure(m / 1024 + 64), "alloc worklist");
-      CK(launch_reduce_km(job->seg_start.p, S, job->skeys, job->perm, job->v.p, job->sums.p, job->cnts.p, k,
-                          job->worklist.p, job->st, job->nsm, s),
-         "reduce km");
+      if (!job->km_partial) {
+        CK(job->worklist.ensure(m / 1024 + 64), "alloc worklist");
+        CK(launch_reduce_km(job->seg_start.p, S, job->skeys, job->perm, job->v.p, job->sums.p, job->cnts.p, k,
+                            job->worklist.p, job->st, job->nsm, s),
+           "reduce km");
+      }
+      const uint32_t* list = job->km_partial ? job->km_list.p : nullptr;
+      const uint32_t nout = job->km_partial ? job->km_nlist : k;
       CK(job->keys_out.ensure(4ULL * k), "alloc keys");
       CK(job->vals_out.ensure(40ULL * k), "alloc vals");
       CK(job->key_off.ensure(k + 1), "alloc key offsets");
       CK(job->val_off.ensure(k + 1), "alloc val offsets");
-      CK(launch_km_finalize(job->sums.p, job->cnts.p, job->cent.p, k, job->vals_out.p, job->val_off.p, job->keys_out.p,
-                            job->key_off.p, s),
+      CK(launch_km_finalize(job->sums.p, job->cnts.p, job->cent.p, k, list, nout, job->vals_out.p, job->val_off.p,
+                            job->keys_out.p, job->key_off.p, s),
          "km finalize");
-      job->out_n = k;
-      job->out_keys_bytes = 4ULL * k;
-      job->out_vals_bytes = 40ULL * k;
+      job->out_n = nout;
+      job->out_keys_bytes = 4ULL * nout;
+      job->out_vals_bytes = 40ULL * nout;
       break;
     }
     case MR_STRINGMATCH: {
@@ -640,6 +666,155 @@ mr_status mr_fetch(mr_job* job, mr_result* out) {
   return MR_OK;
 }
 
+// ---------------------------------------------------------------- multi-GPU exchange (§8(e))
+mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_bytes) {
+  if (!job || !counts) return MR_ERR_INVALID;
+  if (job->state != kMapped && job->state != kCreated) return fail(job, MR_ERR_STATE, "mr_partition_count out of order");
+  CK(cudaSetDevice(job->cfg.device), "set device");
+  const uint32_t R = static_cast<uint32_t>(job->cfg.nranks);
+  const int w = job->cfg.workload;
+  if (w == MR_STRINGMATCH) return fail(job, MR_ERR_UNSUPPORTED, "StringMatch is Map-only: no exchange");
+  const bool combine = (w == MR_KMEANS) || (w == MR_WORDCOUNT && !(job->cfg.flags & MR_FLAG_NO_COMBINE));
+  XSource xs;
+  xs.nranks = R;
+  if (combine) {
+    // combiner (SURVEY §8(e) reading): local group + reduce, exchange partial aggregates
+    mr_status st = mr_group(job);
+    if (st != MR_OK) return st;
+    st = mr_reduce(job);
+    if (st != MR_OK) return st;
+    if (w == MR_WORDCOUNT) {
+      xs.mode = kXSegs;
+      xs.n = job->nseg;
+      xs.keys = job->keys_out.p;
+      xs.key_off = job->key_off.p;
+      xs.counts = job->counts.p;
+    } else {
+      xs.mode = kXKM;
+      xs.n = job->k;
+      xs.sums = job->sums.p;
+      xs.cnts = job->cnts.p;
+    }
+  } else {
+    // raw pairs: settle the Map (capacity check / replay) without grouping
+    CK(read_state(job), "map (async)");
+    DevState* hs = job->st_h.p;
+    if (hs->err & kErrKeyTooLong) return fail(job, MR_ERR_OVERFLOW, "an emitted key exceeds 65535 bytes");
+    uint64_t m = hs->pair_cursor;
+    if (m > job->cap) {
+      job->h.release(); job->kref.release(); job->v.release(); job->cap = 0;
+      CK(ensure_pairs(job, m + m / 8 + 4096), "grow intermediate");
+      CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
+      for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
+      job->stats.replays += job->batches.size();
+      CK(read_state(job), "replay (async)");
+      m = hs->pair_cursor;
+    }
+    job->m = m - hs->pads;
+    job->stats.pairs = m - hs->pads;
+    xs.mode = kXPairs;
+    xs.n = m;
+    xs.kref = job->kref.p;
+    xs.v = job->v.p;
+    xs.vbytes = vbytes_of(w);
+  }
+  CK(job->xcounts.ensure(2 * R), "alloc counts");
+  CK(job->xcursors.ensure(2 * R), "alloc cursors");
+  CK(job->xheapbase.ensure(R), "alloc heap base");
+  CK(job->xcounts_h.ensure(4 * R), "alloc host counts");
+  CK(launch_x_count(xs, job->xcounts.p, job->nsm, job->stream), "partition count");
+  CK(cudaMemcpyAsync(job->xcounts_h.p, job->xcounts.p, 2 * R * 8, cudaMemcpyDeviceToHost, job->stream), "D2H counts");
+  CK(cudaStreamSynchronize(job->stream), "sync counts");
+  unsigned long long* cur = job->xcounts_h.p + 2 * R;   // host staging for cursors
+  unsigned long long e = 0, hb = 0;
+  std::vector<unsigned long long> hbase(R);
+  for (uint32_t r = 0; r < R; ++r) {
+    counts[2 * r] = job->xcounts_h.p[2 * r];
+    counts[2 * r + 1] = job->xcounts_h.p[2 * r + 1];
+    cur[2 * r] = e;
+    cur[2 * r + 1] = hb;
+    hbase[r] = hb;
+    e += counts[2 * r];
+    hb += counts[2 * r + 1];
+  }
+  CK(cudaMemcpyAsync(job->xcursors.p, cur, 2 * R * 8, cudaMemcpyHostToDevice, job->stream), "H2D cursors");
+  CK(cudaMemcpyAsync(job->xheapbase.p, hbase.data(), R * 8, cudaMemcpyHostToDevice, job->stream), "H2D heap base");
+  CK(cudaStreamSynchronize(job->stream), "sync cursors");
+  xs.heap_base = job->xheapbase.p;
+  job->xs = xs;
+  if (entry_bytes) *entry_bytes = (xs.mode == kXKM) ? sizeof(XEntryKM) : sizeof(XEntry);
+  job->state = kPartitioned;
+  return MR_OK;
+}
+
+mr_status mr_partition_write(mr_job* job, void* entries, void* heap) {
+  if (!job) return MR_ERR_INVALID;
+  if (job->state != kPartitioned) return fail(job, MR_ERR_STATE, "mr_partition_write before mr_partition_count");
+  CK(cudaSetDevice(job->cfg.device), "set device");
+  if (job->xs.n && !entries) return fail(job, MR_ERR_INVALID, "entries is NULL");
+  CK(launch_x_scatter(job->xs, job->xcursors.p, static_cast<uint8_t*>(entries), static_cast<uint8_t*>(heap),
+                      job->stream),
+     "partition scatter");
+  return MR_OK;
+}
+
+mr_status mr_ingest(mr_job* job, const void* entries, const void* heap, const uint64_t* recv_counts) {
+  if (!job || !recv_counts) return MR_ERR_INVALID;
+  if (job->state != kPartitioned) return fail(job, MR_ERR_STATE, "mr_ingest before mr_partition_write");
+  CK(cudaSetDevice(job->cfg.device), "set device");
+  const uint32_t R = static_cast<uint32_t>(job->cfg.nranks);
+  std::vector<uint64_t> se(R + 1, 0), sh(R + 1, 0);
+  for (uint32_t r = 0; r < R; ++r) {
+    se[r + 1] = se[r] + recv_counts[2 * r];
+    sh[r + 1] = sh[r] + recv_counts[2 * r + 1];
+  }
+  const uint64_t n = se[R];
+  if (n && !entries) return fail(job, MR_ERR_INVALID, "entries is NULL");
+  cudaStream_t s = job->stream;
+  job->batches.clear();
+  if (job->cfg.workload == MR_KMEANS) {
+    const uint32_t k = job->k;
+    CK(job->sums.ensure(8ULL * k), "alloc sums");
+    CK(job->cnts.ensure(k), "alloc counts");
+    CK(cudaMemsetAsync(job->sums.p, 0, 64ULL * k, s), "memset sums");
+    CK(cudaMemsetAsync(job->cnts.p, 0, 8ULL * k, s), "memset counts");
+    CK(launch_x_ingest_km(entries, n, job->sums.p, job->cnts.p, k, s), "ingest km");
+    std::vector<uint32_t> own;
+    for (uint32_t j = 0; j < k; ++j)
+      if (km_owner(j, R) == static_cast<uint32_t>(job->cfg.rank)) own.push_back(j);
+    CK(job->km_list.ensure(own.size() + 1), "alloc owner list");
+    if (!own.empty())
+      CK(cudaMemcpyAsync(job->km_list.p, own.data(), own.size() * 4, cudaMemcpyHostToDevice, s), "H2D owners");
+    CK(cudaStreamSynchronize(s), "sync owners");
+    job->km_nlist = static_cast<uint32_t>(own.size());
+    job->km_partial = true;
+    job->state = kMapped;
+    return MR_OK;
+  }
+  if (n > job->cap || job->v.n < n * 8) {
+    job->h.release(); job->kref.release(); job->v.release(); job->cap = 0;
+    CK(job->h.ensure(n + 1), "alloc pairs");
+    CK(job->kref.ensure(n + 1), "alloc pairs");
+    CK(job->v.ensure((n + 1) * 8), "alloc pairs");
+    job->cap = n + 1;
+  }
+  CK(job->src_e.ensure(R + 1), "alloc src");
+  CK(job->src_h.ensure(R + 1), "alloc src");
+  CK(cudaMemcpyAsync(job->src_e.p, se.data(), (R + 1) * 8, cudaMemcpyHostToDevice, s), "H2D src");
+  CK(cudaMemcpyAsync(job->src_h.p, sh.data(), (R + 1) * 8, cudaMemcpyHostToDevice, s), "H2D src");
+  CK(launch_x_ingest(entries, static_cast<const uint8_t*>(heap), n, job->src_e.p, job->src_h.p, R, job->h.p,
+                     job->kref.p, reinterpret_cast<uint64_t*>(job->v.p), 0x5EEDB200ULL,
+                     (job->cfg.flags & MR_FLAG_WEAK_HASH_DEBUG) ? 1u : 0u, s),
+     "ingest");
+  CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), s), "reset state");
+  job->tmp_h.p[0] = n;
+  CK(cudaMemcpyAsync(&job->st->pair_cursor, job->tmp_h.p, 8, cudaMemcpyHostToDevice, s), "set pair count");
+  CK(cudaStreamSynchronize(s), "sync ingest");
+  job->ingested = true;
+  job->state = kMapped;
+  return MR_OK;
+}
+
 mr_status mr_get_stats(const mr_job* job, void* stats, size_t bytes) {
   if (!job || !stats) return MR_ERR_INVALID;
   mr_stats st = job->stats;
@@ -651,11 +826,13 @@ mr_status mr_get_stats(const mr_job* job, void* stats, size_t bytes) {
 mr_status mr_job_destroy(mr_job* job) {
   if (!job) return MR_OK;
   cudaSetDevice(job->cfg.device);
-  if (job->stream) cudaStreamSynchronize(job->stream);
+  cudaStreamSynchronize(job->stream);
   for (void* p : job->owned) cudaFree(p);
   for (auto& b : job->host_rec) b.release();
   for (auto& b : job->host_off) b.release();
   job->prof.release();
+  job->xcounts.release(); job->xcursors.release(); job->xheapbase.release(); job->xcounts_h.release();
+  job->src_e.release(); job->src_h.release(); job->km_list.release();
   job->cent.release(); job->h.release(); job->kref.release(); job->tb.release(); job->v.release();
   job->sw.release();
   job->seg_counts.release(); job->tile_base.release(); job->seg_start.release(); job->key_off.release();

@@ -70,6 +70,22 @@ __device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
   asm volatile("ld.volatile.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ uint64_t ld_relaxed_gpu_u64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed_gpu_u64(uint64_t* p, uint64_t v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t ld_acquire_gpu_u64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu_u64(uint64_t* p, uint64_t v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 __device__ __forceinline__ void st_volatile_u64(uint64_t* p, uint64_t v) {
   asm volatile("st.volatile.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
@@ -107,8 +123,10 @@ __device__ __forceinline__ uint64_t hash_bytes(const uint8_t* p, uint32_t len, u
 }
 // Final sort key of a hashed key; weak_hash (MR_FLAG_WEAK_HASH_DEBUG) keeps only 4 bits so
 // that almost every segment collides (tests the verification + re-sort slow path).
+// ~0 is reserved for the flush filler sentinel, so a hashed key never equals it.
 __device__ __forceinline__ uint64_t hashed_key(uint64_t h, bool weak) {
-  return (weak ? (h & 0xFULL) : (h & ~kHashedBit)) | kHashedBit;
+  const uint64_t k = (weak ? (h & 0xFULL) : (h & ~kHashedBit)) | kHashedBit;
+  return k == ~0ULL ? ~0ULL - 1 : k;
 }
 // <= 7 bytes packed little-endian, length in bits 56..63 (1..7): injective, top bit clear.
 __device__ __forceinline__ uint64_t inline_key(uint64_t bytes_le, uint32_t len) {

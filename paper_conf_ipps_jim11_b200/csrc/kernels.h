@@ -24,6 +24,7 @@ struct DevState {
   unsigned long long large_items;  // reduce work list length (large segments x tiles)
   unsigned long long large_done;   // work-list cursor for the persistent large-segment kernel
   unsigned int tile_counter[32];   // dynamic tile ids of the look-back kernels (one per launch slot)
+  unsigned long long pads;         // sentinel filler pairs written by the flushes (sort last, excluded)
 };
 constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u;
 
@@ -97,17 +98,48 @@ cudaError_t launch_key_lengths(const uint64_t* seg_start, uint64_t nseg, const u
 cudaError_t launch_key_copy(const uint64_t* seg_start, uint64_t nseg, const uint32_t* perm, const uint64_t* kref,
                             const uint64_t* key_off, uint8_t* keys, cudaStream_t s);
 cudaError_t launch_reduce_wc(const uint64_t* seg_start, uint64_t nseg, const uint32_t* perm, const uint8_t* v,
-                             uint64_t* counts, uint64_t* worklist, DevState* st, int num_sms, cudaStream_t s);
+                             int vbytes, uint64_t* counts, uint64_t* worklist, DevState* st, int num_sms,
+                             cudaStream_t s);
 cudaError_t launch_reduce_km(const uint64_t* seg_start, uint64_t nseg, const uint64_t* skeys, const uint32_t* perm,
                              const uint8_t* v, double* sums, unsigned long long* cnts, uint32_t k,
                              uint64_t* worklist, DevState* st, int num_sms, cudaStream_t s);
+// list == nullptr: all k clusters; else the nlist cluster ids in `list` (multi-GPU owners)
 cudaError_t launch_km_finalize(const double* sums, const unsigned long long* cnts, const float* centroids,
-                               uint32_t k, uint8_t* vals, uint64_t* val_off, uint8_t* keys, uint64_t* key_off,
-                               cudaStream_t s);
+                               uint32_t k, const uint32_t* list, uint32_t nlist, uint8_t* vals, uint64_t* val_off,
+                               uint8_t* keys, uint64_t* key_off, cudaStream_t s);
 cudaError_t launch_gather_u64(const uint32_t* perm, const uint8_t* v, uint64_t m, uint64_t* out, cudaStream_t s);
 cudaError_t launch_offsets_scaled(const uint64_t* seg_start, uint64_t nseg, uint64_t scale, uint64_t* out,
                                   cudaStream_t s);
 cudaError_t launch_iota_scaled(uint64_t n, uint64_t scale, uint64_t* out, cudaStream_t s);
 cudaError_t launch_rehash(uint64_t* h, const uint64_t* kref, uint64_t m, uint64_t seed, cudaStream_t s);
+
+// ---- multi-GPU exchange (exchange.cu) ----
+constexpr int kMaxRanks = 64;
+enum XMode : int { kXPairs = 0, kXSegs = 1, kXKM = 2 };
+struct XEntry { uint64_t koff_len; uint64_t v; };          // WC / II (16 B)
+struct XEntryKM { uint64_t id, cnt; double sums[8]; };      // KM partial (80 B)
+struct XSource {
+  int mode = kXPairs;
+  uint32_t nranks = 1;
+  uint64_t n = 0;                              // records of the source
+  const uint64_t* kref = nullptr;              // kXPairs
+  const uint8_t* v = nullptr;
+  int vbytes = 8;
+  const uint8_t* keys = nullptr;               // kXSegs
+  const uint64_t* key_off = nullptr;
+  const uint64_t* counts = nullptr;
+  const double* sums = nullptr;                // kXKM
+  const unsigned long long* cnts = nullptr;
+  const unsigned long long* heap_base = nullptr;  // device: heap slice start of every destination
+};
+uint32_t km_owner(uint32_t j, uint32_t nranks);
+cudaError_t launch_x_count(const XSource& S, unsigned long long* counts, int num_sms, cudaStream_t s);
+cudaError_t launch_x_scatter(const XSource& S, unsigned long long* cursors, uint8_t* entries, uint8_t* heap,
+                             cudaStream_t s);
+cudaError_t launch_x_ingest(const void* entries, const uint8_t* heap, uint64_t n, const uint64_t* src_e,
+                            const uint64_t* src_h, uint32_t R, uint64_t* h, uint64_t* kref, uint64_t* v,
+                            uint64_t seed, uint32_t weak, cudaStream_t s);
+cudaError_t launch_x_ingest_km(const void* entries, uint64_t n, double* sums, unsigned long long* cnts, uint32_t k,
+                               cudaStream_t s);
 
 }  // namespace bmr

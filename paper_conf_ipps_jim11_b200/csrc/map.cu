@@ -28,9 +28,11 @@ namespace {
 
 constexpr int kNMap = 16;
 constexpr int kProdWarp = kNMap;
-constexpr int kFlushWarp = kNMap + 1;
-constexpr int kThreads = (kNMap + 2) * 32;
-constexpr int kStages = 3;
+constexpr int kFlushWarp0 = kNMap + 1;   // flush warps kFlushWarp0 .. kFlushWarp0 + kNFlush - 1
+constexpr int kNFlush = 1;
+constexpr int kThreads = (kNMap + 1 + kNFlush) * 32;
+constexpr int kStages = 4;
+constexpr int kLag = 2;           // producer builds the bitmap of tile it - kLag after issuing tile it
 constexpr int kT = 16384;        // owned bytes per tile (text) / bytes per tile (KM)
 constexpr int kLead = 16;        // bytes staged before the tile (previous-byte context)
 constexpr int kHalo = 256;       // bytes staged after the tile (words / matches / URLs crossing it)
@@ -60,26 +62,29 @@ struct StageHdr {
 };
 
 struct OutCtl {
-  unsigned long long cur;        // [generation:32 | count:32]; half = generation & 1
+  unsigned int cur;              // [generation:8 | count:24]; half = generation & 1
+  unsigned int final_seq;        // full generation number of the final flush
   unsigned int committed[2];     // entries fully written into each half (current generation)
   unsigned int fcount[2];        // sealed entry count of each half
-  unsigned int final_gen, is_final;
+  unsigned long long fbase[2];   // global base reserved for the sealed half (one atomic per flush)
+  unsigned int nsealed, is_final;  // sealed generations so far (full count); final flush flag
   uint64_t req[2];               // mbarrier: half sealed -> flush warp
   uint64_t done[2];              // mbarrier: half flushed -> free
 };
 
 struct Layout {
   static constexpr int ctl = 0;                                   // OutCtl
-  static constexpr int hdr = 128;                                 // kStages x 128
+  static constexpr int hdr = 128;                                 // kStages x 128 (<= 4 stages)
   static constexpr int full = hdr + kStages * 128;                // kStages x 8
   static constexpr int empty = full + kStages * 8;
+  static constexpr int ready = empty + kStages * 8;               // kStages x 8 (text: bitmap built)
   static constexpr int bytes = 1024;                              // kStages x kStageBytes
   static constexpr int offs = bytes + kStages * kStageBytes;      // kStages x kOffBytes
   static constexpr int bits = offs + kStages * kOffBytes;         // kStages x kBitBytes
   static constexpr int out = bits + kStages * kBitBytes;          // 2 x kOutHalf
   static constexpr int cent = out + 2 * kOutHalf;                 // KM centroids
 };
-static_assert(Layout::empty + kStages * 8 <= Layout::bytes, "header region overflow");
+static_assert(Layout::ready + kStages * 8 <= Layout::bytes, "header region overflow");
 
 template <int W>
 struct PairFmt {
@@ -114,6 +119,26 @@ struct Params {
 };
 
 constexpr uint32_t kFull = 0xffffffffu;
+
+// ---------------------------------------------------------------- packed fp32 (sm_100a FADD2/FFMA2)
+__device__ __forceinline__ uint64_t f2pack(float a, float b) {
+  uint64_t r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(a), "f"(b));
+  return r;
+}
+__device__ __forceinline__ void f2unpack(uint64_t v, float& a, float& b) {
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(v));
+}
+__device__ __forceinline__ uint64_t f2sub(uint64_t a, uint64_t b) {
+  uint64_t r;
+  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+  return r;
+}
+__device__ __forceinline__ uint64_t f2fma(uint64_t a, uint64_t b, uint64_t c) {
+  uint64_t r;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
+  return r;
+}
 
 // ---------------------------------------------------------------- byte-class helpers
 __device__ __forceinline__ uint32_t movemask4(uint32_t m) {  // 0xFF/0x00 bytes -> 4 bits
@@ -209,8 +234,25 @@ __device__ uint32_t slow_word_len(const Params& P, const TileView& tv, long long
 // first.  Scans the stage 16 bytes at a time, then global memory (slow path).
 __device__ long long find_quote(const Params& P, const TileView& tv, long long q0, long long p_marker) {
   const long long N = static_cast<long long>(P.nbytes);
+  const long long lim = min(tv.stg_hi, N);
   long long q = q0;
-  while (q < tv.stg_hi && q < N) {
+  while (q < lim && ((q - tv.sbase) & 3)) {               // align to a 4-byte SMEM word
+    if (tv.is_start(q)) return -1;
+    if (tv.sb[q - tv.sbase] == '"') return q;
+    ++q;
+  }
+  while (q + 4 <= lim) {                                   // 4 bytes per step (SWAR)
+    const long long i = q - tv.sbase;
+    const uint32_t w = *reinterpret_cast<const uint32_t*>(tv.sb + i);
+    const uint32_t st = (tv.bm[i >> 5] >> (i & 31)) & 0xFu;
+    const uint32_t m = eq_mask4(w, 0x22222222u) | st;
+    if (m) {
+      const uint32_t j = __ffs(m) - 1;
+      return ((st >> j) & 1u) ? -1 : q + j;               // record ends first -> unclosed
+    }
+    q += 4;
+  }
+  while (q < lim) {
     if (tv.is_start(q)) return -1;
     if (tv.sb[q - tv.sbase] == '"') return q;
     ++q;
@@ -222,47 +264,129 @@ __device__ long long find_quote(const Params& P, const TileView& tv, long long q
   return -1;
 }
 
-__device__ __forceinline__ uint64_t key_of(const uint8_t* kp, uint32_t len, const Params& P) {
+// Same function as hash_bytes (common.cuh) for a key lying inside the SMEM stage: aligned
+// 4-byte SMEM loads + funnel shifts instead of byte loads.
+__device__ __forceinline__ uint32_t smem_word_at(const uint8_t* sb, uint32_t i) {  // 4 bytes at any i
+  const uint32_t a = i & ~3u, sh = (i & 3u) * 8;
+  const uint32_t w0 = *reinterpret_cast<const uint32_t*>(sb + a);
+  if (!sh) return w0;
+  const uint32_t w1 = *reinterpret_cast<const uint32_t*>(sb + a + 4);
+  return __funnelshift_r(w0, w1, sh);
+}
+__device__ __forceinline__ uint64_t hash_smem(const uint8_t* sb, uint32_t i, uint32_t len, uint64_t seed) {
+  uint64_t h = seed ^ (static_cast<uint64_t>(len) * 0x9E3779B97F4A7C15ULL);
+  uint32_t k = 0;
+  for (; k + 8 <= len; k += 8) {
+    const uint64_t b = static_cast<uint64_t>(smem_word_at(sb, i + k)) |
+                       (static_cast<uint64_t>(smem_word_at(sb, i + k + 4)) << 32);
+    h = mix64(h ^ b) + 0x632BE59BD9B4E019ULL;
+  }
+  if (k < len) {
+    const uint32_t r = len - k;
+    uint64_t b = static_cast<uint64_t>(smem_word_at(sb, i + k));
+    if (r > 4) b |= static_cast<uint64_t>(smem_word_at(sb, i + k + 4)) << 32;
+    b &= (1ULL << (8 * r)) - 1ULL;
+    h = mix64(h ^ b ^ 0xA5A5A5A5ULL);
+  }
+  return mix64(h);
+}
+
+// Sort key of the key bytes [q, q + len): inline when <= 7 bytes, else the 64-bit hash.
+__device__ __forceinline__ uint64_t key_at(const Params& P, const TileView& tv, long long q, uint32_t len) {
+  const bool in_stage = (q + static_cast<long long>(len) <= tv.stg_hi) && (q - tv.sbase + len + 12 <= kStageBytes);
   if (len <= 7) {
     uint64_t b = 0;
-    for (uint32_t i = 0; i < len; ++i) b |= static_cast<uint64_t>(kp[i]) << (8 * i);
+    if (in_stage) {
+      const uint32_t i = static_cast<uint32_t>(q - tv.sbase);
+      b = static_cast<uint64_t>(smem_word_at(tv.sb, i)) | (static_cast<uint64_t>(smem_word_at(tv.sb, i + 4)) << 32);
+    } else {
+      for (uint32_t k = 0; k < len; ++k) b |= static_cast<uint64_t>(P.rec[q + k]) << (8 * k);
+    }
     return inline_key(b, len);
   }
-  return hashed_key(hash_bytes(kp, len, P.hash_seed), (P.flags & 8u) != 0);
+  const uint64_t h = in_stage ? hash_smem(tv.sb, static_cast<uint32_t>(q - tv.sbase), len, P.hash_seed)
+                              : hash_bytes(P.rec + q, len, P.hash_seed);
+  return hashed_key(h, (P.flags & 8u) != 0);
 }
 
 // ---------------------------------------------------------------- emit allocator
+// Shared cursor: 32-bit [generation:8 | count:24] (native ATOMS.ADD).  half = generation & 1.
+// Flush bases are kept multiples of 4 pairs so that every SoA run of a flushed half is 16-byte
+// aligned in global memory and leaves SMEM as one TMA bulk store (cp.async.bulk global<-shared);
+// the <= 3 filler entries carry the workload's sentinel key, which sorts after every real key
+// and is excluded from the groups (DevState::pads).  StringMatch (Map-only, sparse) flushes with
+// plain stores and needs no filler.
 struct Slot { uint32_t half, base; };
+constexpr uint32_t kCntMask = 0xFFFFFFu;
 
-__device__ __forceinline__ Slot reserve(OutCtl* oc, uint32_t cnt, uint32_t cap) {
+template <int W>
+__device__ __forceinline__ uint64_t sentinel_key(const Params& P) {
+  if constexpr (W == kKM) return P.k <= 255 ? 255ULL : 65535ULL;
+  return ~0ULL;
+}
+
+template <int W>
+__device__ void seal(const Params& P, OutCtl* oc, uint8_t* outh, uint32_t gen8, uint32_t h, uint32_t cnt,
+                     bool last) {
+  using F = PairFmt<W>;
+  const uint32_t full_gen = oc->nsealed;                       // full generation number
+  if (!last && full_gen >= 1) mbar_wait(&oc->done[(full_gen - 1) & 1u], ((full_gen - 1) >> 1) & 1u);
+  if (!last) {
+    oc->committed[h ^ 1u] = 0;
+    oc->nsealed = full_gen + 1;
+    __threadfence_block();
+    atomicExch(&oc->cur, ((gen8 + 1) & 0xFFu) << 24);          // other warps continue in the other half
+  } else {
+    oc->final_seq = full_gen;
+    oc->is_final = 1;
+  }
+  uint32_t cnt4 = cnt;
+  if constexpr (W != kSM) {
+    cnt4 = (cnt + 3u) & ~3u;
+    uint8_t* half = outh + h * kOutHalf;
+    for (uint32_t i = cnt; i < cnt4; ++i) {                   // sentinel filler entries
+      reinterpret_cast<uint64_t*>(half)[i] = sentinel_key<W>(P);
+      if constexpr (F::kKref) reinterpret_cast<uint64_t*>(half)[F::kCap + i] = 0;
+    }
+  }
+  unsigned long long gb = 0;
+  if (cnt4) {
+    gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(cnt4));  // ONE global atomic
+    atomicAdd(&P.st->flushes, 1ULL);
+    if (cnt4 != cnt) atomicAdd(&P.st->pads, static_cast<unsigned long long>(cnt4 - cnt));
+  }
+  oc->fcount[h] = cnt4;
+  oc->fbase[h] = gb;
+  __threadfence_block();
+  mbar_arrive(&oc->req[h]);
+}
+
+template <int W>
+__device__ __forceinline__ Slot reserve(const Params& P, OutCtl* oc, uint8_t* outh, uint32_t cnt, uint32_t cap) {
   const uint32_t lane = threadIdx.x & 31;
   for (;;) {
-    unsigned long long old = 0;
-    if (lane == 0) old = atomicAdd(&oc->cur, static_cast<unsigned long long>(cnt));
+    uint32_t old = 0;
+    if (lane == 0) old = atomicAdd(&oc->cur, cnt);
     old = __shfl_sync(kFull, old, 0);
-    const uint32_t gen = static_cast<uint32_t>(old >> 32), base = static_cast<uint32_t>(old);
+    const uint32_t gen = old >> 24, base = old & kCntMask;
     const uint32_t h = gen & 1u;
     if (base + cnt <= cap) return {h, base};
     if (lane == 0) {
       if (base <= cap) {
         // This warp crossed the capacity first: it seals half h (L113 "overflow handling").
         volatile unsigned int* cm = &oc->committed[h];
-        while (*cm != base) __nanosleep(20);
-        if (gen >= 1) mbar_wait(&oc->done[(gen - 1) & 1u], ((gen - 1) >> 1) & 1u);  // other half free
-        oc->committed[h ^ 1u] = 0;
-        oc->fcount[h] = base;
-        __threadfence_block();
-        atomicExch(&oc->cur, static_cast<unsigned long long>(gen + 1) << 32);
-        mbar_arrive(&oc->req[h]);
+        while (*cm != base) __nanosleep(32);
+        seal<W>(P, oc, outh, gen, h, base, false);
       } else {
-        volatile unsigned long long* c = &oc->cur;
-        while (static_cast<uint32_t>(*c >> 32) == gen) __nanosleep(32);
+        volatile unsigned int* c = &oc->cur;
+        while ((*c >> 24) == gen) __nanosleep(128);
       }
     }
     __syncwarp();
   }
 }
 __device__ __forceinline__ void commit(OutCtl* oc, Slot s, uint32_t cnt) {
+  fence_proxy_async_shared();   // generic SMEM writes -> visible to the TMA store of the flush
   __syncwarp();
   if ((threadIdx.x & 31) == 0) {
     __threadfence_block();
@@ -271,6 +395,16 @@ __device__ __forceinline__ void commit(OutCtl* oc, Slot s, uint32_t cnt) {
 }
 
 // ---------------------------------------------------------------- flush warp
+__device__ __forceinline__ void tma_store_1d(void* gdst, const void* ssrc, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gdst), "r"(smem_u32(ssrc)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void tma_store_commit_and_wait_read() {
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+  asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+
 template <int W>
 __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   using F = PairFmt<W>;
@@ -279,43 +413,29 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
     const uint32_t h = f & 1u;
     mbar_wait(&oc->req[h], (f >> 1) & 1u);
     const uint32_t cnt = *reinterpret_cast<volatile unsigned int*>(&oc->fcount[h]);
+    const unsigned long long gb = *reinterpret_cast<volatile unsigned long long*>(&oc->fbase[h]);
     const bool fin = *reinterpret_cast<volatile unsigned int*>(&oc->is_final) &&
-                     *reinterpret_cast<volatile unsigned int*>(&oc->final_gen) == f;
-    if (cnt) {
-      unsigned long long gb = 0;
-      if (lane == 0) {
-        gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(cnt));  // ONE global atomic
-        atomicAdd(&P.st->flushes, 1ULL);
-      }
-      gb = __shfl_sync(kFull, gb, 0);
-      if (gb + cnt <= P.cap_pairs) {
-        const uint8_t* half = smem + Layout::out + h * kOutHalf;
-        const uint64_t* sh = reinterpret_cast<const uint64_t*>(half);
+                     *reinterpret_cast<volatile unsigned int*>(&oc->final_seq) == f;
+    const uint8_t* half = smem + Layout::out + h * kOutHalf;
+    if (cnt && gb + cnt <= P.cap_pairs) {
+      const uint64_t* sh = reinterpret_cast<const uint64_t*>(half);
+      const uint8_t* sv = half + F::kCap * (F::kKref ? 16 : 8);
+      if constexpr (W == kSM) {
         for (uint32_t i = lane; i < cnt; i += 32) P.oh[gb + i] = sh[i];
-        if constexpr (F::kKref) {
-          const uint64_t* sk = sh + F::kCap;
-          for (uint32_t i = lane; i < cnt; i += 32) P.okref[gb + i] = sk[i];
-        }
-        const uint8_t* sv = half + F::kCap * (F::kKref ? 16 : 8);
-        if constexpr (F::kV == 4) {
-          const uint32_t* s4 = reinterpret_cast<const uint32_t*>(sv);
-          uint32_t* g4 = reinterpret_cast<uint32_t*>(P.ov) + gb;
-          for (uint32_t i = lane; i < cnt; i += 32) g4[i] = s4[i];
-        } else if constexpr (F::kV == 8) {
-          const uint64_t* s8 = reinterpret_cast<const uint64_t*>(sv);
-          uint64_t* g8 = reinterpret_cast<uint64_t*>(P.ov) + gb;
-          for (uint32_t i = lane; i < cnt; i += 32) g8[i] = s8[i];
-        } else if constexpr (F::kV == 32) {
-          const uint4* s16 = reinterpret_cast<const uint4*>(sv);
-          uint4* g16 = reinterpret_cast<uint4*>(P.ov) + gb * 2;
-          for (uint32_t i = lane; i < 2 * cnt; i += 32) g16[i] = s16[i];
-        }
+      } else if (lane == 0) {
+        // A4 staging-out as three TMA bulk stores (16-B aligned: gb % 4 == 0, cnt % 4 == 0)
+        fence_proxy_async_shared();
+        tma_store_1d(P.oh + gb, sh, cnt * 8);
+        if constexpr (F::kKref) tma_store_1d(P.okref + gb, sh + F::kCap, cnt * 8);
+        if constexpr (F::kV > 0) tma_store_1d(P.ov + gb * F::kV, sv, cnt * F::kV);
+        tma_store_commit_and_wait_read();          // SMEM may be reused once the stores have read it
       }
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(&oc->done[h]);
     if (fin) break;
   }
+  if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // global writes complete
 }
 
 // ---------------------------------------------------------------- producer warp
@@ -329,6 +449,30 @@ __device__ void stage_copy_edges(uint8_t* d, const uint8_t* g, uint64_t len, uin
   for (uint32_t i = lane; i < tail; i += 32) d[head + body + i] = g[head + body + i];
   body_off = head;
   body_len = body;
+}
+
+// Text tiles: once the TMA of stage s has landed, the producer warp turns the staged offsets
+// slice into the record-start bitmap and releases the stage to the map warps (ready[s]).
+// Done one tile behind the TMA issue, so the copy latency is hidden.
+__device__ void finish_stage(const Params& P, uint8_t* smem, uint32_t it) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout::full);
+  uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout::ready);
+  mbar_wait(&full[s], ph);
+  const StageHdr* hd = reinterpret_cast<const StageHdr*>(smem + Layout::hdr + s * 128);
+  uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout::bits + s * kBitBytes);
+  const uint64_t* soff = reinterpret_cast<const uint64_t*>(smem + Layout::offs + s * kOffBytes + hd->off_shift);
+  const uint64_t ra = hd->ra, cnt = hd->rb - hd->ra;
+  const long long sbase = hd->sbase;
+  const bool staged = hd->off_staged != 0;
+  for (uint64_t r = lane; r < cnt; r += 32) {
+    const uint64_t pos = staged ? soff[r] : P.off[ra + r];
+    const long long i = static_cast<long long>(pos) - sbase;
+    atomicOr(&bm[i >> 5], 1u << (i & 31));
+  }
+  __syncwarp();
+  if (lane == 0) mbar_arrive(&ready[s]);
 }
 
 template <int W>
@@ -409,16 +553,21 @@ __device__ void producer_loop(const Params& P, uint8_t* smem) {
           if (b_len) tma_load_1d(d + b_off, g + b_off, b_len, &full[s]);
           if (o_len) tma_load_1d(so + shift + o_off, og + o_off, o_len, &full[s]);
         }
+        if (it >= kLag) finish_stage(P, smem, it - kLag);
       }
       ++it;
     }
+  }
+  if constexpr (W != kKM) {
+    for (uint32_t j = (it >= kLag ? it - kLag : 0); j < it; ++j) finish_stage(P, smem, j);
   }
   // end-of-work marker
   const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
   mbar_wait(&empty[s], ph ^ 1u);
   if (lane == 0) {
     reinterpret_cast<StageHdr*>(smem + Layout::hdr + s * 128)->t = -1;
-    mbar_arrive(&full[s]);
+    if constexpr (W == kKM) mbar_arrive(&full[s]);
+    else mbar_arrive(reinterpret_cast<uint64_t*>(smem + Layout::ready) + s);
   }
 }
 
@@ -500,7 +649,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
   const uint32_t cnt = __popc(emit_mask);
   const uint32_t total = __reduce_add_sync(kFull, cnt);
   if (total == 0) return;
-  const Slot slot = reserve(oc, total, P.out_cap);
+  const Slot slot = reserve<W>(P, oc, outh, total, P.out_cap);
   uint8_t* half = outh + slot.half * kOutHalf;
   uint64_t* sh = reinterpret_cast<uint64_t*>(half);
   uint64_t* sk = sh + F::kCap;
@@ -519,13 +668,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
       if constexpr (W == kWC) {
         const uint32_t rest = nb >> (j + 1);
         uint32_t len = rest ? static_cast<uint32_t>(__ffs(rest)) : slow_word_len(P, tv, p, p0 + 32);
-        uint64_t key;
-        if (len <= 7) {
-          key = inline_key(window8(x, j), len);
-        } else {
-          const uint8_t* kp = (p + len <= tv.stg_hi) ? tv.sb + (p - tv.sbase) : P.rec + p;
-          key = hashed_key(hash_bytes(kp, len, P.hash_seed), (P.flags & 8u) != 0);
-        }
+        const uint64_t key = (len <= 7) ? inline_key(window8(x, j), len) : key_at(P, tv, p, len);
         if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
         sh[idx] = key;
         sk[idx] = (reinterpret_cast<uint64_t>(P.rec + p) << 16) | len;
@@ -536,9 +679,8 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
         uint32_t len = nth == 0 ? aux[0] : aux[1];
         ++nth;
         const long long q0 = p + 9;
-        const uint8_t* kp = (q0 + len <= tv.stg_hi) ? tv.sb + (q0 - tv.sbase) : P.rec + q0;
         if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
-        sh[idx] = key_of(kp, len, P);
+        sh[idx] = key_at(P, tv, q0, len);
         sk[idx] = (reinterpret_cast<uint64_t>(P.rec + q0) << 16) | len;
         reinterpret_cast<uint64_t*>(sv)[idx] = P.gbase + static_cast<uint64_t>(q0);
       }
@@ -559,7 +701,8 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   const float* cent = reinterpret_cast<const float*>(smem + Layout::cent);
   for (uint32_t it = 0;; ++it) {
     const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
-    mbar_wait(&full[s], ph);
+    if constexpr (W == kKM) mbar_wait(&full[s], ph);
+    else mbar_wait(reinterpret_cast<uint64_t*>(smem + Layout::ready) + s, ph);
     const StageHdr hd = *reinterpret_cast<const StageHdr*>(smem + Layout::hdr + s * 128);
     if (hd.t < 0) break;
     const uint8_t* sb = smem + Layout::bytes + s * kStageBytes;
@@ -576,19 +719,38 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         const float4 b = reinterpret_cast<const float4*>(pt)[1];
         x[0] = a.x; x[1] = a.y; x[2] = a.z; x[3] = a.w; x[4] = b.x; x[5] = b.y; x[6] = b.z; x[7] = b.w;
         float bd = 0.0f;
-        for (uint32_t j = 0; j < P.k; ++j) {   // C-2 KM: fp32 RN, explicit fmaf chain, ties -> lowest j
-          const float4 c0 = reinterpret_cast<const float4*>(cent + j * 8)[0];
-          const float4 c1 = reinterpret_cast<const float4*>(cent + j * 8)[1];
+        // C-2 KM: fp32 RN, explicit chain d = fma(x_t - c_t, x_t - c_t, d) over t = 0..7, ties ->
+        // lowest j.  Two centroids per instruction with packed FADD2/FFMA2 (each lane of the pair
+        // performs exactly the scalar RN operations, so the result is bit-identical).
+        uint64_t X[8];
+#pragma unroll
+        for (int t = 0; t < 8; ++t) X[t] = f2pack(x[t], x[t]);
+        const uint32_t kp = P.k & ~1u;
+        bool first = true;
+#pragma unroll 2
+        for (uint32_t j = 0; j < kp; j += 2) {
+          const ulonglong2* cp = reinterpret_cast<const ulonglong2*>(cent + j * 8);   // pair layout
+          const ulonglong2 q0 = cp[0], q1 = cp[1], q2 = cp[2], q3 = cp[3];
+          const uint64_t C[8] = {q0.x, q0.y, q1.x, q1.y, q2.x, q2.y, q3.x, q3.y};
+          uint64_t D = 0;
+#pragma unroll
+          for (int t = 0; t < 8; ++t) {
+            const uint64_t E = f2sub(X[t], C[t]);
+            D = f2fma(E, E, D);
+          }
+          float d0, d1;
+          f2unpack(D, d0, d1);
+          if (first || d0 < bd) { bd = d0; best = j; }
+          first = false;
+          if (d1 < bd) { bd = d1; best = j + 1; }
+        }
+        if (P.k & 1u) {
+          const uint32_t j = P.k - 1;
+          const float* c = cent + j * 8;   // last centroid stored unpaired
           float d = 0.0f, e;
-          e = __fsub_rn(x[0], c0.x); d = __fmaf_rn(e, e, d);
-          e = __fsub_rn(x[1], c0.y); d = __fmaf_rn(e, e, d);
-          e = __fsub_rn(x[2], c0.z); d = __fmaf_rn(e, e, d);
-          e = __fsub_rn(x[3], c0.w); d = __fmaf_rn(e, e, d);
-          e = __fsub_rn(x[4], c1.x); d = __fmaf_rn(e, e, d);
-          e = __fsub_rn(x[5], c1.y); d = __fmaf_rn(e, e, d);
-          e = __fsub_rn(x[6], c1.z); d = __fmaf_rn(e, e, d);
-          e = __fsub_rn(x[7], c1.w); d = __fmaf_rn(e, e, d);
-          if (j == 0 || d < bd) { bd = d; best = j; }
+#pragma unroll
+          for (int t = 0; t < 8; ++t) { e = __fsub_rn(x[t], c[t]); d = __fmaf_rn(e, e, d); }
+          if (first || d < bd) { bd = d; best = j; }
         }
       }
       const uint32_t m = __ballot_sync(kFull, valid);
@@ -596,7 +758,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       if (lane == 0) mbar_arrive(&empty[s]);   // stage no longer read by this warp
       if (m) {
         const uint32_t total = __popc(m);
-        const Slot slot = reserve(oc, total, P.out_cap);
+        const Slot slot = reserve<W>(P, oc, outh, total, P.out_cap);
         if (valid) {
           const uint32_t idx = slot.base + __popc(m & lanemask_lt());
           uint8_t* half = outh + slot.half * kOutHalf;
@@ -608,16 +770,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         commit(oc, slot, total);
       }
     } else {
-      // record-start bitmap from the staged (or global) offsets slice
-      uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout::bits + s * kBitBytes);
-      const uint64_t* soff = reinterpret_cast<const uint64_t*>(smem + Layout::offs + s * kOffBytes + hd.off_shift);
-      const uint64_t cnt = hd.rb - hd.ra;
-      for (uint64_t r = tid; r < cnt; r += kNMap * 32) {
-        const uint64_t pos = hd.off_staged ? soff[r] : P.off[hd.ra + r];
-        const long long i = static_cast<long long>(pos) - hd.sbase;
-        atomicOr(&bm[i >> 5], 1u << (i & 31));
-      }
-      named_bar_sync(1, kNMap * 32);
+      const uint32_t* bm = reinterpret_cast<const uint32_t*>(smem + Layout::bits + s * kBitBytes);
       TileView tv{sb, bm, hd.sbase, hd.stg_hi};
       for (uint32_t w = warp; w < kNWin; w += kNMap) {
         const long long wp = hd.chunk0 + static_cast<long long>(w) * kWin;
@@ -630,17 +783,11 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       if (lane == 0) mbar_arrive(&empty[s]);
     }
   }
-  // final flush of the partially filled half (all map warps done)
+  // final flush of the partially filled half (all map warps done, nothing pending)
   named_bar_sync(2, kNMap * 32);
   if (threadIdx.x == 0) {
-    const unsigned long long cur = *reinterpret_cast<volatile unsigned long long*>(&oc->cur);
-    const uint32_t gen = static_cast<uint32_t>(cur >> 32), cnt = static_cast<uint32_t>(cur);
-    const uint32_t h = gen & 1u;
-    oc->fcount[h] = cnt;
-    oc->final_gen = gen;
-    oc->is_final = 1;
-    __threadfence_block();
-    mbar_arrive(&oc->req[h]);
+    const uint32_t cur = *reinterpret_cast<volatile unsigned int*>(&oc->cur);
+    seal<W>(P, oc, outh, cur >> 24, (cur >> 24) & 1u, cur & kCntMask, true);
   }
 }
 
@@ -650,25 +797,33 @@ __global__ void __launch_bounds__(kThreads, 1) k_map(Params P) {
   OutCtl* oc = reinterpret_cast<OutCtl*>(smem + Layout::ctl);
   if (threadIdx.x == 0) {
     oc->cur = 0;
+    oc->final_seq = 0;
+    oc->fbase[0] = oc->fbase[1] = 0;
     oc->committed[0] = oc->committed[1] = 0;
     oc->fcount[0] = oc->fcount[1] = 0;
-    oc->final_gen = 0;
+    oc->nsealed = 0;
     oc->is_final = 0;
     mbar_init(&oc->req[0], 1); mbar_init(&oc->req[1], 1);
-    mbar_init(&oc->done[0], 1); mbar_init(&oc->done[1], 1);
+    mbar_init(&oc->done[0], kNFlush); mbar_init(&oc->done[1], kNFlush);
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout::full);
     uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout::empty);
-    for (int s = 0; s < kStages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], kNMap); }
+    uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout::ready);
+    for (int s = 0; s < kStages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], kNMap); mbar_init(&ready[s], 1); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if constexpr (W == kKM) {
     float* cent = reinterpret_cast<float*>(smem + Layout::cent);
-    for (uint32_t i = threadIdx.x; i < P.k * 8; i += blockDim.x) cent[i] = P.cent[i];
+    // pair layout: centroids (2p, 2p+1) interleaved per coordinate -> f32x2 operands
+    for (uint32_t i = threadIdx.x; i < P.k * 8; i += blockDim.x) {
+      const uint32_t j = i / 8, t = i % 8;
+      const uint32_t kp = P.k & ~1u;
+      cent[j < kp ? ((j & ~1u) * 8 + t * 2 + (j & 1u)) : i] = P.cent[i];
+    }
   }
   __syncthreads();
   const uint32_t warp = threadIdx.x >> 5;
   if (warp == kProdWarp) producer_loop<W>(P, smem);
-  else if (warp == kFlushWarp) flush_loop<W>(P, smem, oc);
+  else if (warp >= kFlushWarp0) flush_loop<W>(P, smem, oc);
   else map_loop<W>(P, smem, oc);
 }
 

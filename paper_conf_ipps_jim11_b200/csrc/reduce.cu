@@ -33,42 +33,78 @@ __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
   return v;
 }
 
+// 8 key bytes starting at p (little-endian); reads only the aligned 8-byte words that hold
+// bytes [p, p + need), need <= 8, so it never touches a word outside the key's own words.
+__device__ __forceinline__ uint64_t load8(const uint8_t* p, uint32_t need) {
+  const uintptr_t a = reinterpret_cast<uintptr_t>(p) & ~static_cast<uintptr_t>(7);
+  const uint32_t sh = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(p) & 7u) * 8;
+  const uint64_t w0 = __ldg(reinterpret_cast<const unsigned long long*>(a));
+  if (sh == 0) return w0;
+  uint64_t v = w0 >> sh;
+  if (sh / 8 + need > 8) v |= static_cast<uint64_t>(__ldg(reinterpret_cast<const unsigned long long*>(a + 8))) << (64 - sh);
+  return v;
+}
+
+// Byte equality of two keys given as kref = (address << 16) | length.
 __device__ bool key_bytes_equal(uint64_t ka, uint64_t kb) {
   const uint32_t la = static_cast<uint32_t>(ka & 0xFFFF), lb = static_cast<uint32_t>(kb & 0xFFFF);
   if (la != lb) return false;
   const uint8_t* pa = reinterpret_cast<const uint8_t*>(ka >> 16);
   const uint8_t* pb = reinterpret_cast<const uint8_t*>(kb >> 16);
-  for (uint32_t i = 0; i < la; ++i)
-    if (pa[i] != pb[i]) return false;
+  for (uint32_t i = 0; i < la; i += 8) {
+    const uint32_t need = min(8u, la - i);
+    const uint64_t mask = need == 8 ? ~0ULL : ((1ULL << (8 * need)) - 1ULL);
+    if (((load8(pa + i, need) ^ load8(pb + i, need)) & mask) != 0) return false;
+  }
   return true;
 }
+
+// Each warp owns 512 consecutive sorted positions (16 steps of 32 lanes: coalesced loads);
+// a lane compares its key with the previous position's key (shuffle from the previous lane).
+constexpr int kSegWarp = 32 * kSegIPT;   // positions per warp
 
 __global__ void __launch_bounds__(kSegThreads) k_seg_count(const uint64_t* __restrict__ sk,
                                                          const uint32_t* __restrict__ perm,
                                                          const uint64_t* __restrict__ kref, uint64_t m,
                                                          uint32_t* counts, DevState* st) {
   __shared__ uint32_t red[kSegThreads / 32];
-  const uint64_t base = static_cast<uint64_t>(blockIdx.x) * kSegTile + static_cast<uint64_t>(threadIdx.x) * kSegIPT;
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint64_t wbase = static_cast<uint64_t>(blockIdx.x) * kSegTile + static_cast<uint64_t>(warp) * kSegWarp;
   uint32_t heads = 0, coll = 0;
-  uint64_t prev = (base > 0 && base - 1 < m) ? sk[base - 1] : 0;
+  uint64_t carry_k = (wbase > 0 && wbase - 1 < m) ? sk[wbase - 1] : 0;     // key before this step
+  uint64_t carry_r = 0;                                                     // its kref (if loaded)
+  bool carry_has_r = false;
+#pragma unroll 4
   for (int j = 0; j < kSegIPT; ++j) {
-    const uint64_t i = base + j;
-    if (i >= m) break;
-    const uint64_t k = sk[i];
-    if (i == 0 || k != prev) {
-      ++heads;
-    } else if ((k & kHashedBit) && kref) {
-      if (!key_bytes_equal(kref[perm[i]], kref[perm[i - 1]])) ++coll;
+    const uint64_t i = wbase + static_cast<uint64_t>(j) * 32 + lane;
+    const bool valid = i < m;
+    const uint64_t k = valid ? sk[i] : 0;
+    uint64_t prev = __shfl_up_sync(0xffffffffu, k, 1);
+    if (lane == 0) prev = carry_k;
+    const bool head = valid && (i == 0 || k != prev);
+    heads += head ? 1u : 0u;
+    // byte verification of equal hashed keys (C-3 #13): adjacent pairs inside an equal-hash run
+    const bool hashed_run = valid && kref && (k & kHashedBit) && !head;
+    const bool need_r = valid && kref && (k & kHashedBit);
+    const unsigned any = __ballot_sync(0xffffffffu, need_r);
+    uint64_t r = 0;
+    if (any) {
+      if (need_r) r = kref[perm[i]];
+      uint64_t rp = __shfl_up_sync(0xffffffffu, r, 1);
+      if (lane == 0) rp = carry_has_r ? carry_r : ((hashed_run && i > 0) ? kref[perm[i - 1]] : 0);
+      if (hashed_run && !key_bytes_equal(r, rp)) ++coll;
     }
-    prev = k;
+    carry_k = __shfl_sync(0xffffffffu, k, 31);
+    carry_r = __shfl_sync(0xffffffffu, r, 31);
+    carry_has_r = __shfl_sync(0xffffffffu, need_r ? 1u : 0u, 31) != 0;
   }
   if (coll) atomicAdd(&st->collisions, coll);
-  uint32_t w = __reduce_add_sync(0xffffffffu, heads);
-  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = w;
+  const uint32_t w = __reduce_add_sync(0xffffffffu, heads);
+  if (lane == 0) red[warp] = w;
   __syncthreads();
   if (threadIdx.x == 0) {
     uint32_t t = 0;
-    for (int i = 0; i < kSegThreads / 32; ++i) t += red[i];
+    for (int q = 0; q < kSegThreads / 32; ++q) t += red[q];
     counts[blockIdx.x] = t;
   }
 }
@@ -77,39 +113,45 @@ __global__ void __launch_bounds__(kSegThreads) k_seg_write(const uint64_t* __res
                                                          const uint64_t* __restrict__ tile_base,
                                                          uint64_t* seg_start) {
   __shared__ uint32_t wsum[kSegThreads / 32];
-  const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const uint64_t base = static_cast<uint64_t>(blockIdx.x) * kSegTile + static_cast<uint64_t>(tid) * kSegIPT;
-  uint32_t hm = 0;
-  uint64_t prev = (base > 0 && base - 1 < m) ? sk[base - 1] : 0;
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint64_t wbase = static_cast<uint64_t>(blockIdx.x) * kSegTile + static_cast<uint64_t>(warp) * kSegWarp;
+  // pass 1: heads of this warp's 512 positions (bitmask per step kept in registers)
+  uint32_t hm[kSegIPT];
+  uint32_t wcount = 0;
+  uint64_t carry_k = (wbase > 0 && wbase - 1 < m) ? sk[wbase - 1] : 0;
+#pragma unroll
   for (int j = 0; j < kSegIPT; ++j) {
-    const uint64_t i = base + j;
-    if (i >= m) break;
-    const uint64_t k = sk[i];
-    if (i == 0 || k != prev) hm |= 1u << j;
-    prev = k;
+    const uint64_t i = wbase + static_cast<uint64_t>(j) * 32 + lane;
+    const bool valid = i < m;
+    const uint64_t k = valid ? sk[i] : 0;
+    uint64_t prev = __shfl_up_sync(0xffffffffu, k, 1);
+    if (lane == 0) prev = carry_k;
+    hm[j] = __ballot_sync(0xffffffffu, valid && (i == 0 || k != prev));
+    wcount += __popc(hm[j]);
+    carry_k = __shfl_sync(0xffffffffu, k, 31);
   }
-  const uint32_t c = __popc(hm);
-  const uint32_t inc = warp_inclusive_add(c);
-  if (lane == 31) wsum[warp] = inc;
+  if (lane == 0) wsum[warp] = wcount;
   __syncthreads();
   uint32_t wpre = 0, tot = 0;
   for (int w = 0; w < kSegThreads / 32; ++w) {
     wpre += (w < static_cast<int>(warp)) ? wsum[w] : 0u;
     tot += wsum[w];
   }
-  uint64_t r = tile_base[blockIdx.x] + wpre + inc - c;
-  while (hm) {
-    const int j = __ffs(hm) - 1;
-    hm &= hm - 1;
-    seg_start[r++] = base + j;
+  uint64_t r = tile_base[blockIdx.x] + wpre;
+#pragma unroll
+  for (int j = 0; j < kSegIPT; ++j) {
+    const uint64_t i = wbase + static_cast<uint64_t>(j) * 32 + lane;
+    if ((hm[j] >> lane) & 1u) seg_start[r + __popc(hm[j] & lanemask_lt())] = i;
+    r += __popc(hm[j]);
   }
   const uint64_t tile_end = static_cast<uint64_t>(blockIdx.x + 1) * kSegTile;
-  if (tid == 0 && tile_end >= m) seg_start[tile_base[blockIdx.x] + tot] = m;  // sentinel S -> m
+  if (threadIdx.x == 0 && tile_end >= m) seg_start[tile_base[blockIdx.x] + tot] = m;  // sentinel S -> m
 }
 
 // ---------------------------------------------------------------- WordCount reduce (u64 sums)
+template <typename V>
 __global__ void k_reduce_wc_small(const uint64_t* __restrict__ seg, uint64_t nseg, const uint32_t* __restrict__ perm,
-                                  const uint32_t* __restrict__ v, uint64_t* counts, uint64_t* worklist,
+                                  const V* __restrict__ v, uint64_t* counts, uint64_t* worklist,
                                   DevState* st) {
   const uint64_t gw = (blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x) >> 5;
   const uint64_t nw = (static_cast<uint64_t>(gridDim.x) * blockDim.x) >> 5;
@@ -118,6 +160,7 @@ __global__ void k_reduce_wc_small(const uint64_t* __restrict__ seg, uint64_t nse
     const uint64_t a = seg[s], b = seg[s + 1], size = b - a;
     if (size <= kSmallWC) {
       uint64_t sum = 0;
+#pragma unroll 4
       for (uint64_t i = a + lane; i < b; i += 32) sum += v[perm[i]];
       sum = warp_sum_u64(sum);
       if (lane == 0) counts[s] = sum;
@@ -130,9 +173,10 @@ __global__ void k_reduce_wc_small(const uint64_t* __restrict__ seg, uint64_t nse
   }
 }
 
+template <typename V>
 __global__ void __launch_bounds__(256) k_reduce_wc_large(const uint64_t* __restrict__ seg,
                                                        const uint32_t* __restrict__ perm,
-                                                       const uint32_t* __restrict__ v, uint64_t* counts,
+                                                       const V* __restrict__ v, uint64_t* counts,
                                                        const uint64_t* __restrict__ worklist, DevState* st) {
   __shared__ unsigned long long item;
   __shared__ uint64_t red[8];
@@ -145,6 +189,7 @@ __global__ void __launch_bounds__(256) k_reduce_wc_large(const uint64_t* __restr
     const uint64_t w = worklist[it], s = w >> 24, t = w & 0xFFFFFF;
     const uint64_t a = seg[s] + t * kLargeTile, b = min(seg[s + 1], a + kLargeTile);
     uint64_t sum = 0;
+#pragma unroll 8
     for (uint64_t i = a + threadIdx.x; i < b; i += blockDim.x) sum += v[perm[i]];
     sum = warp_sum_u64(sum);
     if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = sum;
@@ -242,18 +287,21 @@ __global__ void __launch_bounds__(256) k_reduce_km_large(const uint64_t* __restr
 }
 
 __global__ void k_km_finalize(const double* sums, const unsigned long long* cnts, const float* cent, uint32_t k,
-                              uint8_t* vals, uint64_t* val_off, uint8_t* keys, uint64_t* key_off) {
-  const uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
-  if (j > k) return;
-  if (j == k) { val_off[k] = 40ULL * k; key_off[k] = 4ULL * k; return; }
+                              const uint32_t* list, uint32_t nlist, uint8_t* vals, uint64_t* val_off, uint8_t* keys,
+                              uint64_t* key_off) {
+  const uint32_t n = list ? nlist : k;
+  const uint32_t o = blockIdx.x * blockDim.x + threadIdx.x;   // output slot
+  if (o > n) return;
+  if (o == n) { val_off[n] = 40ULL * n; key_off[n] = 4ULL * n; return; }
+  const uint32_t j = list ? list[o] : o;
   const unsigned long long c = cnts[j];
-  float* o = reinterpret_cast<float*>(vals + 40ULL * j);
+  float* out = reinterpret_cast<float*>(vals + 40ULL * o);
   for (int t = 0; t < 8; ++t)
-    o[t] = c ? static_cast<float>(__ddiv_rn(sums[j * 8 + t], static_cast<double>(c))) : cent[j * 8 + t];
-  *reinterpret_cast<unsigned long long*>(vals + 40ULL * j + 32) = c;
-  *reinterpret_cast<uint32_t*>(keys + 4ULL * j) = j;
-  val_off[j] = 40ULL * j;
-  key_off[j] = 4ULL * j;
+    out[t] = c ? static_cast<float>(__ddiv_rn(sums[j * 8 + t], static_cast<double>(c))) : cent[j * 8 + t];
+  *reinterpret_cast<unsigned long long*>(vals + 40ULL * o + 32) = c;
+  *reinterpret_cast<uint32_t*>(keys + 4ULL * o) = j;
+  val_off[o] = 40ULL * o;
+  key_off[o] = 4ULL * o;
 }
 
 // ---------------------------------------------------------------- output assembly
@@ -328,17 +376,24 @@ cudaError_t launch_key_copy(const uint64_t* seg_start, uint64_t nseg, const uint
   return cudaGetLastError();
 }
 cudaError_t launch_reduce_wc(const uint64_t* seg_start, uint64_t nseg, const uint32_t* perm, const uint8_t* v,
-                             uint64_t* counts, uint64_t* worklist, DevState* st, int num_sms, cudaStream_t s) {
+                             int vbytes, uint64_t* counts, uint64_t* worklist, DevState* st, int num_sms,
+                             cudaStream_t s) {
   if (nseg == 0) return cudaSuccess;
   cudaError_t e = cudaMemsetAsync(&st->large_items, 0, 2 * sizeof(unsigned long long), s);
   if (e != cudaSuccess) return e;
   const unsigned g1 = static_cast<unsigned>(std::min<uint64_t>(blocks_for(nseg * 32, 256), 148ULL * 64));
-  k_reduce_wc_small<<<g1, 256, 0, s>>>(seg_start, nseg, perm, reinterpret_cast<const uint32_t*>(v), counts, worklist,
-                                       st);
-  count_launch();
-  k_reduce_wc_large<<<num_sms * 4, 256, 0, s>>>(seg_start, perm, reinterpret_cast<const uint32_t*>(v), counts,
-                                                worklist, st);
-  count_launch();
+  if (vbytes == 4) {
+    k_reduce_wc_small<uint32_t><<<g1, 256, 0, s>>>(seg_start, nseg, perm, reinterpret_cast<const uint32_t*>(v),
+                                                   counts, worklist, st);
+    k_reduce_wc_large<uint32_t><<<num_sms * 4, 256, 0, s>>>(seg_start, perm, reinterpret_cast<const uint32_t*>(v),
+                                                            counts, worklist, st);
+  } else {
+    k_reduce_wc_small<uint64_t><<<g1, 256, 0, s>>>(seg_start, nseg, perm, reinterpret_cast<const uint64_t*>(v),
+                                                   counts, worklist, st);
+    k_reduce_wc_large<uint64_t><<<num_sms * 4, 256, 0, s>>>(seg_start, perm, reinterpret_cast<const uint64_t*>(v),
+                                                            counts, worklist, st);
+  }
+  count_launch(2);
   return cudaGetLastError();
 }
 cudaError_t launch_reduce_km(const uint64_t* seg_start, uint64_t nseg, const uint64_t* skeys, const uint32_t* perm,
@@ -356,8 +411,11 @@ cudaError_t launch_reduce_km(const uint64_t* seg_start, uint64_t nseg, const uin
   return cudaGetLastError();
 }
 cudaError_t launch_km_finalize(const double* sums, const unsigned long long* cnts, const float* centroids, uint32_t k,
-                               uint8_t* vals, uint64_t* val_off, uint8_t* keys, uint64_t* key_off, cudaStream_t s) {
-  k_km_finalize<<<blocks_for(k + 1, 128), 128, 0, s>>>(sums, cnts, centroids, k, vals, val_off, keys, key_off);
+                               const uint32_t* list, uint32_t nlist, uint8_t* vals, uint64_t* val_off, uint8_t* keys,
+                               uint64_t* key_off, cudaStream_t s) {
+  const uint32_t n = list ? nlist : k;
+  k_km_finalize<<<blocks_for(n + 1, 128), 128, 0, s>>>(sums, cnts, centroids, k, list, nlist, vals, val_off, keys,
+                                                       key_off);
   count_launch();
   return cudaGetLastError();
 }

@@ -51,7 +51,7 @@ struct SortSmem {
 };
 
 template <bool kFirst>
-__global__ void __launch_bounds__(kSortThreads) k_onesweep(const uint64_t* __restrict__ keys_in,
+__global__ void __launch_bounds__(kSortThreads, 3) k_onesweep(const uint64_t* __restrict__ keys_in,
                                                          const uint32_t* __restrict__ idx_in,
                                                          uint64_t* __restrict__ keys_out,
                                                          uint32_t* __restrict__ idx_out, uint64_t m,
@@ -68,14 +68,11 @@ __global__ void __launch_bounds__(kSortThreads) k_onesweep(const uint64_t* __res
   const uint64_t tbase = static_cast<uint64_t>(tile) * kSortTile;
   const uint64_t wbase = tbase + static_cast<uint64_t>(warp) * 32 * kSortIPT;
   uint64_t key[kSortIPT];
-  uint32_t idx[kSortIPT];
   uint32_t rank[kSortIPT];
 #pragma unroll
   for (int j = 0; j < kSortIPT; ++j) {
     const uint64_t e = wbase + j * 32 + lane;
-    const bool v = e < m;
-    key[j] = v ? keys_in[e] : ~0ULL;  // padding sorts last (digit 255, after every real key)
-    idx[j] = kFirst ? static_cast<uint32_t>(e) : (v ? idx_in[e] : 0u);
+    key[j] = e < m ? keys_in[e] : ~0ULL;  // padding sorts last (digit 255, after every real key)
   }
   // stable warp-level ranking (element order == (j, lane) order inside the warp)
 #pragma unroll
@@ -88,6 +85,7 @@ __global__ void __launch_bounds__(kSortThreads) k_onesweep(const uint64_t* __res
       before = S.wcnt[warp][d];
       S.wcnt[warp][d] = before + __popc(peers);
     }
+    __syncwarp();   // order this step's counter updates before the next step's reads
     before = __shfl_sync(0xffffffffu, before, leader);
     rank[j] = before + __popc(peers & lanemask_lt());
   }
@@ -116,30 +114,32 @@ __global__ void __launch_bounds__(kSortThreads) k_onesweep(const uint64_t* __res
     uint64_t* my = status + static_cast<uint64_t>(tile) * 256 + d;
     uint32_t excl = 0;
     if (tile == 0) {
-      st_volatile_u64(my, pack_status(epoch, kPrefix, tcount));
+      st_relaxed_gpu_u64(my, pack_status(epoch, kPrefix, tcount));
     } else {
-      st_volatile_u64(my, pack_status(epoch, kAgg, tcount));
+      st_relaxed_gpu_u64(my, pack_status(epoch, kAgg, tcount));
       long long p = static_cast<long long>(tile) - 1;
       while (p >= 0) {
-        const uint64_t s = ld_volatile_u64(status + static_cast<uint64_t>(p) * 256 + d);
+        const uint64_t s = ld_relaxed_gpu_u64(status + static_cast<uint64_t>(p) * 256 + d);
         const uint32_t ep = static_cast<uint32_t>(s >> 34), kind = static_cast<uint32_t>(s >> 32) & 3u;
         if (ep != epoch || kind == 0) continue;
         excl += static_cast<uint32_t>(s);
         if (kind == kPrefix) break;
         --p;
       }
-      st_volatile_u64(my, pack_status(epoch, kPrefix, excl + tcount));
+      st_relaxed_gpu_u64(my, pack_status(epoch, kPrefix, excl + tcount));
     }
     S.goff[d] = bases[d] + excl;
   }
   __syncthreads();
-  // scatter into SMEM in tile-sorted order
+  // scatter into SMEM in tile-sorted order (payload loaded here, after ranking, to keep the
+  // ranking phase's register footprint small)
 #pragma unroll
   for (int j = 0; j < kSortIPT; ++j) {
+    const uint64_t e = wbase + j * 32 + lane;
     const uint32_t d = static_cast<uint32_t>(key[j] >> shift) & 255u;
     const uint32_t lp = S.dstart[d] + S.wcnt[warp][d] + rank[j];
     S.keys[lp] = key[j];
-    S.idx[lp] = idx[j];
+    S.idx[lp] = kFirst ? static_cast<uint32_t>(e) : (e < m ? idx_in[e] : 0u);
   }
   __syncthreads();
   const uint32_t nvalid = static_cast<uint32_t>(min(static_cast<uint64_t>(kSortTile), m - tbase));

@@ -1,0 +1,42 @@
+"""Process-group plumbing for the multi-GPU exchange: byte-count exchange and
+variable-size all-to-all over torch.distributed (NCCL on B200, gloo in the CPU tests).  No
+MapReduce arithmetic here: libbmr's kernels produce and consume the buffers."""
+from __future__ import annotations
+
+import numpy as np
+
+
+def exchange_counts(counts: np.ndarray, group=None) -> np.ndarray:
+    """counts[r] = (entries, heap bytes) this rank sends to rank r -> recv[r] = what rank r sends
+    to this rank.  One all_to_all_single of nranks x 2 int64."""
+    import torch
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    assert counts.shape == (world, 2)
+    dev = _dev(group)
+    send = torch.from_numpy(np.ascontiguousarray(counts, np.int64)).to(dev)
+    recv = torch.empty_like(send)
+    dist.all_to_all_single(recv, send, group=group)
+    return recv.cpu().numpy()
+
+
+def alltoallv(send, send_bytes, recv_bytes, group=None):
+    """Variable all-to-all of a flat uint8 tensor: slice r (send_bytes[r] bytes, in rank order)
+    goes to rank r; returns the concatenation of what every rank sent here, in rank order."""
+    import torch
+    import torch.distributed as dist
+    send_bytes = [int(x) for x in send_bytes]
+    recv_bytes = [int(x) for x in recv_bytes]
+    out = torch.empty(sum(recv_bytes), dtype=torch.uint8, device=send.device)
+    if sum(send_bytes) == 0 and sum(recv_bytes) == 0:
+        return out
+    dist.all_to_all_single(out, send, output_split_sizes=recv_bytes, input_split_sizes=send_bytes, group=group)
+    return out
+
+
+def _dev(group):
+    import torch
+    import torch.distributed as dist
+    if dist.get_backend(group) == "nccl":
+        return torch.device("cuda", torch.cuda.current_device())
+    return torch.device("cpu")
