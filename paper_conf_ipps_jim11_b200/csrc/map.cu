@@ -43,7 +43,8 @@ constexpr int kOffCap = 1024;                  // record offsets staged per tile
 constexpr int kOffBytes = 8320;                // (kOffCap + 2) * 8 rounded up
 constexpr int kBitWords = kStageBytes / 32 + 4;
 constexpr int kBitBytes = 2176;                // >= kBitWords * 4, multiple of 128
-constexpr int kOutHalf = 40960;
+constexpr int kNOut = 4;         // output buffers in the flush ring (generation g uses buffer g % kNOut)
+constexpr int kOutHalf = 20480;  // bytes per output buffer
 constexpr int kKmPts = kT / 32;                // 512 points per KM tile
 
 static_assert(kLead + kT + kHalo + 32 <= kStageBytes, "stage too small");
@@ -64,27 +65,30 @@ struct StageHdr {
 struct OutCtl {
   unsigned int cur;              // [generation:8 | count:24]; half = generation & 1
   unsigned int final_seq;        // full generation number of the final flush
-  unsigned int committed[2];     // entries fully written into each half (current generation)
-  unsigned int fcount[2];        // sealed entry count of each half
-  unsigned long long fbase[2];   // global base reserved for the sealed half (one atomic per flush)
+  unsigned int committed[kNOut];     // entries fully written into each buffer (current generation)
+  unsigned int fcount[kNOut];        // sealed entry count of each buffer
+  unsigned long long fbase[kNOut];   // global base reserved for the sealed buffer (one atomic per flush)
+  unsigned long long nflush, npads;  // per-CTA statistics, added to DevState once at the end
   unsigned int nsealed, is_final;  // sealed generations so far (full count); final flush flag
-  uint64_t req[2];               // mbarrier: half sealed -> flush warp
-  uint64_t done[2];              // mbarrier: half flushed -> free
+  uint64_t req[kNOut];           // mbarrier: buffer sealed -> flush warp
+  uint64_t done[kNOut];          // mbarrier: buffer flushed -> free
 };
 
 struct Layout {
   static constexpr int ctl = 0;                                   // OutCtl
-  static constexpr int hdr = 128;                                 // kStages x 128 (<= 4 stages)
+  static constexpr int hdr = 256;                                 // kStages x 128 (<= 4 stages)
   static constexpr int full = hdr + kStages * 128;                // kStages x 8
   static constexpr int empty = full + kStages * 8;
   static constexpr int ready = empty + kStages * 8;               // kStages x 8 (text: bitmap built)
   static constexpr int bytes = 1024;                              // kStages x kStageBytes
   static constexpr int offs = bytes + kStages * kStageBytes;      // kStages x kOffBytes
   static constexpr int bits = offs + kStages * kOffBytes;         // kStages x kBitBytes
-  static constexpr int out = bits + kStages * kBitBytes;          // 2 x kOutHalf
-  static constexpr int cent = out + 2 * kOutHalf;                 // KM centroids
+  static constexpr int out = bits + kStages * kBitBytes;          // kNOut x kOutHalf
+  static constexpr int cent = out + kNOut * kOutHalf;             // KM centroids
 };
 static_assert(Layout::ready + kStages * 8 <= Layout::bytes, "header region overflow");
+static_assert(sizeof(OutCtl) <= Layout::hdr, "OutCtl overlaps the stage headers");
+static_assert(256 % kNOut == 0, "8-bit generation counter must wrap on a buffer boundary");
 
 template <int W>
 struct PairFmt {
@@ -325,42 +329,29 @@ __device__ __forceinline__ uint64_t sentinel_key(const Params& P) {
   return ~0ULL;
 }
 
+// Seal buffer h of the current generation: switch every warp to the next buffer at once (the
+// in-flight writers of h finish on their own), then hand h to the flush warp.  Only when all
+// kNOut buffers are busy does the sealing warp wait (for the oldest flush).
 template <int W>
-__device__ void seal(const Params& P, OutCtl* oc, uint8_t* outh, uint32_t gen8, uint32_t h, uint32_t cnt,
-                     bool last) {
-  using F = PairFmt<W>;
+__device__ void seal(const Params& P, OutCtl* oc, uint32_t gen8, uint32_t h, uint32_t cnt, bool last) {
   const uint32_t full_gen = oc->nsealed;                       // full generation number
-  if (!last && full_gen >= 1) mbar_wait(&oc->done[(full_gen - 1) & 1u], ((full_gen - 1) >> 1) & 1u);
   if (!last) {
-    oc->committed[h ^ 1u] = 0;
+    if (full_gen + 1 >= kNOut) {                               // next buffer last used by gen q
+      const uint32_t q = full_gen + 1 - kNOut;
+      mbar_wait(&oc->done[q % kNOut], (q / kNOut) & 1u);
+    }
+    oc->committed[(h + 1) % kNOut] = 0;
     oc->nsealed = full_gen + 1;
     __threadfence_block();
-    atomicExch(&oc->cur, ((gen8 + 1) & 0xFFu) << 24);          // other warps continue in the other half
+    atomicExch(&oc->cur, ((gen8 + 1) & 0xFFu) << 24);          // other warps continue in the next buffer
   } else {
     oc->final_seq = full_gen;
     oc->is_final = 1;
   }
-  uint32_t cnt4 = cnt;
-  if constexpr (W != kSM) {
-    cnt4 = (cnt + 3u) & ~3u;
-    uint8_t* half = outh + h * kOutHalf;
-    for (uint32_t i = cnt; i < cnt4; ++i) {                   // sentinel filler entries
-      reinterpret_cast<uint64_t*>(half)[i] = sentinel_key<W>(P);
-      if constexpr (F::kKref) reinterpret_cast<uint64_t*>(half)[F::kCap + i] = 0;
-    }
-  }
-  unsigned long long gb = 0;
-  if (cnt4) {
-    gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(cnt4));  // ONE global atomic
-    atomicAdd(&P.st->flushes, 1ULL);
-    if (cnt4 != cnt) atomicAdd(&P.st->pads, static_cast<unsigned long long>(cnt4 - cnt));
-  }
-  oc->fcount[h] = cnt4;
-  oc->fbase[h] = gb;
+  oc->fcount[h] = cnt;
   __threadfence_block();
   mbar_arrive(&oc->req[h]);
 }
-
 template <int W>
 __device__ __forceinline__ Slot reserve(const Params& P, OutCtl* oc, uint8_t* outh, uint32_t cnt, uint32_t cap) {
   const uint32_t lane = threadIdx.x & 31;
@@ -369,14 +360,12 @@ __device__ __forceinline__ Slot reserve(const Params& P, OutCtl* oc, uint8_t* ou
     if (lane == 0) old = atomicAdd(&oc->cur, cnt);
     old = __shfl_sync(kFull, old, 0);
     const uint32_t gen = old >> 24, base = old & kCntMask;
-    const uint32_t h = gen & 1u;
+    const uint32_t h = gen % kNOut;
     if (base + cnt <= cap) return {h, base};
     if (lane == 0) {
       if (base <= cap) {
         // This warp crossed the capacity first: it seals half h (L113 "overflow handling").
-        volatile unsigned int* cm = &oc->committed[h];
-        while (*cm != base) __nanosleep(32);
-        seal<W>(P, oc, outh, gen, h, base, false);
+        seal<W>(P, oc, gen, h, base, false);
       } else {
         volatile unsigned int* c = &oc->cur;
         while ((*c >> 24) == gen) __nanosleep(128);
@@ -410,13 +399,34 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   using F = PairFmt<W>;
   const uint32_t lane = threadIdx.x & 31;
   for (uint32_t f = 0;; ++f) {
-    const uint32_t h = f & 1u;
-    mbar_wait(&oc->req[h], (f >> 1) & 1u);
-    const uint32_t cnt = *reinterpret_cast<volatile unsigned int*>(&oc->fcount[h]);
-    const unsigned long long gb = *reinterpret_cast<volatile unsigned long long*>(&oc->fbase[h]);
+    const uint32_t h = f % kNOut;
+    mbar_wait(&oc->req[h], (f / kNOut) & 1u);
+    const uint32_t cnt0 = *reinterpret_cast<volatile unsigned int*>(&oc->fcount[h]);
     const bool fin = *reinterpret_cast<volatile unsigned int*>(&oc->is_final) &&
                      *reinterpret_cast<volatile unsigned int*>(&oc->final_seq) == f;
-    const uint8_t* half = smem + Layout::out + h * kOutHalf;
+    uint8_t* half = smem + Layout::out + h * kOutHalf;
+    // the sealed buffer's writers finish on their own: wait until all cnt0 entries are committed
+    if (lane == 0) {
+      volatile unsigned int* cm = &oc->committed[h];
+      while (*cm != cnt0) __nanosleep(32);
+    }
+    __syncwarp();
+    uint32_t cnt = cnt0;
+    if constexpr (W != kSM) {
+      cnt = (cnt0 + 3u) & ~3u;                                  // 4-pair aligned flush (TMA store)
+      if (lane < cnt - cnt0) {                                  // sentinel filler entries
+        reinterpret_cast<uint64_t*>(half)[cnt0 + lane] = sentinel_key<W>(P);
+        if constexpr (F::kKref) reinterpret_cast<uint64_t*>(half)[F::kCap + cnt0 + lane] = 0;
+      }
+    }
+    unsigned long long gb = 0;
+    if (lane == 0 && cnt) {
+      gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(cnt));  // ONE global atomic per flush
+      oc->nflush += 1;
+      oc->npads += cnt - cnt0;
+    }
+    gb = __shfl_sync(kFull, gb, 0);
+    __syncwarp();
     if (cnt && gb + cnt <= P.cap_pairs) {
       const uint64_t* sh = reinterpret_cast<const uint64_t*>(half);
       const uint8_t* sv = half + F::kCap * (F::kKref ? 16 : 8);
@@ -435,7 +445,11 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
     if (lane == 0) mbar_arrive(&oc->done[h]);
     if (fin) break;
   }
-  if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // global writes complete
+  if (lane == 0) {
+    asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // global writes complete
+    atomicAdd(&P.st->flushes, oc->nflush);
+    if (oc->npads) atomicAdd(&P.st->pads, oc->npads);
+  }
 }
 
 // ---------------------------------------------------------------- producer warp
@@ -593,14 +607,25 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
   uint32_t emit_mask = 0;       // bit j: an emission anchored at p0 + j
   uint32_t aux[2] = {0, 0};     // II: closing-quote distance for up to two markers
   uint32_t wm = 0, nb = 0;
+  const uint32_t lane = threadIdx.x & 31;
   if constexpr (W == kWC) {
+    // word bytes of this chunk; the next chunk's mask comes from lane + 1 (same window), so each
+    // lane classifies only its own 16 bytes.  Lane 31 knows nothing beyond its chunk: its words
+    // that do not end inside the chunk take the slow path.
+    uint32_t w16 = 0;
     if (live) {
 #pragma unroll
-      for (int i = 0; i < 8; ++i) wm |= word_mask4(x[i]) << (4 * i);
-      wm &= vm;
-      uint32_t prevw = 0;
-      if (p0 - 1 >= 0 && p0 - 1 < N) prevw = is_word_byte(tv.sb[i0 - 1]) ? 1u : 0u;
-      nb = ~wm | R;                                            // a word cannot continue here
+      for (int i = 0; i < 4; ++i) w16 |= word_mask4(x[i]) << (4 * i);
+    }
+    const uint32_t nxt = __shfl_down_sync(kFull, w16, 1);
+    const uint32_t prv = __shfl_up_sync(kFull, w16, 1);
+    if (live) {
+      const uint32_t known = lane < 31 ? 0xFFFFFFFFu : 0xFFFFu;
+      wm = (w16 | (lane < 31 ? nxt << 16 : 0u)) & vm;
+      uint32_t prevw;
+      if (lane == 0) prevw = (p0 - 1 >= 0 && p0 - 1 < N && is_word_byte(tv.sb[i0 - 1])) ? 1u : 0u;
+      else prevw = (prv >> 15) & 1u;
+      nb = (~wm | R) & known;                                  // a word cannot continue here
       emit_mask = wm & 0xFFFFu & ~(((wm << 1) | prevw) & ~R);  // word starts (C-2 WC)
     }
   } else if constexpr (W == kSM) {
@@ -667,7 +692,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
       const long long p = p0 + j;
       if constexpr (W == kWC) {
         const uint32_t rest = nb >> (j + 1);
-        uint32_t len = rest ? static_cast<uint32_t>(__ffs(rest)) : slow_word_len(P, tv, p, p0 + 32);
+        uint32_t len = rest ? static_cast<uint32_t>(__ffs(rest)) : slow_word_len(P, tv, p, p0 + (lane < 31 ? 32 : 16));
         const uint64_t key = (len <= 7) ? inline_key(window8(x, j), len) : key_at(P, tv, p, len);
         if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
         sh[idx] = key;
@@ -787,7 +812,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   named_bar_sync(2, kNMap * 32);
   if (threadIdx.x == 0) {
     const uint32_t cur = *reinterpret_cast<volatile unsigned int*>(&oc->cur);
-    seal<W>(P, oc, outh, cur >> 24, (cur >> 24) & 1u, cur & kCntMask, true);
+    seal<W>(P, oc, cur >> 24, (cur >> 24) % kNOut, cur & kCntMask, true);
   }
 }
 
@@ -798,13 +823,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_map(Params P) {
   if (threadIdx.x == 0) {
     oc->cur = 0;
     oc->final_seq = 0;
-    oc->fbase[0] = oc->fbase[1] = 0;
-    oc->committed[0] = oc->committed[1] = 0;
-    oc->fcount[0] = oc->fcount[1] = 0;
+    for (int b = 0; b < kNOut; ++b) { oc->fbase[b] = 0; oc->committed[b] = 0; oc->fcount[b] = 0; }
+    oc->nflush = 0;
+    oc->npads = 0;
     oc->nsealed = 0;
     oc->is_final = 0;
-    mbar_init(&oc->req[0], 1); mbar_init(&oc->req[1], 1);
-    mbar_init(&oc->done[0], kNFlush); mbar_init(&oc->done[1], kNFlush);
+    for (int b = 0; b < kNOut; ++b) { mbar_init(&oc->req[b], 1); mbar_init(&oc->done[b], kNFlush); }
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout::full);
     uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout::empty);
     uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout::ready);

@@ -44,25 +44,29 @@ struct SortSmem {
   uint64_t keys[kSortTile];
   uint32_t idx[kSortTile];
   uint32_t wcnt[kWarps][256];
+  uint32_t hist[256];
   uint32_t dstart[256];
   uint32_t goff[256];
   uint32_t wsum[kWarps];
   uint32_t tile;
 };
 
+constexpr int kLookWindow = 4;   // predecessor status words fetched per look-back step
+
 template <bool kFirst>
 __global__ void __launch_bounds__(kSortThreads, 3) k_onesweep(const uint64_t* __restrict__ keys_in,
-                                                         const uint32_t* __restrict__ idx_in,
-                                                         uint64_t* __restrict__ keys_out,
-                                                         uint32_t* __restrict__ idx_out, uint64_t m,
-                                                         uint32_t shift, const uint32_t* __restrict__ bases,
-                                                         uint64_t* status, uint32_t epoch,
-                                                         unsigned int* tile_counter) {
+                                                            const uint32_t* __restrict__ idx_in,
+                                                            uint64_t* __restrict__ keys_out,
+                                                            uint32_t* __restrict__ idx_out, uint64_t m,
+                                                            uint32_t shift, const uint32_t* __restrict__ bases,
+                                                            uint64_t* status, uint32_t epoch,
+                                                            unsigned int* tile_counter) {
   extern __shared__ __align__(16) uint8_t raw[];
   SortSmem& S = *reinterpret_cast<SortSmem*>(raw);
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid == 0) S.tile = atomicAdd(tile_counter, 1u);
   for (uint32_t i = tid; i < kWarps * 256; i += kSortThreads) (&S.wcnt[0][0])[i] = 0;
+  S.hist[tid] = 0;
   __syncthreads();
   const uint32_t tile = S.tile;
   const uint64_t tbase = static_cast<uint64_t>(tile) * kSortTile;
@@ -74,26 +78,32 @@ __global__ void __launch_bounds__(kSortThreads, 3) k_onesweep(const uint64_t* __
     const uint64_t e = wbase + j * 32 + lane;
     key[j] = e < m ? keys_in[e] : ~0ULL;  // padding sorts last (digit 255, after every real key)
   }
-  // stable warp-level ranking (element order == (j, lane) order inside the warp)
+  // 1. tile histogram first, published immediately (early aggregate for the successors)
+#pragma unroll
+  for (int j = 0; j < kSortIPT; ++j) atomicAdd(&S.hist[static_cast<uint32_t>(key[j] >> shift) & 255u], 1u);
+  __syncthreads();
+  const uint32_t d = tid;  // kSortThreads == 256: one digit per thread
+  const uint32_t tcount = S.hist[d];
+  uint64_t* my = status + static_cast<uint64_t>(tile) * 256 + d;
+  st_relaxed_gpu_u64(my, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount));
+  // 2. stable warp-level ranking (element order == (j, lane) order inside the warp)
 #pragma unroll
   for (int j = 0; j < kSortIPT; ++j) {
-    const uint32_t d = static_cast<uint32_t>(key[j] >> shift) & 255u;
-    const uint32_t peers = __match_any_sync(0xffffffffu, d);
+    const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & 255u;
+    const uint32_t peers = __match_any_sync(0xffffffffu, dj);
     const uint32_t leader = __ffs(peers) - 1;
     uint32_t before = 0;
     if (lane == leader) {
-      before = S.wcnt[warp][d];
-      S.wcnt[warp][d] = before + __popc(peers);
+      before = S.wcnt[warp][dj];
+      S.wcnt[warp][dj] = before + __popc(peers);
     }
     __syncwarp();   // order this step's counter updates before the next step's reads
     before = __shfl_sync(0xffffffffu, before, leader);
     rank[j] = before + __popc(peers & lanemask_lt());
   }
   __syncthreads();
-  // per digit: warp-exclusive offsets, tile count, tile-local digit start, global offset
-  uint32_t tcount = 0;
+  // 3. per digit: warp-exclusive offsets and the tile-local digit start
   {
-    const uint32_t d = tid;  // kSortThreads == 256
     uint32_t run = 0;
 #pragma unroll
     for (int w = 0; w < kWarps; ++w) {
@@ -101,52 +111,59 @@ __global__ void __launch_bounds__(kSortThreads, 3) k_onesweep(const uint64_t* __
       S.wcnt[w][d] = run;
       run += c;
     }
-    tcount = run;
-    // block exclusive scan of tcount over digits
     const uint32_t inc = warp_inclusive_add(tcount);
     if (lane == 31) S.wsum[warp] = inc;
-    __syncthreads();
+  }
+  __syncthreads();
+  {
     uint32_t wpre = 0;
 #pragma unroll
     for (int w = 0; w < kWarps; ++w) wpre += (w < static_cast<int>(warp)) ? S.wsum[w] : 0u;
-    S.dstart[d] = wpre + inc - tcount;
-    // decoupled look-back for digit d
-    uint64_t* my = status + static_cast<uint64_t>(tile) * 256 + d;
+    S.dstart[d] = wpre + warp_inclusive_add(tcount) - tcount;
+    // 4. decoupled look-back, kLookWindow predecessors per round trip
     uint32_t excl = 0;
-    if (tile == 0) {
-      st_relaxed_gpu_u64(my, pack_status(epoch, kPrefix, tcount));
-    } else {
-      st_relaxed_gpu_u64(my, pack_status(epoch, kAgg, tcount));
+    if (tile > 0) {
       long long p = static_cast<long long>(tile) - 1;
-      while (p >= 0) {
-        const uint64_t s = ld_relaxed_gpu_u64(status + static_cast<uint64_t>(p) * 256 + d);
-        const uint32_t ep = static_cast<uint32_t>(s >> 34), kind = static_cast<uint32_t>(s >> 32) & 3u;
-        if (ep != epoch || kind == 0) continue;
-        excl += static_cast<uint32_t>(s);
-        if (kind == kPrefix) break;
-        --p;
+      for (;;) {
+        uint64_t sv[kLookWindow];
+#pragma unroll
+        for (int i = 0; i < kLookWindow; ++i)
+          sv[i] = (p - i >= 0) ? ld_relaxed_gpu_u64(status + static_cast<uint64_t>(p - i) * 256 + d) : 0;
+        int adv = 0;
+        bool done = false;
+#pragma unroll
+        for (int i = 0; i < kLookWindow; ++i) {
+          if (done || adv != i) continue;             // stop at the first not-ready / prefix word
+          const uint32_t ep = static_cast<uint32_t>(sv[i] >> 34), kind = static_cast<uint32_t>(sv[i] >> 32) & 3u;
+          if (ep != epoch || kind == 0) continue;     // not ready yet: retry from here
+          excl += static_cast<uint32_t>(sv[i]);
+          ++adv;
+          if (kind == kPrefix) done = true;
+        }
+        if (done) break;
+        p -= adv;
       }
       st_relaxed_gpu_u64(my, pack_status(epoch, kPrefix, excl + tcount));
     }
     S.goff[d] = bases[d] + excl;
   }
   __syncthreads();
-  // scatter into SMEM in tile-sorted order (payload loaded here, after ranking, to keep the
-  // ranking phase's register footprint small)
+  // 5. scatter into SMEM in tile-sorted order (payload loaded here, after ranking)
 #pragma unroll
   for (int j = 0; j < kSortIPT; ++j) {
     const uint64_t e = wbase + j * 32 + lane;
-    const uint32_t d = static_cast<uint32_t>(key[j] >> shift) & 255u;
-    const uint32_t lp = S.dstart[d] + S.wcnt[warp][d] + rank[j];
+    const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & 255u;
+    const uint32_t lp = S.dstart[dj] + S.wcnt[warp][dj] + rank[j];
     S.keys[lp] = key[j];
     S.idx[lp] = kFirst ? static_cast<uint32_t>(e) : (e < m ? idx_in[e] : 0u);
   }
   __syncthreads();
+  // 6. contiguous per-digit runs to global memory
   const uint32_t nvalid = static_cast<uint32_t>(min(static_cast<uint64_t>(kSortTile), m - tbase));
   for (uint32_t i = tid; i < nvalid; i += kSortThreads) {
     const uint64_t k = S.keys[i];
-    const uint32_t d = static_cast<uint32_t>(k >> shift) & 255u;
-    const uint32_t pos = S.goff[d] + (i - S.dstart[d]);
+    const uint32_t dk = static_cast<uint32_t>(k >> shift) & 255u;
+    const uint32_t pos = S.goff[dk] + (i - S.dstart[dk]);
     keys_out[pos] = k;
     idx_out[pos] = S.idx[i];
   }
