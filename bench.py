@@ -260,8 +260,12 @@ def main():
         barrier()
         t0 = time.perf_counter()
         ev0.record(stream)
+        evs = []
         for _ in range(args.steps):
             step()
+            e = torch.cuda.Event(enable_timing=True)
+            e.record(stream)
+            evs.append(e)
             s = job.stats()  # map/hist/sort/seg events are collected at mr_group's synchronisation
             for k in tot:
                 tot[k] += s[k]
@@ -272,6 +276,7 @@ def main():
         wall = time.perf_counter() - t0
         barrier()
     ms = ev0.elapsed_time(ev1) / args.steps
+    step_ms = [ev0.elapsed_time(evs[0])] + [evs[i - 1].elapsed_time(evs[i]) for i in range(1, len(evs))]
     t = torch.tensor([ms], device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -380,6 +385,8 @@ def main():
                           "combiner": inp["wl"] in ("wc", "km")} if exchange else None),
             "gpu_launches": int(tot["kernel_launches"]),
             "clocks": clk.summary(), "wall_s_timed": round(wall, 3),
+            "step_ms": {"min": round(min(step_ms), 3), "median": round(statistics.median(step_ms), 3),
+                        "max": round(max(step_ms), 3)},
         }
         print(json.dumps(line), flush=True)
     job.close()

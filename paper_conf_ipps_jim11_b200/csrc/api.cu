@@ -28,10 +28,12 @@ template <typename T>
 struct DBuf {
   T* p = nullptr;
   uint64_t n = 0;
+  // grow-only with 1/16 headroom: sizes that drift by a few elements between runs (e.g. the
+  // number of flush filler pairs) must not trigger a multi-GB cudaFree/cudaMalloc per step
   cudaError_t ensure(uint64_t need) {
     if (need <= n && p) return cudaSuccess;
     release();
-    const uint64_t cnt = std::max<uint64_t>(need, 1);
+    const uint64_t cnt = std::max<uint64_t>(need + need / 16, 1);
     cudaError_t e = cudaMalloc(reinterpret_cast<void**>(&p), cnt * sizeof(T));
     if (e != cudaSuccess) { p = nullptr; n = 0; cudaGetLastError(); return e; }
     n = cnt;
@@ -212,7 +214,7 @@ struct mr_job {
   uint64_t m = 0, nseg = 0, key_bytes = 0;
   DBuf<uint32_t> seg_counts;
   DBuf<uint64_t> tile_base, seg_start, key_off, val_off, counts, worklist, gathered;
-  DBuf<uint8_t> keys_out, vals_out;
+  DBuf<uint8_t> keys_out, vals_out, vsorted;
   DBuf<double> sums;
   DBuf<unsigned long long> cnts;
   // fetched result
@@ -837,7 +839,7 @@ mr_status mr_job_destroy(mr_job* job) {
   job->sw.release();
   job->seg_counts.release(); job->tile_base.release(); job->seg_start.release(); job->key_off.release();
   job->val_off.release(); job->counts.release(); job->worklist.release(); job->gathered.release();
-  job->keys_out.release(); job->vals_out.release(); job->sums.release(); job->cnts.release();
+  job->keys_out.release(); job->vals_out.release(); job->vsorted.release(); job->sums.release(); job->cnts.release();
   job->keys_h.release(); job->vals_h.release(); job->key_off_h.release(); job->val_off_h.release();
   job->st_h.release(); job->tmp_h.release();
   if (job->st) cudaFree(job->st);

@@ -104,22 +104,40 @@ __host__ __device__ __forceinline__ uint64_t mix64(uint64_t z) {  // murmur3 fin
 }
 constexpr uint64_t kHashedBit = 1ULL << 63;
 
-// Hash of len >= 8 key bytes read through a generic pointer (shared or global).
+// 64-bit key hash over 4-byte little-endian words (last word zero-padded): two 32-bit lanes
+// (murmur3-style rounds) so that the map warps stay on 32-bit IMAD/LOP3; hash_bytes (generic
+// pointer) and the map kernel's SMEM variant feed identical words and agree bit for bit.
+struct KeyHash {
+  uint32_t h1, h2;
+  __device__ __forceinline__ KeyHash(uint64_t seed, uint32_t len)
+      : h1(static_cast<uint32_t>(seed) ^ (len * 0x9E3779B1u)), h2(static_cast<uint32_t>(seed >> 32) + len * 0x85EBCA77u) {}
+  __device__ __forceinline__ void add(uint32_t w) {
+    h1 = __funnelshift_l(h1 ^ (w * 0xCC9E2D51u), h1 ^ (w * 0xCC9E2D51u), 15) * 0x1B873593u;
+    h2 = (h2 + w) * 0x27D4EB2Fu;
+    h2 ^= h2 >> 15;
+  }
+  __device__ __forceinline__ static uint32_t fmix(uint32_t h) {
+    h ^= h >> 16; h *= 0x85EBCA6Bu; h ^= h >> 13; h *= 0xC2B2AE35u; h ^= h >> 16;
+    return h;
+  }
+  __device__ __forceinline__ uint64_t finish() const {
+    return (static_cast<uint64_t>(fmix(h1 + h2)) << 32) | fmix(h2 ^ __funnelshift_l(h1, h1, 7));
+  }
+};
+
+// Hash of key bytes read through a generic pointer (shared or global).
 __device__ __forceinline__ uint64_t hash_bytes(const uint8_t* p, uint32_t len, uint64_t seed) {
-  uint64_t h = seed ^ (static_cast<uint64_t>(len) * 0x9E3779B97F4A7C15ULL);
+  KeyHash hs(seed, len);
   uint32_t i = 0;
-  for (; i + 8 <= len; i += 8) {
-    uint64_t b = 0;
-#pragma unroll
-    for (int k = 0; k < 8; ++k) b |= static_cast<uint64_t>(p[i + k]) << (8 * k);
-    h = mix64(h ^ b) + 0x632BE59BD9B4E019ULL;
-  }
+  for (; i + 4 <= len; i += 4)
+    hs.add(static_cast<uint32_t>(p[i]) | (static_cast<uint32_t>(p[i + 1]) << 8) |
+           (static_cast<uint32_t>(p[i + 2]) << 16) | (static_cast<uint32_t>(p[i + 3]) << 24));
   if (i < len) {
-    uint64_t b = 0;
-    for (int k = 0; i + k < len; ++k) b |= static_cast<uint64_t>(p[i + k]) << (8 * k);
-    h = mix64(h ^ b ^ 0xA5A5A5A5ULL);
+    uint32_t w = 0;
+    for (uint32_t k = 0; i + k < len; ++k) w |= static_cast<uint32_t>(p[i + k]) << (8 * k);
+    hs.add(w);
   }
-  return mix64(h);
+  return hs.finish();
 }
 // Final sort key of a hashed key; weak_hash (MR_FLAG_WEAK_HASH_DEBUG) keeps only 4 bits so
 // that almost every segment collides (tests the verification + re-sort slow path).

@@ -4,21 +4,25 @@
 // collects results in a shared-memory output area and flushes it to global memory with one
 // global atomic per flush.  Its GT200 mechanics (16 KB SMEM, all threads alternating between
 // stage-in / compute / stage-out, software wait-signal flags, yield by dummy global reads) are
-// prior art; the B200 re-derivation here:
+// prior art; the B200 re-derivation here (one 576-thread CTA per SM):
 //   * producer warp (A1/A2): one elected lane issues TMA bulk copies (cp.async.bulk) of the
-//     tile bytes and of the tile's record-offset slice into a 3-stage SMEM ring guarded by
-//     mbarrier full/empty pairs (replaces the barrier-separated staging loop, L68/L85);
+//     tile bytes and of the tile's record-offset slice into an SMEM ring (4 stages, 7 for SM)
+//     guarded by mbarrier full/empty pairs; kLag tiles later the producer turns the staged
+//     offsets into a record-start bitmap and releases the stage (ready mbarrier) — replaces the
+//     barrier-separated staging loop (L68, L85);
 //   * 16 map warps (A3): byte-parallel, record-agnostic scanning — each lane owns a 16-byte
-//     chunk, record boundaries come from a per-stage bitmap built from the staged offsets; the
+//     chunk, record boundaries come from the bitmap; no map-warp barrier at all, so the
 //     per-record imbalance the paper blames for SO overhead (L273) disappears;
-//   * emit allocator (A11/A12, D3/D4): a warp result is reserved with ONE shared 64-bit
-//     atomicAdd on a packed [generation | count] cursor of the active output half;
-//   * overflow (A13, L113): the unique warp whose reservation crosses the half's capacity seals
-//     the half, switches generation (double-buffered halves) and hands the half to the flush
-//     warp through an mbarrier (replaces the wait/signal flag protocol, L96-100);
-//   * flush warp (A4): one global atomicAdd per flush reserves [base, base+k) of the
-//     intermediate SoA arrays, then coalesced stores.  The global cursor counts demand even
-//     past capacity (D7), so the host can grow the buffers and replay the batch.
+//   * emit allocator (A11/A12, D3/D4): a warp result is reserved with ONE shared 32-bit
+//     atomicAdd on a packed [generation:8 | count:24] cursor of the current output buffer;
+//   * overflow (A13, L113): the unique warp whose reservation crosses the buffer's capacity
+//     seals it and switches every warp to the next buffer of a 4-buffer ring at once (replaces
+//     the wait/signal flag protocol, L96-100); it waits only if all buffers are still flushing;
+//   * flush warp (A4): waits for the sealed buffer's in-flight writers, takes ONE global
+//     atomicAdd for the whole buffer, and writes its SoA arrays with TMA bulk stores
+//     (cp.async.bulk.global.shared::cta).  Flushes are rounded to 4 pairs (16-B alignment) with
+//     sentinel filler pairs.  The global cursor counts demand even past capacity (D7), so the
+//     host can grow the buffers and replay the batch.
 #include <cstdio>
 
 #include "common.cuh"
@@ -31,8 +35,6 @@ constexpr int kProdWarp = kNMap;
 constexpr int kFlushWarp0 = kNMap + 1;   // flush warps kFlushWarp0 .. kFlushWarp0 + kNFlush - 1
 constexpr int kNFlush = 1;
 constexpr int kThreads = (kNMap + 1 + kNFlush) * 32;
-constexpr int kStages = 4;
-constexpr int kLag = 2;           // producer builds the bitmap of tile it - kLag after issuing tile it
 constexpr int kT = 16384;        // owned bytes per tile (text) / bytes per tile (KM)
 constexpr int kLead = 16;        // bytes staged before the tile (previous-byte context)
 constexpr int kHalo = 256;       // bytes staged after the tile (words / matches / URLs crossing it)
@@ -44,7 +46,21 @@ constexpr int kOffBytes = 8320;                // (kOffCap + 2) * 8 rounded up
 constexpr int kBitWords = kStageBytes / 32 + 4;
 constexpr int kBitBytes = 2176;                // >= kBitWords * 4, multiple of 128
 constexpr int kNOut = 4;         // output buffers in the flush ring (generation g uses buffer g % kNOut)
-constexpr int kOutHalf = 20480;  // bytes per output buffer
+// Per-workload SMEM budget: StringMatch is read-bound with almost no output -> more input stages
+// (more bytes in flight per SM) and small output buffers; the emitting workloads keep 4 stages
+// and 4 x 20 KB output buffers.
+template <int W>
+struct Cfg {
+  static constexpr int kStages = (W == kSM) ? 7 : 4;
+  static constexpr int kOutHalf = (W == kSM) ? 4096 : 20480;   // bytes per output buffer
+  // the producer builds the bitmap of tile it - kLag right after issuing tile it: kLag stages of
+  // TMA traffic stay in flight per SM while one stage is being consumed
+  static constexpr int kLag = kStages - 2;
+  // WC: per-warp queue of the window's long (hashed) words, hashed by all 32 lanes together
+  // after the emission rounds (a lane-per-word hash inside the rounds diverges: with 7% long
+  // words, 9 in 10 rounds would carry at least one).  <= 64 words of >= 8 bytes fit in 512 B.
+  static constexpr int kHashQ = (W == kWC) ? 64 : 0;
+};
 constexpr int kKmPts = kT / 32;                // 512 points per KM tile
 
 static_assert(kLead + kT + kHalo + 32 <= kStageBytes, "stage too small");
@@ -74,20 +90,23 @@ struct OutCtl {
   uint64_t done[kNOut];          // mbarrier: buffer flushed -> free
 };
 
+template <int W>
 struct Layout {
+  static constexpr int kStages = Cfg<W>::kStages;
   static constexpr int ctl = 0;                                   // OutCtl
-  static constexpr int hdr = 256;                                 // kStages x 128 (<= 4 stages)
+  static constexpr int hdr = 256;                                 // kStages x 128
   static constexpr int full = hdr + kStages * 128;                // kStages x 8
   static constexpr int empty = full + kStages * 8;
   static constexpr int ready = empty + kStages * 8;               // kStages x 8 (text: bitmap built)
-  static constexpr int bytes = 1024;                              // kStages x kStageBytes
+  static constexpr int bytes = 2048;                              // kStages x kStageBytes
   static constexpr int offs = bytes + kStages * kStageBytes;      // kStages x kOffBytes
   static constexpr int bits = offs + kStages * kOffBytes;         // kStages x kBitBytes
-  static constexpr int out = bits + kStages * kBitBytes;          // kNOut x kOutHalf
-  static constexpr int cent = out + kNOut * kOutHalf;             // KM centroids
+  static constexpr int out = bits + kStages * kBitBytes;          // kNOut x Cfg<W>::kOutHalf
+  static constexpr int hq = out + kNOut * Cfg<W>::kOutHalf;       // kNMap x kHashQ x 8 (WC)
+  static constexpr int cent = hq + kNMap * Cfg<W>::kHashQ * 8;    // KM centroids
+  static_assert(ready + kStages * 8 <= bytes, "header region overflow");
+  static_assert(sizeof(OutCtl) <= hdr, "OutCtl overlaps the stage headers");
 };
-static_assert(Layout::ready + kStages * 8 <= Layout::bytes, "header region overflow");
-static_assert(sizeof(OutCtl) <= Layout::hdr, "OutCtl overlaps the stage headers");
 static_assert(256 % kNOut == 0, "8-bit generation counter must wrap on a buffer boundary");
 
 template <int W>
@@ -95,7 +114,7 @@ struct PairFmt {
   static constexpr bool kKref = (W == kWC || W == kII);
   static constexpr int kV = (W == kWC) ? 4 : (W == kSM) ? 0 : (W == kKM) ? 32 : 8;
   static constexpr int kPairBytes = 8 + (kKref ? 8 : 0) + kV;
-  static constexpr uint32_t kCap = (kOutHalf / kPairBytes) & ~3u;
+  static constexpr uint32_t kCap = (Cfg<W>::kOutHalf / kPairBytes) & ~3u;
   // largest single warp reservation: WC 8 words / 16 B, SM 16 matches / 16 B, II 2, KM 1 per lane
   static constexpr uint32_t kMaxReserve = (W == kWC) ? 256 : (W == kSM) ? 512 : 32 * ((W == kII) ? 2 : 1);
   static_assert(kCap >= kMaxReserve, "output half smaller than one warp result");
@@ -119,6 +138,7 @@ struct Params {
   uint32_t flags;
   DevState* st;
   const uint64_t* tb;      // tile bounds
+  const uint8_t* off_end;  // end of the offsets array rounded DOWN to 16 B (aligned TMA limit)
   uint64_t hash_seed;
 };
 
@@ -170,13 +190,11 @@ __device__ __forceinline__ uint32_t bits32(const uint32_t* bm, long long i0) {  
 }
 // select 3 consecutive words x[wi..wi+2] of an 8-word window (wi in 0..3, no local memory)
 __device__ __forceinline__ uint64_t window8(const uint32_t (&x)[8], uint32_t j) {
-  uint32_t wi = j >> 2, sh = (j & 3) * 8, a, b, c;
-  switch (wi) {
-    case 0: a = x[0]; b = x[1]; c = x[2]; break;
-    case 1: a = x[1]; b = x[2]; c = x[3]; break;
-    case 2: a = x[2]; b = x[3]; c = x[4]; break;
-    default: a = x[3]; b = x[4]; c = x[5]; break;
-  }
+  // branch-free selection (selects, not a divergent switch): words j/4 .. j/4 + 2
+  const uint32_t sh = (j & 3) * 8;
+  const bool b2 = (j & 8) != 0, b1 = (j & 4) != 0;
+  const uint32_t w0 = b2 ? x[2] : x[0], w1 = b2 ? x[3] : x[1], w2 = b2 ? x[4] : x[2], w3 = b2 ? x[5] : x[3];
+  const uint32_t a = b1 ? w1 : w0, b = b1 ? w2 : w1, c = b1 ? w3 : w2;
   return (static_cast<uint64_t>(__funnelshift_r(b, c, sh)) << 32) | __funnelshift_r(a, b, sh);
 }
 // 16 bytes starting at j (0..15) of the 8-word window, as 4 words
@@ -215,22 +233,29 @@ struct TileView {
 // Word length for a word at position p whose end lies beyond the 32-byte window [p0, p0+32).
 __device__ uint32_t slow_word_len(const Params& P, const TileView& tv, long long p, long long from) {
   long long q = from;
-  uint64_t rec_end = ~0ULL;
-  bool have_end = false;
   const long long N = static_cast<long long>(P.nbytes);
-  for (;; ++q) {
-    if (q >= N) break;
-    uint32_t c;
-    if (q < tv.stg_hi) {
-      if (tv.is_start(q)) break;
-      c = tv.sb[q - tv.sbase];
-    } else {
-      if (!have_end) { rec_end = next_start_after(P.off, P.n, static_cast<uint64_t>(p)); have_end = true; }
-      if (static_cast<uint64_t>(q) >= rec_end) break;
-      c = P.rec[q];
-    }
-    if (!is_word_byte(c)) break;
+  const long long lim = min(tv.stg_hi, N);
+  // inside the stage: 4 bytes per step (SWAR word classes + bitmap record starts)
+  while (q < lim && ((q - tv.sbase) & 3)) {
+    if (tv.is_start(q) || !is_word_byte(tv.sb[q - tv.sbase])) return static_cast<uint32_t>(q - p);
+    ++q;
   }
+  while (q + 4 <= lim) {
+    const long long i = q - tv.sbase;
+    const uint32_t w = *reinterpret_cast<const uint32_t*>(tv.sb + i);
+    const uint32_t m = ((~word_mask4(w)) & 0xFu) | ((tv.bm[i >> 5] >> (i & 31)) & 0xFu);
+    if (m) return static_cast<uint32_t>(q + (__ffs(m) - 1) - p);
+    q += 4;
+  }
+  while (q < lim) {
+    if (tv.is_start(q) || !is_word_byte(tv.sb[q - tv.sbase])) return static_cast<uint32_t>(q - p);
+    ++q;
+  }
+  if (q >= N) return static_cast<uint32_t>(q - p);
+  // beyond the staged halo (words longer than ~256 bytes): global memory, record end by search
+  const uint64_t rec_end = next_start_after(P.off, P.n, static_cast<uint64_t>(p));
+  for (; q < N && static_cast<uint64_t>(q) < rec_end; ++q)
+    if (!is_word_byte(P.rec[q])) break;
   return static_cast<uint32_t>(q - p);
 }
 
@@ -278,21 +303,11 @@ __device__ __forceinline__ uint32_t smem_word_at(const uint8_t* sb, uint32_t i) 
   return __funnelshift_r(w0, w1, sh);
 }
 __device__ __forceinline__ uint64_t hash_smem(const uint8_t* sb, uint32_t i, uint32_t len, uint64_t seed) {
-  uint64_t h = seed ^ (static_cast<uint64_t>(len) * 0x9E3779B97F4A7C15ULL);
+  KeyHash hs(seed, len);
   uint32_t k = 0;
-  for (; k + 8 <= len; k += 8) {
-    const uint64_t b = static_cast<uint64_t>(smem_word_at(sb, i + k)) |
-                       (static_cast<uint64_t>(smem_word_at(sb, i + k + 4)) << 32);
-    h = mix64(h ^ b) + 0x632BE59BD9B4E019ULL;
-  }
-  if (k < len) {
-    const uint32_t r = len - k;
-    uint64_t b = static_cast<uint64_t>(smem_word_at(sb, i + k));
-    if (r > 4) b |= static_cast<uint64_t>(smem_word_at(sb, i + k + 4)) << 32;
-    b &= (1ULL << (8 * r)) - 1ULL;
-    h = mix64(h ^ b ^ 0xA5A5A5A5ULL);
-  }
-  return mix64(h);
+  for (; k + 4 <= len; k += 4) hs.add(smem_word_at(sb, i + k));
+  if (k < len) hs.add(smem_word_at(sb, i + k) & ((1u << (8 * (len - k))) - 1u));
+  return hs.finish();
 }
 
 // Sort key of the key bytes [q, q + len): inline when <= 7 bytes, else the 64-bit hash.
@@ -404,7 +419,7 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
     const uint32_t cnt0 = *reinterpret_cast<volatile unsigned int*>(&oc->fcount[h]);
     const bool fin = *reinterpret_cast<volatile unsigned int*>(&oc->is_final) &&
                      *reinterpret_cast<volatile unsigned int*>(&oc->final_seq) == f;
-    uint8_t* half = smem + Layout::out + h * kOutHalf;
+    uint8_t* half = smem + Layout<W>::out + h * Cfg<W>::kOutHalf;
     // the sealed buffer's writers finish on their own: wait until all cnt0 entries are committed
     if (lane == 0) {
       volatile unsigned int* cm = &oc->committed[h];
@@ -468,15 +483,17 @@ __device__ void stage_copy_edges(uint8_t* d, const uint8_t* g, uint64_t len, uin
 // Text tiles: once the TMA of stage s has landed, the producer warp turns the staged offsets
 // slice into the record-start bitmap and releases the stage to the map warps (ready[s]).
 // Done one tile behind the TMA issue, so the copy latency is hidden.
+template <int W>
 __device__ void finish_stage(const Params& P, uint8_t* smem, uint32_t it) {
+  constexpr int kStages = Cfg<W>::kStages;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout::full);
-  uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout::ready);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
+  uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout<W>::ready);
   mbar_wait(&full[s], ph);
-  const StageHdr* hd = reinterpret_cast<const StageHdr*>(smem + Layout::hdr + s * 128);
-  uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout::bits + s * kBitBytes);
-  const uint64_t* soff = reinterpret_cast<const uint64_t*>(smem + Layout::offs + s * kOffBytes + hd->off_shift);
+  const StageHdr* hd = reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
+  uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout<W>::bits + s * kBitBytes);
+  const uint64_t* soff = reinterpret_cast<const uint64_t*>(smem + Layout<W>::offs + s * kOffBytes + hd->off_shift);
   const uint64_t ra = hd->ra, cnt = hd->rb - hd->ra;
   const long long sbase = hd->sbase;
   const bool staged = hd->off_staged != 0;
@@ -491,9 +508,10 @@ __device__ void finish_stage(const Params& P, uint8_t* smem, uint32_t it) {
 
 template <int W>
 __device__ void producer_loop(const Params& P, uint8_t* smem) {
+  constexpr int kStages = Cfg<W>::kStages;
   const uint32_t lane = threadIdx.x & 31;
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout::full);
-  uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout::empty);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
+  uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
   uint32_t it = 0;
   const long long N = static_cast<long long>(P.nbytes);
   for (uint64_t t0 = blockIdx.x; t0 < P.ntiles; t0 += 32ULL * gridDim.x) {
@@ -508,10 +526,10 @@ __device__ void producer_loop(const Params& P, uint8_t* smem) {
       const uint64_t ra = __shfl_sync(kFull, my_ra, j), rb = __shfl_sync(kFull, my_rb, j);
       const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
       mbar_wait(&empty[s], ph ^ 1u);
-      StageHdr* hd = reinterpret_cast<StageHdr*>(smem + Layout::hdr + s * 128);
-      uint8_t* sb = smem + Layout::bytes + s * kStageBytes;
+      StageHdr* hd = reinterpret_cast<StageHdr*>(smem + Layout<W>::hdr + s * 128);
+      uint8_t* sb = smem + Layout<W>::bytes + s * kStageBytes;
       uint32_t b_off = 0, b_len = 0, o_off = 0, o_len = 0;
-      uint8_t* so = smem + Layout::offs + s * kOffBytes;
+      uint8_t* so = smem + Layout<W>::offs + s * kOffBytes;
       if constexpr (W == kKM) {
         const uint64_t p_lo = t * kKmPts, p_hi = min(P.n, p_lo + kKmPts);
         const uint8_t* g = P.rec + p_lo * 32;
@@ -538,7 +556,7 @@ __device__ void producer_loop(const Params& P, uint8_t* smem) {
         const uint8_t* g = P.rec + w_lo;
         stage_copy_edges(d, g, static_cast<uint64_t>(max(0LL, stg_hi - w_lo)), lane, b_off, b_len);
         // clear the record-start bitmap (map warps set bits after the full barrier)
-        uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout::bits + s * kBitBytes);
+        uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout<W>::bits + s * kBitBytes);
         for (uint32_t i = lane; i < kBitBytes / 16; i += 32) reinterpret_cast<uint4*>(bm)[i] = make_uint4(0, 0, 0, 0);
         // offsets slice offsets[ra..rb) (record starts in the staged window)
         const uint64_t cnt = rb - ra;
@@ -547,7 +565,21 @@ __device__ void producer_loop(const Params& P, uint8_t* smem) {
         const uint8_t* og = reinterpret_cast<const uint8_t*>(P.off + ra);
         if (staged && cnt) {
           shift = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(og) & 15u);
-          stage_copy_edges(so + shift, og, cnt * 8, lane, o_off, o_len);
+          // Copy the 16-B aligned superset of the slice with TMA alone (no synchronous edge
+          // loads on the producer's critical path) whenever it stays inside offsets[0..n].
+          const uint8_t* a_lo = og - shift;
+          const uint8_t* a_hi = reinterpret_cast<const uint8_t*>(
+              (reinterpret_cast<uintptr_t>(og + cnt * 8) + 15u) & ~static_cast<uintptr_t>(15u));
+          if (a_lo >= reinterpret_cast<const uint8_t*>(P.off) && a_hi <= P.off_end) {
+            o_off = 0;
+            o_len = static_cast<uint32_t>(a_hi - a_lo);
+            og = a_lo;
+            // so + shift still addresses offsets[ra]; the TMA below starts at so (= a_lo)
+          } else {
+            stage_copy_edges(so + shift, og, cnt * 8, lane, o_off, o_len);
+            og = og - shift;
+            o_off += shift;
+          }
         }
         if (lane == 0) {
           hd->t = static_cast<long long>(t);
@@ -565,23 +597,23 @@ __device__ void producer_loop(const Params& P, uint8_t* smem) {
         if (lane == 0) {
           mbar_arrive_expect_tx(&full[s], b_len + o_len);
           if (b_len) tma_load_1d(d + b_off, g + b_off, b_len, &full[s]);
-          if (o_len) tma_load_1d(so + shift + o_off, og + o_off, o_len, &full[s]);
+          if (o_len) tma_load_1d(so + o_off, og + o_off, o_len, &full[s]);
         }
-        if (it >= kLag) finish_stage(P, smem, it - kLag);
+        if (it >= Cfg<W>::kLag) finish_stage<W>(P, smem, it - Cfg<W>::kLag);
       }
       ++it;
     }
   }
   if constexpr (W != kKM) {
-    for (uint32_t j = (it >= kLag ? it - kLag : 0); j < it; ++j) finish_stage(P, smem, j);
+    for (uint32_t j = (it >= Cfg<W>::kLag ? it - Cfg<W>::kLag : 0); j < it; ++j) finish_stage<W>(P, smem, j);
   }
   // end-of-work marker
   const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
   mbar_wait(&empty[s], ph ^ 1u);
   if (lane == 0) {
-    reinterpret_cast<StageHdr*>(smem + Layout::hdr + s * 128)->t = -1;
+    reinterpret_cast<StageHdr*>(smem + Layout<W>::hdr + s * 128)->t = -1;
     if constexpr (W == kKM) mbar_arrive(&full[s]);
-    else mbar_arrive(reinterpret_cast<uint64_t*>(smem + Layout::ready) + s);
+    else mbar_arrive(reinterpret_cast<uint64_t*>(smem + Layout<W>::ready) + s);
   }
 }
 
@@ -675,16 +707,21 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
   const uint32_t total = __reduce_add_sync(kFull, cnt);
   if (total == 0) return;
   const Slot slot = reserve<W>(P, oc, outh, total, P.out_cap);
-  uint8_t* half = outh + slot.half * kOutHalf;
+  uint8_t* half = outh + slot.half * Cfg<W>::kOutHalf;
   uint64_t* sh = reinterpret_cast<uint64_t*>(half);
   uint64_t* sk = sh + F::kCap;
   uint8_t* sv = half + F::kCap * (F::kKref ? 16 : 8);
   uint32_t k = slot.base;
   uint32_t m_left = emit_mask;
   int nth = 0;
+  uint32_t nq = 0;                                   // WC: queued long words of this window
+  uint64_t* hq = reinterpret_cast<uint64_t*>(outh + (Layout<W>::hq - Layout<W>::out)) +
+                 (threadIdx.x >> 5) * Cfg<W>::kHashQ;
   while (__any_sync(kFull, m_left != 0)) {
     const bool act = m_left != 0;
     const uint32_t m = __ballot_sync(kFull, act);
+    bool queue = false;
+    uint64_t qe = 0;
     if (act) {
       const uint32_t j = __ffs(m_left) - 1;
       m_left &= m_left - 1;
@@ -693,9 +730,14 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
       if constexpr (W == kWC) {
         const uint32_t rest = nb >> (j + 1);
         uint32_t len = rest ? static_cast<uint32_t>(__ffs(rest)) : slow_word_len(P, tv, p, p0 + (lane < 31 ? 32 : 16));
-        const uint64_t key = (len <= 7) ? inline_key(window8(x, j), len) : key_at(P, tv, p, len);
         if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
-        sh[idx] = key;
+        if (len <= 7) {
+          sh[idx] = inline_key(window8(x, j), len);
+        } else {                                      // hashed after the rounds, all lanes together
+          queue = true;
+          qe = static_cast<uint64_t>(idx) | (static_cast<uint64_t>(p - tv.sbase) << 16) |
+               (static_cast<uint64_t>(len) << 40);
+        }
         sk[idx] = (reinterpret_cast<uint64_t>(P.rec + p) << 16) | len;
         reinterpret_cast<uint32_t*>(sv)[idx] = 1u;
       } else if constexpr (W == kSM) {
@@ -710,27 +752,42 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
         reinterpret_cast<uint64_t*>(sv)[idx] = P.gbase + static_cast<uint64_t>(q0);
       }
     }
+    if constexpr (W == kWC) {
+      const uint32_t qm = __ballot_sync(kFull, queue);
+      if (queue) hq[nq + __popc(qm & lanemask_lt())] = qe;
+      nq += __popc(qm);
+    }
     k += __popc(m);
+  }
+  if constexpr (W == kWC) {
+    __syncwarp();
+    for (uint32_t q = lane; q < nq; q += 32) {         // lane-parallel hashing of the long words
+      const uint64_t e = hq[q];
+      const uint32_t idx = static_cast<uint32_t>(e & 0xFFFF);
+      const long long p = tv.sbase + static_cast<long long>((e >> 16) & 0xFFFFFF);
+      sh[idx] = key_at(P, tv, p, static_cast<uint32_t>(e >> 40));
+    }
   }
   commit(oc, slot, total);
 }
 
 template <int W>
 __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
+  constexpr int kStages = Cfg<W>::kStages;
   using F = PairFmt<W>;
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t tid = threadIdx.x;  // 0 .. kNMap*32-1
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout::full);
-  uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout::empty);
-  uint8_t* outh = smem + Layout::out;
-  const float* cent = reinterpret_cast<const float*>(smem + Layout::cent);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
+  uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
+  uint8_t* outh = smem + Layout<W>::out;
+  const float* cent = reinterpret_cast<const float*>(smem + Layout<W>::cent);
   for (uint32_t it = 0;; ++it) {
     const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
     if constexpr (W == kKM) mbar_wait(&full[s], ph);
-    else mbar_wait(reinterpret_cast<uint64_t*>(smem + Layout::ready) + s, ph);
-    const StageHdr hd = *reinterpret_cast<const StageHdr*>(smem + Layout::hdr + s * 128);
+    else mbar_wait(reinterpret_cast<uint64_t*>(smem + Layout<W>::ready) + s, ph);
+    const StageHdr hd = *reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
     if (hd.t < 0) break;
-    const uint8_t* sb = smem + Layout::bytes + s * kStageBytes;
+    const uint8_t* sb = smem + Layout<W>::bytes + s * kStageBytes;
     if constexpr (W == kKM) {
       const uint64_t i = static_cast<uint64_t>(hd.lo) + tid;
       const bool valid = i < static_cast<uint64_t>(hd.hi);
@@ -786,7 +843,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         const Slot slot = reserve<W>(P, oc, outh, total, P.out_cap);
         if (valid) {
           const uint32_t idx = slot.base + __popc(m & lanemask_lt());
-          uint8_t* half = outh + slot.half * kOutHalf;
+          uint8_t* half = outh + slot.half * Cfg<W>::kOutHalf;
           reinterpret_cast<uint64_t*>(half)[idx] = best;
           float4* sv = reinterpret_cast<float4*>(half + F::kCap * 8 + static_cast<size_t>(idx) * 32);
           sv[0] = make_float4(x[0], x[1], x[2], x[3]);
@@ -795,7 +852,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         commit(oc, slot, total);
       }
     } else {
-      const uint32_t* bm = reinterpret_cast<const uint32_t*>(smem + Layout::bits + s * kBitBytes);
+      const uint32_t* bm = reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * kBitBytes);
       TileView tv{sb, bm, hd.sbase, hd.stg_hi};
       for (uint32_t w = warp; w < kNWin; w += kNMap) {
         const long long wp = hd.chunk0 + static_cast<long long>(w) * kWin;
@@ -818,8 +875,9 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
 
 template <int W>
 __global__ void __launch_bounds__(kThreads, 1) k_map(Params P) {
+  constexpr int kStages = Cfg<W>::kStages;
   extern __shared__ __align__(128) uint8_t smem[];
-  OutCtl* oc = reinterpret_cast<OutCtl*>(smem + Layout::ctl);
+  OutCtl* oc = reinterpret_cast<OutCtl*>(smem + Layout<W>::ctl);
   if (threadIdx.x == 0) {
     oc->cur = 0;
     oc->final_seq = 0;
@@ -829,14 +887,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_map(Params P) {
     oc->nsealed = 0;
     oc->is_final = 0;
     for (int b = 0; b < kNOut; ++b) { mbar_init(&oc->req[b], 1); mbar_init(&oc->done[b], kNFlush); }
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout::full);
-    uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout::empty);
-    uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout::ready);
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
+    uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
+    uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout<W>::ready);
     for (int s = 0; s < kStages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], kNMap); mbar_init(&ready[s], 1); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if constexpr (W == kKM) {
-    float* cent = reinterpret_cast<float*>(smem + Layout::cent);
+    float* cent = reinterpret_cast<float*>(smem + Layout<W>::cent);
     // pair layout: centroids (2p, 2p+1) interleaved per coordinate -> f32x2 operands
     for (uint32_t i = threadIdx.x; i < P.k * 8; i += blockDim.x) {
       const uint32_t j = i / 8, t = i % 8;
@@ -896,6 +954,9 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.flags = a.flags;
   P.st = a.st;
   P.tb = a.tile_bounds;
+  P.off_end = a.offsets ? reinterpret_cast<const uint8_t*>(
+                              reinterpret_cast<uintptr_t>(a.offsets + a.n + 1) & ~static_cast<uintptr_t>(15u))
+                        : nullptr;
   P.hash_seed = a.hash_seed;
   if (P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
@@ -903,7 +964,7 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
     k_tile_bounds<<<blocks, 256, 0, s>>>(a.offsets, a.n, P.ntiles, P.a0, a.tile_bounds);
     count_launch();
   }
-  const size_t smem = Layout::cent + (W == kKM ? static_cast<size_t>(a.k) * 32 : 0);
+  const size_t smem = Layout<W>::cent + (W == kKM ? static_cast<size_t>(a.k) * 32 : 0);
   cudaError_t e = cudaFuncSetAttribute(k_map<W>, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
   if (e != cudaSuccess) return e;
   int grid = a.grid > 0 ? a.grid : num_sms;

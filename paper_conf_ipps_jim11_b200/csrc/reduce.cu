@@ -149,35 +149,54 @@ __global__ void __launch_bounds__(kSegThreads) k_seg_write(const uint64_t* __res
 }
 
 // ---------------------------------------------------------------- WordCount reduce (u64 sums)
+// Segment-size-aware WC reduce.  A warp takes 32 consecutive segments: tiny ones (<= 32 pairs,
+// the long tail of the Zipf vocabulary) are summed by their own lane (TR, L181); medium ones
+// (<= kSmallWC) by the whole warp in turn; large ones become kLargeTile work items for the
+// block-level kernel below (BR).
+// Segment-size-aware WC reduce (values gathered through perm).  A warp takes 32 consecutive
+// segments: tiny ones (<= 32 pairs, the long tail of the Zipf vocabulary) are summed by their
+// own lane (TR, L181); medium ones (<= kSmallWC) by the whole warp in turn; large ones become
+// kLargeTile work items for the block-level kernel below (BR).
 template <typename V>
 __global__ void k_reduce_wc_small(const uint64_t* __restrict__ seg, uint64_t nseg, const uint32_t* __restrict__ perm,
-                                  const V* __restrict__ v, uint64_t* counts, uint64_t* worklist,
-                                  DevState* st) {
+                                  const V* __restrict__ v, uint64_t* counts, uint64_t* worklist, DevState* st) {
   const uint64_t gw = (blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x) >> 5;
   const uint64_t nw = (static_cast<uint64_t>(gridDim.x) * blockDim.x) >> 5;
   const uint32_t lane = threadIdx.x & 31;
-  for (uint64_t s = gw; s < nseg; s += nw) {
-    const uint64_t a = seg[s], b = seg[s + 1], size = b - a;
-    if (size <= kSmallWC) {
+  for (uint64_t s0 = gw * 32; s0 < nseg; s0 += nw * 32) {
+    const uint64_t s = s0 + lane;
+    uint64_t a = 0, b = 0;
+    if (s < nseg) { a = seg[s]; b = seg[s + 1]; }
+    const uint64_t size = b - a;
+    if (s < nseg && size <= 32) {                       // thread per key set
       uint64_t sum = 0;
-#pragma unroll 4
-      for (uint64_t i = a + lane; i < b; i += 32) sum += v[perm[i]];
-      sum = warp_sum_u64(sum);
-      if (lane == 0) counts[s] = sum;
-    } else if (lane == 0) {
+      for (uint64_t i = a; i < b; ++i) sum += v[perm[i]];
+      counts[s] = sum;
+    } else if (s < nseg && size > kSmallWC) {           // block-level work items
       counts[s] = 0;
       const uint64_t nt = (size + kLargeTile - 1) / kLargeTile;
       const uint64_t at = atomicAdd(&st->large_items, static_cast<unsigned long long>(nt));
       for (uint64_t t = 0; t < nt; ++t) worklist[at + t] = (s << 24) | t;
+    }
+    uint32_t med = __ballot_sync(0xffffffffu, s < nseg && size > 32 && size <= kSmallWC);
+    while (med) {                                        // warp per medium key set
+      const int L = __ffs(med) - 1;
+      med &= med - 1;
+      const uint64_t ma = __shfl_sync(0xffffffffu, a, L), mb = __shfl_sync(0xffffffffu, b, L);
+      uint64_t sum = 0;
+#pragma unroll 4
+      for (uint64_t i = ma + lane; i < mb; i += 32) sum += v[perm[i]];
+      sum = warp_sum_u64(sum);
+      if (lane == 0) counts[s0 + L] = sum;
     }
   }
 }
 
 template <typename V>
 __global__ void __launch_bounds__(256) k_reduce_wc_large(const uint64_t* __restrict__ seg,
-                                                       const uint32_t* __restrict__ perm,
-                                                       const V* __restrict__ v, uint64_t* counts,
-                                                       const uint64_t* __restrict__ worklist, DevState* st) {
+                                                       const uint32_t* __restrict__ perm, const V* __restrict__ v,
+                                                       uint64_t* counts, const uint64_t* __restrict__ worklist,
+                                                       DevState* st) {
   __shared__ unsigned long long item;
   __shared__ uint64_t red[8];
   const unsigned long long nitems = st->large_items;
@@ -381,17 +400,15 @@ cudaError_t launch_reduce_wc(const uint64_t* seg_start, uint64_t nseg, const uin
   if (nseg == 0) return cudaSuccess;
   cudaError_t e = cudaMemsetAsync(&st->large_items, 0, 2 * sizeof(unsigned long long), s);
   if (e != cudaSuccess) return e;
-  const unsigned g1 = static_cast<unsigned>(std::min<uint64_t>(blocks_for(nseg * 32, 256), 148ULL * 64));
+  const unsigned g1 = static_cast<unsigned>(std::min<uint64_t>(blocks_for(nseg, 256), 148ULL * 32));
   if (vbytes == 4) {
-    k_reduce_wc_small<uint32_t><<<g1, 256, 0, s>>>(seg_start, nseg, perm, reinterpret_cast<const uint32_t*>(v),
-                                                   counts, worklist, st);
-    k_reduce_wc_large<uint32_t><<<num_sms * 4, 256, 0, s>>>(seg_start, perm, reinterpret_cast<const uint32_t*>(v),
-                                                            counts, worklist, st);
+    const uint32_t* v4 = reinterpret_cast<const uint32_t*>(v);
+    k_reduce_wc_small<uint32_t><<<g1, 256, 0, s>>>(seg_start, nseg, perm, v4, counts, worklist, st);
+    k_reduce_wc_large<uint32_t><<<num_sms * 4, 256, 0, s>>>(seg_start, perm, v4, counts, worklist, st);
   } else {
-    k_reduce_wc_small<uint64_t><<<g1, 256, 0, s>>>(seg_start, nseg, perm, reinterpret_cast<const uint64_t*>(v),
-                                                   counts, worklist, st);
-    k_reduce_wc_large<uint64_t><<<num_sms * 4, 256, 0, s>>>(seg_start, perm, reinterpret_cast<const uint64_t*>(v),
-                                                            counts, worklist, st);
+    const uint64_t* v8 = reinterpret_cast<const uint64_t*>(v);
+    k_reduce_wc_small<uint64_t><<<g1, 256, 0, s>>>(seg_start, nseg, perm, v8, counts, worklist, st);
+    k_reduce_wc_large<uint64_t><<<num_sms * 4, 256, 0, s>>>(seg_start, perm, v8, counts, worklist, st);
   }
   count_launch(2);
   return cudaGetLastError();

@@ -13,6 +13,8 @@
 //     scattered through SMEM so that global writes are contiguous runs per digit.
 // Look-back status words: [epoch:30 | kind:2 | value:32]; every launch uses a fresh epoch so
 // the status buffer never needs clearing.
+#include <cstdlib>
+
 #include "common.cuh"
 
 namespace bmr {
@@ -43,7 +45,7 @@ __global__ void __launch_bounds__(256) k_hist(const uint64_t* __restrict__ keys,
 struct SortSmem {
   uint64_t keys[kSortTile];
   uint32_t idx[kSortTile];
-  uint32_t wcnt[kWarps][256];
+  uint32_t wcnt[kWarps][256];      // per-warp digit counters, then warp-exclusive offsets
   uint32_t hist[256];
   uint32_t dstart[256];
   uint32_t goff[256];
@@ -53,7 +55,10 @@ struct SortSmem {
 
 constexpr int kLookWindow = 4;   // predecessor status words fetched per look-back step
 
-template <bool kFirst>
+// kVar bit 0: rank with one shared atomic per match group (1) or a read-modify-write of the
+// warp counter per step (0); bit 1: tile histogram by shared atomics before ranking, published
+// as an early aggregate (1), or summed from the warp counters after ranking (0).
+template <bool kFirst, int kVar>
 __global__ void __launch_bounds__(kSortThreads, 3) k_onesweep(const uint64_t* __restrict__ keys_in,
                                                             const uint32_t* __restrict__ idx_in,
                                                             uint64_t* __restrict__ keys_out,
@@ -61,6 +66,7 @@ __global__ void __launch_bounds__(kSortThreads, 3) k_onesweep(const uint64_t* __
                                                             uint32_t shift, const uint32_t* __restrict__ bases,
                                                             uint64_t* status, uint32_t epoch,
                                                             unsigned int* tile_counter) {
+  constexpr bool kAtomicRank = (kVar & 1) != 0, kEarly = (kVar & 2) != 0;
   extern __shared__ __align__(16) uint8_t raw[];
   SortSmem& S = *reinterpret_cast<SortSmem*>(raw);
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -78,28 +84,53 @@ __global__ void __launch_bounds__(kSortThreads, 3) k_onesweep(const uint64_t* __
     const uint64_t e = wbase + j * 32 + lane;
     key[j] = e < m ? keys_in[e] : ~0ULL;  // padding sorts last (digit 255, after every real key)
   }
-  // 1. tile histogram first, published immediately (early aggregate for the successors)
-#pragma unroll
-  for (int j = 0; j < kSortIPT; ++j) atomicAdd(&S.hist[static_cast<uint32_t>(key[j] >> shift) & 255u], 1u);
-  __syncthreads();
   const uint32_t d = tid;  // kSortThreads == 256: one digit per thread
-  const uint32_t tcount = S.hist[d];
+  uint32_t tcount = 0;
   uint64_t* my = status + static_cast<uint64_t>(tile) * 256 + d;
-  st_relaxed_gpu_u64(my, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount));
-  // 2. stable warp-level ranking (element order == (j, lane) order inside the warp)
+  if constexpr (kEarly) {
+    // 1. tile histogram first, published immediately (early aggregate for the successors)
 #pragma unroll
-  for (int j = 0; j < kSortIPT; ++j) {
-    const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & 255u;
-    const uint32_t peers = __match_any_sync(0xffffffffu, dj);
-    const uint32_t leader = __ffs(peers) - 1;
-    uint32_t before = 0;
-    if (lane == leader) {
-      before = S.wcnt[warp][dj];
-      S.wcnt[warp][dj] = before + __popc(peers);
+    for (int j = 0; j < kSortIPT; ++j) atomicAdd(&S.hist[static_cast<uint32_t>(key[j] >> shift) & 255u], 1u);
+    __syncthreads();
+    tcount = S.hist[d];
+    st_relaxed_gpu_u64(my, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount));
+  }
+  // 2. stable warp-level ranking (element order == (j, lane) order inside the warp)
+  if constexpr (kAtomicRank) {
+    // the leader of each match group reserves the group's slots with one shared atomicAdd; a
+    // warp's atomics are applied in issue order, their results are consumed afterwards
+    uint32_t peers[kSortIPT];
+#pragma unroll
+    for (int j = 0; j < kSortIPT; ++j) {
+      const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & 255u;
+      peers[j] = __match_any_sync(0xffffffffu, dj);
+      rank[j] = 0;
+      if (lane == static_cast<uint32_t>(__ffs(peers[j]) - 1)) rank[j] = atomicAdd(&S.wcnt[warp][dj], __popc(peers[j]));
     }
-    __syncwarp();   // order this step's counter updates before the next step's reads
-    before = __shfl_sync(0xffffffffu, before, leader);
-    rank[j] = before + __popc(peers & lanemask_lt());
+#pragma unroll
+    for (int j = 0; j < kSortIPT; ++j)
+      rank[j] = __shfl_sync(0xffffffffu, rank[j], __ffs(peers[j]) - 1) + __popc(peers[j] & lanemask_lt());
+  } else {
+#pragma unroll
+    for (int j = 0; j < kSortIPT; ++j) {
+      const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & 255u;
+      const uint32_t peers = __match_any_sync(0xffffffffu, dj);
+      const uint32_t leader = __ffs(peers) - 1;
+      uint32_t before = 0;
+      if (lane == leader) {
+        before = S.wcnt[warp][dj];
+        S.wcnt[warp][dj] = before + __popc(peers);
+      }
+      __syncwarp();   // order this step's counter updates before the next step's reads
+      before = __shfl_sync(0xffffffffu, before, leader);
+      rank[j] = before + __popc(peers & lanemask_lt());
+    }
+  }
+  __syncthreads();
+  if constexpr (!kEarly) {
+#pragma unroll
+    for (int w = 0; w < kWarps; ++w) tcount += S.wcnt[w][d];
+    st_relaxed_gpu_u64(my, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount));
   }
   __syncthreads();
   // 3. per digit: warp-exclusive offsets and the tile-local digit start
@@ -249,25 +280,45 @@ cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int nu
   return cudaGetLastError();
 }
 
+int sort_variant() {
+  static int v = [] {
+    const char* e = getenv("BMR_SORT_VARIANT");
+    return e ? atoi(e) & 3 : 2;
+  }();
+  return v;
+}
+
+template <bool kFirst, int kVar>
+static void launch_os(unsigned tiles, size_t smem, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
+                      uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
+                      uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
+  cudaFuncSetAttribute(k_onesweep<kFirst, kVar>, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
+  k_onesweep<kFirst, kVar><<<tiles, kSortThreads, smem, s>>>(keys_in, idx_in, keys_out, idx_out, m, shift, bases,
+                                                             status, epoch, tile_counter);
+}
+
 cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out, uint32_t* idx_out,
                             uint64_t m, int digit, const uint32_t* bases, uint64_t* status, uint32_t epoch,
                             unsigned int* tile_counter, cudaStream_t s) {
   if (m == 0) return cudaSuccess;
-  const uint64_t tiles = (m + kSortTile - 1) / kSortTile;
+  const unsigned tiles = static_cast<unsigned>((m + kSortTile - 1) / kSortTile);
   const size_t smem = sizeof(SortSmem);
   cudaError_t e = cudaMemsetAsync(tile_counter, 0, sizeof(unsigned int), s);
   if (e != cudaSuccess) return e;
-  if (idx_in == nullptr) {
-    cudaFuncSetAttribute(k_onesweep<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
-    k_onesweep<true><<<static_cast<unsigned>(tiles), kSortThreads, smem, s>>>(
-        keys_in, nullptr, keys_out, idx_out, m, 8u * digit, bases + 256 * digit, status, epoch, tile_counter);
-    count_launch();
-  } else {
-    cudaFuncSetAttribute(k_onesweep<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
-    k_onesweep<false><<<static_cast<unsigned>(tiles), kSortThreads, smem, s>>>(
-        keys_in, idx_in, keys_out, idx_out, m, 8u * digit, bases + 256 * digit, status, epoch, tile_counter);
-    count_launch();
+  const uint32_t shift = 8u * digit;
+  const uint32_t* b = bases + 256 * digit;
+  const bool first = idx_in == nullptr;
+  switch (sort_variant() | (first ? 4 : 0)) {
+    case 0: launch_os<false, 0>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    case 1: launch_os<false, 1>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    case 2: launch_os<false, 2>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    case 3: launch_os<false, 3>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    case 4: launch_os<true, 0>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    case 5: launch_os<true, 1>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    case 6: launch_os<true, 2>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    default: launch_os<true, 3>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
   }
+  count_launch();
   return cudaGetLastError();
 }
 
