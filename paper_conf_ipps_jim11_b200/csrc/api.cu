@@ -222,6 +222,7 @@ struct mr_job {
   HBuf<uint64_t> key_off_h, val_off_h;
   // multi-GPU exchange (§8(e))
   XSource xs;
+  uint32_t key_bits = 64;         // current sort-key width (WC maps with 48; re-hash -> 64)
   bool ingested = false;          // pairs come from mr_ingest (WC values are u64 partial counts)
   bool km_partial = false;        // KM: sums/cnts hold ingested partials; finalise owned clusters
   int vb_cur = 0;                 // value bytes of the current pairs
@@ -290,6 +291,7 @@ cudaError_t launch_batch(mr_job* job, const Batch& b) {
   a.out.cap = job->cap;
   a.st = job->st;
   a.hash_seed = 0x5EEDB200ULL;
+  a.key_bits = job->key_bits;
   const uint64_t nt = map_tiles(a);
   if (a.workload != kKM) {
     cudaError_t e = job->tb.ensure(2 * nt + 2);
@@ -313,7 +315,8 @@ mr_status do_segments(mr_job* job) {
   CK(job->tile_base.ensure(tiles + 1), "alloc tile base");
   CK(cudaMemsetAsync(&job->st->collisions, 0, sizeof(unsigned int), job->stream), "memset");
   const uint64_t* kref = has_kref(job->cfg.workload) ? job->kref.p : nullptr;
-  CK(launch_seg_count(job->skeys, job->perm, kref, m, job->seg_counts.p, job->st, job->stream), "seg_count");
+  CK(launch_seg_count(job->skeys, job->perm, kref, m, job->seg_counts.p, job->st, job->key_bits, job->stream),
+     "seg_count");
   CK(launch_scan_u32to64(job->seg_counts.p, job->tile_base.p, tiles, &job->st->seg_total, job->sw.status.p,
                          job->sw.epoch++, &job->st->tile_counter[1], job->stream),
      "scan tiles");
@@ -396,6 +399,7 @@ mr_status mr_job_create(const mr_config* cfg, mr_job** out) {
   }
   job->nsm = sm_count(cfg->device);
   job->prof.on = (cfg->flags & MR_FLAG_PROFILE) != 0;
+  job->key_bits = (cfg->workload == MR_WORDCOUNT) ? 48u : 64u;
   job->launches0 = g_kernel_launches.load();
   *out = job;
   return MR_OK;
@@ -410,6 +414,7 @@ mr_status mr_job_reset(mr_job* job) {
   job->host_batches = 0;
   job->ingested = false;
   job->km_partial = false;
+  job->key_bits = (job->cfg.workload == MR_WORDCOUNT) ? 48u : 64u;
   job->prof.collect();
   job->batches.clear();
   job->next_base = 0;
@@ -544,6 +549,7 @@ mr_status mr_group(mr_job* job) {
     if (attempt >= 3) return fail(job, MR_ERR_UNSUPPORTED, "unresolvable 64-bit hash collision");
     // slow path: recompute every hashed key with a fresh full-width hash, then sort again
     CK(launch_rehash(job->h.p, job->kref.p, m_total, 0xC0111DE5ULL + attempt, job->stream), "rehash");
+    job->key_bits = 64;
   }
   job->stats.n_keys = job->nseg;
   Prof::Span sp3{};
@@ -806,7 +812,7 @@ mr_status mr_ingest(mr_job* job, const void* entries, const void* heap, const ui
   CK(cudaMemcpyAsync(job->src_h.p, sh.data(), (R + 1) * 8, cudaMemcpyHostToDevice, s), "H2D src");
   CK(launch_x_ingest(entries, static_cast<const uint8_t*>(heap), n, job->src_e.p, job->src_h.p, R, job->h.p,
                      job->kref.p, reinterpret_cast<uint64_t*>(job->v.p), 0x5EEDB200ULL,
-                     (job->cfg.flags & MR_FLAG_WEAK_HASH_DEBUG) ? 1u : 0u, s),
+                     (job->cfg.flags & MR_FLAG_WEAK_HASH_DEBUG) ? 1u : 0u, job->key_bits, s),
      "ingest");
   CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), s), "reset state");
   job->tmp_h.p[0] = n;

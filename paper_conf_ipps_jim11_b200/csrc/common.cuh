@@ -102,7 +102,6 @@ __host__ __device__ __forceinline__ uint64_t mix64(uint64_t z) {  // murmur3 fin
   z ^= z >> 33;
   return z;
 }
-constexpr uint64_t kHashedBit = 1ULL << 63;
 
 // 64-bit key hash over 4-byte little-endian words (last word zero-padded): two 32-bit lanes
 // (murmur3-style rounds) so that the map warps stay on 32-bit IMAD/LOP3; hash_bytes (generic
@@ -139,16 +138,37 @@ __device__ __forceinline__ uint64_t hash_bytes(const uint8_t* p, uint32_t len, u
   }
   return hs.finish();
 }
-// Final sort key of a hashed key; weak_hash (MR_FLAG_WEAK_HASH_DEBUG) keeps only 4 bits so
-// that almost every segment collides (tests the verification + re-sort slow path).
-// ~0 is reserved for the flush filler sentinel, so a hashed key never equals it.
-__device__ __forceinline__ uint64_t hashed_key(uint64_t h, bool weak) {
-  const uint64_t k = (weak ? (h & 0xFULL) : (h & ~kHashedBit)) | kHashedBit;
-  return k == ~0ULL ? ~0ULL - 1 : k;
+// Sort-key formats.  The key width is 64 bits (II, re-hash slow path) or 48 bits (WC: two LSD
+// passes fewer; digits 6 and 7 are then constant and skipped):
+//   inline  : keys of <= kInlineMax bytes packed little-endian, length in the 3 bits above them
+//             (64: len << 56, <= 7 bytes; 48: len << 40, <= 5 bytes) — injective, top bit clear;
+//   hashed  : longer keys -> hash with the top bit of the width forced to 1 (never collides with
+//             an inline key); equal hashes are verified byte-for-byte at segment time;
+//   sentinel: all ones in the width — flush filler pairs, sorts after every real key.
+__host__ __device__ __forceinline__ uint32_t inline_max(uint32_t bits) { return bits == 48 ? 5u : 7u; }
+__host__ __device__ __forceinline__ uint64_t hashed_bit(uint32_t bits) { return 1ULL << (bits - 1); }
+__host__ __device__ __forceinline__ uint64_t sentinel_of(uint32_t bits) {
+  return bits == 64 ? ~0ULL : ((1ULL << bits) - 1ULL);
 }
-// <= 7 bytes packed little-endian, length in bits 56..63 (1..7): injective, top bit clear.
-__device__ __forceinline__ uint64_t inline_key(uint64_t bytes_le, uint32_t len) {
-  return (bytes_le & ((1ULL << (8 * len)) - 1ULL)) | (static_cast<uint64_t>(len) << 56);
+// WEAK (MR_FLAG_WEAK_HASH_DEBUG) keeps only 4 hash bits so that almost every segment collides
+// (tests the verification + re-sort slow path).
+__device__ __forceinline__ uint64_t hashed_key(uint64_t h, bool weak, uint32_t bits = 64) {
+  const uint64_t hb = hashed_bit(bits);
+  const uint64_t k = (weak ? (h & 0xFULL) : (h & (hb - 1ULL))) | hb;
+  return k == sentinel_of(bits) ? k - 1ULL : k;
+}
+__device__ __forceinline__ uint64_t inline_key(uint64_t bytes_le, uint32_t len, uint32_t bits = 64) {
+  return (bytes_le & ((1ULL << (8 * len)) - 1ULL)) | (static_cast<uint64_t>(len) << (bits - 8));
+}
+// key bytes -> sort key (generic pointer)
+__device__ __forceinline__ uint64_t key_of_bytes(const uint8_t* p, uint32_t len, uint64_t seed, bool weak,
+                                                 uint32_t bits) {
+  if (len <= inline_max(bits)) {
+    uint64_t b = 0;
+    for (uint32_t k = 0; k < len; ++k) b |= static_cast<uint64_t>(p[k]) << (8 * k);
+    return inline_key(b, len, bits);
+  }
+  return hashed_key(hash_bytes(p, len, seed), weak, bits);
 }
 
 // ---------------------------------------------------------------- small scans

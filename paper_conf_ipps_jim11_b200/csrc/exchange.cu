@@ -127,7 +127,7 @@ __global__ void __launch_bounds__(kXThreads) k_x_scatter(XSource S, unsigned lon
 // heap bytes received from each source rank.
 __global__ void k_x_ingest(const XEntry* __restrict__ ent, const uint8_t* heap, uint64_t n, const uint64_t* src_e,
                            const uint64_t* src_h, uint32_t R, uint64_t* h, uint64_t* kref, uint64_t* v,
-                           uint64_t seed, uint32_t weak) {
+                           uint64_t seed, uint32_t weak, uint32_t key_bits) {
   const uint64_t j = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
   if (j >= n) return;
   uint32_t r = 0;
@@ -135,14 +135,7 @@ __global__ void k_x_ingest(const XEntry* __restrict__ ent, const uint8_t* heap, 
   const XEntry x = ent[j];
   const uint32_t klen = static_cast<uint32_t>(x.koff_len & 0xFFFF);
   const uint8_t* kp = heap + src_h[r] + (x.koff_len >> 16);
-  uint64_t key;
-  if (klen <= 7) {
-    uint64_t b = 0;
-    for (uint32_t k = 0; k < klen; ++k) b |= static_cast<uint64_t>(kp[k]) << (8 * k);
-    key = inline_key(b, klen);
-  } else {
-    key = hashed_key(hash_bytes(kp, klen, seed), weak != 0);
-  }
+  const uint64_t key = key_of_bytes(kp, klen, seed, weak != 0, key_bits);
   h[j] = key;
   kref[j] = (reinterpret_cast<uint64_t>(kp) << 16) | klen;
   v[j] = x.v;
@@ -185,10 +178,10 @@ cudaError_t launch_x_scatter(const XSource& S, unsigned long long* cursors, uint
 
 cudaError_t launch_x_ingest(const void* entries, const uint8_t* heap, uint64_t n, const uint64_t* src_e,
                             const uint64_t* src_h, uint32_t R, uint64_t* h, uint64_t* kref, uint64_t* v,
-                            uint64_t seed, uint32_t weak, cudaStream_t s) {
+                            uint64_t seed, uint32_t weak, uint32_t key_bits, cudaStream_t s) {
   if (n == 0) return cudaSuccess;
   k_x_ingest<<<nblocks(n, 256), 256, 0, s>>>(static_cast<const XEntry*>(entries), heap, n, src_e, src_h, R, h, kref,
-                                             v, seed, weak);
+                                             v, seed, weak, key_bits);
   count_launch();
   return cudaGetLastError();
 }

@@ -52,6 +52,7 @@ struct MapArgs {
   DevState* st = nullptr;
   uint64_t* tile_bounds = nullptr;    // scratch: 2 u64 per tile
   uint64_t hash_seed = 0;
+  uint32_t key_bits = 64;             // sort-key width of hashed / inline keys (48 or 64)
   int grid = 0;                       // persistent CTAs (0 = one per SM)
 };
 
@@ -79,7 +80,7 @@ cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uin
 // ---- segments ----
 // heads per sort tile + byte verification of hashed keys; counts[t] = heads in tile t
 cudaError_t launch_seg_count(const uint64_t* skeys, const uint32_t* perm, const uint64_t* kref, uint64_t m,
-                             uint32_t* counts, DevState* st, cudaStream_t s);
+                             uint32_t* counts, DevState* st, uint32_t key_bits, cudaStream_t s);
 // exclusive scan of u64 (in-place allowed); writes total to *total if non-null
 cudaError_t launch_scan_u64(const uint64_t* in, uint64_t* out, uint64_t n, unsigned long long* total,
                             uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s);
@@ -111,6 +112,7 @@ cudaError_t launch_gather_u64(const uint32_t* perm, const uint8_t* v, uint64_t m
 cudaError_t launch_offsets_scaled(const uint64_t* seg_start, uint64_t nseg, uint64_t scale, uint64_t* out,
                                   cudaStream_t s);
 cudaError_t launch_iota_scaled(uint64_t n, uint64_t scale, uint64_t* out, cudaStream_t s);
+// recompute every key in the 64-bit format with a fresh hash seed (collision slow path)
 cudaError_t launch_rehash(uint64_t* h, const uint64_t* kref, uint64_t m, uint64_t seed, cudaStream_t s);
 
 // ---- multi-GPU exchange (exchange.cu) ----
@@ -138,7 +140,7 @@ cudaError_t launch_x_scatter(const XSource& S, unsigned long long* cursors, uint
                              cudaStream_t s);
 cudaError_t launch_x_ingest(const void* entries, const uint8_t* heap, uint64_t n, const uint64_t* src_e,
                             const uint64_t* src_h, uint32_t R, uint64_t* h, uint64_t* kref, uint64_t* v,
-                            uint64_t seed, uint32_t weak, cudaStream_t s);
+                            uint64_t seed, uint32_t weak, uint32_t key_bits, cudaStream_t s);
 cudaError_t launch_x_ingest_km(const void* entries, uint64_t n, double* sums, unsigned long long* cnts, uint32_t k,
                                cudaStream_t s);
 

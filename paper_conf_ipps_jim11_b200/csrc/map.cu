@@ -140,6 +140,7 @@ struct Params {
   const uint64_t* tb;      // tile bounds
   const uint8_t* off_end;  // end of the offsets array rounded DOWN to 16 B (aligned TMA limit)
   uint64_t hash_seed;
+  uint32_t key_bits;       // sort-key width (48 or 64)
 };
 
 constexpr uint32_t kFull = 0xffffffffu;
@@ -310,10 +311,10 @@ __device__ __forceinline__ uint64_t hash_smem(const uint8_t* sb, uint32_t i, uin
   return hs.finish();
 }
 
-// Sort key of the key bytes [q, q + len): inline when <= 7 bytes, else the 64-bit hash.
+// Sort key of the key bytes [q, q + len): inline when short, else the hash (common.cuh).
 __device__ __forceinline__ uint64_t key_at(const Params& P, const TileView& tv, long long q, uint32_t len) {
   const bool in_stage = (q + static_cast<long long>(len) <= tv.stg_hi) && (q - tv.sbase + len + 12 <= kStageBytes);
-  if (len <= 7) {
+  if (len <= inline_max(P.key_bits)) {
     uint64_t b = 0;
     if (in_stage) {
       const uint32_t i = static_cast<uint32_t>(q - tv.sbase);
@@ -321,11 +322,11 @@ __device__ __forceinline__ uint64_t key_at(const Params& P, const TileView& tv, 
     } else {
       for (uint32_t k = 0; k < len; ++k) b |= static_cast<uint64_t>(P.rec[q + k]) << (8 * k);
     }
-    return inline_key(b, len);
+    return inline_key(b, len, P.key_bits);
   }
   const uint64_t h = in_stage ? hash_smem(tv.sb, static_cast<uint32_t>(q - tv.sbase), len, P.hash_seed)
                               : hash_bytes(P.rec + q, len, P.hash_seed);
-  return hashed_key(h, (P.flags & 8u) != 0);
+  return hashed_key(h, (P.flags & 8u) != 0, P.key_bits);
 }
 
 // ---------------------------------------------------------------- emit allocator
@@ -341,7 +342,7 @@ constexpr uint32_t kCntMask = 0xFFFFFFu;
 template <int W>
 __device__ __forceinline__ uint64_t sentinel_key(const Params& P) {
   if constexpr (W == kKM) return P.k <= 255 ? 255ULL : 65535ULL;
-  return ~0ULL;
+  return sentinel_of(P.key_bits);
 }
 
 // Seal buffer h of the current generation: switch every warp to the next buffer at once (the
@@ -731,8 +732,8 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
         const uint32_t rest = nb >> (j + 1);
         uint32_t len = rest ? static_cast<uint32_t>(__ffs(rest)) : slow_word_len(P, tv, p, p0 + (lane < 31 ? 32 : 16));
         if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
-        if (len <= 7) {
-          sh[idx] = inline_key(window8(x, j), len);
+        if (len <= inline_max(P.key_bits)) {
+          sh[idx] = inline_key(window8(x, j), len, P.key_bits);
         } else {                                      // hashed after the rounds, all lanes together
           queue = true;
           qe = static_cast<uint64_t>(idx) | (static_cast<uint64_t>(p - tv.sbase) << 16) |
@@ -958,6 +959,7 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
                               reinterpret_cast<uintptr_t>(a.offsets + a.n + 1) & ~static_cast<uintptr_t>(15u))
                         : nullptr;
   P.hash_seed = a.hash_seed;
+  P.key_bits = a.key_bits;
   if (P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>((P.ntiles + 255) / 256);

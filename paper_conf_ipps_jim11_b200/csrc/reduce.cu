@@ -66,7 +66,7 @@ constexpr int kSegWarp = 32 * kSegIPT;   // positions per warp
 __global__ void __launch_bounds__(kSegThreads) k_seg_count(const uint64_t* __restrict__ sk,
                                                          const uint32_t* __restrict__ perm,
                                                          const uint64_t* __restrict__ kref, uint64_t m,
-                                                         uint32_t* counts, DevState* st) {
+                                                         uint32_t* counts, DevState* st, uint64_t hbit) {
   __shared__ uint32_t red[kSegThreads / 32];
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint64_t wbase = static_cast<uint64_t>(blockIdx.x) * kSegTile + static_cast<uint64_t>(warp) * kSegWarp;
@@ -84,8 +84,8 @@ __global__ void __launch_bounds__(kSegThreads) k_seg_count(const uint64_t* __res
     const bool head = valid && (i == 0 || k != prev);
     heads += head ? 1u : 0u;
     // byte verification of equal hashed keys (C-3 #13): adjacent pairs inside an equal-hash run
-    const bool hashed_run = valid && kref && (k & kHashedBit) && !head;
-    const bool need_r = valid && kref && (k & kHashedBit);
+    const bool hashed_run = valid && kref && (k & hbit) && !head;
+    const bool need_r = valid && kref && (k & hbit);
     const unsigned any = __ballot_sync(0xffffffffu, need_r);
     uint64_t r = 0;
     if (any) {
@@ -357,9 +357,8 @@ __global__ void k_rehash(uint64_t* h, const uint64_t* kref, uint64_t m, uint64_t
   const uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
   if (i >= m) return;
   const uint64_t kr = kref[i];
-  const uint32_t len = static_cast<uint32_t>(kr & 0xFFFF);
-  if (len <= 7) return;  // inline keys are exact already
-  h[i] = hashed_key(hash_bytes(reinterpret_cast<const uint8_t*>(kr >> 16), len, seed), false);
+  if (kr == 0) { h[i] = sentinel_of(64); return; }   // flush filler
+  h[i] = key_of_bytes(reinterpret_cast<const uint8_t*>(kr >> 16), static_cast<uint32_t>(kr & 0xFFFF), seed, false, 64);
 }
 
 inline unsigned blocks_for(uint64_t n, unsigned t) { return static_cast<unsigned>((n + t - 1) / t); }
@@ -367,9 +366,9 @@ inline unsigned blocks_for(uint64_t n, unsigned t) { return static_cast<unsigned
 }  // namespace
 
 cudaError_t launch_seg_count(const uint64_t* skeys, const uint32_t* perm, const uint64_t* kref, uint64_t m,
-                             uint32_t* counts, DevState* st, cudaStream_t s) {
+                             uint32_t* counts, DevState* st, uint32_t key_bits, cudaStream_t s) {
   if (m == 0) return cudaSuccess;
-  k_seg_count<<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, perm, kref, m, counts, st);
+  k_seg_count<<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, perm, kref, m, counts, st, hashed_bit(key_bits));
   count_launch();
   return cudaGetLastError();
 }
