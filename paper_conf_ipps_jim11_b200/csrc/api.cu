@@ -122,9 +122,12 @@ int sm_count(int dev) {
 
 // Radix sort of m keys: writes *out_keys / *out_perm pointing into the workspace (or to
 // `keys` + an identity permutation when every digit is constant).
+// hist_digits > 0: W.hist already holds the histograms of digits [0, hist_digits) (fused into
+// the Map flushes); the remaining digits are known to be constant zero.
 cudaError_t run_sort(SortWork& W, const uint64_t* keys, uint64_t m, const uint64_t** out_keys,
                      const uint32_t** out_perm, DevState* st, int nsm, cudaStream_t s, Prof* prof = nullptr,
-                     double* hist_ms = nullptr, double* pass_ms = nullptr) {
+                     double* hist_ms = nullptr, double* pass_ms = nullptr, int hist_digits = 0,
+                     int key_digits = 8) {
   cudaError_t e;
   if ((e = W.ka.ensure(m)) || (e = W.kb.ensure(m)) || (e = W.ia.ensure(m)) || (e = W.ib.ensure(m))) return e;
   const uint64_t tiles = (m + kSortTile - 1) / kSortTile;
@@ -135,12 +138,20 @@ cudaError_t run_sort(SortWork& W, const uint64_t* keys, uint64_t m, const uint64
   }
   if ((e = W.hist.ensure(8 * 256)) || (e = W.bases.ensure(8 * 256))) return e;
   if ((e = W.hist_h.ensure(8 * 256)) || (e = W.bases_h.ensure(8 * 256))) return e;
-  Prof::Span sp{};
-  if (prof && prof->on) prof->begin(s, sp);
-  if ((e = launch_hist(keys, m, W.hist.p, nsm, s))) return e;
-  if (prof && prof->on) prof->end(s, sp, hist_ms);
+  if (hist_digits == 0) {
+    Prof::Span sp{};
+    if (prof && prof->on) prof->begin(s, sp);
+    if ((e = launch_hist(keys, m, W.hist.p, key_digits, nsm, s))) return e;
+    hist_digits = key_digits;
+    if (prof && prof->on) prof->end(s, sp, hist_ms);
+  }
   if ((e = cudaMemcpyAsync(W.hist_h.p, W.hist.p, 8 * 256 * sizeof(uint32_t), cudaMemcpyDeviceToHost, s))) return e;
   if ((e = cudaStreamSynchronize(s))) return e;
+  if (hist_digits > 0)
+    for (int d = hist_digits; d < 8; ++d) {   // outside the key width (or packed value bits): not sorted
+      for (int b = 0; b < 256; ++b) W.hist_h.p[d * 256 + b] = 0;
+      W.hist_h.p[d * 256] = static_cast<uint32_t>(m);
+    }
   int digits[8];
   int nd = 0;
   for (int d = 0; d < 8; ++d) {
@@ -223,6 +234,9 @@ struct mr_job {
   // multi-GPU exchange (§8(e))
   XSource xs;
   uint32_t key_bits = 64;         // current sort-key width (WC maps with 48; re-hash -> 64)
+  // WC map output with 48-bit keys carries its value in bits 48..63 of the sorted word
+  bool packed() const { return cfg.workload == MR_WORDCOUNT && key_bits == 48 && !ingested; }
+  uint64_t kmask() const { return key_bits == 48 ? ((1ULL << 48) - 1ULL) : ~0ULL; }
   bool ingested = false;          // pairs come from mr_ingest (WC values are u64 partial counts)
   bool km_partial = false;        // KM: sums/cnts hold ingested partials; finalise owned clusters
   int vb_cur = 0;                 // value bytes of the current pairs
@@ -292,6 +306,9 @@ cudaError_t launch_batch(mr_job* job, const Batch& b) {
   a.st = job->st;
   a.hash_seed = 0x5EEDB200ULL;
   a.key_bits = job->key_bits;
+  a.hist = nullptr;   // flush-fused histograms measured slower (one flush warp, 6 atomics per pair)
+  // WC: the emitted value 1 rides in bits 48..63 of the sort word (the sort uses digits 0..5)
+  a.vpack = (job->cfg.workload == MR_WORDCOUNT && job->key_bits == 48) ? (1ULL << 48) : 0;
   const uint64_t nt = map_tiles(a);
   if (a.workload != kKM) {
     cudaError_t e = job->tb.ensure(2 * nt + 2);
@@ -315,7 +332,8 @@ mr_status do_segments(mr_job* job) {
   CK(job->tile_base.ensure(tiles + 1), "alloc tile base");
   CK(cudaMemsetAsync(&job->st->collisions, 0, sizeof(unsigned int), job->stream), "memset");
   const uint64_t* kref = has_kref(job->cfg.workload) ? job->kref.p : nullptr;
-  CK(launch_seg_count(job->skeys, job->perm, kref, m, job->seg_counts.p, job->st, job->key_bits, job->stream),
+  CK(launch_seg_count(job->skeys, job->perm, kref, m, job->seg_counts.p, job->st, job->key_bits, job->kmask(),
+                      job->stream),
      "seg_count");
   CK(launch_scan_u32to64(job->seg_counts.p, job->tile_base.p, tiles, &job->st->seg_total, job->sw.status.p,
                          job->sw.epoch++, &job->st->tile_counter[1], job->stream),
@@ -323,7 +341,7 @@ mr_status do_segments(mr_job* job) {
   CK(read_state(job), "sync segments");
   job->nseg = m ? job->st_h.p->seg_total : 0;
   CK(job->seg_start.ensure(job->nseg + 1), "alloc seg_start");
-  CK(launch_seg_write(job->skeys, m, job->tile_base.p, job->seg_start.p, job->stream), "seg_write");
+  CK(launch_seg_write(job->skeys, m, job->tile_base.p, job->seg_start.p, job->kmask(), job->stream), "seg_write");
   return MR_OK;
 }
 
@@ -426,6 +444,7 @@ mr_status mr_job_reset(mr_job* job) {
   job->stats.capacity_pairs = cap;
   job->launches0 = g_kernel_launches.load();
   CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset state");
+  if (job->sw.hist.p) CK(cudaMemsetAsync(job->sw.hist.p, 0, 8 * 256 * sizeof(uint32_t), job->stream), "zero hist");
   job->state = kCreated;
   return MR_OK;
 }
@@ -457,6 +476,10 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
   if (job->cap == 0) {
     CK(ensure_pairs(job, initial_cap(job, nbytes, n)), "alloc intermediate");
     job->stats.capacity_pairs = job->cap;
+  }
+  if (!job->sw.hist.p) {                      // digit histograms accumulated by the Map flushes
+    CK(job->sw.hist.ensure(8 * 256), "alloc histogram");
+    CK(cudaMemsetAsync(job->sw.hist.p, 0, 8 * 256 * sizeof(uint32_t), job->stream), "zero histogram");
   }
   Batch b{records, offsets, n, nbytes, job->cfg.input_base + job->next_base};
   job->next_base += nbytes;
@@ -515,6 +538,7 @@ mr_status mr_group(mr_job* job) {
     CK(ensure_pairs(job, ncap), "grow intermediate");
     job->stats.capacity_pairs = job->cap;
     CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
+    CK(cudaMemsetAsync(job->sw.hist.p, 0, 8 * 256 * sizeof(uint32_t), job->stream), "zero hist");
     for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
     job->stats.replays += job->batches.size();
     CK(read_state(job), "replay (async)");
@@ -535,7 +559,7 @@ mr_status mr_group(mr_job* job) {
   for (int attempt = 0;; ++attempt) {
     // sentinel keys sort after every real key: the first m sorted positions are the real pairs
     CK(run_sort(job->sw, job->h.p, m_total, &job->skeys, &job->perm, job->st, job->nsm, job->stream, &job->prof,
-                &job->stats.hist_ms, &job->stats.sort_ms),
+                &job->stats.hist_ms, &job->stats.sort_ms, 0, static_cast<int>(job->key_bits / 8)),
        "radix sort");
     job->stats.sort_passes += job->sw.passes;
     Prof::Span sp2{};
@@ -582,8 +606,9 @@ mr_status mr_reduce(mr_job* job) {
     case MR_WORDCOUNT: {
       CK(job->counts.ensure(S + 1), "alloc counts");
       CK(job->worklist.ensure(m / 1024 + 64), "alloc worklist");
-      CK(launch_reduce_wc(job->seg_start.p, S, job->perm, job->v.p, job->ingested ? 8 : 4, job->counts.p,
-                          job->worklist.p, job->st, job->nsm, s),
+      CK(launch_reduce_wc(job->seg_start.p, S, job->skeys, job->perm, job->v.p,
+                          job->packed() ? 2 : (job->ingested ? 1 : 0), job->counts.p, job->worklist.p, job->st,
+                          job->nsm, s),
          "reduce wc");
       CK(job->val_off.ensure(S + 1), "alloc val offsets");
       CK(launch_iota_scaled(S, 8, job->val_off.p, s), "val offsets");
@@ -713,6 +738,7 @@ mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_byte
       job->h.release(); job->kref.release(); job->v.release(); job->cap = 0;
       CK(ensure_pairs(job, m + m / 8 + 4096), "grow intermediate");
       CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
+      CK(cudaMemsetAsync(job->sw.hist.p, 0, 8 * 256 * sizeof(uint32_t), job->stream), "zero hist");
       for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
       job->stats.replays += job->batches.size();
       CK(read_state(job), "replay (async)");

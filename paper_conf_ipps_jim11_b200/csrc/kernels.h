@@ -53,6 +53,8 @@ struct MapArgs {
   uint64_t* tile_bounds = nullptr;    // scratch: 2 u64 per tile
   uint64_t hash_seed = 0;
   uint32_t key_bits = 64;             // sort-key width of hashed / inline keys (48 or 64)
+  uint32_t* hist = nullptr;           // 8 x 256 digit histograms accumulated by the flushes
+  uint64_t vpack = 0;                 // WC: value (1) packed above the 48-bit key (1 << 48), or 0
   int grid = 0;                       // persistent CTAs (0 = one per SM)
 };
 
@@ -71,7 +73,8 @@ struct SortBufs {
   uint64_t cap = 0;
 };
 constexpr int kSortThreads = 256, kSortIPT = 16, kSortTile = kSortThreads * kSortIPT;
-cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int num_sms, cudaStream_t s);
+// histograms of digits [0, nd) (nd = key width / 8); hist must hold 8 x 256 u32
+cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int nd, int num_sms, cudaStream_t s);
 // one LSD pass on digit `digit`; idx_in == nullptr means the identity permutation
 cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
                             uint32_t* idx_out, uint64_t m, int digit, const uint32_t* bases,
@@ -79,15 +82,16 @@ cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uin
 
 // ---- segments ----
 // heads per sort tile + byte verification of hashed keys; counts[t] = heads in tile t
+// kmask: bits of the sorted word that form the key (packed WC values live above bit 48)
 cudaError_t launch_seg_count(const uint64_t* skeys, const uint32_t* perm, const uint64_t* kref, uint64_t m,
-                             uint32_t* counts, DevState* st, uint32_t key_bits, cudaStream_t s);
+                             uint32_t* counts, DevState* st, uint32_t key_bits, uint64_t kmask, cudaStream_t s);
 // exclusive scan of u64 (in-place allowed); writes total to *total if non-null
 cudaError_t launch_scan_u64(const uint64_t* in, uint64_t* out, uint64_t n, unsigned long long* total,
                             uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s);
 cudaError_t launch_scan_u32to64(const uint32_t* in, uint64_t* out, uint64_t n, unsigned long long* total,
                                 uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s);
 cudaError_t launch_seg_write(const uint64_t* skeys, uint64_t m, const uint64_t* tile_base, uint64_t* seg_start,
-                             cudaStream_t s);
+                             uint64_t kmask, cudaStream_t s);
 
 // ---- reduce + output assembly ----
 struct OutBufs {
@@ -98,9 +102,10 @@ cudaError_t launch_key_lengths(const uint64_t* seg_start, uint64_t nseg, const u
                                const uint64_t* kref, uint64_t* lens, cudaStream_t s);
 cudaError_t launch_key_copy(const uint64_t* seg_start, uint64_t nseg, const uint32_t* perm, const uint64_t* kref,
                             const uint64_t* key_off, uint8_t* keys, cudaStream_t s);
-cudaError_t launch_reduce_wc(const uint64_t* seg_start, uint64_t nseg, const uint32_t* perm, const uint8_t* v,
-                             int vbytes, uint64_t* counts, uint64_t* worklist, DevState* st, int num_sms,
-                             cudaStream_t s);
+// vmode 0: u32 values through perm, 1: u64 values through perm, 2: packed in skeys >> 48
+cudaError_t launch_reduce_wc(const uint64_t* seg_start, uint64_t nseg, const uint64_t* skeys, const uint32_t* perm,
+                             const uint8_t* v, int vmode, uint64_t* counts, uint64_t* worklist, DevState* st,
+                             int num_sms, cudaStream_t s);
 cudaError_t launch_reduce_km(const uint64_t* seg_start, uint64_t nseg, const uint64_t* skeys, const uint32_t* perm,
                              const uint8_t* v, double* sums, unsigned long long* cnts, uint32_t k,
                              uint64_t* worklist, DevState* st, int num_sms, cudaStream_t s);

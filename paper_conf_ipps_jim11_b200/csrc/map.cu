@@ -60,6 +60,9 @@ struct Cfg {
   // after the emission rounds (a lane-per-word hash inside the rounds diverges: with 7% long
   // words, 9 in 10 rounds would carry at least one).  <= 64 words of >= 8 bytes fit in 512 B.
   static constexpr int kHashQ = (W == kWC) ? 64 : 0;
+  // a6 fused into a5: the flush warp accumulates the LSD digit histograms of the keys it
+  // flushes (KM ids use 2 digits, text keys 8; StringMatch is not sorted)
+  static constexpr int kHistDigits = (W == kSM) ? 0 : (W == kKM) ? 2 : 8;
 };
 constexpr int kKmPts = kT / 32;                // 512 points per KM tile
 
@@ -103,7 +106,8 @@ struct Layout {
   static constexpr int bits = offs + kStages * kOffBytes;         // kStages x kBitBytes
   static constexpr int out = bits + kStages * kBitBytes;          // kNOut x Cfg<W>::kOutHalf
   static constexpr int hq = out + kNOut * Cfg<W>::kOutHalf;       // kNMap x kHashQ x 8 (WC)
-  static constexpr int cent = hq + kNMap * Cfg<W>::kHashQ * 8;    // KM centroids
+  static constexpr int hist = hq + kNMap * Cfg<W>::kHashQ * 8;    // kHistDigits x 256 x 4
+  static constexpr int cent = hist + Cfg<W>::kHistDigits * 1024;  // KM centroids
   static_assert(ready + kStages * 8 <= bytes, "header region overflow");
   static_assert(sizeof(OutCtl) <= hdr, "OutCtl overlaps the stage headers");
 };
@@ -141,6 +145,8 @@ struct Params {
   const uint8_t* off_end;  // end of the offsets array rounded DOWN to 16 B (aligned TMA limit)
   uint64_t hash_seed;
   uint32_t key_bits;       // sort-key width (48 or 64)
+  uint32_t* hist;          // global 8 x 256 digit histograms (accumulated; nullptr: not fused)
+  uint64_t vpack;          // WC: the emitted value packed above the 48-bit key
 };
 
 constexpr uint32_t kFull = 0xffffffffu;
@@ -435,6 +441,20 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         if constexpr (F::kKref) reinterpret_cast<uint64_t*>(half)[F::kCap + cnt0 + lane] = 0;
       }
     }
+    if constexpr (Cfg<W>::kHistDigits > 0) {
+      if (P.hist) {                                             // digit histograms (fused a6)
+        __syncwarp();
+        uint32_t* hs = reinterpret_cast<uint32_t*>(smem + Layout<W>::hist);
+        const uint64_t* kk = reinterpret_cast<const uint64_t*>(half);
+        const uint32_t nd = min(static_cast<uint32_t>(Cfg<W>::kHistDigits), P.key_bits / 8);
+        for (uint32_t i = lane; i < cnt; i += 32) {
+          const uint64_t key = kk[i];
+#pragma unroll
+          for (uint32_t d = 0; d < static_cast<uint32_t>(Cfg<W>::kHistDigits); ++d)
+            if (d < nd) atomicAdd(&hs[d * 256 + ((key >> (8 * d)) & 255u)], 1u);
+        }
+      }
+    }
     unsigned long long gb = 0;
     if (lane == 0 && cnt) {
       gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(cnt));  // ONE global atomic per flush
@@ -460,6 +480,14 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
     __syncwarp();
     if (lane == 0) mbar_arrive(&oc->done[h]);
     if (fin) break;
+  }
+  if constexpr (Cfg<W>::kHistDigits > 0) {
+    if (P.hist) {
+      __syncwarp();
+      const uint32_t* hs = reinterpret_cast<const uint32_t*>(smem + Layout<W>::hist);
+      for (uint32_t i = lane; i < Cfg<W>::kHistDigits * 256; i += 32)
+        if (hs[i]) atomicAdd(&P.hist[i], hs[i]);
+    }
   }
   if (lane == 0) {
     asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // global writes complete
@@ -733,7 +761,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
         uint32_t len = rest ? static_cast<uint32_t>(__ffs(rest)) : slow_word_len(P, tv, p, p0 + (lane < 31 ? 32 : 16));
         if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
         if (len <= inline_max(P.key_bits)) {
-          sh[idx] = inline_key(window8(x, j), len, P.key_bits);
+          sh[idx] = inline_key(window8(x, j), len, P.key_bits) | P.vpack;
         } else {                                      // hashed after the rounds, all lanes together
           queue = true;
           qe = static_cast<uint64_t>(idx) | (static_cast<uint64_t>(p - tv.sbase) << 16) |
@@ -766,7 +794,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
       const uint64_t e = hq[q];
       const uint32_t idx = static_cast<uint32_t>(e & 0xFFFF);
       const long long p = tv.sbase + static_cast<long long>((e >> 16) & 0xFFFFFF);
-      sh[idx] = key_at(P, tv, p, static_cast<uint32_t>(e >> 40));
+      sh[idx] = key_at(P, tv, p, static_cast<uint32_t>(e >> 40)) | P.vpack;
     }
   }
   commit(oc, slot, total);
@@ -894,6 +922,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_map(Params P) {
     for (int s = 0; s < kStages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], kNMap); mbar_init(&ready[s], 1); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  if constexpr (Cfg<W>::kHistDigits > 0) {
+    uint32_t* hs = reinterpret_cast<uint32_t*>(smem + Layout<W>::hist);
+    for (uint32_t i = threadIdx.x; i < Cfg<W>::kHistDigits * 256; i += blockDim.x) hs[i] = 0;
+  }
   if constexpr (W == kKM) {
     float* cent = reinterpret_cast<float*>(smem + Layout<W>::cent);
     // pair layout: centroids (2p, 2p+1) interleaved per coordinate -> f32x2 operands
@@ -960,6 +992,8 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
                         : nullptr;
   P.hash_seed = a.hash_seed;
   P.key_bits = a.key_bits;
+  P.hist = a.hist;
+  P.vpack = a.vpack;
   if (P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>((P.ntiles + 255) / 256);

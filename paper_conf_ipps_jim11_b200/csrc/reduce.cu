@@ -66,7 +66,8 @@ constexpr int kSegWarp = 32 * kSegIPT;   // positions per warp
 __global__ void __launch_bounds__(kSegThreads) k_seg_count(const uint64_t* __restrict__ sk,
                                                          const uint32_t* __restrict__ perm,
                                                          const uint64_t* __restrict__ kref, uint64_t m,
-                                                         uint32_t* counts, DevState* st, uint64_t hbit) {
+                                                         uint32_t* counts, DevState* st, uint64_t hbit,
+                                                         uint64_t kmask) {
   __shared__ uint32_t red[kSegThreads / 32];
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint64_t wbase = static_cast<uint64_t>(blockIdx.x) * kSegTile + static_cast<uint64_t>(warp) * kSegWarp;
@@ -81,7 +82,7 @@ __global__ void __launch_bounds__(kSegThreads) k_seg_count(const uint64_t* __res
     const uint64_t k = valid ? sk[i] : 0;
     uint64_t prev = __shfl_up_sync(0xffffffffu, k, 1);
     if (lane == 0) prev = carry_k;
-    const bool head = valid && (i == 0 || k != prev);
+    const bool head = valid && (i == 0 || ((k ^ prev) & kmask) != 0);
     heads += head ? 1u : 0u;
     // byte verification of equal hashed keys (C-3 #13): adjacent pairs inside an equal-hash run
     const bool hashed_run = valid && kref && (k & hbit) && !head;
@@ -111,7 +112,7 @@ __global__ void __launch_bounds__(kSegThreads) k_seg_count(const uint64_t* __res
 
 __global__ void __launch_bounds__(kSegThreads) k_seg_write(const uint64_t* __restrict__ sk, uint64_t m,
                                                          const uint64_t* __restrict__ tile_base,
-                                                         uint64_t* seg_start) {
+                                                         uint64_t* seg_start, uint64_t kmask) {
   __shared__ uint32_t wsum[kSegThreads / 32];
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint64_t wbase = static_cast<uint64_t>(blockIdx.x) * kSegTile + static_cast<uint64_t>(warp) * kSegWarp;
@@ -126,7 +127,7 @@ __global__ void __launch_bounds__(kSegThreads) k_seg_write(const uint64_t* __res
     const uint64_t k = valid ? sk[i] : 0;
     uint64_t prev = __shfl_up_sync(0xffffffffu, k, 1);
     if (lane == 0) prev = carry_k;
-    hm[j] = __ballot_sync(0xffffffffu, valid && (i == 0 || k != prev));
+    hm[j] = __ballot_sync(0xffffffffu, valid && (i == 0 || ((k ^ prev) & kmask) != 0));
     wcount += __popc(hm[j]);
     carry_k = __shfl_sync(0xffffffffu, k, 31);
   }
@@ -153,13 +154,24 @@ __global__ void __launch_bounds__(kSegThreads) k_seg_write(const uint64_t* __res
 // the long tail of the Zipf vocabulary) are summed by their own lane (TR, L181); medium ones
 // (<= kSmallWC) by the whole warp in turn; large ones become kLargeTile work items for the
 // block-level kernel below (BR).
-// Segment-size-aware WC reduce (values gathered through perm).  A warp takes 32 consecutive
+// Value of sorted position i: gathered through perm (u32 / u64 value arrays) or, for packed WC
+// pairs, read from the top 16 bits of the sorted 64-bit word itself (no gather at all).
+template <int kMode>   // 0: u32 v[perm[i]], 1: u64 v[perm[i]], 2: packed sk[i] >> 48
+__device__ __forceinline__ uint64_t val_at(const uint64_t* __restrict__ sk, const uint32_t* __restrict__ perm,
+                                           const void* __restrict__ v, uint64_t i) {
+  if constexpr (kMode == 2) return sk[i] >> 48;
+  else if constexpr (kMode == 1) return static_cast<const uint64_t*>(v)[perm[i]];
+  else return static_cast<const uint32_t*>(v)[perm[i]];
+}
+
+// Segment-size-aware WC reduce.  A warp takes 32 consecutive
 // segments: tiny ones (<= 32 pairs, the long tail of the Zipf vocabulary) are summed by their
 // own lane (TR, L181); medium ones (<= kSmallWC) by the whole warp in turn; large ones become
 // kLargeTile work items for the block-level kernel below (BR).
-template <typename V>
-__global__ void k_reduce_wc_small(const uint64_t* __restrict__ seg, uint64_t nseg, const uint32_t* __restrict__ perm,
-                                  const V* __restrict__ v, uint64_t* counts, uint64_t* worklist, DevState* st) {
+template <int kMode>
+__global__ void k_reduce_wc_small(const uint64_t* __restrict__ seg, uint64_t nseg, const uint64_t* __restrict__ sk,
+                                  const uint32_t* __restrict__ perm, const void* __restrict__ v, uint64_t* counts,
+                                  uint64_t* worklist, DevState* st) {
   const uint64_t gw = (blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x) >> 5;
   const uint64_t nw = (static_cast<uint64_t>(gridDim.x) * blockDim.x) >> 5;
   const uint32_t lane = threadIdx.x & 31;
@@ -170,7 +182,7 @@ __global__ void k_reduce_wc_small(const uint64_t* __restrict__ seg, uint64_t nse
     const uint64_t size = b - a;
     if (s < nseg && size <= 32) {                       // thread per key set
       uint64_t sum = 0;
-      for (uint64_t i = a; i < b; ++i) sum += v[perm[i]];
+      for (uint64_t i = a; i < b; ++i) sum += val_at<kMode>(sk, perm, v, i);
       counts[s] = sum;
     } else if (s < nseg && size > kSmallWC) {           // block-level work items
       counts[s] = 0;
@@ -185,16 +197,17 @@ __global__ void k_reduce_wc_small(const uint64_t* __restrict__ seg, uint64_t nse
       const uint64_t ma = __shfl_sync(0xffffffffu, a, L), mb = __shfl_sync(0xffffffffu, b, L);
       uint64_t sum = 0;
 #pragma unroll 4
-      for (uint64_t i = ma + lane; i < mb; i += 32) sum += v[perm[i]];
+      for (uint64_t i = ma + lane; i < mb; i += 32) sum += val_at<kMode>(sk, perm, v, i);
       sum = warp_sum_u64(sum);
       if (lane == 0) counts[s0 + L] = sum;
     }
   }
 }
 
-template <typename V>
+template <int kMode>
 __global__ void __launch_bounds__(256) k_reduce_wc_large(const uint64_t* __restrict__ seg,
-                                                       const uint32_t* __restrict__ perm, const V* __restrict__ v,
+                                                       const uint64_t* __restrict__ sk,
+                                                       const uint32_t* __restrict__ perm, const void* __restrict__ v,
                                                        uint64_t* counts, const uint64_t* __restrict__ worklist,
                                                        DevState* st) {
   __shared__ unsigned long long item;
@@ -209,7 +222,7 @@ __global__ void __launch_bounds__(256) k_reduce_wc_large(const uint64_t* __restr
     const uint64_t a = seg[s] + t * kLargeTile, b = min(seg[s + 1], a + kLargeTile);
     uint64_t sum = 0;
 #pragma unroll 8
-    for (uint64_t i = a + threadIdx.x; i < b; i += blockDim.x) sum += v[perm[i]];
+    for (uint64_t i = a + threadIdx.x; i < b; i += blockDim.x) sum += val_at<kMode>(sk, perm, v, i);
     sum = warp_sum_u64(sum);
     if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = sum;
     __syncthreads();
@@ -366,16 +379,17 @@ inline unsigned blocks_for(uint64_t n, unsigned t) { return static_cast<unsigned
 }  // namespace
 
 cudaError_t launch_seg_count(const uint64_t* skeys, const uint32_t* perm, const uint64_t* kref, uint64_t m,
-                             uint32_t* counts, DevState* st, uint32_t key_bits, cudaStream_t s) {
+                             uint32_t* counts, DevState* st, uint32_t key_bits, uint64_t kmask, cudaStream_t s) {
   if (m == 0) return cudaSuccess;
-  k_seg_count<<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, perm, kref, m, counts, st, hashed_bit(key_bits));
+  k_seg_count<<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, perm, kref, m, counts, st, hashed_bit(key_bits),
+                                                              kmask);
   count_launch();
   return cudaGetLastError();
 }
 cudaError_t launch_seg_write(const uint64_t* skeys, uint64_t m, const uint64_t* tile_base, uint64_t* seg_start,
-                             cudaStream_t s) {
+                             uint64_t kmask, cudaStream_t s) {
   if (m == 0) return cudaMemsetAsync(seg_start, 0, sizeof(uint64_t), s);
-  k_seg_write<<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, m, tile_base, seg_start);
+  k_seg_write<<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, m, tile_base, seg_start, kmask);
   count_launch();
   return cudaGetLastError();
 }
@@ -393,21 +407,22 @@ cudaError_t launch_key_copy(const uint64_t* seg_start, uint64_t nseg, const uint
   count_launch();
   return cudaGetLastError();
 }
-cudaError_t launch_reduce_wc(const uint64_t* seg_start, uint64_t nseg, const uint32_t* perm, const uint8_t* v,
-                             int vbytes, uint64_t* counts, uint64_t* worklist, DevState* st, int num_sms,
-                             cudaStream_t s) {
+cudaError_t launch_reduce_wc(const uint64_t* seg_start, uint64_t nseg, const uint64_t* skeys, const uint32_t* perm,
+                             const uint8_t* v, int vmode, uint64_t* counts, uint64_t* worklist, DevState* st,
+                             int num_sms, cudaStream_t s) {
   if (nseg == 0) return cudaSuccess;
   cudaError_t e = cudaMemsetAsync(&st->large_items, 0, 2 * sizeof(unsigned long long), s);
   if (e != cudaSuccess) return e;
   const unsigned g1 = static_cast<unsigned>(std::min<uint64_t>(blocks_for(nseg, 256), 148ULL * 32));
-  if (vbytes == 4) {
-    const uint32_t* v4 = reinterpret_cast<const uint32_t*>(v);
-    k_reduce_wc_small<uint32_t><<<g1, 256, 0, s>>>(seg_start, nseg, perm, v4, counts, worklist, st);
-    k_reduce_wc_large<uint32_t><<<num_sms * 4, 256, 0, s>>>(seg_start, perm, v4, counts, worklist, st);
+  if (vmode == 2) {
+    k_reduce_wc_small<2><<<g1, 256, 0, s>>>(seg_start, nseg, skeys, perm, v, counts, worklist, st);
+    k_reduce_wc_large<2><<<num_sms * 4, 256, 0, s>>>(seg_start, skeys, perm, v, counts, worklist, st);
+  } else if (vmode == 1) {
+    k_reduce_wc_small<1><<<g1, 256, 0, s>>>(seg_start, nseg, skeys, perm, v, counts, worklist, st);
+    k_reduce_wc_large<1><<<num_sms * 4, 256, 0, s>>>(seg_start, skeys, perm, v, counts, worklist, st);
   } else {
-    const uint64_t* v8 = reinterpret_cast<const uint64_t*>(v);
-    k_reduce_wc_small<uint64_t><<<g1, 256, 0, s>>>(seg_start, nseg, perm, v8, counts, worklist, st);
-    k_reduce_wc_large<uint64_t><<<num_sms * 4, 256, 0, s>>>(seg_start, perm, v8, counts, worklist, st);
+    k_reduce_wc_small<0><<<g1, 256, 0, s>>>(seg_start, nseg, skeys, perm, v, counts, worklist, st);
+    k_reduce_wc_large<0><<<num_sms * 4, 256, 0, s>>>(seg_start, skeys, perm, v, counts, worklist, st);
   }
   count_launch(2);
   return cudaGetLastError();

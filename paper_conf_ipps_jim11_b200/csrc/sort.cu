@@ -13,6 +13,7 @@
 //     scattered through SMEM so that global writes are contiguous runs per digit.
 // Look-back status words: [epoch:30 | kind:2 | value:32]; every launch uses a fresh epoch so
 // the status buffer never needs clearing.
+#include <algorithm>
 #include <cstdlib>
 
 #include "common.cuh"
@@ -27,18 +28,31 @@ __device__ __forceinline__ uint64_t pack_status(uint32_t epoch, uint32_t kind, u
   return (static_cast<uint64_t>(epoch) << 34) | (static_cast<uint64_t>(kind) << 32) | v;
 }
 
-__global__ void __launch_bounds__(256) k_hist(const uint64_t* __restrict__ keys, uint64_t m, uint32_t* hist) {
+// Digit histograms of the first nd digits (nd = key width / 8): one read of the keys, two keys
+// per 16-byte load, shared atomics into a per-block 8 x 256 table.
+__global__ void __launch_bounds__(256) k_hist(const uint64_t* __restrict__ keys, uint64_t m, uint32_t nd,
+                                            uint32_t* hist) {
   __shared__ uint32_t sh[8 * 256];
   for (int i = threadIdx.x; i < 8 * 256; i += blockDim.x) sh[i] = 0;
   __syncthreads();
   const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
-  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i < m; i += stride) {
-    const uint64_t k = __ldcs(keys + i);
+  const uint64_t m2 = m / 2;
+  const ulonglong2* k2 = reinterpret_cast<const ulonglong2*>(keys);
+  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i < m2; i += stride) {
+    const ulonglong2 kk = __ldcs(k2 + i);
 #pragma unroll
-    for (int d = 0; d < 8; ++d) atomicAdd(&sh[d * 256 + ((k >> (8 * d)) & 255u)], 1u);
+    for (uint32_t d = 0; d < 8; ++d) {
+      if (d >= nd) break;
+      atomicAdd(&sh[d * 256 + ((kk.x >> (8 * d)) & 255u)], 1u);
+      atomicAdd(&sh[d * 256 + ((kk.y >> (8 * d)) & 255u)], 1u);
+    }
+  }
+  if ((m & 1) && blockIdx.x == 0 && threadIdx.x == 0) {
+    const uint64_t k = keys[m - 1];
+    for (uint32_t d = 0; d < nd; ++d) atomicAdd(&sh[d * 256 + ((k >> (8 * d)) & 255u)], 1u);
   }
   __syncthreads();
-  for (int i = threadIdx.x; i < 8 * 256; i += blockDim.x)
+  for (int i = threadIdx.x; i < static_cast<int>(nd) * 256; i += blockDim.x)
     if (sh[i]) atomicAdd(&hist[i], sh[i]);
 }
 
@@ -271,11 +285,17 @@ __global__ void __launch_bounds__(kScanThreads) k_scan(const T* __restrict__ in,
 
 }  // namespace
 
-cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int num_sms, cudaStream_t s) {
+cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int nd, int num_sms, cudaStream_t s) {
   cudaError_t e = cudaMemsetAsync(hist, 0, 8 * 256 * sizeof(uint32_t), s);
   if (e != cudaSuccess || m == 0) return e;
-  uint64_t blocks = min(static_cast<uint64_t>(num_sms) * 4, (m + 255) / 256);
-  k_hist<<<static_cast<unsigned>(blocks), 256, 0, s>>>(keys, m, hist);
+  if (reinterpret_cast<uintptr_t>(keys) & 15u) {   // 16-B loads: peel one key off a misaligned start
+    k_hist<<<1, 32, 0, s>>>(keys, 1, static_cast<uint32_t>(nd), hist);
+    count_launch();
+    ++keys;
+    if (--m == 0) return cudaGetLastError();
+  }
+  uint64_t blocks = std::min<uint64_t>(static_cast<uint64_t>(num_sms) * 8, (m / 2 + 255) / 256 + 1);
+  k_hist<<<static_cast<unsigned>(blocks), 256, 0, s>>>(keys, m, static_cast<uint32_t>(nd), hist);
   count_launch();
   return cudaGetLastError();
 }
