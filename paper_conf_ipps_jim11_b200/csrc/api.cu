@@ -130,7 +130,7 @@ cudaError_t run_sort(SortWork& W, const uint64_t* keys, uint64_t m, const uint64
                      int key_digits = 8) {
   cudaError_t e;
   if ((e = W.ka.ensure(m)) || (e = W.kb.ensure(m)) || (e = W.ia.ensure(m)) || (e = W.ib.ensure(m))) return e;
-  const uint64_t tiles = (m + kSortTile - 1) / kSortTile;
+  const uint64_t tiles = (m + sort_tile() - 1) / sort_tile();
   const uint64_t need_status = std::max<uint64_t>(tiles * 256, 3 * ((m + 2047) / 2048) + 3);
   if (W.status.n < need_status) {
     if ((e = W.status.ensure(need_status))) return e;

@@ -72,7 +72,8 @@ struct SortBufs {
   uint32_t* bases = nullptr;   // 8 x 256 exclusive digit bases
   uint64_t cap = 0;
 };
-constexpr int kSortThreads = 256, kSortIPT = 16, kSortTile = kSortThreads * kSortIPT;
+constexpr int kSortThreads = 256;
+int sort_tile();   // keys per onesweep tile (tile shape chosen at start-up, BMR_SORT_CFG)
 // histograms of digits [0, nd) (nd = key width / 8); hist must hold 8 x 256 u32
 cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int nd, int num_sms, cudaStream_t s);
 // one LSD pass on digit `digit`; idx_in == nullptr means the identity permutation

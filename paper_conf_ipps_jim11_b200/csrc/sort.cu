@@ -56,9 +56,11 @@ __global__ void __launch_bounds__(256) k_hist(const uint64_t* __restrict__ keys,
     if (sh[i]) atomicAdd(&hist[i], sh[i]);
 }
 
+template <int IPT>
 struct SortSmem {
-  uint64_t keys[kSortTile];
-  uint32_t idx[kSortTile];
+  static constexpr int kTile = kSortThreads * IPT;
+  uint64_t keys[kTile];
+  uint32_t idx[kTile];
   uint32_t wcnt[kWarps][256];      // per-warp digit counters, then warp-exclusive offsets
   uint32_t hist[256];
   uint32_t dstart[256];
@@ -72,17 +74,19 @@ constexpr int kLookWindow = 4;   // predecessor status words fetched per look-ba
 // kVar bit 0: rank with one shared atomic per match group (1) or a read-modify-write of the
 // warp counter per step (0); bit 1: tile histogram by shared atomics before ranking, published
 // as an early aggregate (1), or summed from the warp counters after ranking (0).
-template <bool kFirst, int kVar>
-__global__ void __launch_bounds__(kSortThreads, 3) k_onesweep(const uint64_t* __restrict__ keys_in,
-                                                            const uint32_t* __restrict__ idx_in,
-                                                            uint64_t* __restrict__ keys_out,
-                                                            uint32_t* __restrict__ idx_out, uint64_t m,
-                                                            uint32_t shift, const uint32_t* __restrict__ bases,
-                                                            uint64_t* status, uint32_t epoch,
-                                                            unsigned int* tile_counter) {
+template <bool kFirst, int kVar, int IPT, int MINB>
+__global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t* __restrict__ keys_in,
+                                                               const uint32_t* __restrict__ idx_in,
+                                                               uint64_t* __restrict__ keys_out,
+                                                               uint32_t* __restrict__ idx_out, uint64_t m,
+                                                               uint32_t shift, const uint32_t* __restrict__ bases,
+                                                               uint64_t* status, uint32_t epoch,
+                                                               unsigned int* tile_counter) {
+  constexpr int kSortIPT = IPT;
+  constexpr int kSortTile = SortSmem<IPT>::kTile;
   constexpr bool kAtomicRank = (kVar & 1) != 0, kEarly = (kVar & 2) != 0;
   extern __shared__ __align__(16) uint8_t raw[];
-  SortSmem& S = *reinterpret_cast<SortSmem*>(raw);
+  SortSmem<IPT>& S = *reinterpret_cast<SortSmem<IPT>*>(raw);
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid == 0) S.tile = atomicAdd(tile_counter, 1u);
   for (uint32_t i = tid; i < kWarps * 256; i += kSortThreads) (&S.wcnt[0][0])[i] = 0;
@@ -307,36 +311,59 @@ int sort_variant() {
   }();
   return v;
 }
+// tile shape: 0 = 16 keys/thread, 3 CTAs/SM; 1 = 12 keys, 4 CTAs; 2 = 20 keys, 2 CTAs; 3 = 8 keys, 6 CTAs
+int sort_cfg() {
+  static int c = [] {
+    const char* e = getenv("BMR_SORT_CFG");
+    return e ? atoi(e) & 3 : 0;
+  }();
+  return c;
+}
+static const int kCfgIPT[4] = {16, 12, 20, 8};
+int sort_tile() { return kSortThreads * kCfgIPT[sort_cfg()]; }
 
-template <bool kFirst, int kVar>
-static void launch_os(unsigned tiles, size_t smem, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
+template <bool kFirst, int kVar, int IPT, int MINB>
+static void launch_os(unsigned tiles, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
                       uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
                       uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
-  cudaFuncSetAttribute(k_onesweep<kFirst, kVar>, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
-  k_onesweep<kFirst, kVar><<<tiles, kSortThreads, smem, s>>>(keys_in, idx_in, keys_out, idx_out, m, shift, bases,
-                                                             status, epoch, tile_counter);
+  const size_t smem = sizeof(SortSmem<IPT>);
+  cudaFuncSetAttribute(k_onesweep<kFirst, kVar, IPT, MINB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       static_cast<int>(smem));
+  k_onesweep<kFirst, kVar, IPT, MINB><<<tiles, kSortThreads, smem, s>>>(keys_in, idx_in, keys_out, idx_out, m, shift,
+                                                                         bases, status, epoch, tile_counter);
+}
+
+template <bool kFirst, int kVar>
+static void launch_cfg(unsigned tiles, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
+                       uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
+                       uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
+  switch (sort_cfg()) {
+    case 1: launch_os<kFirst, kVar, 12, 4>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch, tile_counter, s); break;
+    case 2: launch_os<kFirst, kVar, 20, 2>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch, tile_counter, s); break;
+    case 3: launch_os<kFirst, kVar, 8, 6>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch, tile_counter, s); break;
+    default: launch_os<kFirst, kVar, 16, 3>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch, tile_counter, s); break;
+  }
 }
 
 cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out, uint32_t* idx_out,
                             uint64_t m, int digit, const uint32_t* bases, uint64_t* status, uint32_t epoch,
                             unsigned int* tile_counter, cudaStream_t s) {
   if (m == 0) return cudaSuccess;
-  const unsigned tiles = static_cast<unsigned>((m + kSortTile - 1) / kSortTile);
-  const size_t smem = sizeof(SortSmem);
+  const unsigned tiles = static_cast<unsigned>((m + sort_tile() - 1) / sort_tile());
   cudaError_t e = cudaMemsetAsync(tile_counter, 0, sizeof(unsigned int), s);
   if (e != cudaSuccess) return e;
   const uint32_t shift = 8u * digit;
   const uint32_t* b = bases + 256 * digit;
   const bool first = idx_in == nullptr;
   switch (sort_variant() | (first ? 4 : 0)) {
-    case 0: launch_os<false, 0>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    case 1: launch_os<false, 1>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    case 2: launch_os<false, 2>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    case 3: launch_os<false, 3>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    case 4: launch_os<true, 0>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    case 5: launch_os<true, 1>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    case 6: launch_os<true, 2>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    default: launch_os<true, 3>(tiles, smem, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    case 0: launch_cfg<false, 0>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    case 1: launch_cfg<false, 1>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    case 2: launch_cfg<false, 2>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    case 3: launch_cfg<false, 3>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    case 4: launch_cfg<true, 0>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    case 5: launch_cfg<true, 1>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    case 6: launch_cfg<true, 2>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+    default: launch_cfg<true, 3>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
   }
   count_launch();
   return cudaGetLastError();
