@@ -124,13 +124,17 @@ int sm_count(int dev) {
 // `keys` + an identity permutation when every digit is constant).
 // hist_digits > 0: W.hist already holds the histograms of digits [0, hist_digits) (fused into
 // the Map flushes); the remaining digits are known to be constant zero.
+// out_perm == nullptr: keys only (no permutation payload is carried).
 cudaError_t run_sort(SortWork& W, const uint64_t* keys, uint64_t m, const uint64_t** out_keys,
                      const uint32_t** out_perm, DevState* st, int nsm, cudaStream_t s, Prof* prof = nullptr,
                      double* hist_ms = nullptr, double* pass_ms = nullptr, int hist_digits = 0,
                      int key_digits = 8) {
   cudaError_t e;
-  if ((e = W.ka.ensure(m)) || (e = W.kb.ensure(m)) || (e = W.ia.ensure(m)) || (e = W.ib.ensure(m))) return e;
-  const uint64_t tiles = (m + sort_tile() - 1) / sort_tile();
+  const bool pay = out_perm != nullptr;
+  if ((e = W.ka.ensure(m)) || (e = W.kb.ensure(m))) return e;
+  if (pay && ((e = W.ia.ensure(m)) || (e = W.ib.ensure(m)))) return e;
+  const uint64_t min_tile = std::min(sort_tile(), sort_tile_keys());
+  const uint64_t tiles = (m + min_tile - 1) / min_tile;
   const uint64_t need_status = std::max<uint64_t>(tiles * 256, 3 * ((m + 2047) / 2048) + 3);
   if (W.status.n < need_status) {
     if ((e = W.status.ensure(need_status))) return e;
@@ -167,8 +171,10 @@ cudaError_t run_sort(SortWork& W, const uint64_t* keys, uint64_t m, const uint64
   }
   W.passes = nd;
   if (nd == 0) {
-    k_iota_u32<<<static_cast<unsigned>((m + 255) / 256 + 1), 256, 0, s>>>(W.ia.p, m);
     *out_keys = keys;
+    if (!pay) return cudaSuccess;
+    k_iota_u32<<<static_cast<unsigned>((m + 255) / 256 + 1), 256, 0, s>>>(W.ia.p, m);
+    count_launch();
     *out_perm = W.ia.p;
     return cudaGetLastError();
   }
@@ -179,7 +185,7 @@ cudaError_t run_sort(SortWork& W, const uint64_t* keys, uint64_t m, const uint64
   if (prof && prof->on) prof->begin(s, sp2);
   for (int p = 0; p < nd; ++p) {
     uint64_t* kout = (p & 1) ? W.kb.p : W.ka.p;
-    uint32_t* iout = (p & 1) ? W.ib.p : W.ia.p;
+    uint32_t* iout = pay ? ((p & 1) ? W.ib.p : W.ia.p) : nullptr;
     if ((e = launch_onesweep(kin, iin, kout, iout, m, digits[p], W.bases.p, W.status.p, W.epoch++,
                              &st->tile_counter[0], s)))
       return e;
@@ -188,7 +194,7 @@ cudaError_t run_sort(SortWork& W, const uint64_t* keys, uint64_t m, const uint64
   }
   if (prof && prof->on) prof->end(s, sp2, pass_ms);
   *out_keys = kin;
-  *out_perm = iin;
+  if (pay) *out_perm = iin;
   return cudaSuccess;
 }
 
@@ -219,10 +225,18 @@ struct mr_job {
   size_t host_batches = 0;
   Prof prof;
   unsigned long long launches0 = 0;
-  SortWork sw;
+  SortWork sw, swb;
   const uint64_t* skeys = nullptr;
   const uint32_t* perm = nullptr;
   uint64_t m = 0, nseg = 0, key_bytes = 0;
+  // WC hashed stream (the exact stream uses h / skeys / seg_start): pairs, sorted, segments
+  DBuf<uint64_t> hb, krefb, seg_startb;
+  uint64_t cap_b = 0, mb = 0, nseg_a = 0, nseg_b = 0;
+  const uint64_t* skeysb = nullptr;
+  const uint32_t* permb = nullptr;
+  uint32_t key_bits_b = 48;
+  DBuf<uint64_t> scan_status;     // look-back words of the single-pass scans (epoch-tagged)
+  uint32_t scan_epoch = 1;
   DBuf<uint32_t> seg_counts;
   DBuf<uint64_t> tile_base, seg_start, key_off, val_off, counts, worklist, gathered;
   DBuf<uint8_t> keys_out, vals_out, vsorted;
@@ -234,9 +248,9 @@ struct mr_job {
   // multi-GPU exchange (§8(e))
   XSource xs;
   uint32_t key_bits = 64;         // current sort-key width (WC maps with 48; re-hash -> 64)
-  // WC map output with 48-bit keys carries its value in bits 48..63 of the sorted word
-  bool packed() const { return cfg.workload == MR_WORDCOUNT && key_bits == 48 && !ingested; }
-  uint64_t kmask() const { return key_bits == 48 ? ((1ULL << 48) - 1ULL) : ~0ULL; }
+  // WC Map output = exact stream + hashed stream (values 1, not stored); ingested WC pairs are
+  // one general stream (key, kref, u64 partial count) like II
+  bool split() const { return cfg.workload == MR_WORDCOUNT && !ingested; }
   bool ingested = false;          // pairs come from mr_ingest (WC values are u64 partial counts)
   bool km_partial = false;        // KM: sums/cnts hold ingested partials; finalise owned clusters
   int vb_cur = 0;                 // value bytes of the current pairs
@@ -276,14 +290,23 @@ uint64_t initial_cap(const mr_job* job, uint64_t nbytes, uint64_t n) {
   }
 }
 
-cudaError_t ensure_pairs(mr_job* job, uint64_t cap) {
+// cap_b: WC hashed-stream capacity (0 for the other workloads)
+cudaError_t ensure_pairs(mr_job* job, uint64_t cap, uint64_t cap_b) {
   cudaError_t e;
   if ((e = job->h.ensure(cap))) return e;
   if (has_kref(job->cfg.workload) && (e = job->kref.ensure(cap))) return e;
   const int vb = vbytes_of(job->cfg.workload);
   if (vb && (e = job->v.ensure(cap * vb))) return e;
   job->cap = cap;
+  if (cap_b) {
+    if ((e = job->hb.ensure(cap_b)) || (e = job->krefb.ensure(cap_b))) return e;
+  }
+  job->cap_b = cap_b;
   return cudaSuccess;
+}
+void release_pairs(mr_job* job) {
+  job->h.release(); job->kref.release(); job->v.release(); job->hb.release(); job->krefb.release();
+  job->cap = job->cap_b = 0;
 }
 
 cudaError_t launch_batch(mr_job* job, const Batch& b) {
@@ -303,12 +326,12 @@ cudaError_t launch_batch(mr_job* job, const Batch& b) {
   a.out.kref = job->kref.p;
   a.out.v = job->v.p;
   a.out.cap = job->cap;
+  a.out.hb = job->hb.p;
+  a.out.krefb = job->krefb.p;
+  a.out.cap_b = job->cap_b;
   a.st = job->st;
   a.hash_seed = 0x5EEDB200ULL;
   a.key_bits = job->key_bits;
-  a.hist = nullptr;   // flush-fused histograms measured slower (one flush warp, 6 atomics per pair)
-  // WC: the emitted value 1 rides in bits 48..63 of the sort word (the sort uses digits 0..5)
-  a.vpack = (job->cfg.workload == MR_WORDCOUNT && job->key_bits == 48) ? (1ULL << 48) : 0;
   const uint64_t nt = map_tiles(a);
   if (a.workload != kKM) {
     cudaError_t e = job->tb.ensure(2 * nt + 2);
@@ -325,23 +348,60 @@ cudaError_t read_state(mr_job* job) {
   return cudaStreamSynchronize(job->stream);
 }
 
-mr_status do_segments(mr_job* job) {
-  const uint64_t m = job->m;
+// Look-back workspace for a scan of n elements (k_scan: 2048 per tile, 3 words per tile).
+cudaError_t scan_ws(mr_job* job, uint64_t n, uint64_t** status, uint32_t* epoch) {
+  const uint64_t need = 3 * ((n + 2047) / 2048) + 3;
+  if (job->scan_status.n < need || !job->scan_status.p) {
+    cudaError_t e = job->scan_status.ensure(need);
+    if (e == cudaSuccess) e = cudaMemsetAsync(job->scan_status.p, 0, job->scan_status.n * 8, job->stream);
+    if (e != cudaSuccess) return e;
+  }
+  *status = job->scan_status.p;
+  *epoch = job->scan_epoch++;
+  return cudaSuccess;
+}
+
+// Segment heads of one sorted stream -> seg_start[0..nseg] (seg_start[nseg] = m).
+mr_status do_segments(mr_job* job, const uint64_t* skeys, const uint32_t* perm, const uint64_t* kref, uint64_t m,
+                      uint32_t key_bits, DBuf<uint64_t>& seg_start, uint64_t& nseg) {
   const uint64_t tiles = (m + 4095) / 4096;
   CK(job->seg_counts.ensure(tiles + 1), "alloc seg counts");
   CK(job->tile_base.ensure(tiles + 1), "alloc tile base");
   CK(cudaMemsetAsync(&job->st->collisions, 0, sizeof(unsigned int), job->stream), "memset");
-  const uint64_t* kref = has_kref(job->cfg.workload) ? job->kref.p : nullptr;
-  CK(launch_seg_count(job->skeys, job->perm, kref, m, job->seg_counts.p, job->st, job->key_bits, job->kmask(),
-                      job->stream),
-     "seg_count");
-  CK(launch_scan_u32to64(job->seg_counts.p, job->tile_base.p, tiles, &job->st->seg_total, job->sw.status.p,
-                         job->sw.epoch++, &job->st->tile_counter[1], job->stream),
+  CK(launch_seg_count(skeys, perm, kref, m, job->seg_counts.p, job->st, key_bits, ~0ULL, job->stream), "seg_count");
+  uint64_t* ss;
+  uint32_t ep;
+  CK(scan_ws(job, tiles, &ss, &ep), "alloc scan workspace");
+  CK(launch_scan_u32to64(job->seg_counts.p, job->tile_base.p, tiles, &job->st->seg_total, ss, ep,
+                         &job->st->tile_counter[1], job->stream),
      "scan tiles");
   CK(read_state(job), "sync segments");
-  job->nseg = m ? job->st_h.p->seg_total : 0;
-  CK(job->seg_start.ensure(job->nseg + 1), "alloc seg_start");
-  CK(launch_seg_write(job->skeys, m, job->tile_base.p, job->seg_start.p, job->kmask(), job->stream), "seg_write");
+  nseg = m ? job->st_h.p->seg_total : 0;
+  CK(seg_start.ensure(nseg + 1), "alloc seg_start");
+  CK(launch_seg_write(skeys, m, job->tile_base.p, seg_start.p, ~0ULL, job->stream), "seg_write");
+  return MR_OK;
+}
+
+// D7: settle the Map of every batch.  The cursors counted demand past capacity: grow the pair
+// buffers and replay every batch.  Leaves the final DevState in st_h.
+mr_status settle_map(mr_job* job) {
+  CK(read_state(job), "map (async)");
+  DevState* hs = job->st_h.p;
+  if (hs->err & kErrKeyTooLong) return fail(job, MR_ERR_OVERFLOW, "an emitted key exceeds 65535 bytes");
+  const uint64_t m = hs->pair_cursor, mb = job->split() ? hs->pair_cursor_b : 0;
+  if (m > job->cap || mb > job->cap_b) {
+    const uint64_t ncap = std::max(job->cap, m + m / 8 + 4096);
+    const uint64_t ncap_b = job->split() ? std::max(job->cap_b, mb + mb / 8 + 4096) : 0;
+    release_pairs(job);
+    CK(ensure_pairs(job, ncap, ncap_b), "grow intermediate");
+    job->stats.capacity_pairs = job->cap + job->cap_b;
+    CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
+    for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
+    job->stats.replays += job->batches.size();
+    CK(read_state(job), "replay (async)");
+    if (hs->pair_cursor > job->cap || (job->split() && hs->pair_cursor_b > job->cap_b))
+      return fail(job, MR_ERR_OOM, "replay still overflows");
+  }
   return MR_OK;
 }
 
@@ -433,6 +493,10 @@ mr_status mr_job_reset(mr_job* job) {
   job->ingested = false;
   job->km_partial = false;
   job->key_bits = (job->cfg.workload == MR_WORDCOUNT) ? 48u : 64u;
+  job->key_bits_b = 48;
+  job->mb = job->nseg_a = job->nseg_b = 0;
+  job->skeysb = nullptr;
+  job->permb = nullptr;
   job->prof.collect();
   job->batches.clear();
   job->next_base = 0;
@@ -444,7 +508,6 @@ mr_status mr_job_reset(mr_job* job) {
   job->stats.capacity_pairs = cap;
   job->launches0 = g_kernel_launches.load();
   CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset state");
-  if (job->sw.hist.p) CK(cudaMemsetAsync(job->sw.hist.p, 0, 8 * 256 * sizeof(uint32_t), job->stream), "zero hist");
   job->state = kCreated;
   return MR_OK;
 }
@@ -474,12 +537,11 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
   }
   if (nbytes && !records) return fail(job, MR_ERR_INVALID, "records is NULL");
   if (job->cap == 0) {
-    CK(ensure_pairs(job, initial_cap(job, nbytes, n)), "alloc intermediate");
-    job->stats.capacity_pairs = job->cap;
-  }
-  if (!job->sw.hist.p) {                      // digit histograms accumulated by the Map flushes
-    CK(job->sw.hist.ensure(8 * 256), "alloc histogram");
-    CK(cudaMemsetAsync(job->sw.hist.p, 0, 8 * 256 * sizeof(uint32_t), job->stream), "zero histogram");
+    // WC: ~1 word per 6 bytes, a few % of them longer than 7 bytes (hashed stream)
+    const uint64_t cap_b = job->cfg.workload != MR_WORDCOUNT ? 0
+                           : job->cfg.max_pairs_hint ? job->cfg.max_pairs_hint : nbytes / 24 + 4096;
+    CK(ensure_pairs(job, initial_cap(job, nbytes, n), cap_b), "alloc intermediate");
+    job->stats.capacity_pairs = job->cap + job->cap_b;
   }
   Batch b{records, offsets, n, nbytes, job->cfg.input_base + job->next_base};
   job->next_base += nbytes;
@@ -527,63 +589,98 @@ mr_status mr_group(mr_job* job) {
     job->state = kGrouped;
     return MR_OK;
   }
-  CK(read_state(job), "map (async)");
+  mr_status st = settle_map(job);
+  if (st != MR_OK) return st;
   DevState* hs = job->st_h.p;
-  if (hs->err & kErrKeyTooLong) return fail(job, MR_ERR_OVERFLOW, "an emitted key exceeds 65535 bytes");
-  uint64_t m = hs->pair_cursor;
-  if (m > job->cap) {
-    // D7: the cursor counted demand past capacity -> grow and replay every batch
-    const uint64_t ncap = m + m / 8 + 4096;
-    job->h.release(); job->kref.release(); job->v.release(); job->cap = 0;
-    CK(ensure_pairs(job, ncap), "grow intermediate");
-    job->stats.capacity_pairs = job->cap;
-    CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
-    CK(cudaMemsetAsync(job->sw.hist.p, 0, 8 * 256 * sizeof(uint32_t), job->stream), "zero hist");
-    for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
-    job->stats.replays += job->batches.size();
-    CK(read_state(job), "replay (async)");
-    m = hs->pair_cursor;
-    if (m > job->cap) return fail(job, MR_ERR_OOM, "replay still overflows");
-  }
-  const uint64_t m_total = m;            // includes the flush filler pairs (sentinel keys)
-  m -= hs->pads;
+  const bool split = job->split();
+  const uint64_t m_total = hs->pair_cursor;            // includes the flush filler pairs (sentinel keys)
+  const uint64_t m = m_total - hs->pads;
+  const uint64_t mb = split ? hs->pair_cursor_b : 0;
   job->m = m;
-  job->stats.pairs = m;
+  job->mb = mb;
+  job->stats.pairs = m + mb;
+  job->stats.pairs_hashed = mb;
   job->stats.flushes = hs->flushes;
-  if (m_total >= (1ULL << 32) - 1) return fail(job, MR_ERR_UNSUPPORTED, ">= 2^32 intermediate pairs in one group");
+  if (m_total >= (1ULL << 32) - 1 || mb >= (1ULL << 32) - 1)
+    return fail(job, MR_ERR_UNSUPPORTED, ">= 2^32 intermediate pairs in one group");
   if (job->cfg.workload == MR_STRINGMATCH) {  // Map-only
     job->nseg = m;
     job->state = kGrouped;
     return MR_OK;
   }
-  for (int attempt = 0;; ++attempt) {
-    // sentinel keys sort after every real key: the first m sorted positions are the real pairs
-    CK(run_sort(job->sw, job->h.p, m_total, &job->skeys, &job->perm, job->st, job->nsm, job->stream, &job->prof,
-                &job->stats.hist_ms, &job->stats.sort_ms, 0, static_cast<int>(job->key_bits / 8)),
-       "radix sort");
+  job->nseg_b = 0;
+  job->skeysb = nullptr;
+  job->permb = nullptr;
+  if (split) {
+    // exact stream: keys only (the key is the record), no byte verification needed
+    CK(run_sort(job->sw, job->h.p, m_total, &job->skeys, nullptr, job->st, job->nsm, job->stream, &job->prof,
+                &job->stats.hist_ms, &job->stats.sort_keys_ms, 0, 6),
+       "radix sort (exact)");
     job->stats.sort_passes += job->sw.passes;
-    Prof::Span sp2{};
-    if (job->prof.on) job->prof.begin(job->stream, sp2);
-    mr_status s = do_segments(job);
-    if (s != MR_OK) return s;
-    if (job->prof.on) job->prof.end(job->stream, sp2, &job->stats.seg_ms);
-    const uint32_t coll = hs->collisions;
-    if (coll == 0) break;
-    job->stats.collisions += coll;
-    if (attempt >= 3) return fail(job, MR_ERR_UNSUPPORTED, "unresolvable 64-bit hash collision");
-    // slow path: recompute every hashed key with a fresh full-width hash, then sort again
-    CK(launch_rehash(job->h.p, job->kref.p, m_total, 0xC0111DE5ULL + attempt, job->stream), "rehash");
-    job->key_bits = 64;
+    job->stats.sort_passes_keys += job->sw.passes;
+    job->perm = nullptr;
+    Prof::Span sp{};
+    if (job->prof.on) job->prof.begin(job->stream, sp);
+    st = do_segments(job, job->skeys, nullptr, nullptr, m, 48, job->seg_start, job->nseg_a);
+    if (st != MR_OK) return st;
+    if (job->prof.on) job->prof.end(job->stream, sp, &job->stats.seg_ms);
   }
+  // general stream (II / KM / ingested WC) or the WC hashed stream: sort with the permutation,
+  // verify equal hashes byte for byte, re-hash and re-sort on a collision (slow path)
+  {
+    uint64_t* keys = split ? job->hb.p : job->h.p;
+    const uint64_t* kref = split ? job->krefb.p : (has_kref(job->cfg.workload) || job->ingested ? job->kref.p : nullptr);
+    const uint64_t n = split ? mb : m_total;
+    const uint64_t nreal = split ? mb : m;
+    uint32_t& kbits = split ? job->key_bits_b : job->key_bits;
+    SortWork& W = split ? job->swb : job->sw;
+    const uint64_t** sk = split ? &job->skeysb : &job->skeys;
+    const uint32_t** pm = split ? &job->permb : &job->perm;
+    DBuf<uint64_t>& seg = split ? job->seg_startb : job->seg_start;
+    uint64_t& ns = split ? job->nseg_b : job->nseg_a;
+    for (int attempt = 0;; ++attempt) {
+      // sentinel keys sort after every real key: the first nreal sorted positions are the real pairs
+      CK(run_sort(W, keys, n, sk, pm, job->st, job->nsm, job->stream, &job->prof, &job->stats.hist_ms,
+                  &job->stats.sort_ms, 0, static_cast<int>(kbits / 8)),
+         "radix sort");
+      job->stats.sort_passes += W.passes;
+      Prof::Span sp2{};
+      if (job->prof.on) job->prof.begin(job->stream, sp2);
+      st = do_segments(job, *sk, *pm, kref, nreal, kbits, seg, ns);
+      if (st != MR_OK) return st;
+      if (job->prof.on) job->prof.end(job->stream, sp2, &job->stats.seg_ms);
+      const uint32_t coll = hs->collisions;
+      if (coll == 0) break;
+      job->stats.collisions += coll;
+      if (attempt >= 3) return fail(job, MR_ERR_UNSUPPORTED, "unresolvable 64-bit hash collision");
+      // slow path: recompute every hashed key with a fresh full-width hash, then sort again
+      CK(launch_rehash(keys, kref, n, 0xC0111DE5ULL + attempt, job->stream), "rehash");
+      kbits = 64;
+    }
+    if (!split) { job->nseg_a = ns; }
+  }
+  job->nseg = job->nseg_a + job->nseg_b;
   job->stats.n_keys = job->nseg;
   Prof::Span sp3{};
   if (job->prof.on) job->prof.begin(job->stream, sp3);
   if (job->cfg.workload == MR_WORDCOUNT || job->cfg.workload == MR_INVINDEX) {
     CK(job->key_off.ensure(job->nseg + 1), "alloc key offsets");
-    CK(launch_key_lengths(job->seg_start.p, job->nseg, job->perm, job->kref.p, job->key_off.p, job->stream), "key lengths");
+    if (split) {
+      CK(launch_key_lengths_exact(job->seg_start.p, job->nseg_a, job->skeys, job->key_off.p, job->stream),
+         "key lengths (exact)");
+      CK(launch_key_lengths(job->seg_startb.p, job->nseg_b, job->permb, job->krefb.p, job->key_off.p + job->nseg_a,
+                            job->stream),
+         "key lengths (hashed)");
+    } else {
+      CK(launch_key_lengths(job->seg_start.p, job->nseg, job->perm, job->kref.p, job->key_off.p, job->stream),
+         "key lengths");
+    }
+    uint64_t* ss;
+    uint32_t ep;
+    CK(scan_ws(job, job->nseg, &ss, &ep), "alloc scan workspace");
     CK(launch_scan_u64(job->key_off.p, job->key_off.p, job->nseg,
-                       reinterpret_cast<unsigned long long*>(job->key_off.p + job->nseg), job->sw.status.p,
-                       job->sw.epoch++, &job->st->tile_counter[2], job->stream),
+                       reinterpret_cast<unsigned long long*>(job->key_off.p + job->nseg), ss, ep,
+                       &job->st->tile_counter[2], job->stream),
        "scan key lengths");
     CK(cudaMemcpyAsync(job->tmp_h.p, job->key_off.p + job->nseg, 8, cudaMemcpyDeviceToHost, job->stream), "read key bytes");
     CK(cudaStreamSynchronize(job->stream), "sync key bytes");
@@ -605,15 +702,27 @@ mr_status mr_reduce(mr_job* job) {
   switch (job->cfg.workload) {
     case MR_WORDCOUNT: {
       CK(job->counts.ensure(S + 1), "alloc counts");
-      CK(job->worklist.ensure(m / 1024 + 64), "alloc worklist");
-      CK(launch_reduce_wc(job->seg_start.p, S, job->skeys, job->perm, job->v.p,
-                          job->packed() ? 2 : (job->ingested ? 1 : 0), job->counts.p, job->worklist.p, job->st,
-                          job->nsm, s),
-         "reduce wc");
+      CK(job->keys_out.ensure(job->key_bytes + 1), "alloc keys");
+      if (job->split()) {
+        // every Map value is 1: a key's count is its segment length (exact stream first, then
+        // the hashed stream; the output order is the sorted order of each stream)
+        CK(launch_seg_lengths(job->seg_start.p, job->nseg_a, job->counts.p, s), "counts (exact)");
+        CK(launch_seg_lengths(job->seg_startb.p, job->nseg_b, job->counts.p + job->nseg_a, s), "counts (hashed)");
+        CK(launch_key_decode(job->seg_start.p, job->nseg_a, job->skeys, job->key_off.p, job->keys_out.p, s),
+           "key decode");
+        CK(launch_key_copy(job->seg_startb.p, job->nseg_b, job->permb, job->krefb.p, job->key_off.p + job->nseg_a,
+                           job->keys_out.p, s),
+           "key copy");
+      } else {
+        CK(job->worklist.ensure(m / 1024 + 64), "alloc worklist");
+        CK(launch_reduce_wc(job->seg_start.p, S, job->skeys, job->perm, job->v.p, 1, job->counts.p, job->worklist.p,
+                            job->st, job->nsm, s),
+           "reduce wc");
+        CK(launch_key_copy(job->seg_start.p, S, job->perm, job->kref.p, job->key_off.p, job->keys_out.p, s),
+           "key copy");
+      }
       CK(job->val_off.ensure(S + 1), "alloc val offsets");
       CK(launch_iota_scaled(S, 8, job->val_off.p, s), "val offsets");
-      CK(job->keys_out.ensure(job->key_bytes + 1), "alloc keys");
-      CK(launch_key_copy(job->seg_start.p, S, job->perm, job->kref.p, job->key_off.p, job->keys_out.p, s), "key copy");
       job->out_n = S;
       job->out_keys_bytes = job->key_bytes;
       job->out_vals_bytes = S * 8;
@@ -730,27 +839,26 @@ mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_byte
     }
   } else {
     // raw pairs: settle the Map (capacity check / replay) without grouping
-    CK(read_state(job), "map (async)");
+    mr_status st = settle_map(job);
+    if (st != MR_OK) return st;
     DevState* hs = job->st_h.p;
-    if (hs->err & kErrKeyTooLong) return fail(job, MR_ERR_OVERFLOW, "an emitted key exceeds 65535 bytes");
-    uint64_t m = hs->pair_cursor;
-    if (m > job->cap) {
-      job->h.release(); job->kref.release(); job->v.release(); job->cap = 0;
-      CK(ensure_pairs(job, m + m / 8 + 4096), "grow intermediate");
-      CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
-      CK(cudaMemsetAsync(job->sw.hist.p, 0, 8 * 256 * sizeof(uint32_t), job->stream), "zero hist");
-      for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
-      job->stats.replays += job->batches.size();
-      CK(read_state(job), "replay (async)");
-      m = hs->pair_cursor;
-    }
+    const uint64_t m = hs->pair_cursor;
     job->m = m - hs->pads;
-    job->stats.pairs = m - hs->pads;
-    xs.mode = kXPairs;
-    xs.n = m;
-    xs.kref = job->kref.p;
-    xs.v = job->v.p;
-    xs.vbytes = vbytes_of(w);
+    job->mb = job->split() ? hs->pair_cursor_b : 0;
+    job->stats.pairs = job->m + job->mb;
+    if (job->split()) {
+      xs.mode = kXSplit;
+      xs.hx = job->h.p;
+      xs.nx = m;
+      xs.n = m + job->mb;
+      xs.kref = job->krefb.p;
+    } else {
+      xs.mode = kXPairs;
+      xs.n = m;
+      xs.kref = job->kref.p;
+      xs.v = job->v.p;
+      xs.vbytes = vbytes_of(w);
+    }
   }
   CK(job->xcounts.ensure(2 * R), "alloc counts");
   CK(job->xcursors.ensure(2 * R), "alloc cursors");
@@ -825,8 +933,8 @@ mr_status mr_ingest(mr_job* job, const void* entries, const void* heap, const ui
     job->state = kMapped;
     return MR_OK;
   }
-  if (n > job->cap || job->v.n < n * 8) {
-    job->h.release(); job->kref.release(); job->v.release(); job->cap = 0;
+  if (n > job->cap || job->v.n < n * 8 || job->kref.n < n) {
+    release_pairs(job);
     CK(job->h.ensure(n + 1), "alloc pairs");
     CK(job->kref.ensure(n + 1), "alloc pairs");
     CK(job->v.ensure((n + 1) * 8), "alloc pairs");
@@ -853,6 +961,7 @@ mr_status mr_get_stats(const mr_job* job, void* stats, size_t bytes) {
   if (!job || !stats) return MR_ERR_INVALID;
   mr_stats st = job->stats;
   st.kernel_launches = g_kernel_launches.load() - job->launches0;
+  st.sort_ms += st.sort_keys_ms;   // sort_ms covers both streams
   std::memcpy(stats, &st, std::min(bytes, sizeof(mr_stats)));
   return MR_OK;
 }
@@ -867,8 +976,8 @@ mr_status mr_job_destroy(mr_job* job) {
   job->prof.release();
   job->xcounts.release(); job->xcursors.release(); job->xheapbase.release(); job->xcounts_h.release();
   job->src_e.release(); job->src_h.release(); job->km_list.release();
-  job->cent.release(); job->h.release(); job->kref.release(); job->tb.release(); job->v.release();
-  job->sw.release();
+  job->cent.release(); release_pairs(job); job->tb.release();
+  job->sw.release(); job->swb.release(); job->seg_startb.release(); job->scan_status.release();
   job->seg_counts.release(); job->tile_base.release(); job->seg_start.release(); job->key_off.release();
   job->val_off.release(); job->counts.release(); job->worklist.release(); job->gathered.release();
   job->keys_out.release(); job->vals_out.release(); job->vsorted.release(); job->sums.release(); job->cnts.release();

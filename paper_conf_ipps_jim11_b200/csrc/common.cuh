@@ -142,6 +142,7 @@ __device__ __forceinline__ uint64_t hash_bytes(const uint8_t* p, uint32_t len, u
 // passes fewer; digits 6 and 7 are then constant and skipped):
 //   inline  : keys of <= kInlineMax bytes packed little-endian, length in the 3 bits above them
 //             (64: len << 56, <= 7 bytes; 48: len << 40, <= 5 bytes) — injective, top bit clear;
+//   alnum   : (48 only) [0-9A-Za-z] keys of 6..7 bytes, 6-bit symbol codes, len << 43;
 //   hashed  : longer keys -> hash with the top bit of the width forced to 1 (never collides with
 //             an inline key); equal hashes are verified byte-for-byte at segment time;
 //   sentinel: all ones in the width — flush filler pairs, sorts after every real key.
@@ -160,13 +161,54 @@ __device__ __forceinline__ uint64_t hashed_key(uint64_t h, bool weak, uint32_t b
 __device__ __forceinline__ uint64_t inline_key(uint64_t bytes_le, uint32_t len, uint32_t bits = 64) {
   return (bytes_le & ((1ULL << (8 * len)) - 1ULL)) | (static_cast<uint64_t>(len) << (bits - 8));
 }
+// 48-bit (WordCount) keys of 6..7 bytes: a WC word is [0-9A-Za-z]+ (C-3 #1), so each symbol
+// has a 6-bit code (1..62) and 7 symbols (42 bits) plus the length at bits 43..45 pack
+// injectively — disjoint from the byte-packed keys (< 2^43) and the hashed ones (bit 47).
+__device__ __forceinline__ bool alnum_byte(uint32_t c) {
+  return (c - '0' < 10u) || (c - 'A' < 26u) || (c - 'a' < 26u);
+}
+__device__ __forceinline__ uint64_t alnum_key48(uint64_t bytes_le, uint32_t len) {
+  // SWAR: per byte code = c - 47 - 7 [c > '9'] - 6 [c > 'Z'], then bytes beyond len cleared and
+  // the eight 6-bit codes compressed (byte -> 12-bit pairs -> 24-bit quads -> 48 bits).
+  const auto codes = [](uint32_t w) {
+    const uint32_t g9 = __vcmpgtu4(w, 0x39393939u) & 0x07070707u;
+    const uint32_t gz = __vcmpgtu4(w, 0x5A5A5A5Au) & 0x06060606u;
+    return __vsub4(__vsub4(__vsub4(w, 0x2F2F2F2Fu), g9), gz);
+  };
+  uint64_t x = (static_cast<uint64_t>(codes(static_cast<uint32_t>(bytes_le >> 32))) << 32) |
+               codes(static_cast<uint32_t>(bytes_le));
+  x &= (1ULL << (8 * len)) - 1ULL;  // len <= 7
+  x = (x & 0x003F003F003F003FULL) | ((x >> 2) & 0x0FC00FC00FC00FC0ULL);
+  x = (x & 0x00000FFF00000FFFULL) | ((x >> 4) & 0x00FFF00000FFF000ULL);
+  x = (x & 0x0000000000FFFFFFULL) | ((x >> 8) & 0x0000FFFFFF000000ULL);
+  return x | (static_cast<uint64_t>(len) << 43);
+}
+// Inverse of the 48-bit exact formats (inline <= 5 bytes, alnum 6..7): key bytes little-endian.
+__device__ __forceinline__ uint64_t exact_key_bytes48(uint64_t key, uint32_t& len) {
+  if (key < (1ULL << 43)) {
+    len = static_cast<uint32_t>(key >> 40) & 7u;
+    return key & ((1ULL << 40) - 1ULL);
+  }
+  len = static_cast<uint32_t>(key >> 43) & 7u;
+  uint64_t b = 0;
+  for (uint32_t i = 0; i < len; ++i) {
+    const uint32_t c = static_cast<uint32_t>(key >> (6 * i)) & 63u;
+    b |= static_cast<uint64_t>(c <= 10 ? c + 47u : (c <= 36 ? c + 54u : c + 60u)) << (8 * i);
+  }
+  return b;
+}
 // key bytes -> sort key (generic pointer)
 __device__ __forceinline__ uint64_t key_of_bytes(const uint8_t* p, uint32_t len, uint64_t seed, bool weak,
                                                  uint32_t bits) {
-  if (len <= inline_max(bits)) {
+  if (len <= inline_max(bits) || (bits == 48 && len <= 7)) {
     uint64_t b = 0;
-    for (uint32_t k = 0; k < len; ++k) b |= static_cast<uint64_t>(p[k]) << (8 * k);
-    return inline_key(b, len, bits);
+    bool alnum = true;
+    for (uint32_t k = 0; k < len; ++k) {
+      b |= static_cast<uint64_t>(p[k]) << (8 * k);
+      alnum = alnum && alnum_byte(p[k]);
+    }
+    if (len <= inline_max(bits)) return inline_key(b, len, bits);
+    if (alnum) return alnum_key48(b, len);
   }
   return hashed_key(hash_bytes(p, len, seed), weak, bits);
 }

@@ -28,18 +28,35 @@ __device__ __forceinline__ uint32_t dest_of_id(uint64_t id, uint32_t R) {
   return static_cast<uint32_t>(mix64(id ^ kPartSeed) % R);
 }
 
-// Record i of the source: key bytes (ptr, len), value, destination, heap bytes.
+// Record i of the source: key bytes (ptr, len — or inline bytes), value, destination, heap bytes.
 struct Rec {
   const uint8_t* kp;
+  uint64_t kin;   // key bytes of an exact WC key (kp == nullptr)
   uint32_t klen;
   uint64_t v;
   uint32_t dest;
   uint32_t heap;  // bytes in the heap (key length rounded up to 8)
+  __device__ __forceinline__ uint8_t byte(uint32_t k) const {
+    return kp ? kp[k] : static_cast<uint8_t>(kin >> (8 * k));
+  }
 };
 
 __device__ __forceinline__ Rec get_rec(const XSource& S, uint64_t i) {
   Rec r{};
-  if (S.mode == kXPairs) {
+  if (S.mode == kXSplit) {           // WC Map output: exact stream, then hashed stream; value 1
+    r.v = 1;
+    if (i < S.nx) {
+      const uint64_t key = S.hx[i];
+      if (key == sentinel_of(48)) { r.dest = ~0u; return r; }   // flush filler
+      r.kin = exact_key_bytes48(key, r.klen);
+      r.dest = dest_of_bytes(reinterpret_cast<const uint8_t*>(&r.kin), r.klen, S.nranks);
+      r.heap = (r.klen + 7u) & ~7u;
+      return r;
+    }
+    const uint64_t kr = S.kref[i - S.nx];
+    r.kp = reinterpret_cast<const uint8_t*>(kr >> 16);
+    r.klen = static_cast<uint32_t>(kr & 0xFFFF);
+  } else if (S.mode == kXPairs) {
     const uint64_t kr = S.kref[i];   // 0 = flush filler (sentinel) pair: not a record
     if (kr == 0) { r.dest = ~0u; return r; }
     r.kp = reinterpret_cast<const uint8_t*>(kr >> 16);
@@ -120,7 +137,7 @@ __global__ void __launch_bounds__(kXThreads) k_x_scatter(XSource S, unsigned lon
   o->koff_len = ((hoff - S.heap_base[r.dest]) << 16) | r.klen;
   o->v = r.v;
   uint8_t* hp = heap + hoff;
-  for (uint32_t k = 0; k < r.klen; ++k) hp[k] = r.kp[k];
+  for (uint32_t k = 0; k < r.klen; ++k) hp[k] = r.byte(k);
 }
 
 // Received entries -> SoA pairs.  src_e / src_h: exclusive prefixes (R + 1) of the entries /

@@ -25,15 +25,21 @@ struct DevState {
   unsigned long long large_done;   // work-list cursor for the persistent large-segment kernel
   unsigned int tile_counter[32];   // dynamic tile ids of the look-back kernels (one per launch slot)
   unsigned long long pads;         // sentinel filler pairs written by the flushes (sort last, excluded)
+  unsigned long long pair_cursor_b;  // WC hashed stream: demand in pairs
 };
 constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u;
 
 // Intermediate pairs, SoA in HBM (SURVEY §8(a) layout): sort key, key reference, value.
+// WordCount Map output is two streams: exact keys (h only: the key is the record, value 1) and
+// hashed keys (hb + krefb); see map.cu.
 struct PairBufs {
   uint64_t* h = nullptr;     // 64-bit sort key (inline key / hash / SM offset / KM id)
   uint64_t* kref = nullptr;  // (device address of key bytes << 16) | key length
   uint8_t* v = nullptr;      // value bytes (vbytes per pair)
   uint64_t cap = 0;          // capacity in pairs
+  uint64_t* hb = nullptr;    // WC hashed stream: keys, key references, capacity
+  uint64_t* krefb = nullptr;
+  uint64_t cap_b = 0;
 };
 
 struct MapArgs {
@@ -53,12 +59,10 @@ struct MapArgs {
   uint64_t* tile_bounds = nullptr;    // scratch: 2 u64 per tile
   uint64_t hash_seed = 0;
   uint32_t key_bits = 64;             // sort-key width of hashed / inline keys (48 or 64)
-  uint32_t* hist = nullptr;           // 8 x 256 digit histograms accumulated by the flushes
-  uint64_t vpack = 0;                 // WC: value (1) packed above the 48-bit key (1 << 48), or 0
   int grid = 0;                       // persistent CTAs (0 = one per SM)
 };
 
-int vbytes_of(int workload);                 // value bytes per pair
+int vbytes_of(int workload);                 // value bytes per pair (WC Map output: none, value 1)
 bool has_kref(int workload);
 uint64_t map_tiles(const MapArgs& a);        // number of tiles of a batch
 cudaError_t launch_map(const MapArgs& a, int num_sms, cudaStream_t s);
@@ -74,9 +78,11 @@ struct SortBufs {
 };
 constexpr int kSortThreads = 256;
 int sort_tile();   // keys per onesweep tile (tile shape chosen at start-up, BMR_SORT_CFG)
+int sort_tile_keys();   // the same for the keys-only passes
 // histograms of digits [0, nd) (nd = key width / 8); hist must hold 8 x 256 u32
 cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int nd, int num_sms, cudaStream_t s);
-// one LSD pass on digit `digit`; idx_in == nullptr means the identity permutation
+// one LSD pass on digit `digit`; idx_in == nullptr means the identity permutation;
+// idx_out == nullptr: keys only (no payload)
 cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
                             uint32_t* idx_out, uint64_t m, int digit, const uint32_t* bases,
                             uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s);
@@ -114,6 +120,12 @@ cudaError_t launch_reduce_km(const uint64_t* seg_start, uint64_t nseg, const uin
 cudaError_t launch_km_finalize(const double* sums, const unsigned long long* cnts, const float* centroids,
                                uint32_t k, const uint32_t* list, uint32_t nlist, uint8_t* vals, uint64_t* val_off,
                                uint8_t* keys, uint64_t* key_off, cudaStream_t s);
+// WC exact stream: counts = segment lengths; key lengths / bytes decoded from the sorted keys
+cudaError_t launch_seg_lengths(const uint64_t* seg_start, uint64_t nseg, uint64_t* out, cudaStream_t s);
+cudaError_t launch_key_lengths_exact(const uint64_t* seg_start, uint64_t nseg, const uint64_t* skeys, uint64_t* lens,
+                                     cudaStream_t s);
+cudaError_t launch_key_decode(const uint64_t* seg_start, uint64_t nseg, const uint64_t* skeys, const uint64_t* key_off,
+                              uint8_t* keys, cudaStream_t s);
 cudaError_t launch_gather_u64(const uint32_t* perm, const uint8_t* v, uint64_t m, uint64_t* out, cudaStream_t s);
 cudaError_t launch_offsets_scaled(const uint64_t* seg_start, uint64_t nseg, uint64_t scale, uint64_t* out,
                                   cudaStream_t s);
@@ -123,14 +135,16 @@ cudaError_t launch_rehash(uint64_t* h, const uint64_t* kref, uint64_t m, uint64_
 
 // ---- multi-GPU exchange (exchange.cu) ----
 constexpr int kMaxRanks = 64;
-enum XMode : int { kXPairs = 0, kXSegs = 1, kXKM = 2 };
+enum XMode : int { kXPairs = 0, kXSegs = 1, kXKM = 2, kXSplit = 3 };
 struct XEntry { uint64_t koff_len; uint64_t v; };          // WC / II (16 B)
 struct XEntryKM { uint64_t id, cnt; double sums[8]; };      // KM partial (80 B)
 struct XSource {
   int mode = kXPairs;
   uint32_t nranks = 1;
   uint64_t n = 0;                              // records of the source
-  const uint64_t* kref = nullptr;              // kXPairs
+  const uint64_t* kref = nullptr;              // kXPairs; kXSplit: hashed-stream krefs
+  const uint64_t* hx = nullptr;                // kXSplit: exact-stream keys (nx of them, first)
+  uint64_t nx = 0;
   const uint8_t* v = nullptr;
   int vbytes = 8;
   const uint8_t* keys = nullptr;               // kXSegs

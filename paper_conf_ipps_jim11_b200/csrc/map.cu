@@ -58,12 +58,15 @@ struct Cfg {
   static constexpr int kLag = kStages - 2;
   // WC: per-warp queue of the window's long (hashed) words, hashed by all 32 lanes together
   // after the emission rounds (a lane-per-word hash inside the rounds diverges: with 7% long
-  // words, 9 in 10 rounds would carry at least one).  <= 64 words of >= 8 bytes fit in 512 B.
+  // words, 9 in 10 rounds would carry at least one).  A window holds at most 512 / 8 starts of
+  // words longer than kWcExact bytes.
   static constexpr int kHashQ = (W == kWC) ? 64 : 0;
-  // a6 fused into a5: the flush warp accumulates the LSD digit histograms of the keys it
-  // flushes (KM ids use 2 digits, text keys 8; StringMatch is not sorted)
-  static constexpr int kHistDigits = (W == kSM) ? 0 : (W == kKM) ? 2 : 8;
 };
+// WC words of <= kWcExact bytes get an exact 48-bit key (byte-packed <= 5, alnum-packed 6..7,
+// common.cuh) and travel in the exact stream (8-B entries: the key is the whole record); longer
+// words are hashed and travel with their key reference in the hashed stream (16-B entries).
+constexpr uint32_t kWcExact = 7;
+static_assert(kWin / (kWcExact + 1) <= Cfg<kWC>::kHashQ, "hash queue too small");
 constexpr int kKmPts = kT / 32;                // 512 points per KM tile
 
 static_assert(kLead + kT + kHalo + 32 <= kStageBytes, "stage too small");
@@ -106,21 +109,25 @@ struct Layout {
   static constexpr int bits = offs + kStages * kOffBytes;         // kStages x kBitBytes
   static constexpr int out = bits + kStages * kBitBytes;          // kNOut x Cfg<W>::kOutHalf
   static constexpr int hq = out + kNOut * Cfg<W>::kOutHalf;       // kNMap x kHashQ x 8 (WC)
-  static constexpr int hist = hq + kNMap * Cfg<W>::kHashQ * 8;    // kHistDigits x 256 x 4
-  static constexpr int cent = hist + Cfg<W>::kHistDigits * 1024;  // KM centroids
+  static constexpr int cent = hq + kNMap * Cfg<W>::kHashQ * 8;    // KM centroids
   static_assert(ready + kStages * 8 <= bytes, "header region overflow");
   static_assert(sizeof(OutCtl) <= hdr, "OutCtl overlaps the stage headers");
 };
-static_assert(256 % kNOut == 0, "8-bit generation counter must wrap on a buffer boundary");
+static_assert(64 % kNOut == 0, "6-bit generation counter must wrap on a buffer boundary");
 
+// Output-buffer formats.  SM / KM / II: SoA runs [keys | krefs | values] of kCap entries.
+// WC: exact-key entries (u64 key) fill the buffer from the bottom, hashed entries (u64 key, u64
+// kref) from the top; capacity is counted in 8-byte units (exact 1, hashed 2).  WC values are
+// all 1 and are not stored: a key's count is its segment length.
 template <int W>
 struct PairFmt {
-  static constexpr bool kKref = (W == kWC || W == kII);
-  static constexpr int kV = (W == kWC) ? 4 : (W == kSM) ? 0 : (W == kKM) ? 32 : 8;
+  static constexpr bool kKref = (W == kII);
+  static constexpr int kV = (W == kKM) ? 32 : (W == kII) ? 8 : 0;
   static constexpr int kPairBytes = 8 + (kKref ? 8 : 0) + kV;
-  static constexpr uint32_t kCap = (Cfg<W>::kOutHalf / kPairBytes) & ~3u;
-  // largest single warp reservation: WC 8 words / 16 B, SM 16 matches / 16 B, II 2, KM 1 per lane
-  static constexpr uint32_t kMaxReserve = (W == kWC) ? 256 : (W == kSM) ? 512 : 32 * ((W == kII) ? 2 : 1);
+  static constexpr uint32_t kCap = (W == kWC) ? (Cfg<W>::kOutHalf / 8 - 2) : (Cfg<W>::kOutHalf / kPairBytes) & ~3u;
+  // largest single warp reservation (units): WC <= 512 starts in 512 B (+1 crossing word, 2
+  // units), SM 16 matches / 16 B, II 2, KM 1 per lane
+  static constexpr uint32_t kMaxReserve = (W == kWC) ? 576 : (W == kSM) ? 512 : 32 * ((W == kII) ? 2 : 1);
   static_assert(kCap >= kMaxReserve, "output half smaller than one warp result");
 };
 
@@ -138,6 +145,9 @@ struct Params {
   uint64_t* okref;
   uint8_t* ov;
   uint64_t cap_pairs;
+  uint64_t* ohb;           // WC hashed stream: keys, krefs, capacity
+  uint64_t* okrefb;
+  uint64_t cap_b;
   uint32_t out_cap;        // per-half capacity actually used (FORCE_TINY_OUT shrinks it)
   uint32_t flags;
   DevState* st;
@@ -145,8 +155,6 @@ struct Params {
   const uint8_t* off_end;  // end of the offsets array rounded DOWN to 16 B (aligned TMA limit)
   uint64_t hash_seed;
   uint32_t key_bits;       // sort-key width (48 or 64)
-  uint32_t* hist;          // global 8 x 256 digit histograms (accumulated; nullptr: not fused)
-  uint64_t vpack;          // WC: the emitted value packed above the 48-bit key
 };
 
 constexpr uint32_t kFull = 0xffffffffu;
@@ -342,8 +350,24 @@ __device__ __forceinline__ uint64_t key_at(const Params& P, const TileView& tv, 
 // the <= 3 filler entries carry the workload's sentinel key, which sorts after every real key
 // and is excluded from the groups (DevState::pads).  StringMatch (Map-only, sparse) flushes with
 // plain stores and needs no filler.
-struct Slot { uint32_t half, base; };
-constexpr uint32_t kCntMask = 0xFFFFFFu;
+// Shared cursor: 32-bit [generation:6 | cb:12 | ca:14].  ca counts entries (WC: exact-key
+// entries), cb the WC hashed entries; one atomicAdd reserves both.  Field bounds: a buffer holds
+// <= 2558 units and at most kNMap reservations of <= kMaxReserve overshoot it before the seal.
+struct Slot { uint32_t half, base; };   // base: packed (cb << 14 | ca) at the reservation
+constexpr uint32_t kGenShift = 26, kCbShift = 14;
+constexpr uint32_t kCaMask = (1u << kCbShift) - 1u, kCbMask = (1u << (kGenShift - kCbShift)) - 1u;
+constexpr uint32_t kCntBits = (1u << kGenShift) - 1u;
+__device__ __forceinline__ uint32_t cur_gen(uint32_t c) { return c >> kGenShift; }
+__device__ __forceinline__ uint32_t cur_ca(uint32_t c) { return c & kCaMask; }
+__device__ __forceinline__ uint32_t cur_cb(uint32_t c) { return (c >> kCbShift) & kCbMask; }
+template <int W>
+__device__ __forceinline__ uint32_t units(uint32_t c) {   // buffer space of packed counts
+  if constexpr (W == kWC) return cur_ca(c) + 2u * cur_cb(c);
+  else return cur_ca(c);
+}
+static_assert(PairFmt<kWC>::kCap + kNMap * PairFmt<kWC>::kMaxReserve <= kCaMask, "ca field overflow");
+static_assert(PairFmt<kWC>::kCap / 2 + kNMap * 64 <= kCbMask, "cb field overflow");
+static_assert(PairFmt<kSM>::kCap + kNMap * PairFmt<kSM>::kMaxReserve <= kCaMask, "ca field overflow");
 
 template <int W>
 __device__ __forceinline__ uint64_t sentinel_key(const Params& P) {
@@ -365,7 +389,7 @@ __device__ void seal(const Params& P, OutCtl* oc, uint32_t gen8, uint32_t h, uin
     oc->committed[(h + 1) % kNOut] = 0;
     oc->nsealed = full_gen + 1;
     __threadfence_block();
-    atomicExch(&oc->cur, ((gen8 + 1) & 0xFFu) << 24);          // other warps continue in the next buffer
+    atomicExch(&oc->cur, ((gen8 + 1) & 0x3Fu) << kGenShift);   // other warps continue in the next buffer
   } else {
     oc->final_seq = full_gen;
     oc->is_final = 1;
@@ -374,6 +398,7 @@ __device__ void seal(const Params& P, OutCtl* oc, uint32_t gen8, uint32_t h, uin
   __threadfence_block();
   mbar_arrive(&oc->req[h]);
 }
+// cnt: packed counts (cb << 14 | ca); cap: buffer capacity in units
 template <int W>
 __device__ __forceinline__ Slot reserve(const Params& P, OutCtl* oc, uint8_t* outh, uint32_t cnt, uint32_t cap) {
   const uint32_t lane = threadIdx.x & 31;
@@ -381,16 +406,18 @@ __device__ __forceinline__ Slot reserve(const Params& P, OutCtl* oc, uint8_t* ou
     uint32_t old = 0;
     if (lane == 0) old = atomicAdd(&oc->cur, cnt);
     old = __shfl_sync(kFull, old, 0);
-    const uint32_t gen = old >> 24, base = old & kCntMask;
+    const uint32_t gen = cur_gen(old), base = old & kCntBits;
     const uint32_t h = gen % kNOut;
-    if (base + cnt <= cap) return {h, base};
+    const uint32_t u0 = units<W>(base);
+    if (u0 + units<W>(cnt) <= cap) return {h, base};
     if (lane == 0) {
-      if (base <= cap) {
-        // This warp crossed the capacity first: it seals half h (L113 "overflow handling").
+      if (u0 <= cap) {
+        // This warp crossed the capacity first (units grow monotonically within a generation):
+        // it seals half h (L113 "overflow handling").
         seal<W>(P, oc, gen, h, base, false);
       } else {
         volatile unsigned int* c = &oc->cur;
-        while ((*c >> 24) == gen) __nanosleep(128);
+        while (cur_gen(*c) == gen) __nanosleep(128);
       }
     }
     __syncwarp();
@@ -433,35 +460,28 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       while (*cm != cnt0) __nanosleep(32);
     }
     __syncwarp();
-    uint32_t cnt = cnt0;
-    if constexpr (W != kSM) {
-      cnt = (cnt0 + 3u) & ~3u;                                  // 4-pair aligned flush (TMA store)
-      if (lane < cnt - cnt0) {                                  // sentinel filler entries
-        reinterpret_cast<uint64_t*>(half)[cnt0 + lane] = sentinel_key<W>(P);
-        if constexpr (F::kKref) reinterpret_cast<uint64_t*>(half)[F::kCap + cnt0 + lane] = 0;
+    const uint32_t ca0 = cur_ca(cnt0);
+    const uint32_t cb = (W == kWC) ? cur_cb(cnt0) : 0u;
+    uint32_t cnt = ca0;
+    if constexpr (W == kWC) {
+      cnt = (ca0 + 1u) & ~1u;                                   // 16-B aligned exact run (TMA store)
+      if (lane == 0 && cnt != ca0) reinterpret_cast<uint64_t*>(half)[ca0] = sentinel_key<W>(P);
+    } else if constexpr (W != kSM) {
+      cnt = (ca0 + 3u) & ~3u;                                   // 4-pair aligned flush (TMA store)
+      if (lane < cnt - ca0) {                                   // sentinel filler entries
+        reinterpret_cast<uint64_t*>(half)[ca0 + lane] = sentinel_key<W>(P);
+        if constexpr (F::kKref) reinterpret_cast<uint64_t*>(half)[F::kCap + ca0 + lane] = 0;
       }
     }
-    if constexpr (Cfg<W>::kHistDigits > 0) {
-      if (P.hist) {                                             // digit histograms (fused a6)
-        __syncwarp();
-        uint32_t* hs = reinterpret_cast<uint32_t*>(smem + Layout<W>::hist);
-        const uint64_t* kk = reinterpret_cast<const uint64_t*>(half);
-        const uint32_t nd = min(static_cast<uint32_t>(Cfg<W>::kHistDigits), P.key_bits / 8);
-        for (uint32_t i = lane; i < cnt; i += 32) {
-          const uint64_t key = kk[i];
-#pragma unroll
-          for (uint32_t d = 0; d < static_cast<uint32_t>(Cfg<W>::kHistDigits); ++d)
-            if (d < nd) atomicAdd(&hs[d * 256 + ((key >> (8 * d)) & 255u)], 1u);
-        }
-      }
-    }
-    unsigned long long gb = 0;
-    if (lane == 0 && cnt) {
-      gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(cnt));  // ONE global atomic per flush
-      oc->nflush += 1;
-      oc->npads += cnt - cnt0;
+    unsigned long long gb = 0, gbb = 0;
+    if (lane == 0) {
+      if (cnt) gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(cnt));  // ONE global atomic per run
+      if (cb) gbb = atomicAdd(&P.st->pair_cursor_b, static_cast<unsigned long long>(cb));
+      oc->nflush += (cnt || cb) ? 1 : 0;
+      oc->npads += cnt - ca0;
     }
     gb = __shfl_sync(kFull, gb, 0);
+    gbb = __shfl_sync(kFull, gbb, 0);
     __syncwarp();
     if (cnt && gb + cnt <= P.cap_pairs) {
       const uint64_t* sh = reinterpret_cast<const uint64_t*>(half);
@@ -469,7 +489,7 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       if constexpr (W == kSM) {
         for (uint32_t i = lane; i < cnt; i += 32) P.oh[gb + i] = sh[i];
       } else if (lane == 0) {
-        // A4 staging-out as three TMA bulk stores (16-B aligned: gb % 4 == 0, cnt % 4 == 0)
+        // A4 staging-out as TMA bulk stores (16-B aligned: gb and cnt even / multiples of 4)
         fence_proxy_async_shared();
         tma_store_1d(P.oh + gb, sh, cnt * 8);
         if constexpr (F::kKref) tma_store_1d(P.okref + gb, sh + F::kCap, cnt * 8);
@@ -477,17 +497,21 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         tma_store_commit_and_wait_read();          // SMEM may be reused once the stores have read it
       }
     }
+    if constexpr (W == kWC) {
+      // hashed entries (key, kref) from the top of the buffer -> the two SoA arrays of the
+      // hashed stream (a few % of the pairs: plain coalesced stores)
+      if (cb && gbb + cb <= P.cap_b) {
+        const ulonglong2* top = reinterpret_cast<const ulonglong2*>(half + Cfg<W>::kOutHalf);
+        for (uint32_t i = lane; i < cb; i += 32) {
+          const ulonglong2 e = top[-1 - static_cast<int>(i)];
+          P.ohb[gbb + i] = e.x;
+          P.okrefb[gbb + i] = e.y;
+        }
+      }
+    }
     __syncwarp();
     if (lane == 0) mbar_arrive(&oc->done[h]);
     if (fin) break;
-  }
-  if constexpr (Cfg<W>::kHistDigits > 0) {
-    if (P.hist) {
-      __syncwarp();
-      const uint32_t* hs = reinterpret_cast<const uint32_t*>(smem + Layout<W>::hist);
-      for (uint32_t i = lane; i < Cfg<W>::kHistDigits * 256; i += 32)
-        if (hs[i]) atomicAdd(&P.hist[i], hs[i]);
-    }
   }
   if (lane == 0) {
     asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // global writes complete
@@ -647,6 +671,73 @@ __device__ void producer_loop(const Params& P, uint8_t* smem) {
 }
 
 // ---------------------------------------------------------------- map warps
+// WordCount emission of one warp window.  Each start is classified BEFORE the reservation: a
+// word is exact iff it ends within kWcExact bytes (nb bit q: a word cannot continue at q, so the
+// word at j ends at the first nb bit above j).  Only a lane's highest start can lack a visible
+// end; it is measured by the slow path up front.  One shared atomic reserves ta exact entries
+// and tb hashed entries; the rounds write exact keys directly and queue the hashed words, which
+// all 32 lanes then hash together.
+__device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* outh, const TileView& tv,
+                                        const uint32_t (&x)[8], long long p0, uint32_t emit_mask, uint32_t nb) {
+  const uint32_t lane = threadIdx.x & 31;
+  uint32_t len_slow = 0, slow_bit = 0;
+  if (emit_mask) {
+    const uint32_t jh = 31 - __clz(emit_mask);
+    if ((nb >> (jh + 1)) == 0) {
+      slow_bit = 1u << jh;
+      len_slow = slow_word_len(P, tv, p0 + jh, p0 + (lane < 31 ? 32 : 16));
+    }
+  }
+  uint32_t near = 0;                                   // bit j: an nb bit in (j, j + kWcExact]
+#pragma unroll
+  for (uint32_t d = 1; d <= kWcExact; ++d) near |= nb >> d;
+  uint32_t longm = emit_mask & ~near & ~slow_bit;
+  if (slow_bit && len_slow > kWcExact) longm |= slow_bit;
+  const uint32_t nl = __popc(longm);
+  const uint32_t tot = __reduce_add_sync(kFull, (__popc(emit_mask) - nl) | (nl << 16));
+  if (tot == 0) return;
+  const uint32_t packed = (tot & 0xFFFFu) | ((tot >> 16) << kCbShift);
+  const Slot slot = reserve<kWC>(P, oc, outh, packed, P.out_cap);
+  uint8_t* half = outh + slot.half * Cfg<kWC>::kOutHalf;
+  uint64_t* sh = reinterpret_cast<uint64_t*>(half);
+  ulonglong2* top = reinterpret_cast<ulonglong2*>(half + Cfg<kWC>::kOutHalf);   // hashed entry i: top[-1 - i]
+  uint64_t* hq = reinterpret_cast<uint64_t*>(outh + (Layout<kWC>::hq - Layout<kWC>::out)) +
+                 (threadIdx.x >> 5) * Cfg<kWC>::kHashQ;
+  const uint32_t kb0 = cur_cb(slot.base);
+  uint32_t ka = cur_ca(slot.base), nq = 0;
+  uint32_t m_left = emit_mask;
+  while (__any_sync(kFull, m_left != 0)) {
+    const bool act = m_left != 0;
+    uint32_t j = 0, len = 0;
+    if (act) {
+      j = __ffs(m_left) - 1;
+      m_left &= m_left - 1;
+      const uint32_t rest = nb >> (j + 1);
+      len = rest ? static_cast<uint32_t>(__ffs(rest)) : len_slow;
+    }
+    const bool ex = act && len <= kWcExact;
+    const uint32_t ma = __ballot_sync(kFull, ex), mb = __ballot_sync(kFull, act && !ex);
+    if (ex) {
+      const uint64_t b = window8(x, j);     // an exact word lies inside the 32 loaded bytes
+      sh[ka + __popc(ma & lanemask_lt())] = len <= inline_max(48) ? inline_key(b, len, 48) : alnum_key48(b, len);
+    } else if (act) {
+      if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
+      hq[nq + __popc(mb & lanemask_lt())] = static_cast<uint64_t>(p0 + j - tv.sbase) | (static_cast<uint64_t>(len) << 24);
+    }
+    ka += __popc(ma);
+    nq += __popc(mb);
+  }
+  __syncwarp();
+  for (uint32_t q = lane; q < nq; q += 32) {           // lane-parallel hashing of the long words
+    const uint64_t e = hq[q];
+    const long long p = tv.sbase + static_cast<long long>(e & 0xFFFFFF);
+    const uint32_t len = static_cast<uint32_t>(e >> 24);
+    top[-1 - static_cast<int>(kb0 + q)] =
+        make_ulonglong2(key_at(P, tv, p, len), (reinterpret_cast<uint64_t>(P.rec + p) << 16) | len);
+  }
+  commit(oc, slot, packed);
+}
+
 template <int W>
 __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, const TileView& tv,
                                 long long p0, long long i0, bool live) {
@@ -731,9 +822,12 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
       }
     }
   }
+  if constexpr (W == kWC) {
+    emit_wc(P, oc, outh, tv, x, p0, emit_mask, nb);
+    return;
+  }
   // ---- reserve one warp result, then lane-major emission rounds
-  const uint32_t cnt = __popc(emit_mask);
-  const uint32_t total = __reduce_add_sync(kFull, cnt);
+  const uint32_t total = __reduce_add_sync(kFull, __popc(emit_mask));
   if (total == 0) return;
   const Slot slot = reserve<W>(P, oc, outh, total, P.out_cap);
   uint8_t* half = outh + slot.half * Cfg<W>::kOutHalf;
@@ -743,33 +837,15 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
   uint32_t k = slot.base;
   uint32_t m_left = emit_mask;
   int nth = 0;
-  uint32_t nq = 0;                                   // WC: queued long words of this window
-  uint64_t* hq = reinterpret_cast<uint64_t*>(outh + (Layout<W>::hq - Layout<W>::out)) +
-                 (threadIdx.x >> 5) * Cfg<W>::kHashQ;
   while (__any_sync(kFull, m_left != 0)) {
     const bool act = m_left != 0;
     const uint32_t m = __ballot_sync(kFull, act);
-    bool queue = false;
-    uint64_t qe = 0;
     if (act) {
       const uint32_t j = __ffs(m_left) - 1;
       m_left &= m_left - 1;
       const uint32_t idx = k + __popc(m & lanemask_lt());
       const long long p = p0 + j;
-      if constexpr (W == kWC) {
-        const uint32_t rest = nb >> (j + 1);
-        uint32_t len = rest ? static_cast<uint32_t>(__ffs(rest)) : slow_word_len(P, tv, p, p0 + (lane < 31 ? 32 : 16));
-        if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
-        if (len <= inline_max(P.key_bits)) {
-          sh[idx] = inline_key(window8(x, j), len, P.key_bits) | P.vpack;
-        } else {                                      // hashed after the rounds, all lanes together
-          queue = true;
-          qe = static_cast<uint64_t>(idx) | (static_cast<uint64_t>(p - tv.sbase) << 16) |
-               (static_cast<uint64_t>(len) << 40);
-        }
-        sk[idx] = (reinterpret_cast<uint64_t>(P.rec + p) << 16) | len;
-        reinterpret_cast<uint32_t*>(sv)[idx] = 1u;
-      } else if constexpr (W == kSM) {
+      if constexpr (W == kSM) {
         sh[idx] = P.gbase + static_cast<uint64_t>(p);
       } else if constexpr (W == kII) {
         uint32_t len = nth == 0 ? aux[0] : aux[1];
@@ -781,21 +857,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
         reinterpret_cast<uint64_t*>(sv)[idx] = P.gbase + static_cast<uint64_t>(q0);
       }
     }
-    if constexpr (W == kWC) {
-      const uint32_t qm = __ballot_sync(kFull, queue);
-      if (queue) hq[nq + __popc(qm & lanemask_lt())] = qe;
-      nq += __popc(qm);
-    }
     k += __popc(m);
-  }
-  if constexpr (W == kWC) {
-    __syncwarp();
-    for (uint32_t q = lane; q < nq; q += 32) {         // lane-parallel hashing of the long words
-      const uint64_t e = hq[q];
-      const uint32_t idx = static_cast<uint32_t>(e & 0xFFFF);
-      const long long p = tv.sbase + static_cast<long long>((e >> 16) & 0xFFFFFF);
-      sh[idx] = key_at(P, tv, p, static_cast<uint32_t>(e >> 40)) | P.vpack;
-    }
   }
   commit(oc, slot, total);
 }
@@ -898,7 +960,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   named_bar_sync(2, kNMap * 32);
   if (threadIdx.x == 0) {
     const uint32_t cur = *reinterpret_cast<volatile unsigned int*>(&oc->cur);
-    seal<W>(P, oc, cur >> 24, (cur >> 24) % kNOut, cur & kCntMask, true);
+    seal<W>(P, oc, cur_gen(cur), cur_gen(cur) % kNOut, cur & kCntBits, true);
   }
 }
 
@@ -921,10 +983,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_map(Params P) {
     uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout<W>::ready);
     for (int s = 0; s < kStages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], kNMap); mbar_init(&ready[s], 1); }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  if constexpr (Cfg<W>::kHistDigits > 0) {
-    uint32_t* hs = reinterpret_cast<uint32_t*>(smem + Layout<W>::hist);
-    for (uint32_t i = threadIdx.x; i < Cfg<W>::kHistDigits * 256; i += blockDim.x) hs[i] = 0;
   }
   if constexpr (W == kKM) {
     float* cent = reinterpret_cast<float*>(smem + Layout<W>::cent);
@@ -992,8 +1050,9 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
                         : nullptr;
   P.hash_seed = a.hash_seed;
   P.key_bits = a.key_bits;
-  P.hist = a.hist;
-  P.vpack = a.vpack;
+  P.ohb = a.out.hb;
+  P.okrefb = a.out.krefb;
+  P.cap_b = a.out.cap_b;
   if (P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>((P.ntiles + 255) / 256);
@@ -1012,8 +1071,8 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
 
 }  // namespace
 
-int vbytes_of(int w) { return w == kWC ? 4 : w == kSM ? 0 : w == kKM ? 32 : 8; }
-bool has_kref(int w) { return w == kWC || w == kII; }
+int vbytes_of(int w) { return w == kKM ? 32 : w == kII ? 8 : 0; }
+bool has_kref(int w) { return w == kII; }
 
 uint64_t map_tiles(const MapArgs& a) {
   if (a.workload == kKM) return (a.n + kKmPts - 1) / kKmPts;

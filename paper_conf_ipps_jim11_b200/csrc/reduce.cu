@@ -354,6 +354,28 @@ __global__ void k_key_copy(const uint64_t* seg, uint64_t nseg, const uint32_t* p
   uint8_t* dst = keys + key_off[s];
   for (uint32_t i = lane; i < len; i += 32) dst[i] = src[i];
 }
+// WC exact stream: the key is the record (value 1) -> count = segment length, key bytes decoded
+// from the key itself.
+__global__ void k_seg_lengths(const uint64_t* seg, uint64_t nseg, uint64_t* out) {
+  const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (s < nseg) out[s] = seg[s + 1] - seg[s];
+}
+__global__ void k_key_lengths_exact(const uint64_t* seg, uint64_t nseg, const uint64_t* sk, uint64_t* lens) {
+  const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (s >= nseg) return;
+  uint32_t len;
+  exact_key_bytes48(sk[seg[s]], len);
+  lens[s] = len;
+}
+__global__ void k_key_decode(const uint64_t* seg, uint64_t nseg, const uint64_t* sk, const uint64_t* key_off,
+                             uint8_t* keys) {
+  const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (s >= nseg) return;
+  uint32_t len;
+  const uint64_t b = exact_key_bytes48(sk[seg[s]], len);
+  uint8_t* dst = keys + key_off[s];
+  for (uint32_t i = 0; i < len; ++i) dst[i] = static_cast<uint8_t>(b >> (8 * i));
+}
 __global__ void k_gather_u64(const uint32_t* perm, const uint64_t* v, uint64_t m, uint64_t* out) {
   const uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
   if (i < m) out[i] = v[perm[i]];
@@ -447,6 +469,26 @@ cudaError_t launch_km_finalize(const double* sums, const unsigned long long* cnt
   const uint32_t n = list ? nlist : k;
   k_km_finalize<<<blocks_for(n + 1, 128), 128, 0, s>>>(sums, cnts, centroids, k, list, nlist, vals, val_off, keys,
                                                        key_off);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_seg_lengths(const uint64_t* seg_start, uint64_t nseg, uint64_t* out, cudaStream_t s) {
+  if (nseg == 0) return cudaSuccess;
+  k_seg_lengths<<<blocks_for(nseg, 256), 256, 0, s>>>(seg_start, nseg, out);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_key_lengths_exact(const uint64_t* seg_start, uint64_t nseg, const uint64_t* skeys, uint64_t* lens,
+                                     cudaStream_t s) {
+  if (nseg == 0) return cudaSuccess;
+  k_key_lengths_exact<<<blocks_for(nseg, 256), 256, 0, s>>>(seg_start, nseg, skeys, lens);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_key_decode(const uint64_t* seg_start, uint64_t nseg, const uint64_t* skeys, const uint64_t* key_off,
+                              uint8_t* keys, cudaStream_t s) {
+  if (nseg == 0) return cudaSuccess;
+  k_key_decode<<<blocks_for(nseg, 256), 256, 0, s>>>(seg_start, nseg, skeys, key_off, keys);
   count_launch();
   return cudaGetLastError();
 }

@@ -56,11 +56,11 @@ __global__ void __launch_bounds__(256) k_hist(const uint64_t* __restrict__ keys,
     if (sh[i]) atomicAdd(&hist[i], sh[i]);
 }
 
-template <int IPT>
+template <int IPT, bool kPay>
 struct SortSmem {
   static constexpr int kTile = kSortThreads * IPT;
   uint64_t keys[kTile];
-  uint32_t idx[kTile];
+  uint32_t idx[kPay ? kTile : 1];
   uint32_t wcnt[kWarps][256];      // per-warp digit counters, then warp-exclusive offsets
   uint32_t hist[256];
   uint32_t dstart[256];
@@ -74,7 +74,8 @@ constexpr int kLookWindow = 4;   // predecessor status words fetched per look-ba
 // kVar bit 0: rank with one shared atomic per match group (1) or a read-modify-write of the
 // warp counter per step (0); bit 1: tile histogram by shared atomics before ranking, published
 // as an early aggregate (1), or summed from the warp counters after ranking (0).
-template <bool kFirst, int kVar, int IPT, int MINB>
+// kPay: carry the u32 permutation payload (false: keys only, idx_in / idx_out unused).
+template <bool kFirst, int kVar, int IPT, int MINB, bool kPay>
 __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t* __restrict__ keys_in,
                                                                const uint32_t* __restrict__ idx_in,
                                                                uint64_t* __restrict__ keys_out,
@@ -83,10 +84,10 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t*
                                                                uint64_t* status, uint32_t epoch,
                                                                unsigned int* tile_counter) {
   constexpr int kSortIPT = IPT;
-  constexpr int kSortTile = SortSmem<IPT>::kTile;
+  constexpr int kSortTile = SortSmem<IPT, kPay>::kTile;
   constexpr bool kAtomicRank = (kVar & 1) != 0, kEarly = (kVar & 2) != 0;
   extern __shared__ __align__(16) uint8_t raw[];
-  SortSmem<IPT>& S = *reinterpret_cast<SortSmem<IPT>*>(raw);
+  SortSmem<IPT, kPay>& S = *reinterpret_cast<SortSmem<IPT, kPay>*>(raw);
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid == 0) S.tile = atomicAdd(tile_counter, 1u);
   for (uint32_t i = tid; i < kWarps * 256; i += kSortThreads) (&S.wcnt[0][0])[i] = 0;
@@ -204,7 +205,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t*
     const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & 255u;
     const uint32_t lp = S.dstart[dj] + S.wcnt[warp][dj] + rank[j];
     S.keys[lp] = key[j];
-    S.idx[lp] = kFirst ? static_cast<uint32_t>(e) : (e < m ? idx_in[e] : 0u);
+    if constexpr (kPay) S.idx[lp] = kFirst ? static_cast<uint32_t>(e) : (e < m ? idx_in[e] : 0u);
   }
   __syncthreads();
   // 6. contiguous per-digit runs to global memory
@@ -214,7 +215,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t*
     const uint32_t dk = static_cast<uint32_t>(k >> shift) & 255u;
     const uint32_t pos = S.goff[dk] + (i - S.dstart[dk]);
     keys_out[pos] = k;
-    idx_out[pos] = S.idx[i];
+    if constexpr (kPay) idx_out[pos] = S.idx[i];
   }
 }
 
@@ -321,53 +322,74 @@ int sort_cfg() {
 }
 static const int kCfgIPT[4] = {16, 12, 20, 8};
 int sort_tile() { return kSortThreads * kCfgIPT[sort_cfg()]; }
+static const int kCfgIPTKeys[4] = {16, 12, 16, 24};
+int sort_tile_keys() { return kSortThreads * kCfgIPTKeys[sort_cfg()]; }
 
-template <bool kFirst, int kVar, int IPT, int MINB>
+template <bool kFirst, int kVar, int IPT, int MINB, bool kPay>
 static void launch_os(unsigned tiles, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
                       uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
                       uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
-  const size_t smem = sizeof(SortSmem<IPT>);
-  cudaFuncSetAttribute(k_onesweep<kFirst, kVar, IPT, MINB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  const size_t smem = sizeof(SortSmem<IPT, kPay>);
+  cudaFuncSetAttribute(k_onesweep<kFirst, kVar, IPT, MINB, kPay>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        static_cast<int>(smem));
-  k_onesweep<kFirst, kVar, IPT, MINB><<<tiles, kSortThreads, smem, s>>>(keys_in, idx_in, keys_out, idx_out, m, shift,
-                                                                         bases, status, epoch, tile_counter);
+  k_onesweep<kFirst, kVar, IPT, MINB, kPay><<<tiles, kSortThreads, smem, s>>>(keys_in, idx_in, keys_out, idx_out, m,
+                                                                               shift, bases, status, epoch,
+                                                                               tile_counter);
 }
 
+#define BMR_OS_ARGS tiles, keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch, tile_counter, s
 template <bool kFirst, int kVar>
 static void launch_cfg(unsigned tiles, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
                        uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
                        uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
   switch (sort_cfg()) {
-    case 1: launch_os<kFirst, kVar, 12, 4>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch, tile_counter, s); break;
-    case 2: launch_os<kFirst, kVar, 20, 2>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch, tile_counter, s); break;
-    case 3: launch_os<kFirst, kVar, 8, 6>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch, tile_counter, s); break;
-    default: launch_os<kFirst, kVar, 16, 3>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch, tile_counter, s); break;
+    case 1: launch_os<kFirst, kVar, 12, 4, true>(BMR_OS_ARGS); break;
+    case 2: launch_os<kFirst, kVar, 20, 2, true>(BMR_OS_ARGS); break;
+    case 3: launch_os<kFirst, kVar, 8, 6, true>(BMR_OS_ARGS); break;
+    default: launch_os<kFirst, kVar, 16, 3, true>(BMR_OS_ARGS); break;
+  }
+}
+// keys only (8 B per key per direction): the tile shape is the same, the SMEM image smaller
+static void launch_keys_only(unsigned tiles, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
+                             uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
+                             uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
+  switch (sort_cfg()) {
+    case 1: launch_os<false, 2, 12, 4, false>(BMR_OS_ARGS); break;
+    case 2: launch_os<false, 2, 16, 4, false>(BMR_OS_ARGS); break;
+    case 3: launch_os<false, 2, 24, 2, false>(BMR_OS_ARGS); break;
+    default: launch_os<false, 2, 16, 3, false>(BMR_OS_ARGS); break;
   }
 }
 
 cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out, uint32_t* idx_out,
-                            uint64_t m, int digit, const uint32_t* bases, uint64_t* status, uint32_t epoch,
+                            uint64_t m, int digit, const uint32_t* bases_all, uint64_t* status, uint32_t epoch,
                             unsigned int* tile_counter, cudaStream_t s) {
   if (m == 0) return cudaSuccess;
-  const unsigned tiles = static_cast<unsigned>((m + sort_tile() - 1) / sort_tile());
+  const uint64_t tile = idx_out ? sort_tile() : sort_tile_keys();
+  const unsigned tiles = static_cast<unsigned>((m + tile - 1) / tile);
   cudaError_t e = cudaMemsetAsync(tile_counter, 0, sizeof(unsigned int), s);
   if (e != cudaSuccess) return e;
   const uint32_t shift = 8u * digit;
-  const uint32_t* b = bases + 256 * digit;
+  const uint32_t* bases = bases_all + 256 * digit;
   const bool first = idx_in == nullptr;
-  switch (sort_variant() | (first ? 4 : 0)) {
-    case 0: launch_cfg<false, 0>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    case 1: launch_cfg<false, 1>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    case 2: launch_cfg<false, 2>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    case 3: launch_cfg<false, 3>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    case 4: launch_cfg<true, 0>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    case 5: launch_cfg<true, 1>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    case 6: launch_cfg<true, 2>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
-    default: launch_cfg<true, 3>(tiles, keys_in, idx_in, keys_out, idx_out, m, shift, b, status, epoch, tile_counter, s); break;
+  if (idx_out == nullptr) {
+    launch_keys_only(BMR_OS_ARGS);
+  } else {
+    switch (sort_variant() | (first ? 4 : 0)) {
+      case 0: launch_cfg<false, 0>(BMR_OS_ARGS); break;
+      case 1: launch_cfg<false, 1>(BMR_OS_ARGS); break;
+      case 2: launch_cfg<false, 2>(BMR_OS_ARGS); break;
+      case 3: launch_cfg<false, 3>(BMR_OS_ARGS); break;
+      case 4: launch_cfg<true, 0>(BMR_OS_ARGS); break;
+      case 5: launch_cfg<true, 1>(BMR_OS_ARGS); break;
+      case 6: launch_cfg<true, 2>(BMR_OS_ARGS); break;
+      default: launch_cfg<true, 3>(BMR_OS_ARGS); break;
+    }
   }
   count_launch();
   return cudaGetLastError();
 }
+#undef BMR_OS_ARGS
 
 template <typename T>
 static cudaError_t scan_impl(const T* in, uint64_t* out, uint64_t n, unsigned long long* total, uint64_t* status,
