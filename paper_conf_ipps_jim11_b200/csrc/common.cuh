@@ -142,7 +142,8 @@ __device__ __forceinline__ uint64_t hash_bytes(const uint8_t* p, uint32_t len, u
 // passes fewer; digits 6 and 7 are then constant and skipped):
 //   inline  : keys of <= kInlineMax bytes packed little-endian, length in the 3 bits above them
 //             (64: len << 56, <= 7 bytes; 48: len << 40, <= 5 bytes) — injective, top bit clear;
-//   alnum   : (48 only) [0-9A-Za-z] keys of 6..7 bytes, 6-bit symbol codes, len << 43;
+//   alnum   : (48 only) [0-9A-Za-z] keys of 6..7 bytes: 2^43 | 6-bit symbol codes (1..62, so
+//             the length is implied) — every exact 48-bit key is < 2^44 (five 9-bit digits);
 //   hashed  : longer keys -> hash with the top bit of the width forced to 1 (never collides with
 //             an inline key); equal hashes are verified byte-for-byte at segment time;
 //   sentinel: all ones in the width — flush filler pairs, sorts after every real key.
@@ -162,8 +163,9 @@ __device__ __forceinline__ uint64_t inline_key(uint64_t bytes_le, uint32_t len, 
   return (bytes_le & ((1ULL << (8 * len)) - 1ULL)) | (static_cast<uint64_t>(len) << (bits - 8));
 }
 // 48-bit (WordCount) keys of 6..7 bytes: a WC word is [0-9A-Za-z]+ (C-3 #1), so each symbol
-// has a 6-bit code (1..62) and 7 symbols (42 bits) plus the length at bits 43..45 pack
-// injectively — disjoint from the byte-packed keys (< 2^43) and the hashed ones (bit 47).
+// has a nonzero 6-bit code (1..62); 6 or 7 codes (<= 42 bits, the highest nonzero code gives
+// the length) above a 2^43 tag pack injectively — disjoint from the byte-packed keys (< 2^43)
+// and from the hashed ones (bit 47).
 __device__ __forceinline__ bool alnum_byte(uint32_t c) {
   return (c - '0' < 10u) || (c - 'A' < 26u) || (c - 'a' < 26u);
 }
@@ -181,7 +183,7 @@ __device__ __forceinline__ uint64_t alnum_key48(uint64_t bytes_le, uint32_t len)
   x = (x & 0x003F003F003F003FULL) | ((x >> 2) & 0x0FC00FC00FC00FC0ULL);
   x = (x & 0x00000FFF00000FFFULL) | ((x >> 4) & 0x00FFF00000FFF000ULL);
   x = (x & 0x0000000000FFFFFFULL) | ((x >> 8) & 0x0000FFFFFF000000ULL);
-  return x | (static_cast<uint64_t>(len) << 43);
+  return x | (1ULL << 43);
 }
 // Inverse of the 48-bit exact formats (inline <= 5 bytes, alnum 6..7): key bytes little-endian.
 __device__ __forceinline__ uint64_t exact_key_bytes48(uint64_t key, uint32_t& len) {
@@ -189,7 +191,8 @@ __device__ __forceinline__ uint64_t exact_key_bytes48(uint64_t key, uint32_t& le
     len = static_cast<uint32_t>(key >> 40) & 7u;
     return key & ((1ULL << 40) - 1ULL);
   }
-  len = static_cast<uint32_t>(key >> 43) & 7u;
+  const uint64_t codes = key & ((1ULL << 42) - 1ULL);
+  len = codes ? static_cast<uint32_t>(63 - __clzll(static_cast<long long>(codes))) / 6u + 1u : 0u;
   uint64_t b = 0;
   for (uint32_t i = 0; i < len; ++i) {
     const uint32_t c = static_cast<uint32_t>(key >> (6 * i)) & 63u;

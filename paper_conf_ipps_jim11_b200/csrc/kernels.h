@@ -77,14 +77,17 @@ struct SortBufs {
   uint64_t cap = 0;
 };
 constexpr int kSortThreads = 256;
+constexpr int kBinStride = 512;   // histogram / base tables: 8 digits x kBinStride bins (digits of 8 or 9 bits)
 int sort_tile();   // keys per onesweep tile (tile shape chosen at start-up, BMR_SORT_CFG)
 int sort_tile_keys();   // the same for the keys-only passes
-// histograms of digits [0, nd) (nd = key width / 8); hist must hold 8 x 256 u32
-cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int nd, int num_sms, cudaStream_t s);
-// one LSD pass on digit `digit`; idx_in == nullptr means the identity permutation;
-// idx_out == nullptr: keys only (no payload)
+// histograms of digits [0, nd) of `bits` bits each (8 or 9); hist holds 8 x kBinStride u32
+cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int nd, int bits, int num_sms,
+                        cudaStream_t s);
+// one LSD pass on digit `digit` of `bits` bits (8, or 9 for keys-only passes); idx_in ==
+// nullptr means the identity permutation; idx_out == nullptr: keys only (no payload).
+// bases: 8 x kBinStride table of global digit bases; status: tiles x 2^bits look-back words
 cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
-                            uint32_t* idx_out, uint64_t m, int digit, const uint32_t* bases,
+                            uint32_t* idx_out, uint64_t m, int digit, int bits, const uint32_t* bases,
                             uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s);
 
 // ---- segments ----

@@ -63,6 +63,7 @@ __device__ bool key_bytes_equal(uint64_t ka, uint64_t kb) {
 // a lane compares its key with the previous position's key (shuffle from the previous lane).
 constexpr int kSegWarp = 32 * kSegIPT;   // positions per warp
 
+template <bool kVerify>
 __global__ void __launch_bounds__(kSegThreads) k_seg_count(const uint64_t* __restrict__ sk,
                                                          const uint32_t* __restrict__ perm,
                                                          const uint64_t* __restrict__ kref, uint64_t m,
@@ -84,20 +85,22 @@ __global__ void __launch_bounds__(kSegThreads) k_seg_count(const uint64_t* __res
     if (lane == 0) prev = carry_k;
     const bool head = valid && (i == 0 || ((k ^ prev) & kmask) != 0);
     heads += head ? 1u : 0u;
-    // byte verification of equal hashed keys (C-3 #13): adjacent pairs inside an equal-hash run
-    const bool hashed_run = valid && kref && (k & hbit) && !head;
-    const bool need_r = valid && kref && (k & hbit);
-    const unsigned any = __ballot_sync(0xffffffffu, need_r);
-    uint64_t r = 0;
-    if (any) {
-      if (need_r) r = kref[perm[i]];
-      uint64_t rp = __shfl_up_sync(0xffffffffu, r, 1);
-      if (lane == 0) rp = carry_has_r ? carry_r : ((hashed_run && i > 0) ? kref[perm[i - 1]] : 0);
-      if (hashed_run && !key_bytes_equal(r, rp)) ++coll;
-    }
     carry_k = __shfl_sync(0xffffffffu, k, 31);
-    carry_r = __shfl_sync(0xffffffffu, r, 31);
-    carry_has_r = __shfl_sync(0xffffffffu, need_r ? 1u : 0u, 31) != 0;
+    if constexpr (kVerify) {
+      // byte verification of equal hashed keys (C-3 #13): adjacent pairs inside an equal-hash run
+      const bool hashed_run = valid && (k & hbit) && !head;
+      const bool need_r = valid && (k & hbit);
+      const unsigned any = __ballot_sync(0xffffffffu, need_r);
+      uint64_t r = 0;
+      if (any) {
+        if (need_r) r = kref[perm[i]];
+        uint64_t rp = __shfl_up_sync(0xffffffffu, r, 1);
+        if (lane == 0) rp = carry_has_r ? carry_r : ((hashed_run && i > 0) ? kref[perm[i - 1]] : 0);
+        if (hashed_run && !key_bytes_equal(r, rp)) ++coll;
+      }
+      carry_r = __shfl_sync(0xffffffffu, r, 31);
+      carry_has_r = __shfl_sync(0xffffffffu, need_r ? 1u : 0u, 31) != 0;
+    }
   }
   if (coll) atomicAdd(&st->collisions, coll);
   const uint32_t w = __reduce_add_sync(0xffffffffu, heads);
@@ -403,8 +406,12 @@ inline unsigned blocks_for(uint64_t n, unsigned t) { return static_cast<unsigned
 cudaError_t launch_seg_count(const uint64_t* skeys, const uint32_t* perm, const uint64_t* kref, uint64_t m,
                              uint32_t* counts, DevState* st, uint32_t key_bits, uint64_t kmask, cudaStream_t s) {
   if (m == 0) return cudaSuccess;
-  k_seg_count<<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, perm, kref, m, counts, st, hashed_bit(key_bits),
-                                                              kmask);
+  if (kref)
+    k_seg_count<true><<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, perm, kref, m, counts, st,
+                                                                      hashed_bit(key_bits), kmask);
+  else   // keys-only streams: equal keys are equal records, nothing to verify
+    k_seg_count<false><<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, perm, kref, m, counts, st,
+                                                                       hashed_bit(key_bits), kmask);
   count_launch();
   return cudaGetLastError();
 }

@@ -28,13 +28,14 @@ __device__ __forceinline__ uint64_t pack_status(uint32_t epoch, uint32_t kind, u
   return (static_cast<uint64_t>(epoch) << 34) | (static_cast<uint64_t>(kind) << 32) | v;
 }
 
-// Digit histograms of the first nd digits (nd = key width / 8): one read of the keys, two keys
-// per 16-byte load, shared atomics into a per-block 8 x 256 table.
+// Digit histograms of the first nd digits of `bits` bits (8 or 9): one read of the keys, two
+// keys per 16-byte load, shared atomics into a per-block nd x 512 table (stride kBinStride).
 __global__ void __launch_bounds__(256) k_hist(const uint64_t* __restrict__ keys, uint64_t m, uint32_t nd,
-                                            uint32_t* hist) {
-  __shared__ uint32_t sh[8 * 256];
-  for (int i = threadIdx.x; i < 8 * 256; i += blockDim.x) sh[i] = 0;
+                                            uint32_t bits, uint32_t* hist) {
+  __shared__ uint32_t sh[8 * kBinStride];
+  for (int i = threadIdx.x; i < 8 * kBinStride; i += blockDim.x) sh[i] = 0;
   __syncthreads();
+  const uint64_t mask = (1ULL << bits) - 1ULL;
   const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
   const uint64_t m2 = m / 2;
   const ulonglong2* k2 = reinterpret_cast<const ulonglong2*>(keys);
@@ -43,39 +44,41 @@ __global__ void __launch_bounds__(256) k_hist(const uint64_t* __restrict__ keys,
 #pragma unroll
     for (uint32_t d = 0; d < 8; ++d) {
       if (d >= nd) break;
-      atomicAdd(&sh[d * 256 + ((kk.x >> (8 * d)) & 255u)], 1u);
-      atomicAdd(&sh[d * 256 + ((kk.y >> (8 * d)) & 255u)], 1u);
+      atomicAdd(&sh[d * kBinStride + ((kk.x >> (bits * d)) & mask)], 1u);
+      atomicAdd(&sh[d * kBinStride + ((kk.y >> (bits * d)) & mask)], 1u);
     }
   }
   if ((m & 1) && blockIdx.x == 0 && threadIdx.x == 0) {
     const uint64_t k = keys[m - 1];
-    for (uint32_t d = 0; d < nd; ++d) atomicAdd(&sh[d * 256 + ((k >> (8 * d)) & 255u)], 1u);
+    for (uint32_t d = 0; d < nd; ++d) atomicAdd(&sh[d * kBinStride + ((k >> (bits * d)) & mask)], 1u);
   }
   __syncthreads();
-  for (int i = threadIdx.x; i < static_cast<int>(nd) * 256; i += blockDim.x)
+  for (int i = threadIdx.x; i < static_cast<int>(nd) * kBinStride; i += blockDim.x)
     if (sh[i]) atomicAdd(&hist[i], sh[i]);
 }
 
-template <int IPT, bool kPay>
+template <int IPT, bool kPay, int kBins>
 struct SortSmem {
   static constexpr int kTile = kSortThreads * IPT;
   uint64_t keys[kTile];
   uint32_t idx[kPay ? kTile : 1];
-  uint32_t wcnt[kWarps][256];      // per-warp digit counters, then warp-exclusive offsets
-  uint32_t hist[256];
-  uint32_t dstart[256];
-  uint32_t goff[256];
+  uint32_t wcnt[kWarps][kBins];    // per-warp digit counters, then warp-exclusive offsets
+  uint32_t hist[kBins];
+  uint32_t dstart[kBins];
+  uint32_t goff[kBins];
   uint32_t wsum[kWarps];
   uint32_t tile;
 };
 
-constexpr int kLookWindow = 4;   // predecessor status words fetched per look-back step
 
+// One LSD pass over the digit [shift, shift + kBits) (kBits 8: 256 bins, one digit per thread;
+// kBits 9: 512 bins, two adjacent digits per thread).
 // kVar bit 0: rank with one shared atomic per match group (1) or a read-modify-write of the
 // warp counter per step (0); bit 1: tile histogram by shared atomics before ranking, published
 // as an early aggregate (1), or summed from the warp counters after ranking (0).
 // kPay: carry the u32 permutation payload (false: keys only, idx_in / idx_out unused).
-template <bool kFirst, int kVar, int IPT, int MINB, bool kPay>
+// kLookWindow: predecessor status words fetched per look-back step (per digit).
+template <bool kFirst, int kVar, int IPT, int MINB, bool kPay, int kBits, int kLookWindow = 4>
 __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t* __restrict__ keys_in,
                                                                const uint32_t* __restrict__ idx_in,
                                                                uint64_t* __restrict__ keys_out,
@@ -83,15 +86,20 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t*
                                                                uint32_t shift, const uint32_t* __restrict__ bases,
                                                                uint64_t* status, uint32_t epoch,
                                                                unsigned int* tile_counter) {
+  constexpr int kBins = 1 << kBits, kDPT = kBins / kSortThreads;
+  constexpr uint32_t kMask = kBins - 1;
   constexpr int kSortIPT = IPT;
-  constexpr int kSortTile = SortSmem<IPT, kPay>::kTile;
+  using Smem = SortSmem<IPT, kPay, kBins>;
+  constexpr int kSortTile = Smem::kTile;
   constexpr bool kAtomicRank = (kVar & 1) != 0, kEarly = (kVar & 2) != 0;
+  constexpr bool kBackoff = (kVar & 4) != 0, kMatchHist = (kVar & 8) != 0;
+  static_assert(kDPT >= 1 && kDPT * kSortThreads == kBins, "bins must be a multiple of the block size");
   extern __shared__ __align__(16) uint8_t raw[];
-  SortSmem<IPT, kPay>& S = *reinterpret_cast<SortSmem<IPT, kPay>*>(raw);
+  Smem& S = *reinterpret_cast<Smem*>(raw);
   const uint32_t tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid == 0) S.tile = atomicAdd(tile_counter, 1u);
-  for (uint32_t i = tid; i < kWarps * 256; i += kSortThreads) (&S.wcnt[0][0])[i] = 0;
-  S.hist[tid] = 0;
+  for (uint32_t i = tid; i < kWarps * kBins; i += kSortThreads) (&S.wcnt[0][0])[i] = 0;
+  for (uint32_t i = tid; i < kBins; i += kSortThreads) S.hist[i] = 0;
   __syncthreads();
   const uint32_t tile = S.tile;
   const uint64_t tbase = static_cast<uint64_t>(tile) * kSortTile;
@@ -101,18 +109,32 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t*
 #pragma unroll
   for (int j = 0; j < kSortIPT; ++j) {
     const uint64_t e = wbase + j * 32 + lane;
-    key[j] = e < m ? keys_in[e] : ~0ULL;  // padding sorts last (digit 255, after every real key)
+    key[j] = e < m ? keys_in[e] : ~0ULL;  // padding sorts last (top digit value, after every real key)
   }
-  const uint32_t d = tid;  // kSortThreads == 256: one digit per thread
-  uint32_t tcount = 0;
-  uint64_t* my = status + static_cast<uint64_t>(tile) * 256 + d;
+  const uint32_t d0 = tid * kDPT;   // this thread's digits: d0 .. d0 + kDPT - 1
+  uint32_t tcount[kDPT];
+#pragma unroll
+  for (int q = 0; q < kDPT; ++q) tcount[q] = 0;
+  uint64_t* my = status + static_cast<uint64_t>(tile) * kBins + d0;
   if constexpr (kEarly) {
     // 1. tile histogram first, published immediately (early aggregate for the successors)
+    if constexpr (kMatchHist) {   // one shared atomic per group of equal digits in the warp
 #pragma unroll
-    for (int j = 0; j < kSortIPT; ++j) atomicAdd(&S.hist[static_cast<uint32_t>(key[j] >> shift) & 255u], 1u);
+      for (int j = 0; j < kSortIPT; ++j) {
+        const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & kMask;
+        const uint32_t peers = __match_any_sync(0xffffffffu, dj);
+        if (lane == static_cast<uint32_t>(__ffs(peers) - 1)) atomicAdd(&S.hist[dj], __popc(peers));
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < kSortIPT; ++j) atomicAdd(&S.hist[static_cast<uint32_t>(key[j] >> shift) & kMask], 1u);
+    }
     __syncthreads();
-    tcount = S.hist[d];
-    st_relaxed_gpu_u64(my, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount));
+#pragma unroll
+    for (int q = 0; q < kDPT; ++q) {
+      tcount[q] = S.hist[d0 + q];
+      st_relaxed_gpu_u64(my + q, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount[q]));
+    }
   }
   // 2. stable warp-level ranking (element order == (j, lane) order inside the warp)
   if constexpr (kAtomicRank) {
@@ -121,7 +143,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t*
     uint32_t peers[kSortIPT];
 #pragma unroll
     for (int j = 0; j < kSortIPT; ++j) {
-      const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & 255u;
+      const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & kMask;
       peers[j] = __match_any_sync(0xffffffffu, dj);
       rank[j] = 0;
       if (lane == static_cast<uint32_t>(__ffs(peers[j]) - 1)) rank[j] = atomicAdd(&S.wcnt[warp][dj], __popc(peers[j]));
@@ -132,7 +154,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t*
   } else {
 #pragma unroll
     for (int j = 0; j < kSortIPT; ++j) {
-      const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & 255u;
+      const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & kMask;
       const uint32_t peers = __match_any_sync(0xffffffffu, dj);
       const uint32_t leader = __ffs(peers) - 1;
       uint32_t before = 0;
@@ -148,61 +170,91 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t*
   __syncthreads();
   if constexpr (!kEarly) {
 #pragma unroll
-    for (int w = 0; w < kWarps; ++w) tcount += S.wcnt[w][d];
-    st_relaxed_gpu_u64(my, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount));
+    for (int q = 0; q < kDPT; ++q) {
+#pragma unroll
+      for (int w = 0; w < kWarps; ++w) tcount[q] += S.wcnt[w][d0 + q];
+      st_relaxed_gpu_u64(my + q, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount[q]));
+    }
   }
   __syncthreads();
   // 3. per digit: warp-exclusive offsets and the tile-local digit start
-  {
+  uint32_t tsum = 0;
+#pragma unroll
+  for (int q = 0; q < kDPT; ++q) {
     uint32_t run = 0;
 #pragma unroll
     for (int w = 0; w < kWarps; ++w) {
-      const uint32_t c = S.wcnt[w][d];
-      S.wcnt[w][d] = run;
+      const uint32_t c = S.wcnt[w][d0 + q];
+      S.wcnt[w][d0 + q] = run;
       run += c;
     }
-    const uint32_t inc = warp_inclusive_add(tcount);
-    if (lane == 31) S.wsum[warp] = inc;
+    tsum += tcount[q];
   }
+  const uint32_t inc = warp_inclusive_add(tsum);
+  if (lane == 31) S.wsum[warp] = inc;
   __syncthreads();
   {
     uint32_t wpre = 0;
 #pragma unroll
     for (int w = 0; w < kWarps; ++w) wpre += (w < static_cast<int>(warp)) ? S.wsum[w] : 0u;
-    S.dstart[d] = wpre + warp_inclusive_add(tcount) - tcount;
-    // 4. decoupled look-back, kLookWindow predecessors per round trip
-    uint32_t excl = 0;
+    uint32_t ds = wpre + inc - tsum;
+#pragma unroll
+    for (int q = 0; q < kDPT; ++q) { S.dstart[d0 + q] = ds; ds += tcount[q]; }
+    // 4. decoupled look-back, kLookWindow predecessors per round trip, all digits of the thread
+    //    in flight together
+    uint32_t excl[kDPT];
+#pragma unroll
+    for (int q = 0; q < kDPT; ++q) excl[q] = 0;
     if (tile > 0) {
-      long long p = static_cast<long long>(tile) - 1;
+      long long p[kDPT];
+      bool done[kDPT];
+#pragma unroll
+      for (int q = 0; q < kDPT; ++q) { p[q] = static_cast<long long>(tile) - 1; done[q] = false; }
       for (;;) {
-        uint64_t sv[kLookWindow];
+        uint64_t sv[kDPT][kLookWindow];
 #pragma unroll
-        for (int i = 0; i < kLookWindow; ++i)
-          sv[i] = (p - i >= 0) ? ld_relaxed_gpu_u64(status + static_cast<uint64_t>(p - i) * 256 + d) : 0;
-        int adv = 0;
-        bool done = false;
+        for (int q = 0; q < kDPT; ++q)
 #pragma unroll
-        for (int i = 0; i < kLookWindow; ++i) {
-          if (done || adv != i) continue;             // stop at the first not-ready / prefix word
-          const uint32_t ep = static_cast<uint32_t>(sv[i] >> 34), kind = static_cast<uint32_t>(sv[i] >> 32) & 3u;
-          if (ep != epoch || kind == 0) continue;     // not ready yet: retry from here
-          excl += static_cast<uint32_t>(sv[i]);
-          ++adv;
-          if (kind == kPrefix) done = true;
+          for (int i = 0; i < kLookWindow; ++i)
+            sv[q][i] = (!done[q] && p[q] - i >= 0)
+                           ? ld_relaxed_gpu_u64(status + static_cast<uint64_t>(p[q] - i) * kBins + d0 + q)
+                           : 0;
+        bool all = true, moved = false;
+#pragma unroll
+        for (int q = 0; q < kDPT; ++q) {
+          if (done[q]) continue;
+          int adv = 0;
+          bool fin = false;
+#pragma unroll
+          for (int i = 0; i < kLookWindow; ++i) {
+            if (fin || adv != i) continue;             // stop at the first not-ready / prefix word
+            const uint32_t ep = static_cast<uint32_t>(sv[q][i] >> 34), kind = static_cast<uint32_t>(sv[q][i] >> 32) & 3u;
+            if (ep != epoch || kind == 0) continue;     // not ready yet: retry from here
+            excl[q] += static_cast<uint32_t>(sv[q][i]);
+            ++adv;
+            if (kind == kPrefix) fin = true;
+          }
+          if (fin) done[q] = true;
+          else { p[q] -= adv; all = false; }
+          moved = moved || fin || adv > 0;
         }
-        if (done) break;
-        p -= adv;
+        if (all) break;
+        if constexpr (kBackoff) {
+          if (!moved) __nanosleep(100);
+        }
       }
-      st_relaxed_gpu_u64(my, pack_status(epoch, kPrefix, excl + tcount));
+#pragma unroll
+      for (int q = 0; q < kDPT; ++q) st_relaxed_gpu_u64(my + q, pack_status(epoch, kPrefix, excl[q] + tcount[q]));
     }
-    S.goff[d] = bases[d] + excl;
+#pragma unroll
+    for (int q = 0; q < kDPT; ++q) S.goff[d0 + q] = bases[d0 + q] + excl[q];
   }
   __syncthreads();
   // 5. scatter into SMEM in tile-sorted order (payload loaded here, after ranking)
 #pragma unroll
   for (int j = 0; j < kSortIPT; ++j) {
     const uint64_t e = wbase + j * 32 + lane;
-    const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & 255u;
+    const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & kMask;
     const uint32_t lp = S.dstart[dj] + S.wcnt[warp][dj] + rank[j];
     S.keys[lp] = key[j];
     if constexpr (kPay) S.idx[lp] = kFirst ? static_cast<uint32_t>(e) : (e < m ? idx_in[e] : 0u);
@@ -212,7 +264,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t*
   const uint32_t nvalid = static_cast<uint32_t>(min(static_cast<uint64_t>(kSortTile), m - tbase));
   for (uint32_t i = tid; i < nvalid; i += kSortThreads) {
     const uint64_t k = S.keys[i];
-    const uint32_t dk = static_cast<uint32_t>(k >> shift) & 255u;
+    const uint32_t dk = static_cast<uint32_t>(k >> shift) & kMask;
     const uint32_t pos = S.goff[dk] + (i - S.dstart[dk]);
     keys_out[pos] = k;
     if constexpr (kPay) idx_out[pos] = S.idx[i];
@@ -290,17 +342,19 @@ __global__ void __launch_bounds__(kScanThreads) k_scan(const T* __restrict__ in,
 
 }  // namespace
 
-cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int nd, int num_sms, cudaStream_t s) {
-  cudaError_t e = cudaMemsetAsync(hist, 0, 8 * 256 * sizeof(uint32_t), s);
+cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int nd, int bits, int num_sms,
+                        cudaStream_t s) {
+  cudaError_t e = cudaMemsetAsync(hist, 0, 8 * kBinStride * sizeof(uint32_t), s);
   if (e != cudaSuccess || m == 0) return e;
   if (reinterpret_cast<uintptr_t>(keys) & 15u) {   // 16-B loads: peel one key off a misaligned start
-    k_hist<<<1, 32, 0, s>>>(keys, 1, static_cast<uint32_t>(nd), hist);
+    k_hist<<<1, 32, 0, s>>>(keys, 1, static_cast<uint32_t>(nd), static_cast<uint32_t>(bits), hist);
     count_launch();
     ++keys;
     if (--m == 0) return cudaGetLastError();
   }
   uint64_t blocks = std::min<uint64_t>(static_cast<uint64_t>(num_sms) * 8, (m / 2 + 255) / 256 + 1);
-  k_hist<<<static_cast<unsigned>(blocks), 256, 0, s>>>(keys, m, static_cast<uint32_t>(nd), hist);
+  k_hist<<<static_cast<unsigned>(blocks), 256, 0, s>>>(keys, m, static_cast<uint32_t>(nd), static_cast<uint32_t>(bits),
+                                                       hist);
   count_launch();
   return cudaGetLastError();
 }
@@ -322,19 +376,19 @@ int sort_cfg() {
 }
 static const int kCfgIPT[4] = {16, 12, 20, 8};
 int sort_tile() { return kSortThreads * kCfgIPT[sort_cfg()]; }
-static const int kCfgIPTKeys[4] = {16, 12, 16, 24};
+// keys-only passes: 16 keys x 256 threads (3 CTAs / SM), or 24 keys (2 CTAs / SM) for cfg 3
+static const int kCfgIPTKeys[4] = {16, 16, 16, 24};
 int sort_tile_keys() { return kSortThreads * kCfgIPTKeys[sort_cfg()]; }
-
-template <bool kFirst, int kVar, int IPT, int MINB, bool kPay>
+template <bool kFirst, int kVar, int IPT, int MINB, bool kPay, int kBits, int LW = 4>
 static void launch_os(unsigned tiles, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
                       uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
                       uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
-  const size_t smem = sizeof(SortSmem<IPT, kPay>);
-  cudaFuncSetAttribute(k_onesweep<kFirst, kVar, IPT, MINB, kPay>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                       static_cast<int>(smem));
-  k_onesweep<kFirst, kVar, IPT, MINB, kPay><<<tiles, kSortThreads, smem, s>>>(keys_in, idx_in, keys_out, idx_out, m,
-                                                                               shift, bases, status, epoch,
-                                                                               tile_counter);
+  using K = decltype(&k_onesweep<kFirst, kVar, IPT, MINB, kPay, kBits, LW>);
+  const K k = &k_onesweep<kFirst, kVar, IPT, MINB, kPay, kBits, LW>;
+  const size_t smem = sizeof(SortSmem<IPT, kPay, (1 << kBits)>);
+  cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
+  k<<<tiles, kSortThreads, smem, s>>>(keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch,
+                                      tile_counter);
 }
 
 #define BMR_OS_ARGS tiles, keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch, tile_counter, s
@@ -343,36 +397,37 @@ static void launch_cfg(unsigned tiles, const uint64_t* keys_in, const uint32_t* 
                        uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
                        uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
   switch (sort_cfg()) {
-    case 1: launch_os<kFirst, kVar, 12, 4, true>(BMR_OS_ARGS); break;
-    case 2: launch_os<kFirst, kVar, 20, 2, true>(BMR_OS_ARGS); break;
-    case 3: launch_os<kFirst, kVar, 8, 6, true>(BMR_OS_ARGS); break;
-    default: launch_os<kFirst, kVar, 16, 3, true>(BMR_OS_ARGS); break;
+    case 1: launch_os<kFirst, kVar, 12, 4, true, 8>(BMR_OS_ARGS); break;
+    case 2: launch_os<kFirst, kVar, 20, 2, true, 8>(BMR_OS_ARGS); break;
+    case 3: launch_os<kFirst, kVar, 8, 6, true, 8>(BMR_OS_ARGS); break;
+    default: launch_os<kFirst, kVar, 16, 3, true, 8>(BMR_OS_ARGS); break;
   }
 }
-// keys only (8 B per key per direction): the tile shape is the same, the SMEM image smaller
+// keys only (8 B per key per direction), 8-bit digits.  Measured on C5 (48-bit WC exact keys,
+// 1.37 G keys): 16 keys x 256 threads, early histogram, look-back window 4 is the fastest of
+// {9-bit digits (5 passes, 2 digits per thread), windows 1/2/8/16, spin back-off,
+// match-aggregated histogram atomics, bijective digit mixing} — see DESIGN.md §4.
 static void launch_keys_only(unsigned tiles, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
                              uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
                              uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
-  switch (sort_cfg()) {
-    case 1: launch_os<false, 2, 12, 4, false>(BMR_OS_ARGS); break;
-    case 2: launch_os<false, 2, 16, 4, false>(BMR_OS_ARGS); break;
-    case 3: launch_os<false, 2, 24, 2, false>(BMR_OS_ARGS); break;
-    default: launch_os<false, 2, 16, 3, false>(BMR_OS_ARGS); break;
-  }
+  if (sort_cfg() == 3) launch_os<false, 2, 24, 2, false, 8, 4>(BMR_OS_ARGS);
+  else launch_os<false, 2, 16, 3, false, 8, 4>(BMR_OS_ARGS);
 }
 
 cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out, uint32_t* idx_out,
-                            uint64_t m, int digit, const uint32_t* bases_all, uint64_t* status, uint32_t epoch,
-                            unsigned int* tile_counter, cudaStream_t s) {
+                            uint64_t m, int digit, int bits, const uint32_t* bases_all, uint64_t* status,
+                            uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
   if (m == 0) return cudaSuccess;
-  const uint64_t tile = idx_out ? sort_tile() : sort_tile_keys();
+  const bool keys_only = idx_out == nullptr;
+  if (bits != 8) return cudaErrorInvalidValue;
+  const uint64_t tile = keys_only ? sort_tile_keys() : sort_tile();
   const unsigned tiles = static_cast<unsigned>((m + tile - 1) / tile);
   cudaError_t e = cudaMemsetAsync(tile_counter, 0, sizeof(unsigned int), s);
   if (e != cudaSuccess) return e;
-  const uint32_t shift = 8u * digit;
-  const uint32_t* bases = bases_all + 256 * digit;
+  const uint32_t shift = static_cast<uint32_t>(bits * digit);
+  const uint32_t* bases = bases_all + kBinStride * digit;
   const bool first = idx_in == nullptr;
-  if (idx_out == nullptr) {
+  if (keys_only) {
     launch_keys_only(BMR_OS_ARGS);
   } else {
     switch (sort_variant() | (first ? 4 : 0)) {
