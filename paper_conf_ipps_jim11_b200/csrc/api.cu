@@ -629,7 +629,7 @@ mr_status mr_group(mr_job* job) {
   if (split) {
     // exact stream: keys only (the key is the record), no byte verification needed
     CK(run_sort(job->sw, job->h.p, m_total, &job->skeys, nullptr, job->st, job->nsm, job->stream, &job->prof,
-                &job->stats.hist_ms, &job->stats.sort_keys_ms, 44),   // exact keys < 2^44 (common.cuh)
+                &job->stats.hist_ms, &job->stats.sort_keys_ms, kExactBits),   // exact keys < 2^30
        "radix sort (exact)");
     job->stats.sort_passes += job->sw.passes;
     job->stats.sort_passes_keys += job->sw.passes;

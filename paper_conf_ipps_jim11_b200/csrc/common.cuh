@@ -142,11 +142,10 @@ __device__ __forceinline__ uint64_t hash_bytes(const uint8_t* p, uint32_t len, u
 // passes fewer; digits 6 and 7 are then constant and skipped):
 //   inline  : keys of <= kInlineMax bytes packed little-endian, length in the 3 bits above them
 //             (64: len << 56, <= 7 bytes; 48: len << 40, <= 5 bytes) — injective, top bit clear;
-//   alnum   : (48 only) [0-9A-Za-z] keys of 6..7 bytes: 2^43 | 6-bit symbol codes (1..62, so
-//             the length is implied) — every exact 48-bit key is < 2^44 (five 9-bit digits);
 //   hashed  : longer keys -> hash with the top bit of the width forced to 1 (never collides with
 //             an inline key); equal hashes are verified byte-for-byte at segment time;
 //   sentinel: all ones in the width — flush filler pairs, sorts after every real key.
+// The WordCount exact stream (map.cu) uses its own 30-bit format, exact_key30 below.
 __host__ __device__ __forceinline__ uint32_t inline_max(uint32_t bits) { return bits == 48 ? 5u : 7u; }
 __host__ __device__ __forceinline__ uint64_t hashed_bit(uint32_t bits) { return 1ULL << (bits - 1); }
 __host__ __device__ __forceinline__ uint64_t sentinel_of(uint32_t bits) {
@@ -162,37 +161,33 @@ __device__ __forceinline__ uint64_t hashed_key(uint64_t h, bool weak, uint32_t b
 __device__ __forceinline__ uint64_t inline_key(uint64_t bytes_le, uint32_t len, uint32_t bits = 64) {
   return (bytes_le & ((1ULL << (8 * len)) - 1ULL)) | (static_cast<uint64_t>(len) << (bits - 8));
 }
-// 48-bit (WordCount) keys of 6..7 bytes: a WC word is [0-9A-Za-z]+ (C-3 #1), so each symbol
-// has a nonzero 6-bit code (1..62); 6 or 7 codes (<= 42 bits, the highest nonzero code gives
-// the length) above a 2^43 tag pack injectively — disjoint from the byte-packed keys (< 2^43)
-// and from the hashed ones (bit 47).
-__device__ __forceinline__ bool alnum_byte(uint32_t c) {
-  return (c - '0' < 10u) || (c - 'A' < 26u) || (c - 'a' < 26u);
+
+// WordCount exact keys: a WC word is [0-9A-Za-z]+ (C-3 #1), so every symbol has a nonzero 6-bit
+// code: '0'-'9' -> 1..10, 'A'-'Z' -> 11..36, 'a'-'z' -> 37..62.  A word of <= 5 symbols packs
+// injectively into 30 bits (symbol i at bits 6i; the highest nonzero code gives the length):
+// four 8-bit LSD digits.  Codes of 4 bytes at once: code = low nibble + base[high nibble], the
+// 5-entry base table looked up with one byte permute (PRMT) indexed by the high nibbles.
+__device__ __forceinline__ uint32_t exact_codes4(uint32_t w) {
+  const uint32_t hi = (w >> 4) & 0x0F0F0F0Fu;                  // 3 digit, 4-5 upper, 6-7 lower
+  const uint32_t h2 = hi | (hi >> 4);
+  const uint32_t sel = (h2 & 0xFFu) | ((h2 >> 8) & 0xFF00u);   // four selector nibbles
+  // table bytes 3..7 = {1, 10, 26, 36, 52}: '0' (low 0) -> 1, 'A' (low 1) -> 11, 'P' (low 0) -> 26,
+  // 'a' (low 1) -> 37, 'p' (low 0) -> 52
+  const uint32_t base = __byte_perm(0x01000000u, 0x34241A0Au, sel);
+  return (w & 0x0F0F0F0Fu) + base;                             // <= 62 per byte: no carries
 }
-__device__ __forceinline__ uint64_t alnum_key48(uint64_t bytes_le, uint32_t len) {
-  // SWAR: per byte code = c - 47 - 7 [c > '9'] - 6 [c > 'Z'], then bytes beyond len cleared and
-  // the eight 6-bit codes compressed (byte -> 12-bit pairs -> 24-bit quads -> 48 bits).
-  const auto codes = [](uint32_t w) {
-    const uint32_t g9 = __vcmpgtu4(w, 0x39393939u) & 0x07070707u;
-    const uint32_t gz = __vcmpgtu4(w, 0x5A5A5A5Au) & 0x06060606u;
-    return __vsub4(__vsub4(__vsub4(w, 0x2F2F2F2Fu), g9), gz);
-  };
-  uint64_t x = (static_cast<uint64_t>(codes(static_cast<uint32_t>(bytes_le >> 32))) << 32) |
-               codes(static_cast<uint32_t>(bytes_le));
-  x &= (1ULL << (8 * len)) - 1ULL;  // len <= 7
-  x = (x & 0x003F003F003F003FULL) | ((x >> 2) & 0x0FC00FC00FC00FC0ULL);
-  x = (x & 0x00000FFF00000FFFULL) | ((x >> 4) & 0x00FFF00000FFF000ULL);
-  x = (x & 0x0000000000FFFFFFULL) | ((x >> 8) & 0x0000FFFFFF000000ULL);
-  return x | (1ULL << 43);
+__device__ __forceinline__ uint64_t exact_key30(uint64_t bytes_le, uint32_t len) {   // len 1..5
+  uint64_t x = (static_cast<uint64_t>(exact_codes4(static_cast<uint32_t>(bytes_le >> 32))) << 32) |
+               exact_codes4(static_cast<uint32_t>(bytes_le));
+  x &= (1ULL << (8 * len)) - 1ULL;
+  x = (x & 0x003F003F003F003FULL) | ((x >> 2) & 0x0FC00FC00FC00FC0ULL);   // byte pairs -> 12 bits
+  x = (x & 0x00000FFF00000FFFULL) | ((x >> 4) & 0x00FFF00000FFF000ULL);   // -> 24 bits
+  x = (x & 0x0000000000FFFFFFULL) | ((x >> 8) & 0x0000FFFFFF000000ULL);   // -> 48 bits
+  return x;
 }
-// Inverse of the 48-bit exact formats (inline <= 5 bytes, alnum 6..7): key bytes little-endian.
-__device__ __forceinline__ uint64_t exact_key_bytes48(uint64_t key, uint32_t& len) {
-  if (key < (1ULL << 43)) {
-    len = static_cast<uint32_t>(key >> 40) & 7u;
-    return key & ((1ULL << 40) - 1ULL);
-  }
-  const uint64_t codes = key & ((1ULL << 42) - 1ULL);
-  len = codes ? static_cast<uint32_t>(63 - __clzll(static_cast<long long>(codes))) / 6u + 1u : 0u;
+// Inverse: key bytes little-endian and the length.
+__device__ __forceinline__ uint64_t exact_key_bytes(uint64_t key, uint32_t& len) {
+  len = key ? static_cast<uint32_t>(63 - __clzll(static_cast<long long>(key))) / 6u + 1u : 0u;
   uint64_t b = 0;
   for (uint32_t i = 0; i < len; ++i) {
     const uint32_t c = static_cast<uint32_t>(key >> (6 * i)) & 63u;
@@ -200,18 +195,13 @@ __device__ __forceinline__ uint64_t exact_key_bytes48(uint64_t key, uint32_t& le
   }
   return b;
 }
-// key bytes -> sort key (generic pointer)
+// key bytes -> sort key (generic pointer), inline / hashed formats
 __device__ __forceinline__ uint64_t key_of_bytes(const uint8_t* p, uint32_t len, uint64_t seed, bool weak,
                                                  uint32_t bits) {
-  if (len <= inline_max(bits) || (bits == 48 && len <= 7)) {
+  if (len <= inline_max(bits)) {
     uint64_t b = 0;
-    bool alnum = true;
-    for (uint32_t k = 0; k < len; ++k) {
-      b |= static_cast<uint64_t>(p[k]) << (8 * k);
-      alnum = alnum && alnum_byte(p[k]);
-    }
-    if (len <= inline_max(bits)) return inline_key(b, len, bits);
-    if (alnum) return alnum_key48(b, len);
+    for (uint32_t k = 0; k < len; ++k) b |= static_cast<uint64_t>(p[k]) << (8 * k);
+    return inline_key(b, len, bits);
   }
   return hashed_key(hash_bytes(p, len, seed), weak, bits);
 }

@@ -48,7 +48,7 @@ __device__ __forceinline__ Rec get_rec(const XSource& S, uint64_t i) {
     if (i < S.nx) {
       const uint64_t key = S.hx[i];
       if (key == sentinel_of(48)) { r.dest = ~0u; return r; }   // flush filler
-      r.kin = exact_key_bytes48(key, r.klen);
+      r.kin = exact_key_bytes(key, r.klen);
       r.dest = dest_of_bytes(reinterpret_cast<const uint8_t*>(&r.kin), r.klen, S.nranks);
       r.heap = (r.klen + 7u) & ~7u;
       return r;

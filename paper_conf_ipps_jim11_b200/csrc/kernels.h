@@ -12,6 +12,9 @@ extern std::atomic<unsigned long long> g_kernel_launches;
 inline void count_launch(unsigned n = 1) { g_kernel_launches.fetch_add(n, std::memory_order_relaxed); }
 
 enum Workload : int { kWC = 1, kSM = 2, kKM = 3, kII = 4 };
+// WordCount exact stream: words of <= kExactMax bytes, keys < 2^kExactBits (common.cuh)
+constexpr uint32_t kExactMax = 5;
+constexpr uint32_t kExactBits = 30;
 
 // Device-resident job state (one per job).
 struct DevState {

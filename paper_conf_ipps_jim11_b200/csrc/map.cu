@@ -57,16 +57,16 @@ struct Cfg {
   // TMA traffic stay in flight per SM while one stage is being consumed
   static constexpr int kLag = kStages - 2;
   // WC: per-warp queue of the window's long (hashed) words, hashed by all 32 lanes together
-  // after the emission rounds (a lane-per-word hash inside the rounds diverges: with 7% long
-  // words, 9 in 10 rounds would carry at least one).  A window holds at most 512 / 8 starts of
-  // words longer than kWcExact bytes.
-  static constexpr int kHashQ = (W == kWC) ? 64 : 0;
+  // after the emission rounds (a lane-per-word hash inside the rounds diverges: with 10% long
+  // words, most rounds would carry at least one).  A window holds at most 512 / 6 + 1 starts
+  // of words longer than kWcExact bytes.
+  static constexpr int kHashQ = (W == kWC) ? 96 : 0;
 };
-// WC words of <= kWcExact bytes get an exact 48-bit key (byte-packed <= 5, alnum-packed 6..7,
-// common.cuh) and travel in the exact stream (8-B entries: the key is the whole record); longer
-// words are hashed and travel with their key reference in the hashed stream (16-B entries).
-constexpr uint32_t kWcExact = 7;
-static_assert(kWin / (kWcExact + 1) <= Cfg<kWC>::kHashQ, "hash queue too small");
+// WC words of <= kWcExact bytes get an exact 30-bit key (common.cuh exact_key30) and travel in
+// the exact stream (8-B entries: the key is the whole record); longer words are hashed and
+// travel with their key reference in the hashed stream (16-B entries).
+constexpr uint32_t kWcExact = kExactMax;
+static_assert(kWin / (kWcExact + 1) + 1 <= Cfg<kWC>::kHashQ, "hash queue too small");
 constexpr int kKmPts = kT / 32;                // 512 points per KM tile
 
 static_assert(kLead + kT + kHalo + 32 <= kStageBytes, "stage too small");
@@ -366,7 +366,7 @@ __device__ __forceinline__ uint32_t units(uint32_t c) {   // buffer space of pac
   else return cur_ca(c);
 }
 static_assert(PairFmt<kWC>::kCap + kNMap * PairFmt<kWC>::kMaxReserve <= kCaMask, "ca field overflow");
-static_assert(PairFmt<kWC>::kCap / 2 + kNMap * 64 <= kCbMask, "cb field overflow");
+static_assert(PairFmt<kWC>::kCap / 2 + kNMap * Cfg<kWC>::kHashQ <= kCbMask, "cb field overflow");
 static_assert(PairFmt<kSM>::kCap + kNMap * PairFmt<kSM>::kMaxReserve <= kCaMask, "ca field overflow");
 
 template <int W>
@@ -719,7 +719,7 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
     const uint32_t ma = __ballot_sync(kFull, ex), mb = __ballot_sync(kFull, act && !ex);
     if (ex) {
       const uint64_t b = window8(x, j);     // an exact word lies inside the 32 loaded bytes
-      sh[ka + __popc(ma & lanemask_lt())] = len <= inline_max(48) ? inline_key(b, len, 48) : alnum_key48(b, len);
+      sh[ka + __popc(ma & lanemask_lt())] = exact_key30(b, len);
     } else if (act) {
       if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
       hq[nq + __popc(mb & lanemask_lt())] = static_cast<uint64_t>(p0 + j - tv.sbase) | (static_cast<uint64_t>(len) << 24);

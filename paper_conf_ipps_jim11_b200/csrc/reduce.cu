@@ -367,7 +367,7 @@ __global__ void k_key_lengths_exact(const uint64_t* seg, uint64_t nseg, const ui
   const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
   if (s >= nseg) return;
   uint32_t len;
-  exact_key_bytes48(sk[seg[s]], len);
+  exact_key_bytes(sk[seg[s]], len);
   lens[s] = len;
 }
 __global__ void k_key_decode(const uint64_t* seg, uint64_t nseg, const uint64_t* sk, const uint64_t* key_off,
@@ -375,7 +375,7 @@ __global__ void k_key_decode(const uint64_t* seg, uint64_t nseg, const uint64_t*
   const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
   if (s >= nseg) return;
   uint32_t len;
-  const uint64_t b = exact_key_bytes48(sk[seg[s]], len);
+  const uint64_t b = exact_key_bytes(sk[seg[s]], len);
   uint8_t* dst = keys + key_off[s];
   for (uint32_t i = 0; i < len; ++i) dst[i] = static_cast<uint8_t>(b >> (8 * i));
 }
