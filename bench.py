@@ -187,21 +187,24 @@ def run_reference(args, rank, world):
 def algorithmic(inp, st, steps):
     """Algorithmic bytes per step of each phase.
 
-    WordCount Map output is two streams: exact keys (8 B, sorted keys-only: 8 B read + 8 B
-    written per pass) and hashed keys (key + kref, 16 B; sorted with a u32 permutation:
-    24 B per pass, the first pass reads no permutation)."""
+    WordCount Map output is three streams: exact keys (words <= 5 bytes) and mid keys (6..8
+    bytes) are bare 8-B keys sorted keys-only (8 B read + 8 B written per pass); hashed keys
+    (longer words) carry a key reference (16 B) and sort with a u32 permutation (24 B per pass,
+    the first pass reads no permutation)."""
     wl = inp["wl"]
     m = st["pairs"] / steps
     mh = st["pairs_hashed"] / steps
-    mx = m - mh
+    mc = st["pairs_mid"] / steps
+    mx = m - mh - mc
     n = inp["n"]
     off_b = 8 * (n + 1) if inp["offsets"] is not None else 0
     px = st["sort_passes_keys"] / steps
+    pc = st["sort_passes_mid"] / steps
     passes = st["sort_passes"] / steps
     if wl == "wc":
-        map_b = inp["nbytes"] + off_b + mx * 8 + mh * 16
-        ph = passes - px
-        sort_b = px * 16 * mx + ((ph * 24 - 4) * mh if ph else 0.0)
+        map_b = inp["nbytes"] + off_b + (mx + mc) * 8 + mh * 16
+        ph = passes - px - pc
+        sort_b = px * 16 * mx + pc * 16 * mc + ((ph * 24 - 4) * mh if ph else 0.0)
     else:
         map_b = inp["nbytes"] + off_b + m * {"sm": 8, "km": 40, "ii": 24}[wl]
         sort_b = (passes * 24 - 4) * m if passes else 0.0   # first pass reads no payload
@@ -268,7 +271,7 @@ def main():
     # timed region: K steps, per-phase device times from the job's CUDA events
     acc = {k: 0.0 for k in ("map_ms", "hist_ms", "sort_ms", "seg_ms", "sort_keys_ms")}
     tot = {"pairs": 0, "sort_passes": 0, "kernel_launches": 0, "flushes": 0, "n_keys": 0, "pairs_hashed": 0,
-           "sort_passes_keys": 0}
+           "sort_passes_keys": 0, "pairs_mid": 0, "sort_passes_mid": 0}
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         barrier()
@@ -399,6 +402,8 @@ def main():
             "map": {"achieved_gbs": round(map_ach, 1), "frac": round(map_ach / hbm, 4),
                     "bytes_per_step": int(alg["map"])},
             "pairs_per_step": int(alg["pairs"]), "sort_passes": alg["passes"],
+            "wc_streams": ({"exact": int(alg["pairs_exact"]), "mid": int(tot["pairs_mid"] / args.steps),
+                            "hashed": int(tot["pairs_hashed"] / args.steps)} if inp["wl"] == "wc" else None),
             "distinct_keys": int(tot["n_keys"] / args.steps),
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "exchange": ({"kind": "hash all-to-all over NCCL (torch.distributed)", "send_bytes_per_rank": xbytes[0],

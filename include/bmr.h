@@ -96,12 +96,16 @@ typedef struct {
   uint64_t kernel_launches;/* libbmr kernels launched since create / reset */
   /* MR_FLAG_PROFILE: device time per phase (CUDA events on the job stream), ms */
   double map_ms, hist_ms, sort_ms, seg_ms, reduce_ms;
-  /* WordCount two-stream Map output: pairs of the hashed stream (included in
+  /* WordCount Map output streams: pairs of the hashed stream (included in
    * `pairs`), LSD passes of the keys-only exact-stream sort (included in `sort_passes`) and
    * their device time (included in `sort_ms`) */
   uint64_t pairs_hashed;
   uint64_t sort_passes_keys;
   double sort_keys_ms;
+  /* WordCount mid stream (6..8-byte words, exact 48-bit keys, sorted keys-only): pairs and LSD
+   * passes (included in `pairs` / `sort_passes`; its device time is in `sort_ms`) */
+  uint64_t pairs_mid;
+  uint64_t sort_passes_mid;
 } mr_stats;
 
 /* State machine: CREATED -> mr_map x k (batches append) -> mr_group -> mr_reduce -> mr_fetch

@@ -63,7 +63,8 @@ class Stats(C.Structure):
     _fields_ = [(n, C.c_uint64) for n in ("pairs", "flushes", "replays", "n_keys", "collisions", "sort_passes",
                                           "map_tiles", "input_bytes", "capacity_pairs", "kernel_launches")] + \
                [(n, C.c_double) for n in ("map_ms", "hist_ms", "sort_ms", "seg_ms", "reduce_ms")] + \
-               [("pairs_hashed", C.c_uint64), ("sort_passes_keys", C.c_uint64), ("sort_keys_ms", C.c_double)]
+               [("pairs_hashed", C.c_uint64), ("sort_passes_keys", C.c_uint64), ("sort_keys_ms", C.c_double),
+                ("pairs_mid", C.c_uint64), ("sort_passes_mid", C.c_uint64)]
 
 
 _LIB = None

@@ -221,7 +221,7 @@ struct mr_job {
   size_t host_batches = 0;
   Prof prof;
   unsigned long long launches0 = 0;
-  SortWork sw, swb;
+  SortWork sw, swb, swc;
   const uint64_t* skeys = nullptr;
   const uint32_t* perm = nullptr;
   uint64_t m = 0, nseg = 0, key_bytes = 0;
@@ -229,6 +229,11 @@ struct mr_job {
   DBuf<uint64_t> hb, krefb, seg_startb;
   uint64_t* sega = nullptr;       // exact-stream segment starts (in the free sort buffer)
   uint64_t cap_b = 0, mb = 0, nseg_a = 0, nseg_b = 0;
+  // WC mid stream (6..8-byte words, exact 48-bit keys, keys only)
+  DBuf<uint64_t> hc;
+  uint64_t cap_c = 0, mc = 0, nseg_c = 0;
+  const uint64_t* skeysc = nullptr;
+  uint64_t* segc = nullptr;
   const uint64_t* skeysb = nullptr;
   const uint32_t* permb = nullptr;
   uint32_t key_bits_b = 48;
@@ -287,8 +292,8 @@ uint64_t initial_cap(const mr_job* job, uint64_t nbytes, uint64_t n) {
   }
 }
 
-// cap_b: WC hashed-stream capacity (0 for the other workloads)
-cudaError_t ensure_pairs(mr_job* job, uint64_t cap, uint64_t cap_b) {
+// cap_b / cap_c: WC hashed / mid stream capacities (0 for the other workloads)
+cudaError_t ensure_pairs(mr_job* job, uint64_t cap, uint64_t cap_b, uint64_t cap_c) {
   cudaError_t e;
   if ((e = job->h.ensure(cap))) return e;
   if (has_kref(job->cfg.workload) && (e = job->kref.ensure(cap))) return e;
@@ -299,11 +304,14 @@ cudaError_t ensure_pairs(mr_job* job, uint64_t cap, uint64_t cap_b) {
     if ((e = job->hb.ensure(cap_b)) || (e = job->krefb.ensure(cap_b))) return e;
   }
   job->cap_b = cap_b;
+  if (cap_c && (e = job->hc.ensure(cap_c))) return e;
+  job->cap_c = cap_c;
   return cudaSuccess;
 }
 void release_pairs(mr_job* job) {
   job->h.release(); job->kref.release(); job->v.release(); job->hb.release(); job->krefb.release();
-  job->cap = job->cap_b = 0;
+  job->hc.release();
+  job->cap = job->cap_b = job->cap_c = 0;
 }
 
 cudaError_t launch_batch(mr_job* job, const Batch& b) {
@@ -326,6 +334,8 @@ cudaError_t launch_batch(mr_job* job, const Batch& b) {
   a.out.hb = job->hb.p;
   a.out.krefb = job->krefb.p;
   a.out.cap_b = job->cap_b;
+  a.out.hc = job->hc.p;
+  a.out.cap_c = job->cap_c;
   a.st = job->st;
   a.hash_seed = 0x5EEDB200ULL;
   a.key_bits = job->key_bits;
@@ -404,17 +414,20 @@ mr_status settle_map(mr_job* job) {
   DevState* hs = job->st_h.p;
   if (hs->err & kErrKeyTooLong) return fail(job, MR_ERR_OVERFLOW, "an emitted key exceeds 65535 bytes");
   const uint64_t m = hs->pair_cursor, mb = job->split() ? hs->pair_cursor_b : 0;
-  if (m > job->cap || mb > job->cap_b) {
+  const uint64_t mc = job->split() ? hs->pair_cursor_c : 0;
+  if (m > job->cap || mb > job->cap_b || mc > job->cap_c) {
     const uint64_t ncap = std::max(job->cap, m + m / 8 + 4096);
     const uint64_t ncap_b = job->split() ? std::max(job->cap_b, mb + mb / 8 + 4096) : 0;
+    const uint64_t ncap_c = job->split() ? std::max(job->cap_c, mc + mc / 8 + 4096) : 0;
     release_pairs(job);
-    CK(ensure_pairs(job, ncap, ncap_b), "grow intermediate");
-    job->stats.capacity_pairs = job->cap + job->cap_b;
+    CK(ensure_pairs(job, ncap, ncap_b, ncap_c), "grow intermediate");
+    job->stats.capacity_pairs = job->cap + job->cap_b + job->cap_c;
     CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
     for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
     job->stats.replays += job->batches.size();
     CK(read_state(job), "replay (async)");
-    if (hs->pair_cursor > job->cap || (job->split() && hs->pair_cursor_b > job->cap_b))
+    if (hs->pair_cursor > job->cap ||
+        (job->split() && (hs->pair_cursor_b > job->cap_b || hs->pair_cursor_c > job->cap_c)))
       return fail(job, MR_ERR_OOM, "replay still overflows");
   }
   return MR_OK;
@@ -509,7 +522,9 @@ mr_status mr_job_reset(mr_job* job) {
   job->km_partial = false;
   job->key_bits = (job->cfg.workload == MR_WORDCOUNT) ? 48u : 64u;
   job->key_bits_b = 48;
-  job->mb = job->nseg_a = job->nseg_b = 0;
+  job->mb = job->nseg_a = job->nseg_b = job->mc = job->nseg_c = 0;
+  job->skeysc = nullptr;
+  job->segc = nullptr;
   job->skeysb = nullptr;
   job->permb = nullptr;
   job->prof.collect();
@@ -553,10 +568,12 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
   if (nbytes && !records) return fail(job, MR_ERR_INVALID, "records is NULL");
   if (job->cap == 0) {
     // WC: ~1 word per 6 bytes, a few % of them longer than 7 bytes (hashed stream)
-    const uint64_t cap_b = job->cfg.workload != MR_WORDCOUNT ? 0
-                           : job->cfg.max_pairs_hint ? job->cfg.max_pairs_hint : nbytes / 24 + 4096;
-    CK(ensure_pairs(job, initial_cap(job, nbytes, n), cap_b), "alloc intermediate");
-    job->stats.capacity_pairs = job->cap + job->cap_b;
+    const bool wc = job->cfg.workload == MR_WORDCOUNT;
+    const uint64_t hint = job->cfg.max_pairs_hint;
+    const uint64_t cap_b = !wc ? 0 : hint ? hint : nbytes / 48 + 4096;
+    const uint64_t cap_c = !wc ? 0 : hint ? hint : nbytes / 32 + 4096;
+    CK(ensure_pairs(job, initial_cap(job, nbytes, n), cap_b, cap_c), "alloc intermediate");
+    job->stats.capacity_pairs = job->cap + job->cap_b + job->cap_c;
   }
   Batch b{records, offsets, n, nbytes, job->cfg.input_base + job->next_base};
   job->next_base += nbytes;
@@ -611,21 +628,26 @@ mr_status mr_group(mr_job* job) {
   const uint64_t m_total = hs->pair_cursor;            // includes the flush filler pairs (sentinel keys)
   const uint64_t m = m_total - hs->pads;
   const uint64_t mb = split ? hs->pair_cursor_b : 0;
+  const uint64_t mc = split ? hs->pair_cursor_c : 0;
   job->m = m;
   job->mb = mb;
-  job->stats.pairs = m + mb;
+  job->mc = mc;
+  job->stats.pairs = m + mb + mc;
   job->stats.pairs_hashed = mb;
+  job->stats.pairs_mid = mc;
   job->stats.flushes = hs->flushes;
-  if (m_total >= (1ULL << 32) - 1 || mb >= (1ULL << 32) - 1)
+  if (m_total >= (1ULL << 32) - 1 || mb >= (1ULL << 32) - 1 || mc >= (1ULL << 32) - 1)
     return fail(job, MR_ERR_UNSUPPORTED, ">= 2^32 intermediate pairs in one group");
   if (job->cfg.workload == MR_STRINGMATCH) {  // Map-only
     job->nseg = m;
     job->state = kGrouped;
     return MR_OK;
   }
-  job->nseg_b = 0;
+  job->nseg_b = job->nseg_c = 0;
   job->skeysb = nullptr;
   job->permb = nullptr;
+  job->skeysc = nullptr;
+  job->segc = nullptr;
   if (split) {
     // exact stream: keys only (the key is the record), no byte verification needed
     CK(run_sort(job->sw, job->h.p, m_total, &job->skeys, nullptr, job->st, job->nsm, job->stream, &job->prof,
@@ -643,6 +665,18 @@ mr_status mr_group(mr_job* job) {
     st = do_segments_into(job, job->skeys, m, job->sega, job->nseg_a);
     if (st != MR_OK) return st;
     if (job->prof.on) job->prof.end(job->stream, sp, &job->stats.seg_ms);
+    // mid stream: exact 48-bit keys, keys only (no fillers: plain stores)
+    CK(run_sort(job->swc, job->hc.p, mc, &job->skeysc, nullptr, job->st, job->nsm, job->stream, &job->prof,
+                &job->stats.hist_ms, &job->stats.sort_ms, kMidBits),
+       "radix sort (mid)");
+    job->stats.sort_passes += job->swc.passes;
+    job->stats.sort_passes_mid += job->swc.passes;
+    Prof::Span spc{};
+    if (job->prof.on) job->prof.begin(job->stream, spc);
+    job->segc = (job->skeysc == job->swc.ka.p) ? job->swc.kb.p : job->swc.ka.p;
+    st = do_segments_into(job, job->skeysc, mc, job->segc, job->nseg_c);
+    if (st != MR_OK) return st;
+    if (job->prof.on) job->prof.end(job->stream, spc, &job->stats.seg_ms);
   }
   // general stream (II / KM / ingested WC) or the WC hashed stream: sort with the permutation,
   // verify equal hashes byte for byte, re-hash and re-sort on a collision (slow path)
@@ -678,7 +712,7 @@ mr_status mr_group(mr_job* job) {
     }
     if (!split) { job->nseg_a = ns; }
   }
-  job->nseg = job->nseg_a + job->nseg_b;
+  job->nseg = job->nseg_a + job->nseg_c + job->nseg_b;
   job->stats.n_keys = job->nseg;
   Prof::Span sp3{};
   if (job->prof.on) job->prof.begin(job->stream, sp3);
@@ -687,7 +721,10 @@ mr_status mr_group(mr_job* job) {
     if (split) {
       CK(launch_key_lengths_exact(job->sega, job->nseg_a, job->skeys, job->key_off.p, job->stream),
          "key lengths (exact)");
-      CK(launch_key_lengths(job->seg_startb.p, job->nseg_b, job->permb, job->krefb.p, job->key_off.p + job->nseg_a,
+      CK(launch_key_lengths_exact(job->segc, job->nseg_c, job->skeysc, job->key_off.p + job->nseg_a, job->stream),
+         "key lengths (mid)");
+      CK(launch_key_lengths(job->seg_startb.p, job->nseg_b, job->permb, job->krefb.p,
+                            job->key_off.p + job->nseg_a + job->nseg_c,
                             job->stream),
          "key lengths (hashed)");
     } else {
@@ -726,10 +763,15 @@ mr_status mr_reduce(mr_job* job) {
         // every Map value is 1: a key's count is its segment length (exact stream first, then
         // the hashed stream; the output order is the sorted order of each stream)
         CK(launch_seg_lengths(job->sega, job->nseg_a, job->counts.p, s), "counts (exact)");
-        CK(launch_seg_lengths(job->seg_startb.p, job->nseg_b, job->counts.p + job->nseg_a, s), "counts (hashed)");
+        CK(launch_seg_lengths(job->segc, job->nseg_c, job->counts.p + job->nseg_a, s), "counts (mid)");
+        CK(launch_seg_lengths(job->seg_startb.p, job->nseg_b, job->counts.p + job->nseg_a + job->nseg_c, s),
+           "counts (hashed)");
+        CK(launch_key_decode(job->segc, job->nseg_c, job->skeysc, job->key_off.p + job->nseg_a, job->keys_out.p, s),
+           "key decode (mid)");
         CK(launch_key_decode(job->sega, job->nseg_a, job->skeys, job->key_off.p, job->keys_out.p, s),
            "key decode");
-        CK(launch_key_copy(job->seg_startb.p, job->nseg_b, job->permb, job->krefb.p, job->key_off.p + job->nseg_a,
+        CK(launch_key_copy(job->seg_startb.p, job->nseg_b, job->permb, job->krefb.p,
+                           job->key_off.p + job->nseg_a + job->nseg_c,
                            job->keys_out.p, s),
            "key copy");
       } else {
@@ -864,12 +906,15 @@ mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_byte
     const uint64_t m = hs->pair_cursor;
     job->m = m - hs->pads;
     job->mb = job->split() ? hs->pair_cursor_b : 0;
-    job->stats.pairs = job->m + job->mb;
+    job->mc = job->split() ? hs->pair_cursor_c : 0;
+    job->stats.pairs = job->m + job->mb + job->mc;
     if (job->split()) {
       xs.mode = kXSplit;
       xs.hx = job->h.p;
       xs.nx = m;
-      xs.n = m + job->mb;
+      xs.hc = job->hc.p;
+      xs.nc = job->mc;
+      xs.n = m + job->mc + job->mb;
       xs.kref = job->krefb.p;
     } else {
       xs.mode = kXPairs;
@@ -996,7 +1041,7 @@ mr_status mr_job_destroy(mr_job* job) {
   job->xcounts.release(); job->xcursors.release(); job->xheapbase.release(); job->xcounts_h.release();
   job->src_e.release(); job->src_h.release(); job->km_list.release();
   job->cent.release(); release_pairs(job); job->tb.release();
-  job->sw.release(); job->swb.release(); job->seg_startb.release(); job->scan_status.release();
+  job->sw.release(); job->swb.release(); job->swc.release(); job->seg_startb.release(); job->scan_status.release();
   job->seg_counts.release(); job->tile_base.release(); job->seg_start.release(); job->key_off.release();
   job->val_off.release(); job->counts.release(); job->worklist.release(); job->gathered.release();
   job->keys_out.release(); job->vals_out.release(); job->vsorted.release(); job->sums.release(); job->cnts.release();

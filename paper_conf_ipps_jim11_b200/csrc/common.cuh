@@ -145,7 +145,7 @@ __device__ __forceinline__ uint64_t hash_bytes(const uint8_t* p, uint32_t len, u
 //   hashed  : longer keys -> hash with the top bit of the width forced to 1 (never collides with
 //             an inline key); equal hashes are verified byte-for-byte at segment time;
 //   sentinel: all ones in the width — flush filler pairs, sorts after every real key.
-// The WordCount exact stream (map.cu) uses its own 30-bit format, exact_key30 below.
+// The WordCount exact and mid streams (map.cu) use the 6-bit symbol codes of exact_key below.
 __host__ __device__ __forceinline__ uint32_t inline_max(uint32_t bits) { return bits == 48 ? 5u : 7u; }
 __host__ __device__ __forceinline__ uint64_t hashed_bit(uint32_t bits) { return 1ULL << (bits - 1); }
 __host__ __device__ __forceinline__ uint64_t sentinel_of(uint32_t bits) {
@@ -163,10 +163,11 @@ __device__ __forceinline__ uint64_t inline_key(uint64_t bytes_le, uint32_t len, 
 }
 
 // WordCount exact keys: a WC word is [0-9A-Za-z]+ (C-3 #1), so every symbol has a nonzero 6-bit
-// code: '0'-'9' -> 1..10, 'A'-'Z' -> 11..36, 'a'-'z' -> 37..62.  A word of <= 5 symbols packs
-// injectively into 30 bits (symbol i at bits 6i; the highest nonzero code gives the length):
-// four 8-bit LSD digits.  Codes of 4 bytes at once: code = low nibble + base[high nibble], the
-// 5-entry base table looked up with one byte permute (PRMT) indexed by the high nibbles.
+// code: '0'-'9' -> 1..10, 'A'-'Z' -> 11..36, 'a'-'z' -> 37..62.  A word of L <= 8 symbols packs
+// injectively into 6L bits (symbol i at bits 6i; the highest nonzero code gives the length):
+// <= 5 symbols -> 30 bits (four 8-bit LSD digits), 6..8 symbols -> 48 bits (six digits).  Codes
+// of 4 bytes at once: code = low nibble + base[high nibble], the 5-entry base table looked up
+// with one byte permute (PRMT) indexed by the high nibbles.
 __device__ __forceinline__ uint32_t exact_codes4(uint32_t w) {
   const uint32_t hi = (w >> 4) & 0x0F0F0F0Fu;                  // 3 digit, 4-5 upper, 6-7 lower
   const uint32_t h2 = hi | (hi >> 4);
@@ -176,10 +177,10 @@ __device__ __forceinline__ uint32_t exact_codes4(uint32_t w) {
   const uint32_t base = __byte_perm(0x01000000u, 0x34241A0Au, sel);
   return (w & 0x0F0F0F0Fu) + base;                             // <= 62 per byte: no carries
 }
-__device__ __forceinline__ uint64_t exact_key30(uint64_t bytes_le, uint32_t len) {   // len 1..5
+__device__ __forceinline__ uint64_t exact_key(uint64_t bytes_le, uint32_t len) {   // len 1..8
   uint64_t x = (static_cast<uint64_t>(exact_codes4(static_cast<uint32_t>(bytes_le >> 32))) << 32) |
                exact_codes4(static_cast<uint32_t>(bytes_le));
-  x &= (1ULL << (8 * len)) - 1ULL;
+  if (len < 8) x &= (1ULL << (8 * len)) - 1ULL;
   x = (x & 0x003F003F003F003FULL) | ((x >> 2) & 0x0FC00FC00FC00FC0ULL);   // byte pairs -> 12 bits
   x = (x & 0x00000FFF00000FFFULL) | ((x >> 4) & 0x00FFF00000FFF000ULL);   // -> 24 bits
   x = (x & 0x0000000000FFFFFFULL) | ((x >> 8) & 0x0000FFFFFF000000ULL);   // -> 48 bits

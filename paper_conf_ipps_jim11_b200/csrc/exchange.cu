@@ -43,17 +43,17 @@ struct Rec {
 
 __device__ __forceinline__ Rec get_rec(const XSource& S, uint64_t i) {
   Rec r{};
-  if (S.mode == kXSplit) {           // WC Map output: exact stream, then hashed stream; value 1
+  if (S.mode == kXSplit) {   // WC Map output: exact, mid, then hashed stream; every value is 1
     r.v = 1;
-    if (i < S.nx) {
-      const uint64_t key = S.hx[i];
-      if (key == sentinel_of(48)) { r.dest = ~0u; return r; }   // flush filler
+    if (i < S.nx + S.nc) {
+      const uint64_t key = i < S.nx ? S.hx[i] : S.hc[i - S.nx];
+      if (key == sentinel_of(48)) { r.dest = ~0u; return r; }   // flush filler (exact stream)
       r.kin = exact_key_bytes(key, r.klen);
       r.dest = dest_of_bytes(reinterpret_cast<const uint8_t*>(&r.kin), r.klen, S.nranks);
       r.heap = (r.klen + 7u) & ~7u;
       return r;
     }
-    const uint64_t kr = S.kref[i - S.nx];
+    const uint64_t kr = S.kref[i - S.nx - S.nc];
     r.kp = reinterpret_cast<const uint8_t*>(kr >> 16);
     r.klen = static_cast<uint32_t>(kr & 0xFFFF);
   } else if (S.mode == kXPairs) {

@@ -12,9 +12,10 @@ extern std::atomic<unsigned long long> g_kernel_launches;
 inline void count_launch(unsigned n = 1) { g_kernel_launches.fetch_add(n, std::memory_order_relaxed); }
 
 enum Workload : int { kWC = 1, kSM = 2, kKM = 3, kII = 4 };
-// WordCount exact stream: words of <= kExactMax bytes, keys < 2^kExactBits (common.cuh)
-constexpr uint32_t kExactMax = 5;
-constexpr uint32_t kExactBits = 30;
+// WordCount streams (map.cu): exact (words of <= kExactMax bytes, keys < 2^kExactBits), mid
+// (<= kMidMax bytes, keys < 2^kMidBits), both keys only; longer words hashed with references.
+constexpr uint32_t kExactMax = 5, kExactBits = 30;
+constexpr uint32_t kMidMax = 8, kMidBits = 48;
 
 // Device-resident job state (one per job).
 struct DevState {
@@ -29,6 +30,7 @@ struct DevState {
   unsigned int tile_counter[32];   // dynamic tile ids of the look-back kernels (one per launch slot)
   unsigned long long pads;         // sentinel filler pairs written by the flushes (sort last, excluded)
   unsigned long long pair_cursor_b;  // WC hashed stream: demand in pairs
+  unsigned long long pair_cursor_c;  // WC mid stream: demand in pairs
 };
 constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u;
 
@@ -43,6 +45,8 @@ struct PairBufs {
   uint64_t* hb = nullptr;    // WC hashed stream: keys, key references, capacity
   uint64_t* krefb = nullptr;
   uint64_t cap_b = 0;
+  uint64_t* hc = nullptr;    // WC mid stream: keys, capacity
+  uint64_t cap_c = 0;
 };
 
 struct MapArgs {
@@ -149,8 +153,10 @@ struct XSource {
   uint32_t nranks = 1;
   uint64_t n = 0;                              // records of the source
   const uint64_t* kref = nullptr;              // kXPairs; kXSplit: hashed-stream krefs
-  const uint64_t* hx = nullptr;                // kXSplit: exact-stream keys (nx of them, first)
-  uint64_t nx = 0;
+  const uint64_t* hx = nullptr;                // kXSplit: exact-stream keys (nx of them, first),
+  uint64_t nx = 0;                             //   then the mid-stream keys (nc), then the hashed
+  const uint64_t* hc = nullptr;                //   stream (kref)
+  uint64_t nc = 0;
   const uint8_t* v = nullptr;
   int vbytes = 8;
   const uint8_t* keys = nullptr;               // kXSegs

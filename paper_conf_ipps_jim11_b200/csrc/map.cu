@@ -62,9 +62,11 @@ struct Cfg {
   // of words longer than kWcExact bytes.
   static constexpr int kHashQ = (W == kWC) ? 96 : 0;
 };
-// WC words of <= kWcExact bytes get an exact 30-bit key (common.cuh exact_key30) and travel in
-// the exact stream (8-B entries: the key is the whole record); longer words are hashed and
-// travel with their key reference in the hashed stream (16-B entries).
+// WC words of <= kWcExact bytes get an exact 30-bit key (common.cuh exact_key) and travel in
+// the exact stream (8-B entries: the key is the whole record).  Longer words are queued; in the
+// queue pass words of <= kMidMax bytes get an exact 48-bit key (mid stream, key only), longer
+// ones a hash (hashed stream, with their key reference).  Queued entries are 16 B (key, kref;
+// kref 0 marks a mid-stream key) and the flush warp routes them.
 constexpr uint32_t kWcExact = kExactMax;
 static_assert(kWin / (kWcExact + 1) + 1 <= Cfg<kWC>::kHashQ, "hash queue too small");
 constexpr int kKmPts = kT / 32;                // 512 points per KM tile
@@ -148,6 +150,8 @@ struct Params {
   uint64_t* ohb;           // WC hashed stream: keys, krefs, capacity
   uint64_t* okrefb;
   uint64_t cap_b;
+  uint64_t* ohc;           // WC mid stream: keys, capacity
+  uint64_t cap_c;
   uint32_t out_cap;        // per-half capacity actually used (FORCE_TINY_OUT shrinks it)
   uint32_t flags;
   DevState* st;
@@ -325,6 +329,17 @@ __device__ __forceinline__ uint64_t hash_smem(const uint8_t* sb, uint32_t i, uin
   return hs.finish();
 }
 
+// The <= 8 key bytes [q, q + len) little-endian (bytes beyond len unspecified).
+__device__ __forceinline__ uint64_t bytes8_at(const Params& P, const TileView& tv, long long q, uint32_t len) {
+  if (q + 8 <= tv.stg_hi && q - tv.sbase + 8 + 12 <= kStageBytes) {
+    const uint32_t i = static_cast<uint32_t>(q - tv.sbase);
+    return static_cast<uint64_t>(smem_word_at(tv.sb, i)) | (static_cast<uint64_t>(smem_word_at(tv.sb, i + 4)) << 32);
+  }
+  uint64_t b = 0;
+  for (uint32_t k = 0; k < len; ++k) b |= static_cast<uint64_t>(P.rec[q + k]) << (8 * k);
+  return b;
+}
+
 // Sort key of the key bytes [q, q + len): inline when short, else the hash (common.cuh).
 __device__ __forceinline__ uint64_t key_at(const Params& P, const TileView& tv, long long q, uint32_t len) {
   const bool in_stage = (q + static_cast<long long>(len) <= tv.stg_hi) && (q - tv.sbase + len + 12 <= kStageBytes);
@@ -476,12 +491,10 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
     unsigned long long gb = 0, gbb = 0;
     if (lane == 0) {
       if (cnt) gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(cnt));  // ONE global atomic per run
-      if (cb) gbb = atomicAdd(&P.st->pair_cursor_b, static_cast<unsigned long long>(cb));
       oc->nflush += (cnt || cb) ? 1 : 0;
       oc->npads += cnt - ca0;
     }
     gb = __shfl_sync(kFull, gb, 0);
-    gbb = __shfl_sync(kFull, gbb, 0);
     __syncwarp();
     if (cnt && gb + cnt <= P.cap_pairs) {
       const uint64_t* sh = reinterpret_cast<const uint64_t*>(half);
@@ -498,15 +511,37 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       }
     }
     if constexpr (W == kWC) {
-      // hashed entries (key, kref) from the top of the buffer -> the two SoA arrays of the
-      // hashed stream (a few % of the pairs: plain coalesced stores)
-      if (cb && gbb + cb <= P.cap_b) {
-        const ulonglong2* top = reinterpret_cast<const ulonglong2*>(half + Cfg<W>::kOutHalf);
-        for (uint32_t i = lane; i < cb; i += 32) {
-          const ulonglong2 e = top[-1 - static_cast<int>(i)];
-          P.ohb[gbb + i] = e.x;
-          P.okrefb[gbb + i] = e.y;
+      // queued entries (key, kref) from the top of the buffer: kref 0 -> mid stream (key only),
+      // else hashed stream (key + kref).  Two ballot passes: count, then scatter (plain
+      // coalesced stores; a few % of the pairs).
+      const ulonglong2* top = reinterpret_cast<const ulonglong2*>(half + Cfg<W>::kOutHalf);
+      uint32_t nc = 0;
+      for (uint32_t i0 = 0; i0 < cb; i0 += 32) {
+        const bool v = i0 + lane < cb && top[-1 - static_cast<int>(i0 + lane)].y == 0;
+        nc += __popc(__ballot_sync(kFull, v));
+      }
+      unsigned long long gc = 0;
+      if (lane == 0) {
+        if (cb - nc) gbb = atomicAdd(&P.st->pair_cursor_b, static_cast<unsigned long long>(cb - nc));
+        if (nc) gc = atomicAdd(&P.st->pair_cursor_c, static_cast<unsigned long long>(nc));
+      }
+      gbb = __shfl_sync(kFull, gbb, 0);
+      gc = __shfl_sync(kFull, gc, 0);
+      const bool okb = gbb + (cb - nc) <= P.cap_b, okc = gc + nc <= P.cap_c;
+      uint32_t rb = 0, rc = 0;
+      for (uint32_t i0 = 0; i0 < cb; i0 += 32) {
+        const bool in = i0 + lane < cb;
+        ulonglong2 e = make_ulonglong2(0ULL, 0ULL);
+        if (in) e = top[-1 - static_cast<int>(i0 + lane)];
+        const uint32_t mc = __ballot_sync(kFull, in && e.y == 0), mb = __ballot_sync(kFull, in && e.y != 0);
+        if (in && e.y == 0 && okc) P.ohc[gc + rc + __popc(mc & lanemask_lt())] = e.x;
+        if (in && e.y != 0 && okb) {
+          const uint64_t o = gbb + rb + __popc(mb & lanemask_lt());
+          P.ohb[o] = e.x;
+          P.okrefb[o] = e.y;
         }
+        rc += __popc(mc);
+        rb += __popc(mb);
       }
     }
     __syncwarp();
@@ -719,7 +754,7 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
     const uint32_t ma = __ballot_sync(kFull, ex), mb = __ballot_sync(kFull, act && !ex);
     if (ex) {
       const uint64_t b = window8(x, j);     // an exact word lies inside the 32 loaded bytes
-      sh[ka + __popc(ma & lanemask_lt())] = exact_key30(b, len);
+      sh[ka + __popc(ma & lanemask_lt())] = exact_key(b, len);
     } else if (act) {
       if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
       hq[nq + __popc(mb & lanemask_lt())] = static_cast<uint64_t>(p0 + j - tv.sbase) | (static_cast<uint64_t>(len) << 24);
@@ -728,12 +763,17 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
     nq += __popc(mb);
   }
   __syncwarp();
-  for (uint32_t q = lane; q < nq; q += 32) {           // lane-parallel hashing of the long words
+  for (uint32_t q = lane; q < nq; q += 32) {           // lane-parallel keys of the long words
     const uint64_t e = hq[q];
     const long long p = tv.sbase + static_cast<long long>(e & 0xFFFFFF);
     const uint32_t len = static_cast<uint32_t>(e >> 24);
-    top[-1 - static_cast<int>(kb0 + q)] =
-        make_ulonglong2(key_at(P, tv, p, len), (reinterpret_cast<uint64_t>(P.rec + p) << 16) | len);
+    ulonglong2 ent;
+    if (len <= kMidMax) {                                // mid stream: exact 48-bit key, no kref
+      ent = make_ulonglong2(exact_key(bytes8_at(P, tv, p, len), len), 0ULL);
+    } else {
+      ent = make_ulonglong2(key_at(P, tv, p, len), (reinterpret_cast<uint64_t>(P.rec + p) << 16) | len);
+    }
+    top[-1 - static_cast<int>(kb0 + q)] = ent;
   }
   commit(oc, slot, packed);
 }
@@ -1053,6 +1093,8 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.ohb = a.out.hb;
   P.okrefb = a.out.krefb;
   P.cap_b = a.out.cap_b;
+  P.ohc = a.out.hc;
+  P.cap_c = a.out.cap_c;
   if (P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>((P.ntiles + 255) / 256);
