@@ -640,6 +640,7 @@ mr_status mr_group(mr_job* job) {
     return fail(job, MR_ERR_UNSUPPORTED, ">= 2^32 intermediate pairs in one group");
   if (job->cfg.workload == MR_STRINGMATCH) {  // Map-only
     job->nseg = m;
+    if (job->prof.on) job->prof.collect();      // settle_map synchronised the stream
     job->state = kGrouped;
     return MR_OK;
   }

@@ -41,6 +41,24 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   while (!mbar_try_wait(bar, parity)) {
   }
 }
+// try_wait with an explicit suspend-time hint (ns): the waiting warp stays suspended (instead of
+// re-polling and taking issue slots from the compute warps) until the phase completes or the
+// hint expires.
+__device__ __forceinline__ bool mbar_try_wait_hint(uint64_t* bar, uint32_t parity, uint32_t ns) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity), "r"(ns)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait_idle(uint64_t* bar, uint32_t parity, uint32_t ns = 20000) {
+  while (!mbar_try_wait_hint(bar, parity, ns)) {
+  }
+}
 // TMA 1-D bulk copy global -> shared; dst, src and bytes must be multiples of 16.
 __device__ __forceinline__ void tma_load_1d(void* smem_dst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
   asm volatile(
@@ -185,6 +203,19 @@ __device__ __forceinline__ uint64_t exact_key(uint64_t bytes_le, uint32_t len) {
   x = (x & 0x00000FFF00000FFFULL) | ((x >> 4) & 0x00FFF00000FFF000ULL);   // -> 24 bits
   x = (x & 0x0000000000FFFFFFULL) | ((x >> 8) & 0x0000FFFFFF000000ULL);   // -> 48 bits
   return x;
+}
+// The same key for len 1..5 (the exact stream) on 32-bit operations: codes of bytes 0..3 with
+// one table permute, byte 4 with a second one, 4 codes packed to 24 bits, code 4 on top.
+__device__ __forceinline__ uint32_t exact_key30(uint64_t bytes_le, uint32_t len) {
+  uint32_t c = exact_codes4(static_cast<uint32_t>(bytes_le));
+  if (len < 4) c &= (1u << (8 * len)) - 1u;
+  uint32_t y = (c & 0x003F003Fu) | ((c >> 2) & 0x0FC00FC0u);   // byte pairs -> 12 bits
+  y = (y & 0x00000FFFu) | ((y >> 4) & 0x00FFF000u);            // -> 24 bits
+  if (len == 5) {
+    const uint32_t b4 = static_cast<uint32_t>(bytes_le >> 32) & 0xFFu;
+    y |= ((b4 & 0xFu) + (__byte_perm(0x01000000u, 0x34241A0Au, b4 >> 4) & 0xFFu)) << 24;
+  }
+  return y;
 }
 // Inverse: key bytes little-endian and the length.
 __device__ __forceinline__ uint64_t exact_key_bytes(uint64_t key, uint32_t& len) {

@@ -162,6 +162,7 @@ struct Params {
 };
 
 constexpr uint32_t kFull = 0xffffffffu;
+constexpr uint32_t kReadyWaitNs = 2000;   // map warps: suspend hint while waiting for a staged tile
 
 // ---------------------------------------------------------------- packed fp32 (sm_100a FADD2/FFMA2)
 __device__ __forceinline__ uint64_t f2pack(float a, float b) {
@@ -188,9 +189,14 @@ __device__ __forceinline__ uint32_t movemask4(uint32_t m) {  // 0xFF/0x00 bytes 
   return ((((m >> 7) & 0x01010101u) * 0x01020408u) >> 24) & 0xFu;
 }
 __device__ __forceinline__ uint32_t word_mask4(uint32_t x) {  // [0-9A-Za-z] (C-3 #1)
-  uint32_t dig = __vcmpltu4(__vsub4(x, 0x30303030u), 0x0a0a0a0au);
-  uint32_t alp = __vcmpltu4(__vsub4(x | 0x20202020u, 0x61616161u), 0x1a1a1a1au);
-  return movemask4(dig | alp);
+  // carry-free byte compares on the low 7 bits (bias so that bit 7 flags c >= bound), bytes
+  // >= 0x80 excluded: 4 x (digit or letter) -> 4 bits
+  const uint32_t x7 = x & 0x7F7F7F7Fu;
+  const uint32_t l = x7 | 0x20202020u;                         // letters -> 0x61..0x7A
+  const uint32_t dig = (x7 + 0x50505050u) & ~(x7 + 0x46464646u);   // 0x30 <= c < 0x3A
+  const uint32_t alp = (l + 0x1F1F1F1Fu) & ~(l + 0x05050505u);     // 0x61 <= l < 0x7B
+  const uint32_t m = (dig | alp) & ~x & 0x80808080u;
+  return ((m >> 7) * 0x01020408u) >> 24;
 }
 __device__ __forceinline__ uint32_t eq_mask4(uint32_t x, uint32_t b4) { return movemask4(__vcmpeq4(x, b4)); }
 __device__ __forceinline__ bool is_word_byte(uint32_t c) {
@@ -464,7 +470,7 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   const uint32_t lane = threadIdx.x & 31;
   for (uint32_t f = 0;; ++f) {
     const uint32_t h = f % kNOut;
-    mbar_wait(&oc->req[h], (f / kNOut) & 1u);
+    mbar_wait_idle(&oc->req[h], (f / kNOut) & 1u);
     const uint32_t cnt0 = *reinterpret_cast<volatile unsigned int*>(&oc->fcount[h]);
     const bool fin = *reinterpret_cast<volatile unsigned int*>(&oc->is_final) &&
                      *reinterpret_cast<volatile unsigned int*>(&oc->final_seq) == f;
@@ -613,7 +619,7 @@ __device__ void producer_loop(const Params& P, uint8_t* smem) {
       if (t >= P.ntiles) break;
       const uint64_t ra = __shfl_sync(kFull, my_ra, j), rb = __shfl_sync(kFull, my_rb, j);
       const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
-      mbar_wait(&empty[s], ph ^ 1u);
+      mbar_wait_idle(&empty[s], ph ^ 1u);
       StageHdr* hd = reinterpret_cast<StageHdr*>(smem + Layout<W>::hdr + s * 128);
       uint8_t* sb = smem + Layout<W>::bytes + s * kStageBytes;
       uint32_t b_off = 0, b_len = 0, o_off = 0, o_len = 0;
@@ -754,7 +760,7 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
     const uint32_t ma = __ballot_sync(kFull, ex), mb = __ballot_sync(kFull, act && !ex);
     if (ex) {
       const uint64_t b = window8(x, j);     // an exact word lies inside the 32 loaded bytes
-      sh[ka + __popc(ma & lanemask_lt())] = exact_key(b, len);
+      sh[ka + __popc(ma & lanemask_lt())] = exact_key30(b, len);
     } else if (act) {
       if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
       hq[nq + __popc(mb & lanemask_lt())] = static_cast<uint64_t>(p0 + j - tv.sbase) | (static_cast<uint64_t>(len) << 24);
@@ -915,7 +921,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   for (uint32_t it = 0;; ++it) {
     const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
     if constexpr (W == kKM) mbar_wait(&full[s], ph);
-    else mbar_wait(reinterpret_cast<uint64_t*>(smem + Layout<W>::ready) + s, ph);
+    else mbar_wait_idle(reinterpret_cast<uint64_t*>(smem + Layout<W>::ready) + s, ph, kReadyWaitNs);
     const StageHdr hd = *reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
     if (hd.t < 0) break;
     const uint8_t* sb = smem + Layout<W>::bytes + s * kStageBytes;
