@@ -187,8 +187,9 @@ def run_reference(args, rank, world):
 def algorithmic(inp, st, steps):
     """Algorithmic bytes per step of each phase.
 
-    WordCount Map output is three streams: exact keys (words <= 5 bytes) and mid keys (6..8
-    bytes) are bare 8-B keys sorted keys-only (8 B read + 8 B written per pass); hashed keys
+    WordCount Map output is three streams: exact keys (words <= 5 bytes) are bare 4-B u32 keys
+    sorted keys-only (4 B read + 4 B written per pass); mid keys (6..8 bytes) bare 8-B keys
+    (8 B read + 8 B written per pass); hashed keys
     (longer words) carry a key reference (16 B) and sort with a u32 permutation (24 B per pass,
     the first pass reads no permutation)."""
     wl = inp["wl"]
@@ -202,13 +203,14 @@ def algorithmic(inp, st, steps):
     pc = st["sort_passes_mid"] / steps
     passes = st["sort_passes"] / steps
     if wl == "wc":
-        map_b = inp["nbytes"] + off_b + (mx + mc) * 8 + mh * 16
+        map_b = inp["nbytes"] + off_b + mx * 4 + mc * 8 + mh * 16
         ph = passes - px - pc
-        sort_b = px * 16 * mx + pc * 16 * mc + ((ph * 24 - 4) * mh if ph else 0.0)
+        sort_b = px * 8 * mx + pc * 16 * mc + ((ph * 24 - 4) * mh if ph else 0.0)
     else:
         map_b = inp["nbytes"] + off_b + m * {"sm": 8, "km": 40, "ii": 24}[wl]
         sort_b = (passes * 24 - 4) * m if passes else 0.0   # first pass reads no payload
-    return {"map": map_b, "hist": 8 * m, "sort": sort_b, "passes": passes, "pairs": m, "pairs_exact": mx,
+    hist_b = (4 * mx + 8 * (mc + mh)) if wl == "wc" else 8 * m
+    return {"map": map_b, "hist": hist_b, "sort": sort_b, "passes": passes, "pairs": m, "pairs_exact": mx,
             "passes_keys": px}
 
 
@@ -311,7 +313,7 @@ def main():
     if alg["passes_keys"]:   # WC: the keys-only pass over the exact stream dominates the step
         kname = "k_onesweep (keys-only LSD pass, WC exact stream)"
         sort_launch_ms = per["sort_keys_ms"] / alg["passes_keys"]
-        sort_launch_bytes = 16 * alg["pairs_exact"]
+        sort_launch_bytes = 8 * alg["pairs_exact"]
     else:
         kname = "k_onesweep (LSD pass)"
         sort_launch_ms = per["sort_ms"] / max(alg["passes"], 1)

@@ -103,10 +103,14 @@ struct Batch {
 struct SortWork {
   DBuf<uint64_t> ka, kb, status;
   DBuf<uint32_t> ia, ib, hist, bases;
+  DBuf<uint32_t> ka32, kb32;      // u32 keys-only ping-pong (WC exact stream)
   HBuf<uint32_t> hist_h, bases_h;
   uint32_t epoch = 1;
   uint64_t passes = 0;
-  void release() { ka.release(); kb.release(); status.release(); ia.release(); ib.release(); hist.release(); bases.release(); hist_h.release(); bases_h.release(); }
+  void release() {
+    ka.release(); kb.release(); status.release(); ia.release(); ib.release(); hist.release(); bases.release();
+    hist_h.release(); bases_h.release(); ka32.release(); kb32.release();
+  }
 };
 
 __global__ void k_iota_u32(uint32_t* p, uint64_t n) {
@@ -194,6 +198,65 @@ cudaError_t run_sort(SortWork& W, const uint64_t* keys, uint64_t m, const uint64
   return cudaSuccess;
 }
 
+
+// Keys-only radix sort of m u32 keys on their low key_width bits (the WC exact stream):
+// *out_keys points into the workspace (or at `keys` when every digit is constant).
+cudaError_t run_sort32(SortWork& W, const uint32_t* keys, uint64_t m, const uint32_t** out_keys, DevState* st,
+                       int nsm, cudaStream_t s, Prof* prof, double* hist_ms, double* pass_ms, int key_width) {
+  cudaError_t e;
+  const int bits = 8, bins = 1 << bits;
+  const int ndig = std::min(4, (key_width + bits - 1) / bits);
+  if ((e = W.ka32.ensure(m + 1)) || (e = W.kb32.ensure(m + 1))) return e;
+  const uint64_t tiles = (m + sort_tile_keys32() - 1) / sort_tile_keys32();
+  const uint64_t need_status = tiles * bins;
+  if (W.status.n < need_status || !W.status.p) {
+    if ((e = W.status.ensure(need_status))) return e;
+    if ((e = cudaMemsetAsync(W.status.p, 0, W.status.n * sizeof(uint64_t), s))) return e;
+  }
+  if ((e = W.hist.ensure(8 * kBinStride)) || (e = W.bases.ensure(8 * kBinStride))) return e;
+  if ((e = W.hist_h.ensure(8 * kBinStride)) || (e = W.bases_h.ensure(8 * kBinStride))) return e;
+  {
+    Prof::Span sp{};
+    if (prof && prof->on) prof->begin(s, sp);
+    if ((e = launch_hist32(keys, m, W.hist.p, ndig, bits, nsm, s))) return e;
+    if (prof && prof->on) prof->end(s, sp, hist_ms);
+  }
+  if ((e = cudaMemcpyAsync(W.hist_h.p, W.hist.p, 8 * kBinStride * sizeof(uint32_t), cudaMemcpyDeviceToHost, s)))
+    return e;
+  if ((e = cudaStreamSynchronize(s))) return e;
+  int digits[4];
+  int nd = 0;
+  for (int d = 0; d < ndig; ++d) {
+    uint32_t run = 0;
+    int nonzero = 0;
+    for (int b = 0; b < bins; ++b) {
+      const uint32_t c = W.hist_h.p[d * kBinStride + b];
+      W.bases_h.p[d * kBinStride + b] = run;
+      run += c;
+      nonzero += c ? 1 : 0;
+    }
+    if (nonzero > 1) digits[nd++] = d;  // constant digits are skipped
+  }
+  W.passes = nd;
+  *out_keys = keys;
+  if (nd == 0) return cudaSuccess;
+  if ((e = cudaMemcpyAsync(W.bases.p, W.bases_h.p, 8 * kBinStride * sizeof(uint32_t), cudaMemcpyHostToDevice, s)))
+    return e;
+  const uint32_t* kin = keys;
+  Prof::Span sp2{};
+  if (prof && prof->on) prof->begin(s, sp2);
+  for (int p = 0; p < nd; ++p) {
+    uint32_t* kout = (p & 1) ? W.kb32.p : W.ka32.p;
+    if ((e = launch_onesweep32(kin, kout, m, digits[p], bits, W.bases.p, W.status.p, W.epoch++,
+                               &st->tile_counter[0], s)))
+      return e;
+    kin = kout;
+  }
+  if (prof && prof->on) prof->end(s, sp2, pass_ms);
+  *out_keys = kin;
+  return cudaSuccess;
+}
+
 }  // namespace
 
 struct mr_job {
@@ -211,6 +274,7 @@ struct mr_job {
   HBuf<uint64_t> tmp_h;
   DBuf<float> cent;
   DBuf<uint64_t> h, kref, tb;
+  DBuf<uint32_t> hx;              // WC exact stream keys (u32)
   DBuf<uint8_t> v;
   uint64_t cap = 0;
   std::vector<Batch> batches;
@@ -223,11 +287,13 @@ struct mr_job {
   unsigned long long launches0 = 0;
   SortWork sw, swb, swc;
   const uint64_t* skeys = nullptr;
+  const uint32_t* skeysx = nullptr;   // WC exact stream, sorted (u32)
   const uint32_t* perm = nullptr;
   uint64_t m = 0, nseg = 0, key_bytes = 0;
   // WC hashed stream (the exact stream uses h / skeys / seg_start): pairs, sorted, segments
   DBuf<uint64_t> hb, krefb, seg_startb;
-  uint64_t* sega = nullptr;       // exact-stream segment starts (in the free sort buffer)
+  uint64_t* sega = nullptr;       // exact-stream segment starts (seg_startx)
+  DBuf<uint64_t> seg_startx;
   uint64_t cap_b = 0, mb = 0, nseg_a = 0, nseg_b = 0;
   // WC mid stream (6..8-byte words, exact 48-bit keys, keys only)
   DBuf<uint64_t> hc;
@@ -295,7 +361,11 @@ uint64_t initial_cap(const mr_job* job, uint64_t nbytes, uint64_t n) {
 // cap_b / cap_c: WC hashed / mid stream capacities (0 for the other workloads)
 cudaError_t ensure_pairs(mr_job* job, uint64_t cap, uint64_t cap_b, uint64_t cap_c) {
   cudaError_t e;
-  if ((e = job->h.ensure(cap))) return e;
+  if (job->split()) {
+    if ((e = job->hx.ensure(cap))) return e;
+  } else if ((e = job->h.ensure(cap))) {
+    return e;
+  }
   if (has_kref(job->cfg.workload) && (e = job->kref.ensure(cap))) return e;
   const int vb = vbytes_of(job->cfg.workload);
   if (vb && (e = job->v.ensure(cap * vb))) return e;
@@ -309,7 +379,7 @@ cudaError_t ensure_pairs(mr_job* job, uint64_t cap, uint64_t cap_b, uint64_t cap
   return cudaSuccess;
 }
 void release_pairs(mr_job* job) {
-  job->h.release(); job->kref.release(); job->v.release(); job->hb.release(); job->krefb.release();
+  job->h.release(); job->hx.release(); job->kref.release(); job->v.release(); job->hb.release(); job->krefb.release();
   job->hc.release();
   job->cap = job->cap_b = job->cap_c = 0;
 }
@@ -328,6 +398,7 @@ cudaError_t launch_batch(mr_job* job, const Batch& b) {
   a.centroids = job->cent.p;
   a.k = job->k;
   a.out.h = job->h.p;
+  a.out.hx = job->hx.p;
   a.out.kref = job->kref.p;
   a.out.v = job->v.p;
   a.out.cap = job->cap;
@@ -404,6 +475,25 @@ mr_status do_segments_into(mr_job* job, const uint64_t* skeys, uint64_t m, uint6
   CK(launch_seg_write(skeys, m, job->tile_base.p, seg_start, ~0ULL, job->stream), "seg_write");
   CK(read_state(job), "sync segments");
   nseg = m ? job->st_h.p->seg_total : 0;
+  return MR_OK;
+}
+
+// Keys-only u32 stream (WC exact): heads counted and scanned; seg_start sized from the count.
+mr_status do_segments32(mr_job* job, const uint32_t* skeys, uint64_t m, DBuf<uint64_t>& seg_start, uint64_t& nseg) {
+  const uint64_t tiles = (m + 4095) / 4096;
+  CK(job->seg_counts.ensure(tiles + 1), "alloc seg counts");
+  CK(job->tile_base.ensure(tiles + 1), "alloc tile base");
+  CK(launch_seg_count32(skeys, m, job->seg_counts.p, job->stream), "seg_count");
+  uint64_t* ss;
+  uint32_t ep;
+  CK(scan_ws(job, tiles, &ss, &ep), "alloc scan workspace");
+  CK(launch_scan_u32to64(job->seg_counts.p, job->tile_base.p, tiles, &job->st->seg_total, ss, ep,
+                         &job->st->tile_counter[1], job->stream),
+     "scan tiles");
+  CK(read_state(job), "sync segments");
+  nseg = m ? job->st_h.p->seg_total : 0;
+  CK(seg_start.ensure(nseg + 1), "alloc seg_start");
+  CK(launch_seg_write32(skeys, m, job->tile_base.p, seg_start.p, job->stream), "seg_write");
   return MR_OK;
 }
 
@@ -651,20 +741,20 @@ mr_status mr_group(mr_job* job) {
   job->segc = nullptr;
   if (split) {
     // exact stream: keys only (the key is the record), no byte verification needed
-    CK(run_sort(job->sw, job->h.p, m_total, &job->skeys, nullptr, job->st, job->nsm, job->stream, &job->prof,
-                &job->stats.hist_ms, &job->stats.sort_keys_ms, kExactBits),   // exact keys < 2^30
+    CK(run_sort32(job->sw, job->hx.p, m_total, &job->skeysx, job->st, job->nsm, job->stream, &job->prof,
+                  &job->stats.hist_ms, &job->stats.sort_keys_ms, kExactBits),   // exact keys < 2^30
        "radix sort (exact)");
     job->stats.sort_passes += job->sw.passes;
     job->stats.sort_passes_keys += job->sw.passes;
     job->perm = nullptr;
     Prof::Span sp{};
     if (job->prof.on) job->prof.begin(job->stream, sp);
-    // heads (count, scan, write); seg_start goes to the sort buffer not holding the result.
+    // heads (count, scan, write) into seg_startx.
     // (A single-pass select with a decoupled look-back over the 4096-key tiles measured slower:
     // 5.4 ms against 3.3 + 2.2 ms on C5.)
-    job->sega = (job->skeys == job->sw.ka.p) ? job->sw.kb.p : job->sw.ka.p;
-    st = do_segments_into(job, job->skeys, m, job->sega, job->nseg_a);
+    st = do_segments32(job, job->skeysx, m, job->seg_startx, job->nseg_a);
     if (st != MR_OK) return st;
+    job->sega = job->seg_startx.p;
     if (job->prof.on) job->prof.end(job->stream, sp, &job->stats.seg_ms);
     // mid stream: exact 48-bit keys, keys only (no fillers: plain stores)
     CK(run_sort(job->swc, job->hc.p, mc, &job->skeysc, nullptr, job->st, job->nsm, job->stream, &job->prof,
@@ -720,7 +810,7 @@ mr_status mr_group(mr_job* job) {
   if (job->cfg.workload == MR_WORDCOUNT || job->cfg.workload == MR_INVINDEX) {
     CK(job->key_off.ensure(job->nseg + 1), "alloc key offsets");
     if (split) {
-      CK(launch_key_lengths_exact(job->sega, job->nseg_a, job->skeys, job->key_off.p, job->stream),
+      CK(launch_key_lengths_exact32(job->sega, job->nseg_a, job->skeysx, job->key_off.p, job->stream),
          "key lengths (exact)");
       CK(launch_key_lengths_exact(job->segc, job->nseg_c, job->skeysc, job->key_off.p + job->nseg_a, job->stream),
          "key lengths (mid)");
@@ -769,7 +859,7 @@ mr_status mr_reduce(mr_job* job) {
            "counts (hashed)");
         CK(launch_key_decode(job->segc, job->nseg_c, job->skeysc, job->key_off.p + job->nseg_a, job->keys_out.p, s),
            "key decode (mid)");
-        CK(launch_key_decode(job->sega, job->nseg_a, job->skeys, job->key_off.p, job->keys_out.p, s),
+        CK(launch_key_decode32(job->sega, job->nseg_a, job->skeysx, job->key_off.p, job->keys_out.p, s),
            "key decode");
         CK(launch_key_copy(job->seg_startb.p, job->nseg_b, job->permb, job->krefb.p,
                            job->key_off.p + job->nseg_a + job->nseg_c,
@@ -911,7 +1001,7 @@ mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_byte
     job->stats.pairs = job->m + job->mb + job->mc;
     if (job->split()) {
       xs.mode = kXSplit;
-      xs.hx = job->h.p;
+      xs.hx = job->hx.p;
       xs.nx = m;
       xs.hc = job->hc.p;
       xs.nc = job->mc;
@@ -1042,7 +1132,8 @@ mr_status mr_job_destroy(mr_job* job) {
   job->xcounts.release(); job->xcursors.release(); job->xheapbase.release(); job->xcounts_h.release();
   job->src_e.release(); job->src_h.release(); job->km_list.release();
   job->cent.release(); release_pairs(job); job->tb.release();
-  job->sw.release(); job->swb.release(); job->swc.release(); job->seg_startb.release(); job->scan_status.release();
+  job->sw.release(); job->swb.release(); job->swc.release(); job->seg_startb.release(); job->seg_startx.release();
+  job->scan_status.release();
   job->seg_counts.release(); job->tile_base.release(); job->seg_start.release(); job->key_off.release();
   job->val_off.release(); job->counts.release(); job->worklist.release(); job->gathered.release();
   job->keys_out.release(); job->vals_out.release(); job->vsorted.release(); job->sums.release(); job->cnts.release();

@@ -46,8 +46,8 @@ __device__ __forceinline__ Rec get_rec(const XSource& S, uint64_t i) {
   if (S.mode == kXSplit) {   // WC Map output: exact, mid, then hashed stream; every value is 1
     r.v = 1;
     if (i < S.nx + S.nc) {
-      const uint64_t key = i < S.nx ? S.hx[i] : S.hc[i - S.nx];
-      if (key == sentinel_of(48)) { r.dest = ~0u; return r; }   // flush filler (exact stream)
+      if (i < S.nx && S.hx[i] == 0xFFFFFFFFu) { r.dest = ~0u; return r; }   // flush filler (exact stream)
+      const uint64_t key = i < S.nx ? static_cast<uint64_t>(S.hx[i]) : S.hc[i - S.nx];
       r.kin = exact_key_bytes(key, r.klen);
       r.dest = dest_of_bytes(reinterpret_cast<const uint8_t*>(&r.kin), r.klen, S.nranks);
       r.heap = (r.klen + 7u) & ~7u;

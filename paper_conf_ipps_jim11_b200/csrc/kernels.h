@@ -35,10 +35,11 @@ struct DevState {
 constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u;
 
 // Intermediate pairs, SoA in HBM (SURVEY §8(a) layout): sort key, key reference, value.
-// WordCount Map output is two streams: exact keys (h only: the key is the record, value 1) and
-// hashed keys (hb + krefb); see map.cu.
+// WordCount Map output is three streams: exact keys (hx, u32: the key is the record, value 1),
+// mid keys (hc, u64 exact 48-bit) and hashed keys (hb + krefb); see map.cu.
 struct PairBufs {
   uint64_t* h = nullptr;     // 64-bit sort key (inline key / hash / SM offset / KM id)
+  uint32_t* hx = nullptr;    // WC exact stream: 30-bit exact keys (u32; 0xFFFFFFFF = filler)
   uint64_t* kref = nullptr;  // (device address of key bytes << 16) | key length
   uint8_t* v = nullptr;      // value bytes (vbytes per pair)
   uint64_t cap = 0;          // capacity in pairs
@@ -72,6 +73,8 @@ struct MapArgs {
 int vbytes_of(int workload);                 // value bytes per pair (WC Map output: none, value 1)
 bool has_kref(int workload);
 uint64_t map_tiles(const MapArgs& a);        // number of tiles of a batch
+uint32_t map_prefetch();
+uint32_t map_wait_hint();                     // L2 prefetch distance of the Map producers (BMR_MAP_PF)
 cudaError_t launch_map(const MapArgs& a, int num_sms, cudaStream_t s);
 
 // ---- group-by-key (hash radix sort + segment boundaries) ----
@@ -87,15 +90,22 @@ constexpr int kSortThreads = 256;
 constexpr int kBinStride = 512;   // histogram / base tables: 8 digits x kBinStride bins (digits of 8 or 9 bits)
 int sort_tile();   // keys per onesweep tile (tile shape chosen at start-up, BMR_SORT_CFG)
 int sort_tile_keys();   // the same for the keys-only passes
+int sort_tile_keys32();   // the same for the keys-only passes over u32 keys
 // histograms of digits [0, nd) of `bits` bits each (8 or 9); hist holds 8 x kBinStride u32
 cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int nd, int bits, int num_sms,
                         cudaStream_t s);
+cudaError_t launch_hist32(const uint32_t* keys, uint64_t m, uint32_t* hist, int nd, int bits, int num_sms,
+                          cudaStream_t s);
 // one LSD pass on digit `digit` of `bits` bits (8, or 9 for keys-only passes); idx_in ==
 // nullptr means the identity permutation; idx_out == nullptr: keys only (no payload).
 // bases: 8 x kBinStride table of global digit bases; status: tiles x 2^bits look-back words
 cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
                             uint32_t* idx_out, uint64_t m, int digit, int bits, const uint32_t* bases,
                             uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s);
+// keys-only LSD pass over u32 keys (the WordCount exact stream)
+cudaError_t launch_onesweep32(const uint32_t* keys_in, uint32_t* keys_out, uint64_t m, int digit, int bits,
+                              const uint32_t* bases, uint64_t* status, uint32_t epoch, unsigned int* tile_counter,
+                              cudaStream_t s);
 
 // ---- segments ----
 // heads per sort tile + byte verification of hashed keys; counts[t] = heads in tile t
@@ -109,6 +119,10 @@ cudaError_t launch_scan_u32to64(const uint32_t* in, uint64_t* out, uint64_t n, u
                                 uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s);
 cudaError_t launch_seg_write(const uint64_t* skeys, uint64_t m, const uint64_t* tile_base, uint64_t* seg_start,
                              uint64_t kmask, cudaStream_t s);
+// the same two steps over sorted u32 keys (keys-only, nothing to verify)
+cudaError_t launch_seg_count32(const uint32_t* skeys, uint64_t m, uint32_t* counts, cudaStream_t s);
+cudaError_t launch_seg_write32(const uint32_t* skeys, uint64_t m, const uint64_t* tile_base, uint64_t* seg_start,
+                               cudaStream_t s);
 
 // ---- reduce + output assembly ----
 struct OutBufs {
@@ -136,6 +150,10 @@ cudaError_t launch_key_lengths_exact(const uint64_t* seg_start, uint64_t nseg, c
                                      cudaStream_t s);
 cudaError_t launch_key_decode(const uint64_t* seg_start, uint64_t nseg, const uint64_t* skeys, const uint64_t* key_off,
                               uint8_t* keys, cudaStream_t s);
+cudaError_t launch_key_lengths_exact32(const uint64_t* seg_start, uint64_t nseg, const uint32_t* skeys, uint64_t* lens,
+                                       cudaStream_t s);
+cudaError_t launch_key_decode32(const uint64_t* seg_start, uint64_t nseg, const uint32_t* skeys,
+                                const uint64_t* key_off, uint8_t* keys, cudaStream_t s);
 cudaError_t launch_gather_u64(const uint32_t* perm, const uint8_t* v, uint64_t m, uint64_t* out, cudaStream_t s);
 cudaError_t launch_offsets_scaled(const uint64_t* seg_start, uint64_t nseg, uint64_t scale, uint64_t* out,
                                   cudaStream_t s);
@@ -153,7 +171,7 @@ struct XSource {
   uint32_t nranks = 1;
   uint64_t n = 0;                              // records of the source
   const uint64_t* kref = nullptr;              // kXPairs; kXSplit: hashed-stream krefs
-  const uint64_t* hx = nullptr;                // kXSplit: exact-stream keys (nx of them, first),
+  const uint32_t* hx = nullptr;                // kXSplit: exact-stream keys (nx of them, first),
   uint64_t nx = 0;                             //   then the mid-stream keys (nc), then the hashed
   const uint64_t* hc = nullptr;                //   stream (kref)
   uint64_t nc = 0;

@@ -24,6 +24,7 @@
 //     sentinel filler pairs.  The global cursor counts demand even past capacity (D7), so the
 //     host can grow the buffers and replay the batch.
 #include <cstdio>
+#include <cstdlib>
 
 #include "common.cuh"
 
@@ -31,10 +32,14 @@ namespace bmr {
 namespace {
 
 constexpr int kNMap = 16;
-constexpr int kProdWarp = kNMap;
-constexpr int kFlushWarp0 = kNMap + 1;   // flush warps kFlushWarp0 .. kFlushWarp0 + kNFlush - 1
+// Producer warps kProdWarp0 .. + kNProd - 1: producer p owns the iterations it == p (mod kNProd)
+// (and so the stages s == p (mod kNProd)); one warp alone is latency-bound at ~465 instructions
+// per tile (TMA issue + bitmap), slower than HBM delivers a tile (ncu, C2 round 1).
+constexpr int kNProd = 2;
+constexpr int kProdWarp0 = kNMap;
+constexpr int kFlushWarp0 = kNMap + kNProd;   // flush warps kFlushWarp0 .. kFlushWarp0 + kNFlush - 1
 constexpr int kNFlush = 1;
-constexpr int kThreads = (kNMap + 1 + kNFlush) * 32;
+constexpr int kThreads = (kNMap + kNProd + kNFlush) * 32;
 constexpr int kT = 16384;        // owned bytes per tile (text) / bytes per tile (KM)
 constexpr int kLead = 16;        // bytes staged before the tile (previous-byte context)
 constexpr int kHalo = 256;       // bytes staged after the tile (words / matches / URLs crossing it)
@@ -51,19 +56,20 @@ constexpr int kNOut = 4;         // output buffers in the flush ring (generation
 // and 4 x 20 KB output buffers.
 template <int W>
 struct Cfg {
-  static constexpr int kStages = (W == kSM) ? 7 : 4;
+  static constexpr int kStages = (W == kSM) ? 6 : 4;
   static constexpr int kOutHalf = (W == kSM) ? 4096 : 20480;   // bytes per output buffer
   // the producer builds the bitmap of tile it - kLag right after issuing tile it: kLag stages of
   // TMA traffic stay in flight per SM while one stage is being consumed
   static constexpr int kLag = kStages - 2;
+  static_assert(kStages % kNProd == 0 && kLag % kNProd == 0, "a producer owns every kNProd-th stage");
   // WC: per-warp queue of the window's long (hashed) words, hashed by all 32 lanes together
   // after the emission rounds (a lane-per-word hash inside the rounds diverges: with 10% long
   // words, most rounds would carry at least one).  A window holds at most 512 / 6 + 1 starts
   // of words longer than kWcExact bytes.
   static constexpr int kHashQ = (W == kWC) ? 96 : 0;
 };
-// WC words of <= kWcExact bytes get an exact 30-bit key (common.cuh exact_key) and travel in
-// the exact stream (8-B entries: the key is the whole record).  Longer words are queued; in the
+// WC words of <= kWcExact bytes get an exact 30-bit key (common.cuh exact_key30) and travel in
+// the exact stream (4-B u32 entries: the key is the whole record).  Longer words are queued; in the
 // queue pass words of <= kMidMax bytes get an exact 48-bit key (mid stream, key only), longer
 // ones a hash (hashed stream, with their key reference).  Queued entries are 16 B (key, kref;
 // kref 0 marks a mid-stream key) and the flush warp routes them.
@@ -118,18 +124,19 @@ struct Layout {
 static_assert(64 % kNOut == 0, "6-bit generation counter must wrap on a buffer boundary");
 
 // Output-buffer formats.  SM / KM / II: SoA runs [keys | krefs | values] of kCap entries.
-// WC: exact-key entries (u64 key) fill the buffer from the bottom, hashed entries (u64 key, u64
-// kref) from the top; capacity is counted in 8-byte units (exact 1, hashed 2).  WC values are
-// all 1 and are not stored: a key's count is its segment length.
+// WC: exact-key entries (u32 key) fill the buffer from the bottom, queued long-word entries (u64
+// key, u64 kref) from the top; capacity is counted in 4-byte units (exact 1, queued 4).  WC
+// values are all 1 and are not stored: a key's count is its segment length.
 template <int W>
 struct PairFmt {
   static constexpr bool kKref = (W == kII);
   static constexpr int kV = (W == kKM) ? 32 : (W == kII) ? 8 : 0;
   static constexpr int kPairBytes = 8 + (kKref ? 8 : 0) + kV;
-  static constexpr uint32_t kCap = (W == kWC) ? (Cfg<W>::kOutHalf / 8 - 2) : (Cfg<W>::kOutHalf / kPairBytes) & ~3u;
-  // largest single warp reservation (units): WC <= 512 starts in 512 B (+1 crossing word, 2
-  // units), SM 16 matches / 16 B, II 2, KM 1 per lane
-  static constexpr uint32_t kMaxReserve = (W == kWC) ? 576 : (W == kSM) ? 512 : 32 * ((W == kII) ? 2 : 1);
+  static constexpr uint32_t kCap = (W == kWC) ? (Cfg<W>::kOutHalf / 4 - 4) : (Cfg<W>::kOutHalf / kPairBytes) & ~3u;
+  // largest single warp reservation (units): WC <= 257 word starts in 512 B (a start follows a
+  // delimiter; +1 crossing word) of which <= kHashQ queued (4 units each), SM 16 matches / 16 B,
+  // II 2, KM 1 per lane
+  static constexpr uint32_t kMaxReserve = (W == kWC) ? 257 + 4 * Cfg<kWC>::kHashQ : (W == kSM) ? 512 : 32 * ((W == kII) ? 2 : 1);
   static_assert(kCap >= kMaxReserve, "output half smaller than one warp result");
 };
 
@@ -152,6 +159,7 @@ struct Params {
   uint64_t cap_b;
   uint64_t* ohc;           // WC mid stream: keys, capacity
   uint64_t cap_c;
+  uint32_t* ohx;           // WC exact stream: u32 keys (capacity cap_pairs)
   uint32_t out_cap;        // per-half capacity actually used (FORCE_TINY_OUT shrinks it)
   uint32_t flags;
   DevState* st;
@@ -159,7 +167,16 @@ struct Params {
   const uint8_t* off_end;  // end of the offsets array rounded DOWN to 16 B (aligned TMA limit)
   uint64_t hash_seed;
   uint32_t key_bits;       // sort-key width (48 or 64)
+  uint32_t pf;             // L2 prefetch distance in producer tiles (0: off)
+  uint32_t wait_hint;      // idle mbarrier waits: 1 = try_wait with a suspend-time hint, 0 = plain try_wait
 };
+
+// Idle wait of a role warp on an mbarrier phase (map warps on a staged tile, producers on a free
+// stage, the flush warp on a sealed buffer).
+__device__ __forceinline__ void map_wait(const Params& P, uint64_t* bar, uint32_t parity, uint32_t ns) {
+  if (P.wait_hint) mbar_wait_idle(bar, parity, ns);
+  else mbar_wait(bar, parity);
+}
 
 constexpr uint32_t kFull = 0xffffffffu;
 constexpr uint32_t kReadyWaitNs = 2000;   // map warps: suspend hint while waiting for a staged tile
@@ -383,7 +400,7 @@ __device__ __forceinline__ uint32_t cur_ca(uint32_t c) { return c & kCaMask; }
 __device__ __forceinline__ uint32_t cur_cb(uint32_t c) { return (c >> kCbShift) & kCbMask; }
 template <int W>
 __device__ __forceinline__ uint32_t units(uint32_t c) {   // buffer space of packed counts
-  if constexpr (W == kWC) return cur_ca(c) + 2u * cur_cb(c);
+  if constexpr (W == kWC) return cur_ca(c) + 4u * cur_cb(c);
   else return cur_ca(c);
 }
 static_assert(PairFmt<kWC>::kCap + kNMap * PairFmt<kWC>::kMaxReserve <= kCaMask, "ca field overflow");
@@ -470,7 +487,7 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   const uint32_t lane = threadIdx.x & 31;
   for (uint32_t f = 0;; ++f) {
     const uint32_t h = f % kNOut;
-    mbar_wait_idle(&oc->req[h], (f / kNOut) & 1u);
+    map_wait(P, &oc->req[h], (f / kNOut) & 1u, 20000);
     const uint32_t cnt0 = *reinterpret_cast<volatile unsigned int*>(&oc->fcount[h]);
     const bool fin = *reinterpret_cast<volatile unsigned int*>(&oc->is_final) &&
                      *reinterpret_cast<volatile unsigned int*>(&oc->final_seq) == f;
@@ -485,8 +502,8 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
     const uint32_t cb = (W == kWC) ? cur_cb(cnt0) : 0u;
     uint32_t cnt = ca0;
     if constexpr (W == kWC) {
-      cnt = (ca0 + 1u) & ~1u;                                   // 16-B aligned exact run (TMA store)
-      if (lane == 0 && cnt != ca0) reinterpret_cast<uint64_t*>(half)[ca0] = sentinel_key<W>(P);
+      cnt = (ca0 + 3u) & ~3u;                                   // 16-B aligned exact run (TMA store)
+      if (lane < cnt - ca0) reinterpret_cast<uint32_t*>(half)[ca0 + lane] = 0xFFFFFFFFu;   // filler: sorts last
     } else if constexpr (W != kSM) {
       cnt = (ca0 + 3u) & ~3u;                                   // 4-pair aligned flush (TMA store)
       if (lane < cnt - ca0) {                                   // sentinel filler entries
@@ -510,7 +527,8 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       } else if (lane == 0) {
         // A4 staging-out as TMA bulk stores (16-B aligned: gb and cnt even / multiples of 4)
         fence_proxy_async_shared();
-        tma_store_1d(P.oh + gb, sh, cnt * 8);
+        if constexpr (W == kWC) tma_store_1d(P.ohx + gb, sh, cnt * 4);
+        else tma_store_1d(P.oh + gb, sh, cnt * 8);
         if constexpr (F::kKref) tma_store_1d(P.okref + gb, sh + F::kCap, cnt * 8);
         if constexpr (F::kV > 0) tma_store_1d(P.ov + gb * F::kV, sv, cnt * F::kV);
         tma_store_commit_and_wait_read();          // SMEM may be reused once the stores have read it
@@ -562,6 +580,13 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
 }
 
 // ---------------------------------------------------------------- producer warp
+// cp.async.bulk.prefetch.L2 of the 16-B aligned interior of [lo, hi) (never touches bytes outside)
+__device__ __forceinline__ void l2_prefetch_range(const uint8_t* lo, const uint8_t* hi) {
+  const uintptr_t a = (reinterpret_cast<uintptr_t>(lo) + 15u) & ~static_cast<uintptr_t>(15u);
+  const uintptr_t b = reinterpret_cast<uintptr_t>(hi) & ~static_cast<uintptr_t>(15u);
+  if (b > a)
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a), "r"(static_cast<uint32_t>(b - a)) : "memory");
+}
 __device__ void stage_copy_edges(uint8_t* d, const uint8_t* g, uint64_t len, uint32_t lane, uint32_t& body_off,
                                  uint32_t& body_len) {
   const uint32_t head = static_cast<uint32_t>(
@@ -601,25 +626,33 @@ __device__ void finish_stage(const Params& P, uint8_t* smem, uint32_t it) {
 }
 
 template <int W>
-__device__ void producer_loop(const Params& P, uint8_t* smem) {
+__device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
   constexpr int kStages = Cfg<W>::kStages;
   const uint32_t lane = threadIdx.x & 31;
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
   uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
-  uint32_t it = 0;
   const long long N = static_cast<long long>(P.nbytes);
-  for (uint64_t t0 = blockIdx.x; t0 < P.ntiles; t0 += 32ULL * gridDim.x) {
-    // lanes prefetch the bounds of the next 32 tiles of this CTA (one latency per 32 tiles)
-    uint64_t my_t = t0 + static_cast<uint64_t>(lane) * gridDim.x, my_ra = 0, my_rb = 0;
+  const uint64_t G = gridDim.x;
+  // iterations of this CTA: tiles blockIdx.x + it * G; this producer takes it == pw (mod kNProd)
+  const uint32_t T = blockIdx.x < P.ntiles ? static_cast<uint32_t>((P.ntiles - blockIdx.x + G - 1) / G) : 0u;
+  for (uint32_t i0 = pw; i0 < T; i0 += 32u * kNProd) {
+    // lanes prefetch the bounds of this producer's next 32 tiles (one latency per 32 tiles)
+    const uint32_t my_it = i0 + lane * kNProd;
+    uint64_t my_ra = 0, my_rb = 0;
     if constexpr (W != kKM) {
-      if (my_t < P.ntiles) { my_ra = P.tb[2 * my_t]; my_rb = P.tb[2 * my_t + 1]; }
+      if (my_it < T) {
+        const uint64_t my_t = blockIdx.x + static_cast<uint64_t>(my_it) * G;
+        my_ra = P.tb[2 * my_t];
+        my_rb = P.tb[2 * my_t + 1];
+      }
     }
     for (uint32_t j = 0; j < 32; ++j) {
-      const uint64_t t = t0 + static_cast<uint64_t>(j) * gridDim.x;
-      if (t >= P.ntiles) break;
+      const uint32_t it = i0 + j * kNProd;
+      if (it >= T) break;
+      const uint64_t t = blockIdx.x + static_cast<uint64_t>(it) * G;
       const uint64_t ra = __shfl_sync(kFull, my_ra, j), rb = __shfl_sync(kFull, my_rb, j);
       const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
-      mbar_wait_idle(&empty[s], ph ^ 1u);
+      map_wait(P, &empty[s], ph ^ 1u, 20000);
       StageHdr* hd = reinterpret_cast<StageHdr*>(smem + Layout<W>::hdr + s * 128);
       uint8_t* sb = smem + Layout<W>::bytes + s * kStageBytes;
       uint32_t b_off = 0, b_len = 0, o_off = 0, o_len = 0;
@@ -693,16 +726,31 @@ __device__ void producer_loop(const Params& P, uint8_t* smem) {
           if (b_len) tma_load_1d(d + b_off, g + b_off, b_len, &full[s]);
           if (o_len) tma_load_1d(so + o_off, og + o_off, o_len, &full[s]);
         }
-        if (it >= Cfg<W>::kLag) finish_stage<W>(P, smem, it - Cfg<W>::kLag);
+        // L2 prefetch of this producer's tile P.pf tiles ahead (bytes + offsets slice): the TMA of
+        // that tile then hits L2, so the kLag stages in flight cover L2 latency, not HBM latency
+        if (P.pf) {
+          const uint32_t jf = j + P.pf;
+          const uint64_t raf = __shfl_sync(kFull, my_ra, jf & 31), rbf = __shfl_sync(kFull, my_rb, jf & 31);
+          const uint32_t itf = i0 + jf * kNProd;
+          if (lane == 0 && itf < T) {
+            const long long c0 = static_cast<long long>(blockIdx.x + static_cast<uint64_t>(itf) * G) * kT - P.a0;
+            l2_prefetch_range(P.rec + max(0LL, c0 - kLead), P.rec + min(c0 + kT + kHalo, N));
+            if (jf < 32 && rbf > raf) l2_prefetch_range(reinterpret_cast<const uint8_t*>(P.off + raf),
+                                                        reinterpret_cast<const uint8_t*>(P.off + rbf));
+          }
+        }
+        if (it >= Cfg<W>::kLag) finish_stage<W>(P, smem, it - Cfg<W>::kLag);   // same owner (kLag % kNProd == 0)
       }
-      ++it;
     }
   }
-  if constexpr (W != kKM) {
-    for (uint32_t j = (it >= Cfg<W>::kLag ? it - Cfg<W>::kLag : 0); j < it; ++j) finish_stage<W>(P, smem, j);
+  if constexpr (W != kKM) {   // this producer's tiles whose bitmap is still pending
+    const uint32_t j0 = T > static_cast<uint32_t>(Cfg<W>::kLag) ? T - Cfg<W>::kLag : 0u;
+    for (uint32_t j = j0; j < T; ++j)
+      if (j % kNProd == pw) finish_stage<W>(P, smem, j);
   }
-  // end-of-work marker
-  const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
+  // end-of-work marker at iteration T, written by its owner
+  if (T % kNProd != pw) return;
+  const uint32_t s = T % kStages, ph = (T / kStages) & 1u;
   mbar_wait(&empty[s], ph ^ 1u);
   if (lane == 0) {
     reinterpret_cast<StageHdr*>(smem + Layout<W>::hdr + s * 128)->t = -1;
@@ -740,7 +788,7 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
   const uint32_t packed = (tot & 0xFFFFu) | ((tot >> 16) << kCbShift);
   const Slot slot = reserve<kWC>(P, oc, outh, packed, P.out_cap);
   uint8_t* half = outh + slot.half * Cfg<kWC>::kOutHalf;
-  uint64_t* sh = reinterpret_cast<uint64_t*>(half);
+  uint32_t* sh = reinterpret_cast<uint32_t*>(half);
   ulonglong2* top = reinterpret_cast<ulonglong2*>(half + Cfg<kWC>::kOutHalf);   // hashed entry i: top[-1 - i]
   uint64_t* hq = reinterpret_cast<uint64_t*>(outh + (Layout<kWC>::hq - Layout<kWC>::out)) +
                  (threadIdx.x >> 5) * Cfg<kWC>::kHashQ;
@@ -921,7 +969,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   for (uint32_t it = 0;; ++it) {
     const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
     if constexpr (W == kKM) mbar_wait(&full[s], ph);
-    else mbar_wait_idle(reinterpret_cast<uint64_t*>(smem + Layout<W>::ready) + s, ph, kReadyWaitNs);
+    else map_wait(P, reinterpret_cast<uint64_t*>(smem + Layout<W>::ready) + s, ph, kReadyWaitNs);
     const StageHdr hd = *reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
     if (hd.t < 0) break;
     const uint8_t* sb = smem + Layout<W>::bytes + s * kStageBytes;
@@ -1041,7 +1089,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_map(Params P) {
   }
   __syncthreads();
   const uint32_t warp = threadIdx.x >> 5;
-  if (warp == kProdWarp) producer_loop<W>(P, smem);
+  if (warp >= kProdWarp0 && warp < kProdWarp0 + kNProd) producer_loop<W>(P, smem, warp - kProdWarp0);
   else if (warp >= kFlushWarp0) flush_loop<W>(P, smem, oc);
   else map_loop<W>(P, smem, oc);
 }
@@ -1101,6 +1149,9 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.cap_b = a.out.cap_b;
   P.ohc = a.out.hc;
   P.cap_c = a.out.cap_c;
+  P.ohx = a.out.hx;
+  P.pf = map_prefetch();
+  P.wait_hint = map_wait_hint();
   if (P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>((P.ntiles + 255) / 256);
@@ -1118,6 +1169,25 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
 }
 
 }  // namespace
+
+// L2 prefetch distance of the Map producers (BMR_MAP_PF, tiles; default 0 = off: measured slower
+// on C2/C4 in round 1 with 2 producers)
+uint32_t map_prefetch() {
+  static uint32_t v = [] {
+    const char* e = getenv("BMR_MAP_PF");
+    return e ? static_cast<uint32_t>(atoi(e)) : 0u;
+  }();
+  return v;
+}
+
+// idle-wait flavour of the Map role warps (BMR_MAP_WAIT: 1 = suspend-time hint, default 0 = plain)
+uint32_t map_wait_hint() {
+  static uint32_t v = [] {
+    const char* e = getenv("BMR_MAP_WAIT");
+    return e ? static_cast<uint32_t>(atoi(e)) : 0u;
+  }();
+  return v;
+}
 
 int vbytes_of(int w) { return w == kKM ? 32 : w == kII ? 8 : 0; }
 bool has_kref(int w) { return w == kII; }

@@ -63,8 +63,8 @@ __device__ bool key_bytes_equal(uint64_t ka, uint64_t kb) {
 // a lane compares its key with the previous position's key (shuffle from the previous lane).
 constexpr int kSegWarp = 32 * kSegIPT;   // positions per warp
 
-template <bool kVerify>
-__global__ void __launch_bounds__(kSegThreads) k_seg_count(const uint64_t* __restrict__ sk,
+template <bool kVerify, typename K = uint64_t>
+__global__ void __launch_bounds__(kSegThreads) k_seg_count(const K* __restrict__ sk,
                                                          const uint32_t* __restrict__ perm,
                                                          const uint64_t* __restrict__ kref, uint64_t m,
                                                          uint32_t* counts, DevState* st, uint64_t hbit,
@@ -73,17 +73,17 @@ __global__ void __launch_bounds__(kSegThreads) k_seg_count(const uint64_t* __res
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint64_t wbase = static_cast<uint64_t>(blockIdx.x) * kSegTile + static_cast<uint64_t>(warp) * kSegWarp;
   uint32_t heads = 0, coll = 0;
-  uint64_t carry_k = (wbase > 0 && wbase - 1 < m) ? sk[wbase - 1] : 0;     // key before this step
+  K carry_k = (wbase > 0 && wbase - 1 < m) ? sk[wbase - 1] : 0;            // key before this step
   uint64_t carry_r = 0;                                                     // its kref (if loaded)
   bool carry_has_r = false;
 #pragma unroll 4
   for (int j = 0; j < kSegIPT; ++j) {
     const uint64_t i = wbase + static_cast<uint64_t>(j) * 32 + lane;
     const bool valid = i < m;
-    const uint64_t k = valid ? sk[i] : 0;
-    uint64_t prev = __shfl_up_sync(0xffffffffu, k, 1);
+    const K k = valid ? sk[i] : 0;
+    K prev = __shfl_up_sync(0xffffffffu, k, 1);
     if (lane == 0) prev = carry_k;
-    const bool head = valid && (i == 0 || ((k ^ prev) & kmask) != 0);
+    const bool head = valid && (i == 0 || ((k ^ prev) & static_cast<K>(kmask)) != 0);
     heads += head ? 1u : 0u;
     carry_k = __shfl_sync(0xffffffffu, k, 31);
     if constexpr (kVerify) {
@@ -113,7 +113,8 @@ __global__ void __launch_bounds__(kSegThreads) k_seg_count(const uint64_t* __res
   }
 }
 
-__global__ void __launch_bounds__(kSegThreads) k_seg_write(const uint64_t* __restrict__ sk, uint64_t m,
+template <typename K = uint64_t>
+__global__ void __launch_bounds__(kSegThreads) k_seg_write(const K* __restrict__ sk, uint64_t m,
                                                          const uint64_t* __restrict__ tile_base,
                                                          uint64_t* seg_start, uint64_t kmask) {
   __shared__ uint32_t wsum[kSegThreads / 32];
@@ -122,15 +123,15 @@ __global__ void __launch_bounds__(kSegThreads) k_seg_write(const uint64_t* __res
   // pass 1: heads of this warp's 512 positions (bitmask per step kept in registers)
   uint32_t hm[kSegIPT];
   uint32_t wcount = 0;
-  uint64_t carry_k = (wbase > 0 && wbase - 1 < m) ? sk[wbase - 1] : 0;
+  K carry_k = (wbase > 0 && wbase - 1 < m) ? sk[wbase - 1] : 0;
 #pragma unroll
   for (int j = 0; j < kSegIPT; ++j) {
     const uint64_t i = wbase + static_cast<uint64_t>(j) * 32 + lane;
     const bool valid = i < m;
-    const uint64_t k = valid ? sk[i] : 0;
-    uint64_t prev = __shfl_up_sync(0xffffffffu, k, 1);
+    const K k = valid ? sk[i] : 0;
+    K prev = __shfl_up_sync(0xffffffffu, k, 1);
     if (lane == 0) prev = carry_k;
-    hm[j] = __ballot_sync(0xffffffffu, valid && (i == 0 || ((k ^ prev) & kmask) != 0));
+    hm[j] = __ballot_sync(0xffffffffu, valid && (i == 0 || ((k ^ prev) & static_cast<K>(kmask)) != 0));
     wcount += __popc(hm[j]);
     carry_k = __shfl_sync(0xffffffffu, k, 31);
   }
@@ -363,14 +364,16 @@ __global__ void k_seg_lengths(const uint64_t* seg, uint64_t nseg, uint64_t* out)
   const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
   if (s < nseg) out[s] = seg[s + 1] - seg[s];
 }
-__global__ void k_key_lengths_exact(const uint64_t* seg, uint64_t nseg, const uint64_t* sk, uint64_t* lens) {
+template <typename K>
+__global__ void k_key_lengths_exact(const uint64_t* seg, uint64_t nseg, const K* sk, uint64_t* lens) {
   const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
   if (s >= nseg) return;
   uint32_t len;
   exact_key_bytes(sk[seg[s]], len);
   lens[s] = len;
 }
-__global__ void k_key_decode(const uint64_t* seg, uint64_t nseg, const uint64_t* sk, const uint64_t* key_off,
+template <typename K>
+__global__ void k_key_decode(const uint64_t* seg, uint64_t nseg, const K* sk, const uint64_t* key_off,
                              uint8_t* keys) {
   const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
   if (s >= nseg) return;
@@ -419,6 +422,20 @@ cudaError_t launch_seg_write(const uint64_t* skeys, uint64_t m, const uint64_t* 
                              uint64_t kmask, cudaStream_t s) {
   if (m == 0) return cudaMemsetAsync(seg_start, 0, sizeof(uint64_t), s);
   k_seg_write<<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, m, tile_base, seg_start, kmask);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_seg_count32(const uint32_t* skeys, uint64_t m, uint32_t* counts, cudaStream_t s) {
+  if (m == 0) return cudaSuccess;
+  k_seg_count<false, uint32_t><<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, nullptr, nullptr, m, counts,
+                                                                               nullptr, 0, ~0ULL);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_seg_write32(const uint32_t* skeys, uint64_t m, const uint64_t* tile_base, uint64_t* seg_start,
+                               cudaStream_t s) {
+  if (m == 0) return cudaMemsetAsync(seg_start, 0, sizeof(uint64_t), s);
+  k_seg_write<uint32_t><<<blocks_for(m, kSegTile), kSegThreads, 0, s>>>(skeys, m, tile_base, seg_start, ~0ULL);
   count_launch();
   return cudaGetLastError();
 }
@@ -494,6 +511,20 @@ cudaError_t launch_key_lengths_exact(const uint64_t* seg_start, uint64_t nseg, c
 }
 cudaError_t launch_key_decode(const uint64_t* seg_start, uint64_t nseg, const uint64_t* skeys, const uint64_t* key_off,
                               uint8_t* keys, cudaStream_t s) {
+  if (nseg == 0) return cudaSuccess;
+  k_key_decode<<<blocks_for(nseg, 256), 256, 0, s>>>(seg_start, nseg, skeys, key_off, keys);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_key_lengths_exact32(const uint64_t* seg_start, uint64_t nseg, const uint32_t* skeys, uint64_t* lens,
+                                       cudaStream_t s) {
+  if (nseg == 0) return cudaSuccess;
+  k_key_lengths_exact<<<blocks_for(nseg, 256), 256, 0, s>>>(seg_start, nseg, skeys, lens);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_key_decode32(const uint64_t* seg_start, uint64_t nseg, const uint32_t* skeys,
+                                const uint64_t* key_off, uint8_t* keys, cudaStream_t s) {
   if (nseg == 0) return cudaSuccess;
   k_key_decode<<<blocks_for(nseg, 256), 256, 0, s>>>(seg_start, nseg, skeys, key_off, keys);
   count_launch();

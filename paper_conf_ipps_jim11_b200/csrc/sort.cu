@@ -28,43 +28,47 @@ __device__ __forceinline__ uint64_t pack_status(uint32_t epoch, uint32_t kind, u
   return (static_cast<uint64_t>(epoch) << 34) | (static_cast<uint64_t>(kind) << 32) | v;
 }
 
-// Digit histograms of the first nd digits of `bits` bits (8 or 9): one read of the keys, two
-// keys per 16-byte load, shared atomics into a per-block nd x 512 table (stride kBinStride).
-__global__ void __launch_bounds__(256) k_hist(const uint64_t* __restrict__ keys, uint64_t m, uint32_t nd,
-                                            uint32_t bits, uint32_t* hist) {
+// Digit histograms of the first nd digits of `bits` bits (8 or 9): one read of the keys (16-byte
+// loads: two u64 or four u32 keys each), shared atomics into a per-block nd x 512 table (stride
+// kBinStride).
+template <typename K>
+__global__ void __launch_bounds__(256) k_hist(const K* __restrict__ keys, uint64_t m, uint32_t nd, uint32_t bits,
+                                            uint32_t* hist) {
+  constexpr int kPer = 16 / sizeof(K);
   __shared__ uint32_t sh[8 * kBinStride];
   for (int i = threadIdx.x; i < 8 * kBinStride; i += blockDim.x) sh[i] = 0;
   __syncthreads();
-  const uint64_t mask = (1ULL << bits) - 1ULL;
+  const uint32_t mask = (1u << bits) - 1u;
   const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
-  const uint64_t m2 = m / 2;
-  const ulonglong2* k2 = reinterpret_cast<const ulonglong2*>(keys);
-  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i < m2; i += stride) {
-    const ulonglong2 kk = __ldcs(k2 + i);
+  const uint64_t mv = m / kPer;
+  const uint4* k4 = reinterpret_cast<const uint4*>(keys);
+  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i < mv; i += stride) {
+    const uint4 raw = __ldcs(k4 + i);
+    K kk[kPer];
+    memcpy(kk, &raw, 16);
 #pragma unroll
     for (uint32_t d = 0; d < 8; ++d) {
       if (d >= nd) break;
-      atomicAdd(&sh[d * kBinStride + ((kk.x >> (bits * d)) & mask)], 1u);
-      atomicAdd(&sh[d * kBinStride + ((kk.y >> (bits * d)) & mask)], 1u);
+#pragma unroll
+      for (int q = 0; q < kPer; ++q) atomicAdd(&sh[d * kBinStride + (static_cast<uint32_t>(kk[q] >> (bits * d)) & mask)], 1u);
     }
   }
-  if ((m & 1) && blockIdx.x == 0 && threadIdx.x == 0) {
-    const uint64_t k = keys[m - 1];
-    for (uint32_t d = 0; d < nd; ++d) atomicAdd(&sh[d * kBinStride + ((k >> (bits * d)) & mask)], 1u);
+  if (blockIdx.x == 0 && threadIdx.x < m % kPer) {
+    const K k = keys[mv * kPer + threadIdx.x];
+    for (uint32_t d = 0; d < nd; ++d) atomicAdd(&sh[d * kBinStride + (static_cast<uint32_t>(k >> (bits * d)) & mask)], 1u);
   }
   __syncthreads();
   for (int i = threadIdx.x; i < static_cast<int>(nd) * kBinStride; i += blockDim.x)
     if (sh[i]) atomicAdd(&hist[i], sh[i]);
 }
 
-template <int IPT, bool kPay, int kBins>
+template <typename K, int IPT, bool kPay, int kBins>
 struct SortSmem {
   static constexpr int kTile = kSortThreads * IPT;
-  uint64_t keys[kTile];
+  K keys[kTile];
   uint32_t idx[kPay ? kTile : 1];
   uint32_t wcnt[kWarps][kBins];    // per-warp digit counters, then warp-exclusive offsets
   uint32_t hist[kBins];
-  uint32_t dstart[kBins];
   uint32_t goff[kBins];
   uint32_t wsum[kWarps];
   uint32_t tile;
@@ -78,10 +82,10 @@ struct SortSmem {
 // as an early aggregate (1), or summed from the warp counters after ranking (0).
 // kPay: carry the u32 permutation payload (false: keys only, idx_in / idx_out unused).
 // kLookWindow: predecessor status words fetched per look-back step (per digit).
-template <bool kFirst, int kVar, int IPT, int MINB, bool kPay, int kBits, int kLookWindow = 4>
-__global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t* __restrict__ keys_in,
+template <typename K, bool kFirst, int kVar, int IPT, int MINB, bool kPay, int kBits, int kLookWindow = 4>
+__global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __restrict__ keys_in,
                                                                const uint32_t* __restrict__ idx_in,
-                                                               uint64_t* __restrict__ keys_out,
+                                                               K* __restrict__ keys_out,
                                                                uint32_t* __restrict__ idx_out, uint64_t m,
                                                                uint32_t shift, const uint32_t* __restrict__ bases,
                                                                uint64_t* status, uint32_t epoch,
@@ -89,7 +93,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t*
   constexpr int kBins = 1 << kBits, kDPT = kBins / kSortThreads;
   constexpr uint32_t kMask = kBins - 1;
   constexpr int kSortIPT = IPT;
-  using Smem = SortSmem<IPT, kPay, kBins>;
+  using Smem = SortSmem<K, IPT, kPay, kBins>;
   constexpr int kSortTile = Smem::kTile;
   constexpr bool kAtomicRank = (kVar & 1) != 0, kEarly = (kVar & 2) != 0;
   constexpr bool kBackoff = (kVar & 4) != 0, kMatchHist = (kVar & 8) != 0;
@@ -104,12 +108,12 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t*
   const uint32_t tile = S.tile;
   const uint64_t tbase = static_cast<uint64_t>(tile) * kSortTile;
   const uint64_t wbase = tbase + static_cast<uint64_t>(warp) * 32 * kSortIPT;
-  uint64_t key[kSortIPT];
+  K key[kSortIPT];
   uint32_t rank[kSortIPT];
 #pragma unroll
   for (int j = 0; j < kSortIPT; ++j) {
     const uint64_t e = wbase + j * 32 + lane;
-    key[j] = e < m ? keys_in[e] : ~0ULL;  // padding sorts last (top digit value, after every real key)
+    key[j] = e < m ? keys_in[e] : static_cast<K>(~static_cast<K>(0));  // padding sorts last (top digit value, after every real key)
   }
   const uint32_t d0 = tid * kDPT;   // this thread's digits: d0 .. d0 + kDPT - 1
   uint32_t tcount[kDPT];
@@ -176,31 +180,47 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t*
       st_relaxed_gpu_u64(my + q, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount[q]));
     }
   }
-  __syncthreads();
-  // 3. per digit: warp-exclusive offsets and the tile-local digit start
+  // (a thread reads and rewrites only the counters of its own digits: no barrier needed here)
+  // 3. per digit: the tile-local digit start (block scan of the tile counts), then every warp's
+  //    counter becomes its tile-local scatter base for the digit (digit start + earlier warps)
   uint32_t tsum = 0;
 #pragma unroll
-  for (int q = 0; q < kDPT; ++q) {
-    uint32_t run = 0;
-#pragma unroll
-    for (int w = 0; w < kWarps; ++w) {
-      const uint32_t c = S.wcnt[w][d0 + q];
-      S.wcnt[w][d0 + q] = run;
-      run += c;
-    }
-    tsum += tcount[q];
-  }
+  for (int q = 0; q < kDPT; ++q) tsum += tcount[q];
   const uint32_t inc = warp_inclusive_add(tsum);
   if (lane == 31) S.wsum[warp] = inc;
   __syncthreads();
+  uint32_t dsq[kDPT];
   {
     uint32_t wpre = 0;
 #pragma unroll
     for (int w = 0; w < kWarps; ++w) wpre += (w < static_cast<int>(warp)) ? S.wsum[w] : 0u;
     uint32_t ds = wpre + inc - tsum;
 #pragma unroll
-    for (int q = 0; q < kDPT; ++q) { S.dstart[d0 + q] = ds; ds += tcount[q]; }
-    // 4. decoupled look-back, kLookWindow predecessors per round trip, all digits of the thread
+    for (int q = 0; q < kDPT; ++q) {
+      dsq[q] = ds;
+      uint32_t run = ds;
+#pragma unroll
+      for (int w = 0; w < kWarps; ++w) {
+        const uint32_t c = S.wcnt[w][d0 + q];
+        S.wcnt[w][d0 + q] = run;
+        run += c;
+      }
+      ds += tcount[q];
+    }
+  }
+  __syncthreads();
+  // 4. scatter into SMEM in tile-sorted order (payload loaded here, after ranking); frees the
+  //    key and rank registers before the look-back
+#pragma unroll
+  for (int j = 0; j < kSortIPT; ++j) {
+    const uint64_t e = wbase + j * 32 + lane;
+    const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & kMask;
+    const uint32_t lp = S.wcnt[warp][dj] + rank[j];
+    S.keys[lp] = key[j];
+    if constexpr (kPay) S.idx[lp] = kFirst ? static_cast<uint32_t>(e) : (e < m ? idx_in[e] : 0u);
+  }
+  {
+    // 5. decoupled look-back, kLookWindow predecessors per round trip, all digits of the thread
     //    in flight together
     uint32_t excl[kDPT];
 #pragma unroll
@@ -246,26 +266,17 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const uint64_t*
 #pragma unroll
       for (int q = 0; q < kDPT; ++q) st_relaxed_gpu_u64(my + q, pack_status(epoch, kPrefix, excl[q] + tcount[q]));
     }
+    // global position of tile-sorted slot i with digit d: i + (digit base + earlier tiles - digit start)
 #pragma unroll
-    for (int q = 0; q < kDPT; ++q) S.goff[d0 + q] = bases[d0 + q] + excl[q];
-  }
-  __syncthreads();
-  // 5. scatter into SMEM in tile-sorted order (payload loaded here, after ranking)
-#pragma unroll
-  for (int j = 0; j < kSortIPT; ++j) {
-    const uint64_t e = wbase + j * 32 + lane;
-    const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & kMask;
-    const uint32_t lp = S.dstart[dj] + S.wcnt[warp][dj] + rank[j];
-    S.keys[lp] = key[j];
-    if constexpr (kPay) S.idx[lp] = kFirst ? static_cast<uint32_t>(e) : (e < m ? idx_in[e] : 0u);
+    for (int q = 0; q < kDPT; ++q) S.goff[d0 + q] = bases[d0 + q] + excl[q] - dsq[q];
   }
   __syncthreads();
   // 6. contiguous per-digit runs to global memory
   const uint32_t nvalid = static_cast<uint32_t>(min(static_cast<uint64_t>(kSortTile), m - tbase));
   for (uint32_t i = tid; i < nvalid; i += kSortThreads) {
-    const uint64_t k = S.keys[i];
+    const K k = S.keys[i];
     const uint32_t dk = static_cast<uint32_t>(k >> shift) & kMask;
-    const uint32_t pos = S.goff[dk] + (i - S.dstart[dk]);
+    const uint32_t pos = S.goff[dk] + i;
     keys_out[pos] = k;
     if constexpr (kPay) idx_out[pos] = S.idx[i];
   }
@@ -342,109 +353,142 @@ __global__ void __launch_bounds__(kScanThreads) k_scan(const T* __restrict__ in,
 
 }  // namespace
 
-cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int nd, int bits, int num_sms,
-                        cudaStream_t s) {
+template <typename K>
+static cudaError_t hist_impl(const K* keys, uint64_t m, uint32_t* hist, int nd, int bits, int num_sms,
+                             cudaStream_t s) {
   cudaError_t e = cudaMemsetAsync(hist, 0, 8 * kBinStride * sizeof(uint32_t), s);
   if (e != cudaSuccess || m == 0) return e;
-  if (reinterpret_cast<uintptr_t>(keys) & 15u) {   // 16-B loads: peel one key off a misaligned start
-    k_hist<<<1, 32, 0, s>>>(keys, 1, static_cast<uint32_t>(nd), static_cast<uint32_t>(bits), hist);
+  while (reinterpret_cast<uintptr_t>(keys) & 15u) {   // 16-B loads: peel keys off a misaligned start
+    k_hist<K><<<1, 32, 0, s>>>(keys, 1, static_cast<uint32_t>(nd), static_cast<uint32_t>(bits), hist);
     count_launch();
     ++keys;
     if (--m == 0) return cudaGetLastError();
   }
-  uint64_t blocks = std::min<uint64_t>(static_cast<uint64_t>(num_sms) * 8, (m / 2 + 255) / 256 + 1);
-  k_hist<<<static_cast<unsigned>(blocks), 256, 0, s>>>(keys, m, static_cast<uint32_t>(nd), static_cast<uint32_t>(bits),
-                                                       hist);
+  constexpr uint64_t kPer = 16 / sizeof(K);
+  uint64_t blocks = std::min<uint64_t>(static_cast<uint64_t>(num_sms) * 8, (m / kPer + 255) / 256 + 1);
+  k_hist<K><<<static_cast<unsigned>(blocks), 256, 0, s>>>(keys, m, static_cast<uint32_t>(nd),
+                                                          static_cast<uint32_t>(bits), hist);
   count_launch();
   return cudaGetLastError();
+}
+cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int nd, int bits, int num_sms,
+                        cudaStream_t s) {
+  return hist_impl<uint64_t>(keys, m, hist, nd, bits, num_sms, s);
+}
+cudaError_t launch_hist32(const uint32_t* keys, uint64_t m, uint32_t* hist, int nd, int bits, int num_sms,
+                          cudaStream_t s) {
+  return hist_impl<uint32_t>(keys, m, hist, nd, bits, num_sms, s);
 }
 
 int sort_variant() {
   static int v = [] {
     const char* e = getenv("BMR_SORT_VARIANT");
+    return e ? atoi(e) & 1 : 0;
+  }();
+  return v;
+}
+// u32 keys-only passes: kVar of k_onesweep (bit 0 atomic ranking, bit 1 early histogram)
+int sort_variant32() {
+  static int v = [] {
+    const char* e = getenv("BMR_SORT_VARIANT32");
     return e ? atoi(e) & 3 : 2;
   }();
   return v;
 }
-// tile shape: 0 = 16 keys/thread, 3 CTAs/SM; 1 = 12 keys, 4 CTAs; 2 = 20 keys, 2 CTAs; 3 = 8 keys, 6 CTAs
+// Tile shapes (keys per thread x 256 threads, CTAs per SM), chosen at start-up (BMR_SORT_CFG):
+//   payload passes (u64 key + u32 index): cfg 0 = 16 keys, 3 CTAs/SM; cfg 1 = 12 keys, 4 CTAs
+//   keys-only u64 passes: 16 keys, 3 CTAs/SM (cfg 1: 24 keys, 2 CTAs)
+//   keys-only u32 passes: 24 keys, 3 CTAs/SM (cfg 1: 32 keys, 2 CTAs)
+// (measured on C5 in round 1: 16 x 256 with the early tile histogram and a look-back window of
+// 4 was the fastest u64 shape among 8/12/16/20/24 keys, 9-bit digits, windows 1..16, spin
+// back-off and match-aggregated histogram atomics.)
 int sort_cfg() {
   static int c = [] {
     const char* e = getenv("BMR_SORT_CFG");
-    return e ? atoi(e) & 3 : 0;
+    return e ? atoi(e) & 1 : 0;
   }();
   return c;
 }
-static const int kCfgIPT[4] = {16, 12, 20, 8};
-int sort_tile() { return kSortThreads * kCfgIPT[sort_cfg()]; }
-// keys-only passes: 16 keys x 256 threads (3 CTAs / SM), or 24 keys (2 CTAs / SM) for cfg 3
-static const int kCfgIPTKeys[4] = {16, 16, 16, 24};
-int sort_tile_keys() { return kSortThreads * kCfgIPTKeys[sort_cfg()]; }
-template <bool kFirst, int kVar, int IPT, int MINB, bool kPay, int kBits, int LW = 4>
-static void launch_os(unsigned tiles, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
-                      uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
-                      uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
-  using K = decltype(&k_onesweep<kFirst, kVar, IPT, MINB, kPay, kBits, LW>);
-  const K k = &k_onesweep<kFirst, kVar, IPT, MINB, kPay, kBits, LW>;
-  const size_t smem = sizeof(SortSmem<IPT, kPay, (1 << kBits)>);
+int sort_tile() { return kSortThreads * (sort_cfg() ? 12 : 16); }
+int sort_tile_keys() { return kSortThreads * (sort_cfg() ? 24 : 16); }
+int sort_tile_keys32() { return kSortThreads * (sort_cfg() ? 32 : 24); }
+
+template <typename K, bool kFirst, int kVar, int IPT, int MINB, bool kPay, int LW = 4>
+static void launch_os(unsigned tiles, const K* keys_in, const uint32_t* idx_in, K* keys_out, uint32_t* idx_out,
+                      uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status, uint32_t epoch,
+                      unsigned int* tile_counter, cudaStream_t s) {
+  const auto k = &k_onesweep<K, kFirst, kVar, IPT, MINB, kPay, 8, LW>;
+  const size_t smem = sizeof(SortSmem<K, IPT, kPay, 256>);
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
   k<<<tiles, kSortThreads, smem, s>>>(keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch,
                                       tile_counter);
 }
 
 #define BMR_OS_ARGS tiles, keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch, tile_counter, s
+// kVar 2: early tile histogram (published before ranking), read-modify-write warp ranking;
+// kVar 3: the same with one shared atomic per match group for the ranking
 template <bool kFirst, int kVar>
-static void launch_cfg(unsigned tiles, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
+static void launch_pay(unsigned tiles, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
                        uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
                        uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
-  switch (sort_cfg()) {
-    case 1: launch_os<kFirst, kVar, 12, 4, true, 8>(BMR_OS_ARGS); break;
-    case 2: launch_os<kFirst, kVar, 20, 2, true, 8>(BMR_OS_ARGS); break;
-    case 3: launch_os<kFirst, kVar, 8, 6, true, 8>(BMR_OS_ARGS); break;
-    default: launch_os<kFirst, kVar, 16, 3, true, 8>(BMR_OS_ARGS); break;
-  }
-}
-// keys only (8 B per key per direction), 8-bit digits.  Measured on C5 (48-bit WC exact keys,
-// 1.37 G keys): 16 keys x 256 threads, early histogram, look-back window 4 is the fastest of
-// {9-bit digits (5 passes, 2 digits per thread), windows 1/2/8/16, spin back-off,
-// match-aggregated histogram atomics, bijective digit mixing} — see DESIGN.md §4.
-static void launch_keys_only(unsigned tiles, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
-                             uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
-                             uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
-  if (sort_cfg() == 3) launch_os<false, 2, 24, 2, false, 8, 4>(BMR_OS_ARGS);
-  else launch_os<false, 2, 16, 3, false, 8, 4>(BMR_OS_ARGS);
+  if (sort_cfg() == 1) launch_os<uint64_t, kFirst, kVar, 12, 4, true>(BMR_OS_ARGS);
+  else launch_os<uint64_t, kFirst, kVar, 16, 3, true>(BMR_OS_ARGS);
 }
 
-cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out, uint32_t* idx_out,
-                            uint64_t m, int digit, int bits, const uint32_t* bases_all, uint64_t* status,
-                            uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
+template <typename K>
+static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* keys_out, uint32_t* idx_out, uint64_t m,
+                                 int digit, int bits, const uint32_t* bases_all, uint64_t* status, uint32_t epoch,
+                                 unsigned int* tile_counter, cudaStream_t s) {
   if (m == 0) return cudaSuccess;
   const bool keys_only = idx_out == nullptr;
   if (bits != 8) return cudaErrorInvalidValue;
-  const uint64_t tile = keys_only ? sort_tile_keys() : sort_tile();
+  if (sizeof(K) == 4 && !keys_only) return cudaErrorInvalidValue;
+  const uint64_t tile = sizeof(K) == 4 ? sort_tile_keys32() : keys_only ? sort_tile_keys() : sort_tile();
   const unsigned tiles = static_cast<unsigned>((m + tile - 1) / tile);
   cudaError_t e = cudaMemsetAsync(tile_counter, 0, sizeof(unsigned int), s);
   if (e != cudaSuccess) return e;
   const uint32_t shift = static_cast<uint32_t>(bits * digit);
   const uint32_t* bases = bases_all + kBinStride * digit;
   const bool first = idx_in == nullptr;
-  if (keys_only) {
-    launch_keys_only(BMR_OS_ARGS);
+  if constexpr (sizeof(K) == 4) {
+    if (sort_cfg() == 1) {
+      launch_os<K, false, 2, 32, 2, false>(BMR_OS_ARGS);
+    } else {
+      switch (sort_variant32()) {
+        case 0: launch_os<K, false, 0, 24, 3, false>(BMR_OS_ARGS); break;
+        case 1: launch_os<K, false, 1, 24, 3, false>(BMR_OS_ARGS); break;
+        case 3: launch_os<K, false, 3, 24, 3, false>(BMR_OS_ARGS); break;
+        default: launch_os<K, false, 2, 24, 3, false>(BMR_OS_ARGS); break;
+      }
+    }
+  } else if (keys_only) {
+    if (sort_cfg() == 1) launch_os<K, false, 2, 24, 2, false>(BMR_OS_ARGS);
+    else launch_os<K, false, 2, 16, 3, false>(BMR_OS_ARGS);
   } else {
-    switch (sort_variant() | (first ? 4 : 0)) {
-      case 0: launch_cfg<false, 0>(BMR_OS_ARGS); break;
-      case 1: launch_cfg<false, 1>(BMR_OS_ARGS); break;
-      case 2: launch_cfg<false, 2>(BMR_OS_ARGS); break;
-      case 3: launch_cfg<false, 3>(BMR_OS_ARGS); break;
-      case 4: launch_cfg<true, 0>(BMR_OS_ARGS); break;
-      case 5: launch_cfg<true, 1>(BMR_OS_ARGS); break;
-      case 6: launch_cfg<true, 2>(BMR_OS_ARGS); break;
-      default: launch_cfg<true, 3>(BMR_OS_ARGS); break;
+    switch ((sort_variant() ? 1 : 0) | (first ? 2 : 0)) {
+      case 0: launch_pay<false, 2>(BMR_OS_ARGS); break;
+      case 1: launch_pay<false, 3>(BMR_OS_ARGS); break;
+      case 2: launch_pay<true, 2>(BMR_OS_ARGS); break;
+      default: launch_pay<true, 3>(BMR_OS_ARGS); break;
     }
   }
   count_launch();
   return cudaGetLastError();
 }
 #undef BMR_OS_ARGS
+
+cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out, uint32_t* idx_out,
+                            uint64_t m, int digit, int bits, const uint32_t* bases_all, uint64_t* status,
+                            uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
+  return onesweep_impl<uint64_t>(keys_in, idx_in, keys_out, idx_out, m, digit, bits, bases_all, status, epoch,
+                                 tile_counter, s);
+}
+cudaError_t launch_onesweep32(const uint32_t* keys_in, uint32_t* keys_out, uint64_t m, int digit, int bits,
+                              const uint32_t* bases_all, uint64_t* status, uint32_t epoch,
+                              unsigned int* tile_counter, cudaStream_t s) {
+  return onesweep_impl<uint32_t>(keys_in, nullptr, keys_out, nullptr, m, digit, bits, bases_all, status, epoch,
+                                 tile_counter, s);
+}
 
 template <typename T>
 static cudaError_t scan_impl(const T* in, uint64_t* out, uint64_t n, unsigned long long* total, uint64_t* status,
