@@ -310,30 +310,33 @@ def main():
     per["reduce_ms"] = red / args.steps
     alg = algorithmic(inp, tot, args.steps)
     hbm, peak_kind = load_peaks()
-    if alg["passes_keys"]:   # WC: the keys-only pass over the exact stream dominates the step
-        kname = "k_onesweep (keys-only LSD pass, WC exact stream)"
-        sort_launch_ms = per["sort_keys_ms"] / alg["passes_keys"]
-        sort_launch_bytes = 8 * alg["pairs_exact"]
-    else:
-        kname = "k_onesweep (LSD pass)"
-        sort_launch_ms = per["sort_ms"] / max(alg["passes"], 1)
-        sort_launch_bytes = alg["sort"] / max(alg["passes"], 1)
-    roof = None
-    if alg["passes"]:
-        ach = sort_launch_bytes / (sort_launch_ms / 1e3) / 1e9
-        roof = {"kernel": kname, "bound": "hbm", "achieved": round(ach, 1), "peak": hbm,
-                "peak_kind": peak_kind, "unit": "GB/s", "frac": round(ach / hbm, 4), "traffic": None,
-                "bytes_per_launch": int(sort_launch_bytes), "ms_per_launch": round(sort_launch_ms, 4)}
+    # roofline of the dominant kernel (the larger device-time share of the step): the Map kernel
+    # or the onesweep LSD passes (all sort streams together, per launch)
     map_ach = alg["map"] / (per["map_ms"] / 1e3) / 1e9 if per["map_ms"] else 0.0
+    sort_ms_all = per["sort_ms"]
+    if alg["passes"] and sort_ms_all > per["map_ms"]:
+        if alg["passes_keys"] and per["sort_keys_ms"] > 0.5 * sort_ms_all:
+            kname = "k_onesweep (keys-only u32 LSD pass, WC exact stream)"
+            launch_ms = per["sort_keys_ms"] / alg["passes_keys"]
+            launch_bytes = 8 * alg["pairs_exact"]
+        else:
+            kname = "k_onesweep (LSD pass)"
+            launch_ms = sort_ms_all / alg["passes"]
+            launch_bytes = alg["sort"] / alg["passes"]
+        tkey = "k_onesweep"
+    else:
+        kname, launch_ms, launch_bytes, tkey = "k_map", per["map_ms"], alg["map"], "k_map"
+    ach = launch_bytes / (launch_ms / 1e3) / 1e9 if launch_ms else 0.0
+    roof = {"kernel": kname, "bound": "hbm", "achieved": round(ach, 1), "peak": hbm, "peak_kind": peak_kind,
+            "unit": "GB/s", "frac": round(ach / hbm, 4), "traffic": None, "bytes_per_launch": int(launch_bytes),
+            "ms_per_launch": round(launch_ms, 4),
+            "share_of_step": round((sort_ms_all if tkey == "k_onesweep" else per["map_ms"]) / ms, 3)}
     traffic_p = os.path.join(ROOT, "profiles", "traffic.json")
-    if roof and os.path.exists(traffic_p):
-        tr = json.load(open(traffic_p)).get(args.workload, {}).get("k_onesweep")
+    if os.path.exists(traffic_p):
+        tr = json.load(open(traffic_p)).get(args.workload, {}).get(tkey)
         if tr:
-            roof["traffic"] = tr
-    if roof is None:   # Map-only (SM) or single-digit sort: the Map kernel dominates
-        roof = {"kernel": "k_map", "bound": "hbm", "achieved": round(map_ach, 1), "peak": hbm,
-                "peak_kind": peak_kind, "unit": "GB/s", "frac": round(map_ach / hbm, 4), "traffic": None,
-                "bytes_per_launch": int(alg["map"]), "ms_per_launch": round(per["map_ms"], 4)}
+            roof["traffic"] = tr["bytes_per_launch"]
+            roof["traffic_source"] = tr["source"]
 
     nbytes_all = inp["nbytes"] * world
     value = nbytes_all / (ms_max / 1e3) / 1e9

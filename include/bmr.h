@@ -52,6 +52,7 @@ typedef enum { MR_WORDCOUNT = 1, MR_STRINGMATCH = 2, MR_KMEANS = 3, MR_INVINDEX 
 #define MR_FLAG_NO_COMBINE      0x20u /* multi-GPU: exchange raw pairs (no combiner) */
 #define MR_FLAG_PROFILE         0x40u /* record CUDA events per phase on the job stream (mr_stats *_ms) */
 #define MR_FLAG_OWN_STREAM      0x80u /* ignore cfg.stream: the job creates a private non-blocking stream */
+#define MR_FLAG_NO_MAP_COMBINE  0x100u /* WC: no in-SMEM combiner in the Map (every word is emitted as a pair) */
 
 typedef struct { uint8_t pattern[16]; } mr_sm_params;                      /* StringMatch */
 typedef struct { uint32_t k, dim; const float* centroids; } mr_km_params;  /* KMeans: host ptr, k x dim fp32, dim == 8, 1 <= k <= 1024 */
@@ -106,6 +107,10 @@ typedef struct {
    * passes (included in `pairs` / `sort_passes`; its device time is in `sort_ms`) */
   uint64_t pairs_mid;
   uint64_t sort_passes_mid;
+  /* WordCount in-SMEM combiner: partial (key, count) entries flushed by the
+   * Map CTAs (not included in `pairs`), and the words they absorbed (not emitted as pairs) */
+  uint64_t pairs_partial;
+  uint64_t words_combined;
 } mr_stats;
 
 /* State machine: CREATED -> mr_map x k (batches append) -> mr_group -> mr_reduce -> mr_fetch

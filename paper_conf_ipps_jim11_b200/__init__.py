@@ -23,7 +23,7 @@ WORDCOUNT, STRINGMATCH, KMEANS, INVINDEX = 1, 2, 3, 4
 WORKLOADS = {"wc": WORDCOUNT, "sm": STRINGMATCH, "km": KMEANS, "ii": INVINDEX}
 FLAG_NO_SMEM_IN, FLAG_NO_SMEM_OUT, FLAG_FORCE_TINY_OUT = 0x01, 0x02, 0x04
 FLAG_WEAK_HASH_DEBUG, FLAG_VALIDATE, FLAG_NO_COMBINE = 0x08, 0x10, 0x20
-FLAG_PROFILE, FLAG_OWN_STREAM = 0x40, 0x80
+FLAG_PROFILE, FLAG_OWN_STREAM, FLAG_NO_MAP_COMBINE = 0x40, 0x80, 0x100
 
 STATUS = {0: "MR_OK", 1: "MR_ERR_INVALID", 2: "MR_ERR_STATE", 3: "MR_ERR_OOM", 4: "MR_ERR_OVERFLOW",
           5: "MR_ERR_CUDA", 6: "MR_ERR_NCCL", 7: "MR_ERR_UNSUPPORTED"}
@@ -64,7 +64,8 @@ class Stats(C.Structure):
                                           "map_tiles", "input_bytes", "capacity_pairs", "kernel_launches")] + \
                [(n, C.c_double) for n in ("map_ms", "hist_ms", "sort_ms", "seg_ms", "reduce_ms")] + \
                [("pairs_hashed", C.c_uint64), ("sort_passes_keys", C.c_uint64), ("sort_keys_ms", C.c_double),
-                ("pairs_mid", C.c_uint64), ("sort_passes_mid", C.c_uint64)]
+                ("pairs_mid", C.c_uint64), ("sort_passes_mid", C.c_uint64),
+                ("pairs_partial", C.c_uint64), ("words_combined", C.c_uint64)]
 
 
 _LIB = None

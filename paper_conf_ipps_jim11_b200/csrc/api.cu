@@ -275,6 +275,11 @@ struct mr_job {
   DBuf<float> cent;
   DBuf<uint64_t> h, kref, tb;
   DBuf<uint32_t> hx;              // WC exact stream keys (u32)
+  // WC in-SMEM combiner (f-1): partial entries (key | count << 32), their sort / segments / merge
+  DBuf<uint64_t> hp, seg_startp, psum, pxcounts;
+  DBuf<uint32_t> midx, xkeys;
+  uint64_t cap_p = 0, mp = 0, nseg_p = 0, n_extra = 0;
+  const uint64_t* skeysp = nullptr;
   DBuf<uint8_t> v;
   uint64_t cap = 0;
   std::vector<Batch> batches;
@@ -285,7 +290,7 @@ struct mr_job {
   size_t host_batches = 0;
   Prof prof;
   unsigned long long launches0 = 0;
-  SortWork sw, swb, swc;
+  SortWork sw, swb, swc, swp;
   const uint64_t* skeys = nullptr;
   const uint32_t* skeysx = nullptr;   // WC exact stream, sorted (u32)
   const uint32_t* perm = nullptr;
@@ -319,6 +324,7 @@ struct mr_job {
   // WC Map output = exact stream + hashed stream (values 1, not stored); ingested WC pairs are
   // one general stream (key, kref, u64 partial count) like II
   bool split() const { return cfg.workload == MR_WORDCOUNT && !ingested; }
+  bool comb() const { return split() && !(cfg.flags & MR_FLAG_NO_MAP_COMBINE); }
   bool ingested = false;          // pairs come from mr_ingest (WC values are u64 partial counts)
   bool km_partial = false;        // KM: sums/cnts hold ingested partials; finalise owned clusters
   int vb_cur = 0;                 // value bytes of the current pairs
@@ -379,6 +385,7 @@ cudaError_t ensure_pairs(mr_job* job, uint64_t cap, uint64_t cap_b, uint64_t cap
   return cudaSuccess;
 }
 void release_pairs(mr_job* job) {
+  job->hp.release(); job->cap_p = 0;
   job->h.release(); job->hx.release(); job->kref.release(); job->v.release(); job->hb.release(); job->krefb.release();
   job->hc.release();
   job->cap = job->cap_b = job->cap_c = 0;
@@ -399,6 +406,8 @@ cudaError_t launch_batch(mr_job* job, const Batch& b) {
   a.k = job->k;
   a.out.h = job->h.p;
   a.out.hx = job->hx.p;
+  a.out.hp = job->comb() ? job->hp.p : nullptr;
+  a.out.cap_p = job->cap_p;
   a.out.kref = job->kref.p;
   a.out.v = job->v.p;
   a.out.cap = job->cap;
@@ -461,18 +470,19 @@ mr_status do_segments(mr_job* job, const uint64_t* skeys, const uint32_t* perm, 
 }
 
 // Keys-only stream: heads counted, scanned and written into a caller-provided seg_start (m + 1).
-mr_status do_segments_into(mr_job* job, const uint64_t* skeys, uint64_t m, uint64_t* seg_start, uint64_t& nseg) {
+mr_status do_segments_into(mr_job* job, const uint64_t* skeys, uint64_t m, uint64_t* seg_start, uint64_t& nseg,
+                           uint64_t kmask = ~0ULL) {
   const uint64_t tiles = (m + 4095) / 4096;
   CK(job->seg_counts.ensure(tiles + 1), "alloc seg counts");
   CK(job->tile_base.ensure(tiles + 1), "alloc tile base");
-  CK(launch_seg_count(skeys, nullptr, nullptr, m, job->seg_counts.p, job->st, 48, ~0ULL, job->stream), "seg_count");
+  CK(launch_seg_count(skeys, nullptr, nullptr, m, job->seg_counts.p, job->st, 48, kmask, job->stream), "seg_count");
   uint64_t* ss;
   uint32_t ep;
   CK(scan_ws(job, tiles, &ss, &ep), "alloc scan workspace");
   CK(launch_scan_u32to64(job->seg_counts.p, job->tile_base.p, tiles, &job->st->seg_total, ss, ep,
                          &job->st->tile_counter[1], job->stream),
      "scan tiles");
-  CK(launch_seg_write(skeys, m, job->tile_base.p, seg_start, ~0ULL, job->stream), "seg_write");
+  CK(launch_seg_write(skeys, m, job->tile_base.p, seg_start, kmask, job->stream), "seg_write");
   CK(read_state(job), "sync segments");
   nseg = m ? job->st_h.p->seg_total : 0;
   return MR_OK;
@@ -505,19 +515,26 @@ mr_status settle_map(mr_job* job) {
   if (hs->err & kErrKeyTooLong) return fail(job, MR_ERR_OVERFLOW, "an emitted key exceeds 65535 bytes");
   const uint64_t m = hs->pair_cursor, mb = job->split() ? hs->pair_cursor_b : 0;
   const uint64_t mc = job->split() ? hs->pair_cursor_c : 0;
-  if (m > job->cap || mb > job->cap_b || mc > job->cap_c) {
+  const uint64_t mp = job->comb() ? hs->pair_cursor_p : 0;
+  if (m > job->cap || mb > job->cap_b || mc > job->cap_c || mp > job->cap_p) {
+    const uint64_t ncap_p = job->comb() ? std::max(job->cap_p, mp + mp / 8 + 4096) : 0;
     const uint64_t ncap = std::max(job->cap, m + m / 8 + 4096);
     const uint64_t ncap_b = job->split() ? std::max(job->cap_b, mb + mb / 8 + 4096) : 0;
     const uint64_t ncap_c = job->split() ? std::max(job->cap_c, mc + mc / 8 + 4096) : 0;
     release_pairs(job);
     CK(ensure_pairs(job, ncap, ncap_b, ncap_c), "grow intermediate");
+    if (ncap_p) {
+      CK(job->hp.ensure(ncap_p), "grow partials");
+      job->cap_p = ncap_p;
+    }
     job->stats.capacity_pairs = job->cap + job->cap_b + job->cap_c;
     CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
     for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
     job->stats.replays += job->batches.size();
     CK(read_state(job), "replay (async)");
     if (hs->pair_cursor > job->cap ||
-        (job->split() && (hs->pair_cursor_b > job->cap_b || hs->pair_cursor_c > job->cap_c)))
+        (job->split() && (hs->pair_cursor_b > job->cap_b || hs->pair_cursor_c > job->cap_c)) ||
+        (job->comb() && hs->pair_cursor_p > job->cap_p))
       return fail(job, MR_ERR_OOM, "replay still overflows");
   }
   return MR_OK;
@@ -613,6 +630,8 @@ mr_status mr_job_reset(mr_job* job) {
   job->key_bits = (job->cfg.workload == MR_WORDCOUNT) ? 48u : 64u;
   job->key_bits_b = 48;
   job->mb = job->nseg_a = job->nseg_b = job->mc = job->nseg_c = 0;
+  job->mp = job->nseg_p = job->n_extra = 0;
+  job->skeysp = nullptr;
   job->skeysc = nullptr;
   job->segc = nullptr;
   job->skeysb = nullptr;
@@ -663,6 +682,10 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
     const uint64_t cap_b = !wc ? 0 : hint ? hint : nbytes / 48 + 4096;
     const uint64_t cap_c = !wc ? 0 : hint ? hint : nbytes / 32 + 4096;
     CK(ensure_pairs(job, initial_cap(job, nbytes, n), cap_b, cap_c), "alloc intermediate");
+    if (job->comb()) {   // combiner partials: <= 4096 per CTA per batch (grown + replayed if exceeded)
+      job->cap_p = job->cfg.max_pairs_hint ? job->cfg.max_pairs_hint : 2ULL * 4096 * job->nsm + 4096;
+      CK(job->hp.ensure(job->cap_p), "alloc partials");
+    }
     job->stats.capacity_pairs = job->cap + job->cap_b + job->cap_c;
   }
   Batch b{records, offsets, n, nbytes, job->cfg.input_base + job->next_base};
@@ -722,6 +745,8 @@ mr_status mr_group(mr_job* job) {
   job->m = m;
   job->mb = mb;
   job->mc = mc;
+  job->mp = job->comb() ? hs->pair_cursor_p : 0;
+  job->stats.pairs_partial = job->mp;
   job->stats.pairs = m + mb + mc;
   job->stats.pairs_hashed = mb;
   job->stats.pairs_mid = mc;
@@ -735,6 +760,7 @@ mr_status mr_group(mr_job* job) {
     return MR_OK;
   }
   job->nseg_b = job->nseg_c = 0;
+  job->nseg_p = job->n_extra = 0;   // (ingested jobs have no combiner partials)
   job->skeysb = nullptr;
   job->permb = nullptr;
   job->skeysc = nullptr;
@@ -755,6 +781,32 @@ mr_status mr_group(mr_job* job) {
     st = do_segments32(job, job->skeysx, m, job->seg_startx, job->nseg_a);
     if (st != MR_OK) return st;
     job->sega = job->seg_startx.p;
+    // combiner partials: sort (keys-only, 30-bit key, count above bit 32), segments, then merge
+    // into the exact segments or the extra list of partial-only keys
+    job->nseg_p = job->n_extra = 0;
+    job->skeysp = nullptr;
+    if (job->mp) {
+      const uint64_t mp = job->mp;
+      CK(run_sort(job->swp, job->hp.p, mp, &job->skeysp, nullptr, job->st, job->nsm, job->stream, nullptr,
+                  nullptr, nullptr, kExactBits),
+         "radix sort (partials)");
+      job->stats.sort_passes += job->swp.passes;
+      CK(job->seg_startp.ensure(mp + 1), "alloc partial segments");
+      st = do_segments_into(job, job->skeysp, mp, job->seg_startp.p, job->nseg_p, (1ULL << kExactBits) - 1);
+      if (st != MR_OK) return st;
+      const uint64_t np = job->nseg_p;
+      CK(job->midx.ensure(np + 1), "alloc merge");
+      CK(job->psum.ensure(np + 1), "alloc merge");
+      CK(job->xkeys.ensure(np + 1), "alloc merge");
+      CK(job->pxcounts.ensure(np + 1), "alloc merge");
+      CK(cudaMemsetAsync(&job->st->n_extra, 0, 2 * sizeof(unsigned long long), job->stream), "memset");
+      CK(launch_comb_merge(job->seg_startp.p, np, job->skeysp, job->sega, job->nseg_a, job->skeysx, job->midx.p,
+                           job->psum.p, job->xkeys.p, job->pxcounts.p, &job->st->n_extra, job->stream),
+         "combiner merge");
+      CK(read_state(job), "sync merge");
+      job->n_extra = hs->n_extra;
+      job->stats.words_combined = hs->words_comb;
+    }
     if (job->prof.on) job->prof.end(job->stream, sp, &job->stats.seg_ms);
     // mid stream: exact 48-bit keys, keys only (no fillers: plain stores)
     CK(run_sort(job->swc, job->hc.p, mc, &job->skeysc, nullptr, job->st, job->nsm, job->stream, &job->prof,
@@ -803,19 +855,22 @@ mr_status mr_group(mr_job* job) {
     }
     if (!split) { job->nseg_a = ns; }
   }
-  job->nseg = job->nseg_a + job->nseg_c + job->nseg_b;
+  job->nseg = job->nseg_a + job->n_extra + job->nseg_c + job->nseg_b;
   job->stats.n_keys = job->nseg;
   Prof::Span sp3{};
   if (job->prof.on) job->prof.begin(job->stream, sp3);
   if (job->cfg.workload == MR_WORDCOUNT || job->cfg.workload == MR_INVINDEX) {
     CK(job->key_off.ensure(job->nseg + 1), "alloc key offsets");
     if (split) {
+      const uint64_t na = job->nseg_a + job->n_extra;   // exact segments, then partial-only keys
       CK(launch_key_lengths_exact32(job->sega, job->nseg_a, job->skeysx, job->key_off.p, job->stream),
          "key lengths (exact)");
-      CK(launch_key_lengths_exact(job->segc, job->nseg_c, job->skeysc, job->key_off.p + job->nseg_a, job->stream),
+      CK(launch_key_lengths_list32(job->xkeys.p, job->n_extra, job->key_off.p + job->nseg_a, job->stream),
+         "key lengths (partial-only)");
+      CK(launch_key_lengths_exact(job->segc, job->nseg_c, job->skeysc, job->key_off.p + na, job->stream),
          "key lengths (mid)");
       CK(launch_key_lengths(job->seg_startb.p, job->nseg_b, job->permb, job->krefb.p,
-                            job->key_off.p + job->nseg_a + job->nseg_c,
+                            job->key_off.p + na + job->nseg_c,
                             job->stream),
          "key lengths (hashed)");
     } else {
@@ -853,16 +908,23 @@ mr_status mr_reduce(mr_job* job) {
       if (job->split()) {
         // every Map value is 1: a key's count is its segment length (exact stream first, then
         // the hashed stream; the output order is the sorted order of each stream)
+        const uint64_t na = job->nseg_a + job->n_extra;
         CK(launch_seg_lengths(job->sega, job->nseg_a, job->counts.p, s), "counts (exact)");
-        CK(launch_seg_lengths(job->segc, job->nseg_c, job->counts.p + job->nseg_a, s), "counts (mid)");
-        CK(launch_seg_lengths(job->seg_startb.p, job->nseg_b, job->counts.p + job->nseg_a + job->nseg_c, s),
+        CK(launch_comb_add(job->midx.p, job->psum.p, job->nseg_p, job->counts.p, s), "counts (combined)");
+        if (job->n_extra)
+          CK(cudaMemcpyAsync(job->counts.p + job->nseg_a, job->pxcounts.p, job->n_extra * 8, cudaMemcpyDeviceToDevice, s),
+             "counts (partial-only)");
+        CK(launch_seg_lengths(job->segc, job->nseg_c, job->counts.p + na, s), "counts (mid)");
+        CK(launch_seg_lengths(job->seg_startb.p, job->nseg_b, job->counts.p + na + job->nseg_c, s),
            "counts (hashed)");
-        CK(launch_key_decode(job->segc, job->nseg_c, job->skeysc, job->key_off.p + job->nseg_a, job->keys_out.p, s),
+        CK(launch_key_decode(job->segc, job->nseg_c, job->skeysc, job->key_off.p + na, job->keys_out.p, s),
            "key decode (mid)");
+        CK(launch_key_decode_list32(job->xkeys.p, job->n_extra, job->key_off.p + job->nseg_a, job->keys_out.p, s),
+           "key decode (partial-only)");
         CK(launch_key_decode32(job->sega, job->nseg_a, job->skeysx, job->key_off.p, job->keys_out.p, s),
            "key decode");
         CK(launch_key_copy(job->seg_startb.p, job->nseg_b, job->permb, job->krefb.p,
-                           job->key_off.p + job->nseg_a + job->nseg_c,
+                           job->key_off.p + na + job->nseg_c,
                            job->keys_out.p, s),
            "key copy");
       } else {
@@ -1005,7 +1067,9 @@ mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_byte
       xs.nx = m;
       xs.hc = job->hc.p;
       xs.nc = job->mc;
-      xs.n = m + job->mc + job->mb;
+      xs.hp = job->hp.p;
+      xs.np = job->comb() ? hs->pair_cursor_p : 0;
+      xs.n = m + xs.np + job->mc + job->mb;
       xs.kref = job->krefb.p;
     } else {
       xs.mode = kXPairs;
@@ -1132,6 +1196,8 @@ mr_status mr_job_destroy(mr_job* job) {
   job->xcounts.release(); job->xcursors.release(); job->xheapbase.release(); job->xcounts_h.release();
   job->src_e.release(); job->src_h.release(); job->km_list.release();
   job->cent.release(); release_pairs(job); job->tb.release();
+  job->swp.release(); job->seg_startp.release(); job->psum.release(); job->pxcounts.release();
+  job->midx.release(); job->xkeys.release();
   job->sw.release(); job->swb.release(); job->swc.release(); job->seg_startb.release(); job->seg_startx.release();
   job->scan_status.release();
   job->seg_counts.release(); job->tile_base.release(); job->seg_start.release(); job->key_off.release();

@@ -43,17 +43,25 @@ struct Rec {
 
 __device__ __forceinline__ Rec get_rec(const XSource& S, uint64_t i) {
   Rec r{};
-  if (S.mode == kXSplit) {   // WC Map output: exact, mid, then hashed stream; every value is 1
+  if (S.mode == kXSplit) {   // WC Map output: exact, combiner partials, mid, then hashed stream
     r.v = 1;
-    if (i < S.nx + S.nc) {
+    if (i < S.nx + S.np + S.nc) {
       if (i < S.nx && S.hx[i] == 0xFFFFFFFFu) { r.dest = ~0u; return r; }   // flush filler (exact stream)
-      const uint64_t key = i < S.nx ? static_cast<uint64_t>(S.hx[i]) : S.hc[i - S.nx];
+      uint64_t key;
+      if (i < S.nx) {
+        key = S.hx[i];
+      } else if (i < S.nx + S.np) {   // combiner partial: exact key, value = its count
+        key = S.hp[i - S.nx] & 0x3FFFFFFFULL;
+        r.v = S.hp[i - S.nx] >> 32;
+      } else {
+        key = S.hc[i - S.nx - S.np];
+      }
       r.kin = exact_key_bytes(key, r.klen);
       r.dest = dest_of_bytes(reinterpret_cast<const uint8_t*>(&r.kin), r.klen, S.nranks);
       r.heap = (r.klen + 7u) & ~7u;
       return r;
     }
-    const uint64_t kr = S.kref[i - S.nx - S.nc];
+    const uint64_t kr = S.kref[i - S.nx - S.np - S.nc];
     r.kp = reinterpret_cast<const uint8_t*>(kr >> 16);
     r.klen = static_cast<uint32_t>(kr & 0xFFFF);
   } else if (S.mode == kXPairs) {

@@ -31,6 +31,9 @@ struct DevState {
   unsigned long long pads;         // sentinel filler pairs written by the flushes (sort last, excluded)
   unsigned long long pair_cursor_b;  // WC hashed stream: demand in pairs
   unsigned long long pair_cursor_c;  // WC mid stream: demand in pairs
+  unsigned long long pair_cursor_p;  // WC combiner partials: demand in entries
+  unsigned long long n_extra;        // WC: partial-only keys found by the merge (mr_group)
+  unsigned long long words_comb;     // WC: words absorbed by the combiners (sum of partial counts)
 };
 constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u;
 
@@ -40,6 +43,8 @@ constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u;
 struct PairBufs {
   uint64_t* h = nullptr;     // 64-bit sort key (inline key / hash / SM offset / KM id)
   uint32_t* hx = nullptr;    // WC exact stream: 30-bit exact keys (u32; 0xFFFFFFFF = filler)
+  uint64_t* hp = nullptr;    // WC combiner partials (exact key | count << 32); nullptr = no combiner
+  uint64_t cap_p = 0;
   uint64_t* kref = nullptr;  // (device address of key bytes << 16) | key length
   uint8_t* v = nullptr;      // value bytes (vbytes per pair)
   uint64_t cap = 0;          // capacity in pairs
@@ -74,7 +79,8 @@ int vbytes_of(int workload);                 // value bytes per pair (WC Map out
 bool has_kref(int workload);
 uint64_t map_tiles(const MapArgs& a);        // number of tiles of a batch
 uint32_t map_prefetch();
-uint32_t map_wait_hint();                     // L2 prefetch distance of the Map producers (BMR_MAP_PF)
+uint32_t map_wait_hint();
+uint32_t map_dyn_windows(int workload);                     // L2 prefetch distance of the Map producers (BMR_MAP_PF)
 cudaError_t launch_map(const MapArgs& a, int num_sms, cudaStream_t s);
 
 // ---- group-by-key (hash radix sort + segment boundaries) ----
@@ -155,6 +161,16 @@ cudaError_t launch_key_lengths_exact32(const uint64_t* seg_start, uint64_t nseg,
 cudaError_t launch_key_decode32(const uint64_t* seg_start, uint64_t nseg, const uint32_t* skeys,
                                 const uint64_t* key_off, uint8_t* keys, cudaStream_t s);
 cudaError_t launch_gather_u64(const uint32_t* perm, const uint8_t* v, uint64_t m, uint64_t* out, cudaStream_t s);
+// WC combiner partials (f-1): merge into the exact stream's segments (midx / psum) or the extra
+// list of partial-only keys (xkeys / xcounts, *nextra of them)
+cudaError_t launch_comb_merge(const uint64_t* segp, uint64_t nsegp, const uint64_t* skp, const uint64_t* sega,
+                              uint64_t nsega, const uint32_t* skx, uint32_t* midx, uint64_t* psum, uint32_t* xkeys,
+                              uint64_t* xcounts, unsigned long long* nextra, cudaStream_t s);
+cudaError_t launch_comb_add(const uint32_t* midx, const uint64_t* psum, uint64_t nsegp, uint64_t* counts,
+                            cudaStream_t s);
+cudaError_t launch_key_lengths_list32(const uint32_t* keys, uint64_t n, uint64_t* lens, cudaStream_t s);
+cudaError_t launch_key_decode_list32(const uint32_t* keys, uint64_t n, const uint64_t* key_off, uint8_t* out,
+                                     cudaStream_t s);
 cudaError_t launch_offsets_scaled(const uint64_t* seg_start, uint64_t nseg, uint64_t scale, uint64_t* out,
                                   cudaStream_t s);
 cudaError_t launch_iota_scaled(uint64_t n, uint64_t scale, uint64_t* out, cudaStream_t s);
@@ -175,6 +191,8 @@ struct XSource {
   uint64_t nx = 0;                             //   then the mid-stream keys (nc), then the hashed
   const uint64_t* hc = nullptr;                //   stream (kref)
   uint64_t nc = 0;
+  const uint64_t* hp = nullptr;                // kXSplit: combiner partials (key | count << 32),
+  uint64_t np = 0;                             //   after the exact stream
   const uint8_t* v = nullptr;
   int vbytes = 8;
   const uint8_t* keys = nullptr;               // kXSegs

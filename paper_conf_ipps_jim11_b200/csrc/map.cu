@@ -46,8 +46,6 @@ constexpr int kHalo = 256;       // bytes staged after the tile (words / matches
 constexpr int kWin = 512;        // bytes per warp window = 32 lanes x 16 B
 constexpr int kNWin = kT / kWin;
 constexpr int kStageBytes = 16768;             // >= kLead + kT + kHalo + 32, multiple of 128
-constexpr int kOffCap = 1024;                  // record offsets staged per tile
-constexpr int kOffBytes = 8320;                // (kOffCap + 2) * 8 rounded up
 constexpr int kBitWords = kStageBytes / 32 + 4;
 constexpr int kBitBytes = 2176;                // >= kBitWords * 4, multiple of 128
 constexpr int kNOut = 4;         // output buffers in the flush ring (generation g uses buffer g % kNOut)
@@ -56,8 +54,12 @@ constexpr int kNOut = 4;         // output buffers in the flush ring (generation
 // and 4 x 20 KB output buffers.
 template <int W>
 struct Cfg {
+  // StringMatch (read-bound, almost no output): 6 stages (8 stages with 512 staged offsets each
+  // measured slower on C2: 2.38 against 2.07 ms)
   static constexpr int kStages = (W == kSM) ? 6 : 4;
-  static constexpr int kOutHalf = (W == kSM) ? 4096 : 20480;   // bytes per output buffer
+  static constexpr int kOffCap = 1024;   // record offsets staged per tile (more: read from global)
+  static constexpr int kOffBytes = ((kOffCap + 2) * 8 + 127) / 128 * 128;
+  static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? 12288 : 20480;   // bytes per output buffer
   // the producer builds the bitmap of tile it - kLag right after issuing tile it: kLag stages of
   // TMA traffic stay in flight per SM while one stage is being consumed
   static constexpr int kLag = kStages - 2;
@@ -67,7 +69,16 @@ struct Cfg {
   // words, most rounds would carry at least one).  A window holds at most 512 / 6 + 1 starts
   // of words longer than kWcExact bytes.
   static constexpr int kHashQ = (W == kWC) ? 96 : 0;
+  // WC: per-warp queue of the window's exact keys that missed the combiner (u32), copied into
+  // the output buffer after the one reservation; <= 257 word starts per window
+  static constexpr int kXQ = (W == kWC) ? 264 : 0;
+  // WC: in-SMEM combiner (MapCG-style): kCombSlots u64 entries
+  // (u32 exact keys + u32 counts), direct-mapped, a slot keeps the first key that claims it
+  static constexpr int kCombSlots = (W == kWC) ? 4096 : 0;
 };
+constexpr int kCombBits = 12;
+static_assert(Cfg<kWC>::kCombSlots == (1 << kCombBits), "combiner slots");
+constexpr uint32_t kCombEmpty32 = 0xFFFFFFFFu;   // exact keys are < 2^30
 // WC words of <= kWcExact bytes get an exact 30-bit key (common.cuh exact_key30) and travel in
 // the exact stream (4-B u32 entries: the key is the whole record).  Longer words are queued; in the
 // queue pass words of <= kMidMax bytes get an exact 48-bit key (mid stream, key only), longer
@@ -75,6 +86,7 @@ struct Cfg {
 // kref 0 marks a mid-stream key) and the flush warp routes them.
 constexpr uint32_t kWcExact = kExactMax;
 static_assert(kWin / (kWcExact + 1) + 1 <= Cfg<kWC>::kHashQ, "hash queue too small");
+static_assert(kWin / 2 + 1 <= Cfg<kWC>::kXQ, "exact-key queue too small");
 constexpr int kKmPts = kT / 32;                // 512 points per KM tile
 
 static_assert(kLead + kT + kHalo + 32 <= kStageBytes, "stage too small");
@@ -100,6 +112,7 @@ struct OutCtl {
   unsigned long long fbase[kNOut];   // global base reserved for the sealed buffer (one atomic per flush)
   unsigned long long nflush, npads;  // per-CTA statistics, added to DevState once at the end
   unsigned int nsealed, is_final;  // sealed generations so far (full count); final flush flag
+  unsigned int win_next;         // text: next window (tile * kNWin + window) to hand to a map warp
   uint64_t req[kNOut];           // mbarrier: buffer sealed -> flush warp
   uint64_t done[kNOut];          // mbarrier: buffer flushed -> free
 };
@@ -114,10 +127,12 @@ struct Layout {
   static constexpr int ready = empty + kStages * 8;               // kStages x 8 (text: bitmap built)
   static constexpr int bytes = 2048;                              // kStages x kStageBytes
   static constexpr int offs = bytes + kStages * kStageBytes;      // kStages x kOffBytes
-  static constexpr int bits = offs + kStages * kOffBytes;         // kStages x kBitBytes
+  static constexpr int bits = offs + kStages * Cfg<W>::kOffBytes; // kStages x kBitBytes
   static constexpr int out = bits + kStages * kBitBytes;          // kNOut x Cfg<W>::kOutHalf
   static constexpr int hq = out + kNOut * Cfg<W>::kOutHalf;       // kNMap x kHashQ x 8 (WC)
-  static constexpr int cent = hq + kNMap * Cfg<W>::kHashQ * 8;    // KM centroids
+  static constexpr int xq = hq + kNMap * Cfg<W>::kHashQ * 8;      // kNMap x kXQ x 4 (WC)
+  static constexpr int comb = xq + kNMap * Cfg<W>::kXQ * 4;       // kCombSlots x 8 (WC)
+  static constexpr int cent = comb + Cfg<W>::kCombSlots * 8;      // KM centroids
   static_assert(ready + kStages * 8 <= bytes, "header region overflow");
   static_assert(sizeof(OutCtl) <= hdr, "OutCtl overlaps the stage headers");
 };
@@ -160,6 +175,9 @@ struct Params {
   uint64_t* ohc;           // WC mid stream: keys, capacity
   uint64_t cap_c;
   uint32_t* ohx;           // WC exact stream: u32 keys (capacity cap_pairs)
+  uint64_t* ohp;           // WC combiner partials: (exact key | count << 32), capacity cap_p
+  uint64_t cap_p;
+  uint32_t comb;           // WC: in-SMEM combiner on
   uint32_t out_cap;        // per-half capacity actually used (FORCE_TINY_OUT shrinks it)
   uint32_t flags;
   DevState* st;
@@ -168,14 +186,25 @@ struct Params {
   uint64_t hash_seed;
   uint32_t key_bits;       // sort-key width (48 or 64)
   uint32_t pf;             // L2 prefetch distance in producer tiles (0: off)
-  uint32_t wait_hint;      // idle mbarrier waits: 1 = try_wait with a suspend-time hint, 0 = plain try_wait
+  uint32_t wait_hint;      // idle mbarrier waits: 0 plain try_wait, 1 suspend-time hint, 2 helpers sleep-poll
+  uint32_t dyn;            // text: windows handed out dynamically (1) or in static warp order (0)
 };
 
 // Idle wait of a role warp on an mbarrier phase (map warps on a staged tile, producers on a free
 // stage, the flush warp on a sealed buffer).
 __device__ __forceinline__ void map_wait(const Params& P, uint64_t* bar, uint32_t parity, uint32_t ns) {
-  if (P.wait_hint) mbar_wait_idle(bar, parity, ns);
+  if (P.wait_hint == 1) mbar_wait_idle(bar, parity, ns);
   else mbar_wait(bar, parity);
+}
+// Waits of the helper warps (producers on a free stage, the flush warp on a sealed buffer): with
+// wait_hint == 2 they poll with __nanosleep between attempts, leaving issue slots to the map
+// warps (the Map of the text workloads is issue-bound).
+__device__ __forceinline__ void helper_wait(const Params& P, uint64_t* bar, uint32_t parity, uint32_t sleep_ns) {
+  if (P.wait_hint == 2) {
+    while (!mbar_try_wait(bar, parity)) __nanosleep(sleep_ns);
+  } else {
+    map_wait(P, bar, parity, 20000);
+  }
 }
 
 constexpr uint32_t kFull = 0xffffffffu;
@@ -487,7 +516,7 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   const uint32_t lane = threadIdx.x & 31;
   for (uint32_t f = 0;; ++f) {
     const uint32_t h = f % kNOut;
-    map_wait(P, &oc->req[h], (f / kNOut) & 1u, 20000);
+    helper_wait(P, &oc->req[h], (f / kNOut) & 1u, 64);
     const uint32_t cnt0 = *reinterpret_cast<volatile unsigned int*>(&oc->fcount[h]);
     const bool fin = *reinterpret_cast<volatile unsigned int*>(&oc->is_final) &&
                      *reinterpret_cast<volatile unsigned int*>(&oc->final_seq) == f;
@@ -612,7 +641,8 @@ __device__ void finish_stage(const Params& P, uint8_t* smem, uint32_t it) {
   mbar_wait(&full[s], ph);
   const StageHdr* hd = reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
   uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout<W>::bits + s * kBitBytes);
-  const uint64_t* soff = reinterpret_cast<const uint64_t*>(smem + Layout<W>::offs + s * kOffBytes + hd->off_shift);
+  const uint64_t* soff =
+      reinterpret_cast<const uint64_t*>(smem + Layout<W>::offs + s * Cfg<W>::kOffBytes + hd->off_shift);
   const uint64_t ra = hd->ra, cnt = hd->rb - hd->ra;
   const long long sbase = hd->sbase;
   const bool staged = hd->off_staged != 0;
@@ -652,11 +682,11 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
       const uint64_t t = blockIdx.x + static_cast<uint64_t>(it) * G;
       const uint64_t ra = __shfl_sync(kFull, my_ra, j), rb = __shfl_sync(kFull, my_rb, j);
       const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
-      map_wait(P, &empty[s], ph ^ 1u, 20000);
+      helper_wait(P, &empty[s], ph ^ 1u, 128);
       StageHdr* hd = reinterpret_cast<StageHdr*>(smem + Layout<W>::hdr + s * 128);
       uint8_t* sb = smem + Layout<W>::bytes + s * kStageBytes;
       uint32_t b_off = 0, b_len = 0, o_off = 0, o_len = 0;
-      uint8_t* so = smem + Layout<W>::offs + s * kOffBytes;
+      uint8_t* so = smem + Layout<W>::offs + s * Cfg<W>::kOffBytes;
       if constexpr (W == kKM) {
         const uint64_t p_lo = t * kKmPts, p_hi = min(P.n, p_lo + kKmPts);
         const uint8_t* g = P.rec + p_lo * 32;
@@ -687,7 +717,7 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
         for (uint32_t i = lane; i < kBitBytes / 16; i += 32) reinterpret_cast<uint4*>(bm)[i] = make_uint4(0, 0, 0, 0);
         // offsets slice offsets[ra..rb) (record starts in the staged window)
         const uint64_t cnt = rb - ra;
-        const bool staged = cnt <= kOffCap;
+        const bool staged = cnt <= static_cast<uint64_t>(Cfg<W>::kOffCap);
         uint32_t shift = 0;
         const uint8_t* og = reinterpret_cast<const uint8_t*>(P.off + ra);
         if (staged && cnt) {
@@ -760,6 +790,18 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
 }
 
 // ---------------------------------------------------------------- map warps
+// Combiner probe (f-1): adds one occurrence of exact key `key` to its slot if the slot holds the
+// key or is free (claimed by a 32-bit CAS); false = the slot belongs to another key (emit
+// normally).  Keys and counts are separate u32 arrays: 32-bit shared atomics are native (a
+// 64-bit shared atomicAdd is a CAS spin loop, which serialises on the Zipf head's slots).
+__device__ __forceinline__ bool comb_add(uint32_t* ckey, uint32_t key) {
+  const uint32_t slot = (key * 0x9E3779B1u) >> (32 - kCombBits);
+  uint32_t v = *reinterpret_cast<volatile uint32_t*>(ckey + slot);
+  if (v == kCombEmpty32) v = atomicCAS(ckey + slot, kCombEmpty32, key);
+  if (v != key && v != kCombEmpty32) return false;
+  atomicAdd(ckey + Cfg<kWC>::kCombSlots + slot, 1u);   // count array follows the key array
+  return true;
+}
 // WordCount emission of one warp window.  Each start is classified BEFORE the reservation: a
 // word is exact iff it ends within kWcExact bytes (nb bit q: a word cannot continue at q, so the
 // word at j ends at the first nb bit above j).  Only a lane's highest start can lack a visible
@@ -782,18 +824,14 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
   for (uint32_t d = 1; d <= kWcExact; ++d) near |= nb >> d;
   uint32_t longm = emit_mask & ~near & ~slow_bit;
   if (slow_bit && len_slow > kWcExact) longm |= slow_bit;
-  const uint32_t nl = __popc(longm);
-  const uint32_t tot = __reduce_add_sync(kFull, (__popc(emit_mask) - nl) | (nl << 16));
-  if (tot == 0) return;
-  const uint32_t packed = (tot & 0xFFFFu) | ((tot >> 16) << kCbShift);
-  const Slot slot = reserve<kWC>(P, oc, outh, packed, P.out_cap);
-  uint8_t* half = outh + slot.half * Cfg<kWC>::kOutHalf;
-  uint32_t* sh = reinterpret_cast<uint32_t*>(half);
-  ulonglong2* top = reinterpret_cast<ulonglong2*>(half + Cfg<kWC>::kOutHalf);   // hashed entry i: top[-1 - i]
+  (void)longm;
+  if (__all_sync(kFull, emit_mask == 0)) return;
   uint64_t* hq = reinterpret_cast<uint64_t*>(outh + (Layout<kWC>::hq - Layout<kWC>::out)) +
                  (threadIdx.x >> 5) * Cfg<kWC>::kHashQ;
-  const uint32_t kb0 = cur_cb(slot.base);
-  uint32_t ka = cur_ca(slot.base), nq = 0;
+  uint32_t* xq = reinterpret_cast<uint32_t*>(outh + (Layout<kWC>::xq - Layout<kWC>::out)) +
+                 (threadIdx.x >> 5) * Cfg<kWC>::kXQ;
+  uint32_t* ctab = reinterpret_cast<uint32_t*>(outh + (Layout<kWC>::comb - Layout<kWC>::out));
+  uint32_t nx = 0, nq = 0;
   uint32_t m_left = emit_mask;
   while (__any_sync(kFull, m_left != 0)) {
     const bool act = m_left != 0;
@@ -804,18 +842,31 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
       const uint32_t rest = nb >> (j + 1);
       len = rest ? static_cast<uint32_t>(__ffs(rest)) : len_slow;
     }
-    const bool ex = act && len <= kWcExact;
-    const uint32_t ma = __ballot_sync(kFull, ex), mb = __ballot_sync(kFull, act && !ex);
+    bool ex = act && len <= kWcExact;
+    uint32_t key = 0;
     if (ex) {
-      const uint64_t b = window8(x, j);     // an exact word lies inside the 32 loaded bytes
-      sh[ka + __popc(ma & lanemask_lt())] = exact_key30(b, len);
-    } else if (act) {
+      key = exact_key30(window8(x, j), len);   // an exact word lies inside the 32 loaded bytes
+      if (P.comb && comb_add(ctab, key)) ex = false;   // absorbed by the combiner
+    }
+    const uint32_t ma = __ballot_sync(kFull, ex), mb = __ballot_sync(kFull, act && len > kWcExact);
+    if (ex) {
+      xq[nx + __popc(ma & lanemask_lt())] = key;
+    } else if (act && len > kWcExact) {
       if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
       hq[nq + __popc(mb & lanemask_lt())] = static_cast<uint64_t>(p0 + j - tv.sbase) | (static_cast<uint64_t>(len) << 24);
     }
-    ka += __popc(ma);
+    nx += __popc(ma);
     nq += __popc(mb);
   }
+  if (nx + nq == 0) return;
+  const uint32_t packed = nx | (nq << kCbShift);
+  const Slot slot = reserve<kWC>(P, oc, outh, packed, P.out_cap);
+  uint8_t* half = outh + slot.half * Cfg<kWC>::kOutHalf;
+  uint32_t* sh = reinterpret_cast<uint32_t*>(half);
+  ulonglong2* top = reinterpret_cast<ulonglong2*>(half + Cfg<kWC>::kOutHalf);   // hashed entry i: top[-1 - i]
+  const uint32_t kb0 = cur_cb(slot.base), ka = cur_ca(slot.base);
+  __syncwarp();
+  for (uint32_t i = lane; i < nx; i += 32) sh[ka + i] = xq[i];
   __syncwarp();
   for (uint32_t q = lane; q < nq; q += 32) {           // lane-parallel keys of the long words
     const uint64_t e = hq[q];
@@ -892,12 +943,20 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
       }
     }
   } else if constexpr (W == kII) {
+    // markers of this lane's chunk, then the closing quote of each marker by a warp-cooperative
+    // search: every lane publishes its 16-bit "stop" mask (a '"' or a record start) and a marker
+    // finds the first stop at or after its URL start with two shuffles (the URL ends at the first
+    // '"' unless the record ends first, C-3 #9); only URLs leaving the 512-B window scan onwards.
+    uint32_t mk = 0, st16 = 0;
     if (live) {
-      uint32_t cand = 0;
+      uint32_t cand = 0, qm = 0;
 #pragma unroll
-      for (int i = 0; i < 4; ++i) cand |= eq_mask4(x[i], 0x3C3C3C3Cu) << (4 * i);  // '<'
+      for (int i = 0; i < 4; ++i) {
+        cand |= eq_mask4(x[i], 0x3C3C3C3Cu) << (4 * i);  // '<'
+        qm |= eq_mask4(x[i], 0x22222222u) << (4 * i);    // '"'
+      }
       cand &= vm & 0xFFFFu;
-      int nm = 0;
+      st16 = ((qm & vm) | R) & 0xFFFFu;
       while (cand) {
         const uint32_t j = __ffs(cand) - 1;
         cand &= cand - 1;
@@ -907,12 +966,40 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
         window16(x, j, w);
         // "<a href=\"" little-endian: 3C 61 20 68 | 72 65 66 3D | 22
         if (w[0] != 0x6820613Cu || w[1] != 0x3D666572u || (w[2] & 0xFFu) != 0x22u) continue;
-        const long long q0 = p0 + j + 9;
-        const long long q = find_quote(P, tv, q0, p0 + j);
-        if (q > q0 && nm < 2) {
-          aux[nm++] = static_cast<uint32_t>(q - q0);
-          emit_mask |= 1u << j;
-        }
+        mk |= 1u << j;
+      }
+    }
+    const uint32_t lanes_st = __ballot_sync(kFull, st16 != 0);
+    const uint32_t r16 = R & 0xFFFFu;
+    const long long wp = p0 - static_cast<long long>(lane) * 16;   // window start
+    int nm = 0;
+    for (int mi = 0; mi < 2; ++mi) {          // a 9-byte marker: at most two start in 16 bytes
+      if (!__any_sync(kFull, mk != 0)) break;
+      const bool has = mk != 0;
+      const uint32_t j = has ? static_cast<uint32_t>(__ffs(mk) - 1) : 0u;
+      if (has) mk &= mk - 1;
+      const uint32_t a = lane * 16 + j + 9;   // window offset of the URL start
+      const uint32_t T = min(a >> 4, 31u);
+      const uint32_t sT = __shfl_sync(kFull, st16, T), rT = __shfl_sync(kFull, r16, T);
+      const uint32_t cT = a < static_cast<uint32_t>(kWin) ? (sT >> (a & 15u)) << (a & 15u) : 0u;
+      const uint32_t later = T < 31 ? (lanes_st & ~((2u << T) - 1u)) : 0u;
+      const uint32_t F = later ? static_cast<uint32_t>(__ffs(later) - 1) : 31u;
+      const uint32_t sF = __shfl_sync(kFull, st16, F), rF = __shfl_sync(kFull, r16, F);
+      if (!has) continue;
+      const long long q0 = p0 + j + 9;
+      long long q;
+      if (cT) {
+        const uint32_t b = __ffs(cT) - 1;
+        q = ((rT >> b) & 1u) ? -1 : wp + T * 16 + b;     // record ends first -> unclosed
+      } else if (later && a < static_cast<uint32_t>(kWin)) {
+        const uint32_t b = __ffs(sF) - 1;
+        q = ((rF >> b) & 1u) ? -1 : wp + F * 16 + b;
+      } else {                                           // no stop in the window: scan onwards
+        q = find_quote(P, tv, max(q0, wp + kWin), p0 + j);
+      }
+      if (q > q0 && nm < 2) {
+        aux[nm++] = static_cast<uint32_t>(q - q0);
+        emit_mask |= 1u << j;
       }
     }
   }
@@ -966,7 +1053,27 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
   uint8_t* outh = smem + Layout<W>::out;
   const float* cent = reinterpret_cast<const float*>(smem + Layout<W>::cent);
+  // Text: windows are handed out dynamically (one shared atomic per 512-B window, in tile order),
+  // so a warp that drew cheap windows takes the next one instead of idling until the slowest
+  // warp of the tile is done; a stage is released after all kNWin of its windows (empty[s]
+  // counts windows).  KM: one point per map lane, kNMap arrivals per stage.
+  // (P.dyn == 0: static order, warp w takes windows w and w + kNMap of every tile)
+  static_assert(kNWin == 2 * kNMap, "static window order assumes two windows per warp and tile");
+  uint32_t kseq = 0;
   for (uint32_t it = 0;; ++it) {
+    uint32_t w = 0;
+    if constexpr (W != kKM) {
+      uint32_t g = 0;
+      if (P.dyn) {
+        if (lane == 0) g = atomicAdd(&oc->win_next, 1u);
+        g = __shfl_sync(kFull, g, 0);
+      } else {
+        g = (kseq >> 1) * kNWin + warp + (kseq & 1u) * kNMap;
+        ++kseq;
+      }
+      it = g / kNWin;
+      w = g % kNWin;
+    }
     const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
     if constexpr (W == kKM) mbar_wait(&full[s], ph);
     else map_wait(P, reinterpret_cast<uint64_t*>(smem + Layout<W>::ready) + s, ph, kReadyWaitNs);
@@ -1039,9 +1146,8 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
     } else {
       const uint32_t* bm = reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * kBitBytes);
       TileView tv{sb, bm, hd.sbase, hd.stg_hi};
-      for (uint32_t w = warp; w < kNWin; w += kNMap) {
-        const long long wp = hd.chunk0 + static_cast<long long>(w) * kWin;
-        if (wp >= hd.hi) break;                       // warp-uniform
+      const long long wp = hd.chunk0 + static_cast<long long>(w) * kWin;
+      if (wp < hd.hi) {                               // warp-uniform
         const long long p0 = wp + lane * 16;
         const bool live = (p0 + 16 > 0) && (p0 < static_cast<long long>(P.nbytes));
         emit_text_chunk<W>(P, oc, outh, tv, p0, p0 - hd.sbase, live);
@@ -1052,6 +1158,22 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   }
   // final flush of the partially filled half (all map warps done, nothing pending)
   named_bar_sync(2, kNMap * 32);
+  if constexpr (W == kWC) {
+    if (P.comb) {   // combiner partials -> global (one atomic per warp step; demand counted past capacity)
+      const uint32_t* ctab = reinterpret_cast<const uint32_t*>(smem + Layout<W>::comb);
+      for (uint32_t i0 = warp * 32; i0 < static_cast<uint32_t>(Cfg<W>::kCombSlots); i0 += kNMap * 32) {
+        const uint32_t k = ctab[i0 + lane], c = ctab[Cfg<W>::kCombSlots + i0 + lane];
+        const uint64_t v = static_cast<uint64_t>(k) | (static_cast<uint64_t>(c) << 32);
+        const uint32_t mv = __ballot_sync(kFull, k != kCombEmpty32);
+        if (!mv) continue;
+        unsigned long long gb = 0;
+        if (lane == 0) gb = atomicAdd(&P.st->pair_cursor_p, static_cast<unsigned long long>(__popc(mv)));
+        gb = __shfl_sync(kFull, gb, 0);
+        const uint64_t o = gb + __popc(mv & lanemask_lt());
+        if (k != kCombEmpty32 && o < P.cap_p) P.ohp[o] = v;
+      }
+    }
+  }
   if (threadIdx.x == 0) {
     const uint32_t cur = *reinterpret_cast<volatile unsigned int*>(&oc->cur);
     seal<W>(P, oc, cur_gen(cur), cur_gen(cur) % kNOut, cur & kCntBits, true);
@@ -1071,12 +1193,24 @@ __global__ void __launch_bounds__(kThreads, 1) k_map(Params P) {
     oc->npads = 0;
     oc->nsealed = 0;
     oc->is_final = 0;
+    oc->win_next = 0;
     for (int b = 0; b < kNOut; ++b) { mbar_init(&oc->req[b], 1); mbar_init(&oc->done[b], kNFlush); }
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
     uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
     uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout<W>::ready);
-    for (int s = 0; s < kStages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], kNMap); mbar_init(&ready[s], 1); }
+    for (int s = 0; s < kStages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], W == kKM ? kNMap : kNWin);   // text: one arrival per window
+      mbar_init(&ready[s], 1);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if constexpr (W == kWC) {
+    uint32_t* ctab = reinterpret_cast<uint32_t*>(smem + Layout<W>::comb);   // keys, then counts
+    for (uint32_t i = threadIdx.x; i < static_cast<uint32_t>(Cfg<W>::kCombSlots); i += blockDim.x) {
+      ctab[i] = kCombEmpty32;
+      ctab[Cfg<W>::kCombSlots + i] = 0;
+    }
   }
   if constexpr (W == kKM) {
     float* cent = reinterpret_cast<float*>(smem + Layout<W>::cent);
@@ -1150,8 +1284,12 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.ohc = a.out.hc;
   P.cap_c = a.out.cap_c;
   P.ohx = a.out.hx;
+  P.ohp = a.out.hp;
+  P.cap_p = a.out.cap_p;
+  P.comb = (W == kWC && a.out.hp != nullptr) ? 1u : 0u;
   P.pf = map_prefetch();
   P.wait_hint = map_wait_hint();
+  P.dyn = map_dyn_windows(W);
   if (P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>((P.ntiles + 255) / 256);
@@ -1180,13 +1318,24 @@ uint32_t map_prefetch() {
   return v;
 }
 
-// idle-wait flavour of the Map role warps (BMR_MAP_WAIT: 1 = suspend-time hint, default 0 = plain)
+// idle-wait flavour of the Map role warps (BMR_MAP_WAIT: 0 = plain try_wait, 1 = suspend-time
+// hint, 2 = plain for the map warps and __nanosleep polling for the producers / flush warp)
 uint32_t map_wait_hint() {
   static uint32_t v = [] {
     const char* e = getenv("BMR_MAP_WAIT");
     return e ? static_cast<uint32_t>(atoi(e)) : 0u;
   }();
   return v;
+}
+
+// text window scheduling (BMR_MAP_DYN: 0 static, 1 dynamic; default: dynamic except StringMatch,
+// whose windows are uniformly cheap -- measured on C2/C4/C5 in round 1)
+uint32_t map_dyn_windows(int w) {
+  static int v = [] {
+    const char* e = getenv("BMR_MAP_DYN");
+    return e ? atoi(e) : -1;
+  }();
+  return v >= 0 ? static_cast<uint32_t>(v) : (w == kSM ? 0u : 1u);
 }
 
 int vbytes_of(int w) { return w == kKM ? 32 : w == kII ? 8 : 0; }

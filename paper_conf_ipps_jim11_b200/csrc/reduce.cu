@@ -382,6 +382,55 @@ __global__ void k_key_decode(const uint64_t* seg, uint64_t nseg, const K* sk, co
   uint8_t* dst = keys + key_off[s];
   for (uint32_t i = 0; i < len; ++i) dst[i] = static_cast<uint8_t>(b >> (8 * i));
 }
+// WC combiner partials (f-1), after their own sort + segments: the summed count of every partial
+// key, then a binary search of the key among the exact stream's segment keys (ascending).  Found:
+// midx = that segment (its count is augmented in mr_reduce); not found: the key is appended to
+// the extra list (keys that only the combiner saw).
+__global__ void k_comb_merge(const uint64_t* __restrict__ segp, uint64_t nsegp, const uint64_t* __restrict__ skp,
+                             const uint64_t* __restrict__ sega, uint64_t nsega, const uint32_t* __restrict__ skx,
+                             uint32_t* midx, uint64_t* psum, uint32_t* xkeys, uint64_t* xcounts,
+                             unsigned long long* nextra) {   // nextra[1]: words absorbed (sum of counts)
+  const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (s >= nsegp) return;
+  const uint64_t a = segp[s], b = segp[s + 1];
+  const uint32_t key = static_cast<uint32_t>(skp[a] & 0x3FFFFFFFULL);
+  uint64_t sum = 0;
+  for (uint64_t i = a; i < b; ++i) sum += skp[i] >> 32;
+  atomicAdd(nextra + 1, static_cast<unsigned long long>(sum));
+  uint64_t lo = 0, hi = nsega;   // first exact segment with key >= `key`
+  while (lo < hi) {
+    const uint64_t mid = (lo + hi) >> 1;
+    if (skx[sega[mid]] < key) lo = mid + 1; else hi = mid;
+  }
+  if (lo < nsega && skx[sega[lo]] == key) {
+    midx[s] = static_cast<uint32_t>(lo);
+    psum[s] = sum;
+  } else {
+    midx[s] = 0xFFFFFFFFu;
+    const unsigned long long e = atomicAdd(nextra, 1ULL);
+    xkeys[e] = key;
+    xcounts[e] = sum;
+  }
+}
+__global__ void k_comb_add(const uint32_t* midx, const uint64_t* psum, uint64_t nsegp, uint64_t* counts) {
+  const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (s < nsegp && midx[s] != 0xFFFFFFFFu) counts[midx[s]] += psum[s];   // distinct keys: distinct targets
+}
+__global__ void k_key_lengths_list32(const uint32_t* keys, uint64_t n, uint64_t* lens) {
+  const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (s >= n) return;
+  uint32_t len;
+  exact_key_bytes(keys[s], len);
+  lens[s] = len;
+}
+__global__ void k_key_decode_list32(const uint32_t* keys, uint64_t n, const uint64_t* key_off, uint8_t* out) {
+  const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (s >= n) return;
+  uint32_t len;
+  const uint64_t b = exact_key_bytes(keys[s], len);
+  uint8_t* dst = out + key_off[s];
+  for (uint32_t i = 0; i < len; ++i) dst[i] = static_cast<uint8_t>(b >> (8 * i));
+}
 __global__ void k_gather_u64(const uint32_t* perm, const uint64_t* v, uint64_t m, uint64_t* out) {
   const uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
   if (i < m) out[i] = v[perm[i]];
@@ -527,6 +576,35 @@ cudaError_t launch_key_decode32(const uint64_t* seg_start, uint64_t nseg, const 
                                 const uint64_t* key_off, uint8_t* keys, cudaStream_t s) {
   if (nseg == 0) return cudaSuccess;
   k_key_decode<<<blocks_for(nseg, 256), 256, 0, s>>>(seg_start, nseg, skeys, key_off, keys);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_comb_merge(const uint64_t* segp, uint64_t nsegp, const uint64_t* skp, const uint64_t* sega,
+                              uint64_t nsega, const uint32_t* skx, uint32_t* midx, uint64_t* psum, uint32_t* xkeys,
+                              uint64_t* xcounts, unsigned long long* nextra, cudaStream_t s) {
+  if (nsegp == 0) return cudaSuccess;
+  k_comb_merge<<<blocks_for(nsegp, 256), 256, 0, s>>>(segp, nsegp, skp, sega, nsega, skx, midx, psum, xkeys, xcounts,
+                                                      nextra);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_comb_add(const uint32_t* midx, const uint64_t* psum, uint64_t nsegp, uint64_t* counts,
+                            cudaStream_t s) {
+  if (nsegp == 0) return cudaSuccess;
+  k_comb_add<<<blocks_for(nsegp, 256), 256, 0, s>>>(midx, psum, nsegp, counts);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_key_lengths_list32(const uint32_t* keys, uint64_t n, uint64_t* lens, cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  k_key_lengths_list32<<<blocks_for(n, 256), 256, 0, s>>>(keys, n, lens);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_key_decode_list32(const uint32_t* keys, uint64_t n, const uint64_t* key_off, uint8_t* out,
+                                     cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  k_key_decode_list32<<<blocks_for(n, 256), 256, 0, s>>>(keys, n, key_off, out);
   count_launch();
   return cudaGetLastError();
 }

@@ -43,7 +43,7 @@ def test_c5_wordcount_8gib_vs_ground_truth():
     ko, vo = r["key_offsets"], r["val_offsets"]
     keys, vals = bytes(r["keys"]), r["vals"].view(np.uint64)
     assert r["n_keys"] == int((hist > 0).sum())
-    assert int(vals.sum()) == int(hist.sum()) == st["pairs"]
+    assert int(vals.sum()) == int(hist.sum()) == st["pairs"] + st["words_combined"]
     # every (word, count) equals the drawn-rank histogram (spellings are unique per rank)
     want = {pygen.word(i): int(c) for i in np.nonzero(hist)[0].tolist() for c in [hist[i]]}
     got = {keys[ko[i]:ko[i + 1]]: int(vals[i]) for i in range(r["n_keys"])}

@@ -53,7 +53,8 @@ def same(workload, batches, gkw=None, okw=None):
         assert np.array_equal(dg, do)
     else:
         assert dg == do
-    assert st["pairs"] == o["pairs"]
+    # WC: words absorbed by the in-SMEM combiner are not emitted as pairs
+    assert st["pairs"] + st["words_combined"] == o["pairs"]
     return dg, st
 
 
@@ -128,11 +129,36 @@ def test_wc_force_tiny_out_and_weak_hash():
     g = pygen.host_text(pygen.spec_wc(1_000_000, 5), 2)
     b = [(g["data"], g["offsets"], g["n"])]
     base, _ = same("wc", b)
-    tiny, st = same("wc", b, gkw={"flags": bmr.FLAG_FORCE_TINY_OUT})
-    assert st["flushes"] > 500            # 576-unit buffers instead of 2558
+    tiny, st = same("wc", b, gkw={"flags": bmr.FLAG_FORCE_TINY_OUT | bmr.FLAG_NO_MAP_COMBINE})
+    assert st["flushes"] > 500            # 641-unit buffers instead of 3068
+    tiny2, _ = same("wc", b, gkw={"flags": bmr.FLAG_FORCE_TINY_OUT})
+    assert tiny2 == tiny
     weak, st2 = same("wc", b, gkw={"flags": bmr.FLAG_WEAK_HASH_DEBUG})
     assert st2["collisions"] > 0          # verification found the forced collisions
     assert base == tiny == weak
+
+
+def test_wc_map_combiner_on_and_off():
+    # f-1: the in-SMEM combiner absorbs most repeated short words; the result must not depend on it
+    g = pygen.host_text(pygen.spec_wc(1_000_000, 5), 24)
+    b = [(g["data"], g["offsets"], g["n"])]
+    on, st_on = same("wc", b)
+    off, st_off = same("wc", b, gkw={"flags": bmr.FLAG_NO_MAP_COMBINE})
+    assert on == off
+    assert st_off["words_combined"] == 0 and st_off["pairs_partial"] == 0
+    assert st_on["words_combined"] > st_on["pairs"] // 4 and st_on["pairs_partial"] > 0
+    assert st_on["pairs"] + st_on["words_combined"] == st_off["pairs"]
+
+
+def test_wc_combiner_partials_replay_and_multibatch():
+    # tiny capacities: the exact, partial and hashed streams all overflow and the batches replay
+    g = pygen.host_text(pygen.spec_wc(10_000, 3), 3)
+    data, off = g["data"], g["offsets"]
+    cuts = [0, g["n"] // 4, g["n"] // 2, g["n"]]
+    b = [(data[int(off[a]):int(off[c])], off[a:c + 1] - off[a], c - a) for a, c in zip(cuts, cuts[1:])]
+    got, st = same("wc", b, gkw={"max_pairs_hint": 2000})
+    assert st["replays"] >= 3 and st["words_combined"] > 0
+    assert got == decode("wc", ora("wc", [(data, off, g["n"])]))
 
 
 def test_wc_replay_on_overflow():
@@ -195,6 +221,19 @@ def test_sm_self_overlap_and_boundaries():
     data, off = make_records(recs)
     got, _ = same("sm", [(data, off, len(recs))], gkw={"pattern": pat}, okw={"pattern": pat})
     assert len(got) == 985 + 0 + 1 + 25 + (20_000 - 15)
+
+
+def test_sm_short_records_offsets_from_global():
+    # ~4-byte records: > 512 record starts per 16 KiB tile, so the producers read the tile's
+    # offsets from global memory instead of staging them (StringMatch stages at most 512)
+    rng = np.random.default_rng(7)
+    pat = b"#needle:0123456#"
+    recs = [bytes(rng.integers(97, 100, size=int(rng.integers(0, 8)), dtype=np.uint8)) for _ in range(60_000)]
+    for i in rng.choice(len(recs), 300, replace=False).tolist():
+        recs[i] = b"x" + pat + b"y"
+    data, off = make_records(recs)
+    got, _ = same("sm", [(data, off, len(recs))], gkw={"pattern": pat}, okw={"pattern": pat})
+    assert len(got) == 300
 
 
 def test_sm_input_base_and_multibatch():
