@@ -816,7 +816,7 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
     const uint32_t jh = 31 - __clz(emit_mask);
     if ((nb >> (jh + 1)) == 0) {
       slow_bit = 1u << jh;
-      len_slow = slow_word_len(P, tv, p0 + jh, p0 + (lane < 31 ? 32 : 16));
+      len_slow = slow_word_len(P, tv, p0 + jh, p0 + 32);
     }
   }
   uint32_t near = 0;                                   // bit j: an nb bit in (j, j + kWcExact]
@@ -907,18 +907,24 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
   const uint32_t lane = threadIdx.x & 31;
   if constexpr (W == kWC) {
     // word bytes of this chunk; the next chunk's mask comes from lane + 1 (same window), so each
-    // lane classifies only its own 16 bytes.  Lane 31 knows nothing beyond its chunk: its words
-    // that do not end inside the chunk take the slow path.
+    // lane classifies only its own 16 bytes.  Lane 31 classifies the 16 bytes after the window
+    // itself (already loaded: x[4..7]); only words running past the 32 loaded bytes take the slow
+    // path.
     uint32_t w16 = 0;
     if (live) {
 #pragma unroll
       for (int i = 0; i < 4; ++i) w16 |= word_mask4(x[i]) << (4 * i);
     }
-    const uint32_t nxt = __shfl_down_sync(kFull, w16, 1);
+    uint32_t nxt = __shfl_down_sync(kFull, w16, 1);
     const uint32_t prv = __shfl_up_sync(kFull, w16, 1);
     if (live) {
-      const uint32_t known = lane < 31 ? 0xFFFFFFFFu : 0xFFFFu;
-      wm = (w16 | (lane < 31 ? nxt << 16 : 0u)) & vm;
+      if (lane == 31) {
+        nxt = 0;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) nxt |= word_mask4(x[4 + i]) << (4 * i);
+      }
+      const uint32_t known = 0xFFFFFFFFu;
+      wm = (w16 | (nxt << 16)) & vm;
       uint32_t prevw;
       if (lane == 0) prevw = (p0 - 1 >= 0 && p0 - 1 < N && is_word_byte(tv.sb[i0 - 1])) ? 1u : 0u;
       else prevw = (prv >> 15) & 1u;
