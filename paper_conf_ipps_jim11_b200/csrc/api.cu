@@ -324,7 +324,12 @@ struct mr_job {
   // WC Map output = exact stream + hashed stream (values 1, not stored); ingested WC pairs are
   // one general stream (key, kref, u64 partial count) like II
   bool split() const { return cfg.workload == MR_WORDCOUNT && !ingested; }
-  bool comb() const { return split() && !(cfg.flags & MR_FLAG_NO_MAP_COMBINE); }
+  bool wc_comb() const { return split() && !(cfg.flags & MR_FLAG_NO_MAP_COMBINE); }
+  // KM: the Map accumulates the cluster sums itself (k <= 64; not for ingested partials)
+  bool km_comb() const {
+    return cfg.workload == MR_KMEANS && k <= 64 && !km_partial && !(cfg.flags & MR_FLAG_NO_MAP_COMBINE);
+  }
+  bool km_combined = false;       // KM: sums / cnts were produced by the Map combiner
   bool ingested = false;          // pairs come from mr_ingest (WC values are u64 partial counts)
   bool km_partial = false;        // KM: sums/cnts hold ingested partials; finalise owned clusters
   int vb_cur = 0;                 // value bytes of the current pairs
@@ -406,7 +411,9 @@ cudaError_t launch_batch(mr_job* job, const Batch& b) {
   a.k = job->k;
   a.out.h = job->h.p;
   a.out.hx = job->hx.p;
-  a.out.hp = job->comb() ? job->hp.p : nullptr;
+  a.out.hp = job->wc_comb() ? job->hp.p : nullptr;
+  a.out.km_sums = job->km_comb() ? job->sums.p : nullptr;
+  a.out.km_cnts = job->km_comb() ? job->cnts.p : nullptr;
   a.out.cap_p = job->cap_p;
   a.out.kref = job->kref.p;
   a.out.v = job->v.p;
@@ -515,9 +522,9 @@ mr_status settle_map(mr_job* job) {
   if (hs->err & kErrKeyTooLong) return fail(job, MR_ERR_OVERFLOW, "an emitted key exceeds 65535 bytes");
   const uint64_t m = hs->pair_cursor, mb = job->split() ? hs->pair_cursor_b : 0;
   const uint64_t mc = job->split() ? hs->pair_cursor_c : 0;
-  const uint64_t mp = job->comb() ? hs->pair_cursor_p : 0;
+  const uint64_t mp = job->wc_comb() ? hs->pair_cursor_p : 0;
   if (m > job->cap || mb > job->cap_b || mc > job->cap_c || mp > job->cap_p) {
-    const uint64_t ncap_p = job->comb() ? std::max(job->cap_p, mp + mp / 8 + 4096) : 0;
+    const uint64_t ncap_p = job->wc_comb() ? std::max(job->cap_p, mp + mp / 8 + 4096) : 0;
     const uint64_t ncap = std::max(job->cap, m + m / 8 + 4096);
     const uint64_t ncap_b = job->split() ? std::max(job->cap_b, mb + mb / 8 + 4096) : 0;
     const uint64_t ncap_c = job->split() ? std::max(job->cap_c, mc + mc / 8 + 4096) : 0;
@@ -529,12 +536,16 @@ mr_status settle_map(mr_job* job) {
     }
     job->stats.capacity_pairs = job->cap + job->cap_b + job->cap_c;
     CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
+    if (job->km_comb()) {
+      CK(cudaMemsetAsync(job->sums.p, 0, 64ULL * job->k, job->stream), "reset sums");
+      CK(cudaMemsetAsync(job->cnts.p, 0, 8ULL * job->k, job->stream), "reset counts");
+    }
     for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
     job->stats.replays += job->batches.size();
     CK(read_state(job), "replay (async)");
     if (hs->pair_cursor > job->cap ||
         (job->split() && (hs->pair_cursor_b > job->cap_b || hs->pair_cursor_c > job->cap_c)) ||
-        (job->comb() && hs->pair_cursor_p > job->cap_p))
+        (job->wc_comb() && hs->pair_cursor_p > job->cap_p))
       return fail(job, MR_ERR_OOM, "replay still overflows");
   }
   return MR_OK;
@@ -627,6 +638,7 @@ mr_status mr_job_reset(mr_job* job) {
   job->host_batches = 0;
   job->ingested = false;
   job->km_partial = false;
+  job->km_combined = false;
   job->key_bits = (job->cfg.workload == MR_WORDCOUNT) ? 48u : 64u;
   job->key_bits_b = 48;
   job->mb = job->nseg_a = job->nseg_b = job->mc = job->nseg_c = 0;
@@ -682,11 +694,17 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
     const uint64_t cap_b = !wc ? 0 : hint ? hint : nbytes / 48 + 4096;
     const uint64_t cap_c = !wc ? 0 : hint ? hint : nbytes / 32 + 4096;
     CK(ensure_pairs(job, initial_cap(job, nbytes, n), cap_b, cap_c), "alloc intermediate");
-    if (job->comb()) {   // combiner partials: <= 4096 per CTA per batch (grown + replayed if exceeded)
+    if (job->wc_comb()) {   // combiner partials: <= 4096 per CTA per batch (grown + replayed if exceeded)
       job->cap_p = job->cfg.max_pairs_hint ? job->cfg.max_pairs_hint : 2ULL * 4096 * job->nsm + 4096;
       CK(job->hp.ensure(job->cap_p), "alloc partials");
     }
     job->stats.capacity_pairs = job->cap + job->cap_b + job->cap_c;
+  }
+  if (job->batches.empty() && job->km_comb()) {   // KM combiner accumulators (summed over batches)
+    CK(job->sums.ensure(8ULL * job->k), "alloc sums");
+    CK(job->cnts.ensure(job->k), "alloc counts");
+    CK(cudaMemsetAsync(job->sums.p, 0, 64ULL * job->k, job->stream), "zero sums");
+    CK(cudaMemsetAsync(job->cnts.p, 0, 8ULL * job->k, job->stream), "zero counts");
   }
   Batch b{records, offsets, n, nbytes, job->cfg.input_base + job->next_base};
   job->next_base += nbytes;
@@ -745,7 +763,7 @@ mr_status mr_group(mr_job* job) {
   job->m = m;
   job->mb = mb;
   job->mc = mc;
-  job->mp = job->comb() ? hs->pair_cursor_p : 0;
+  job->mp = job->wc_comb() ? hs->pair_cursor_p : 0;
   job->stats.pairs_partial = job->mp;
   job->stats.pairs = m + mb + mc;
   job->stats.pairs_hashed = mb;
@@ -753,6 +771,16 @@ mr_status mr_group(mr_job* job) {
   job->stats.flushes = hs->flushes;
   if (m_total >= (1ULL << 32) - 1 || mb >= (1ULL << 32) - 1 || mc >= (1ULL << 32) - 1)
     return fail(job, MR_ERR_UNSUPPORTED, ">= 2^32 intermediate pairs in one group");
+  if (job->km_comb()) {   // KM combiner: the Map produced the cluster sums; nothing to group
+    uint64_t pts = 0;
+    for (const Batch& b : job->batches) pts += b.n;
+    job->stats.words_combined = pts;
+    job->km_combined = true;
+    job->nseg = job->k;
+    if (job->prof.on) job->prof.collect();
+    job->state = kGrouped;
+    return MR_OK;
+  }
   if (job->cfg.workload == MR_STRINGMATCH) {  // Map-only
     job->nseg = m;
     if (job->prof.on) job->prof.collect();      // settle_map synchronised the stream
@@ -958,7 +986,7 @@ mr_status mr_reduce(mr_job* job) {
       const uint32_t k = job->k;
       CK(job->sums.ensure(8ULL * k), "alloc sums");
       CK(job->cnts.ensure(k), "alloc counts");
-      if (!job->km_partial) {
+      if (!job->km_partial && !job->km_combined) {
         CK(job->worklist.ensure(m / 1024 + 64), "alloc worklist");
         CK(launch_reduce_km(job->seg_start.p, S, job->skeys, job->perm, job->v.p, job->sums.p, job->cnts.p, k,
                             job->worklist.p, job->st, job->nsm, s),
@@ -1068,7 +1096,7 @@ mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_byte
       xs.hc = job->hc.p;
       xs.nc = job->mc;
       xs.hp = job->hp.p;
-      xs.np = job->comb() ? hs->pair_cursor_p : 0;
+      xs.np = job->wc_comb() ? hs->pair_cursor_p : 0;
       xs.n = m + xs.np + job->mc + job->mb;
       xs.kref = job->krefb.p;
     } else {

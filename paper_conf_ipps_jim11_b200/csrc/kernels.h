@@ -45,6 +45,8 @@ struct PairBufs {
   uint32_t* hx = nullptr;    // WC exact stream: 30-bit exact keys (u32; 0xFFFFFFFF = filler)
   uint64_t* hp = nullptr;    // WC combiner partials (exact key | count << 32); nullptr = no combiner
   uint64_t cap_p = 0;
+  double* km_sums = nullptr;             // KM combiner: cluster sums / counts accumulated by the
+  unsigned long long* km_cnts = nullptr; //   Map itself (nullptr = emit (id, point) pairs)
   uint64_t* kref = nullptr;  // (device address of key bytes << 16) | key length
   uint8_t* v = nullptr;      // value bytes (vbytes per pair)
   uint64_t cap = 0;          // capacity in pairs

@@ -31,15 +31,19 @@
 namespace bmr {
 namespace {
 
+// Map warps per CTA: KMeans 16 (one 32-point slice each of a 512-point tile); the text workloads
+// 24 (their Map is issue-bound on dependent integer chains: more warps per scheduler hide them)
 constexpr int kNMap = 16;
+constexpr int kNMapText = 24;
+template <int W>
+constexpr int nmap() { return W == 3 ? kNMap : kNMapText; }
 // Producer warps kProdWarp0 .. + kNProd - 1: producer p owns the iterations it == p (mod kNProd)
 // (and so the stages s == p (mod kNProd)); one warp alone is latency-bound at ~465 instructions
 // per tile (TMA issue + bitmap), slower than HBM delivers a tile (ncu, C2 round 1).
 constexpr int kNProd = 2;
-constexpr int kProdWarp0 = kNMap;
-constexpr int kFlushWarp0 = kNMap + kNProd;   // flush warps kFlushWarp0 .. kFlushWarp0 + kNFlush - 1
-constexpr int kNFlush = 1;
-constexpr int kThreads = (kNMap + kNProd + kNFlush) * 32;
+constexpr int kNFlush = 1;   // warps: map 0 .. nmap-1, producers nmap .. nmap+kNProd-1, then flush
+template <int W>
+constexpr int threads_of() { return (nmap<W>() + kNProd + kNFlush) * 32; }
 constexpr int kT = 16384;        // owned bytes per tile (text) / bytes per tile (KM)
 constexpr int kLead = 16;        // bytes staged before the tile (previous-byte context)
 constexpr int kHalo = 256;       // bytes staged after the tile (words / matches / URLs crossing it)
@@ -59,7 +63,7 @@ struct Cfg {
   static constexpr int kStages = (W == kSM) ? 6 : 4;
   static constexpr int kOffCap = 1024;   // record offsets staged per tile (more: read from global)
   static constexpr int kOffBytes = ((kOffCap + 2) * 8 + 127) / 128 * 128;
-  static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? 12288 : 20480;   // bytes per output buffer
+  static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? 10240 : 20480;   // bytes per output buffer
   // the producer builds the bitmap of tile it - kLag right after issuing tile it: kLag stages of
   // TMA traffic stay in flight per SM while one stage is being consumed
   static constexpr int kLag = kStages - 2;
@@ -88,6 +92,10 @@ constexpr uint32_t kWcExact = kExactMax;
 static_assert(kWin / (kWcExact + 1) + 1 <= Cfg<kWC>::kHashQ, "hash queue too small");
 static_assert(kWin / 2 + 1 <= Cfg<kWC>::kXQ, "exact-key queue too small");
 constexpr int kKmPts = kT / 32;                // 512 points per KM tile
+// KM combiner (k <= kKmCombMax): per-warp fp32 accumulators [kNMap][64][8] + counts [kNMap][64]
+// in the (otherwise unused for KM) offsets + bitmap stage regions
+constexpr int kKmCombMax = 64;
+constexpr int kKmWaccBytes = kNMap * kKmCombMax * 8 * 4;
 
 static_assert(kLead + kT + kHalo + 32 <= kStageBytes, "stage too small");
 static_assert(kBitWords * 4 <= kBitBytes, "bitmap too small");
@@ -129,14 +137,19 @@ struct Layout {
   static constexpr int offs = bytes + kStages * kStageBytes;      // kStages x kOffBytes
   static constexpr int bits = offs + kStages * Cfg<W>::kOffBytes; // kStages x kBitBytes
   static constexpr int out = bits + kStages * kBitBytes;          // kNOut x Cfg<W>::kOutHalf
-  static constexpr int hq = out + kNOut * Cfg<W>::kOutHalf;       // kNMap x kHashQ x 8 (WC)
-  static constexpr int xq = hq + kNMap * Cfg<W>::kHashQ * 8;      // kNMap x kXQ x 4 (WC)
-  static constexpr int comb = xq + kNMap * Cfg<W>::kXQ * 4;       // kCombSlots x 8 (WC)
+  static constexpr int hq = out + kNOut * Cfg<W>::kOutHalf;       // nmap x kHashQ x 8 (WC)
+  static constexpr int xq = hq + nmap<W>() * Cfg<W>::kHashQ * 8;  // nmap x kXQ x 4 (WC)
+  static constexpr int comb = xq + nmap<W>() * Cfg<W>::kXQ * 4;   // kCombSlots x 8 (WC)
   static constexpr int cent = comb + Cfg<W>::kCombSlots * 8;      // KM centroids
   static_assert(ready + kStages * 8 <= bytes, "header region overflow");
   static_assert(sizeof(OutCtl) <= hdr, "OutCtl overlaps the stage headers");
 };
 static_assert(64 % kNOut == 0, "6-bit generation counter must wrap on a buffer boundary");
+static_assert(Layout<kWC>::cent <= 232448 && Layout<kSM>::cent <= 232448 && Layout<kII>::cent <= 232448 &&
+                  Layout<kKM>::cent + 1024 * 32 <= 232448,
+              "SMEM layout exceeds 227 KB per CTA");
+static_assert(kKmWaccBytes + kNMap * kKmCombMax * 4 <= Layout<kKM>::out - Layout<kKM>::offs,
+              "KM combiner accumulators exceed the offsets + bitmap regions");
 
 // Output-buffer formats.  SM / KM / II: SoA runs [keys | krefs | values] of kCap entries.
 // WC: exact-key entries (u32 key) fill the buffer from the bottom, queued long-word entries (u64
@@ -177,7 +190,9 @@ struct Params {
   uint32_t* ohx;           // WC exact stream: u32 keys (capacity cap_pairs)
   uint64_t* ohp;           // WC combiner partials: (exact key | count << 32), capacity cap_p
   uint64_t cap_p;
-  uint32_t comb;           // WC: in-SMEM combiner on
+  uint32_t comb;           // WC / KM: in-SMEM combiner on
+  double* km_sums;         // KM combiner: job accumulators (k x 8 fp64, k u64), zeroed by the host
+  unsigned long long* km_cnts;
   uint32_t out_cap;        // per-half capacity actually used (FORCE_TINY_OUT shrinks it)
   uint32_t flags;
   DevState* st;
@@ -432,9 +447,11 @@ __device__ __forceinline__ uint32_t units(uint32_t c) {   // buffer space of pac
   if constexpr (W == kWC) return cur_ca(c) + 4u * cur_cb(c);
   else return cur_ca(c);
 }
-static_assert(PairFmt<kWC>::kCap + kNMap * PairFmt<kWC>::kMaxReserve <= kCaMask, "ca field overflow");
-static_assert(PairFmt<kWC>::kCap / 2 + kNMap * Cfg<kWC>::kHashQ <= kCbMask, "cb field overflow");
-static_assert(PairFmt<kSM>::kCap + kNMap * PairFmt<kSM>::kMaxReserve <= kCaMask, "ca field overflow");
+// WC: a reservation carries <= kWin / 2 + 1 exact entries (ca) and <= kHashQ queued ones (cb)
+static_assert(PairFmt<kWC>::kCap + kNMapText * (kWin / 2 + 1) <= kCaMask, "ca field overflow");
+static_assert(PairFmt<kWC>::kCap / 4 + kNMapText * Cfg<kWC>::kHashQ <= kCbMask, "cb field overflow");
+static_assert(PairFmt<kSM>::kCap + kNMapText * PairFmt<kSM>::kMaxReserve <= kCaMask, "ca field overflow");
+static_assert(PairFmt<kII>::kCap + kNMapText * PairFmt<kII>::kMaxReserve <= kCaMask, "ca field overflow");
 
 template <int W>
 __device__ __forceinline__ uint64_t sentinel_key(const Params& P) {
@@ -1063,9 +1080,19 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   // so a warp that drew cheap windows takes the next one instead of idling until the slowest
   // warp of the tile is done; a stage is released after all kNWin of its windows (empty[s]
   // counts windows).  KM: one point per map lane, kNMap arrivals per stage.
-  // (P.dyn == 0: static order, warp w takes windows w and w + kNMap of every tile)
-  static_assert(kNWin == 2 * kNMap, "static window order assumes two windows per warp and tile");
-  uint32_t kseq = 0;
+  // KM combiner: lane-owned fp64 sums / counts of clusters lane, lane + 32 (k <= kKmCombMax)
+  double kacc[kKmCombMax / 32][8];
+  unsigned long long kcnt[kKmCombMax / 32];
+#pragma unroll
+  for (int q = 0; q < kKmCombMax / 32; ++q) {
+    kcnt[q] = 0;
+#pragma unroll
+    for (int t = 0; t < 8; ++t) kacc[q][t] = 0.0;
+  }
+  // (P.dyn == 0: static order, map warp w takes windows w, w + nmap, w + 2 nmap, ... of the CTA's
+  // window sequence)
+  uint32_t kseq = 0, have_it = ~0u;
+  StageHdr hd{};
   for (uint32_t it = 0;; ++it) {
     uint32_t w = 0;
     if constexpr (W != kKM) {
@@ -1074,16 +1101,19 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         if (lane == 0) g = atomicAdd(&oc->win_next, 1u);
         g = __shfl_sync(kFull, g, 0);
       } else {
-        g = (kseq >> 1) * kNWin + warp + (kseq & 1u) * kNMap;
+        g = warp + kseq * static_cast<uint32_t>(nmap<W>());
         ++kseq;
       }
       it = g / kNWin;
       w = g % kNWin;
     }
     const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
-    if constexpr (W == kKM) mbar_wait(&full[s], ph);
-    else map_wait(P, reinterpret_cast<uint64_t*>(smem + Layout<W>::ready) + s, ph, kReadyWaitNs);
-    const StageHdr hd = *reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
+    if (it != have_it) {   // a warp's consecutive windows are mostly in one tile: wait + header once
+      if constexpr (W == kKM) mbar_wait(&full[s], ph);
+      else map_wait(P, reinterpret_cast<uint64_t*>(smem + Layout<W>::ready) + s, ph, kReadyWaitNs);
+      hd = *reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
+      have_it = it;
+    }
     if (hd.t < 0) break;
     const uint8_t* sb = smem + Layout<W>::bytes + s * kStageBytes;
     if constexpr (W == kKM) {
@@ -1136,7 +1166,35 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       const uint32_t m = __ballot_sync(kFull, valid);
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[s]);   // stage no longer read by this warp
-      if (m) {
+      if (P.comb) {
+        // f-1 combiner: fp32 per-warp cluster sums of this tile (<= 32 points per partial, as
+        // in the sorted Reduce, reading 5), folded into lane-owned fp64 registers
+        float* wacc = reinterpret_cast<float*>(smem + Layout<W>::offs) + warp * (kKmCombMax * 8);
+        uint32_t* wcnt = reinterpret_cast<uint32_t*>(smem + Layout<W>::offs + kKmWaccBytes) + warp * kKmCombMax;
+        if (valid) {
+#pragma unroll
+          for (int t = 0; t < 8; ++t) atomicAdd(wacc + t * kKmCombMax + best, x[t]);   // [dim][cluster]: no bank conflicts
+          atomicAdd(wcnt + best, 1u);
+        }
+        __syncwarp();
+#pragma unroll
+        for (int q = 0; q < kKmCombMax / 32; ++q) {
+          const uint32_t c = lane + 32 * q;
+          if (c < P.k) {
+            const uint32_t nc = wcnt[c];
+            if (nc) {
+              wcnt[c] = 0;
+              kcnt[q] += nc;
+#pragma unroll
+              for (int t = 0; t < 8; ++t) {
+                kacc[q][t] += static_cast<double>(wacc[t * kKmCombMax + c]);
+                wacc[t * kKmCombMax + c] = 0.0f;
+              }
+            }
+          }
+        }
+        __syncwarp();
+      } else if (m) {
         const uint32_t total = __popc(m);
         const Slot slot = reserve<W>(P, oc, outh, total, P.out_cap);
         if (valid) {
@@ -1162,12 +1220,25 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       if (lane == 0) mbar_arrive(&empty[s]);
     }
   }
+  if constexpr (W == kKM) {
+    if (P.comb) {   // this lane's clusters -> global fp64 sums / u64 counts (job accumulators)
+#pragma unroll
+      for (int q = 0; q < kKmCombMax / 32; ++q) {
+        const uint32_t c = lane + 32 * q;
+        if (c < P.k && kcnt[q]) {
+          atomicAdd(P.km_cnts + c, kcnt[q]);
+#pragma unroll
+          for (int t = 0; t < 8; ++t) atomicAdd(P.km_sums + c * 8 + t, kacc[q][t]);
+        }
+      }
+    }
+  }
   // final flush of the partially filled half (all map warps done, nothing pending)
-  named_bar_sync(2, kNMap * 32);
+  named_bar_sync(2, nmap<W>() * 32);
   if constexpr (W == kWC) {
     if (P.comb) {   // combiner partials -> global (one atomic per warp step; demand counted past capacity)
       const uint32_t* ctab = reinterpret_cast<const uint32_t*>(smem + Layout<W>::comb);
-      for (uint32_t i0 = warp * 32; i0 < static_cast<uint32_t>(Cfg<W>::kCombSlots); i0 += kNMap * 32) {
+      for (uint32_t i0 = warp * 32; i0 < static_cast<uint32_t>(Cfg<W>::kCombSlots); i0 += nmap<W>() * 32) {
         const uint32_t k = ctab[i0 + lane], c = ctab[Cfg<W>::kCombSlots + i0 + lane];
         const uint64_t v = static_cast<uint64_t>(k) | (static_cast<uint64_t>(c) << 32);
         const uint32_t mv = __ballot_sync(kFull, k != kCombEmpty32);
@@ -1187,7 +1258,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
 }
 
 template <int W>
-__global__ void __launch_bounds__(kThreads, 1) k_map(Params P) {
+__global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
   constexpr int kStages = Cfg<W>::kStages;
   extern __shared__ __align__(128) uint8_t smem[];
   OutCtl* oc = reinterpret_cast<OutCtl*>(smem + Layout<W>::ctl);
@@ -1219,6 +1290,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_map(Params P) {
     }
   }
   if constexpr (W == kKM) {
+    if (P.comb) {
+      uint32_t* z = reinterpret_cast<uint32_t*>(smem + Layout<W>::offs);
+      for (uint32_t i = threadIdx.x; i < static_cast<uint32_t>(kKmWaccBytes / 4 + kNMap * kKmCombMax); i += blockDim.x)
+        z[i] = 0;
+    }
     float* cent = reinterpret_cast<float*>(smem + Layout<W>::cent);
     // pair layout: centroids (2p, 2p+1) interleaved per coordinate -> f32x2 operands
     for (uint32_t i = threadIdx.x; i < P.k * 8; i += blockDim.x) {
@@ -1229,8 +1305,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_map(Params P) {
   }
   __syncthreads();
   const uint32_t warp = threadIdx.x >> 5;
-  if (warp >= kProdWarp0 && warp < kProdWarp0 + kNProd) producer_loop<W>(P, smem, warp - kProdWarp0);
-  else if (warp >= kFlushWarp0) flush_loop<W>(P, smem, oc);
+  if (warp >= static_cast<uint32_t>(nmap<W>()) && warp < static_cast<uint32_t>(nmap<W>() + kNProd))
+    producer_loop<W>(P, smem, warp - nmap<W>());
+  else if (warp >= static_cast<uint32_t>(nmap<W>() + kNProd)) flush_loop<W>(P, smem, oc);
   else map_loop<W>(P, smem, oc);
 }
 
@@ -1292,7 +1369,9 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.ohx = a.out.hx;
   P.ohp = a.out.hp;
   P.cap_p = a.out.cap_p;
-  P.comb = (W == kWC && a.out.hp != nullptr) ? 1u : 0u;
+  P.comb = (W == kWC && a.out.hp != nullptr) || (W == kKM && a.out.km_sums != nullptr && a.k <= kKmCombMax) ? 1u : 0u;
+  P.km_sums = a.out.km_sums;
+  P.km_cnts = a.out.km_cnts;
   P.pf = map_prefetch();
   P.wait_hint = map_wait_hint();
   P.dyn = map_dyn_windows(W);
@@ -1307,7 +1386,7 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   if (e != cudaSuccess) return e;
   int grid = a.grid > 0 ? a.grid : num_sms;
   if (static_cast<uint64_t>(grid) > P.ntiles) grid = static_cast<int>(P.ntiles);
-  k_map<W><<<grid, kThreads, smem, s>>>(P);
+  k_map<W><<<grid, threads_of<W>(), smem, s>>>(P);
   count_launch();
   return cudaGetLastError();
 }

@@ -405,13 +405,15 @@ int sort_variant32() {
 int sort_cfg() {
   static int c = [] {
     const char* e = getenv("BMR_SORT_CFG");
-    return e ? atoi(e) & 1 : 0;
+    return e ? atoi(e) & 3 : 0;
   }();
   return c;
 }
-int sort_tile() { return kSortThreads * (sort_cfg() ? 12 : 16); }
-int sort_tile_keys() { return kSortThreads * (sort_cfg() ? 24 : 16); }
-int sort_tile_keys32() { return kSortThreads * (sort_cfg() ? 32 : 24); }
+// u32 keys-only shapes (keys per thread, CTAs per SM): cfg 0 (24, 3), 1 (32, 2), 2 (16, 4), 3 (24, 2)
+static const int kIPT32[4] = {24, 32, 16, 24};
+int sort_tile() { return kSortThreads * (sort_cfg() == 1 ? 12 : 16); }
+int sort_tile_keys() { return kSortThreads * (sort_cfg() == 1 ? 24 : 16); }
+int sort_tile_keys32() { return kSortThreads * kIPT32[sort_cfg()]; }
 
 template <typename K, bool kFirst, int kVar, int IPT, int MINB, bool kPay, int LW = 4>
 static void launch_os(unsigned tiles, const K* keys_in, const uint32_t* idx_in, K* keys_out, uint32_t* idx_out,
@@ -431,7 +433,7 @@ template <bool kFirst, int kVar>
 static void launch_pay(unsigned tiles, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
                        uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
                        uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
-  if (sort_cfg() == 1) launch_os<uint64_t, kFirst, kVar, 12, 4, true>(BMR_OS_ARGS);
+  if (sort_cfg() == 1) launch_os<uint64_t, kFirst, kVar, 12, 4, true>(BMR_OS_ARGS);   // cfg 1: 12 keys, 4 CTAs
   else launch_os<uint64_t, kFirst, kVar, 16, 3, true>(BMR_OS_ARGS);
 }
 
@@ -453,6 +455,10 @@ static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* ke
   if constexpr (sizeof(K) == 4) {
     if (sort_cfg() == 1) {
       launch_os<K, false, 2, 32, 2, false>(BMR_OS_ARGS);
+    } else if (sort_cfg() == 2) {
+      launch_os<K, false, 2, 16, 4, false>(BMR_OS_ARGS);
+    } else if (sort_cfg() == 3) {
+      launch_os<K, false, 2, 24, 2, false>(BMR_OS_ARGS);
     } else {
       switch (sort_variant32()) {
         case 0: launch_os<K, false, 0, 24, 3, false>(BMR_OS_ARGS); break;
@@ -462,7 +468,7 @@ static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* ke
       }
     }
   } else if (keys_only) {
-    if (sort_cfg() == 1) launch_os<K, false, 2, 24, 2, false>(BMR_OS_ARGS);
+    if (sort_cfg() == 1) launch_os<K, false, 2, 24, 2, false>(BMR_OS_ARGS);   // cfg 1: 24 keys, 2 CTAs
     else launch_os<K, false, 2, 16, 3, false>(BMR_OS_ARGS);
   } else {
     switch ((sort_variant() ? 1 : 0) | (first ? 2 : 0)) {

@@ -272,12 +272,31 @@ def test_km_generator_blobs():
     assert int(cnt.sum()) == n
 
 
-@pytest.mark.parametrize("k", [1, 7, 32, 300])
-def test_km_random_quantised(k):
+@pytest.mark.parametrize("flags", [0, bmr.FLAG_NO_MAP_COMBINE], ids=["combiner", "sorted"])
+@pytest.mark.parametrize("k", [1, 7, 32, 64, 65, 300])
+def test_km_random_quantised(k, flags):
+    # k <= 64: the Map's in-SMEM combiner (f-1) unless NO_MAP_COMBINE; k > 64: sort + reduce
     rng = np.random.default_rng(k)
     pts = (rng.integers(-60_000, 60_000, size=(20_000, 8)) / 1024.0).astype(np.float32)
     cen = (rng.integers(-60_000, 60_000, size=(k, 8)) / 1024.0).astype(np.float32)
-    km_check(pts, cen)
+    km_check(pts, cen, flags=flags)
+
+
+def test_km_combiner_multibatch():
+    spec = pygen.KMSpec()
+    pts = pygen.host_km(spec, 32 * 3000 + 5)
+    _, init = pygen.km_centres(spec)
+    data = pts.view(np.uint8).reshape(-1)
+    cut = 32 * 1234 * 32
+    b = [(data[:cut], None, cut // 32), (data[cut:], None, len(pts) - cut // 32)]
+    r, st = gpu("km", b, centroids=init)
+    assert st["pairs"] == 0 and st["words_combined"] == len(pts)
+    o = ora("km", [(data, None, len(pts))], centroids=init)
+    cg, ng = decode("km", r)
+    co, no = decode("km", o)
+    assert np.array_equal(ng, no)
+    floor = np.abs(pts.astype(np.float64)).mean(0)
+    assert np.all(np.abs(cg.astype(np.float64) - co) <= KM_RTOL * np.maximum(np.abs(co), floor[None, :]))
 
 
 def test_km_empty_and_tiny():
@@ -290,7 +309,7 @@ def test_km_force_tiny_out():
     spec = pygen.KMSpec()
     pts = pygen.host_km(spec, 32 * 500)
     _, init = pygen.km_centres(spec)
-    km_check(pts, init, flags=bmr.FLAG_FORCE_TINY_OUT)
+    km_check(pts, init, flags=bmr.FLAG_FORCE_TINY_OUT | bmr.FLAG_NO_MAP_COMBINE)
 
 
 # ------------------------------------------------------------------ InvertedIndex
