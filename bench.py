@@ -207,7 +207,12 @@ def algorithmic(inp, st, steps):
         ph = passes - px - pc
         sort_b = px * 8 * mx + pc * 16 * mc + ((ph * 24 - 4) * mh if ph else 0.0)
     else:
-        map_b = inp["nbytes"] + off_b + m * {"sm": 8, "km": 40, "ii": 24}[wl]
+        if wl == "sm":   # lazy record directory: offsets are read only around pattern candidates
+            off_b = 0
+        if wl == "km" and st.get("words_combined", 0):   # KM combiner: no pairs written
+            map_b = inp["nbytes"]
+        else:
+            map_b = inp["nbytes"] + off_b + m * {"sm": 8, "km": 40, "ii": 24}[wl]
         sort_b = (passes * 24 - 4) * m if passes else 0.0   # first pass reads no payload
     hist_b = (4 * mx + 8 * (mc + mh)) if wl == "wc" else 8 * m
     return {"map": map_b, "hist": hist_b, "sort": sort_b, "passes": passes, "pairs": m, "pairs_exact": mx,
@@ -273,7 +278,7 @@ def main():
     # timed region: K steps, per-phase device times from the job's CUDA events
     acc = {k: 0.0 for k in ("map_ms", "hist_ms", "sort_ms", "seg_ms", "sort_keys_ms")}
     tot = {"pairs": 0, "sort_passes": 0, "kernel_launches": 0, "flushes": 0, "n_keys": 0, "pairs_hashed": 0,
-           "sort_passes_keys": 0, "pairs_mid": 0, "sort_passes_mid": 0}
+           "sort_passes_keys": 0, "pairs_mid": 0, "sort_passes_mid": 0, "words_combined": 0, "pairs_partial": 0}
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         barrier()
@@ -408,7 +413,9 @@ def main():
                     "bytes_per_step": int(alg["map"])},
             "pairs_per_step": int(alg["pairs"]), "sort_passes": alg["passes"],
             "wc_streams": ({"exact": int(alg["pairs_exact"]), "mid": int(tot["pairs_mid"] / args.steps),
-                            "hashed": int(tot["pairs_hashed"] / args.steps)} if inp["wl"] == "wc" else None),
+                            "hashed": int(tot["pairs_hashed"] / args.steps),
+                            "partials": int(tot["pairs_partial"] / args.steps)} if inp["wl"] == "wc" else None),
+            "map_combiner": {"words_or_points_absorbed": int(tot["words_combined"] / args.steps)},
             "distinct_keys": int(tot["n_keys"] / args.steps),
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "exchange": ({"kind": "hash all-to-all over NCCL (torch.distributed)", "send_bytes_per_rank": xbytes[0],

@@ -62,6 +62,11 @@ struct Cfg {
   // measured slower on C2: 2.38 against 2.07 ms)
   static constexpr int kStages = (W == kSM) ? 6 : 4;
   static constexpr int kOffCap = 1024;   // record offsets staged per tile (more: read from global)
+  // StringMatch reads the record directory lazily: record boundaries matter only where the
+  // pattern's first byte matches (planted, rare), so no offsets are staged and no bitmap is built;
+  // a candidate checks for a record start inside its 16 bytes by a binary search over the tile's
+  // offsets slice in global memory.  The producers only issue the byte TMA.
+  static constexpr bool kLazyDir = (W == kSM);
   static constexpr int kOffBytes = ((kOffCap + 2) * 8 + 127) / 128 * 128;
   static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? 10240 : 20480;   // bytes per output buffer
   // the producer builds the bitmap of tile it - kLag right after issuing tile it: kLag stages of
@@ -310,6 +315,7 @@ struct TileView {
   const uint8_t* sb;       // stage bytes
   const uint32_t* bm;      // record-start bitmap
   long long sbase, stg_hi;
+  unsigned long long ra, rb;   // the tile's record starts offsets[ra..rb) (lazy directory)
   __device__ bool is_start(long long q) const {
     long long i = q - sbase;
     return (bm[i >> 5] >> (i & 31)) & 1u;
@@ -730,11 +736,13 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
         const uint8_t* g = P.rec + w_lo;
         stage_copy_edges(d, g, static_cast<uint64_t>(max(0LL, stg_hi - w_lo)), lane, b_off, b_len);
         // clear the record-start bitmap (map warps set bits after the full barrier)
-        uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout<W>::bits + s * kBitBytes);
-        for (uint32_t i = lane; i < kBitBytes / 16; i += 32) reinterpret_cast<uint4*>(bm)[i] = make_uint4(0, 0, 0, 0);
+        if constexpr (!Cfg<W>::kLazyDir) {
+          uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout<W>::bits + s * kBitBytes);
+          for (uint32_t i = lane; i < kBitBytes / 16; i += 32) reinterpret_cast<uint4*>(bm)[i] = make_uint4(0, 0, 0, 0);
+        }
         // offsets slice offsets[ra..rb) (record starts in the staged window)
         const uint64_t cnt = rb - ra;
-        const bool staged = cnt <= static_cast<uint64_t>(Cfg<W>::kOffCap);
+        const bool staged = !Cfg<W>::kLazyDir && cnt <= static_cast<uint64_t>(Cfg<W>::kOffCap);
         uint32_t shift = 0;
         const uint8_t* og = reinterpret_cast<const uint8_t*>(P.off + ra);
         if (staged && cnt) {
@@ -786,11 +794,13 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
                                                         reinterpret_cast<const uint8_t*>(P.off + rbf));
           }
         }
-        if (it >= Cfg<W>::kLag) finish_stage<W>(P, smem, it - Cfg<W>::kLag);   // same owner (kLag % kNProd == 0)
+        if constexpr (!Cfg<W>::kLazyDir) {
+          if (it >= Cfg<W>::kLag) finish_stage<W>(P, smem, it - Cfg<W>::kLag);   // same owner (kLag % kNProd == 0)
+        }
       }
     }
   }
-  if constexpr (W != kKM) {   // this producer's tiles whose bitmap is still pending
+  if constexpr (W != kKM && !Cfg<W>::kLazyDir) {   // this producer's tiles whose bitmap is still pending
     const uint32_t j0 = T > static_cast<uint32_t>(Cfg<W>::kLag) ? T - Cfg<W>::kLag : 0u;
     for (uint32_t j = j0; j < T; ++j)
       if (j % kNProd == pw) finish_stage<W>(P, smem, j);
@@ -801,7 +811,7 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
   mbar_wait(&empty[s], ph ^ 1u);
   if (lane == 0) {
     reinterpret_cast<StageHdr*>(smem + Layout<W>::hdr + s * 128)->t = -1;
-    if constexpr (W == kKM) mbar_arrive(&full[s]);
+    if constexpr (W == kKM || Cfg<W>::kLazyDir) mbar_arrive(&full[s]);
     else mbar_arrive(reinterpret_cast<uint64_t*>(smem + Layout<W>::ready) + s);
   }
 }
@@ -913,7 +923,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
     x[0] = c0.x; x[1] = c0.y; x[2] = c0.z; x[3] = c0.w;
     x[4] = c1.x; x[5] = c1.y; x[6] = c1.z; x[7] = c1.w;
     vm = range_mask32(p0, 0, N);
-    R = bits32(tv.bm, i0);
+    if constexpr (!Cfg<W>::kLazyDir) R = bits32(tv.bm, i0);
   } else {
 #pragma unroll
     for (int i = 0; i < 8; ++i) x[i] = 0;
@@ -959,10 +969,18 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
         const uint32_t j = __ffs(cand) - 1;
         cand &= cand - 1;
         if (p0 + j + 16 > N) continue;
-        if ((R >> (j + 1)) & 0x7FFFu) continue;             // match must lie inside one record
         uint32_t w[4];
         window16(x, j, w);
-        if (w[0] == P.pat[0] && w[1] == P.pat[1] && w[2] == P.pat[2] && w[3] == P.pat[3]) emit_mask |= 1u << j;
+        if (w[0] != P.pat[0] || w[1] != P.pat[1] || w[2] != P.pat[2] || w[3] != P.pat[3]) continue;
+        // the match must lie inside one record: no record start in (p, p + 15] (lazy directory)
+        unsigned long long lo = tv.ra, hi = tv.rb;
+        const unsigned long long p = static_cast<unsigned long long>(p0 + j);
+        while (lo < hi) {                                   // first record start > p in the slice
+          const unsigned long long mid = (lo + hi) >> 1;
+          if (P.off[mid] > p) hi = mid; else lo = mid + 1;
+        }
+        if (lo < tv.rb && P.off[lo] <= p + 15) continue;   // (offsets[rb] lies beyond the halo)
+        emit_mask |= 1u << j;
       }
     }
   } else if constexpr (W == kII) {
@@ -1109,7 +1127,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
     }
     const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
     if (it != have_it) {   // a warp's consecutive windows are mostly in one tile: wait + header once
-      if constexpr (W == kKM) mbar_wait(&full[s], ph);
+      if constexpr (W == kKM || Cfg<W>::kLazyDir) mbar_wait(&full[s], ph);
       else map_wait(P, reinterpret_cast<uint64_t*>(smem + Layout<W>::ready) + s, ph, kReadyWaitNs);
       hd = *reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
       have_it = it;
@@ -1209,7 +1227,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       }
     } else {
       const uint32_t* bm = reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * kBitBytes);
-      TileView tv{sb, bm, hd.sbase, hd.stg_hi};
+      TileView tv{sb, bm, hd.sbase, hd.stg_hi, hd.ra, hd.rb};
       const long long wp = hd.chunk0 + static_cast<long long>(w) * kWin;
       if (wp < hd.hi) {                               // warp-uniform
         const long long p0 = wp + lane * 16;
