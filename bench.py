@@ -229,6 +229,9 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--units", type=int, default=0, help="override pages (text) / points (KM) per GPU")
+    ap.add_argument("--mode", default="SIO", choices=["SIO", "SO", "SI", "G"],
+                    help="Map memory-usage mode (PAPER.md L129-135 ablation, SURVEY §8(f) f-2)")
+    ap.add_argument("--no-map-combine", action="store_true", help="literal north-star order (no Map combiner)")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -257,7 +260,11 @@ def main():
         WORKLOADS[args.workload] = (w[0], w[1] + f" [reduced: {args.units} units]", args.units)
     inp = make_input(args.workload, rank, dev)
     torch.cuda.synchronize()
-    job = bmr.Job(inp["wl"], **job_kwargs(inp, bmr.FLAG_PROFILE, local, rank, world))
+    mode_flags = {"SIO": 0, "SO": bmr.FLAG_NO_SMEM_IN, "SI": bmr.FLAG_NO_SMEM_OUT,
+                  "G": bmr.FLAG_NO_SMEM_IN | bmr.FLAG_NO_SMEM_OUT}[args.mode]
+    if args.no_map_combine:
+        mode_flags |= bmr.FLAG_NO_MAP_COMBINE
+    job = bmr.Job(inp["wl"], **job_kwargs(inp, bmr.FLAG_PROFILE | mode_flags, local, rank, world))
     stream = torch.cuda.current_stream()
     exchange = world > 1 and inp["wl"] != "sm"      # SM is Map-only: no exchange
     xbytes = [0]
@@ -356,7 +363,7 @@ def main():
             h_off = torch.empty(inp["offsets"].numel(), dtype=torch.int64, pin_memory=True)
             h_off.copy_(inp["offsets"])
         torch.cuda.synchronize()
-        job_e = bmr.Job(inp["wl"], **job_kwargs(inp, 0, local, rank, world))
+        job_e = bmr.Job(inp["wl"], **job_kwargs(inp, mode_flags, local, rank, world))
         d2h = 0
 
         def estep():
@@ -405,7 +412,8 @@ def main():
             "dtype": "f32" if wl == "km" else "u8", "data": "synthetic",
             "config": {"workload": args.workload, "description": WORKLOADS[args.workload][1],
                        "input_bytes_per_gpu": inp["nbytes"], "records_per_gpu": inp["n"],
-                       "l2": "inputs larger than L2 (no flush needed)", "parallelism": f"dp{world}"},
+                       "l2": "inputs larger than L2 (no flush needed)", "parallelism": f"dp{world}",
+                       "map_mode": args.mode, "map_combiner": not args.no_map_combine},
             "records_per_s": round(inp["n"] * world / (ms_max / 1e3), 1),
             "hbm_frac_end_to_end": round((alg["map"] + alg["hist"] + alg["sort"]) / (ms_max / 1e3) / 1e9 / hbm, 4),
             "phases_ms": {k[:-3]: round(v, 3) for k, v in per.items()},

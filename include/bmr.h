@@ -44,8 +44,9 @@ typedef enum {
 typedef enum { MR_WORDCOUNT = 1, MR_STRINGMATCH = 2, MR_KMEANS = 3, MR_INVINDEX = 4 } mr_workload;
 
 /* Flags */
-#define MR_FLAG_NO_SMEM_IN      0x01u /* reserved: SO ablation (L134) */
-#define MR_FLAG_NO_SMEM_OUT     0x02u /* reserved: SI ablation (L135) */
+#define MR_FLAG_NO_SMEM_IN      0x01u /* SO ablation (L134): map warps read record bytes from global memory */
+#define MR_FLAG_NO_SMEM_OUT     0x02u /* SI ablation (L135): one global atomic per warp result, direct HBM writes */
+                                      /* both = G (L173); neither = SIO, the default (L133, C-3 #18) */
 #define MR_FLAG_FORCE_TINY_OUT  0x04u /* output half = one warp result: every warp result overflows (L113) */
 #define MR_FLAG_WEAK_HASH_DEBUG 0x08u /* 4-bit key hash: forces collisions, exercises verification */
 #define MR_FLAG_VALIDATE        0x10u /* host-side argument validation of offsets (reads them back) */

@@ -208,6 +208,11 @@ struct Params {
   uint32_t pf;             // L2 prefetch distance in producer tiles (0: off)
   uint32_t wait_hint;      // idle mbarrier waits: 0 plain try_wait, 1 suspend-time hint, 2 helpers sleep-poll
   uint32_t dyn;            // text: windows handed out dynamically (1) or in static warp order (0)
+  // memory-mode ablations (§IV-C): so = no input staging
+  // (map warps read record bytes from global memory; the record directory is still staged),
+  // si = no output staging (each warp result is appended to global memory with one global
+  // atomic per warp, L135 / L171-173); both = the paper's G mode
+  uint32_t so, si;
 };
 
 // Idle wait of a role warp on an mbarrier phase (map warps on a staged tile, producers on a free
@@ -714,7 +719,7 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
         const uint64_t p_lo = t * kKmPts, p_hi = min(P.n, p_lo + kKmPts);
         const uint8_t* g = P.rec + p_lo * 32;
         uint8_t* d = sb + (reinterpret_cast<uintptr_t>(g) & 15u);   // same 16-B phase as the source
-        stage_copy_edges(d, g, (p_hi - p_lo) * 32, lane, b_off, b_len);
+        if (!P.so) stage_copy_edges(d, g, (p_hi - p_lo) * 32, lane, b_off, b_len);
         if (lane == 0) {
           hd->t = static_cast<long long>(t);
           hd->lo = static_cast<long long>(p_lo);
@@ -734,7 +739,7 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
         // stage bytes [w_lo, stg_hi) at sb + (w_lo - sbase); (rec + sbase) is 16-B aligned
         uint8_t* d = sb + (w_lo - sbase);
         const uint8_t* g = P.rec + w_lo;
-        stage_copy_edges(d, g, static_cast<uint64_t>(max(0LL, stg_hi - w_lo)), lane, b_off, b_len);
+        if (!P.so) stage_copy_edges(d, g, static_cast<uint64_t>(max(0LL, stg_hi - w_lo)), lane, b_off, b_len);
         // clear the record-start bitmap (map warps set bits after the full barrier)
         if constexpr (!Cfg<W>::kLazyDir) {
           uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout<W>::bits + s * kBitBytes);
@@ -886,6 +891,42 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
     nq += __popc(mb);
   }
   if (nx + nq == 0) return;
+  if (P.si) {   // SI / G ablation: append straight to the three global streams, one atomic each
+    __syncwarp();
+    unsigned long long gx = 0;
+    if (lane == 0 && nx) gx = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(nx));
+    gx = __shfl_sync(kFull, gx, 0);
+    for (uint32_t i = lane; i < nx; i += 32)
+      if (gx + i < P.cap_pairs) P.ohx[gx + i] = xq[i];
+    for (uint32_t q0 = 0; q0 < nq; q0 += 32) {
+      const uint32_t q = q0 + lane;
+      const bool in = q < nq;
+      ulonglong2 ent = make_ulonglong2(0ULL, 0ULL);
+      if (in) {
+        const uint64_t e = hq[q];
+        const long long p = tv.sbase + static_cast<long long>(e & 0xFFFFFF);
+        const uint32_t len = static_cast<uint32_t>(e >> 24);
+        ent = len <= kMidMax ? make_ulonglong2(exact_key(bytes8_at(P, tv, p, len), len), 0ULL)
+                             : make_ulonglong2(key_at(P, tv, p, len), (reinterpret_cast<uint64_t>(P.rec + p) << 16) | len);
+      }
+      const uint32_t mc = __ballot_sync(kFull, in && ent.y == 0), mbm = __ballot_sync(kFull, in && ent.y != 0);
+      unsigned long long gc = 0, gbb = 0;
+      if (lane == 0) {
+        if (mc) gc = atomicAdd(&P.st->pair_cursor_c, static_cast<unsigned long long>(__popc(mc)));
+        if (mbm) gbb = atomicAdd(&P.st->pair_cursor_b, static_cast<unsigned long long>(__popc(mbm)));
+      }
+      gc = __shfl_sync(kFull, gc, 0);
+      gbb = __shfl_sync(kFull, gbb, 0);
+      if (in && ent.y == 0) {
+        const uint64_t o = gc + __popc(mc & lanemask_lt());
+        if (o < P.cap_c) P.ohc[o] = ent.x;
+      } else if (in) {
+        const uint64_t o = gbb + __popc(mbm & lanemask_lt());
+        if (o < P.cap_b) { P.ohb[o] = ent.x; P.okrefb[o] = ent.y; }
+      }
+    }
+    return;
+  }
   const uint32_t packed = nx | (nq << kCbShift);
   const Slot slot = reserve<kWC>(P, oc, outh, packed, P.out_cap);
   uint8_t* half = outh + slot.half * Cfg<kWC>::kOutHalf;
@@ -918,10 +959,29 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
   uint32_t x[8];
   uint32_t vm = 0, R = 0;
   if (live) {
-    const uint4 c0 = *reinterpret_cast<const uint4*>(tv.sb + i0);
-    const uint4 c1 = *reinterpret_cast<const uint4*>(tv.sb + i0 + 16);
-    x[0] = c0.x; x[1] = c0.y; x[2] = c0.z; x[3] = c0.w;
-    x[4] = c1.x; x[5] = c1.y; x[6] = c1.z; x[7] = c1.w;
+    if (P.so) {   // SO / G ablation: the 32 bytes straight from global memory (rec + p0 is 16-B aligned)
+      if (p0 >= 0 && p0 + 32 <= N) {
+        const uint4 c0 = __ldg(reinterpret_cast<const uint4*>(P.rec + p0));
+        const uint4 c1 = __ldg(reinterpret_cast<const uint4*>(P.rec + p0 + 16));
+        x[0] = c0.x; x[1] = c0.y; x[2] = c0.z; x[3] = c0.w;
+        x[4] = c1.x; x[5] = c1.y; x[6] = c1.z; x[7] = c1.w;
+      } else {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          uint32_t w = 0;
+          for (int b = 0; b < 4; ++b) {
+            const long long q = p0 + 4 * i + b;
+            if (q >= 0 && q < N) w |= static_cast<uint32_t>(P.rec[q]) << (8 * b);
+          }
+          x[i] = w;
+        }
+      }
+    } else {
+      const uint4 c0 = *reinterpret_cast<const uint4*>(tv.sb + i0);
+      const uint4 c1 = *reinterpret_cast<const uint4*>(tv.sb + i0 + 16);
+      x[0] = c0.x; x[1] = c0.y; x[2] = c0.z; x[3] = c0.w;
+      x[4] = c1.x; x[5] = c1.y; x[6] = c1.z; x[7] = c1.w;
+    }
     vm = range_mask32(p0, 0, N);
     if constexpr (!Cfg<W>::kLazyDir) R = bits32(tv.bm, i0);
   } else {
@@ -953,7 +1013,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
       const uint32_t known = 0xFFFFFFFFu;
       wm = (w16 | (nxt << 16)) & vm;
       uint32_t prevw;
-      if (lane == 0) prevw = (p0 - 1 >= 0 && p0 - 1 < N && is_word_byte(tv.sb[i0 - 1])) ? 1u : 0u;
+      if (lane == 0) prevw = (p0 - 1 >= 0 && p0 - 1 < N && is_word_byte(P.so ? P.rec[p0 - 1] : tv.sb[i0 - 1])) ? 1u : 0u;
       else prevw = (prv >> 15) & 1u;
       nb = (~wm | R) & known;                                  // a word cannot continue here
       emit_mask = wm & 0xFFFFu & ~(((wm << 1) | prevw) & ~R);  // word starts (C-2 WC)
@@ -1051,12 +1111,27 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
   // ---- reserve one warp result, then lane-major emission rounds
   const uint32_t total = __reduce_add_sync(kFull, __popc(emit_mask));
   if (total == 0) return;
-  const Slot slot = reserve<W>(P, oc, outh, total, P.out_cap);
-  uint8_t* half = outh + slot.half * Cfg<W>::kOutHalf;
-  uint64_t* sh = reinterpret_cast<uint64_t*>(half);
-  uint64_t* sk = sh + F::kCap;
-  uint8_t* sv = half + F::kCap * (F::kKref ? 16 : 8);
-  uint32_t k = slot.base;
+  Slot slot{0, 0};
+  uint64_t* sh;
+  uint64_t* sk;
+  uint8_t* sv;
+  uint64_t k, cap = ~0ULL;
+  if (P.si) {   // SI / G ablation: one global atomic per warp result, lanes write HBM directly
+    unsigned long long gb = 0;
+    if (lane == 0) gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(total));
+    k = __shfl_sync(kFull, gb, 0);
+    sh = P.oh;
+    sk = P.okref;
+    sv = P.ov;
+    cap = P.cap_pairs;
+  } else {
+    slot = reserve<W>(P, oc, outh, total, P.out_cap);
+    uint8_t* half = outh + slot.half * Cfg<W>::kOutHalf;
+    sh = reinterpret_cast<uint64_t*>(half);
+    sk = sh + F::kCap;
+    sv = half + F::kCap * (F::kKref ? 16 : 8);
+    k = slot.base;
+  }
   uint32_t m_left = emit_mask;
   int nth = 0;
   while (__any_sync(kFull, m_left != 0)) {
@@ -1065,23 +1140,26 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
     if (act) {
       const uint32_t j = __ffs(m_left) - 1;
       m_left &= m_left - 1;
-      const uint32_t idx = k + __popc(m & lanemask_lt());
+      const uint64_t idx = k + __popc(m & lanemask_lt());
       const long long p = p0 + j;
       if constexpr (W == kSM) {
-        sh[idx] = P.gbase + static_cast<uint64_t>(p);
+        if (idx < cap) sh[idx] = P.gbase + static_cast<uint64_t>(p);
       } else if constexpr (W == kII) {
         uint32_t len = nth == 0 ? aux[0] : aux[1];
         ++nth;
         const long long q0 = p + 9;
         if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
-        sh[idx] = key_at(P, tv, q0, len);
-        sk[idx] = (reinterpret_cast<uint64_t>(P.rec + q0) << 16) | len;
-        reinterpret_cast<uint64_t*>(sv)[idx] = P.gbase + static_cast<uint64_t>(q0);
+        const uint64_t key = key_at(P, tv, q0, len);
+        if (idx < cap) {
+          sh[idx] = key;
+          sk[idx] = (reinterpret_cast<uint64_t>(P.rec + q0) << 16) | len;
+          reinterpret_cast<uint64_t*>(sv)[idx] = P.gbase + static_cast<uint64_t>(q0);
+        }
       }
     }
     k += __popc(m);
   }
-  commit(oc, slot, total);
+  if (!P.si) commit(oc, slot, total);
 }
 
 template <int W>
@@ -1143,8 +1221,9 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       float x[8];
       uint32_t best = 0;
       if (valid) {
-        const float4 a = reinterpret_cast<const float4*>(pt)[0];
-        const float4 b = reinterpret_cast<const float4*>(pt)[1];
+        const float4* src = P.so ? reinterpret_cast<const float4*>(P.rec + i * 32) : reinterpret_cast<const float4*>(pt);
+        const float4 a = P.so ? __ldg(src) : src[0];
+        const float4 b = P.so ? __ldg(src + 1) : src[1];
         x[0] = a.x; x[1] = a.y; x[2] = a.z; x[3] = a.w; x[4] = b.x; x[5] = b.y; x[6] = b.z; x[7] = b.w;
         float bd = 0.0f;
         // C-2 KM: fp32 RN, explicit chain d = fma(x_t - c_t, x_t - c_t, d) over t = 0..7, ties ->
@@ -1212,6 +1291,17 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
           }
         }
         __syncwarp();
+      } else if (m && P.si) {   // SI / G ablation: global append per warp result
+        unsigned long long gb = 0;
+        if (lane == 0) gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(__popc(m)));
+        gb = __shfl_sync(kFull, gb, 0);
+        const uint64_t o = gb + __popc(m & lanemask_lt());
+        if (valid && o < P.cap_pairs) {
+          P.oh[o] = best;
+          float4* gv = reinterpret_cast<float4*>(P.ov + o * 32);
+          gv[0] = make_float4(x[0], x[1], x[2], x[3]);
+          gv[1] = make_float4(x[4], x[5], x[6], x[7]);
+        }
       } else if (m) {
         const uint32_t total = __popc(m);
         const Slot slot = reserve<W>(P, oc, outh, total, P.out_cap);
@@ -1227,7 +1317,8 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       }
     } else {
       const uint32_t* bm = reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * kBitBytes);
-      TileView tv{sb, bm, hd.sbase, hd.stg_hi, hd.ra, hd.rb};
+      // (SO: an empty stage makes every helper read global memory)
+      TileView tv{sb, bm, hd.sbase, P.so ? hd.sbase : hd.stg_hi, hd.ra, hd.rb};
       const long long wp = hd.chunk0 + static_cast<long long>(w) * kWin;
       if (wp < hd.hi) {                               // warp-uniform
         const long long p0 = wp + lane * 16;
@@ -1393,6 +1484,8 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.pf = map_prefetch();
   P.wait_hint = map_wait_hint();
   P.dyn = map_dyn_windows(W);
+  P.so = (a.flags & 1u) ? 1u : 0u;   // MR_FLAG_NO_SMEM_IN
+  P.si = (a.flags & 2u) ? 1u : 0u;   // MR_FLAG_NO_SMEM_OUT
   if (P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>((P.ntiles + 255) / 256);

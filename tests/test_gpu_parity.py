@@ -161,6 +161,38 @@ def test_wc_combiner_partials_replay_and_multibatch():
     assert got == decode("wc", ora("wc", [(data, off, g["n"])]))
 
 
+MODES = {"SO": bmr.FLAG_NO_SMEM_IN, "SI": bmr.FLAG_NO_SMEM_OUT, "G": bmr.FLAG_NO_SMEM_IN | bmr.FLAG_NO_SMEM_OUT}
+
+
+@pytest.mark.parametrize("mode", sorted(MODES))
+def test_memory_modes_wc_ii_sm(mode):
+    # f-2: the paper's memory-usage modes (SO / SI / G, L129-135, L171-175) on the same kernel
+    # give the SIO result for every text workload, incl. ragged tails and capacity replays
+    f = MODES[mode]
+    g = pygen.host_text(pygen.spec_wc(1_000_000, 5), 3)
+    b = [(g["data"], g["offsets"], g["n"])]
+    assert same("wc", b, gkw={"flags": f})[0] == same("wc", b)[0]
+    same("wc", b, gkw={"flags": f, "max_pairs_hint": 5000})
+    data, off = make_records(_mixed_length_records(9, 3000))
+    same("wc", [(data, off, len(off) - 1)], gkw={"flags": f | bmr.FLAG_NO_MAP_COMBINE})
+    gi = pygen.host_text(pygen.spec_ii(4), 2)
+    same("ii", [(gi["data"], gi["offsets"], gi["n"])], gkw={"flags": f})
+    spec = pygen.spec_sm(plant_ppm=50_000)
+    gs = pygen.host_text(spec, 2, truth=True)
+    got, _ = same("sm", [(gs["data"], gs["offsets"], gs["n"])], gkw={"pattern": spec.pattern, "flags": f},
+                  okw={"pattern": spec.pattern})
+    assert np.array_equal(got, gs["plants"])
+
+
+@pytest.mark.parametrize("mode", sorted(MODES))
+def test_memory_modes_km(mode):
+    spec = pygen.KMSpec()
+    pts = pygen.host_km(spec, 32 * 700 + 3)
+    _, init = pygen.km_centres(spec)
+    km_check(pts, init, flags=MODES[mode])
+    km_check(pts, init, flags=MODES[mode] | bmr.FLAG_NO_MAP_COMBINE)
+
+
 def test_wc_replay_on_overflow():
     g = pygen.host_text(pygen.spec_wc(10_000, 1), 1)
     got, st = same("wc", [(g["data"], g["offsets"], g["n"])], gkw={"max_pairs_hint": 1000})

@@ -31,8 +31,9 @@ def raw(rep):
     return rows[0], rows[1], rows[2:]
 
 
-def top_stalls(rep, n=6):
-    out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+def top_stalls(rep, idx=0, n=6):
+    out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass",
+                          "--launch-skip", str(idx), "--launch-count", "1"],
                          capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
     if len(rows) < 3:
@@ -75,13 +76,13 @@ def main():
     with open(out, "w") as f:
         for rep in sys.argv[2:]:
             h, units, rows = raw(rep)
-            for r in rows:
+            for idx, r in enumerate(rows):
                 f.write(f"## {rep.split('/')[-1]} — {r[h.index('Kernel Name')][:120]}\n\n")
                 for m, label in METRICS:
                     if m in h:
                         f.write(f"- {label}: {r[h.index(m)]} {units[h.index(m)]}\n")
                 f.write("\nTop SASS stall sites (share of warp-stall samples, executions, instruction):\n\n")
-                for share, inst, src in top_stalls(rep):
+                for share, inst, src in top_stalls(rep, idx):
                     f.write(f"- {share:5.1f}%  x{inst}  `{src[:90]}`\n")
                 f.write("\n")
 
