@@ -96,7 +96,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
   using Smem = SortSmem<K, IPT, kPay, kBins>;
   constexpr int kSortTile = Smem::kTile;
   constexpr bool kAtomicRank = (kVar & 1) != 0, kEarly = (kVar & 2) != 0;
-  constexpr bool kBackoff = (kVar & 4) != 0, kMatchHist = (kVar & 8) != 0;
+  constexpr bool kBackoff = (kVar & 4) != 0, kMatchHist = (kVar & 8) != 0, kBallotPeers = (kVar & 16) != 0;
   static_assert(kDPT >= 1 && kDPT * kSortThreads == kBins, "bins must be a multiple of the block size");
   extern __shared__ __align__(16) uint8_t raw[];
   Smem& S = *reinterpret_cast<Smem*>(raw);
@@ -159,7 +159,20 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
 #pragma unroll
     for (int j = 0; j < kSortIPT; ++j) {
       const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & kMask;
-      const uint32_t peers = __match_any_sync(0xffffffffu, dj);
+      uint32_t peers;
+      if constexpr (kBallotPeers) {
+        // lanes with the same digit by bit slicing: kBits ballots (short latency, independent of
+        // the other steps) instead of match.any (ncu: 49% of the stall samples wait on MATCH)
+        peers = 0xffffffffu;
+#pragma unroll
+        for (int b = 0; b < kBits; ++b) {
+          const bool bit = (dj >> b) & 1u;
+          const uint32_t bal = __ballot_sync(0xffffffffu, bit);
+          peers &= bit ? bal : ~bal;
+        }
+      } else {
+        peers = __match_any_sync(0xffffffffu, dj);
+      }
       const uint32_t leader = __ffs(peers) - 1;
       uint32_t before = 0;
       if (lane == leader) {
@@ -391,7 +404,7 @@ int sort_variant() {
 int sort_variant32() {
   static int v = [] {
     const char* e = getenv("BMR_SORT_VARIANT32");
-    return e ? atoi(e) & 3 : 2;
+    return e ? atoi(e) : 2;
   }();
   return v;
 }
@@ -413,7 +426,8 @@ int sort_cfg() {
 static const int kIPT32[4] = {24, 32, 16, 24};
 int sort_tile() { return kSortThreads * (sort_cfg() == 1 ? 12 : 16); }
 int sort_tile_keys() { return kSortThreads * (sort_cfg() == 1 ? 24 : 16); }
-int sort_tile_keys32() { return kSortThreads * kIPT32[sort_cfg()]; }
+int sort_variant32();
+int sort_tile_keys32() { return kSortThreads * (sort_variant32() == 19 ? 16 : kIPT32[sort_cfg()]); }
 
 template <typename K, bool kFirst, int kVar, int IPT, int MINB, bool kPay, int LW = 4>
 static void launch_os(unsigned tiles, const K* keys_in, const uint32_t* idx_in, K* keys_out, uint32_t* idx_out,
@@ -464,6 +478,8 @@ static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* ke
         case 0: launch_os<K, false, 0, 24, 3, false>(BMR_OS_ARGS); break;
         case 1: launch_os<K, false, 1, 24, 3, false>(BMR_OS_ARGS); break;
         case 3: launch_os<K, false, 3, 24, 3, false>(BMR_OS_ARGS); break;
+        case 18: launch_os<K, false, 18, 24, 3, false>(BMR_OS_ARGS); break;
+        case 19: launch_os<K, false, 18, 16, 3, false>(BMR_OS_ARGS); break;
         default: launch_os<K, false, 2, 24, 3, false>(BMR_OS_ARGS); break;
       }
     }
