@@ -137,6 +137,17 @@ mr_status mr_map(mr_job* job, const uint8_t* records, const uint64_t* offsets, u
  * memory on the job stream (the end-to-end path of bench.py). */
 mr_status mr_map_host(mr_job* job, const uint8_t* records, const uint64_t* offsets, uint64_t n);
 
+/* Map HOST text whose records are its '\n'-terminated lines (the record model of the text
+ * configs, Table II "a line"): record i ends with the i-th '\n' (inclusive); bytes after
+ * the last '\n' form one more record.  Equivalent to mr_map_host(text, offsets, n) with those
+ * offsets, without an offsets array crossing the host link: the library copies the text in
+ * batches (~256 MiB, ending after a '\n') on its own copy stream and, per batch, derives the
+ * offsets on the device and runs the Map while the next batch is in flight.  `text` (caller-
+ * owned) must stay valid until the call returns; pin it (cudaHostRegister / cudaMallocHost) for
+ * the copies to overlap.  Each batch becomes one mapped batch (SM/II offsets stay global).
+ * MR_ERR_INVALID for fixed-stride workloads (KM) or text == NULL with nbytes > 0. */
+mr_status mr_map_host_lines(mr_job* job, const uint8_t* text, uint64_t nbytes);
+
 /* Group by key (§8(a) a6-a8): capacity check (grow + replay on overflow), digit histogram,
  * onesweep LSD passes over non-constant digits, segment boundaries with byte verification of
  * hashed keys (re-sort with a fresh hash on collision).  Synchronises the stream. */

@@ -28,7 +28,7 @@ FLAG_PROFILE, FLAG_OWN_STREAM, FLAG_NO_MAP_COMBINE = 0x40, 0x80, 0x100
 STATUS = {0: "MR_OK", 1: "MR_ERR_INVALID", 2: "MR_ERR_STATE", 3: "MR_ERR_OOM", 4: "MR_ERR_OVERFLOW",
           5: "MR_ERR_CUDA", 6: "MR_ERR_NCCL", 7: "MR_ERR_UNSUPPORTED"}
 
-EXPORTS = ("mr_job_create", "mr_map", "mr_map_host", "mr_group", "mr_reduce", "mr_fetch", "mr_job_reset",
+EXPORTS = ("mr_job_create", "mr_map", "mr_map_host", "mr_map_host_lines", "mr_group", "mr_reduce", "mr_fetch", "mr_job_reset",
            "mr_get_stats", "mr_job_destroy", "mr_status_string", "mr_last_error", "mr_sort_u64",
            "mr_partition_count", "mr_partition_write", "mr_ingest")
 
@@ -82,6 +82,7 @@ def lib() -> C.CDLL:
         L.mr_job_create.argtypes = [C.POINTER(Config), C.POINTER(vp)]
         L.mr_map.argtypes = [vp, vp, vp, u64]
         L.mr_map_host.argtypes = [vp, vp, vp, u64]
+        L.mr_map_host_lines.argtypes = [vp, vp, u64]
         for f in ("mr_group", "mr_reduce", "mr_job_reset", "mr_job_destroy"):
             getattr(L, f).argtypes = [vp]
         L.mr_fetch.argtypes = [vp, C.POINTER(Result)]
@@ -174,6 +175,11 @@ class Job:
         if n is None:
             n = (len(offsets) - 1) if offsets is not None else records.size // 32
         self._check(lib().mr_map_host(self.h, _ptr(records), _ptr(offsets), n))
+
+    def map_host_lines(self, text: np.ndarray):
+        """Host text whose records are its '\n'-terminated lines (offsets derived on the device,
+        copies overlapped with the Map; pin `text` for the overlap)."""
+        self._check(lib().mr_map_host_lines(self.h, _ptr(text), int(text.size)))
 
     def group(self):
         self._check(lib().mr_group(self.h))

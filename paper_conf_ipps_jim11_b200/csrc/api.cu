@@ -288,6 +288,8 @@ struct mr_job {
   std::vector<DBuf<uint8_t>> host_rec;   // device copies made by mr_map_host (reused after reset)
   std::vector<DBuf<uint64_t>> host_off;
   size_t host_batches = 0;
+  cudaStream_t cstream = nullptr;        // copy stream of mr_map_host_lines
+  std::vector<cudaEvent_t> line_ev;
   Prof prof;
   unsigned long long launches0 = 0;
   SortWork sw, swb, swc, swp;
@@ -742,6 +744,87 @@ mr_status mr_map_host(mr_job* job, const uint8_t* records, const uint64_t* offse
     doff = job->host_off[i].p;
   }
   return map_common(job, job->host_rec[i].p, doff, n);
+}
+
+// mr_map_host_lines batch size (BMR_LINE_CHUNK bytes, default 256 MiB): copies of batch b + 1
+// overlap the line split and Map of batch b
+static uint64_t line_chunk() {   // read per call (tests shrink it to force many batches)
+  const char* e = getenv("BMR_LINE_CHUNK");
+  return e ? std::max<uint64_t>(strtoull(e, nullptr, 10), 64) : (256ULL << 20);
+}
+
+mr_status mr_map_host_lines(mr_job* job, const uint8_t* text, uint64_t nbytes) {
+  const uint64_t kLineChunk = line_chunk();
+  if (!job) return MR_ERR_INVALID;
+  if (job->cfg.record_stride > 0) return fail(job, MR_ERR_INVALID, "mr_map_host_lines: text workloads only");
+  if (nbytes && !text) return fail(job, MR_ERR_INVALID, "text is NULL");
+  CK(cudaSetDevice(job->cfg.device), "set device");
+  if (!job->cstream) {
+    CK(cudaStreamCreateWithFlags(&job->cstream, cudaStreamNonBlocking), "copy stream");
+  }
+  // batches of ~kLineChunk bytes ending after a '\n' (host-side memrchr on the caller's text)
+  std::vector<uint64_t> cut{0};
+  while (cut.back() < nbytes) {
+    uint64_t end = std::min(nbytes, cut.back() + kLineChunk);
+    if (end < nbytes) {
+      const void* nl = memrchr(text + cut.back(), '\n', end - cut.back());
+      if (nl) end = static_cast<const uint8_t*>(nl) - text + 1;
+      else {  // a line longer than a chunk: extend to its end
+        const void* f = memchr(text + end, '\n', nbytes - end);
+        end = f ? static_cast<const uint8_t*>(f) - text + 1 : nbytes;
+      }
+    }
+    cut.push_back(end);
+  }
+  const size_t nb = cut.size() - 1;
+  const size_t ti = job->host_batches++;
+  if (job->host_rec.size() <= ti) { job->host_rec.resize(ti + 1); job->host_off.resize(ti + 1); }
+  CK(job->host_rec[ti].ensure(nbytes + 64), "alloc device text");
+  uint8_t* dtext = job->host_rec[ti].p;
+  // copies on the copy stream, one event per batch; the job stream waits per batch
+  if (job->line_ev.size() < nb) {
+    const size_t old = job->line_ev.size();
+    job->line_ev.resize(nb);
+    for (size_t b = old; b < nb; ++b) CK(cudaEventCreateWithFlags(&job->line_ev[b], cudaEventDisableTiming), "event");
+  }
+  CK(cudaEventRecord(job->line_ev[0], job->stream), "event");   // copies start after earlier work
+  CK(cudaStreamWaitEvent(job->cstream, job->line_ev[0], 0), "wait");
+  for (size_t b = 0; b < nb; ++b) {
+    CK(cudaMemcpyAsync(dtext + cut[b], text + cut[b], cut[b + 1] - cut[b], cudaMemcpyHostToDevice, job->cstream),
+       "H2D text");
+    CK(cudaEventRecord(job->line_ev[b], job->cstream), "event");
+  }
+  for (size_t b = 0; b < nb; ++b) {
+    const uint64_t lo = cut[b], hi = cut[b + 1];
+    CK(cudaStreamWaitEvent(job->stream, job->line_ev[b], 0), "wait text");
+    const uint64_t tiles = line_tiles(lo, hi);
+    CK(job->seg_counts.ensure(tiles + 1), "alloc line counts");
+    CK(job->tile_base.ensure(tiles + 1), "alloc line bases");
+    CK(launch_line_count(dtext, lo, hi, job->seg_counts.p, job->stream), "line count");
+    uint64_t* ss;
+    uint32_t ep;
+    CK(scan_ws(job, tiles, &ss, &ep), "alloc scan workspace");
+    CK(launch_scan_u32to64(job->seg_counts.p, job->tile_base.p, tiles, &job->st->seg_total, ss, ep,
+                           &job->st->tile_counter[1], job->stream),
+       "scan line counts");
+    CK(read_state(job), "sync line count");
+    const uint64_t nl = job->st_h.p->seg_total;
+    const bool open_end = text[hi - 1] != '\n';
+    const uint64_t n = nl + (open_end ? 1 : 0);
+    const size_t oi = job->host_batches++;
+    if (job->host_rec.size() <= oi) { job->host_rec.resize(oi + 1); job->host_off.resize(oi + 1); }
+    CK(job->host_off[oi].ensure(n + 1), "alloc device offsets");
+    uint64_t* off = job->host_off[oi].p;
+    CK(cudaMemsetAsync(off, 0, 8, job->stream), "offsets[0]");
+    CK(launch_line_write(dtext, lo, hi, job->tile_base.p, off, job->stream), "line offsets");
+    if (open_end) {
+      job->tmp_h.p[1] = hi - lo;
+      CK(cudaMemcpyAsync(off + n, job->tmp_h.p + 1, 8, cudaMemcpyHostToDevice, job->stream), "offsets[n]");
+    }
+    mr_status st = map_common(job, dtext + lo, off, n);
+    if (st != MR_OK) return st;
+  }
+  return MR_OK;
 }
 
 mr_status mr_group(mr_job* job) {
@@ -1234,6 +1317,8 @@ mr_status mr_job_destroy(mr_job* job) {
   job->keys_h.release(); job->vals_h.release(); job->key_off_h.release(); job->val_off_h.release();
   job->st_h.release(); job->tmp_h.release();
   if (job->st) cudaFree(job->st);
+  for (cudaEvent_t e : job->line_ev) cudaEventDestroy(e);
+  if (job->cstream) cudaStreamDestroy(job->cstream);
   if (job->own_stream && job->stream) cudaStreamDestroy(job->stream);
   cudaGetLastError();
   delete job;

@@ -179,6 +179,12 @@ cudaError_t launch_iota_scaled(uint64_t n, uint64_t scale, uint64_t* out, cudaSt
 // recompute every key in the 64-bit format with a fresh hash seed (collision slow path)
 cudaError_t launch_rehash(uint64_t* h, const uint64_t* kref, uint64_t m, uint64_t seed, cudaStream_t s);
 
+// ---- record directory of '\n'-terminated text (lines.cu) ----
+uint64_t line_tiles(uint64_t lo, uint64_t hi);
+cudaError_t launch_line_count(const uint8_t* base, uint64_t lo, uint64_t hi, uint32_t* counts, cudaStream_t s);
+cudaError_t launch_line_write(const uint8_t* base, uint64_t lo, uint64_t hi, const uint64_t* tile_base, uint64_t* off,
+                              cudaStream_t s);
+
 // ---- multi-GPU exchange (exchange.cu) ----
 constexpr int kMaxRanks = 64;
 enum XMode : int { kXPairs = 0, kXSegs = 1, kXKM = 2, kXSplit = 3 };

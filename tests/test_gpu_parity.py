@@ -193,6 +193,32 @@ def test_memory_modes_km(mode):
     km_check(pts, init, flags=MODES[mode] | bmr.FLAG_NO_MAP_COMBINE)
 
 
+@pytest.mark.parametrize("chunk", [None, 100_000, 4_096])
+def test_map_host_lines_equals_offsets(chunk, monkeypatch):
+    # mr_map_host_lines: the device-derived line directory (in batches overlapped with the copies)
+    # gives the same result as the host offsets, incl. an unterminated last line and lines longer
+    # than a batch
+    if chunk:
+        monkeypatch.setenv("BMR_LINE_CHUNK", str(chunk))
+    g = pygen.host_text(pygen.spec_wc(1_000_000, 5), 2)
+    text = np.concatenate([g["data"], np.frombuffer(b"tail words " * 700 + b"no newline", np.uint8)])
+    off = np.concatenate([g["offsets"], np.array([len(text)], np.uint64)])
+    n = len(off) - 1
+    for wl, kw in (("wc", {}), ("ii", {}), ("sm", {"pattern": b"tail words tail "})):
+        with bmr.Job(wl, **kw) as job:
+            job.map_host_lines(text)
+            job.group()
+            job.reduce()
+            got = decode(wl, job.fetch())
+            st = job.stats()
+        want = decode(wl, ora(wl, [(text, off, n)], **({"pattern": kw["pattern"]} if wl == "sm" else {})))
+        if wl == "sm":
+            assert np.array_equal(got, want) and len(got) > 0
+        else:
+            assert got == want
+        assert st["input_bytes"] == len(text)
+
+
 def test_wc_replay_on_overflow():
     g = pygen.host_text(pygen.spec_wc(10_000, 1), 1)
     got, st = same("wc", [(g["data"], g["offsets"], g["n"])], gkw={"max_pairs_hint": 1000})
