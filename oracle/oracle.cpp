@@ -17,6 +17,9 @@
 //   Workloads (C-2; "Word Count ... String Match ... Inverted Index ... KMeans"):
 //     WC  word = maximal [0-9A-Za-z] run inside a record; emit (word, u32 1); reduce = u64 sum.
 //     SM  every j with j+16 <= len and rec[j..j+16) == P: emit u64 global offset (overlaps count).
+//     SML (SM per line, the paper's own output, L125 "search a line for the keyword; emit the
+//         line if found"): a record with at least one such j emits the u64 global offset of its
+//         first byte, once (Map-only).
 //     KM  d_j = fmaf chain of (x_t - c_jt)^2 in fp32 RN, argmin with ties -> lowest j; emit
 //         (u32 j, 32-B point); reduce: cnt (u64), sum in fp64, c'_j = (float)(sum/cnt),
 //         empty cluster keeps c_j; output all k clusters.
@@ -34,7 +37,7 @@
 
 namespace {
 
-enum { WC = 1, SM = 2, KM = 3, II = 4 };
+enum { WC = 1, SM = 2, KM = 3, II = 4, SML = 5 };
 
 struct Job {
   int workload = 0;
@@ -74,6 +77,14 @@ void map_sm(Job& J, const uint8_t* b, uint64_t len, uint64_t gpos) {
   if (len < 16) return;
   for (uint64_t j = 0; j + 16 <= len; ++j)
     if (std::memcmp(b + j, J.pattern, 16) == 0) J.pairs.emplace_back(u64_bytes(gpos + j), std::string());
+}
+
+void map_sml(Job& J, const uint8_t* b, uint64_t len, uint64_t gpos) {
+  for (uint64_t j = 0; j + 16 <= len; ++j)
+    if (std::memcmp(b + j, J.pattern, 16) == 0) {
+      J.pairs.emplace_back(u64_bytes(gpos), std::string());
+      return;
+    }
 }
 
 void map_km(Job& J, const uint8_t* b, uint64_t len) {
@@ -120,7 +131,7 @@ void push(Job& J, const std::string& k, const std::string& v) {
 void reduce(Job& J) {
   J.keys.clear(); J.vals.clear();
   J.key_off.assign(1, 0); J.val_off.assign(1, 0);
-  if (J.workload == SM) {  // Map-only; canonical = offsets ascending
+  if (J.workload == SM || J.workload == SML) {  // Map-only; canonical = offsets ascending
     std::vector<uint64_t> o;
     o.reserve(J.pairs.size());
     for (auto& p : J.pairs) o.push_back(bytes_u64(p.first));
@@ -181,7 +192,7 @@ typedef struct {
 } oracle_result;
 
 void* oracle_create(int workload, const uint8_t* pattern16, uint32_t k, const float* centroids) {
-  if (workload < WC || workload > II) return nullptr;
+  if (workload < WC || workload > SML) return nullptr;
   Job* J = new Job();
   J->workload = workload;
   if (pattern16) std::memcpy(J->pattern, pattern16, 16);
@@ -206,6 +217,7 @@ int oracle_map(void* job, const uint8_t* records, const uint64_t* offsets, uint6
     switch (J->workload) {
       case WC: map_wc(*J, b, e - a); break;
       case SM: map_sm(*J, b, e - a, batch_base + a); break;
+      case SML: map_sml(*J, b, e - a, batch_base + a); break;
       case KM: map_km(*J, b, e - a); break;
       case II: map_ii(*J, b, e - a, batch_base + a); break;
     }

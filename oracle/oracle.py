@@ -12,8 +12,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-WC, SM, KM, II = 1, 2, 3, 4
-NAMES = {"wc": WC, "sm": SM, "km": KM, "ii": II}
+WC, SM, KM, II, SML = 1, 2, 3, 4, 5
+NAMES = {"wc": WC, "sm": SM, "km": KM, "ii": II, "sml": SML}   # sml: StringMatch per line (L125)
 
 
 class _Result(C.Structure):

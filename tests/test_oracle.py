@@ -114,6 +114,31 @@ def test_sm_bruteforce_tiny(seed):
     assert np.array_equal(got, exp)
 
 
+@pytest.mark.parametrize("seed", range(4))
+def test_sm_lines_bruteforce(seed):
+    # the paper's per-line StringMatch (L125: "emit the line if found"): Python `in` per record
+    rng = np.random.default_rng(300 + seed)
+    pat = b"abababababababab"
+    recs = []
+    for _ in range(60):
+        r = bytearray(rng.choice(list(b"ab "), size=int(rng.integers(0, 70))).tolist())
+        for _ in range(int(rng.integers(0, 3))):
+            if len(r) >= 16:
+                j = int(rng.integers(0, len(r) - 15))
+                r[j:j + 16] = pat
+        recs.append(bytes(r))
+    data, off = make_records(recs)
+    base = 77
+    got = decode("sm", oracle.run("sml", [(data, off, len(recs), 0, base)], pattern=pat))
+    exp = np.array([base + int(off[i]) for i, r in enumerate(recs) if pat in r], np.uint64)
+    assert np.array_equal(got, exp) and len(exp) > 0
+    # every line of the per-offset output's records, once
+    per_off = decode("sm", oracle.run("sm", [(data, off, len(recs), 0, base)], pattern=pat))
+    starts = np.array([base + int(o) for o in off[:-1]], np.uint64)
+    rec_of = np.searchsorted(starts, per_off, side="right") - 1
+    assert np.array_equal(np.unique(starts[rec_of]), got)
+
+
 def test_sm_self_overlap_985():
     data, off = make_records([b"a" * 1000])
     got = decode("sm", oracle.run("sm", [(data, off, 1, 0, 0)], pattern=b"a" * 16))
