@@ -54,6 +54,8 @@ typedef enum { MR_WORDCOUNT = 1, MR_STRINGMATCH = 2, MR_KMEANS = 3, MR_INVINDEX 
 #define MR_FLAG_PROFILE         0x40u /* record CUDA events per phase on the job stream (mr_stats *_ms) */
 #define MR_FLAG_OWN_STREAM      0x80u /* ignore cfg.stream: the job creates a private non-blocking stream */
 #define MR_FLAG_NO_MAP_COMBINE  0x100u /* WC: no in-SMEM combiner in the Map (every word is emitted as a pair) */
+#define MR_FLAG_SM_LINES        0x200u /* SM: the paper's per-line output (L125): the global offset of every
+                                          record containing the pattern, once (grouped by key) */
 
 typedef struct { uint8_t pattern[16]; } mr_sm_params;                      /* StringMatch */
 typedef struct { uint32_t k, dim; const float* centroids; } mr_km_params;  /* KMeans: host ptr, k x dim fp32, dim == 8, 1 <= k <= 1024 */

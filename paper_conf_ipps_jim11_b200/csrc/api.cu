@@ -864,6 +864,21 @@ mr_status mr_group(mr_job* job) {
     job->state = kGrouped;
     return MR_OK;
   }
+  if (job->cfg.workload == MR_STRINGMATCH && (job->cfg.flags & MR_FLAG_SM_LINES)) {
+    // per-line output (L125): one record start per match -> sort + unique (the group-by path)
+    CK(run_sort(job->sw, job->h.p, m, &job->skeys, nullptr, job->st, job->nsm, job->stream, &job->prof,
+                &job->stats.hist_ms, &job->stats.sort_ms, 64),
+       "radix sort (lines)");
+    job->stats.sort_passes += job->sw.passes;
+    job->perm = nullptr;
+    CK(job->seg_start.ensure(m + 1), "alloc segments");
+    st = do_segments_into(job, job->skeys, m, job->seg_start.p, job->nseg);
+    if (st != MR_OK) return st;
+    job->stats.n_keys = job->nseg;
+    if (job->prof.on) job->prof.collect();
+    job->state = kGrouped;
+    return MR_OK;
+  }
   if (job->cfg.workload == MR_STRINGMATCH) {  // Map-only
     job->nseg = m;
     if (job->prof.on) job->prof.collect();      // settle_map synchronised the stream
@@ -1090,12 +1105,18 @@ mr_status mr_reduce(mr_job* job) {
       break;
     }
     case MR_STRINGMATCH: {
-      CK(job->key_off.ensure(m + 1), "alloc key offsets");
-      CK(job->val_off.ensure(m + 1), "alloc val offsets");
-      CK(launch_iota_scaled(m, 8, job->key_off.p, s), "key offsets");
-      CK(cudaMemsetAsync(job->val_off.p, 0, (m + 1) * 8, s), "val offsets");
-      job->out_n = m;
-      job->out_keys_bytes = m * 8;
+      const uint64_t n = S;   // matches, or (per-line output) distinct record starts
+      if (job->cfg.flags & MR_FLAG_SM_LINES) {
+        CK(job->keys_out.ensure(8 * n + 8), "alloc keys");
+        CK(launch_seg_keys(job->seg_start.p, n, job->skeys, reinterpret_cast<uint64_t*>(job->keys_out.p), s),
+           "line keys");
+      }
+      CK(job->key_off.ensure(n + 1), "alloc key offsets");
+      CK(job->val_off.ensure(n + 1), "alloc val offsets");
+      CK(launch_iota_scaled(n, 8, job->key_off.p, s), "key offsets");
+      CK(cudaMemsetAsync(job->val_off.p, 0, (n + 1) * 8, s), "val offsets");
+      job->out_n = n;
+      job->out_keys_bytes = n * 8;
       job->out_vals_bytes = 0;
       break;
     }
@@ -1115,7 +1136,9 @@ mr_status mr_fetch(mr_job* job, mr_result* out) {
   CK(job->vals_h.ensure(job->out_vals_bytes + 1), "alloc host vals");
   CK(job->key_off_h.ensure(n + 1), "alloc host key offsets");
   CK(job->val_off_h.ensure(n + 1), "alloc host val offsets");
-  const uint8_t* dkeys = job->cfg.workload == MR_STRINGMATCH ? reinterpret_cast<const uint8_t*>(job->h.p) : job->keys_out.p;
+  const uint8_t* dkeys = (job->cfg.workload == MR_STRINGMATCH && !(job->cfg.flags & MR_FLAG_SM_LINES))
+                             ? reinterpret_cast<const uint8_t*>(job->h.p)
+                             : job->keys_out.p;
   const uint8_t* dvals = job->cfg.workload == MR_WORDCOUNT ? reinterpret_cast<const uint8_t*>(job->counts.p)
                          : job->cfg.workload == MR_INVINDEX ? reinterpret_cast<const uint8_t*>(job->gathered.p)
                                                             : job->vals_out.p;

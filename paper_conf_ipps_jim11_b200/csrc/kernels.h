@@ -163,6 +163,7 @@ cudaError_t launch_key_lengths_exact32(const uint64_t* seg_start, uint64_t nseg,
 cudaError_t launch_key_decode32(const uint64_t* seg_start, uint64_t nseg, const uint32_t* skeys,
                                 const uint64_t* key_off, uint8_t* keys, cudaStream_t s);
 cudaError_t launch_gather_u64(const uint32_t* perm, const uint8_t* v, uint64_t m, uint64_t* out, cudaStream_t s);
+cudaError_t launch_seg_keys(const uint64_t* seg, uint64_t nseg, const uint64_t* sk, uint64_t* out, cudaStream_t s);
 // WC combiner partials (f-1): merge into the exact stream's segments (midx / psum) or the extra
 // list of partial-only keys (xkeys / xcounts, *nextra of them)
 cudaError_t launch_comb_merge(const uint64_t* segp, uint64_t nsegp, const uint64_t* skp, const uint64_t* sega,

@@ -213,6 +213,7 @@ struct Params {
   // si = no output staging (each warp result is appended to global memory with one global
   // atomic per warp, L135 / L171-173); both = the paper's G mode
   uint32_t so, si;
+  uint32_t sm_lines;       // StringMatch: emit the matching record's start (MR_FLAG_SM_LINES)
 };
 
 // Idle wait of a role warp on an mbarrier phase (map warps on a staged tile, producers on a free
@@ -1143,7 +1144,16 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
       const uint64_t idx = k + __popc(m & lanemask_lt());
       const long long p = p0 + j;
       if constexpr (W == kSM) {
-        if (idx < cap) sh[idx] = P.gbase + static_cast<uint64_t>(p);
+        uint64_t key = static_cast<uint64_t>(p);
+        if (P.sm_lines) {   // the paper's per-line output (L125): the match's record start instead
+          unsigned long long lo = tv.ra, hi = tv.rb;
+          while (lo < hi) {
+            const unsigned long long mid = (lo + hi) >> 1;
+            if (P.off[mid] > key) hi = mid; else lo = mid + 1;
+          }
+          key = P.off[lo - 1];   // lo >= 1: offsets[0] = 0 <= p
+        }
+        if (idx < cap) sh[idx] = P.gbase + key;
       } else if constexpr (W == kII) {
         uint32_t len = nth == 0 ? aux[0] : aux[1];
         ++nth;
@@ -1486,6 +1496,7 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.dyn = map_dyn_windows(W);
   P.so = (a.flags & 1u) ? 1u : 0u;   // MR_FLAG_NO_SMEM_IN
   P.si = (a.flags & 2u) ? 1u : 0u;   // MR_FLAG_NO_SMEM_OUT
+  P.sm_lines = (W == kSM && (a.flags & 0x200u)) ? 1u : 0u;   // MR_FLAG_SM_LINES
   if (P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>((P.ntiles + 255) / 256);

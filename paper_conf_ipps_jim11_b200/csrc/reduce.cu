@@ -431,6 +431,11 @@ __global__ void k_key_decode_list32(const uint32_t* keys, uint64_t n, const uint
   uint8_t* dst = out + key_off[s];
   for (uint32_t i = 0; i < len; ++i) dst[i] = static_cast<uint8_t>(b >> (8 * i));
 }
+// keys at the segment heads of a sorted keys-only stream (SM per-line output: unique record starts)
+__global__ void k_seg_keys(const uint64_t* seg, uint64_t nseg, const uint64_t* sk, uint64_t* out) {
+  const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
+  if (s < nseg) out[s] = sk[seg[s]];
+}
 __global__ void k_gather_u64(const uint32_t* perm, const uint64_t* v, uint64_t m, uint64_t* out) {
   const uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
   if (i < m) out[i] = v[perm[i]];
@@ -605,6 +610,12 @@ cudaError_t launch_key_decode_list32(const uint32_t* keys, uint64_t n, const uin
                                      cudaStream_t s) {
   if (n == 0) return cudaSuccess;
   k_key_decode_list32<<<blocks_for(n, 256), 256, 0, s>>>(keys, n, key_off, out);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_seg_keys(const uint64_t* seg, uint64_t nseg, const uint64_t* sk, uint64_t* out, cudaStream_t s) {
+  if (nseg == 0) return cudaSuccess;
+  k_seg_keys<<<blocks_for(nseg, 256), 256, 0, s>>>(seg, nseg, sk, out);
   count_launch();
   return cudaGetLastError();
 }

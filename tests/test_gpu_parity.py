@@ -294,6 +294,23 @@ def test_sm_short_records_offsets_from_global():
     assert len(got) == 300
 
 
+@pytest.mark.parametrize("flags", [0, bmr.FLAG_NO_SMEM_IN | bmr.FLAG_NO_SMEM_OUT], ids=["SIO", "G"])
+def test_sm_per_line_output(flags):
+    # f-4: the paper's own StringMatch output (L125: emit the line if found) = oracle "sml"
+    pat = b"a" * 16
+    recs = [b"a" * 1000, b"a" * 15, b"a" * 16, b"", b"b" + b"a" * 40, b"xyz" * 50, b"a" * 20_000, b"a" * 17]
+    rng = np.random.default_rng(3)
+    recs += [bytes(rng.choice(list(b"ab"), size=int(rng.integers(0, 40)), p=[0.9, 0.1]).tolist()) for _ in range(3000)]
+    data, off = make_records(recs)
+    half = len(recs) // 2
+    b = [(data[: int(off[half])], off[: half + 1], half), (data[int(off[half]):], off[half:] - off[half], len(recs) - half)]
+    g, st = gpu("sm", b, pattern=pat, flags=bmr.FLAG_SM_LINES | flags, input_base=5)
+    o = oracle.run("sml", [(data, off, len(recs), 0, 5)], pattern=pat)
+    got, want = decode("sm", g), decode("sm", o)
+    assert np.array_equal(got, want) and len(want) > 5
+    assert st["n_keys"] == len(want) and st["pairs"] >= len(want)
+
+
 def test_sm_input_base_and_multibatch():
     spec = pygen.spec_sm(plant_ppm=50_000)
     g = pygen.host_text(spec, 2, truth=True)
