@@ -373,7 +373,7 @@ def main():
                 job_e.shuffle()
             job_e.group()
             job_e.reduce()
-            r = job_e.fetch()
+            r = job_e.fetch(copy=False)   # the D2H into job-owned pinned memory, no extra host copy
             return r["keys"].nbytes + r["vals"].nbytes + r["key_offsets"].nbytes + r["val_offsets"].nbytes
 
         estep()

@@ -114,10 +114,11 @@ def _ptr(x) -> int:
     raise TypeError(type(x))
 
 
-def _copy(addr, nbytes, dtype=np.uint8):
+def _copy(addr, nbytes, dtype=np.uint8, copy=True):
     if nbytes == 0:
         return np.zeros(0, dtype)
-    return np.frombuffer((C.c_uint8 * nbytes).from_address(addr), np.uint8).copy().view(dtype)
+    a = np.frombuffer((C.c_uint8 * nbytes).from_address(addr), np.uint8)
+    return (a.copy() if copy else a).view(dtype)
 
 
 class Job:
@@ -187,14 +188,16 @@ class Job:
     def reduce(self):
         self._check(lib().mr_reduce(self.h))
 
-    def fetch(self) -> dict:
+    def fetch(self, copy: bool = True) -> dict:
+        """The result (mr_result encoding).  copy=False returns views of the job-owned pinned host
+        buffers (valid until the next call on this job, as in the C ABI)."""
         r = Result()
         self._check(lib().mr_fetch(self.h, C.byref(r)))
         n = int(r.n_keys)
-        ko = _copy(r.key_offsets, 8 * (n + 1), np.uint64)
-        vo = _copy(r.val_offsets, 8 * (n + 1), np.uint64)
-        return {"n_keys": n, "keys": _copy(r.keys, int(ko[-1])), "key_offsets": ko,
-                "vals": _copy(r.vals, int(vo[-1])), "val_offsets": vo}
+        ko = _copy(r.key_offsets, 8 * (n + 1), np.uint64, copy)
+        vo = _copy(r.val_offsets, 8 * (n + 1), np.uint64, copy)
+        return {"n_keys": n, "keys": _copy(r.keys, int(ko[-1]), np.uint8, copy), "key_offsets": ko,
+                "vals": _copy(r.vals, int(vo[-1]), np.uint8, copy), "val_offsets": vo}
 
     def run(self, *batches) -> dict:
         for b in batches:

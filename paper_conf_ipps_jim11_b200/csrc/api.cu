@@ -665,7 +665,10 @@ mr_status mr_job_reset(mr_job* job) {
   return MR_OK;
 }
 
-static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t* offsets, uint64_t n) {
+// known_nbytes: the batch length when the caller knows it (mr_map_host_lines), else ~0 (read
+// offsets[n] back from the device)
+static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t* offsets, uint64_t n,
+                            uint64_t known_nbytes = ~0ULL) {
   if (job->state != kCreated && job->state != kMapped) return fail(job, MR_ERR_STATE, "mr_map after mr_group");
   const bool fixed = job->cfg.record_stride > 0;
   if (fixed != (offsets == nullptr)) return fail(job, MR_ERR_INVALID, "offsets must be NULL iff record_stride > 0");
@@ -675,6 +678,8 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
   uint64_t nbytes = 0;
   if (fixed) {
     nbytes = n * job->cfg.record_stride;
+  } else if (known_nbytes != ~0ULL && !(job->cfg.flags & MR_FLAG_VALIDATE)) {
+    nbytes = known_nbytes;
   } else {
     CK(cudaMemcpyAsync(job->tmp_h.p, offsets + n, sizeof(uint64_t), cudaMemcpyDeviceToHost, job->stream), "read offsets[n]");
     if (job->cfg.flags & MR_FLAG_VALIDATE) {
@@ -821,7 +826,7 @@ mr_status mr_map_host_lines(mr_job* job, const uint8_t* text, uint64_t nbytes) {
       job->tmp_h.p[1] = hi - lo;
       CK(cudaMemcpyAsync(off + n, job->tmp_h.p + 1, 8, cudaMemcpyHostToDevice, job->stream), "offsets[n]");
     }
-    mr_status st = map_common(job, dtext + lo, off, n);
+    mr_status st = map_common(job, dtext + lo, off, n, hi - lo);
     if (st != MR_OK) return st;
   }
   return MR_OK;
