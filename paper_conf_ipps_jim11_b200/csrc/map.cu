@@ -58,16 +58,17 @@ constexpr int kNOut = 4;         // output buffers in the flush ring (generation
 // and 4 x 20 KB output buffers.
 template <int W>
 struct Cfg {
-  // StringMatch (read-bound, almost no output): 6 stages (8 stages with 512 staged offsets each
-  // measured slower on C2: 2.38 against 2.07 ms)
-  static constexpr int kStages = (W == kSM) ? 6 : 4;
-  static constexpr int kOffCap = 1024;   // record offsets staged per tile (more: read from global)
+  // StringMatch (read-bound, almost no output, lazy record directory below: no offsets or bitmap
+  // regions): 8 stages of bytes in flight
+  static constexpr int kStages = (W == kSM) ? 8 : 4;
+  static constexpr int kOffCap = (W == kSM) ? 0 : 1024;   // record offsets staged per tile (more: read from global)
   // StringMatch reads the record directory lazily: record boundaries matter only where the
   // pattern's first byte matches (planted, rare), so no offsets are staged and no bitmap is built;
   // a candidate checks for a record start inside its 16 bytes by a binary search over the tile's
   // offsets slice in global memory.  The producers only issue the byte TMA.
   static constexpr bool kLazyDir = (W == kSM);
-  static constexpr int kOffBytes = ((kOffCap + 2) * 8 + 127) / 128 * 128;
+  static constexpr int kOffBytes = (W == kSM) ? 0 : ((kOffCap + 2) * 8 + 127) / 128 * 128;
+  static constexpr int kBits = (W == kSM) ? 0 : kBitBytes;   // record-start bitmap bytes per stage
   static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? 10240 : 20480;   // bytes per output buffer
   // the producer builds the bitmap of tile it - kLag right after issuing tile it: kLag stages of
   // TMA traffic stay in flight per SM while one stage is being consumed
@@ -141,7 +142,7 @@ struct Layout {
   static constexpr int bytes = 2048;                              // kStages x kStageBytes
   static constexpr int offs = bytes + kStages * kStageBytes;      // kStages x kOffBytes
   static constexpr int bits = offs + kStages * Cfg<W>::kOffBytes; // kStages x kBitBytes
-  static constexpr int out = bits + kStages * kBitBytes;          // kNOut x Cfg<W>::kOutHalf
+  static constexpr int out = bits + kStages * Cfg<W>::kBits;      // kNOut x Cfg<W>::kOutHalf
   static constexpr int hq = out + kNOut * Cfg<W>::kOutHalf;       // nmap x kHashQ x 8 (WC)
   static constexpr int xq = hq + nmap<W>() * Cfg<W>::kHashQ * 8;  // nmap x kXQ x 4 (WC)
   static constexpr int comb = xq + nmap<W>() * Cfg<W>::kXQ * 4;   // kCombSlots x 8 (WC)
@@ -669,7 +670,7 @@ __device__ void finish_stage(const Params& P, uint8_t* smem, uint32_t it) {
   uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout<W>::ready);
   mbar_wait(&full[s], ph);
   const StageHdr* hd = reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
-  uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout<W>::bits + s * kBitBytes);
+  uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits);
   const uint64_t* soff =
       reinterpret_cast<const uint64_t*>(smem + Layout<W>::offs + s * Cfg<W>::kOffBytes + hd->off_shift);
   const uint64_t ra = hd->ra, cnt = hd->rb - hd->ra;
@@ -743,8 +744,8 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
         if (!P.so) stage_copy_edges(d, g, static_cast<uint64_t>(max(0LL, stg_hi - w_lo)), lane, b_off, b_len);
         // clear the record-start bitmap (map warps set bits after the full barrier)
         if constexpr (!Cfg<W>::kLazyDir) {
-          uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout<W>::bits + s * kBitBytes);
-          for (uint32_t i = lane; i < kBitBytes / 16; i += 32) reinterpret_cast<uint4*>(bm)[i] = make_uint4(0, 0, 0, 0);
+          uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits);
+          for (uint32_t i = lane; i < Cfg<W>::kBits / 16; i += 32) reinterpret_cast<uint4*>(bm)[i] = make_uint4(0, 0, 0, 0);
         }
         // offsets slice offsets[ra..rb) (record starts in the staged window)
         const uint64_t cnt = rb - ra;
@@ -1022,10 +1023,20 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
   } else if constexpr (W == kSM) {
     if (live) {
       const uint32_t b0 = (P.pat[0] & 0xFFu) * 0x01010101u;
-      uint32_t cand = 0;
+      // any byte equal to the pattern's first byte?  (exact has-zero-byte test on x ^ b0: the
+      // first byte is rare in text, so the per-byte mask is computed only when one exists)
+      uint32_t any = 0;
 #pragma unroll
-      for (int i = 0; i < 4; ++i) cand |= eq_mask4(x[i], b0) << (4 * i);
-      cand &= vm & 0xFFFFu;
+      for (int i = 0; i < 4; ++i) {
+        const uint32_t t = x[i] ^ b0;
+        any |= (t - 0x01010101u) & ~t & 0x80808080u;
+      }
+      uint32_t cand = 0;
+      if (any) {
+#pragma unroll
+        for (int i = 0; i < 4; ++i) cand |= eq_mask4(x[i], b0) << (4 * i);
+        cand &= vm & 0xFFFFu;
+      }
       while (cand) {
         const uint32_t j = __ffs(cand) - 1;
         cand &= cand - 1;
@@ -1326,7 +1337,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         commit(oc, slot, total);
       }
     } else {
-      const uint32_t* bm = reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * kBitBytes);
+      const uint32_t* bm = reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits);
       // (SO: an empty stage makes every helper read global memory)
       TileView tv{sb, bm, hd.sbase, P.so ? hd.sbase : hd.stg_hi, hd.ra, hd.rb};
       const long long wp = hd.chunk0 + static_cast<long long>(w) * kWin;
