@@ -712,6 +712,12 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
       const uint64_t t = blockIdx.x + static_cast<uint64_t>(it) * G;
       const uint64_t ra = __shfl_sync(kFull, my_ra, j), rb = __shfl_sync(kFull, my_rb, j);
       const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
+      // release the bitmap of tile it - kLag (its bytes have landed) BEFORE blocking on a free
+      // stage: that wait lasts until the oldest tile's last window is done, and the map warps
+      // need the next tile meanwhile
+      if constexpr (W != kKM && !Cfg<W>::kLazyDir) {
+        if (it >= static_cast<uint32_t>(Cfg<W>::kLag)) finish_stage<W>(P, smem, it - Cfg<W>::kLag);   // same owner
+      }
       helper_wait(P, &empty[s], ph ^ 1u, 128);
       StageHdr* hd = reinterpret_cast<StageHdr*>(smem + Layout<W>::hdr + s * 128);
       uint8_t* sb = smem + Layout<W>::bytes + s * kStageBytes;
@@ -801,9 +807,7 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
                                                         reinterpret_cast<const uint8_t*>(P.off + rbf));
           }
         }
-        if constexpr (!Cfg<W>::kLazyDir) {
-          if (it >= Cfg<W>::kLag) finish_stage<W>(P, smem, it - Cfg<W>::kLag);   // same owner (kLag % kNProd == 0)
-        }
+
       }
     }
   }

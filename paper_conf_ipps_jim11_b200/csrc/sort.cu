@@ -427,7 +427,10 @@ static const int kIPT32[4] = {24, 32, 16, 24};
 int sort_tile() { return kSortThreads * (sort_cfg() == 1 ? 12 : 16); }
 int sort_tile_keys() { return kSortThreads * (sort_cfg() == 1 ? 24 : 16); }
 int sort_variant32();
-int sort_tile_keys32() { return kSortThreads * (sort_variant32() == 19 ? 16 : kIPT32[sort_cfg()]); }
+int sort_tile_keys32() {
+  const int v = sort_variant32();
+  return kSortThreads * (v == 19 || v == 21 ? 16 : v == 20 ? 20 : kIPT32[sort_cfg()]);
+}
 
 template <typename K, bool kFirst, int kVar, int IPT, int MINB, bool kPay, int LW = 4>
 static void launch_os(unsigned tiles, const K* keys_in, const uint32_t* idx_in, K* keys_out, uint32_t* idx_out,
@@ -480,6 +483,8 @@ static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* ke
         case 3: launch_os<K, false, 3, 24, 3, false>(BMR_OS_ARGS); break;
         case 18: launch_os<K, false, 18, 24, 3, false>(BMR_OS_ARGS); break;
         case 19: launch_os<K, false, 18, 16, 3, false>(BMR_OS_ARGS); break;
+        case 20: launch_os<K, false, 2, 20, 3, false>(BMR_OS_ARGS); break;
+        case 21: launch_os<K, false, 2, 16, 3, false>(BMR_OS_ARGS); break;
         default: launch_os<K, false, 2, 24, 3, false>(BMR_OS_ARGS); break;
       }
     }
