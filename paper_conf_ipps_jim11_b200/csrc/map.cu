@@ -50,6 +50,7 @@ constexpr int kHalo = 256;       // bytes staged after the tile (words / matches
 constexpr int kWin = 512;        // bytes per warp window = 32 lanes x 16 B
 constexpr int kNWin = kT / kWin;
 constexpr int kStageBytes = 16768;             // >= kLead + kT + kHalo + 32, multiple of 128
+static_assert(kStageBytes <= (1 << 15), "WC long-word queue entries hold a 15-bit stage offset");
 constexpr int kBitWords = kStageBytes / 32 + 4;
 constexpr int kBitBytes = 2176;                // >= kBitWords * 4, multiple of 128
 constexpr int kNOut = 4;         // output buffers in the flush ring (generation g uses buffer g % kNOut)
@@ -69,7 +70,7 @@ struct Cfg {
   static constexpr bool kLazyDir = (W == kSM);
   static constexpr int kOffBytes = (W == kSM) ? 0 : ((kOffCap + 2) * 8 + 127) / 128 * 128;
   static constexpr int kBits = (W == kSM) ? 0 : kBitBytes;   // record-start bitmap bytes per stage
-  static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? 10240 : 20480;   // bytes per output buffer
+  static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? 12288 : 20480;   // bytes per output buffer
   // the producer builds the bitmap of tile it - kLag right after issuing tile it: kLag stages of
   // TMA traffic stay in flight per SM while one stage is being consumed
   static constexpr int kLag = kStages - 2;
@@ -143,8 +144,8 @@ struct Layout {
   static constexpr int offs = bytes + kStages * kStageBytes;      // kStages x kOffBytes
   static constexpr int bits = offs + kStages * Cfg<W>::kOffBytes; // kStages x kBitBytes
   static constexpr int out = bits + kStages * Cfg<W>::kBits;      // kNOut x Cfg<W>::kOutHalf
-  static constexpr int hq = out + kNOut * Cfg<W>::kOutHalf;       // nmap x kHashQ x 8 (WC)
-  static constexpr int xq = hq + nmap<W>() * Cfg<W>::kHashQ * 8;  // nmap x kXQ x 4 (WC)
+  static constexpr int hq = out + kNOut * Cfg<W>::kOutHalf;       // nmap x kHashQ x 4 (WC)
+  static constexpr int xq = hq + nmap<W>() * Cfg<W>::kHashQ * 4;  // nmap x kXQ x 4 (WC)
   static constexpr int comb = xq + nmap<W>() * Cfg<W>::kXQ * 4;   // kCombSlots x 8 (WC)
   static constexpr int cent = comb + Cfg<W>::kCombSlots * 8;      // KM centroids
   static_assert(ready + kStages * 8 <= bytes, "header region overflow");
@@ -864,7 +865,7 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
   if (slow_bit && len_slow > kWcExact) longm |= slow_bit;
   (void)longm;
   if (__all_sync(kFull, emit_mask == 0)) return;
-  uint64_t* hq = reinterpret_cast<uint64_t*>(outh + (Layout<kWC>::hq - Layout<kWC>::out)) +
+  uint32_t* hq = reinterpret_cast<uint32_t*>(outh + (Layout<kWC>::hq - Layout<kWC>::out)) +
                  (threadIdx.x >> 5) * Cfg<kWC>::kHashQ;
   uint32_t* xq = reinterpret_cast<uint32_t*>(outh + (Layout<kWC>::xq - Layout<kWC>::out)) +
                  (threadIdx.x >> 5) * Cfg<kWC>::kXQ;
@@ -891,7 +892,8 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
       xq[nx + __popc(ma & lanemask_lt())] = key;
     } else if (act && len > kWcExact) {
       if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
-      hq[nq + __popc(mb & lanemask_lt())] = static_cast<uint64_t>(p0 + j - tv.sbase) | (static_cast<uint64_t>(len) << 24);
+      // u32 queue entry: stage offset (< 2^15) | length << 15 (<= 0xFFFF)
+      hq[nq + __popc(mb & lanemask_lt())] = static_cast<uint32_t>(p0 + j - tv.sbase) | (len << 15);
     }
     nx += __popc(ma);
     nq += __popc(mb);
@@ -909,9 +911,9 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
       const bool in = q < nq;
       ulonglong2 ent = make_ulonglong2(0ULL, 0ULL);
       if (in) {
-        const uint64_t e = hq[q];
-        const long long p = tv.sbase + static_cast<long long>(e & 0xFFFFFF);
-        const uint32_t len = static_cast<uint32_t>(e >> 24);
+        const uint32_t e = hq[q];
+        const long long p = tv.sbase + static_cast<long long>(e & 0x7FFFu);
+        const uint32_t len = e >> 15;
         ent = len <= kMidMax ? make_ulonglong2(exact_key(bytes8_at(P, tv, p, len), len), 0ULL)
                              : make_ulonglong2(key_at(P, tv, p, len), (reinterpret_cast<uint64_t>(P.rec + p) << 16) | len);
       }
@@ -943,9 +945,9 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
   for (uint32_t i = lane; i < nx; i += 32) sh[ka + i] = xq[i];
   __syncwarp();
   for (uint32_t q = lane; q < nq; q += 32) {           // lane-parallel keys of the long words
-    const uint64_t e = hq[q];
-    const long long p = tv.sbase + static_cast<long long>(e & 0xFFFFFF);
-    const uint32_t len = static_cast<uint32_t>(e >> 24);
+    const uint32_t e = hq[q];
+    const long long p = tv.sbase + static_cast<long long>(e & 0x7FFFu);
+    const uint32_t len = e >> 15;
     ulonglong2 ent;
     if (len <= kMidMax) {                                // mid stream: exact 48-bit key, no kref
       ent = make_ulonglong2(exact_key(bytes8_at(P, tv, p, len), len), 0ULL);

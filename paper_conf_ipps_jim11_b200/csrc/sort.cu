@@ -429,7 +429,7 @@ int sort_tile_keys() { return kSortThreads * (sort_cfg() == 1 ? 24 : 16); }
 int sort_variant32();
 int sort_tile_keys32() {
   const int v = sort_variant32();
-  return kSortThreads * (v == 19 || v == 21 ? 16 : v == 20 ? 20 : kIPT32[sort_cfg()]);
+  return kSortThreads * (v == 19 || v == 21 || v == 22 ? 16 : v == 20 ? 20 : kIPT32[sort_cfg()]);
 }
 
 template <typename K, bool kFirst, int kVar, int IPT, int MINB, bool kPay, int LW = 4>
@@ -485,6 +485,8 @@ static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* ke
         case 19: launch_os<K, false, 18, 16, 3, false>(BMR_OS_ARGS); break;
         case 20: launch_os<K, false, 2, 20, 3, false>(BMR_OS_ARGS); break;
         case 21: launch_os<K, false, 2, 16, 3, false>(BMR_OS_ARGS); break;
+        case 22: launch_os<K, false, 2, 16, 3, false, 8>(BMR_OS_ARGS); break;
+        case 23: launch_os<K, false, 2, 24, 3, false, 8>(BMR_OS_ARGS); break;
         default: launch_os<K, false, 2, 24, 3, false>(BMR_OS_ARGS); break;
       }
     }
