@@ -82,7 +82,8 @@ bool has_kref(int workload);
 uint64_t map_tiles(const MapArgs& a);        // number of tiles of a batch
 uint32_t map_prefetch();
 uint32_t map_wait_hint();
-uint32_t map_dyn_windows(int workload);                     // L2 prefetch distance of the Map producers (BMR_MAP_PF)
+uint32_t map_dyn_windows(int workload);
+uint32_t map_wc_balanced();                     // L2 prefetch distance of the Map producers (BMR_MAP_PF)
 cudaError_t launch_map(const MapArgs& a, int num_sms, cudaStream_t s);
 
 // ---- group-by-key (hash radix sort + segment boundaries) ----

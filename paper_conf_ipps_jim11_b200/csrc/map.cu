@@ -216,6 +216,7 @@ struct Params {
   // atomic per warp, L135 / L171-173); both = the paper's G mode
   uint32_t so, si;
   uint32_t sm_lines;       // StringMatch: emit the matching record's start (MR_FLAG_SM_LINES)
+  uint32_t wc_bal;         // WordCount: balanced two-phase emission (BMR_WC_BAL, default on)
 };
 
 // Idle wait of a role warp on an mbarrier phase (map warps on a staged tile, producers on a free
@@ -871,6 +872,50 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
                  (threadIdx.x >> 5) * Cfg<kWC>::kXQ;
   uint32_t* ctab = reinterpret_cast<uint32_t*>(outh + (Layout<kWC>::comb - Layout<kWC>::out));
   uint32_t nx = 0, nq = 0;
+  if (P.wc_bal && !P.so) {
+    // Balanced emission.  Phase 1: each lane writes a descriptor (stage offset | length << 15)
+    // of every word it starts at the word's warp rank (cheap divergent loop); phase 2: the warp
+    // processes the descriptors 32 at a time (rounds = words / 32 instead of the busiest lane's
+    // word count), reading the word bytes from the stage.  Phase 2 compacts the exact keys that
+    // miss the combiner into the same queue (its writes stay below the round being read).
+    const uint32_t cnt = __popc(emit_mask);
+    const uint32_t incl = warp_inclusive_add(cnt);
+    const uint32_t W = __shfl_sync(kFull, incl, 31);
+    if (W == 0) return;
+    uint32_t k = incl - cnt;
+    const uint32_t i0 = static_cast<uint32_t>(p0 - tv.sbase);
+    for (uint32_t m = emit_mask; m; m &= m - 1) {
+      const uint32_t j = __ffs(m) - 1;
+      const uint32_t rest = nb >> (j + 1);
+      uint32_t len = rest ? static_cast<uint32_t>(__ffs(rest)) : len_slow;
+      if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
+      xq[k++] = (i0 + j) | (len << 15);
+    }
+    __syncwarp();
+    for (uint32_t b = 0; b < W; b += 32) {
+      const bool act = b + lane < W;
+      const uint32_t d = act ? xq[b + lane] : 0u;
+      __syncwarp();                            // this round's reads before the compacting writes
+      const uint32_t len = d >> 15, pos = d & 0x7FFFu;
+      bool ex = act && len <= kWcExact;
+      uint32_t key = 0;
+      if (ex) {   // the <= 5 word bytes from the stage: two aligned words cover [pos, pos + 5)
+        const uint32_t a = pos & ~3u, sh = (pos & 3u) * 8;
+        const uint32_t w0 = *reinterpret_cast<const uint32_t*>(tv.sb + a);
+        const uint32_t w1 = *reinterpret_cast<const uint32_t*>(tv.sb + a + 4);
+        const uint64_t bts = static_cast<uint64_t>(__funnelshift_r(w0, w1, sh)) | (static_cast<uint64_t>(w1 >> sh) << 32);
+        key = exact_key30(bts, len);
+        if (P.comb && comb_add(ctab, key)) ex = false;   // absorbed by the combiner
+      }
+      const bool lg = act && len > kWcExact;
+      const uint32_t ma = __ballot_sync(kFull, ex), mb = __ballot_sync(kFull, lg);
+      if (ex) xq[nx + __popc(ma & lanemask_lt())] = key;
+      else if (lg) hq[nq + __popc(mb & lanemask_lt())] = d;
+      nx += __popc(ma);
+      nq += __popc(mb);
+      __syncwarp();
+    }
+  } else {
   uint32_t m_left = emit_mask;
   while (__any_sync(kFull, m_left != 0)) {
     const bool act = m_left != 0;
@@ -897,6 +942,7 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
     }
     nx += __popc(ma);
     nq += __popc(mb);
+  }
   }
   if (nx + nq == 0) return;
   if (P.si) {   // SI / G ablation: append straight to the three global streams, one atomic each
@@ -1514,6 +1560,7 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.so = (a.flags & 1u) ? 1u : 0u;   // MR_FLAG_NO_SMEM_IN
   P.si = (a.flags & 2u) ? 1u : 0u;   // MR_FLAG_NO_SMEM_OUT
   P.sm_lines = (W == kSM && (a.flags & 0x200u)) ? 1u : 0u;   // MR_FLAG_SM_LINES
+  P.wc_bal = map_wc_balanced();
   if (P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>((P.ntiles + 255) / 256);
@@ -1560,6 +1607,15 @@ uint32_t map_dyn_windows(int w) {
     return e ? atoi(e) : -1;
   }();
   return v >= 0 ? static_cast<uint32_t>(v) : (w == kSM ? 0u : 1u);
+}
+
+// WordCount emission: balanced two-phase rounds (BMR_WC_BAL=1, default) or lane-serial rounds (0)
+uint32_t map_wc_balanced() {
+  static uint32_t v = [] {
+    const char* e = getenv("BMR_WC_BAL");
+    return e ? static_cast<uint32_t>(atoi(e)) : 1u;
+  }();
+  return v;
 }
 
 int vbytes_of(int w) { return w == kKM ? 32 : w == kII ? 8 : 0; }
