@@ -16,7 +16,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libbmr.so")
+LIB_PATH = os.environ.get("BMR_LIB") or os.path.join(_HERE, "libbmr.so")   # BMR_LIB: variant builds (sweeps)
 
 MR_ABI_VERSION = 1
 WORDCOUNT, STRINGMATCH, KMEANS, INVINDEX = 1, 2, 3, 4

@@ -80,7 +80,7 @@ struct MapArgs {
 int vbytes_of(int workload);                 // value bytes per pair (WC Map output: none, value 1)
 bool has_kref(int workload);
 uint64_t map_tiles(const MapArgs& a);        // number of tiles of a batch
-uint32_t map_prefetch();
+uint32_t map_prefetch(int w);
 uint32_t map_wait_hint();
 uint32_t map_dyn_windows(int workload);
 uint32_t map_wc_balanced();                     // L2 prefetch distance of the Map producers (BMR_MAP_PF)

@@ -57,11 +57,14 @@ constexpr int kNOut = 4;         // output buffers in the flush ring (generation
 // Per-workload SMEM budget: StringMatch is read-bound with almost no output -> more input stages
 // (more bytes in flight per SM) and small output buffers; the emitting workloads keep 4 stages
 // and 4 x 20 KB output buffers.
+#ifndef BMR_SM_STAGES
+#define BMR_SM_STAGES 12   // StringMatch stages in flight per SM (12 x 16.4 KiB)
+#endif
 template <int W>
 struct Cfg {
   // StringMatch (read-bound, almost no output, lazy record directory below: no offsets or bitmap
   // regions): 8 stages of bytes in flight
-  static constexpr int kStages = (W == kSM) ? 8 : 4;
+  static constexpr int kStages = (W == kSM) ? BMR_SM_STAGES : 4;
   static constexpr int kOffCap = (W == kSM) ? 0 : 1024;   // record offsets staged per tile (more: read from global)
   // StringMatch reads the record directory lazily: record boundaries matter only where the
   // pattern's first byte matches (planted, rare), so no offsets are staged and no bitmap is built;
@@ -140,7 +143,7 @@ struct Layout {
   static constexpr int full = hdr + kStages * 128;                // kStages x 8
   static constexpr int empty = full + kStages * 8;
   static constexpr int ready = empty + kStages * 8;               // kStages x 8 (text: bitmap built)
-  static constexpr int bytes = 2048;                              // kStages x kStageBytes
+  static constexpr int bytes = (ready + kStages * 8 <= 2048) ? 2048 : (ready + kStages * 8 + 127) / 128 * 128;   // kStages x kStageBytes
   static constexpr int offs = bytes + kStages * kStageBytes;      // kStages x kOffBytes
   static constexpr int bits = offs + kStages * Cfg<W>::kOffBytes; // kStages x kBitBytes
   static constexpr int out = bits + kStages * Cfg<W>::kBits;      // kNOut x Cfg<W>::kOutHalf
@@ -148,7 +151,6 @@ struct Layout {
   static constexpr int xq = hq + nmap<W>() * Cfg<W>::kHashQ * 4;  // nmap x kXQ x 4 (WC)
   static constexpr int comb = xq + nmap<W>() * Cfg<W>::kXQ * 4;   // kCombSlots x 8 (WC)
   static constexpr int cent = comb + Cfg<W>::kCombSlots * 8;      // KM centroids
-  static_assert(ready + kStages * 8 <= bytes, "header region overflow");
   static_assert(sizeof(OutCtl) <= hdr, "OutCtl overlaps the stage headers");
 };
 static_assert(64 % kNOut == 0, "6-bit generation counter must wrap on a buffer boundary");
@@ -1235,6 +1237,72 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
   if (!P.si) commit(oc, slot, total);
 }
 
+// StringMatch map warps (default SIO, static order): super-windows of kSmSub 512-B windows.  The
+// pattern's first byte is rare in text, so each lane first runs the exact has-byte test over its
+// kSmSub 16-B chunks (one LDS.128 + 3 ALU ops per 4 bytes); only a 512-B window in which some
+// lane saw the byte runs the full per-byte path (emit_text_chunk: candidate mask, 16-byte
+// compare, record check, emission).  The per-window bookkeeping (window index, stage header,
+// range masks, the warp reduction of the emission count) is paid once per 2 KiB instead of per
+// 512 B (ncu, C2 round 1: it was ~80% of the Map's instructions).
+constexpr int kSmSub = 4, kNSup = kNWin / kSmSub;
+__device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
+  constexpr int W = kSM;
+  constexpr int kStages = Cfg<W>::kStages;
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
+  uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
+  uint8_t* outh = smem + Layout<W>::out;
+  const uint32_t b0 = (P.pat[0] & 0xFFu) * 0x01010101u;
+  const long long N = static_cast<long long>(P.nbytes);
+  // this CTA's iterations (as producer_loop): a warp's super-windows are nmap apart and may skip
+  // whole tiles (kNSup < nmap), so it must stop at T itself rather than wait for the end marker
+  const uint64_t G = gridDim.x;
+  const uint32_t T = blockIdx.x < P.ntiles ? static_cast<uint32_t>((P.ntiles - blockIdx.x + G - 1) / G) : 0u;
+  uint32_t have_it = ~0u;
+  StageHdr hd{};
+  for (uint32_t kseq = 0;; ++kseq) {
+    const uint32_t g = warp + kseq * static_cast<uint32_t>(nmap<W>());
+    const uint32_t it = g / kNSup, sw = g % kNSup;
+    if (it >= T) break;
+    const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
+    if (it != have_it) {
+      mbar_wait(&full[s], ph);
+      hd = *reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
+      have_it = it;
+    }
+    if (hd.t < 0) break;
+    const uint8_t* sb = smem + Layout<W>::bytes + s * kStageBytes;
+    const long long wp0 = hd.chunk0 + static_cast<long long>(sw) * (kSmSub * kWin);
+    // has-byte test (exact: (t - 0x01..) & ~t & 0x80.. is non-zero iff t has a zero byte); bytes
+    // outside [0, N) only cause a spurious slow-path visit, which masks them exactly
+    uint32_t anym = 0;
+    const uint8_t* c0 = sb + (wp0 - hd.sbase) + lane * 16;
+#pragma unroll
+    for (int k = 0; k < kSmSub; ++k) {
+      const uint4 c = *reinterpret_cast<const uint4*>(c0 + k * kWin);
+      const uint32_t t0 = c.x ^ b0, t1 = c.y ^ b0, t2 = c.z ^ b0, t3 = c.w ^ b0;
+      const uint32_t a = ((t0 - 0x01010101u) & ~t0) | ((t1 - 0x01010101u) & ~t1) | ((t2 - 0x01010101u) & ~t2) |
+                         ((t3 - 0x01010101u) & ~t3);
+      anym |= ((a & 0x80808080u) ? 1u : 0u) << k;
+    }
+    uint32_t need = 0;
+#pragma unroll
+    for (int k = 0; k < kSmSub; ++k) need |= (__any_sync(kFull, (anym >> k) & 1u) ? 1u : 0u) << k;
+    while (need) {                                     // warp-uniform
+      const int k = __ffs(need) - 1;
+      need &= need - 1;
+      const long long wp = wp0 + static_cast<long long>(k) * kWin;
+      if (wp >= hd.hi) break;
+      TileView tv{sb, nullptr, hd.sbase, hd.stg_hi, hd.ra, hd.rb};
+      const long long p0 = wp + lane * 16;
+      const bool live = (p0 + 16 > 0) && (p0 < N);
+      emit_text_chunk<W>(P, oc, outh, tv, p0, p0 - hd.sbase, live);
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive_cnt(&empty[s], kSmSub);
+  }
+}
+
 template <int W>
 __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   constexpr int kStages = Cfg<W>::kStages;
@@ -1262,7 +1330,11 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   // window sequence)
   uint32_t kseq = 0, have_it = ~0u;
   StageHdr hd{};
-  for (uint32_t it = 0;; ++it) {
+  const bool sm_fast = W == kSM && !P.so && !P.dyn;
+  if constexpr (W == kSM) {
+    if (sm_fast) sm_fast_loop(P, smem, oc);
+  }
+  for (uint32_t it = 0; !sm_fast; ++it) {
     uint32_t w = 0;
     if constexpr (W != kKM) {
       uint32_t g = 0;
@@ -1554,7 +1626,7 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.comb = (W == kWC && a.out.hp != nullptr) || (W == kKM && a.out.km_sums != nullptr && a.k <= kKmCombMax) ? 1u : 0u;
   P.km_sums = a.out.km_sums;
   P.km_cnts = a.out.km_cnts;
-  P.pf = map_prefetch();
+  P.pf = map_prefetch(W);
   P.wait_hint = map_wait_hint();
   P.dyn = map_dyn_windows(W);
   P.so = (a.flags & 1u) ? 1u : 0u;   // MR_FLAG_NO_SMEM_IN
@@ -1581,12 +1653,14 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
 
 // L2 prefetch distance of the Map producers (BMR_MAP_PF, tiles; default 0 = off: measured slower
 // on C2/C4 in round 1 with 2 producers)
-uint32_t map_prefetch() {
-  static uint32_t v = [] {
+// L2 prefetch distance of the producers in tiles (BMR_MAP_PF; default: 2 for StringMatch, whose
+// Map is a pure read stream -- C2 0.467 -> 0.495 of HBM, round 1 sweep -- else off)
+uint32_t map_prefetch(int w) {
+  static int v = [] {
     const char* e = getenv("BMR_MAP_PF");
-    return e ? static_cast<uint32_t>(atoi(e)) : 0u;
+    return e ? atoi(e) : -1;
   }();
-  return v;
+  return v >= 0 ? static_cast<uint32_t>(v) : (w == kSM ? 2u : 0u);
 }
 
 // idle-wait flavour of the Map role warps (BMR_MAP_WAIT: 0 = plain try_wait, 1 = suspend-time

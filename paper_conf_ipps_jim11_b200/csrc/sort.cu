@@ -97,6 +97,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
   constexpr int kSortTile = Smem::kTile;
   constexpr bool kAtomicRank = (kVar & 1) != 0, kEarly = (kVar & 2) != 0;
   constexpr bool kBackoff = (kVar & 4) != 0, kMatchHist = (kVar & 8) != 0, kBallotPeers = (kVar & 16) != 0;
+  constexpr bool kBallotAll = (kVar & 32) != 0;
   static_assert(kDPT >= 1 && kDPT * kSortThreads == kBins, "bins must be a multiple of the block size");
   extern __shared__ __align__(16) uint8_t raw[];
   Smem& S = *reinterpret_cast<Smem*>(raw);
@@ -120,6 +121,44 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
 #pragma unroll
   for (int q = 0; q < kDPT; ++q) tcount[q] = 0;
   uint64_t* my = status + static_cast<uint64_t>(tile) * kBins + d0;
+  if constexpr (kBallotAll) {
+    // kVar bit 5: peer masks from kBits ballots per key (no match.any: ncu C5 round 1 put 48% of
+    // the stall samples on the instruction consuming the MATCH result).  Per key group (equal
+    // digits in the warp) the highest lane issues one shared atomic for the tile histogram and
+    // one for the warp's digit counter; a warp's atomics to one counter are applied in issue
+    // order (j order), so ranks stay stable.  The tile histogram is published right after.
+#pragma unroll
+    for (int j0 = 0; j0 < kSortIPT; j0 += 8) {
+      uint32_t peers[8];
+#pragma unroll
+      for (int j = j0; j < j0 + 8 && j < kSortIPT; ++j) {
+        const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & kMask;
+        uint32_t pm = 0xffffffffu;
+#pragma unroll
+        for (int b = 0; b < kBits; ++b) {
+          const uint32_t bal = __ballot_sync(0xffffffffu, (dj >> b) & 1u);
+          pm &= ((dj >> b) & 1u) ? bal : ~bal;
+        }
+        peers[j - j0] = pm;
+        rank[j] = 0;
+        if (lane == 31u - __clz(pm)) {
+          if constexpr (kEarly) atomicAdd(&S.hist[dj], __popc(pm));
+          rank[j] = atomicAdd(&S.wcnt[warp][dj], __popc(pm));
+        }
+      }
+#pragma unroll
+      for (int j = j0; j < j0 + 8 && j < kSortIPT; ++j)
+        rank[j] = __shfl_sync(0xffffffffu, rank[j], 31 - __clz(peers[j - j0])) + __popc(peers[j - j0] & lanemask_lt());
+    }
+    if constexpr (kEarly) {
+      __syncthreads();
+#pragma unroll
+      for (int q = 0; q < kDPT; ++q) {
+        tcount[q] = S.hist[d0 + q];
+        st_relaxed_gpu_u64(my + q, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount[q]));
+      }
+    }
+  } else {
   if constexpr (kEarly) {
     // 1. tile histogram first, published immediately (early aggregate for the successors)
     if constexpr (kMatchHist) {   // one shared atomic per group of equal digits in the warp
@@ -184,6 +223,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
       rank[j] = before + __popc(peers & lanemask_lt());
     }
   }
+  }   // !kBallotAll
   __syncthreads();
   if constexpr (!kEarly) {
 #pragma unroll
@@ -286,6 +326,26 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
   __syncthreads();
   // 6. contiguous per-digit runs to global memory
   const uint32_t nvalid = static_cast<uint32_t>(min(static_cast<uint64_t>(kSortTile), m - tbase));
+  if (nvalid == static_cast<uint32_t>(kSortTile)) {
+    // full tile: unrolled in groups of 8, so the SMEM reads of 8 elements are in flight together
+    // (a rolled loop serialises LDS key -> LDS goff -> STG per element)
+#pragma unroll
+    for (int j0 = 0; j0 < kSortIPT; j0 += 8) {
+      K kk[8];
+      uint32_t pp[8];
+#pragma unroll
+      for (int j = 0; j < 8 && j0 + j < kSortIPT; ++j) kk[j] = S.keys[(j0 + j) * kSortThreads + tid];
+#pragma unroll
+      for (int j = 0; j < 8 && j0 + j < kSortIPT; ++j)
+        pp[j] = S.goff[static_cast<uint32_t>(kk[j] >> shift) & kMask] + (j0 + j) * kSortThreads + tid;
+#pragma unroll
+      for (int j = 0; j < 8 && j0 + j < kSortIPT; ++j) {
+        keys_out[pp[j]] = kk[j];
+        if constexpr (kPay) idx_out[pp[j]] = S.idx[(j0 + j) * kSortThreads + tid];
+      }
+    }
+    return;
+  }
   for (uint32_t i = tid; i < nvalid; i += kSortThreads) {
     const K k = S.keys[i];
     const uint32_t dk = static_cast<uint32_t>(k >> shift) & kMask;
@@ -429,7 +489,8 @@ int sort_tile_keys() { return kSortThreads * (sort_cfg() == 1 ? 24 : 16); }
 int sort_variant32();
 int sort_tile_keys32() {
   const int v = sort_variant32();
-  return kSortThreads * (v == 19 || v == 21 || v == 22 ? 16 : v == 20 ? 20 : kIPT32[sort_cfg()]);
+  return kSortThreads * (v == 19 || v == 21 || v == 22 || v == 35 || v == 36 ? 16 : v == 20 ? 20 : v == 37 ? 32
+                                                                                          : kIPT32[sort_cfg()]);
 }
 
 template <typename K, bool kFirst, int kVar, int IPT, int MINB, bool kPay, int LW = 4>
@@ -487,6 +548,14 @@ static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* ke
         case 21: launch_os<K, false, 2, 16, 3, false>(BMR_OS_ARGS); break;
         case 22: launch_os<K, false, 2, 16, 3, false, 8>(BMR_OS_ARGS); break;
         case 23: launch_os<K, false, 2, 24, 3, false, 8>(BMR_OS_ARGS); break;
+        case 34: launch_os<K, false, 34, 24, 3, false>(BMR_OS_ARGS); break;   // ballot peers, early hist, leader atomics
+        case 35: launch_os<K, false, 34, 16, 3, false>(BMR_OS_ARGS); break;
+        case 36: launch_os<K, false, 34, 16, 4, false>(BMR_OS_ARGS); break;
+        case 37: launch_os<K, false, 34, 32, 2, false>(BMR_OS_ARGS); break;
+        case 38: launch_os<K, false, 34, 24, 3, false, 8>(BMR_OS_ARGS); break;    // look-back windows 8 / 16 / 32
+        case 39: launch_os<K, false, 34, 24, 3, false, 16>(BMR_OS_ARGS); break;
+        case 40: launch_os<K, false, 34, 24, 3, false, 32>(BMR_OS_ARGS); break;
+        case 41: launch_os<K, false, 2, 24, 3, false, 16>(BMR_OS_ARGS); break;
         default: launch_os<K, false, 2, 24, 3, false>(BMR_OS_ARGS); break;
       }
     }

@@ -1,0 +1,16 @@
+#!/bin/bash
+# Build a libbmr variant with extra -D flags into variants/libbmr_<name>.so (sweeps: BMR_LIB=...).
+# usage: tools/build_variant.sh NAME "-DFOO=1 -DBAR=2"
+set -e
+name=$1; defs=$2
+mkdir -p build/var_$name variants
+NVFLAGS="-O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -lineinfo -Xcompiler -fPIC --expt-relaxed-constexpr -ftz=false -prec-div=true -prec-sqrt=true"
+objs=""
+for f in paper_conf_ipps_jim11_b200/csrc/*.cu; do
+  b=$(basename $f .cu)
+  nvcc $NVFLAGS $defs -Iinclude -c -o build/var_$name/$b.o $f &
+  objs="$objs build/var_$name/$b.o"
+done
+wait
+nvcc -gencode arch=compute_100a,code=sm_100a -shared --cudart static -o variants/libbmr_$name.so $objs
+echo variants/libbmr_$name.so
