@@ -34,9 +34,18 @@ namespace {
 // Map warps per CTA: KMeans 16 (one 32-point slice each of a 512-point tile); the text workloads
 // 24 (their Map is issue-bound on dependent integer chains: more warps per scheduler hide them)
 constexpr int kNMap = 16;
+#ifndef BMR_SM_NMAP
+#define BMR_SM_NMAP 24   // StringMatch map warps
+#endif
+#ifndef BMR_SM_WAIT_NS
+#define BMR_SM_WAIT_NS 1000   // StringMatch map warps: suspend-time hint of the stage wait (0: spin)
+#endif
+#ifndef BMR_SM_SUB
+#define BMR_SM_SUB 4     // StringMatch 512-B windows per map-warp super-window
+#endif
 constexpr int kNMapText = 24;
 template <int W>
-constexpr int nmap() { return W == 3 ? kNMap : kNMapText; }
+constexpr int nmap() { return W == 3 ? kNMap : W == 2 ? BMR_SM_NMAP : kNMapText; }
 // Producer warps kProdWarp0 .. + kNProd - 1: producer p owns the iterations it == p (mod kNProd)
 // (and so the stages s == p (mod kNProd)); one warp alone is latency-bound at ~465 instructions
 // per tile (TMA issue + bitmap), slower than HBM delivers a tile (ncu, C2 round 1).
@@ -807,8 +816,8 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
           if (lane == 0 && itf < T) {
             const long long c0 = static_cast<long long>(blockIdx.x + static_cast<uint64_t>(itf) * G) * kT - P.a0;
             l2_prefetch_range(P.rec + max(0LL, c0 - kLead), P.rec + min(c0 + kT + kHalo, N));
-            if (jf < 32 && rbf > raf) l2_prefetch_range(reinterpret_cast<const uint8_t*>(P.off + raf),
-                                                        reinterpret_cast<const uint8_t*>(P.off + rbf));
+            if (!Cfg<W>::kLazyDir && jf < 32 && rbf > raf)   // (SM stages no offsets)
+              l2_prefetch_range(reinterpret_cast<const uint8_t*>(P.off + raf), reinterpret_cast<const uint8_t*>(P.off + rbf));
           }
         }
 
@@ -1244,7 +1253,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
 // compare, record check, emission).  The per-window bookkeeping (window index, stage header,
 // range masks, the warp reduction of the emission count) is paid once per 2 KiB instead of per
 // 512 B (ncu, C2 round 1: it was ~80% of the Map's instructions).
-constexpr int kSmSub = 4, kNSup = kNWin / kSmSub;
+constexpr int kSmSub = BMR_SM_SUB, kNSup = kNWin / kSmSub;
 __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   constexpr int W = kSM;
   constexpr int kStages = Cfg<W>::kStages;
@@ -1266,7 +1275,10 @@ __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl
     if (it >= T) break;
     const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
     if (it != have_it) {
-      mbar_wait(&full[s], ph);
+      // suspended wait (try_wait with a time hint): spinning map warps took 30% of the issued
+      // instructions (ncu C2), competing with the producers for issue slots
+      if (BMR_SM_WAIT_NS) mbar_wait_idle(&full[s], ph, BMR_SM_WAIT_NS);
+      else mbar_wait(&full[s], ph);
       hd = *reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
       have_it = it;
     }
@@ -1288,18 +1300,95 @@ __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl
     uint32_t need = 0;
 #pragma unroll
     for (int k = 0; k < kSmSub; ++k) need |= (__any_sync(kFull, (anym >> k) & 1u) ? 1u : 0u) << k;
+    // Rare path, part 1 (stage reads only): 16-byte compares at the first-byte candidates of the
+    // windows that have any; a lane keeps the global positions of its (<= 2 per 16 B) matches.
+    uint64_t mp[2];
+    uint32_t nm = 0;
     while (need) {                                     // warp-uniform
       const int k = __ffs(need) - 1;
       need &= need - 1;
-      const long long wp = wp0 + static_cast<long long>(k) * kWin;
-      if (wp >= hd.hi) break;
-      TileView tv{sb, nullptr, hd.sbase, hd.stg_hi, hd.ra, hd.rb};
-      const long long p0 = wp + lane * 16;
-      const bool live = (p0 + 16 > 0) && (p0 < N);
-      emit_text_chunk<W>(P, oc, outh, tv, p0, p0 - hd.sbase, live);
+      const long long p0 = wp0 + static_cast<long long>(k) * kWin + lane * 16;
+      if (!((anym >> k) & 1u)) continue;
+      const uint8_t* c = c0 + k * kWin;
+      const uint4 u0 = *reinterpret_cast<const uint4*>(c), u1 = *reinterpret_cast<const uint4*>(c + 16);
+      const uint32_t x[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
+      uint32_t cand = 0;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) cand |= eq_mask4(x[i], b0) << (4 * i);
+      cand &= range_mask32(p0, 0, min(N, hd.hi) ) & 0xFFFFu;   // own bytes of this tile, inside the input
+      while (cand) {
+        const uint32_t j = __ffs(cand) - 1;
+        cand &= cand - 1;
+        if (p0 + j + 16 > N) continue;
+        uint32_t w[4];
+        window16(x, j, w);
+        if (w[0] != P.pat[0] || w[1] != P.pat[1] || w[2] != P.pat[2] || w[3] != P.pat[3]) continue;
+        if (nm < 2) mp[nm] = static_cast<uint64_t>(p0 + j);
+        ++nm;   // (16-byte pattern whose first byte recurs: > 2 matches per 16 B -> fallback below)
+      }
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive_cnt(&empty[s], kSmSub);
+    const bool over = __any_sync(kFull, nm > 2);
+    const StageHdr h = hd;
+    // the stage is no longer read: release it before the global-memory record checks, so a
+    // match never holds up the stage ring (ncu C2: the per-lane binary search over global
+    // offsets stalled the in-order stage release)
+    if (!over) {
+      __syncwarp();
+      if (lane == 0) mbar_arrive_cnt(&empty[s], kSmSub);
+    } else {
+      // rare self-overlapping pattern (e.g. a run of one byte): the general per-window path
+      for (int k = 0; k < kSmSub; ++k) {
+        const long long wp = wp0 + static_cast<long long>(k) * kWin;
+        if (wp >= h.hi || !__any_sync(kFull, (anym >> k) & 1u)) continue;
+        TileView tv{sb, nullptr, h.sbase, h.stg_hi, h.ra, h.rb};
+        const long long p0 = wp + lane * 16;
+        emit_text_chunk<W>(P, oc, outh, tv, p0, p0 - h.sbase, (p0 + 16 > 0) && (p0 < N));
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive_cnt(&empty[s], kSmSub);
+      continue;
+    }
+    // Rare path, part 2: each match, one at a time with the whole warp: the first record start
+    // after p by a two-round warp-cooperative search of offsets[ra, rb) (32 samples, then <= 32
+    // entries), then emission of p (or its record start, MR_FLAG_SM_LINES) when no record start
+    // lies in (p, p + 15] (C-3 #3: a match lies inside one record).
+    for (;;) {
+      const uint32_t bal = __ballot_sync(kFull, nm > 0);
+      if (!bal) break;
+      const uint32_t src = __ffs(bal) - 1;
+      const unsigned long long p = __shfl_sync(kFull, static_cast<unsigned long long>(mp[0]), src);
+      if (lane == src) { mp[0] = mp[1]; --nm; }
+      unsigned long long lo = h.ra, hi = h.rb;       // first i in [lo, hi) with off[i] > p (hi if none)
+      while (hi - lo > 32) {
+        const unsigned long long step = (hi - lo + 31) / 32;
+        const unsigned long long i = lo + lane * step;
+        const uint32_t gt = __ballot_sync(kFull, i >= hi || P.off[i] > p);
+        if (gt == 0) { lo = lo + 31 * step + 1; continue; }
+        const uint32_t f = __ffs(gt) - 1;
+        if (f == 0) { hi = lo; break; }
+        hi = min(hi, lo + f * step);
+        lo = lo + (f - 1) * step + 1;
+      }
+      if (hi > lo) {
+        const unsigned long long i = lo + lane;
+        const uint32_t gt = __ballot_sync(kFull, i >= hi || P.off[i] > p);
+        hi = gt ? lo + (__ffs(gt) - 1) : hi;
+      }
+      const unsigned long long u = hi;               // (offsets[rb] lies beyond the halo)
+      const bool ok = !(u < h.rb && P.off[u] <= p + 15);
+      if (!ok) continue;
+      const uint64_t key = P.gbase + (P.sm_lines ? P.off[u - 1] : p);   // u >= 1: offsets[0] = 0 <= p
+      if (P.si) {
+        if (lane == 0) {
+          const unsigned long long g = atomicAdd(&P.st->pair_cursor, 1ULL);
+          if (g < P.cap_pairs) P.oh[g] = key;
+        }
+      } else {
+        const Slot slot = reserve<W>(P, oc, outh, 1u, P.out_cap);
+        if (lane == 0) reinterpret_cast<uint64_t*>(outh + slot.half * Cfg<W>::kOutHalf)[slot.base] = key;
+        commit(oc, slot, 1u);
+      }
+    }
   }
 }
 
@@ -1653,14 +1742,15 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
 
 // L2 prefetch distance of the Map producers (BMR_MAP_PF, tiles; default 0 = off: measured slower
 // on C2/C4 in round 1 with 2 producers)
-// L2 prefetch distance of the producers in tiles (BMR_MAP_PF; default: 2 for StringMatch, whose
-// Map is a pure read stream -- C2 0.467 -> 0.495 of HBM, round 1 sweep -- else off)
+// L2 prefetch distance of the producers in tiles (BMR_MAP_PF; default off: with the StringMatch
+// record checks moved after the stage release it no longer helps, C2 round 1 sweep 0/1/2/4)
 uint32_t map_prefetch(int w) {
   static int v = [] {
     const char* e = getenv("BMR_MAP_PF");
     return e ? atoi(e) : -1;
   }();
-  return v >= 0 ? static_cast<uint32_t>(v) : (w == kSM ? 2u : 0u);
+  (void)w;
+  return v >= 0 ? static_cast<uint32_t>(v) : 0u;
 }
 
 // idle-wait flavour of the Map role warps (BMR_MAP_WAIT: 0 = plain try_wait, 1 = suspend-time
