@@ -247,8 +247,9 @@ cudaError_t run_sort32(SortWork& W, const uint32_t* keys, uint64_t m, const uint
   if (prof && prof->on) prof->begin(s, sp2);
   for (int p = 0; p < nd; ++p) {
     uint32_t* kout = (p & 1) ? W.kb32.p : W.ka32.p;
+    const int rk = choose_rank_kind32(W.hist_h.p + digits[p] * kBinStride, m, p == 0);
     if ((e = launch_onesweep32(kin, kout, m, digits[p], bits, W.bases.p, W.status.p, W.epoch++,
-                               &st->tile_counter[0], s)))
+                               &st->tile_counter[0], s, rk)))
       return e;
     kin = kout;
   }

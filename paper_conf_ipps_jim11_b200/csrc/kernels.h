@@ -114,7 +114,10 @@ cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uin
 // keys-only LSD pass over u32 keys (the WordCount exact stream)
 cudaError_t launch_onesweep32(const uint32_t* keys_in, uint32_t* keys_out, uint64_t m, int digit, int bits,
                               const uint32_t* bases, uint64_t* status, uint32_t epoch, unsigned int* tile_counter,
-                              cudaStream_t s);
+                              cudaStream_t s, int rank_kind = 0);
+// ranking kind of a u32 pass from its digit histogram (hist[0..255], m keys): 66 (shared-memory
+// match masks) for a first pass whose digits of 32 keys are mostly distinct, else 2 (match.any)
+int choose_rank_kind32(const uint32_t* hist, uint64_t m, bool first_pass);
 
 // ---- segments ----
 // heads per sort tile + byte verification of hashed keys; counts[t] = heads in tile t

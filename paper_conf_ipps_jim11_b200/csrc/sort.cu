@@ -14,6 +14,8 @@
 // Look-back status words: [epoch:30 | kind:2 | value:32]; every launch uses a fresh epoch so
 // the status buffer never needs clearing.
 #include <algorithm>
+#include <cmath>
+#include <cstdio>
 #include <cstdlib>
 
 #include "common.cuh"
@@ -62,9 +64,10 @@ __global__ void __launch_bounds__(256) k_hist(const K* __restrict__ keys, uint64
     if (sh[i]) atomicAdd(&hist[i], sh[i]);
 }
 
-template <typename K, int IPT, bool kPay, int kBins>
+template <typename K, int IPT, bool kPay, int kBins, int kSlots = 0>
 struct SortSmem {
   static constexpr int kTile = kSortThreads * IPT;
+  uint32_t mm[kSlots > 0 ? kSlots : 1][kWarps][kSlots > 0 ? kBins : 1];   // match masks (kVar bit 6)
   K keys[kTile];
   uint32_t idx[kPay ? kTile : 1];
   uint32_t wcnt[kWarps][kBins];    // per-warp digit counters, then warp-exclusive offsets
@@ -93,11 +96,14 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
   constexpr int kBins = 1 << kBits, kDPT = kBins / kSortThreads;
   constexpr uint32_t kMask = kBins - 1;
   constexpr int kSortIPT = IPT;
-  using Smem = SortSmem<K, IPT, kPay, kBins>;
+  constexpr int kSlots = (kVar & 64) ? 4 : 0;
+  using Smem = SortSmem<K, IPT, kPay, kBins, kSlots>;
   constexpr int kSortTile = Smem::kTile;
   constexpr bool kAtomicRank = (kVar & 1) != 0, kEarly = (kVar & 2) != 0;
   constexpr bool kBackoff = (kVar & 4) != 0, kMatchHist = (kVar & 8) != 0, kBallotPeers = (kVar & 16) != 0;
-  constexpr bool kBallotAll = (kVar & 32) != 0;
+  constexpr bool kBallotAll = (kVar & 32) != 0, kOrMatch = (kVar & 64) != 0;
+  // diagnostics only (tools/micro/sort_bench; wrong output): 128 = no look-back, 256 = no global write
+  constexpr bool kDiagNoLook = (kVar & 128) != 0, kDiagNoWrite = (kVar & 256) != 0;
   static_assert(kDPT >= 1 && kDPT * kSortThreads == kBins, "bins must be a multiple of the block size");
   extern __shared__ __align__(16) uint8_t raw[];
   Smem& S = *reinterpret_cast<Smem*>(raw);
@@ -105,6 +111,8 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
   if (tid == 0) S.tile = atomicAdd(tile_counter, 1u);
   for (uint32_t i = tid; i < kWarps * kBins; i += kSortThreads) (&S.wcnt[0][0])[i] = 0;
   for (uint32_t i = tid; i < kBins; i += kSortThreads) S.hist[i] = 0;
+  if constexpr (kOrMatch)
+    for (uint32_t i = tid; i < kSlots * kWarps * kBins; i += kSortThreads) (&S.mm[0][0][0])[i] = 0;
   __syncthreads();
   const uint32_t tile = S.tile;
   const uint64_t tbase = static_cast<uint64_t>(tile) * kSortTile;
@@ -121,7 +129,53 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
 #pragma unroll
   for (int q = 0; q < kDPT; ++q) tcount[q] = 0;
   uint64_t* my = status + static_cast<uint64_t>(tile) * kBins + d0;
-  if constexpr (kBallotAll) {
+  if constexpr (kOrMatch) {
+    // kVar bit 6: peer masks through shared memory (one RED.OR of the lane bit per key into a
+    // per-warp digit slot, read back after a warp barrier, cleared by the group's leader), 4
+    // slots so that 4 keys of a thread are matched per round; the leader issues the tile
+    // histogram and warp-counter atomics (applied in issue order: stable ranks).
+#pragma unroll
+    for (int j0 = 0; j0 < kSortIPT; j0 += kSlots) {
+      uint32_t pm[kSlots];
+#pragma unroll
+      for (int q = 0; q < kSlots; ++q) {
+        if (j0 + q >= kSortIPT) break;
+        const uint32_t dj = static_cast<uint32_t>(key[j0 + q] >> shift) & kMask;
+        atomicOr(&S.mm[q][warp][dj], 1u << lane);
+      }
+      __syncwarp();
+#pragma unroll
+      for (int q = 0; q < kSlots; ++q) {
+        if (j0 + q >= kSortIPT) break;
+        pm[q] = S.mm[q][warp][static_cast<uint32_t>(key[j0 + q] >> shift) & kMask];
+      }
+      __syncwarp();
+#pragma unroll
+      for (int q = 0; q < kSlots; ++q) {
+        if (j0 + q >= kSortIPT) break;
+        const uint32_t dj = static_cast<uint32_t>(key[j0 + q] >> shift) & kMask;
+        rank[j0 + q] = 0;
+        if (lane == 31u - __clz(pm[q])) {
+          S.mm[q][warp][dj] = 0;
+          if constexpr (kEarly) atomicAdd(&S.hist[dj], __popc(pm[q]));
+          rank[j0 + q] = atomicAdd(&S.wcnt[warp][dj], __popc(pm[q]));
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < kSlots; ++q) {
+        if (j0 + q >= kSortIPT) break;
+        rank[j0 + q] = __shfl_sync(0xffffffffu, rank[j0 + q], 31 - __clz(pm[q])) + __popc(pm[q] & lanemask_lt());
+      }
+    }
+    if constexpr (kEarly) {
+      __syncthreads();
+#pragma unroll
+      for (int q = 0; q < kDPT; ++q) {
+        tcount[q] = S.hist[d0 + q];
+        st_relaxed_gpu_u64(my + q, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount[q]));
+      }
+    }
+  } else if constexpr (kBallotAll) {
     // kVar bit 5: peer masks from kBits ballots per key (no match.any: ncu C5 round 1 put 48% of
     // the stall samples on the instruction consuming the MATCH result).  Per key group (equal
     // digits in the warp) the highest lane issues one shared atomic for the tile histogram and
@@ -278,7 +332,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
     uint32_t excl[kDPT];
 #pragma unroll
     for (int q = 0; q < kDPT; ++q) excl[q] = 0;
-    if (tile > 0) {
+    if (tile > 0 && !kDiagNoLook) {
       long long p[kDPT];
       bool done[kDPT];
 #pragma unroll
@@ -326,6 +380,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
   __syncthreads();
   // 6. contiguous per-digit runs to global memory
   const uint32_t nvalid = static_cast<uint32_t>(min(static_cast<uint64_t>(kSortTile), m - tbase));
+  if constexpr (kDiagNoWrite) return;
   if (nvalid == static_cast<uint32_t>(kSortTile)) {
     // full tile: unrolled in groups of 8, so the SMEM reads of 8 elements are in flight together
     // (a rolled loop serialises LDS key -> LDS goff -> STG per element)
@@ -484,12 +539,31 @@ int sort_cfg() {
 }
 // u32 keys-only shapes (keys per thread, CTAs per SM): cfg 0 (24, 3), 1 (32, 2), 2 (16, 4), 3 (24, 2)
 static const int kIPT32[4] = {24, 32, 16, 24};
+// u32 pass ranking by digit statistics: E = expected number of distinct digits among 32 keys
+// (sum over bins of 1 - (1 - p_b)^32).  match.any slows down with many distinct values per warp,
+// the shared-memory OR masks with many equal ones (same-address atomics serialise); measured with
+// tools/micro/sort_bench (round 1): first pass over Zipf keys (E 28.6) 3.37 vs 4.59 ms.  Only the
+// first pass sees the input order: after it, equal keys are adjacent and the warps' digits are
+// far less diverse than E says (later passes: match 2.4-3.4 ms, OR masks 3.8-4.6 ms), so they
+// keep match.any.  BMR_SORT_ADAPT = threshold on E (default 24; 0 disables: env variant).
+int choose_rank_kind32(const uint32_t* hist, uint64_t m, bool first_pass) {
+  static double thr = [] {
+    const char* e = getenv("BMR_SORT_ADAPT");
+    return e ? atof(e) : 24.0;
+  }();
+  if (thr <= 0 || m == 0) return 0;
+  double e = 0;
+  for (int b = 0; b < 256; ++b) e += 1.0 - std::pow(1.0 - static_cast<double>(hist[b]) / static_cast<double>(m), 32);
+  if (getenv("BMR_SORT_DEBUG")) fprintf(stderr, "[bmr] u32 pass: E[distinct digits / 32 keys] = %.2f\n", e);
+  return (first_pass && e >= thr) ? 66 : 2;
+}
+
 int sort_tile() { return kSortThreads * (sort_cfg() == 1 ? 12 : 16); }
 int sort_tile_keys() { return kSortThreads * (sort_cfg() == 1 ? 24 : 16); }
 int sort_variant32();
 int sort_tile_keys32() {
   const int v = sort_variant32();
-  return kSortThreads * (v == 19 || v == 21 || v == 22 || v == 35 || v == 36 ? 16 : v == 20 ? 20 : v == 37 ? 32
+  return kSortThreads * (v == 19 || v == 21 || v == 22 || v == 35 || v == 36 || v == 67 || v == 68 ? 16 : v == 20 ? 20 : v == 37 ? 32
                                                                                           : kIPT32[sort_cfg()]);
 }
 
@@ -498,7 +572,7 @@ static void launch_os(unsigned tiles, const K* keys_in, const uint32_t* idx_in, 
                       uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status, uint32_t epoch,
                       unsigned int* tile_counter, cudaStream_t s) {
   const auto k = &k_onesweep<K, kFirst, kVar, IPT, MINB, kPay, 8, LW>;
-  const size_t smem = sizeof(SortSmem<K, IPT, kPay, 256>);
+  const size_t smem = sizeof(SortSmem<K, IPT, kPay, 256, (kVar & 64) ? 4 : 0>);
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
   k<<<tiles, kSortThreads, smem, s>>>(keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch,
                                       tile_counter);
@@ -514,6 +588,9 @@ static void launch_pay(unsigned tiles, const uint64_t* keys_in, const uint32_t* 
   if (sort_cfg() == 1) launch_os<uint64_t, kFirst, kVar, 12, 4, true>(BMR_OS_ARGS);   // cfg 1: 12 keys, 4 CTAs
   else launch_os<uint64_t, kFirst, kVar, 16, 3, true>(BMR_OS_ARGS);
 }
+
+// per-pass ranking choice of the u32 passes (launch_onesweep32's rank_kind; <= 0: BMR_SORT_VARIANT32)
+static thread_local int g_rank_kind = 0;
 
 template <typename K>
 static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* keys_out, uint32_t* idx_out, uint64_t m,
@@ -538,7 +615,7 @@ static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* ke
     } else if (sort_cfg() == 3) {
       launch_os<K, false, 2, 24, 2, false>(BMR_OS_ARGS);
     } else {
-      switch (sort_variant32()) {
+      switch (g_rank_kind > 0 ? g_rank_kind : sort_variant32()) {
         case 0: launch_os<K, false, 0, 24, 3, false>(BMR_OS_ARGS); break;
         case 1: launch_os<K, false, 1, 24, 3, false>(BMR_OS_ARGS); break;
         case 3: launch_os<K, false, 3, 24, 3, false>(BMR_OS_ARGS); break;
@@ -556,6 +633,15 @@ static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* ke
         case 39: launch_os<K, false, 34, 24, 3, false, 16>(BMR_OS_ARGS); break;
         case 40: launch_os<K, false, 34, 24, 3, false, 32>(BMR_OS_ARGS); break;
         case 41: launch_os<K, false, 2, 24, 3, false, 16>(BMR_OS_ARGS); break;
+        case 130: launch_os<K, false, 130, 24, 3, false>(BMR_OS_ARGS); break;   // diagnostics (wrong output)
+        case 258: launch_os<K, false, 258, 24, 3, false>(BMR_OS_ARGS); break;
+        case 386: launch_os<K, false, 386, 24, 3, false>(BMR_OS_ARGS); break;
+        case 194: launch_os<K, false, 194, 24, 3, false>(BMR_OS_ARGS); break;
+        case 322: launch_os<K, false, 322, 24, 3, false>(BMR_OS_ARGS); break;
+        case 66: launch_os<K, false, 66, 24, 3, false>(BMR_OS_ARGS); break;   // RED.OR match masks, 4 slots
+        case 67: launch_os<K, false, 66, 16, 3, false>(BMR_OS_ARGS); break;
+        case 68: launch_os<K, false, 66, 16, 4, false>(BMR_OS_ARGS); break;
+        case 69: launch_os<K, false, 66, 24, 2, false>(BMR_OS_ARGS); break;
         default: launch_os<K, false, 2, 24, 3, false>(BMR_OS_ARGS); break;
       }
     }
@@ -583,7 +669,8 @@ cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uin
 }
 cudaError_t launch_onesweep32(const uint32_t* keys_in, uint32_t* keys_out, uint64_t m, int digit, int bits,
                               const uint32_t* bases_all, uint64_t* status, uint32_t epoch,
-                              unsigned int* tile_counter, cudaStream_t s) {
+                              unsigned int* tile_counter, cudaStream_t s, int rank_kind) {
+  g_rank_kind = rank_kind;
   return onesweep_impl<uint32_t>(keys_in, nullptr, keys_out, nullptr, m, digit, bits, bases_all, status, epoch,
                                  tile_counter, s);
 }
