@@ -37,6 +37,9 @@ constexpr int kNMap = 16;
 #ifndef BMR_SM_NMAP
 #define BMR_SM_NMAP 24   // StringMatch map warps
 #endif
+#ifndef BMR_WC_COMB_PROBES
+#define BMR_WC_COMB_PROBES 1   // WordCount combiner probes per word (2: C5 absorbs 4.6% more words but the Map costs 0.9 ms more than the sort saves)
+#endif
 #ifndef BMR_SM_WAIT_NS
 #define BMR_SM_WAIT_NS 1000   // StringMatch map warps: suspend-time hint of the stage wait (0: spin)
 #endif
@@ -845,13 +848,22 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
 // key or is free (claimed by a 32-bit CAS); false = the slot belongs to another key (emit
 // normally).  Keys and counts are separate u32 arrays: 32-bit shared atomics are native (a
 // 64-bit shared atomicAdd is a CAS spin loop, which serialises on the Zipf head's slots).
+// BMR_WC_COMB_PROBES probes (home slot, home ^ 1, ...): with 2, a key whose home slot belongs to
+// another key gets a second chance (measured on C5, round 1: not worth its Map instructions).  Slots are never freed within a batch,
+// so a key lives in at most one of its two slots; partials are summed per key anyway.
 __device__ __forceinline__ bool comb_add(uint32_t* ckey, uint32_t key) {
-  const uint32_t slot = (key * 0x9E3779B1u) >> (32 - kCombBits);
-  uint32_t v = *reinterpret_cast<volatile uint32_t*>(ckey + slot);
-  if (v == kCombEmpty32) v = atomicCAS(ckey + slot, kCombEmpty32, key);
-  if (v != key && v != kCombEmpty32) return false;
-  atomicAdd(ckey + Cfg<kWC>::kCombSlots + slot, 1u);   // count array follows the key array
-  return true;
+  const uint32_t home = (key * 0x9E3779B1u) >> (32 - kCombBits);
+#pragma unroll
+  for (uint32_t probe = 0; probe < BMR_WC_COMB_PROBES; ++probe) {
+    const uint32_t slot = home ^ probe;
+    uint32_t v = *reinterpret_cast<volatile uint32_t*>(ckey + slot);
+    if (v == kCombEmpty32) v = atomicCAS(ckey + slot, kCombEmpty32, key);
+    if (v == key || v == kCombEmpty32) {
+      atomicAdd(ckey + Cfg<kWC>::kCombSlots + slot, 1u);   // count array follows the key array
+      return true;
+    }
+  }
+  return false;
 }
 // WordCount emission of one warp window.  Each start is classified BEFORE the reservation: a
 // word is exact iff it ends within kWcExact bytes (nb bit q: a word cannot continue at q, so the
