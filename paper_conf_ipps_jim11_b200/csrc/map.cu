@@ -1135,6 +1135,19 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
     // search: every lane publishes its 16-bit "stop" mask (a '"' or a record start) and a marker
     // finds the first stop at or after its URL start with two shuffles (the URL ends at the first
     // '"' unless the record ends first, C-3 #9); only URLs leaving the 512-B window scan onwards.
+    // '<' is rare in the text outside markers: a window without one in any lane emits nothing
+    // (exact has-byte test, 3 ALU ops per 4 bytes, before the per-byte masks)
+    {
+      uint32_t a = 0;
+      if (live) {
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const uint32_t t = x[i] ^ 0x3C3C3C3Cu;
+          a |= (t - 0x01010101u) & ~t;
+        }
+      }
+      if (!__any_sync(kFull, (a & 0x80808080u) != 0)) return;
+    }
     uint32_t mk = 0, st16 = 0;
     if (live) {
       uint32_t cand = 0, qm = 0;
