@@ -702,7 +702,7 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
     const uint64_t cap_b = !wc ? 0 : hint ? hint : nbytes / 48 + 4096;
     const uint64_t cap_c = !wc ? 0 : hint ? hint : nbytes / 32 + 4096;
     CK(ensure_pairs(job, initial_cap(job, nbytes, n), cap_b, cap_c), "alloc intermediate");
-    if (job->wc_comb()) {   // combiner partials: <= 4096 per CTA per batch (grown + replayed if exceeded)
+    if (job->wc_comb()) {   // combiner partials: <= 2^kCombBits per CTA per batch (grown + replayed if exceeded)
       job->cap_p = job->cfg.max_pairs_hint ? job->cfg.max_pairs_hint : 2ULL * 4096 * job->nsm + 4096;
       CK(job->hp.ensure(job->cap_p), "alloc partials");
     }

@@ -37,6 +37,17 @@ constexpr int kNMap = 16;
 #ifndef BMR_SM_NMAP
 #define BMR_SM_NMAP 24   // StringMatch map warps
 #endif
+#ifndef BMR_WC_COMB_BITS
+#define BMR_WC_COMB_BITS 13     // WordCount combiner: 2^bits direct-mapped slots (u32 key + u32 count);
+                                // 13 (64 KB): C5 exact stream 672 M -> 599 M keys, step 47.4 -> 46.2 ms
+#endif
+#ifndef BMR_WC_OUT_BYTES
+#define BMR_WC_OUT_BYTES 8192   // WordCount output buffer bytes (x kNOut; 12 KB -> 8 KB: no measurable Map cost)
+#endif
+#ifndef BMR_WC_OFFCAP
+#define BMR_WC_OFFCAP 640       // WordCount: record offsets staged per tile (C1/C5 lines >= 27 B: <= 617 per
+                                // staged window; denser tiles read offsets from global memory)
+#endif
 #ifndef BMR_WC_COMB_PROBES
 #define BMR_WC_COMB_PROBES 1   // WordCount combiner probes per word (2: C5 absorbs 4.6% more words but the Map costs 0.9 ms more than the sort saves)
 #endif
@@ -77,7 +88,7 @@ struct Cfg {
   // StringMatch (read-bound, almost no output, lazy record directory below: no offsets or bitmap
   // regions): 8 stages of bytes in flight
   static constexpr int kStages = (W == kSM) ? BMR_SM_STAGES : 4;
-  static constexpr int kOffCap = (W == kSM) ? 0 : 1024;   // record offsets staged per tile (more: read from global)
+  static constexpr int kOffCap = (W == kSM) ? 0 : (W == kWC) ? BMR_WC_OFFCAP : 1024;   // record offsets staged per tile (more: read from global)
   // StringMatch reads the record directory lazily: record boundaries matter only where the
   // pattern's first byte matches (planted, rare), so no offsets are staged and no bitmap is built;
   // a candidate checks for a record start inside its 16 bytes by a binary search over the tile's
@@ -85,7 +96,7 @@ struct Cfg {
   static constexpr bool kLazyDir = (W == kSM);
   static constexpr int kOffBytes = (W == kSM) ? 0 : ((kOffCap + 2) * 8 + 127) / 128 * 128;
   static constexpr int kBits = (W == kSM) ? 0 : kBitBytes;   // record-start bitmap bytes per stage
-  static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? 12288 : 20480;   // bytes per output buffer
+  static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? BMR_WC_OUT_BYTES : 20480;   // bytes per output buffer
   // the producer builds the bitmap of tile it - kLag right after issuing tile it: kLag stages of
   // TMA traffic stay in flight per SM while one stage is being consumed
   static constexpr int kLag = kStages - 2;
@@ -100,9 +111,9 @@ struct Cfg {
   static constexpr int kXQ = (W == kWC) ? 264 : 0;
   // WC: in-SMEM combiner (MapCG-style): kCombSlots u64 entries
   // (u32 exact keys + u32 counts), direct-mapped, a slot keeps the first key that claims it
-  static constexpr int kCombSlots = (W == kWC) ? 4096 : 0;
+  static constexpr int kCombSlots = (W == kWC) ? (1 << BMR_WC_COMB_BITS) : 0;
 };
-constexpr int kCombBits = 12;
+constexpr int kCombBits = BMR_WC_COMB_BITS;
 static_assert(Cfg<kWC>::kCombSlots == (1 << kCombBits), "combiner slots");
 constexpr uint32_t kCombEmpty32 = 0xFFFFFFFFu;   // exact keys are < 2^30
 // WC words of <= kWcExact bytes get an exact 30-bit key (common.cuh exact_key30) and travel in
