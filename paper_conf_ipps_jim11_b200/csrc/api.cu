@@ -186,8 +186,9 @@ cudaError_t run_sort(SortWork& W, const uint64_t* keys, uint64_t m, const uint64
   for (int p = 0; p < nd; ++p) {
     uint64_t* kout = (p & 1) ? W.kb.p : W.ka.p;
     uint32_t* iout = pay ? ((p & 1) ? W.ib.p : W.ia.p) : nullptr;
+    const int rk = pay ? 0 : choose_rank_kind32(W.hist_h.p + digits[p] * kBinStride, m, p == 0);
     if ((e = launch_onesweep(kin, iin, kout, iout, m, digits[p], bits, W.bases.p, W.status.p, W.epoch++,
-                             &st->tile_counter[0], s)))
+                             &st->tile_counter[0], s, rk)))
       return e;
     kin = kout;
     iin = iout;

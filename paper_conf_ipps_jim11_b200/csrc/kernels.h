@@ -110,7 +110,8 @@ cudaError_t launch_hist32(const uint32_t* keys, uint64_t m, uint32_t* hist, int 
 // bases: 8 x kBinStride table of global digit bases; status: tiles x 2^bits look-back words
 cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
                             uint32_t* idx_out, uint64_t m, int digit, int bits, const uint32_t* bases,
-                            uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s);
+                            uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s,
+                            int rank_kind = 0);   // 66: OR-mask ranking (keys-only passes), else match.any
 // keys-only LSD pass over u32 keys (the WordCount exact stream)
 cudaError_t launch_onesweep32(const uint32_t* keys_in, uint32_t* keys_out, uint64_t m, int digit, int bits,
                               const uint32_t* bases, uint64_t* status, uint32_t epoch, unsigned int* tile_counter,

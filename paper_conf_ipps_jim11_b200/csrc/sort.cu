@@ -646,7 +646,8 @@ static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* ke
       }
     }
   } else if (keys_only) {
-    if (sort_cfg() == 1) launch_os<K, false, 2, 24, 2, false>(BMR_OS_ARGS);   // cfg 1: 24 keys, 2 CTAs
+    if (g_rank_kind == 66) launch_os<K, false, 66, 16, 3, false>(BMR_OS_ARGS);   // OR-mask ranking (first pass)
+    else if (sort_cfg() == 1) launch_os<K, false, 2, 24, 2, false>(BMR_OS_ARGS);   // cfg 1: 24 keys, 2 CTAs
     else launch_os<K, false, 2, 16, 3, false>(BMR_OS_ARGS);
   } else {
     switch ((sort_variant() ? 1 : 0) | (first ? 2 : 0)) {
@@ -663,7 +664,8 @@ static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* ke
 
 cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out, uint32_t* idx_out,
                             uint64_t m, int digit, int bits, const uint32_t* bases_all, uint64_t* status,
-                            uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
+                            uint32_t epoch, unsigned int* tile_counter, cudaStream_t s, int rank_kind) {
+  g_rank_kind = rank_kind;
   return onesweep_impl<uint64_t>(keys_in, idx_in, keys_out, idx_out, m, digit, bits, bases_all, status, epoch,
                                  tile_counter, s);
 }
