@@ -51,12 +51,16 @@ __device__ bool key_bytes_equal(uint64_t ka, uint64_t kb) {
   if (la != lb) return false;
   const uint8_t* pa = reinterpret_cast<const uint8_t*>(ka >> 16);
   const uint8_t* pb = reinterpret_cast<const uint8_t*>(kb >> 16);
+  // no early exit inside the loop: equal keys (the common case) read every chunk anyway, and
+  // independent iterations let the loads of several chunks be in flight together
+  uint64_t diff = 0;
+#pragma unroll 4
   for (uint32_t i = 0; i < la; i += 8) {
     const uint32_t need = min(8u, la - i);
     const uint64_t mask = need == 8 ? ~0ULL : ((1ULL << (8 * need)) - 1ULL);
-    if (((load8(pa + i, need) ^ load8(pb + i, need)) & mask) != 0) return false;
+    diff |= (load8(pa + i, need) ^ load8(pb + i, need)) & mask;
   }
-  return true;
+  return diff == 0;
 }
 
 // Each warp owns 512 consecutive sorted positions (16 steps of 32 lanes: coalesced loads);
