@@ -26,6 +26,8 @@
 #include <cstdio>
 #include <cstdlib>
 
+#include <climits>
+
 #include "common.cuh"
 
 namespace bmr {
@@ -105,7 +107,7 @@ struct Cfg {
   // after the emission rounds (a lane-per-word hash inside the rounds diverges: with 10% long
   // words, most rounds would carry at least one).  A window holds at most 512 / 6 + 1 starts
   // of words longer than kWcExact bytes.
-  static constexpr int kHashQ = (W == kWC) ? 96 : 0;
+  static constexpr int kHashQ = (W == kWC) ? 96 : (W == kII) ? 192 : 0;   // II: URL queue, 64 x (u64 pos + u32 len)
   // WC: per-warp queue of the window's exact keys that missed the combiner (u32), copied into
   // the output buffer after the one reservation; <= 257 word starts per window
   static constexpr int kXQ = (W == kWC) ? 264 : 0;
@@ -1039,9 +1041,43 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
   commit(oc, slot, packed);
 }
 
+// InvertedIndex URL queue (per map warp, in the hq region): the markers of a window are queued as
+// (URL position, length) and the queue is drained 32..64 entries at a time, one entry per lane:
+// key (inline or the hash of the URL bytes, read from global memory so the stage can go), one
+// reservation, SoA stores.  A window holds about one URL, so hashing it in the window's emission
+// round left 31 lanes idle for the whole hash (ncu C4 round 1: ~15% of the Map's instructions).
+__device__ __forceinline__ uint64_t* ii_qpos(uint8_t* outh) {
+  return reinterpret_cast<uint64_t*>(outh + (Layout<kII>::hq - Layout<kII>::out)) +
+         (threadIdx.x >> 5) * (Cfg<kII>::kHashQ / 2);
+}
+__device__ void ii_drain(const Params& P, OutCtl* oc, uint8_t* outh, uint32_t& qn) {
+  using F = PairFmt<kII>;
+  if (qn == 0) return;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t* qpos = ii_qpos(outh);
+  const uint32_t* qlen = reinterpret_cast<const uint32_t*>(qpos + 64);
+  __syncwarp();
+  const Slot slot = reserve<kII>(P, oc, outh, qn, P.out_cap);
+  uint8_t* half = outh + slot.half * Cfg<kII>::kOutHalf;
+  uint64_t* sh = reinterpret_cast<uint64_t*>(half);
+  uint64_t* sk = sh + F::kCap;
+  uint64_t* sv = reinterpret_cast<uint64_t*>(half + F::kCap * 16);
+  const TileView gv{nullptr, nullptr, 0, LLONG_MIN, 0, 0};   // key bytes from global memory
+  for (uint32_t e = lane; e < qn; e += 32) {
+    const long long q0 = static_cast<long long>(qpos[e]);
+    const uint32_t len = qlen[e];
+    const uint32_t idx = slot.base + e;
+    sh[idx] = key_at(P, gv, q0, len);
+    sk[idx] = (reinterpret_cast<uint64_t>(P.rec + q0) << 16) | len;
+    sv[idx] = P.gbase + static_cast<uint64_t>(q0);
+  }
+  commit(oc, slot, qn);
+  qn = 0;
+}
+
 template <int W>
 __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, const TileView& tv,
-                                long long p0, long long i0, bool live) {
+                                long long p0, long long i0, bool live, uint32_t& qn) {
   using F = PairFmt<W>;
   const long long N = static_cast<long long>(P.nbytes);
   uint32_t x[8];
@@ -1219,6 +1255,31 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
     emit_wc(P, oc, outh, tv, x, p0, emit_mask, nb);
     return;
   }
+  if constexpr (W == kII) {
+    if (!P.si) {   // queue the URLs (drained lane-parallel, see ii_drain)
+      const uint32_t cnt = __popc(emit_mask);   // <= 2 markers start in 16 bytes
+      const uint32_t incl = warp_inclusive_add(cnt);
+      const uint32_t tot = __shfl_sync(kFull, incl, 31);
+      if (tot == 0) return;
+      if (qn + tot > 64) ii_drain(P, oc, outh, qn);
+      uint64_t* qpos = ii_qpos(outh);
+      uint32_t* qlen = reinterpret_cast<uint32_t*>(qpos + 64);
+      uint32_t k = qn + incl - cnt;
+      int nth = 0;
+      for (uint32_t m = emit_mask; m; m &= m - 1) {
+        const uint32_t j = __ffs(m) - 1;
+        uint32_t len = nth == 0 ? aux[0] : aux[1];
+        ++nth;
+        if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
+        qpos[k] = static_cast<uint64_t>(p0 + j + 9);
+        qlen[k] = len;
+        ++k;
+      }
+      qn += tot;
+      if (qn >= 32) ii_drain(P, oc, outh, qn);
+      return;
+    }
+  }
   // ---- reserve one warp result, then lane-major emission rounds
   const uint32_t total = __reduce_add_sync(kFull, __popc(emit_mask));
   if (total == 0) return;
@@ -1378,7 +1439,8 @@ __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl
         if (wp >= h.hi || !__any_sync(kFull, (anym >> k) & 1u)) continue;
         TileView tv{sb, nullptr, h.sbase, h.stg_hi, h.ra, h.rb};
         const long long p0 = wp + lane * 16;
-        emit_text_chunk<W>(P, oc, outh, tv, p0, p0 - h.sbase, (p0 + 16 > 0) && (p0 < N));
+        uint32_t qn_unused = 0;
+        emit_text_chunk<W>(P, oc, outh, tv, p0, p0 - h.sbase, (p0 + 16 > 0) && (p0 < N), qn_unused);
       }
       __syncwarp();
       if (lane == 0) mbar_arrive_cnt(&empty[s], kSmSub);
@@ -1454,6 +1516,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   // (P.dyn == 0: static order, map warp w takes windows w, w + nmap, w + 2 nmap, ... of the CTA's
   // window sequence)
   uint32_t kseq = 0, have_it = ~0u;
+  uint32_t qn = 0;   // II: queued URLs of this warp (ii_drain)
   StageHdr hd{};
   const bool sm_fast = W == kSM && !P.so && !P.dyn;
   if constexpr (W == kSM) {
@@ -1593,7 +1656,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       if (wp < hd.hi) {                               // warp-uniform
         const long long p0 = wp + lane * 16;
         const bool live = (p0 + 16 > 0) && (p0 < static_cast<long long>(P.nbytes));
-        emit_text_chunk<W>(P, oc, outh, tv, p0, p0 - hd.sbase, live);
+        emit_text_chunk<W>(P, oc, outh, tv, p0, p0 - hd.sbase, live, qn);
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[s]);
@@ -1612,6 +1675,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       }
     }
   }
+  if constexpr (W == kII) ii_drain(P, oc, outh, qn);   // this warp's last queued URLs
   // final flush of the partially filled half (all map warps done, nothing pending)
   named_bar_sync(2, nmap<W>() * 32);
   if constexpr (W == kWC) {
