@@ -53,6 +53,9 @@ constexpr int kNMap = 16;
 #ifndef BMR_WC_COMB_PROBES
 #define BMR_WC_COMB_PROBES 1   // WordCount combiner probes per word (2: C5 absorbs 4.6% more words but the Map costs 0.9 ms more than the sort saves)
 #endif
+#ifndef BMR_SM_DYN
+#define BMR_SM_DYN 1   // StringMatch super-windows: 0 static round-robin, 1 shared counter (C2 Map 1.03 -> 0.81 ms)
+#endif
 #ifndef BMR_SM_WAIT_NS
 #define BMR_SM_WAIT_NS 1000   // StringMatch map warps: suspend-time hint of the stage wait (0: spin)
 #endif
@@ -1367,7 +1370,14 @@ __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl
   uint32_t have_it = ~0u;
   StageHdr hd{};
   for (uint32_t kseq = 0;; ++kseq) {
-    const uint32_t g = warp + kseq * static_cast<uint32_t>(nmap<W>());
+    uint32_t g;
+    if (BMR_SM_DYN) {   // super-windows from a shared counter: a warp busy with a match's record
+      uint32_t gg = 0;  // check does not hold up the super-windows it would own in static order
+      if (lane == 0) gg = atomicAdd(&oc->win_next, 1u);
+      g = __shfl_sync(kFull, gg, 0);
+    } else {
+      g = warp + kseq * static_cast<uint32_t>(nmap<W>());
+    }
     const uint32_t it = g / kNSup, sw = g % kNSup;
     if (it >= T) break;
     const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
