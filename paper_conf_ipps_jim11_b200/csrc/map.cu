@@ -1346,7 +1346,8 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
   if (!P.si) commit(oc, slot, total);
 }
 
-// StringMatch map warps (default SIO, static order): super-windows of kSmSub 512-B windows.  The
+// StringMatch map warps (all memory modes): super-windows of kSmSub 512-B windows, handed out
+// from a shared counter (BMR_SM_DYN) or in a static round-robin.  The
 // pattern's first byte is rare in text, so each lane first runs the exact has-byte test over its
 // kSmSub 16-B chunks (one LDS.128 + 3 ALU ops per 4 bytes); only a 512-B window in which some
 // lane saw the byte runs the full per-byte path (emit_text_chunk: candidate mask, 16-byte
@@ -1396,9 +1397,18 @@ __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl
     // outside [0, N) only cause a spurious slow-path visit, which masks them exactly
     uint32_t anym = 0;
     const uint8_t* c0 = sb + (wp0 - hd.sbase) + lane * 16;
+    // SO / G ablation (MR_FLAG_NO_SMEM_IN): the same loads from global memory (the stage is empty)
+    auto ld16 = [&](long long q, const uint8_t* sp) -> uint4 {
+      if (!P.so) return *reinterpret_cast<const uint4*>(sp);
+      if (q >= 0 && q + 16 <= N) return __ldg(reinterpret_cast<const uint4*>(P.rec + q));   // rec + q: 16-B aligned
+      uint32_t w[4] = {0, 0, 0, 0};
+      for (int b = 0; b < 16; ++b)
+        if (q + b >= 0 && q + b < N) w[b >> 2] |= static_cast<uint32_t>(P.rec[q + b]) << (8 * (b & 3));
+      return make_uint4(w[0], w[1], w[2], w[3]);
+    };
 #pragma unroll
     for (int k = 0; k < kSmSub; ++k) {
-      const uint4 c = *reinterpret_cast<const uint4*>(c0 + k * kWin);
+      const uint4 c = ld16(wp0 + k * kWin + lane * 16, c0 + k * kWin);
       const uint32_t t0 = c.x ^ b0, t1 = c.y ^ b0, t2 = c.z ^ b0, t3 = c.w ^ b0;
       const uint32_t a = ((t0 - 0x01010101u) & ~t0) | ((t1 - 0x01010101u) & ~t1) | ((t2 - 0x01010101u) & ~t2) |
                          ((t3 - 0x01010101u) & ~t3);
@@ -1417,7 +1427,7 @@ __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl
       const long long p0 = wp0 + static_cast<long long>(k) * kWin + lane * 16;
       if (!((anym >> k) & 1u)) continue;
       const uint8_t* c = c0 + k * kWin;
-      const uint4 u0 = *reinterpret_cast<const uint4*>(c), u1 = *reinterpret_cast<const uint4*>(c + 16);
+      const uint4 u0 = ld16(p0, c), u1 = ld16(p0 + 16, c + 16);
       const uint32_t x[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
       uint32_t cand = 0;
 #pragma unroll
@@ -1528,7 +1538,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   uint32_t kseq = 0, have_it = ~0u;
   uint32_t qn = 0;   // II: queued URLs of this warp (ii_drain)
   StageHdr hd{};
-  const bool sm_fast = W == kSM && !P.so && !P.dyn;
+  const bool sm_fast = W == kSM && !P.dyn;
   if constexpr (W == kSM) {
     if (sm_fast) sm_fast_loop(P, smem, oc);
   }
