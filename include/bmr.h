@@ -192,6 +192,28 @@ mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_byte
 mr_status mr_partition_write(mr_job* job, void* entries, void* heap);
 mr_status mr_ingest(mr_job* job, const void* entries, const void* heap, const uint64_t* recv_counts);
 
+/* ---- Fused Map flush + shuffle over peer memory, InvertedIndex ----
+ * Instead of partition + all-to-all, the Map's flush appends every record straight to the
+ * receive window of its destination rank (same destination function as mr_partition_*): per
+ * warp and destination one atomic pair on the window cursor, then the 16-byte entry
+ * (heap offset << 16 | key length, u64 value) and the key bytes (8-byte aligned records).
+ * A window = entries (16-B aligned, entry_cap x 16 B) + heap (8-B aligned, heap_cap bytes) +
+ * cursor (2 x u64: entries, heap bytes appended; counts demand past the capacity), all device
+ * memory the CALLER owns and zeroes, addressable from this process: a peer GPU's buffers opened
+ * through CUDA IPC (NVLink stores and atomics), or same-GPU buffers (virtual ranks, tests).
+ *   mr_set_xwindows(job, R, entries[R], heaps[R], cursors[R], entry_cap, heap_cap) — host arrays
+ *     of device pointers, window r = rank r; CREATED state (before mr_map); R = 0 disables.
+ *     MR_ERR_INVALID: not InvertedIndex, NULL / misaligned pointer, R > 64.
+ *   mr_map ... (the records leave through the windows; nothing stays local)
+ *   all ranks' Maps complete (caller's barrier), then on every rank
+ *   mr_ingest_xwindow(job, own_entries, own_heap, own_cursor, entry_cap, heap_cap): reads the
+ *     cursor, MR_ERR_OOM if the window overflowed (nothing ingested; re-run with larger windows),
+ *     else ingests like mr_ingest -> MAPPED; then mr_group / mr_reduce / mr_fetch. */
+mr_status mr_set_xwindows(mr_job* job, uint32_t nranks, void* const* entries, void* const* heaps,
+                          uint64_t* const* cursors, uint64_t entry_cap, uint64_t heap_cap);
+mr_status mr_ingest_xwindow(mr_job* job, const void* entries, const void* heap, const uint64_t* cursor,
+                            uint64_t entry_cap, uint64_t heap_cap);
+
 /* Group-by primitive exposed for testing (§8(a) a7): stable LSD radix sort of n u64 device
  * keys; writes the sorted keys and the u32 permutation (perm[i] = source index of the i-th
  * key).  Synchronises `stream`. n < 2^32. */

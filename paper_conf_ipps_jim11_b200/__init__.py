@@ -30,7 +30,28 @@ STATUS = {0: "MR_OK", 1: "MR_ERR_INVALID", 2: "MR_ERR_STATE", 3: "MR_ERR_OOM", 4
 
 EXPORTS = ("mr_job_create", "mr_map", "mr_map_host", "mr_map_host_lines", "mr_group", "mr_reduce", "mr_fetch", "mr_job_reset",
            "mr_get_stats", "mr_job_destroy", "mr_status_string", "mr_last_error", "mr_sort_u64",
-           "mr_partition_count", "mr_partition_write", "mr_ingest")
+           "mr_partition_count", "mr_partition_write", "mr_ingest", "mr_set_xwindows", "mr_ingest_xwindow")
+
+
+class XWindow:
+    """A receive window of the fused Map flush (f-3): device buffers for entry_cap 16-byte entries,
+    heap_cap key bytes and the 2 x u64 cursor, owned here (torch tensors on `device`)."""
+
+    def __init__(self, entry_cap: int, heap_cap: int, device=None):
+        import torch
+        dev = device if device is not None else torch.device("cuda", torch.cuda.current_device())
+        self.entry_cap, self.heap_cap = int(entry_cap), int(heap_cap)
+        self.entries = torch.empty(max(self.entry_cap, 1) * 16, dtype=torch.uint8, device=dev)
+        self.heap = torch.empty(max(self.heap_cap, 8), dtype=torch.uint8, device=dev)
+        self.cursor = torch.zeros(2, dtype=torch.int64, device=dev)
+
+    def reset(self):
+        self.cursor.zero_()
+
+    def used(self):
+        """(entries, heap bytes) appended so far (demand; may exceed the capacity)."""
+        c = self.cursor.cpu().tolist()
+        return int(c[0]), int(c[1])
 
 
 class MRError(RuntimeError):
@@ -95,6 +116,8 @@ def lib() -> C.CDLL:
         L.mr_partition_count.argtypes = [vp, vp, C.POINTER(u64)]
         L.mr_partition_write.argtypes = [vp, vp, vp]
         L.mr_ingest.argtypes = [vp, vp, vp, vp]
+        L.mr_set_xwindows.argtypes = [vp, C.c_uint32, vp, vp, vp, u64, u64]
+        L.mr_ingest_xwindow.argtypes = [vp, vp, vp, vp, u64, u64]
         for f in EXPORTS:
             if f not in ("mr_status_string", "mr_last_error"):
                 getattr(L, f).restype = C.c_int
@@ -227,6 +250,27 @@ class Job:
         rc = np.ascontiguousarray(recv_counts, np.int64).astype(np.uint64).reshape(-1)
         self._recv = (entries, heap, rc)
         self._check(lib().mr_ingest(self.h, _ptr(entries), _ptr(heap), _ptr(rc)))
+
+    # ---- fused Map flush + shuffle (mr_set_xwindows / mr_ingest_xwindow) ----
+    def set_xwindows(self, windows):
+        """Register one receive window per destination rank (list of XWindow, rank order) before
+        map(): InvertedIndex records then leave the Map straight through them."""
+        n = len(windows)
+        arr = (C.c_void_p * max(n, 1))
+        ents = arr(*[w.entries.data_ptr() for w in windows])
+        heaps = arr(*[w.heap.data_ptr() for w in windows])
+        curs = arr(*[w.cursor.data_ptr() for w in windows])
+        ecap = windows[0].entry_cap if n else 0
+        hcap = windows[0].heap_cap if n else 0
+        self._xwin = list(windows)
+        self._check(lib().mr_set_xwindows(self.h, n, C.cast(ents, C.c_void_p), C.cast(heaps, C.c_void_p),
+                                          C.cast(curs, C.c_void_p), ecap, hcap))
+
+    def ingest_xwindow(self, w):
+        """Ingest this rank's own receive window after every rank's Map completed."""
+        self._recv = (w,)
+        self._check(lib().mr_ingest_xwindow(self.h, _ptr(w.entries), _ptr(w.heap), _ptr(w.cursor),
+                                            w.entry_cap, w.heap_cap))
 
     def shuffle(self, group=None):
         """One all-to-all exchange over torch.distributed (NCCL on GPUs): partition -> exchange

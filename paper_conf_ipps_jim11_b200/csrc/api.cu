@@ -340,6 +340,8 @@ struct mr_job {
   DBuf<unsigned long long> xcounts, xcursors, xheapbase;
   HBuf<unsigned long long> xcounts_h;
   DBuf<uint64_t> src_e, src_h;
+  DBuf<XWindow> xwin;             // f-3: receive windows of the fused Map flush (InvertedIndex)
+  uint32_t xranks = 0;
   DBuf<uint32_t> km_list;
   uint32_t km_nlist = 0;
   uint64_t out_keys_bytes = 0, out_vals_bytes = 0, out_n = 0;
@@ -430,6 +432,8 @@ cudaError_t launch_batch(mr_job* job, const Batch& b) {
   a.st = job->st;
   a.hash_seed = 0x5EEDB200ULL;
   a.key_bits = job->key_bits;
+  a.xwin = job->xranks ? job->xwin.p : nullptr;
+  a.xranks = job->xranks;
   const uint64_t nt = map_tiles(a);
   if (a.workload != kKM) {
     cudaError_t e = job->tb.ensure(2 * nt + 2);
@@ -1317,6 +1321,51 @@ mr_status mr_ingest(mr_job* job, const void* entries, const void* heap, const ui
   return MR_OK;
 }
 
+mr_status mr_set_xwindows(mr_job* job, uint32_t nranks, void* const* entries, void* const* heaps,
+                          uint64_t* const* cursors, uint64_t entry_cap, uint64_t heap_cap) {
+  if (!job) return MR_ERR_INVALID;
+  if (nranks == 0) { job->xranks = 0; return MR_OK; }
+  if (job->cfg.workload != MR_INVINDEX) return fail(job, MR_ERR_INVALID, "fused windows: InvertedIndex only");
+  if (nranks > static_cast<uint32_t>(kMaxRanks) || !entries || !heaps || !cursors)
+    return fail(job, MR_ERR_INVALID, "bad window arrays");
+  if (job->state != kCreated) return fail(job, MR_ERR_STATE, "mr_set_xwindows after mr_map");
+  std::vector<XWindow> w(nranks);
+  for (uint32_t r = 0; r < nranks; ++r) {
+    if (!entries[r] || !heaps[r] || !cursors[r] || (reinterpret_cast<uintptr_t>(entries[r]) & 15u) ||
+        (reinterpret_cast<uintptr_t>(heaps[r]) & 7u) || (reinterpret_cast<uintptr_t>(cursors[r]) & 7u))
+      return fail(job, MR_ERR_INVALID, "window pointer NULL or misaligned");
+    w[r] = XWindow{static_cast<uint8_t*>(entries[r]), static_cast<uint8_t*>(heaps[r]),
+                   reinterpret_cast<unsigned long long*>(cursors[r]), entry_cap, heap_cap};
+  }
+  CK(cudaSetDevice(job->cfg.device), "set device");
+  CK(job->xwin.ensure(nranks), "alloc windows");
+  CK(cudaMemcpyAsync(job->xwin.p, w.data(), nranks * sizeof(XWindow), cudaMemcpyHostToDevice, job->stream),
+     "H2D windows");
+  CK(cudaStreamSynchronize(job->stream), "sync windows");
+  job->xranks = nranks;
+  return MR_OK;
+}
+
+mr_status mr_ingest_xwindow(mr_job* job, const void* entries, const void* heap, const uint64_t* cursor,
+                            uint64_t entry_cap, uint64_t heap_cap) {
+  if (!job || !cursor) return MR_ERR_INVALID;
+  if (job->cfg.workload != MR_INVINDEX) return fail(job, MR_ERR_INVALID, "fused windows: InvertedIndex only");
+  if (job->state != kMapped && job->state != kCreated)
+    return fail(job, MR_ERR_STATE, "mr_ingest_xwindow after mr_group");
+  CK(cudaSetDevice(job->cfg.device), "set device");
+  uint64_t c[2] = {0, 0};
+  CK(cudaMemcpy(c, cursor, sizeof(c), cudaMemcpyDeviceToHost), "D2H window cursor");
+  if (c[0] > entry_cap || c[1] > heap_cap)
+    return fail(job, MR_ERR_OOM, "receive window overflow: " + std::to_string(c[0]) + " entries / " +
+                                          std::to_string(c[1]) + " heap bytes needed");
+  const uint32_t R = static_cast<uint32_t>(std::max(1, job->cfg.nranks));
+  std::vector<uint64_t> counts(2 * R, 0);
+  counts[0] = c[0];   // one contiguous block (source order is irrelevant after the sort)
+  counts[1] = c[1];
+  job->state = kPartitioned;
+  return mr_ingest(job, entries, heap, counts.data());
+}
+
 mr_status mr_get_stats(const mr_job* job, void* stats, size_t bytes) {
   if (!job || !stats) return MR_ERR_INVALID;
   mr_stats st = job->stats;
@@ -1335,7 +1384,7 @@ mr_status mr_job_destroy(mr_job* job) {
   for (auto& b : job->host_off) b.release();
   job->prof.release();
   job->xcounts.release(); job->xcursors.release(); job->xheapbase.release(); job->xcounts_h.release();
-  job->src_e.release(); job->src_h.release(); job->km_list.release();
+  job->src_e.release(); job->src_h.release(); job->km_list.release(); job->xwin.release();
   job->cent.release(); release_pairs(job); job->tb.release();
   job->swp.release(); job->seg_startp.release(); job->psum.release(); job->pxcounts.release();
   job->midx.release(); job->xkeys.release();

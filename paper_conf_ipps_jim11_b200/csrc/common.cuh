@@ -159,6 +159,13 @@ __device__ __forceinline__ uint64_t hash_bytes(const uint8_t* p, uint32_t len, u
   }
   return hs.finish();
 }
+
+// Destination rank of a key in the multi-GPU exchange: from the key BYTES, so it is
+// the same on every rank and for every code path (partition pass, fused Map flush).
+constexpr uint64_t kPartSeed = 0x9A27D11EB200ULL;
+__device__ __forceinline__ uint32_t dest_of_bytes(const uint8_t* p, uint32_t len, uint32_t R) {
+  return static_cast<uint32_t>(mix64(hash_bytes(p, len, kPartSeed) ^ 0x51ULL) % R);
+}
 // Sort-key formats.  The key width is 64 bits (II, re-hash slow path) or 48 bits (WC: two LSD
 // passes fewer; digits 6 and 7 are then constant and skipped):
 //   inline  : keys of <= kInlineMax bytes packed little-endian, length in the 3 bits above them

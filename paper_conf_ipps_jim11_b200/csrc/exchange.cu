@@ -18,12 +18,7 @@
 namespace bmr {
 namespace {
 
-constexpr uint64_t kPartSeed = 0x9A27D11EB200ULL;
 constexpr int kXThreads = 256;
-
-__device__ __forceinline__ uint32_t dest_of_bytes(const uint8_t* p, uint32_t len, uint32_t R) {
-  return static_cast<uint32_t>(mix64(hash_bytes(p, len, kPartSeed) ^ 0x51ULL) % R);
-}
 __device__ __forceinline__ uint32_t dest_of_id(uint64_t id, uint32_t R) {
   return static_cast<uint32_t>(mix64(id ^ kPartSeed) % R);
 }

@@ -57,6 +57,16 @@ struct PairBufs {
   uint64_t cap_c = 0;
 };
 
+// f-3 fused exchange: a destination rank's receive window (device pointers valid in this
+// process: a peer GPU's buffers opened through CUDA IPC, or same-GPU buffers for virtual ranks).
+// cursor[0] = entries appended, cursor[1] = heap bytes appended (demand, may pass the capacity).
+struct XWindow {
+  uint8_t* entries;                 // XEntry[ecap]
+  uint8_t* heap;                    // key bytes, hcap bytes (8-B aligned records)
+  unsigned long long* cursor;       // 2 x u64
+  uint64_t ecap, hcap;
+};
+
 struct MapArgs {
   int workload = 0;
   uint32_t flags = 0;
@@ -75,6 +85,8 @@ struct MapArgs {
   uint64_t hash_seed = 0;
   uint32_t key_bits = 64;             // sort-key width of hashed / inline keys (48 or 64)
   int grid = 0;                       // persistent CTAs (0 = one per SM)
+  const XWindow* xwin = nullptr;      // f-3: InvertedIndex records go straight to these R windows
+  uint32_t xranks = 0;
 };
 
 int vbytes_of(int workload);                 // value bytes per pair (WC Map output: none, value 1)

@@ -247,6 +247,8 @@ struct Params {
   uint32_t so, si;
   uint32_t sm_lines;       // StringMatch: emit the matching record's start (MR_FLAG_SM_LINES)
   uint32_t wc_bal;         // WordCount: balanced two-phase emission (BMR_WC_BAL, default on)
+  const XWindow* xwin;     // f-3: InvertedIndex records appended straight to these windows
+  uint32_t xranks;         // number of windows (0: local output)
 };
 
 // Idle wait of a role warp on an mbarrier phase (map warps on a staged tile, producers on a free
@@ -1053,6 +1055,58 @@ __device__ __forceinline__ uint64_t* ii_qpos(uint8_t* outh) {
   return reinterpret_cast<uint64_t*>(outh + (Layout<kII>::hq - Layout<kII>::out)) +
          (threadIdx.x >> 5) * (Cfg<kII>::kHashQ / 2);
 }
+// f-3: fused Map flush + shuffle.  The drained URLs go straight to the receive
+// window of their destination rank (dest_of_bytes of the URL bytes, as in the partition pass):
+// per destination one pair of atomics per warp (entries, heap bytes) on the window's cursor —
+// over NVLink when the window lives on a peer GPU — then the 16-B entry and the key bytes are
+// stored into it.  No local pairs, no partition pass, no all-to-all: the transfer overlaps the
+// Map.  Demand past a window's capacity is still counted (mr_ingest_xwindow reports it).
+__device__ void ii_drain_xwin(const Params& P, uint32_t qn, const uint64_t* qpos, const uint32_t* qlen) {
+  const uint32_t lane = threadIdx.x & 31;
+  for (uint32_t e0 = 0; e0 < qn; e0 += 32) {
+    const uint32_t e = e0 + lane;
+    const bool in = e < qn;
+    const long long q0 = in ? static_cast<long long>(qpos[e]) : 0;
+    const uint32_t len = in ? qlen[e] : 0u;
+    const uint8_t* kp = P.rec + q0;
+    const uint32_t d = in ? dest_of_bytes(kp, len, P.xranks) : ~0u;
+    const uint32_t hb = (len + 7u) & ~7u;
+    unsigned long long ie = 0, ih = 0;
+    for (uint32_t r = 0; r < P.xranks; ++r) {
+      const uint32_t m = __ballot_sync(kFull, d == r);
+      if (!m) continue;
+      const uint32_t hv = d == r ? hb : 0u;
+      const uint32_t incl = warp_inclusive_add(hv);
+      const uint32_t tot = __shfl_sync(kFull, incl, 31);
+      const uint32_t leader = __ffs(m) - 1;
+      unsigned long long be = 0, bh = 0;
+      if (lane == leader) {
+        be = atomicAdd(P.xwin[r].cursor, static_cast<unsigned long long>(__popc(m)));
+        bh = atomicAdd(P.xwin[r].cursor + 1, static_cast<unsigned long long>(tot));
+      }
+      be = __shfl_sync(kFull, be, leader);
+      bh = __shfl_sync(kFull, bh, leader);
+      if (d == r) {
+        ie = be + __popc(m & lanemask_lt());
+        ih = bh + incl - hv;
+      }
+    }
+    if (in) {
+      const XWindow w = P.xwin[d];
+      if (ie < w.ecap && ih + hb <= w.hcap) {
+        XEntry* o = reinterpret_cast<XEntry*>(w.entries) + ie;
+        o->koff_len = (static_cast<uint64_t>(ih) << 16) | len;
+        o->v = P.gbase + static_cast<uint64_t>(q0);
+        for (uint32_t k = 0; k < len; k += 8) {   // heap records are 8-B aligned
+          uint64_t b = 0;
+          for (uint32_t t = 0; t < 8 && k + t < len; ++t) b |= static_cast<uint64_t>(kp[k + t]) << (8 * t);
+          *reinterpret_cast<uint64_t*>(w.heap + ih + k) = b;
+        }
+      }
+    }
+  }
+}
+
 __device__ void ii_drain(const Params& P, OutCtl* oc, uint8_t* outh, uint32_t& qn) {
   using F = PairFmt<kII>;
   if (qn == 0) return;
@@ -1060,6 +1114,12 @@ __device__ void ii_drain(const Params& P, OutCtl* oc, uint8_t* outh, uint32_t& q
   const uint64_t* qpos = ii_qpos(outh);
   const uint32_t* qlen = reinterpret_cast<const uint32_t*>(qpos + 64);
   __syncwarp();
+  if (P.xranks) {
+    ii_drain_xwin(P, qn, qpos, qlen);
+    __syncwarp();
+    qn = 0;
+    return;
+  }
   const Slot slot = reserve<kII>(P, oc, outh, qn, P.out_cap);
   uint8_t* half = outh + slot.half * Cfg<kII>::kOutHalf;
   uint64_t* sh = reinterpret_cast<uint64_t*>(half);
@@ -1259,7 +1319,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
     return;
   }
   if constexpr (W == kII) {
-    if (!P.si) {   // queue the URLs (drained lane-parallel, see ii_drain)
+    if (!P.si || P.xranks) {   // queue the URLs (drained lane-parallel, see ii_drain)
       const uint32_t cnt = __popc(emit_mask);   // <= 2 markers start in 16 bytes
       const uint32_t incl = warp_inclusive_add(cnt);
       const uint32_t tot = __shfl_sync(kFull, incl, 31);
@@ -1824,6 +1884,8 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
                         : nullptr;
   P.hash_seed = a.hash_seed;
   P.key_bits = a.key_bits;
+  P.xwin = a.xwin;
+  P.xranks = (W == kII) ? a.xranks : 0u;
   P.ohb = a.out.hb;
   P.okrefb = a.out.krefb;
   P.cap_b = a.out.cap_b;

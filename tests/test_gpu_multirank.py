@@ -122,3 +122,55 @@ def test_km_multirank(R):
     assert np.array_equal(cnt, no)
     floor = np.abs(pts.astype(np.float64)).mean(0)
     assert np.all(np.abs(cen.astype(np.float64) - co) <= 1e-5 * np.maximum(np.abs(co), floor[None]))
+
+
+def run_fused_ii(shards, R, entry_cap=1 << 20, heap_cap=64 << 20):
+    """f-3: every rank's Map appends its records straight into the destination ranks' receive
+    windows (here all on one GPU); after all Maps, every rank ingests its own window."""
+    wins = [bmr.XWindow(entry_cap, heap_cap) for _ in range(R)]
+    jobs, keep = [], []
+    for r in range(R):
+        g = shards[r]
+        job = bmr.Job("ii", rank=r, nranks=R, input_base=g["base"])
+        job.set_xwindows(wins)
+        d = torch.from_numpy(g["data"]).cuda()
+        o = torch.from_numpy(g["offsets"].view(np.int64)).cuda()
+        keep.append((d, o))
+        job.map(d, o, g["n"])
+        jobs.append(job)
+    torch.cuda.synchronize()   # every rank's Map (and so every window) is complete
+    return jobs, wins, keep
+
+
+@pytest.mark.parametrize("R", [1, 2, 3])
+def test_ii_fused_xwindows(R):
+    spec = pygen.spec_ii(4)
+    sh = shards_text(spec, 6, R)
+    jobs, wins, keep = run_fused_ii(sh, R)
+    outs = []
+    for r in range(R):
+        jobs[r].ingest_xwindow(wins[r])
+    for job in jobs:
+        job.group()
+        job.reduce()
+        outs.append(job.fetch())
+        job.close()
+    got = union_dict(outs, "ii")
+    whole = pygen.host_text(spec, 6)
+    res = oracle.run("ii", [(whole["data"], whole["offsets"], whole["n"], 0, 0)])
+    exp = decode("ii", res)
+    assert got == exp
+    # every record left through a window, and only there
+    assert sum(w.used()[0] for w in wins) == sum(len(v) for v in exp.values())
+    # the same records as the partition + all-to-all path
+    assert got == union_dict(run_virtual("ii", sh, R), "ii")
+
+
+def test_ii_fused_xwindow_overflow():
+    spec = pygen.spec_ii(4)
+    sh = shards_text(spec, 2, 2)
+    jobs, wins, keep = run_fused_ii(sh, 2, entry_cap=16, heap_cap=1 << 20)
+    with pytest.raises(bmr.MRError, match="MR_ERR_OOM"):
+        jobs[0].ingest_xwindow(wins[0])
+    for job in jobs:
+        job.close()
