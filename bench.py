@@ -232,6 +232,9 @@ def main():
     ap.add_argument("--mode", default="SIO", choices=["SIO", "SO", "SI", "G"],
                     help="Map memory-usage mode (PAPER.md L129-135 ablation, SURVEY §8(f) f-2)")
     ap.add_argument("--no-map-combine", action="store_true", help="literal north-star order (no Map combiner)")
+    ap.add_argument("--xchg", default="a2a", choices=["a2a", "fused"],
+                    help="InvertedIndex exchange: partition + all-to-all (a2a) or the fused Map flush into "
+                         "receive windows (f-3; one GPU: the rank's own window, timed with its ingest)")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -268,10 +271,22 @@ def main():
     stream = torch.cuda.current_stream()
     exchange = world > 1 and inp["wl"] != "sm"      # SM is Map-only: no exchange
     xbytes = [0]
+    xwin = None
+    if args.xchg == "fused":
+        if inp["wl"] != "ii" or world > 1:
+            raise SystemExit("--xchg fused: InvertedIndex on one GPU (multi-GPU windows need CUDA IPC plumbing)")
+        xwin = bmr.XWindow(inp["nbytes"] // 48 + 4096, inp["nbytes"] // 4 + 65536, device=torch.device(dev))
+        job.set_xwindows([xwin])
+        exchange = False
 
     def step():
         job.reset()
-        job.map(inp["data"], inp["offsets"], inp["n"])
+        if xwin is not None:   # f-3: the Map's flush appends the records to the window, then ingest
+            xwin.reset()
+            job.map(inp["data"], inp["offsets"], inp["n"])
+            job.ingest_xwindow(xwin)
+        else:
+            job.map(inp["data"], inp["offsets"], inp["n"])
         if exchange:  # one hash all-to-all over NCCL
             xbytes[0] = job.shuffle()
         job.group()
@@ -428,7 +443,9 @@ def main():
             "distinct_keys": int(tot["n_keys"] / args.steps),
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "exchange": ({"kind": "hash all-to-all over NCCL (torch.distributed)", "send_bytes_per_rank": xbytes[0],
-                          "combiner": inp["wl"] in ("wc", "km")} if exchange else None),
+                          "combiner": inp["wl"] in ("wc", "km")} if exchange else
+                         ({"kind": "fused Map flush into the receive window (f-3), one rank",
+                           "window_entries_heap": list(xwin.used())} if xwin is not None else None)),
             "gpu_launches": int(tot["kernel_launches"]),
             "clocks": clk.summary(), "wall_s_timed": round(wall, 3),
             "step_ms": {"min": round(min(step_ms), 3), "median": round(statistics.median(step_ms), 3),

@@ -160,11 +160,38 @@ __device__ __forceinline__ uint64_t hash_bytes(const uint8_t* p, uint32_t len, u
   return hs.finish();
 }
 
+// `need` (1..8) bytes at p, little-endian, from 8-byte aligned loads only (never touching an
+// 8-byte word that holds none of the needed bytes); bytes beyond `need` are unspecified.
+__device__ __forceinline__ uint64_t load8(const uint8_t* p, uint32_t need) {
+  const uintptr_t a = reinterpret_cast<uintptr_t>(p) & ~static_cast<uintptr_t>(7);
+  const uint32_t sh = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(p) & 7u) * 8;
+  const uint64_t w0 = __ldg(reinterpret_cast<const unsigned long long*>(a));
+  if (sh == 0) return w0;
+  uint64_t v = w0 >> sh;
+  if (sh / 8 + need > 8) v |= static_cast<uint64_t>(__ldg(reinterpret_cast<const unsigned long long*>(a + 8))) << (64 - sh);
+  return v;
+}
+// hash_bytes of key bytes in global memory, read 8 bytes at a time (same words, same result).
+__device__ __forceinline__ uint64_t hash_bytes_g(const uint8_t* p, uint32_t len, uint64_t seed) {
+  KeyHash hs(seed, len);
+  for (uint32_t k = 0; k < len; k += 8) {
+    const uint32_t need = min(8u, len - k);
+    uint64_t v = load8(p + k, need);
+    if (need < 8) v &= (1ULL << (8 * need)) - 1ULL;
+    hs.add(static_cast<uint32_t>(v));
+    if (k + 4 < len) hs.add(static_cast<uint32_t>(v >> 32));
+  }
+  return hs.finish();
+}
+
 // Destination rank of a key in the multi-GPU exchange: from the key BYTES, so it is
 // the same on every rank and for every code path (partition pass, fused Map flush).
 constexpr uint64_t kPartSeed = 0x9A27D11EB200ULL;
 __device__ __forceinline__ uint32_t dest_of_bytes(const uint8_t* p, uint32_t len, uint32_t R) {
   return static_cast<uint32_t>(mix64(hash_bytes(p, len, kPartSeed) ^ 0x51ULL) % R);
+}
+__device__ __forceinline__ uint32_t dest_of_bytes_g(const uint8_t* p, uint32_t len, uint32_t R) {   // global p
+  return static_cast<uint32_t>(mix64(hash_bytes_g(p, len, kPartSeed) ^ 0x51ULL) % R);
 }
 // Sort-key formats.  The key width is 64 bits (II, re-hash slow path) or 48 bits (WC: two LSD
 // passes fewer; digits 6 and 7 are then constant and skipped):

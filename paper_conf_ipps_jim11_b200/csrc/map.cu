@@ -1069,7 +1069,7 @@ __device__ void ii_drain_xwin(const Params& P, uint32_t qn, const uint64_t* qpos
     const long long q0 = in ? static_cast<long long>(qpos[e]) : 0;
     const uint32_t len = in ? qlen[e] : 0u;
     const uint8_t* kp = P.rec + q0;
-    const uint32_t d = in ? dest_of_bytes(kp, len, P.xranks) : ~0u;
+    const uint32_t d = in ? dest_of_bytes_g(kp, len, P.xranks) : ~0u;
     const uint32_t hb = (len + 7u) & ~7u;
     unsigned long long ie = 0, ih = 0;
     for (uint32_t r = 0; r < P.xranks; ++r) {
@@ -1097,11 +1097,8 @@ __device__ void ii_drain_xwin(const Params& P, uint32_t qn, const uint64_t* qpos
         XEntry* o = reinterpret_cast<XEntry*>(w.entries) + ie;
         o->koff_len = (static_cast<uint64_t>(ih) << 16) | len;
         o->v = P.gbase + static_cast<uint64_t>(q0);
-        for (uint32_t k = 0; k < len; k += 8) {   // heap records are 8-B aligned
-          uint64_t b = 0;
-          for (uint32_t t = 0; t < 8 && k + t < len; ++t) b |= static_cast<uint64_t>(kp[k + t]) << (8 * t);
-          *reinterpret_cast<uint64_t*>(w.heap + ih + k) = b;
-        }
+        for (uint32_t k = 0; k < len; k += 8)   // heap records are 8-B aligned
+          *reinterpret_cast<uint64_t*>(w.heap + ih + k) = load8(kp + k, min(8u, len - k));
       }
     }
   }

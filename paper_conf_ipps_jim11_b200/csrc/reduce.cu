@@ -35,15 +35,6 @@ __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
 
 // 8 key bytes starting at p (little-endian); reads only the aligned 8-byte words that hold
 // bytes [p, p + need), need <= 8, so it never touches a word outside the key's own words.
-__device__ __forceinline__ uint64_t load8(const uint8_t* p, uint32_t need) {
-  const uintptr_t a = reinterpret_cast<uintptr_t>(p) & ~static_cast<uintptr_t>(7);
-  const uint32_t sh = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(p) & 7u) * 8;
-  const uint64_t w0 = __ldg(reinterpret_cast<const unsigned long long*>(a));
-  if (sh == 0) return w0;
-  uint64_t v = w0 >> sh;
-  if (sh / 8 + need > 8) v |= static_cast<uint64_t>(__ldg(reinterpret_cast<const unsigned long long*>(a + 8))) << (64 - sh);
-  return v;
-}
 
 // Byte equality of two keys given as kref = (address << 16) | length.
 __device__ bool key_bytes_equal(uint64_t ka, uint64_t kb) {
