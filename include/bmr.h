@@ -214,6 +214,21 @@ mr_status mr_set_xwindows(mr_job* job, uint32_t nranks, void* const* entries, vo
 mr_status mr_ingest_xwindow(mr_job* job, const void* entries, const void* heap, const uint64_t* cursor,
                             uint64_t entry_cap, uint64_t heap_cap);
 
+/* Device memory and CUDA IPC helpers for windows shared between processes (one per GPU):
+ * mr_dev_alloc: cudaMalloc of >= bytes on `device` (a whole allocation, so its IPC handle maps
+ * it at offset 0; MR_ERR_OOM).  mr_dev_free / mr_dev_zero / mr_dev_copy (synchronous,
+ * cudaMemcpyDefault).  mr_ipc_handle: the MR_IPC_HANDLE_BYTES-byte handle of an mr_dev_alloc
+ * pointer (host buffer out).  mr_ipc_open: maps another process's handle on `device` (peer
+ * access enabled lazily: NVLink on B200 boxes); mr_ipc_close unmaps.  Failures -> MR_ERR_CUDA. */
+#define MR_IPC_HANDLE_BYTES 64
+mr_status mr_dev_alloc(int device, uint64_t bytes, void** dptr);
+mr_status mr_dev_free(void* dptr);
+mr_status mr_dev_zero(void* dptr, uint64_t bytes);
+mr_status mr_dev_copy(void* dst, const void* src, uint64_t bytes);
+mr_status mr_ipc_handle(const void* dptr, void* handle);
+mr_status mr_ipc_open(int device, const void* handle, void** dptr);
+mr_status mr_ipc_close(void* dptr);
+
 /* Group-by primitive exposed for testing (§8(a) a7): stable LSD radix sort of n u64 device
  * keys; writes the sorted keys and the u32 permutation (perm[i] = source index of the i-th
  * key).  Synchronises `stream`. n < 2^32. */

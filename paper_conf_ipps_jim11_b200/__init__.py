@@ -30,28 +30,88 @@ STATUS = {0: "MR_OK", 1: "MR_ERR_INVALID", 2: "MR_ERR_STATE", 3: "MR_ERR_OOM", 4
 
 EXPORTS = ("mr_job_create", "mr_map", "mr_map_host", "mr_map_host_lines", "mr_group", "mr_reduce", "mr_fetch", "mr_job_reset",
            "mr_get_stats", "mr_job_destroy", "mr_status_string", "mr_last_error", "mr_sort_u64",
-           "mr_partition_count", "mr_partition_write", "mr_ingest", "mr_set_xwindows", "mr_ingest_xwindow")
+           "mr_partition_count", "mr_partition_write", "mr_ingest", "mr_set_xwindows", "mr_ingest_xwindow",
+           "mr_dev_alloc", "mr_dev_free", "mr_dev_zero", "mr_dev_copy", "mr_ipc_handle", "mr_ipc_open", "mr_ipc_close")
 
 
 class XWindow:
-    """A receive window of the fused Map flush (f-3): device buffers for entry_cap 16-byte entries,
-    heap_cap key bytes and the 2 x u64 cursor, owned here (torch tensors on `device`)."""
+    """A receive window of the fused Map flush (f-3): entry_cap 16-byte entries, heap_cap key bytes
+    and the 2 x u64 cursor.  ipc=False: torch tensors on `device` (same-process ranks); ipc=True:
+    one mr_dev_alloc block [cursor | entries | heap] whose CUDA IPC handle other processes open
+    (XWindow.open_peer), so their Maps store into it over NVLink."""
 
-    def __init__(self, entry_cap: int, heap_cap: int, device=None):
+    _HDR = 256
+
+    def __init__(self, entry_cap: int, heap_cap: int, device=None, ipc: bool = False):
         import torch
         dev = device if device is not None else torch.device("cuda", torch.cuda.current_device())
         self.entry_cap, self.heap_cap = int(entry_cap), int(heap_cap)
-        self.entries = torch.empty(max(self.entry_cap, 1) * 16, dtype=torch.uint8, device=dev)
-        self.heap = torch.empty(max(self.heap_cap, 8), dtype=torch.uint8, device=dev)
-        self.cursor = torch.zeros(2, dtype=torch.int64, device=dev)
+        self.ipc, self.peer, self._base = ipc, False, 0
+        if not ipc:
+            self.entries = torch.empty(max(self.entry_cap, 1) * 16, dtype=torch.uint8, device=dev)
+            self.heap = torch.empty(max(self.heap_cap, 8), dtype=torch.uint8, device=dev)
+            self.cursor = torch.zeros(2, dtype=torch.int64, device=dev)
+            self.entries_ptr, self.heap_ptr = self.entries.data_ptr(), self.heap.data_ptr()
+            self.cursor_ptr = self.cursor.data_ptr()
+            return
+        self.device = dev.index if dev.index is not None else torch.cuda.current_device()
+        p = C.c_void_p()
+        st = lib().mr_dev_alloc(self.device, self._bytes(), C.byref(p))
+        if st:
+            raise MRError(st, "mr_dev_alloc")
+        self._base = p.value
+        self._set_ptrs(self._base)
+        self.reset()
+
+    def _bytes(self):
+        return self._HDR + max(self.entry_cap, 1) * 16 + ((max(self.heap_cap, 8) + 255) // 256) * 256
+
+    def _set_ptrs(self, base):
+        self.cursor_ptr = base
+        self.entries_ptr = base + self._HDR
+        self.heap_ptr = base + self._HDR + max(self.entry_cap, 1) * 16
+
+    def ipc_handle(self) -> bytes:
+        """(handle bytes, entry_cap, heap_cap) for another process to open this window."""
+        h = C.create_string_buffer(64)
+        st = lib().mr_ipc_handle(self._base, h)
+        if st:
+            raise MRError(st, "mr_ipc_handle")
+        return h.raw
+
+    @classmethod
+    def open_peer(cls, handle: bytes, entry_cap: int, heap_cap: int, device: int):
+        """Map another process's window (its ipc_handle) into this process."""
+        w = cls.__new__(cls)
+        w.entry_cap, w.heap_cap, w.ipc, w.peer, w.device = int(entry_cap), int(heap_cap), True, True, device
+        p = C.c_void_p()
+        st = lib().mr_ipc_open(device, C.create_string_buffer(handle, 64), C.byref(p))
+        if st:
+            raise MRError(st, "mr_ipc_open")
+        w._base = p.value
+        w._set_ptrs(w._base)
+        return w
 
     def reset(self):
-        self.cursor.zero_()
+        if self.ipc:
+            st = lib().mr_dev_zero(self.cursor_ptr, 16)
+            if st:
+                raise MRError(st, "mr_dev_zero")
+        else:
+            self.cursor.zero_()
 
     def used(self):
         """(entries, heap bytes) appended so far (demand; may exceed the capacity)."""
-        c = self.cursor.cpu().tolist()
+        c = np.zeros(2, np.uint64)
+        st = lib().mr_dev_copy(c.ctypes.data, self.cursor_ptr, 16)
+        if st:
+            raise MRError(st, "mr_dev_copy")
         return int(c[0]), int(c[1])
+
+    def close(self):
+        if self.ipc and self._base:
+            (lib().mr_ipc_close if self.peer else lib().mr_dev_free)(self._base)
+            self._base = 0
 
 
 class MRError(RuntimeError):
@@ -118,6 +178,13 @@ def lib() -> C.CDLL:
         L.mr_ingest.argtypes = [vp, vp, vp, vp]
         L.mr_set_xwindows.argtypes = [vp, C.c_uint32, vp, vp, vp, u64, u64]
         L.mr_ingest_xwindow.argtypes = [vp, vp, vp, vp, u64, u64]
+        L.mr_dev_alloc.argtypes = [C.c_int, u64, vp]
+        L.mr_dev_free.argtypes = [vp]
+        L.mr_dev_zero.argtypes = [vp, u64]
+        L.mr_dev_copy.argtypes = [vp, vp, u64]
+        L.mr_ipc_handle.argtypes = [vp, vp]
+        L.mr_ipc_open.argtypes = [C.c_int, vp, vp]
+        L.mr_ipc_close.argtypes = [vp]
         for f in EXPORTS:
             if f not in ("mr_status_string", "mr_last_error"):
                 getattr(L, f).restype = C.c_int
@@ -257,9 +324,9 @@ class Job:
         map(): InvertedIndex records then leave the Map straight through them."""
         n = len(windows)
         arr = (C.c_void_p * max(n, 1))
-        ents = arr(*[w.entries.data_ptr() for w in windows])
-        heaps = arr(*[w.heap.data_ptr() for w in windows])
-        curs = arr(*[w.cursor.data_ptr() for w in windows])
+        ents = arr(*[w.entries_ptr for w in windows])
+        heaps = arr(*[w.heap_ptr for w in windows])
+        curs = arr(*[w.cursor_ptr for w in windows])
         ecap = windows[0].entry_cap if n else 0
         hcap = windows[0].heap_cap if n else 0
         self._xwin = list(windows)
@@ -269,8 +336,7 @@ class Job:
     def ingest_xwindow(self, w):
         """Ingest this rank's own receive window after every rank's Map completed."""
         self._recv = (w,)
-        self._check(lib().mr_ingest_xwindow(self.h, _ptr(w.entries), _ptr(w.heap), _ptr(w.cursor),
-                                            w.entry_cap, w.heap_cap))
+        self._check(lib().mr_ingest_xwindow(self.h, w.entries_ptr, w.heap_ptr, w.cursor_ptr, w.entry_cap, w.heap_cap))
 
     def shuffle(self, group=None):
         """One all-to-all exchange over torch.distributed (NCCL on GPUs): partition -> exchange

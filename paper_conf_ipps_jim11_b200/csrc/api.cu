@@ -1366,6 +1366,54 @@ mr_status mr_ingest_xwindow(mr_job* job, const void* entries, const void* heap, 
   return mr_ingest(job, entries, heap, counts.data());
 }
 
+// ---- device memory + CUDA IPC helpers for receive windows shared between processes ----
+mr_status mr_dev_alloc(int device, uint64_t bytes, void** dptr) {
+  if (!dptr) return MR_ERR_INVALID;
+  *dptr = nullptr;
+  if (cudaSetDevice(device) != cudaSuccess) { cudaGetLastError(); return MR_ERR_CUDA; }
+  if (cudaMalloc(dptr, std::max<uint64_t>(bytes, 256)) != cudaSuccess) { cudaGetLastError(); *dptr = nullptr; return MR_ERR_OOM; }
+  return MR_OK;
+}
+mr_status mr_dev_free(void* dptr) {
+  if (dptr && cudaFree(dptr) != cudaSuccess) { cudaGetLastError(); return MR_ERR_CUDA; }
+  return MR_OK;
+}
+mr_status mr_dev_copy(void* dst, const void* src, uint64_t bytes) {   // synchronous, any direction
+  if (bytes && (!dst || !src)) return MR_ERR_INVALID;
+  if (bytes && cudaMemcpy(dst, src, bytes, cudaMemcpyDefault) != cudaSuccess) { cudaGetLastError(); return MR_ERR_CUDA; }
+  return MR_OK;
+}
+mr_status mr_dev_zero(void* dptr, uint64_t bytes) {
+  if (bytes && !dptr) return MR_ERR_INVALID;
+  if (bytes && cudaMemset(dptr, 0, bytes) != cudaSuccess) { cudaGetLastError(); return MR_ERR_CUDA; }
+  return MR_OK;
+}
+mr_status mr_ipc_handle(const void* dptr, void* handle) {
+  if (!dptr || !handle) return MR_ERR_INVALID;
+  cudaIpcMemHandle_t h;
+  if (cudaIpcGetMemHandle(&h, const_cast<void*>(dptr)) != cudaSuccess) { cudaGetLastError(); return MR_ERR_CUDA; }
+  static_assert(sizeof(h) == MR_IPC_HANDLE_BYTES, "IPC handle size");
+  std::memcpy(handle, &h, sizeof(h));
+  return MR_OK;
+}
+mr_status mr_ipc_open(int device, const void* handle, void** dptr) {
+  if (!handle || !dptr) return MR_ERR_INVALID;
+  *dptr = nullptr;
+  cudaIpcMemHandle_t h;
+  std::memcpy(&h, handle, sizeof(h));
+  if (cudaSetDevice(device) != cudaSuccess) { cudaGetLastError(); return MR_ERR_CUDA; }
+  if (cudaIpcOpenMemHandle(dptr, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+    cudaGetLastError();
+    *dptr = nullptr;
+    return MR_ERR_CUDA;
+  }
+  return MR_OK;
+}
+mr_status mr_ipc_close(void* dptr) {
+  if (dptr && cudaIpcCloseMemHandle(dptr) != cudaSuccess) { cudaGetLastError(); return MR_ERR_CUDA; }
+  return MR_OK;
+}
+
 mr_status mr_get_stats(const mr_job* job, void* stats, size_t bytes) {
   if (!job || !stats) return MR_ERR_INVALID;
   mr_stats st = job->stats;

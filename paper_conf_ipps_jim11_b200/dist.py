@@ -40,3 +40,17 @@ def _dev(group):
     if dist.get_backend(group) == "nccl":
         return torch.device("cuda", torch.cuda.current_device())
     return torch.device("cpu")
+
+
+def open_xwindows(own, group=None):
+    """f-3 plumbing: every rank publishes the CUDA IPC handle of its own receive window (an
+    XWindow(ipc=True)) with one all_gather_object; returns the rank-ordered window list for
+    Job.set_xwindows (own window for this rank, mapped peer windows for the others).  Close the
+    peer windows (XWindow.close) after the last Map that uses them."""
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    mine = (own.ipc_handle(), own.entry_cap, own.heap_cap)
+    alls = [None] * world
+    dist.all_gather_object(alls, mine, group=group)
+    from . import XWindow
+    return [own if r == rank else XWindow.open_peer(h, ec, hc, own.device) for r, (h, ec, hc) in enumerate(alls)]
