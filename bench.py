@@ -273,17 +273,28 @@ def main():
     xbytes = [0]
     xwin = None
     if args.xchg == "fused":
-        if inp["wl"] != "ii" or world > 1:
-            raise SystemExit("--xchg fused: InvertedIndex on one GPU (multi-GPU windows need CUDA IPC plumbing)")
-        xwin = bmr.XWindow(inp["nbytes"] // 48 + 4096, inp["nbytes"] // 4 + 65536, device=torch.device(dev))
-        job.set_xwindows([xwin])
+        if inp["wl"] != "ii":
+            raise SystemExit("--xchg fused: InvertedIndex only")
+        # every rank's receive window holds what all ranks may send it (uniform hash partition;
+        # 2x headroom for skew)
+        ecap = 2 * inp["nbytes"] // 48 + 4096
+        hcap = 2 * inp["nbytes"] // 4 + 65536
+        if world > 1:   # windows shared through CUDA IPC: the Maps store into peers over NVLink
+            from paper_conf_ipps_jim11_b200 import dist as D
+            xwin = bmr.XWindow(ecap, hcap, device=torch.device(dev), ipc=True)
+            job.set_xwindows(D.open_xwindows(xwin))
+        else:
+            xwin = bmr.XWindow(ecap, hcap, device=torch.device(dev))
+            job.set_xwindows([xwin])
         exchange = False
 
     def step():
         job.reset()
-        if xwin is not None:   # f-3: the Map's flush appends the records to the window, then ingest
+        if xwin is not None:   # f-3: the Maps append the records to the owners' windows, then ingest
             xwin.reset()
+            barrier()          # every window is empty before any rank maps
             job.map(inp["data"], inp["offsets"], inp["n"])
+            barrier()          # every rank's records have landed
             job.ingest_xwindow(xwin)
         else:
             job.map(inp["data"], inp["offsets"], inp["n"])
@@ -444,7 +455,7 @@ def main():
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "exchange": ({"kind": "hash all-to-all over NCCL (torch.distributed)", "send_bytes_per_rank": xbytes[0],
                           "combiner": inp["wl"] in ("wc", "km")} if exchange else
-                         ({"kind": "fused Map flush into the receive window (f-3), one rank",
+                         ({"kind": "fused Map flush into the owners' receive windows (f-3, CUDA IPC / NVLink)",
                            "window_entries_heap": list(xwin.used())} if xwin is not None else None)),
             "gpu_launches": int(tot["kernel_launches"]),
             "clocks": clk.summary(), "wall_s_timed": round(wall, 3),
