@@ -21,3 +21,12 @@ spec = pygen.KMSpec(); pts = pygen.host_km(spec, 4096); _, init = pygen.km_centr
 with bmr.Job("km", centroids=init) as job:
     d = torch.from_numpy(pts.view(np.uint8).reshape(-1)).cuda()
     job.map(d, None, 4096); job.group(); job.reduce(); print("km", job.fetch()["n_keys"])
+# SM dense plants (the stage-released record check) and the fused exchange window (f-3)
+run("sm", pygen.spec_sm(20000, dense=True) if "dense" in pygen.spec_sm.__code__.co_varnames else pygen.spec_sm(20000), 2,
+    pattern=pygen.SM_PATTERN)
+g = pygen.host_text(pygen.spec_ii(4), 2)
+d = torch.from_numpy(g["data"]).cuda(); o = torch.from_numpy(g["offsets"].view(np.int64)).cuda()
+w = bmr.XWindow(1 << 16, 1 << 22)
+with bmr.Job("ii") as job:
+    job.set_xwindows([w]); job.map(d, o, g["n"]); torch.cuda.synchronize(); job.ingest_xwindow(w)
+    job.group(); job.reduce(); print("ii fused", job.fetch()["n_keys"])
