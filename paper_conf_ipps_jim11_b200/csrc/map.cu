@@ -50,6 +50,10 @@ constexpr int kNMap = 16;
 #define BMR_WC_OFFCAP 640       // WordCount: record offsets staged per tile (C1/C5 lines >= 27 B: <= 617 per
                                 // staged window; denser tiles read offsets from global memory)
 #endif
+#ifndef BMR_KM_UNROLL
+#define BMR_KM_UNROLL 2   // KMeans: centroid pairs per unrolled distance-loop iteration
+#endif
+constexpr int kKmUnroll = BMR_KM_UNROLL;
 #ifndef BMR_WC_COMB_PROBES
 #define BMR_WC_COMB_PROBES 1   // WordCount combiner probes per word (2: C5 absorbs 4.6% more words but the Map costs 0.9 ms more than the sort saves)
 #endif
@@ -1644,7 +1648,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         for (int t = 0; t < 8; ++t) X[t] = f2pack(x[t], x[t]);
         const uint32_t kp = P.k & ~1u;
         bool first = true;
-#pragma unroll 2
+#pragma unroll kKmUnroll
         for (uint32_t j = 0; j < kp; j += 2) {
           const ulonglong2* cp = reinterpret_cast<const ulonglong2*>(cent + j * 8);   // pair layout
           const ulonglong2 q0 = cp[0], q1 = cp[1], q2 = cp[2], q3 = cp[3];
