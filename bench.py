@@ -3,6 +3,7 @@
 % HBM roofline, vs the CPU oracle).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C5|C4|C3|C2|C1] [--impl reference]
+                    [--mode SIO|SO|SI|G] [--no-map-combine] [--xchg a2a|fused] [--units U]
 
 One step = one pass of the whole hot path (tile scheduling, stage-in,
 user map, emit, flush, digit histogram, onesweep passes, segment boundaries, reduce + output
@@ -11,7 +12,9 @@ assembly) over one shard of synthetic input already resident in HBM.  Default wo
 "1/2/4/8 B200" is quoted on that exercises every row (C2 StringMatch is Map-only).
 Prints ONE JSON line on rank 0.  Timing: W warm-up steps, then K steps bracketed by barrier +
 cuda.synchronize, CUDA events on the job stream, max over ranks.  Inputs (8 GiB) exceed L2
-(126 MB), so no extra flush is needed.
+(126 MB), so no extra flush is needed.  At N > 1 the exchange is the partition + all-to-all over
+NCCL, or with --xchg fused (InvertedIndex) the Maps store straight into the owners' receive
+windows through CUDA IPC.
 """
 from __future__ import annotations
 

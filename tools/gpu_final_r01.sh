@@ -11,6 +11,7 @@ for w in C5 C2 C3 C4; do
   timeout 600 python bench.py --workload $w --steps 5 --warmup 3 > $O/bench_$w.json 2> $O/bench_$w.err
 done
 timeout 300 python bench.py --impl reference --steps 2 --warmup 3 > $O/bench_reference_C5.json 2> $O/bench_reference_C5.err
+timeout 300 python bench.py --workload C4 --xchg fused --steps 5 --warmup 3 --e2e-steps 0 --no-cpu-baseline > $O/bench_C4_fused_xchg.json 2> $O/bench_C4_fused.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $O/launches_C5.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline --e2e-steps 0 > $O/ncu_launch.log 2>&1
 B="python bench.py --steps 1 --warmup 0 --e2e-steps 0 --no-cpu-baseline"
 N="ncu --set full --clock-control none --import-source on"
