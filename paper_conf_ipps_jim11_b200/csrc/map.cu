@@ -1416,6 +1416,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
 // range masks, the warp reduction of the emission count) is paid once per 2 KiB instead of per
 // 512 B (ncu, C2 round 1: it was ~80% of the Map's instructions).
 constexpr int kSmSub = BMR_SM_SUB, kNSup = kNWin / kSmSub;
+template <bool kSO>
 __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   constexpr int W = kSM;
   constexpr int kStages = Cfg<W>::kStages;
@@ -1460,7 +1461,7 @@ __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl
     const uint8_t* c0 = sb + (wp0 - hd.sbase) + lane * 16;
     // SO / G ablation (MR_FLAG_NO_SMEM_IN): the same loads from global memory (the stage is empty)
     auto ld16 = [&](long long q, const uint8_t* sp) -> uint4 {
-      if (!P.so) return *reinterpret_cast<const uint4*>(sp);
+      if constexpr (!kSO) return *reinterpret_cast<const uint4*>(sp);
       if (q >= 0 && q + 16 <= N) return __ldg(reinterpret_cast<const uint4*>(P.rec + q));   // rec + q: 16-B aligned
       uint32_t w[4] = {0, 0, 0, 0};
       for (int b = 0; b < 16; ++b)
@@ -1601,7 +1602,10 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   StageHdr hd{};
   const bool sm_fast = W == kSM && !P.dyn;
   if constexpr (W == kSM) {
-    if (sm_fast) sm_fast_loop(P, smem, oc);
+    if (sm_fast) {   // (SO / G ablation: a separate instantiation, no per-load mode test on the SIO path)
+      if (P.so) sm_fast_loop<true>(P, smem, oc);
+      else sm_fast_loop<false>(P, smem, oc);
+    }
   }
   for (uint32_t it = 0; !sm_fast; ++it) {
     uint32_t w = 0;
