@@ -91,7 +91,32 @@ __global__ void __launch_bounds__(kSegThreads) k_seg_count(const K* __restrict__
         if (need_r) r = kref[perm[i]];
         uint64_t rp = __shfl_up_sync(0xffffffffu, r, 1);
         if (lane == 0) rp = carry_has_r ? carry_r : ((hashed_run && i > 0) ? kref[perm[i - 1]] : 0);
-        if (hashed_run && !key_bytes_equal(r, rp)) ++coll;
+        // keys of <= 16 bytes: every lane reads its OWN key bytes once and compares them with
+        // the previous lane's by shuffles (one random read per element instead of two; C5's long
+        // words; longer keys such as C4's URLs keep the two-pointer comparison)
+        const uint32_t len = static_cast<uint32_t>(r & 0xFFFF);
+        uint64_t b[2] = {0, 0};
+        if (need_r && len <= 16) {
+          const uint8_t* kp = reinterpret_cast<const uint8_t*>(r >> 16);
+#pragma unroll
+          for (int q = 0; q < 2; ++q) {
+            const uint32_t off = 8u * q;
+            if (off < len) {
+              const uint32_t need = min(8u, len - off);
+              b[q] = load8(kp + off, need) & (need == 8 ? ~0ULL : ((1ULL << (8 * need)) - 1ULL));
+            }
+          }
+        }
+        uint64_t pb[2];
+#pragma unroll
+        for (int q = 0; q < 2; ++q) pb[q] = __shfl_up_sync(0xffffffffu, b[q], 1);
+        const uint32_t plen = static_cast<uint32_t>(rp & 0xFFFF);
+        if (hashed_run) {
+          bool eq;
+          if (lane != 0 && len <= 16 && plen <= 16) eq = len == plen && b[0] == pb[0] && b[1] == pb[1];
+          else eq = key_bytes_equal(r, rp);
+          if (!eq) ++coll;
+        }
       }
       carry_r = __shfl_sync(0xffffffffu, r, 31);
       carry_has_r = __shfl_sync(0xffffffffu, need_r ? 1u : 0u, 31) != 0;
