@@ -421,3 +421,21 @@ def test_sort_u64_matches_stable_sort(n, bits):
     ref_v, ref_i = torch.sort(flip, stable=True)
     assert torch.equal(perm.long(), ref_i)
     assert torch.equal(ks, k[ref_i])
+
+
+def test_wc_job_reuse_across_sizes():
+    """A job reused across runs of different sizes (grow-only buffers sized by the previous run:
+    segment starts, sort workspaces, combiner partials) stays exact."""
+    small = pygen.host_text(pygen.spec_wc(1_000_000, 5), 1)
+    big = pygen.host_text(pygen.spec_wc(1_000_000, 5), 6)
+    with bmr.Job("wc") as job:
+        outs = []
+        for g in (small, small, big, big):
+            d, o = dev(g["data"], g["offsets"])
+            job.reset()
+            job.map(d, o, g["n"])
+            job.group()
+            job.reduce()
+            outs.append(decode("wc", job.fetch()))
+    assert outs[0] == outs[1] == decode("wc", ora("wc", [(small["data"], small["offsets"], small["n"])]))
+    assert outs[2] == outs[3] == decode("wc", ora("wc", [(big["data"], big["offsets"], big["n"])]))
