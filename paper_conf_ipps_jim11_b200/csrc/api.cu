@@ -631,7 +631,7 @@ mr_status mr_job_create(const mr_config* cfg, mr_job** out) {
   }
   job->nsm = sm_count(cfg->device);
   job->prof.on = (cfg->flags & MR_FLAG_PROFILE) != 0;
-  job->key_bits = (cfg->workload == MR_WORDCOUNT) ? 48u : 64u;
+  job->key_bits = (cfg->workload == MR_WORDCOUNT || cfg->workload == MR_INVINDEX) ? 48u : 64u;
   job->launches0 = g_kernel_launches.load();
   *out = job;
   return MR_OK;
@@ -647,7 +647,7 @@ mr_status mr_job_reset(mr_job* job) {
   job->ingested = false;
   job->km_partial = false;
   job->km_combined = false;
-  job->key_bits = (job->cfg.workload == MR_WORDCOUNT) ? 48u : 64u;
+  job->key_bits = (job->cfg.workload == MR_WORDCOUNT || job->cfg.workload == MR_INVINDEX) ? 48u : 64u;
   job->key_bits_b = 48;
   job->mb = job->nseg_a = job->nseg_b = job->mc = job->nseg_c = 0;
   job->mp = job->nseg_p = job->n_extra = 0;
