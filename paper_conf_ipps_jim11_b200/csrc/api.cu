@@ -186,7 +186,7 @@ cudaError_t run_sort(SortWork& W, const uint64_t* keys, uint64_t m, const uint64
   for (int p = 0; p < nd; ++p) {
     uint64_t* kout = (p & 1) ? W.kb.p : W.ka.p;
     uint32_t* iout = pay ? ((p & 1) ? W.ib.p : W.ia.p) : nullptr;
-    const int rk = pay ? 0 : choose_rank_kind32(W.hist_h.p + digits[p] * kBinStride, m, p == 0);
+    const int rk = pay ? kRankMatch : choose_rank_kind32(W.hist_h.p + digits[p] * kBinStride, m, p == 0);
     if ((e = launch_onesweep(kin, iin, kout, iout, m, digits[p], bits, W.bases.p, W.status.p, W.epoch++,
                              &st->tile_counter[0], s, rk)))
       return e;
@@ -528,6 +528,7 @@ mr_status settle_map(mr_job* job) {
   CK(read_state(job), "map (async)");
   DevState* hs = job->st_h.p;
   if (hs->err & kErrKeyTooLong) return fail(job, MR_ERR_OVERFLOW, "an emitted key exceeds 65535 bytes");
+  if (job->ingested) return MR_OK;   // ingested pairs: exact count, written into buffers sized for it
   const uint64_t m = hs->pair_cursor, mb = job->split() ? hs->pair_cursor_b : 0;
   const uint64_t mc = job->split() ? hs->pair_cursor_c : 0;
   const uint64_t mp = job->wc_comb() ? hs->pair_cursor_p : 0;
@@ -769,6 +770,11 @@ mr_status mr_map_host_lines(mr_job* job, const uint8_t* text, uint64_t nbytes) {
   if (!job) return MR_ERR_INVALID;
   if (job->cfg.record_stride > 0) return fail(job, MR_ERR_INVALID, "mr_map_host_lines: text workloads only");
   if (nbytes && !text) return fail(job, MR_ERR_INVALID, "text is NULL");
+  if (job->state != kCreated && job->state != kMapped) return fail(job, MR_ERR_STATE, "mr_map after mr_group");
+  if (nbytes == 0) {   // no records: nothing to copy or map
+    job->state = kMapped;
+    return MR_OK;
+  }
   CK(cudaSetDevice(job->cfg.device), "set device");
   if (!job->cstream) {
     CK(cudaStreamCreateWithFlags(&job->cstream, cudaStreamNonBlocking), "copy stream");
@@ -1297,13 +1303,13 @@ mr_status mr_ingest(mr_job* job, const void* entries, const void* heap, const ui
     job->state = kMapped;
     return MR_OK;
   }
-  if (n > job->cap || job->v.n < n * 8 || job->kref.n < n) {
-    release_pairs(job);
-    CK(job->h.ensure(n + 1), "alloc pairs");
-    CK(job->kref.ensure(n + 1), "alloc pairs");
-    CK(job->v.ensure((n + 1) * 8), "alloc pairs");
-    job->cap = n + 1;
-  }
+  // The ingested stream lives in h / kref / v (u64 values).  The Map's own buffers stay as they
+  // are (a WordCount job's split streams hx / hb / hc / hp are untouched), so the job can be reset
+  // and mapped again; the ingested count is exact, so settle_map skips the capacity check.
+  CK(job->h.ensure(n + 1), "alloc pairs");
+  CK(job->kref.ensure(n + 1), "alloc pairs");
+  CK(job->v.ensure((n + 1) * 8), "alloc pairs");
+  if (!job->split()) job->cap = std::min<uint64_t>(std::min(job->h.n, job->kref.n), job->v.n / 8);
   CK(job->src_e.ensure(R + 1), "alloc src");
   CK(job->src_h.ensure(R + 1), "alloc src");
   CK(cudaMemcpyAsync(job->src_e.p, se.data(), (R + 1) * 8, cudaMemcpyHostToDevice, s), "H2D src");
@@ -1353,8 +1359,13 @@ mr_status mr_ingest_xwindow(mr_job* job, const void* entries, const void* heap, 
   if (job->state != kMapped && job->state != kCreated)
     return fail(job, MR_ERR_STATE, "mr_ingest_xwindow after mr_group");
   CK(cudaSetDevice(job->cfg.device), "set device");
-  uint64_t c[2] = {0, 0};
-  CK(cudaMemcpy(c, cursor, sizeof(c), cudaMemcpyDeviceToHost), "D2H window cursor");
+  // this rank's Map errors first (read_state synchronises the job stream): a URL clamped to
+  // 65535 bytes in the Map's queue must reject the batch here too, as settle_map does
+  CK(read_state(job), "map (async)");
+  if (job->st_h.p->err & kErrKeyTooLong) return fail(job, MR_ERR_OVERFLOW, "an emitted key exceeds 65535 bytes");
+  uint64_t* c = job->tmp_h.p + 2;
+  CK(cudaMemcpyAsync(c, cursor, 2 * sizeof(uint64_t), cudaMemcpyDeviceToHost, job->stream), "D2H window cursor");
+  CK(cudaStreamSynchronize(job->stream), "sync window cursor");
   if (c[0] > entry_cap || c[1] > heap_cap)
     return fail(job, MR_ERR_OOM, "receive window overflow: " + std::to_string(c[0]) + " entries / " +
                                           std::to_string(c[1]) + " heap bytes needed");

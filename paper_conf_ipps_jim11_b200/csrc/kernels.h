@@ -109,9 +109,12 @@ struct SortBufs {
 };
 constexpr int kSortThreads = 256;
 constexpr int kBinStride = 512;   // histogram / base tables: 8 digits x kBinStride bins (digits of 8 or 9 bits)
-int sort_tile();   // keys per onesweep tile (tile shape chosen at start-up, BMR_SORT_CFG)
-int sort_tile_keys();   // the same for the keys-only passes
+int sort_tile();          // keys per onesweep tile (payload passes)
+int sort_tile_keys();     // the same for the keys-only passes
 int sort_tile_keys32();   // the same for the keys-only passes over u32 keys
+// ranking of a onesweep pass: match.any groups, or shared-memory OR match masks (a first pass
+// whose 32-key groups carry many distinct digits)
+constexpr int kRankMatch = 0, kRankOrMask = 1;
 // histograms of digits [0, nd) of `bits` bits each (8 or 9); hist holds 8 x kBinStride u32
 cudaError_t launch_hist(const uint64_t* keys, uint64_t m, uint32_t* hist, int nd, int bits, int num_sms,
                         cudaStream_t s);
@@ -123,13 +126,13 @@ cudaError_t launch_hist32(const uint32_t* keys, uint64_t m, uint32_t* hist, int 
 cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
                             uint32_t* idx_out, uint64_t m, int digit, int bits, const uint32_t* bases,
                             uint64_t* status, uint32_t epoch, unsigned int* tile_counter, cudaStream_t s,
-                            int rank_kind = 0);   // 66: OR-mask ranking (keys-only passes), else match.any
+                            int rank_kind = kRankMatch);   // kRankOrMask: keys-only passes only
 // keys-only LSD pass over u32 keys (the WordCount exact stream)
 cudaError_t launch_onesweep32(const uint32_t* keys_in, uint32_t* keys_out, uint64_t m, int digit, int bits,
                               const uint32_t* bases, uint64_t* status, uint32_t epoch, unsigned int* tile_counter,
-                              cudaStream_t s, int rank_kind = 0);
-// ranking kind of a u32 pass from its digit histogram (hist[0..255], m keys): 66 (shared-memory
-// match masks) for a first pass whose digits of 32 keys are mostly distinct, else 2 (match.any)
+                              cudaStream_t s, int rank_kind = kRankMatch);
+// ranking kind of a keys-only pass from its digit histogram (hist[0..255], m keys): kRankOrMask
+// for a first pass whose digits of 32 keys are mostly distinct, else kRankMatch
 int choose_rank_kind32(const uint32_t* hist, uint64_t m, bool first_pass);
 
 // ---- segments ----

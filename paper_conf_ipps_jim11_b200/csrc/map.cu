@@ -4,22 +4,23 @@
 // collects results in a shared-memory output area and flushes it to global memory with one
 // global atomic per flush.  Its GT200 mechanics (16 KB SMEM, all threads alternating between
 // stage-in / compute / stage-out, software wait-signal flags, yield by dummy global reads) are
-// prior art; the B200 re-derivation here (one 576-thread CTA per SM):
-//   * producer warp (A1/A2): one elected lane issues TMA bulk copies (cp.async.bulk) of the
-//     tile bytes and of the tile's record-offset slice into an SMEM ring (4 stages, 7 for SM)
-//     guarded by mbarrier full/empty pairs; kLag tiles later the producer turns the staged
-//     offsets into a record-start bitmap and releases the stage (ready mbarrier) — replaces the
-//     barrier-separated staging loop (L68, L85);
-//   * 16 map warps (A3): byte-parallel, record-agnostic scanning — each lane owns a 16-byte
-//     chunk, record boundaries come from the bitmap; no map-warp barrier at all, so the
-//     per-record imbalance the paper blames for SO overhead (L273) disappears;
+// prior art; the B200 re-derivation here (one persistent CTA per SM):
+//   * two producer warps (A1/A2): an elected lane issues TMA bulk copies (cp.async.bulk) of the
+//     tile bytes and of the tile's record-offset slice into an SMEM ring (4 stages; StringMatch
+//     12 stages of bytes only) guarded by mbarrier full/empty pairs; kLag tiles later the
+//     producer turns the staged offsets into a record-start bitmap and releases the stage
+//     (ready mbarrier) — replaces the barrier-separated staging loop (L68, L85);
+//   * map warps (A3; 24 for the text workloads, 16 for KMeans): byte-parallel, record-agnostic
+//     scanning — each lane owns a 16-byte chunk of a 512-B window, record boundaries come from
+//     the bitmap; no map-warp barrier at all, so the per-record imbalance the paper blames for
+//     SO overhead (L273) disappears;
 //   * emit allocator (A11/A12, D3/D4): a warp result is reserved with ONE shared 32-bit
-//     atomicAdd on a packed [generation:8 | count:24] cursor of the current output buffer;
+//     atomicAdd on a packed [generation:6 | cb:12 | ca:14] cursor of the current output buffer;
 //   * overflow (A13, L113): the unique warp whose reservation crosses the buffer's capacity
 //     seals it and switches every warp to the next buffer of a 4-buffer ring at once (replaces
 //     the wait/signal flag protocol, L96-100); it waits only if all buffers are still flushing;
-//   * flush warp (A4): waits for the sealed buffer's in-flight writers, takes ONE global
-//     atomicAdd for the whole buffer, and writes its SoA arrays with TMA bulk stores
+//   * flush warp (A4): waits (acquire loads) for the sealed buffer's in-flight writers, takes ONE
+//     global atomicAdd for the whole buffer, and writes its SoA arrays with TMA bulk stores
 //     (cp.async.bulk.global.shared::cta).  Flushes are rounded to 4 pairs (16-B alignment) with
 //     sentinel filler pairs.  The global cursor counts demand even past capacity (D7), so the
 //     host can grow the buffers and replay the batch.
@@ -73,9 +74,17 @@ constexpr int nmap() { return W == 3 ? kNMap : W == 2 ? BMR_SM_NMAP : kNMapText;
 // (and so the stages s == p (mod kNProd)); one warp alone is latency-bound at ~465 instructions
 // per tile (TMA issue + bitmap), slower than HBM delivers a tile (ncu, C2 round 1).
 constexpr int kNProd = 2;
-constexpr int kNFlush = 1;   // warps: map 0 .. nmap-1, producers nmap .. nmap+kNProd-1, then flush
+// Flush warps (flush_loop takes generations f == fw mod nflush).  One: a second WordCount flush
+// warp removed the map warps' spinning on sealed buffers but cost the Map more than it saved
+// (C5 Map 20.4 -> 21.3 ms, round 2: a 28th warp lowers the register budget of every warp).
+// Warps: map 0 .. nmap-1, producers nmap .. nmap+kNProd-1, then the flush warps.
+#ifndef BMR_WC_NFLUSH
+#define BMR_WC_NFLUSH 1u
+#endif
 template <int W>
-constexpr int threads_of() { return (nmap<W>() + kNProd + kNFlush) * 32; }
+constexpr uint32_t nflush() { return W == kWC ? BMR_WC_NFLUSH : 1u; }
+template <int W>
+constexpr int threads_of() { return (nmap<W>() + kNProd + static_cast<int>(nflush<W>())) * 32; }
 constexpr int kT = 16384;        // owned bytes per tile (text) / bytes per tile (KM)
 constexpr int kLead = 16;        // bytes staged before the tile (previous-byte context)
 constexpr int kHalo = 256;       // bytes staged after the tile (words / matches / URLs crossing it)
@@ -155,12 +164,11 @@ struct StageHdr {
 };
 
 struct OutCtl {
-  unsigned int cur;              // [generation:8 | count:24]; half = generation & 1
+  unsigned int cur;              // [generation:6 | cb:12 | ca:14]; buffer = generation % kNOut
   unsigned int final_seq;        // full generation number of the final flush
   unsigned int committed[kNOut];     // entries fully written into each buffer (current generation)
   unsigned int fcount[kNOut];        // sealed entry count of each buffer
   unsigned long long fbase[kNOut];   // global base reserved for the sealed buffer (one atomic per flush)
-  unsigned long long nflush, npads;  // per-CTA statistics, added to DevState once at the end
   unsigned int nsealed, is_final;  // sealed generations so far (full count); final flush flag
   unsigned int win_next;         // text: next window (tile * kNWin + window) to hand to a map warp
   uint64_t req[kNOut];           // mbarrier: buffer sealed -> flush warp
@@ -251,6 +259,7 @@ struct Params {
   uint32_t so, si;
   uint32_t sm_lines;       // StringMatch: emit the matching record's start (MR_FLAG_SM_LINES)
   uint32_t wc_bal;         // WordCount: balanced two-phase emission (BMR_WC_BAL, default on)
+  uint32_t wc_fast;        // WordCount: wc_map_loop / wc_window (BMR_WC_FAST, default on)
   const XWindow* xwin;     // f-3: InvertedIndex records appended straight to these windows
   uint32_t xranks;         // number of windows (0: local output)
 };
@@ -477,7 +486,6 @@ __device__ __forceinline__ uint64_t key_at(const Params& P, const TileView& tv, 
 }
 
 // ---------------------------------------------------------------- emit allocator
-// Shared cursor: 32-bit [generation:8 | count:24] (native ATOMS.ADD).  half = generation & 1.
 // Flush bases are kept multiples of 4 pairs so that every SoA run of a flushed half is 16-byte
 // aligned in global memory and leaves SMEM as one TMA bulk store (cp.async.bulk global<-shared);
 // the <= 3 filler entries carry the workload's sentinel key, which sorts after every real key
@@ -551,8 +559,7 @@ __device__ __forceinline__ Slot reserve(const Params& P, OutCtl* oc, uint8_t* ou
         // it seals half h (L113 "overflow handling").
         seal<W>(P, oc, gen, h, base, false);
       } else {
-        volatile unsigned int* c = &oc->cur;
-        while (cur_gen(*c) == gen) __nanosleep(128);
+        while (cur_gen(ld_acquire_cta_shared_u32(&oc->cur)) == gen) __nanosleep(128);
       }
     }
     __syncwarp();
@@ -573,26 +580,39 @@ __device__ __forceinline__ void tma_store_1d(void* gdst, const void* ssrc, uint3
                "r"(bytes)
                : "memory");
 }
-__device__ __forceinline__ void tma_store_commit_and_wait_read() {
-  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-  asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
-}
 
+// Flush warps (A4, L113): flush warp fw of nflush<W>() takes the sealed generations
+// f == fw (mod nflush).  Per buffer: wait for its committed writers (acquire), pad the exact run
+// to 16 B, count the queued WC entries per stream (SMEM only), then ONE round of global atomics
+// (one lane per stream: all three reservations in flight together), the TMA bulk store of the
+// buffer's SoA runs, the routed stores of the queued entries while the TMA reads SMEM, and only
+// then the wait for the TMA's reads before the buffer is handed back.
 template <int W>
-__device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
+__device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc, uint32_t fw) {
   using F = PairFmt<W>;
+  constexpr uint32_t NF = nflush<W>();
   const uint32_t lane = threadIdx.x & 31;
-  for (uint32_t f = 0;; ++f) {
+  unsigned long long nflushes = 0, npads = 0;
+  for (uint32_t f = fw;; f += NF) {
     const uint32_t h = f % kNOut;
-    helper_wait(P, &oc->req[h], (f / kNOut) & 1u, 64);
-    const uint32_t cnt0 = *reinterpret_cast<volatile unsigned int*>(&oc->fcount[h]);
-    const bool fin = *reinterpret_cast<volatile unsigned int*>(&oc->is_final) &&
-                     *reinterpret_cast<volatile unsigned int*>(&oc->final_seq) == f;
+    // wait for generation f to be sealed; with several flush warps the one waiting past the
+    // final generation sees the final flag instead (no arrival ever comes for it)
+    bool past = false;
+    // (suspended try_wait: a polling flush warp would take issue slots from the map warps)
+    while (!mbar_try_wait_hint(&oc->req[h], (f / kNOut) & 1u, 2000)) {
+      if (NF > 1 && ld_acquire_cta_shared_u32(&oc->is_final) && ld_acquire_cta_shared_u32(&oc->final_seq) < f) {
+        past = true;
+        break;
+      }
+    }
+    if (past) break;
+    // (the sealing warp wrote these before its release-arrive on req[h]; the wait above acquires)
+    const bool fin = ld_acquire_cta_shared_u32(&oc->is_final) && ld_acquire_cta_shared_u32(&oc->final_seq) == f;
+    const uint32_t cnt0 = ld_acquire_cta_shared_u32(&oc->fcount[h]);
     uint8_t* half = smem + Layout<W>::out + h * Cfg<W>::kOutHalf;
     // the sealed buffer's writers finish on their own: wait until all cnt0 entries are committed
     if (lane == 0) {
-      volatile unsigned int* cm = &oc->committed[h];
-      while (*cm != cnt0) __nanosleep(32);
+      while (ld_acquire_cta_shared_u32(&oc->committed[h]) != cnt0) __nanosleep(32);
     }
     __syncwarp();
     const uint32_t ca0 = cur_ca(cnt0);
@@ -608,46 +628,49 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         if constexpr (F::kKref) reinterpret_cast<uint64_t*>(half)[F::kCap + ca0 + lane] = 0;
       }
     }
-    unsigned long long gb = 0, gbb = 0;
-    if (lane == 0) {
-      if (cnt) gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(cnt));  // ONE global atomic per run
-      oc->nflush += (cnt || cb) ? 1 : 0;
-      oc->npads += cnt - ca0;
+    // WC queued entries (key, kref) at the top of the buffer: kref 0 -> mid stream (key only),
+    // else hashed stream (key + kref)
+    const ulonglong2* top = reinterpret_cast<const ulonglong2*>(half + Cfg<W>::kOutHalf);
+    uint32_t nc = 0;
+    if constexpr (W == kWC) {
+      for (uint32_t i0 = 0; i0 < cb; i0 += 32) {
+        const bool v = i0 + lane < cb && top[-1 - static_cast<int>(i0 + lane)].y == 0;
+        nc += __popc(__ballot_sync(kFull, v));
+      }
     }
-    gb = __shfl_sync(kFull, gb, 0);
-    __syncwarp();
+    // one global atomic per stream run (L113), issued by lanes 0 / 1 / 2 together
+    unsigned long long g = 0;
+    {
+      unsigned long long* cur = lane == 0 ? &P.st->pair_cursor : lane == 1 ? &P.st->pair_cursor_b : &P.st->pair_cursor_c;
+      const uint32_t want = lane == 0 ? cnt : lane == 1 ? cb - nc : nc;
+      if (lane < 3 && want) g = atomicAdd(cur, static_cast<unsigned long long>(want));
+    }
+    const unsigned long long gb = __shfl_sync(kFull, g, 0);
+    nflushes += (cnt || cb) ? 1 : 0;
+    npads += cnt - ca0;
+    bool tma = false;
     if (cnt && gb + cnt <= P.cap_pairs) {
       const uint64_t* sh = reinterpret_cast<const uint64_t*>(half);
       const uint8_t* sv = half + F::kCap * (F::kKref ? 16 : 8);
       if constexpr (W == kSM) {
         for (uint32_t i = lane; i < cnt; i += 32) P.oh[gb + i] = sh[i];
-      } else if (lane == 0) {
-        // A4 staging-out as TMA bulk stores (16-B aligned: gb and cnt even / multiples of 4)
-        fence_proxy_async_shared();
-        if constexpr (W == kWC) tma_store_1d(P.ohx + gb, sh, cnt * 4);
-        else tma_store_1d(P.oh + gb, sh, cnt * 8);
-        if constexpr (F::kKref) tma_store_1d(P.okref + gb, sh + F::kCap, cnt * 8);
-        if constexpr (F::kV > 0) tma_store_1d(P.ov + gb * F::kV, sv, cnt * F::kV);
-        tma_store_commit_and_wait_read();          // SMEM may be reused once the stores have read it
+      } else {
+        tma = true;
+        fence_proxy_async_shared();   // every lane's filler writes -> visible to the TMA store
+        __syncwarp();
+        if (lane == 0) {
+          // A4 staging-out as TMA bulk stores (16-B aligned: gb and cnt even / multiples of 4)
+          if constexpr (W == kWC) tma_store_1d(P.ohx + gb, sh, cnt * 4);
+          else tma_store_1d(P.oh + gb, sh, cnt * 8);
+          if constexpr (F::kKref) tma_store_1d(P.okref + gb, sh + F::kCap, cnt * 8);
+          if constexpr (F::kV > 0) tma_store_1d(P.ov + gb * F::kV, sv, cnt * F::kV);
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
       }
     }
     if constexpr (W == kWC) {
-      // queued entries (key, kref) from the top of the buffer: kref 0 -> mid stream (key only),
-      // else hashed stream (key + kref).  Two ballot passes: count, then scatter (plain
-      // coalesced stores; a few % of the pairs).
-      const ulonglong2* top = reinterpret_cast<const ulonglong2*>(half + Cfg<W>::kOutHalf);
-      uint32_t nc = 0;
-      for (uint32_t i0 = 0; i0 < cb; i0 += 32) {
-        const bool v = i0 + lane < cb && top[-1 - static_cast<int>(i0 + lane)].y == 0;
-        nc += __popc(__ballot_sync(kFull, v));
-      }
-      unsigned long long gc = 0;
-      if (lane == 0) {
-        if (cb - nc) gbb = atomicAdd(&P.st->pair_cursor_b, static_cast<unsigned long long>(cb - nc));
-        if (nc) gc = atomicAdd(&P.st->pair_cursor_c, static_cast<unsigned long long>(nc));
-      }
-      gbb = __shfl_sync(kFull, gbb, 0);
-      gc = __shfl_sync(kFull, gc, 0);
+      // routed plain stores (coalesced per 32 entries), overlapping the TMA store's SMEM reads
+      const unsigned long long gbb = __shfl_sync(kFull, g, 1), gc = __shfl_sync(kFull, g, 2);
       const bool okb = gbb + (cb - nc) <= P.cap_b, okc = gc + nc <= P.cap_c;
       uint32_t rb = 0, rc = 0;
       for (uint32_t i0 = 0; i0 < cb; i0 += 32) {
@@ -665,14 +688,15 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         rb += __popc(mb);
       }
     }
+    if (tma && lane == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // SMEM reusable
     __syncwarp();
     if (lane == 0) mbar_arrive(&oc->done[h]);
     if (fin) break;
   }
   if (lane == 0) {
     asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // global writes complete
-    atomicAdd(&P.st->flushes, oc->nflush);
-    if (oc->npads) atomicAdd(&P.st->pads, oc->npads);
+    atomicAdd(&P.st->flushes, nflushes);
+    if (npads) atomicAdd(&P.st->pads, npads);
   }
 }
 
@@ -1048,6 +1072,172 @@ __device__ __forceinline__ void emit_wc(const Params& P, OutCtl* oc, uint8_t* ou
     top[-1 - static_cast<int>(kb0 + q)] = ent;
   }
   commit(oc, slot, packed);
+}
+
+// ---------------------------------------------------------------- WordCount fast path (SIO)
+// The same computation as emit_text_chunk<kWC> + emit_wc (balanced mode) for one 512-B window,
+// written for instruction count: no lane-0 / lane-31 divergent sections (every lane loads the
+// byte before its chunk and classifies the next 16 bytes itself), one loop over the word starts
+// that files exact and long words into separate queues (so the combiner rounds see exact words
+// only), branch-free exact keys, predicated lane-0 shared atomics.
+__device__ __forceinline__ uint32_t lane0_atom_add_shared(uint32_t* a, uint32_t v) {
+  uint32_t old = 0;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.eq.u32 p, %2, 0;\n\t"
+      "@p atom.shared.add.u32 %0, [%1], %3;\n\t}"
+      : "+r"(old)
+      : "r"(smem_u32(a)), "r"(threadIdx.x & 31u), "r"(v)
+      : "memory");
+  return __shfl_sync(kFull, old, 0);
+}
+__device__ __forceinline__ void lane0_mbar_arrive(uint64_t* bar) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.eq.u32 p, %1, 0;\n\t"
+      "@p mbarrier.arrive.shared::cta.b64 _, [%0];\n\t}" ::"r"(smem_u32(bar)),
+      "r"(threadIdx.x & 31u)
+      : "memory");
+}
+// exact_key30 (common.cuh) without branches: lo = word bytes 0..3, b4 = byte 4, len 1..5
+__device__ __forceinline__ uint32_t exact_key30_bf(uint32_t lo, uint32_t b4, uint32_t len) {
+  uint32_t c = exact_codes4(lo) & (0xFFFFFFFFu >> (32u - 8u * min(len, 4u)));
+  uint32_t y = (c & 0x003F003Fu) | ((c >> 2) & 0x0FC00FC0u);   // byte pairs -> 12 bits
+  y = (y & 0x00000FFFu) | ((y >> 4) & 0x00FFF000u);            // -> 24 bits
+  const uint32_t c4 = (b4 & 0xFu) + __byte_perm(0x01000000u, 0x34241A0Au, (b4 >> 4) & 0xFu);
+  return y | (len == 5u ? (c4 << 24) : 0u);
+}
+
+// One 512-B window [p0w, p0w + 512) of a WordCount tile (lane = 16-byte chunk).  tv: the stage.
+__device__ __forceinline__ void wc_window(const Params& P, OutCtl* oc, uint8_t* outh, const TileView& tv,
+                                          long long p0w, uint32_t* xq, uint32_t* hq, uint32_t* ctab) {
+  const uint32_t lane = threadIdx.x & 31;
+  const long long N = static_cast<long long>(P.nbytes);
+  const long long p0 = p0w + 16 * lane;
+  const uint32_t i0 = static_cast<uint32_t>(p0 - tv.sbase);   // 16-B aligned stage offset
+  const uint4 c0 = *reinterpret_cast<const uint4*>(tv.sb + i0);
+  const uint4 c1 = *reinterpret_cast<const uint4*>(tv.sb + i0 + 16);   // next chunk (lane 31: the halo)
+  const uint32_t pb = tv.sb[i0 - 1];                                    // byte before the chunk (lead bytes)
+  uint32_t wm = word_mask4(c0.x) | (word_mask4(c0.y) << 4) | (word_mask4(c0.z) << 8) | (word_mask4(c0.w) << 12) |
+                (word_mask4(c1.x) << 16) | (word_mask4(c1.y) << 20) | (word_mask4(c1.z) << 24) |
+                (word_mask4(c1.w) << 28);
+  const bool edge = p0w < 0 || p0w + kWin + 16 > N;   // warp-uniform: only the input's first / last window
+  if (edge) wm &= range_mask32(p0, 0, N);
+  const uint32_t R = bits32(tv.bm, i0);                // record starts at p0 .. p0 + 31
+  const uint32_t prevw = (p0 > 0 && is_word_byte(pb)) ? 1u : 0u;
+  const uint32_t nb = ~wm | R;                          // a word cannot continue here
+  const uint32_t S = wm & 0xFFFFu & ~(((wm << 1) | prevw) & ~R);   // word starts (C-2 WC)
+  const uint32_t near = (nb >> 1) | (nb >> 2) | (nb >> 3) | (nb >> 4) | (nb >> 5);   // ends within 5 bytes
+  // only the lane's highest start can lack a visible end (no stop in the 31 - j bytes after it)
+  uint32_t len_slow = 0;
+  if (S) {
+    const uint32_t jh = 31 - __clz(S);
+    if ((nb >> (jh + 1)) == 0) len_slow = slow_word_len(P, tv, p0 + jh, p0 + 32);
+  }
+  const uint32_t cx = __popc(S & near), cl = __popc(S & ~near);
+  const uint32_t v = cx | (cl << 16);
+  const uint32_t incl = warp_inclusive_add(v);
+  const uint32_t tot = __shfl_sync(kFull, incl, 31);
+  if (tot == 0) return;
+  const uint32_t Wx = tot & 0xFFFFu, nl = tot >> 16;
+  // phase 1: descriptors at the words' warp ranks — exact words (stage offset | len << 16) into
+  // xq, long words (stage offset | len << 15) into hq
+  {
+    uint32_t kx = (incl - v) & 0xFFFFu, kl = (incl - v) >> 16;
+    for (uint32_t m = S; m; m &= m - 1) {
+      const uint32_t j = __ffs(m) - 1;
+      const uint32_t rest = nb >> (j + 1);
+      const uint32_t len = rest ? static_cast<uint32_t>(__ffs(rest)) : len_slow;
+      const bool ex = (near >> j) & 1u;
+      const uint32_t pos = i0 + j;
+      const uint32_t ll = min(len, 0xFFFFu);
+      uint32_t* dst = ex ? xq + kx : hq + kl;
+      *dst = ex ? (pos | (len << 16)) : (pos | (ll << 15));
+      kx += ex ? 1u : 0u;
+      kl += ex ? 0u : 1u;
+      if (len > 0xFFFFu) atomicOr(&P.st->err, kErrKeyTooLong);
+    }
+  }
+  __syncwarp();
+  // phase 2: exact words 32 at a time: key from the stage, combiner probe, misses compacted into xq
+  uint32_t nx = 0;
+  for (uint32_t b = 0; b < Wx; b += 32) {
+    const bool act = b + lane < Wx;
+    const uint32_t d = act ? xq[b + lane] : 0u;
+    __syncwarp();                            // this round's reads before the compacting writes
+    const uint32_t pos = d & 0xFFFFu, len = d >> 16;
+    const uint32_t a = pos & ~3u, sh = (pos & 3u) * 8;
+    const uint32_t w0 = *reinterpret_cast<const uint32_t*>(tv.sb + a);
+    const uint32_t w1 = *reinterpret_cast<const uint32_t*>(tv.sb + a + 4);
+    const uint32_t key = exact_key30_bf(__funnelshift_r(w0, w1, sh), (w1 >> sh) & 0xFFu, max(len, 1u));
+    bool miss = act;
+    if (act && P.comb) miss = !comb_add(ctab, key);
+    const uint32_t ma = __ballot_sync(kFull, miss);
+    if (miss) xq[nx + __popc(ma & lanemask_lt())] = key;
+    nx += __popc(ma);
+  }
+  if (nx + nl == 0) return;
+  const uint32_t packed = nx | (nl << kCbShift);
+  const Slot slot = reserve<kWC>(P, oc, outh, packed, P.out_cap);
+  uint8_t* half = outh + slot.half * Cfg<kWC>::kOutHalf;
+  uint32_t* sh = reinterpret_cast<uint32_t*>(half);
+  ulonglong2* top = reinterpret_cast<ulonglong2*>(half + Cfg<kWC>::kOutHalf);   // queued entry i: top[-1 - i]
+  const uint32_t kb0 = cur_cb(slot.base), ka = cur_ca(slot.base);
+  __syncwarp();
+  for (uint32_t i = lane; i < nx; i += 32) sh[ka + i] = xq[i];
+  for (uint32_t q = lane; q < nl; q += 32) {           // lane-parallel keys of the long words
+    const uint32_t e = hq[q];
+    const long long p = tv.sbase + static_cast<long long>(e & 0x7FFFu);
+    const uint32_t len = e >> 15;
+    ulonglong2 ent;
+    if (len <= kMidMax) {                                // mid stream: exact 48-bit key, no kref
+      ent = make_ulonglong2(exact_key(bytes8_at(P, tv, p, len), len), 0ULL);
+    } else {
+      ent = make_ulonglong2(key_at(P, tv, p, len), (reinterpret_cast<uint64_t>(P.rec + p) << 16) | len);
+    }
+    top[-1 - static_cast<int>(kb0 + q)] = ent;
+  }
+  commit(oc, slot, packed);
+}
+
+// WordCount map warps in SIO mode: windows from the shared counter (tile order), the stage
+// header read once per tile change, the window loop of wc_window.
+__device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
+  constexpr int W = kWC;
+  constexpr int kStages = Cfg<W>::kStages;
+  const uint32_t warp = threadIdx.x >> 5;
+  uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
+  uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout<W>::ready);
+  uint8_t* outh = smem + Layout<W>::out;
+  uint32_t* hq = reinterpret_cast<uint32_t*>(smem + Layout<kWC>::hq) + warp * Cfg<kWC>::kHashQ;
+  uint32_t* xq = reinterpret_cast<uint32_t*>(smem + Layout<kWC>::xq) + warp * Cfg<kWC>::kXQ;
+  uint32_t* ctab = reinterpret_cast<uint32_t*>(smem + Layout<kWC>::comb);
+  uint32_t have_it = ~0u;
+  long long t = 0, sbase = 0, hi = 0, stg_hi = 0;
+  for (;;) {
+    const uint32_t g = lane0_atom_add_shared(&oc->win_next, 1u);
+    const uint32_t it = g / kNWin, w = g % kNWin;
+    const uint32_t s = it % kStages;
+    if (it != have_it) {   // wait for the tile's record-start bitmap, then its header
+      map_wait(P, ready + s, (it / kStages) & 1u, kReadyWaitNs);
+      const StageHdr* hd = reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
+      t = hd->t;
+      sbase = hd->sbase;
+      hi = hd->hi;
+      stg_hi = hd->stg_hi;
+      have_it = it;
+    }
+    if (t < 0) break;
+    const long long wp = sbase + kLead + static_cast<long long>(w) * kWin;
+    if (wp < hi) {   // warp-uniform
+      const TileView tv{smem + Layout<W>::bytes + s * kStageBytes,
+                        reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits), sbase, stg_hi, 0,
+                        0};
+      wc_window(P, oc, outh, tv, wp, xq, hq, ctab);
+    }
+    __syncwarp();
+    lane0_mbar_arrive(&empty[s]);
+  }
 }
 
 // InvertedIndex URL queue (per map warp, in the hq region): the markers of a window are queued as
@@ -1600,14 +1790,18 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   uint32_t kseq = 0, have_it = ~0u;
   uint32_t qn = 0;   // II: queued URLs of this warp (ii_drain)
   StageHdr hd{};
-  const bool sm_fast = W == kSM && !P.dyn;
+  bool fast = W == kSM && !P.dyn;
   if constexpr (W == kSM) {
-    if (sm_fast) {   // (SO / G ablation: a separate instantiation, no per-load mode test on the SIO path)
+    if (fast) {   // (SO / G ablation: a separate instantiation, no per-load mode test on the SIO path)
       if (P.so) sm_fast_loop<true>(P, smem, oc);
       else sm_fast_loop<false>(P, smem, oc);
     }
   }
-  for (uint32_t it = 0; !sm_fast; ++it) {
+  if constexpr (W == kWC) {
+    fast = !P.so && !P.si && P.wc_bal && P.dyn && P.wc_fast;
+    if (fast) wc_map_loop(P, smem, oc);
+  }
+  for (uint32_t it = 0; !fast; ++it) {
     uint32_t w = 0;
     if constexpr (W != kKM) {
       uint32_t g = 0;
@@ -1780,7 +1974,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
     }
   }
   if (threadIdx.x == 0) {
-    const uint32_t cur = *reinterpret_cast<volatile unsigned int*>(&oc->cur);
+    const uint32_t cur = ld_acquire_cta_shared_u32(&oc->cur);
     seal<W>(P, oc, cur_gen(cur), cur_gen(cur) % kNOut, cur & kCntBits, true);
   }
 }
@@ -1794,12 +1988,10 @@ __global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
     oc->cur = 0;
     oc->final_seq = 0;
     for (int b = 0; b < kNOut; ++b) { oc->fbase[b] = 0; oc->committed[b] = 0; oc->fcount[b] = 0; }
-    oc->nflush = 0;
-    oc->npads = 0;
     oc->nsealed = 0;
     oc->is_final = 0;
     oc->win_next = 0;
-    for (int b = 0; b < kNOut; ++b) { mbar_init(&oc->req[b], 1); mbar_init(&oc->done[b], kNFlush); }
+    for (int b = 0; b < kNOut; ++b) { mbar_init(&oc->req[b], 1); mbar_init(&oc->done[b], 1); }
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
     uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
     uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout<W>::ready);
@@ -1835,7 +2027,7 @@ __global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
   const uint32_t warp = threadIdx.x >> 5;
   if (warp >= static_cast<uint32_t>(nmap<W>()) && warp < static_cast<uint32_t>(nmap<W>() + kNProd))
     producer_loop<W>(P, smem, warp - nmap<W>());
-  else if (warp >= static_cast<uint32_t>(nmap<W>() + kNProd)) flush_loop<W>(P, smem, oc);
+  else if (warp >= static_cast<uint32_t>(nmap<W>() + kNProd)) flush_loop<W>(P, smem, oc, warp - nmap<W>() - kNProd);
   else map_loop<W>(P, smem, oc);
 }
 
@@ -1909,6 +2101,13 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.si = (a.flags & 2u) ? 1u : 0u;   // MR_FLAG_NO_SMEM_OUT
   P.sm_lines = (W == kSM && (a.flags & 0x200u)) ? 1u : 0u;   // MR_FLAG_SM_LINES
   P.wc_bal = map_wc_balanced();
+  {
+    static uint32_t fast = [] {
+      const char* e = getenv("BMR_WC_FAST");
+      return e ? static_cast<uint32_t>(atoi(e)) : 1u;
+    }();
+    P.wc_fast = fast;
+  }
   if (P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>((P.ntiles + 255) / 256);

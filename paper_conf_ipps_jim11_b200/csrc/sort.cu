@@ -67,7 +67,7 @@ __global__ void __launch_bounds__(256) k_hist(const K* __restrict__ keys, uint64
 template <typename K, int IPT, bool kPay, int kBins, int kSlots = 0>
 struct SortSmem {
   static constexpr int kTile = kSortThreads * IPT;
-  uint32_t mm[kSlots > 0 ? kSlots : 1][kWarps][kSlots > 0 ? kBins : 1];   // match masks (kVar bit 6)
+  uint32_t mm[kSlots > 0 ? kSlots : 1][kWarps][kSlots > 0 ? kBins : 1];   // match masks (kOrMatch)
   K keys[kTile];
   uint32_t idx[kPay ? kTile : 1];
   uint32_t wcnt[kWarps][kBins];    // per-warp digit counters, then warp-exclusive offsets
@@ -78,14 +78,14 @@ struct SortSmem {
 };
 
 
-// One LSD pass over the digit [shift, shift + kBits) (kBits 8: 256 bins, one digit per thread;
-// kBits 9: 512 bins, two adjacent digits per thread).
-// kVar bit 0: rank with one shared atomic per match group (1) or a read-modify-write of the
-// warp counter per step (0); bit 1: tile histogram by shared atomics before ranking, published
-// as an early aggregate (1), or summed from the warp counters after ranking (0).
+// One LSD pass over the digit [shift, shift + 8) (256 bins, one digit per thread).
+// kOrMatch: rank with shared-memory match masks (one RED.OR of the lane bit per key into a
+// per-warp digit slot, 4 slots in flight) instead of match.any — faster for a first pass whose
+// 32-key groups carry many distinct digits (choose_rank_kind32).
 // kPay: carry the u32 permutation payload (false: keys only, idx_in / idx_out unused).
-// kLookWindow: predecessor status words fetched per look-back step (per digit).
-template <typename K, bool kFirst, int kVar, int IPT, int MINB, bool kPay, int kBits, int kLookWindow = 4>
+// The tile histogram is built before the ranking and published at once as the tile's early
+// aggregate; kLookWindow predecessor status words are fetched per look-back step (per digit).
+template <typename K, bool kFirst, bool kOrMatch, int IPT, int MINB, bool kPay, int kLookWindow = 4>
 __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __restrict__ keys_in,
                                                                const uint32_t* __restrict__ idx_in,
                                                                K* __restrict__ keys_out,
@@ -93,17 +93,12 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
                                                                uint32_t shift, const uint32_t* __restrict__ bases,
                                                                uint64_t* status, uint32_t epoch,
                                                                unsigned int* tile_counter) {
-  constexpr int kBins = 1 << kBits, kDPT = kBins / kSortThreads;
+  constexpr int kBins = 256, kDPT = kBins / kSortThreads;
   constexpr uint32_t kMask = kBins - 1;
   constexpr int kSortIPT = IPT;
-  constexpr int kSlots = (kVar & 64) ? 4 : 0;
+  constexpr int kSlots = kOrMatch ? 4 : 0;
   using Smem = SortSmem<K, IPT, kPay, kBins, kSlots>;
   constexpr int kSortTile = Smem::kTile;
-  constexpr bool kAtomicRank = (kVar & 1) != 0, kEarly = (kVar & 2) != 0;
-  constexpr bool kBackoff = (kVar & 4) != 0, kMatchHist = (kVar & 8) != 0, kBallotPeers = (kVar & 16) != 0;
-  constexpr bool kBallotAll = (kVar & 32) != 0, kOrMatch = (kVar & 64) != 0;
-  // diagnostics only (tools/micro/sort_bench; wrong output): 128 = no look-back, 256 = no global write
-  constexpr bool kDiagNoLook = (kVar & 128) != 0, kDiagNoWrite = (kVar & 256) != 0;
   static_assert(kDPT >= 1 && kDPT * kSortThreads == kBins, "bins must be a multiple of the block size");
   extern __shared__ __align__(16) uint8_t raw[];
   Smem& S = *reinterpret_cast<Smem*>(raw);
@@ -126,14 +121,11 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
   }
   const uint32_t d0 = tid * kDPT;   // this thread's digits: d0 .. d0 + kDPT - 1
   uint32_t tcount[kDPT];
-#pragma unroll
-  for (int q = 0; q < kDPT; ++q) tcount[q] = 0;
   uint64_t* my = status + static_cast<uint64_t>(tile) * kBins + d0;
   if constexpr (kOrMatch) {
-    // kVar bit 6: peer masks through shared memory (one RED.OR of the lane bit per key into a
-    // per-warp digit slot, read back after a warp barrier, cleared by the group's leader), 4
-    // slots so that 4 keys of a thread are matched per round; the leader issues the tile
-    // histogram and warp-counter atomics (applied in issue order: stable ranks).
+    // peer masks through shared memory (read back after a warp barrier, cleared by the group's
+    // leader); the leader issues the tile histogram and warp-counter atomics (applied in issue
+    // order: stable ranks)
 #pragma unroll
     for (int j0 = 0; j0 < kSortIPT; j0 += kSlots) {
       uint32_t pm[kSlots];
@@ -157,7 +149,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
         rank[j0 + q] = 0;
         if (lane == 31u - __clz(pm[q])) {
           S.mm[q][warp][dj] = 0;
-          if constexpr (kEarly) atomicAdd(&S.hist[dj], __popc(pm[q]));
+          atomicAdd(&S.hist[dj], __popc(pm[q]));
           rank[j0 + q] = atomicAdd(&S.wcnt[warp][dj], __popc(pm[q]));
         }
       }
@@ -167,105 +159,28 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
         rank[j0 + q] = __shfl_sync(0xffffffffu, rank[j0 + q], 31 - __clz(pm[q])) + __popc(pm[q] & lanemask_lt());
       }
     }
-    if constexpr (kEarly) {
-      __syncthreads();
-#pragma unroll
-      for (int q = 0; q < kDPT; ++q) {
-        tcount[q] = S.hist[d0 + q];
-        st_relaxed_gpu_u64(my + q, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount[q]));
-      }
-    }
-  } else if constexpr (kBallotAll) {
-    // kVar bit 5: peer masks from kBits ballots per key (no match.any: ncu C5 round 1 put 48% of
-    // the stall samples on the instruction consuming the MATCH result).  Per key group (equal
-    // digits in the warp) the highest lane issues one shared atomic for the tile histogram and
-    // one for the warp's digit counter; a warp's atomics to one counter are applied in issue
-    // order (j order), so ranks stay stable.  The tile histogram is published right after.
-#pragma unroll
-    for (int j0 = 0; j0 < kSortIPT; j0 += 8) {
-      uint32_t peers[8];
-#pragma unroll
-      for (int j = j0; j < j0 + 8 && j < kSortIPT; ++j) {
-        const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & kMask;
-        uint32_t pm = 0xffffffffu;
-#pragma unroll
-        for (int b = 0; b < kBits; ++b) {
-          const uint32_t bal = __ballot_sync(0xffffffffu, (dj >> b) & 1u);
-          pm &= ((dj >> b) & 1u) ? bal : ~bal;
-        }
-        peers[j - j0] = pm;
-        rank[j] = 0;
-        if (lane == 31u - __clz(pm)) {
-          if constexpr (kEarly) atomicAdd(&S.hist[dj], __popc(pm));
-          rank[j] = atomicAdd(&S.wcnt[warp][dj], __popc(pm));
-        }
-      }
-#pragma unroll
-      for (int j = j0; j < j0 + 8 && j < kSortIPT; ++j)
-        rank[j] = __shfl_sync(0xffffffffu, rank[j], 31 - __clz(peers[j - j0])) + __popc(peers[j - j0] & lanemask_lt());
-    }
-    if constexpr (kEarly) {
-      __syncthreads();
-#pragma unroll
-      for (int q = 0; q < kDPT; ++q) {
-        tcount[q] = S.hist[d0 + q];
-        st_relaxed_gpu_u64(my + q, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount[q]));
-      }
-    }
-  } else {
-  if constexpr (kEarly) {
-    // 1. tile histogram first, published immediately (early aggregate for the successors)
-    if constexpr (kMatchHist) {   // one shared atomic per group of equal digits in the warp
-#pragma unroll
-      for (int j = 0; j < kSortIPT; ++j) {
-        const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & kMask;
-        const uint32_t peers = __match_any_sync(0xffffffffu, dj);
-        if (lane == static_cast<uint32_t>(__ffs(peers) - 1)) atomicAdd(&S.hist[dj], __popc(peers));
-      }
-    } else {
-#pragma unroll
-      for (int j = 0; j < kSortIPT; ++j) atomicAdd(&S.hist[static_cast<uint32_t>(key[j] >> shift) & kMask], 1u);
-    }
     __syncthreads();
 #pragma unroll
     for (int q = 0; q < kDPT; ++q) {
       tcount[q] = S.hist[d0 + q];
       st_relaxed_gpu_u64(my + q, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount[q]));
     }
-  }
-  // 2. stable warp-level ranking (element order == (j, lane) order inside the warp)
-  if constexpr (kAtomicRank) {
-    // the leader of each match group reserves the group's slots with one shared atomicAdd; a
-    // warp's atomics are applied in issue order, their results are consumed afterwards
-    uint32_t peers[kSortIPT];
-#pragma unroll
-    for (int j = 0; j < kSortIPT; ++j) {
-      const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & kMask;
-      peers[j] = __match_any_sync(0xffffffffu, dj);
-      rank[j] = 0;
-      if (lane == static_cast<uint32_t>(__ffs(peers[j]) - 1)) rank[j] = atomicAdd(&S.wcnt[warp][dj], __popc(peers[j]));
-    }
-#pragma unroll
-    for (int j = 0; j < kSortIPT; ++j)
-      rank[j] = __shfl_sync(0xffffffffu, rank[j], __ffs(peers[j]) - 1) + __popc(peers[j] & lanemask_lt());
   } else {
+    // 1. tile histogram first, published immediately (early aggregate for the successors)
+#pragma unroll
+    for (int j = 0; j < kSortIPT; ++j) atomicAdd(&S.hist[static_cast<uint32_t>(key[j] >> shift) & kMask], 1u);
+    __syncthreads();
+#pragma unroll
+    for (int q = 0; q < kDPT; ++q) {
+      tcount[q] = S.hist[d0 + q];
+      st_relaxed_gpu_u64(my + q, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount[q]));
+    }
+    // 2. stable warp-level ranking (element order == (j, lane) order inside the warp): match.any
+    //    groups, the group leader reads and advances the warp's digit counter
 #pragma unroll
     for (int j = 0; j < kSortIPT; ++j) {
       const uint32_t dj = static_cast<uint32_t>(key[j] >> shift) & kMask;
-      uint32_t peers;
-      if constexpr (kBallotPeers) {
-        // lanes with the same digit by bit slicing: kBits ballots (short latency, independent of
-        // the other steps) instead of match.any (ncu: 49% of the stall samples wait on MATCH)
-        peers = 0xffffffffu;
-#pragma unroll
-        for (int b = 0; b < kBits; ++b) {
-          const bool bit = (dj >> b) & 1u;
-          const uint32_t bal = __ballot_sync(0xffffffffu, bit);
-          peers &= bit ? bal : ~bal;
-        }
-      } else {
-        peers = __match_any_sync(0xffffffffu, dj);
-      }
+      const uint32_t peers = __match_any_sync(0xffffffffu, dj);
       const uint32_t leader = __ffs(peers) - 1;
       uint32_t before = 0;
       if (lane == leader) {
@@ -277,16 +192,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
       rank[j] = before + __popc(peers & lanemask_lt());
     }
   }
-  }   // !kBallotAll
   __syncthreads();
-  if constexpr (!kEarly) {
-#pragma unroll
-    for (int q = 0; q < kDPT; ++q) {
-#pragma unroll
-      for (int w = 0; w < kWarps; ++w) tcount[q] += S.wcnt[w][d0 + q];
-      st_relaxed_gpu_u64(my + q, pack_status(epoch, tile == 0 ? kPrefix : kAgg, tcount[q]));
-    }
-  }
   // (a thread reads and rewrites only the counters of its own digits: no barrier needed here)
   // 3. per digit: the tile-local digit start (block scan of the tile counts), then every warp's
   //    counter becomes its tile-local scatter base for the digit (digit start + earlier warps)
@@ -332,7 +238,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
     uint32_t excl[kDPT];
 #pragma unroll
     for (int q = 0; q < kDPT; ++q) excl[q] = 0;
-    if (tile > 0 && !kDiagNoLook) {
+    if (tile > 0) {
       long long p[kDPT];
       bool done[kDPT];
 #pragma unroll
@@ -346,7 +252,7 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
             sv[q][i] = (!done[q] && p[q] - i >= 0)
                            ? ld_relaxed_gpu_u64(status + static_cast<uint64_t>(p[q] - i) * kBins + d0 + q)
                            : 0;
-        bool all = true, moved = false;
+        bool all = true;
 #pragma unroll
         for (int q = 0; q < kDPT; ++q) {
           if (done[q]) continue;
@@ -363,12 +269,8 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
           }
           if (fin) done[q] = true;
           else { p[q] -= adv; all = false; }
-          moved = moved || fin || adv > 0;
         }
         if (all) break;
-        if constexpr (kBackoff) {
-          if (!moved) __nanosleep(100);
-        }
       }
 #pragma unroll
       for (int q = 0; q < kDPT; ++q) st_relaxed_gpu_u64(my + q, pack_status(epoch, kPrefix, excl[q] + tcount[q]));
@@ -380,7 +282,6 @@ __global__ void __launch_bounds__(kSortThreads, MINB) k_onesweep(const K* __rest
   __syncthreads();
   // 6. contiguous per-digit runs to global memory
   const uint32_t nvalid = static_cast<uint32_t>(min(static_cast<uint64_t>(kSortTile), m - tbase));
-  if constexpr (kDiagNoWrite) return;
   if (nvalid == static_cast<uint32_t>(kSortTile)) {
     // full tile: unrolled in groups of 8, so the SMEM reads of 8 elements are in flight together
     // (a rolled loop serialises LDS key -> LDS goff -> STG per element)
@@ -508,94 +409,48 @@ cudaError_t launch_hist32(const uint32_t* keys, uint64_t m, uint32_t* hist, int 
   return hist_impl<uint32_t>(keys, m, hist, nd, bits, num_sms, s);
 }
 
-int sort_variant() {
-  static int v = [] {
-    const char* e = getenv("BMR_SORT_VARIANT");
-    return e ? atoi(e) & 1 : 0;
-  }();
-  return v;
-}
-// u32 keys-only passes: kVar of k_onesweep (bit 0 atomic ranking, bit 1 early histogram)
-int sort_variant32() {
-  static int v = [] {
-    const char* e = getenv("BMR_SORT_VARIANT32");
-    return e ? atoi(e) : 2;
-  }();
-  return v;
-}
-// Tile shapes (keys per thread x 256 threads, CTAs per SM), chosen at start-up (BMR_SORT_CFG):
-//   payload passes (u64 key + u32 index): cfg 0 = 16 keys, 3 CTAs/SM; cfg 1 = 12 keys, 4 CTAs
-//   keys-only u64 passes: 16 keys, 3 CTAs/SM (cfg 1: 24 keys, 2 CTAs)
-//   keys-only u32 passes: 24 keys, 3 CTAs/SM (cfg 1: 32 keys, 2 CTAs)
-// (measured on C5 in round 1: 16 x 256 with the early tile histogram and a look-back window of
-// 4 was the fastest u64 shape among 8/12/16/20/24 keys, 9-bit digits, windows 1..16, spin
-// back-off and match-aggregated histogram atomics.)
-int sort_cfg() {
-  static int c = [] {
-    const char* e = getenv("BMR_SORT_CFG");
-    return e ? atoi(e) & 3 : 0;
-  }();
-  return c;
-}
-// u32 keys-only shapes (keys per thread, CTAs per SM): cfg 0 (24, 3), 1 (32, 2), 2 (16, 4), 3 (24, 2)
-static const int kIPT32[4] = {24, 32, 16, 24};
+// Tile shapes (keys per thread x 256 threads, CTAs per SM), measured on C5 in round 1 (16 keys
+// with the early tile histogram and a look-back window of 4 was the fastest u64 shape among
+// 8/12/16/20/24 keys, 9-bit digits, windows 1..16, spin back-off and match-aggregated histogram
+// atomics; 24 keys x 3 CTAs the fastest u32 keys-only shape among 16/20/24/32; ballot-sliced
+// peer masks and larger look-back windows were slower — tools/micro/sort_bench.cu):
+//   payload passes (u64 key + u32 index): 16 keys, 3 CTAs/SM
+//   keys-only u64 passes: 16 keys, 3 CTAs/SM; keys-only u32 passes: 24 keys, 3 CTAs/SM
+constexpr int kIptPay = 16, kIptKeys = 16, kIptKeys32 = 24;
 // u32 pass ranking by digit statistics: E = expected number of distinct digits among 32 keys
 // (sum over bins of 1 - (1 - p_b)^32).  match.any slows down with many distinct values per warp,
 // the shared-memory OR masks with many equal ones (same-address atomics serialise); measured with
 // tools/micro/sort_bench (round 1): first pass over Zipf keys (E 28.6) 3.37 vs 4.59 ms.  Only the
 // first pass sees the input order: after it, equal keys are adjacent and the warps' digits are
 // far less diverse than E says (later passes: match 2.4-3.4 ms, OR masks 3.8-4.6 ms), so they
-// keep match.any.  BMR_SORT_ADAPT = threshold on E (default 24; 0 disables: env variant).
+// keep match.any.  Threshold 24 on E.
 int choose_rank_kind32(const uint32_t* hist, uint64_t m, bool first_pass) {
-  static double thr = [] {
-    const char* e = getenv("BMR_SORT_ADAPT");
-    return e ? atof(e) : 24.0;
-  }();
-  if (thr <= 0 || m == 0) return 0;
+  if (m == 0) return kRankMatch;
   double e = 0;
   for (int b = 0; b < 256; ++b) e += 1.0 - std::pow(1.0 - static_cast<double>(hist[b]) / static_cast<double>(m), 32);
-  if (getenv("BMR_SORT_DEBUG")) fprintf(stderr, "[bmr] u32 pass: E[distinct digits / 32 keys] = %.2f\n", e);
-  return (first_pass && e >= thr) ? 66 : 2;
+  return (first_pass && e >= 24.0) ? kRankOrMask : kRankMatch;
 }
 
-int sort_tile() { return kSortThreads * (sort_cfg() == 1 ? 12 : 16); }
-int sort_tile_keys() { return kSortThreads * (sort_cfg() == 1 ? 24 : 16); }
-int sort_variant32();
-int sort_tile_keys32() {
-  const int v = sort_variant32();
-  return kSortThreads * (v == 19 || v == 21 || v == 22 || v == 35 || v == 36 || v == 67 || v == 68 ? 16 : v == 20 ? 20 : v == 37 ? 32
-                                                                                          : kIPT32[sort_cfg()]);
-}
+int sort_tile() { return kSortThreads * kIptPay; }
+int sort_tile_keys() { return kSortThreads * kIptKeys; }
+int sort_tile_keys32() { return kSortThreads * kIptKeys32; }
 
-template <typename K, bool kFirst, int kVar, int IPT, int MINB, bool kPay, int LW = 4>
+template <typename K, bool kFirst, bool kOrMatch, int IPT, int MINB, bool kPay>
 static void launch_os(unsigned tiles, const K* keys_in, const uint32_t* idx_in, K* keys_out, uint32_t* idx_out,
                       uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status, uint32_t epoch,
                       unsigned int* tile_counter, cudaStream_t s) {
-  const auto k = &k_onesweep<K, kFirst, kVar, IPT, MINB, kPay, 8, LW>;
-  const size_t smem = sizeof(SortSmem<K, IPT, kPay, 256, (kVar & 64) ? 4 : 0>);
+  const auto k = &k_onesweep<K, kFirst, kOrMatch, IPT, MINB, kPay>;
+  const size_t smem = sizeof(SortSmem<K, IPT, kPay, 256, kOrMatch ? 4 : 0>);
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
   k<<<tiles, kSortThreads, smem, s>>>(keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch,
                                       tile_counter);
 }
 
 #define BMR_OS_ARGS tiles, keys_in, idx_in, keys_out, idx_out, m, shift, bases, status, epoch, tile_counter, s
-// kVar 2: early tile histogram (published before ranking), read-modify-write warp ranking;
-// kVar 3: the same with one shared atomic per match group for the ranking
-template <bool kFirst, int kVar>
-static void launch_pay(unsigned tiles, const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out,
-                       uint32_t* idx_out, uint64_t m, uint32_t shift, const uint32_t* bases, uint64_t* status,
-                       uint32_t epoch, unsigned int* tile_counter, cudaStream_t s) {
-  if (sort_cfg() == 1) launch_os<uint64_t, kFirst, kVar, 12, 4, true>(BMR_OS_ARGS);   // cfg 1: 12 keys, 4 CTAs
-  else launch_os<uint64_t, kFirst, kVar, 16, 3, true>(BMR_OS_ARGS);
-}
-
-// per-pass ranking choice of the u32 passes (launch_onesweep32's rank_kind; <= 0: BMR_SORT_VARIANT32)
-static thread_local int g_rank_kind = 0;
-
 template <typename K>
 static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* keys_out, uint32_t* idx_out, uint64_t m,
                                  int digit, int bits, const uint32_t* bases_all, uint64_t* status, uint32_t epoch,
-                                 unsigned int* tile_counter, cudaStream_t s) {
+                                 unsigned int* tile_counter, cudaStream_t s, int rank_kind) {
   if (m == 0) return cudaSuccess;
   const bool keys_only = idx_out == nullptr;
   if (bits != 8) return cudaErrorInvalidValue;
@@ -606,56 +461,17 @@ static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* ke
   if (e != cudaSuccess) return e;
   const uint32_t shift = static_cast<uint32_t>(bits * digit);
   const uint32_t* bases = bases_all + kBinStride * digit;
-  const bool first = idx_in == nullptr;
+  const bool orm = rank_kind == kRankOrMask;
   if constexpr (sizeof(K) == 4) {
-    if (sort_cfg() == 1) {
-      launch_os<K, false, 2, 32, 2, false>(BMR_OS_ARGS);
-    } else if (sort_cfg() == 2) {
-      launch_os<K, false, 2, 16, 4, false>(BMR_OS_ARGS);
-    } else if (sort_cfg() == 3) {
-      launch_os<K, false, 2, 24, 2, false>(BMR_OS_ARGS);
-    } else {
-      switch (g_rank_kind > 0 ? g_rank_kind : sort_variant32()) {
-        case 0: launch_os<K, false, 0, 24, 3, false>(BMR_OS_ARGS); break;
-        case 1: launch_os<K, false, 1, 24, 3, false>(BMR_OS_ARGS); break;
-        case 3: launch_os<K, false, 3, 24, 3, false>(BMR_OS_ARGS); break;
-        case 18: launch_os<K, false, 18, 24, 3, false>(BMR_OS_ARGS); break;
-        case 19: launch_os<K, false, 18, 16, 3, false>(BMR_OS_ARGS); break;
-        case 20: launch_os<K, false, 2, 20, 3, false>(BMR_OS_ARGS); break;
-        case 21: launch_os<K, false, 2, 16, 3, false>(BMR_OS_ARGS); break;
-        case 22: launch_os<K, false, 2, 16, 3, false, 8>(BMR_OS_ARGS); break;
-        case 23: launch_os<K, false, 2, 24, 3, false, 8>(BMR_OS_ARGS); break;
-        case 34: launch_os<K, false, 34, 24, 3, false>(BMR_OS_ARGS); break;   // ballot peers, early hist, leader atomics
-        case 35: launch_os<K, false, 34, 16, 3, false>(BMR_OS_ARGS); break;
-        case 36: launch_os<K, false, 34, 16, 4, false>(BMR_OS_ARGS); break;
-        case 37: launch_os<K, false, 34, 32, 2, false>(BMR_OS_ARGS); break;
-        case 38: launch_os<K, false, 34, 24, 3, false, 8>(BMR_OS_ARGS); break;    // look-back windows 8 / 16 / 32
-        case 39: launch_os<K, false, 34, 24, 3, false, 16>(BMR_OS_ARGS); break;
-        case 40: launch_os<K, false, 34, 24, 3, false, 32>(BMR_OS_ARGS); break;
-        case 41: launch_os<K, false, 2, 24, 3, false, 16>(BMR_OS_ARGS); break;
-        case 130: launch_os<K, false, 130, 24, 3, false>(BMR_OS_ARGS); break;   // diagnostics (wrong output)
-        case 258: launch_os<K, false, 258, 24, 3, false>(BMR_OS_ARGS); break;
-        case 386: launch_os<K, false, 386, 24, 3, false>(BMR_OS_ARGS); break;
-        case 194: launch_os<K, false, 194, 24, 3, false>(BMR_OS_ARGS); break;
-        case 322: launch_os<K, false, 322, 24, 3, false>(BMR_OS_ARGS); break;
-        case 66: launch_os<K, false, 66, 24, 3, false>(BMR_OS_ARGS); break;   // RED.OR match masks, 4 slots
-        case 67: launch_os<K, false, 66, 16, 3, false>(BMR_OS_ARGS); break;
-        case 68: launch_os<K, false, 66, 16, 4, false>(BMR_OS_ARGS); break;
-        case 69: launch_os<K, false, 66, 24, 2, false>(BMR_OS_ARGS); break;
-        default: launch_os<K, false, 2, 24, 3, false>(BMR_OS_ARGS); break;
-      }
-    }
+    if (orm) launch_os<K, false, true, kIptKeys32, 3, false>(BMR_OS_ARGS);
+    else launch_os<K, false, false, kIptKeys32, 3, false>(BMR_OS_ARGS);
   } else if (keys_only) {
-    if (g_rank_kind == 66) launch_os<K, false, 66, 16, 3, false>(BMR_OS_ARGS);   // OR-mask ranking (first pass)
-    else if (sort_cfg() == 1) launch_os<K, false, 2, 24, 2, false>(BMR_OS_ARGS);   // cfg 1: 24 keys, 2 CTAs
-    else launch_os<K, false, 2, 16, 3, false>(BMR_OS_ARGS);
+    if (orm) launch_os<K, false, true, kIptKeys, 3, false>(BMR_OS_ARGS);
+    else launch_os<K, false, false, kIptKeys, 3, false>(BMR_OS_ARGS);
+  } else if (idx_in == nullptr) {   // first payload pass: identity permutation
+    launch_os<K, true, false, kIptPay, 3, true>(BMR_OS_ARGS);
   } else {
-    switch ((sort_variant() ? 1 : 0) | (first ? 2 : 0)) {
-      case 0: launch_pay<false, 2>(BMR_OS_ARGS); break;
-      case 1: launch_pay<false, 3>(BMR_OS_ARGS); break;
-      case 2: launch_pay<true, 2>(BMR_OS_ARGS); break;
-      default: launch_pay<true, 3>(BMR_OS_ARGS); break;
-    }
+    launch_os<K, false, false, kIptPay, 3, true>(BMR_OS_ARGS);
   }
   count_launch();
   return cudaGetLastError();
@@ -665,16 +481,14 @@ static cudaError_t onesweep_impl(const K* keys_in, const uint32_t* idx_in, K* ke
 cudaError_t launch_onesweep(const uint64_t* keys_in, const uint32_t* idx_in, uint64_t* keys_out, uint32_t* idx_out,
                             uint64_t m, int digit, int bits, const uint32_t* bases_all, uint64_t* status,
                             uint32_t epoch, unsigned int* tile_counter, cudaStream_t s, int rank_kind) {
-  g_rank_kind = rank_kind;
   return onesweep_impl<uint64_t>(keys_in, idx_in, keys_out, idx_out, m, digit, bits, bases_all, status, epoch,
-                                 tile_counter, s);
+                                 tile_counter, s, rank_kind);
 }
 cudaError_t launch_onesweep32(const uint32_t* keys_in, uint32_t* keys_out, uint64_t m, int digit, int bits,
                               const uint32_t* bases_all, uint64_t* status, uint32_t epoch,
                               unsigned int* tile_counter, cudaStream_t s, int rank_kind) {
-  g_rank_kind = rank_kind;
   return onesweep_impl<uint32_t>(keys_in, nullptr, keys_out, nullptr, m, digit, bits, bases_all, status, epoch,
-                                 tile_counter, s);
+                                 tile_counter, s, rank_kind);
 }
 
 template <typename T>

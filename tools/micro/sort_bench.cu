@@ -1,7 +1,7 @@
 // Microbenchmark of the u32 keys-only onesweep passes (links build/sort.o): m random keys of
-// `bits` bits, Zipf-like or uniform; times the histogram and each LSD pass with CUDA events for
-// the variants given on the command line (BMR_SORT_VARIANT32 is read once per process, so run one
-// variant per process).  usage: sort_bench M_millions key_bits zipf(0/1)
+// `bits` bits, Zipf-like or uniform; times the histogram and each LSD pass with CUDA events,
+// every pass ranked with match.any (rank 0) or the shared-memory OR masks (rank 1).
+// usage: sort_bench M_millions key_bits zipf(0/1) rank(0/1)
 #include <cstdio>
 #include <cstdlib>
 #include <vector>
@@ -26,6 +26,7 @@ __global__ void gen(uint32_t* k, uint64_t m, uint32_t bits, int zipf) {
 int main(int argc, char** argv) {
   const uint64_t m = (uint64_t)(argc > 1 ? atof(argv[1]) : 672) * 1000000ull;
   const int bits = argc > 2 ? atoi(argv[2]) : 30, zipf = argc > 3 ? atoi(argv[3]) : 1;
+  const int rank = argc > 4 ? atoi(argv[4]) : 0;
   uint32_t *a, *b, *c, *hist, *bases; uint64_t* status; unsigned* tc;
   cudaMalloc(&a, m * 4); cudaMalloc(&b, m * 4); cudaMalloc(&c, m * 4);
   cudaMalloc(&hist, 8 * kBinStride * 4); cudaMalloc(&bases, 8 * kBinStride * 4);
@@ -52,7 +53,7 @@ int main(int argc, char** argv) {
     for (int d = 0; d < 4; ++d) {
       uint32_t* kout = (d & 1) ? c : b;
       cudaEventRecord(e0);
-      launch_onesweep32(kin, kout, m, d, 8, bases, status, epoch++, tc, 0);
+      launch_onesweep32(kin, kout, m, d, 8, bases, status, epoch++, tc, 0, rank ? kRankOrMask : kRankMatch);
       cudaEventRecord(e1); cudaEventSynchronize(e1); cudaEventElapsedTime(&ms, e0, e1);
       tot += ms;
       if (rep == 2) printf("pass %d %.3f ms (%.1f GB/s)\n", d, ms, m * 8.0 / ms / 1e6);
