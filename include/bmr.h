@@ -69,7 +69,9 @@ typedef struct {
   const void* params;        /* mr_sm_params* / mr_km_params* / NULL; copied at create */
   uint64_t input_base;       /* global byte offset of this rank's first record (SM/II offsets are global) */
   int rank, nranks;          /* nranks == 1: single GPU */
-  void* nccl_comm;           /* reserved (the exchange is moved by the caller, see mr_ingest) */
+  void* nccl_comm;           /* nranks > 1: an NCCL communicator over the nranks processes (one per GPU)
+                                from mr_comm_init — mr_group then performs the exchange itself; NULL:
+                                the caller moves the bytes (mr_partition_count / _write / mr_ingest) */
   uint64_t max_pairs_hint;   /* initial intermediate capacity in pairs (0: heuristic) */
   uint64_t heap_bytes_hint;  /* reserved */
   uint32_t flags;            /* MR_FLAG_* */
@@ -114,6 +116,11 @@ typedef struct {
    * Map CTAs (not included in `pairs`), and the words they absorbed (not emitted as pairs) */
   uint64_t pairs_partial;
   uint64_t words_combined;
+  /* the exchange inside mr_group (nranks > 1 with nccl_comm): bytes sent / received by this rank
+   * (entries + key bytes; WC / KM after the local combiner) and its device time (MR_FLAG_PROFILE) */
+  uint64_t xchg_send_bytes;
+  uint64_t xchg_recv_bytes;
+  double xchg_ms;
 } mr_stats;
 
 /* State machine: CREATED -> mr_map x k (batches append) -> mr_group -> mr_reduce -> mr_fetch
@@ -152,7 +159,13 @@ mr_status mr_map_host_lines(mr_job* job, const uint8_t* text, uint64_t nbytes);
 
 /* Group by key (§8(a) a6-a8): capacity check (grow + replay on overflow), digit histogram,
  * onesweep LSD passes over non-constant digits, segment boundaries with byte verification of
- * hashed keys (re-sort with a fresh hash on collision).  Synchronises the stream. */
+ * hashed keys (re-sort with a fresh hash on collision).  Synchronises the stream.
+ * nranks > 1 with cfg.nccl_comm: first the exchange —
+ * partition by destination rank mix64(hash of the key bytes) mod nranks (WC / KM after a local
+ * group + reduce, the combiner; II and MR_FLAG_NO_COMBINE WC raw pairs), ncclAlltoAll of the
+ * count matrix, one NCCL group of send / recv for the entries and key bytes, ingest — then the
+ * local group of the keys this rank owns.  Collective: every rank of the communicator calls
+ * mr_group.  MR_ERR_NCCL on a communication failure (detail in mr_last_error). */
 mr_status mr_group(mr_job* job);
 
 /* Reduce (§8(a) a9) and device-side output assembly.  Asynchronous. */
@@ -177,8 +190,9 @@ const char* mr_last_error(const mr_job* job);
  * global).  Records are routed to rank mix64(hash of the key bytes) mod nranks.  WC and KM first
  * run the local group + reduce as a combiner (the original MapReduce combiner; the paper uses
  * none) unless MR_FLAG_NO_COMBINE (WC only); II exchanges raw pairs.  StringMatch
- * is Map-only and has no exchange (MR_ERR_UNSUPPORTED).  The caller moves the bytes (e.g.
- * torch.distributed all_to_all_single over NCCL):
+ * is Map-only and has no exchange (MR_ERR_UNSUPPORTED).  With cfg.nccl_comm, mr_group runs these
+ * steps itself over NCCL; without it the caller moves the bytes (e.g. torch.distributed
+ * all_to_all_single, gloo in CPU-staged tests) through:
  *   1. mr_partition_count(job, counts, &entry_bytes): counts[2r] = entries for rank r,
  *      counts[2r+1] = heap bytes for rank r (host array of 2*nranks u64); synchronises.
  *   2. caller allocates device buffers of sum(entries)*entry_bytes and sum(heap) bytes;
@@ -191,6 +205,21 @@ const char* mr_last_error(const mr_job* job);
 mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_bytes);
 mr_status mr_partition_write(mr_job* job, void* entries, void* heap);
 mr_status mr_ingest(mr_job* job, const void* entries, const void* heap, const uint64_t* recv_counts);
+
+/* ---- NCCL communicator for the exchange inside mr_group ----
+ * libnccl.so.2 is loaded at run time (BMR_NCCL_LIB, else the copy already in the process — e.g.
+ * torch's — else the loader's): no link-time dependency, single-GPU jobs never load it.
+ *   mr_comm_unique_id(id): rank 0 fills MR_NCCL_ID_BYTES bytes (host buffer), which the caller
+ *     broadcasts to every rank (e.g. torch.distributed.broadcast_object_list);
+ *   mr_comm_init(id, nranks, rank, device, &comm): collective over the nranks processes; comm is
+ *     an ncclComm_t owned by the caller, passed to jobs as mr_config.nccl_comm;
+ *   mr_comm_destroy(comm) after the last job using it (NULL-safe).
+ * MR_ERR_NCCL if NCCL cannot be loaded or fails; mr_comm_backend() names the loaded NCCL. */
+#define MR_NCCL_ID_BYTES 128
+mr_status mr_comm_unique_id(void* id);
+mr_status mr_comm_init(const void* id, int nranks, int rank, int device, void** comm);
+mr_status mr_comm_destroy(void* comm);
+const char* mr_comm_backend(void);
 
 /* ---- Fused Map flush + shuffle over peer memory, InvertedIndex ----
  * Instead of partition + all-to-all, the Map's flush appends every record straight to the

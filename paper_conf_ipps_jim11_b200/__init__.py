@@ -31,7 +31,9 @@ STATUS = {0: "MR_OK", 1: "MR_ERR_INVALID", 2: "MR_ERR_STATE", 3: "MR_ERR_OOM", 4
 EXPORTS = ("mr_job_create", "mr_map", "mr_map_host", "mr_map_host_lines", "mr_group", "mr_reduce", "mr_fetch", "mr_job_reset",
            "mr_get_stats", "mr_job_destroy", "mr_status_string", "mr_last_error", "mr_sort_u64",
            "mr_partition_count", "mr_partition_write", "mr_ingest", "mr_set_xwindows", "mr_ingest_xwindow",
-           "mr_dev_alloc", "mr_dev_free", "mr_dev_zero", "mr_dev_copy", "mr_ipc_handle", "mr_ipc_open", "mr_ipc_close")
+           "mr_dev_alloc", "mr_dev_free", "mr_dev_zero", "mr_dev_copy", "mr_ipc_handle", "mr_ipc_open", "mr_ipc_close",
+           "mr_comm_unique_id", "mr_comm_init", "mr_comm_destroy", "mr_comm_backend")
+MR_NCCL_ID_BYTES = 128
 
 
 class XWindow:
@@ -146,7 +148,8 @@ class Stats(C.Structure):
                [(n, C.c_double) for n in ("map_ms", "hist_ms", "sort_ms", "seg_ms", "reduce_ms")] + \
                [("pairs_hashed", C.c_uint64), ("sort_passes_keys", C.c_uint64), ("sort_keys_ms", C.c_double),
                 ("pairs_mid", C.c_uint64), ("sort_passes_mid", C.c_uint64),
-                ("pairs_partial", C.c_uint64), ("words_combined", C.c_uint64)]
+                ("pairs_partial", C.c_uint64), ("words_combined", C.c_uint64),
+                ("xchg_send_bytes", C.c_uint64), ("xchg_recv_bytes", C.c_uint64), ("xchg_ms", C.c_double)]
 
 
 _LIB = None
@@ -158,6 +161,14 @@ def lib() -> C.CDLL:
     if _LIB is None:
         if not os.path.exists(LIB_PATH):
             raise RuntimeError(f"{LIB_PATH} not built: run __graft_entry__.build()")
+        if "BMR_NCCL_LIB" not in os.environ:   # the NCCL torch bundles (libbmr dlopens it for mr_group's exchange)
+            try:
+                import nvidia.nccl
+                cand = os.path.join(list(nvidia.nccl.__path__)[0], "lib", "libnccl.so.2")
+                if os.path.exists(cand):
+                    os.environ["BMR_NCCL_LIB"] = cand
+            except ImportError:
+                pass
         L = C.CDLL(LIB_PATH)
         vp, u64 = C.c_void_p, C.c_uint64
         L.mr_job_create.argtypes = [C.POINTER(Config), C.POINTER(vp)]
@@ -185,8 +196,13 @@ def lib() -> C.CDLL:
         L.mr_ipc_handle.argtypes = [vp, vp]
         L.mr_ipc_open.argtypes = [C.c_int, vp, vp]
         L.mr_ipc_close.argtypes = [vp]
+        L.mr_comm_unique_id.argtypes = [vp]
+        L.mr_comm_init.argtypes = [vp, C.c_int, C.c_int, C.c_int, C.POINTER(vp)]
+        L.mr_comm_destroy.argtypes = [vp]
+        L.mr_comm_backend.argtypes = []
+        L.mr_comm_backend.restype = C.c_char_p
         for f in EXPORTS:
-            if f not in ("mr_status_string", "mr_last_error"):
+            if f not in ("mr_status_string", "mr_last_error", "mr_comm_backend"):
                 getattr(L, f).restype = C.c_int
         _LIB = L
     return _LIB
@@ -211,12 +227,52 @@ def _copy(addr, nbytes, dtype=np.uint8, copy=True):
     return (a.copy() if copy else a).view(dtype)
 
 
+class Comm:
+    """An NCCL communicator created by libbmr (mr_comm_unique_id / mr_comm_init) for the exchange
+    inside mr_group: ``Job(..., comm=c)``.  ``Comm.from_torch()`` forms it over the default
+    torch.distributed group (the 128-byte id travels by broadcast_object_list: plumbing only)."""
+
+    def __init__(self, uid: bytes, nranks: int, rank: int, device: int):
+        p = C.c_void_p()
+        st = lib().mr_comm_init(C.create_string_buffer(uid, MR_NCCL_ID_BYTES), nranks, rank, device, C.byref(p))
+        if st:
+            raise MRError(st, f"mr_comm_init ({lib().mr_comm_backend().decode()})")
+        self.ptr, self.nranks, self.rank, self.device = p.value, nranks, rank, device
+
+    @staticmethod
+    def unique_id() -> bytes:
+        b = C.create_string_buffer(MR_NCCL_ID_BYTES)
+        st = lib().mr_comm_unique_id(b)
+        if st:
+            raise MRError(st, f"mr_comm_unique_id ({lib().mr_comm_backend().decode()})")
+        return b.raw
+
+    @classmethod
+    def from_torch(cls, group=None, device: int | None = None):
+        import torch
+        import torch.distributed as dist
+        rank, world = dist.get_rank(group), dist.get_world_size(group)
+        obj = [cls.unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
+        return cls(obj[0], world, rank, torch.cuda.current_device() if device is None else device)
+
+    @staticmethod
+    def backend() -> str:
+        return lib().mr_comm_backend().decode()
+
+    def close(self):
+        if getattr(self, "ptr", None):
+            lib().mr_comm_destroy(self.ptr)
+            self.ptr = None
+
+
 class Job:
-    """One MapReduce job (mr_job).  ``workload`` in {"wc", "sm", "km", "ii"}."""
+    """One MapReduce job (mr_job).  ``workload`` in {"wc", "sm", "km", "ii"}.  With ``comm`` (a
+    Comm over ``nranks`` processes) mr_group performs the multi-GPU exchange itself."""
 
     def __init__(self, workload: str, device: int = 0, stream=None, pattern: bytes | None = None,
                  centroids: np.ndarray | None = None, input_base: int = 0, flags: int = 0,
-                 max_pairs_hint: int = 0, rank: int = 0, nranks: int = 1):
+                 max_pairs_hint: int = 0, rank: int = 0, nranks: int = 1, comm: Comm | None = None):
         L = lib()
         self.workload = workload
         cfg = Config()
@@ -230,6 +286,10 @@ class Job:
         cfg.input_base = input_base
         cfg.rank, cfg.nranks = rank, nranks
         self.rank, self.nranks = rank, nranks
+        if comm is not None:
+            assert comm.nranks == nranks and comm.rank == rank, "comm does not match (rank, nranks)"
+            cfg.nccl_comm = comm.ptr
+        self.comm = comm
         cfg.max_pairs_hint = max_pairs_hint
         cfg.flags = flags
         self._keep = []

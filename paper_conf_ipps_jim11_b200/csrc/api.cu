@@ -14,6 +14,7 @@
 #include <vector>
 
 #include "bmr.h"
+#include "comm.h"
 #include "kernels.h"
 
 using namespace bmr;
@@ -341,6 +342,11 @@ struct mr_job {
   HBuf<unsigned long long> xcounts_h;
   DBuf<uint64_t> src_e, src_h;
   DBuf<XWindow> xwin;             // f-3: receive windows of the fused Map flush (InvertedIndex)
+  // the exchange inside mr_group (nranks > 1 with cfg.nccl_comm): send / receive buffers (the
+  // received heap holds the key bytes the ingested pairs reference until mr_reduce completes)
+  DBuf<uint8_t> xsend_e, xsend_h, xrecv_e, xrecv_h;
+  DBuf<uint64_t> xrecv_counts;
+  bool in_exchange = false;       // mr_group called by the exchange's own combiner step
   uint32_t xranks = 0;
   DBuf<uint32_t> km_list;
   uint32_t km_nlist = 0;
@@ -558,6 +564,65 @@ mr_status settle_map(mr_job* job) {
       return fail(job, MR_ERR_OOM, "replay still overflows");
   }
   return MR_OK;
+}
+
+}  // namespace
+
+extern "C" mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_bytes);
+extern "C" mr_status mr_partition_write(mr_job* job, void* entries, void* heap);
+extern "C" mr_status mr_ingest(mr_job* job, const void* entries, const void* heap, const uint64_t* recv_counts);
+
+namespace {
+
+// The one exchange of the multi-GPU group-by (SURVEY §8(b) mr_group with R > 1, §8(e); PAPER.md
+// L51-52: the shuffle between Map and Reduce is the framework's): partition by destination rank
+// (WC / KM: after the local combiner), ncclAlltoAll of the R x (entries, heap bytes) count
+// matrix, then ONE NCCL group of send / recv pairs for the entry and key-byte slices, all on the
+// job stream, then mr_ingest of what arrived.  Synchronises twice (the counts size the receive
+// buffers; the ingest needs the received counts on the host).
+mr_status exchange(mr_job* job) {
+  const NcclApi* a = nccl_api();
+  if (!a->ok) return fail(job, MR_ERR_NCCL, "NCCL unavailable: " + a->err);
+  const int R = job->cfg.nranks;
+  void* comm = job->cfg.nccl_comm;
+  cudaStream_t s = job->stream;
+  std::vector<uint64_t> cnt(2 * R), rc(2 * R);
+  uint64_t eb = 0;
+  job->in_exchange = true;
+  mr_status st = mr_partition_count(job, cnt.data(), &eb);   // (its local group + reduce time their own phases)
+  job->in_exchange = false;
+  if (st != MR_OK) return st;
+  Prof::Span sp{};
+  if (job->prof.on) job->prof.begin(s, sp);
+  std::vector<uint64_t> se(R + 1, 0), sh(R + 1, 0), re(R + 1, 0), rh(R + 1, 0);
+  for (int r = 0; r < R; ++r) {
+    se[r + 1] = se[r] + cnt[2 * r] * eb;
+    sh[r + 1] = sh[r] + cnt[2 * r + 1];
+  }
+  CK(job->xsend_e.ensure(se[R] + 16), "alloc send entries");
+  CK(job->xsend_h.ensure(sh[R] + 16), "alloc send heap");
+  st = mr_partition_write(job, job->xsend_e.p, job->xsend_h.p);
+  if (st != MR_OK) return st;
+  CK(job->xrecv_counts.ensure(2 * R), "alloc receive counts");
+  int nr = 0;
+  CK(nccl_alltoall_u64x2(a, reinterpret_cast<const uint64_t*>(job->xcounts.p), job->xrecv_counts.p, R, comm, s, &nr),
+     "count exchange");
+  if (nr) return fail(job, MR_ERR_NCCL, "ncclAlltoAll (counts): " + nccl_error(a, nr));
+  CK(cudaMemcpyAsync(rc.data(), job->xrecv_counts.p, 2 * R * 8, cudaMemcpyDeviceToHost, s), "D2H receive counts");
+  CK(cudaStreamSynchronize(s), "sync count exchange");
+  for (int r = 0; r < R; ++r) {
+    re[r + 1] = re[r] + rc[2 * r] * eb;
+    rh[r + 1] = rh[r] + rc[2 * r + 1];
+  }
+  CK(job->xrecv_e.ensure(re[R] + 16), "alloc receive entries");
+  CK(job->xrecv_h.ensure(rh[R] + 16), "alloc receive heap");
+  nr = nccl_alltoallv2(a, job->xsend_e.p, se.data(), job->xrecv_e.p, re.data(), job->xsend_h.p, sh.data(),
+                       job->xrecv_h.p, rh.data(), R, comm, s);
+  if (nr) return fail(job, MR_ERR_NCCL, "NCCL send/recv: " + nccl_error(a, nr));
+  job->stats.xchg_send_bytes += se[R] + sh[R];
+  job->stats.xchg_recv_bytes += re[R] + rh[R];
+  if (job->prof.on) job->prof.end(s, sp, &job->stats.xchg_ms);
+  return mr_ingest(job, job->xrecv_e.p, job->xrecv_h.p, rc.data());
 }
 
 }  // namespace
@@ -848,6 +913,11 @@ mr_status mr_group(mr_job* job) {
   if (!job) return MR_ERR_INVALID;
   if (job->state != kMapped && job->state != kCreated) return fail(job, MR_ERR_STATE, "mr_group out of order");
   CK(cudaSetDevice(job->cfg.device), "set device");
+  if (job->cfg.nranks > 1 && job->cfg.nccl_comm && !job->in_exchange && !job->ingested && !job->km_partial &&
+      job->cfg.workload != MR_STRINGMATCH) {
+    mr_status xs = exchange(job);   // -> ingested pairs (or KM partials) of the keys this rank owns
+    if (xs != MR_OK) return xs;
+  }
   if (job->km_partial) {           // ingested KM partials: grouping happened at the owner (atomics)
     job->state = kGrouped;
     return MR_OK;
@@ -1444,6 +1514,8 @@ mr_status mr_job_destroy(mr_job* job) {
   job->prof.release();
   job->xcounts.release(); job->xcursors.release(); job->xheapbase.release(); job->xcounts_h.release();
   job->src_e.release(); job->src_h.release(); job->km_list.release(); job->xwin.release();
+  job->xsend_e.release(); job->xsend_h.release(); job->xrecv_e.release(); job->xrecv_h.release();
+  job->xrecv_counts.release();
   job->cent.release(); release_pairs(job); job->tb.release();
   job->swp.release(); job->seg_startp.release(); job->psum.release(); job->pxcounts.release();
   job->midx.release(); job->xkeys.release();

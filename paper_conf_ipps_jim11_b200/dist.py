@@ -30,6 +30,11 @@ def alltoallv(send, send_bytes, recv_bytes, group=None):
     out = torch.empty(sum(recv_bytes), dtype=torch.uint8, device=send.device)
     if sum(send_bytes) == 0 and sum(recv_bytes) == 0:
         return out
+    if send.is_cuda and dist.get_backend(group) != "nccl":   # gloo: staged through host memory
+        tmp = torch.empty(sum(recv_bytes), dtype=torch.uint8)
+        dist.all_to_all_single(tmp, send.cpu(), output_split_sizes=recv_bytes, input_split_sizes=send_bytes,
+                               group=group)
+        return tmp.to(send.device)
     dist.all_to_all_single(out, send, output_split_sizes=recv_bytes, input_split_sizes=send_bytes, group=group)
     return out
 
