@@ -56,6 +56,11 @@ typedef enum { MR_WORDCOUNT = 1, MR_STRINGMATCH = 2, MR_KMEANS = 3, MR_INVINDEX 
 #define MR_FLAG_NO_MAP_COMBINE  0x100u /* WC: no in-SMEM combiner in the Map (every word is emitted as a pair) */
 #define MR_FLAG_SM_LINES        0x200u /* SM: the paper's per-line output (L125): the global offset of every
                                           record containing the pattern, once (grouped by key) */
+#define MR_FLAG_BATCH_COMBINE   0x400u /* WC: each mapped batch is grouped + reduced (combined) when the next
+                                          one is mapped — mr_map then synchronises — and its (key, count)
+                                          partials kept; mr_group merges the partials (exact sums).  For
+                                          jobs larger than one group (>= 2^32 pairs) or HBM: batched
+                                          processing "at another level" (L74).  Ignored by SM / KM / II. */
 
 typedef struct { uint8_t pattern[16]; } mr_sm_params;                      /* StringMatch */
 typedef struct { uint32_t k, dim; const float* centroids; } mr_km_params;  /* KMeans: host ptr, k x dim fp32, dim == 8, 1 <= k <= 1024 */

@@ -24,6 +24,7 @@ WORKLOADS = {"wc": WORDCOUNT, "sm": STRINGMATCH, "km": KMEANS, "ii": INVINDEX}
 FLAG_NO_SMEM_IN, FLAG_NO_SMEM_OUT, FLAG_FORCE_TINY_OUT = 0x01, 0x02, 0x04
 FLAG_WEAK_HASH_DEBUG, FLAG_VALIDATE, FLAG_NO_COMBINE = 0x08, 0x10, 0x20
 FLAG_PROFILE, FLAG_OWN_STREAM, FLAG_NO_MAP_COMBINE, FLAG_SM_LINES = 0x40, 0x80, 0x100, 0x200
+FLAG_BATCH_COMBINE = 0x400
 
 STATUS = {0: "MR_OK", 1: "MR_ERR_INVALID", 2: "MR_ERR_STATE", 3: "MR_ERR_OOM", 4: "MR_ERR_OVERFLOW",
           5: "MR_ERR_CUDA", 6: "MR_ERR_NCCL", 7: "MR_ERR_UNSUPPORTED"}

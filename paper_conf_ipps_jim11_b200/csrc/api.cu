@@ -347,6 +347,16 @@ struct mr_job {
   DBuf<uint8_t> xsend_e, xsend_h, xrecv_e, xrecv_h;
   DBuf<uint64_t> xrecv_counts;
   bool in_exchange = false;       // mr_group called by the exchange's own combiner step
+  bool exchanged = false;         // this run's pairs already went through an exchange (mr_ingest)
+  // WC batch combine (MR_FLAG_BATCH_COMBINE, SURVEY §8(e) strong scaling; "batched
+  // processing at another level"): every batch is grouped + reduced when the next one is mapped
+  // (or at mr_group) and its (key, count) partials appended to an arena of 16-B entries + key
+  // bytes; mr_group then ingests the arena and groups the partials (counts summed exactly)
+  DBuf<uint8_t> acc_e, acc_h;
+  uint64_t acc_ne = 0, acc_nh = 0;
+  uint32_t nfolds = 0;
+  bool in_fold = false;
+  mr_stats fold_stats{};          // per-group counters of the folded batches (added at the end)
   uint32_t xranks = 0;
   DBuf<uint32_t> km_list;
   uint32_t km_nlist = 0;
@@ -571,6 +581,11 @@ mr_status settle_map(mr_job* job) {
 extern "C" mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_bytes);
 extern "C" mr_status mr_partition_write(mr_job* job, void* entries, void* heap);
 extern "C" mr_status mr_ingest(mr_job* job, const void* entries, const void* heap, const uint64_t* recv_counts);
+namespace {
+mr_status ingest_impl(mr_job* job, const void* entries, const void* heap, const uint64_t* recv_counts, uint32_t R);
+mr_status fold(mr_job* job);
+mr_status fold_finish(mr_job* job);
+}
 
 namespace {
 
@@ -622,7 +637,88 @@ mr_status exchange(mr_job* job) {
   job->stats.xchg_send_bytes += se[R] + sh[R];
   job->stats.xchg_recv_bytes += re[R] + rh[R];
   if (job->prof.on) job->prof.end(s, sp, &job->stats.xchg_ms);
-  return mr_ingest(job, job->xrecv_e.p, job->xrecv_h.p, rc.data());
+  job->exchanged = true;
+  return ingest_impl(job, job->xrecv_e.p, job->xrecv_h.p, rc.data(), static_cast<uint32_t>(R));
+}
+
+// grow a device byte arena to >= need bytes, keeping its first `used` bytes
+cudaError_t grow_keep(DBuf<uint8_t>& b, uint64_t used, uint64_t need, cudaStream_t s) {
+  if (need <= b.n && b.p) return cudaSuccess;
+  DBuf<uint8_t> nb;
+  cudaError_t e = nb.ensure(std::max<uint64_t>(need, 2 * b.n));
+  if (e != cudaSuccess) return e;
+  if (used && (e = cudaMemcpyAsync(nb.p, b.p, used, cudaMemcpyDeviceToDevice, s)) != cudaSuccess) return e;
+  if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return e;
+  b.release();
+  b = nb;
+  nb.p = nullptr;
+  nb.n = 0;
+  return cudaSuccess;
+}
+
+// WC batch combine: group + reduce the batches mapped since the last fold (the local combiner,
+// exact integer sums) and append their (key, count) partials to the arena; the job is then ready
+// to map the next batch.  Synchronises.
+mr_status fold(mr_job* job) {
+  cudaStream_t s = job->stream;
+  job->in_fold = true;
+  mr_status st = mr_group(job);
+  if (st == MR_OK) st = mr_reduce(job);
+  job->in_fold = false;
+  if (st != MR_OK) return st;
+  mr_stats& f = job->fold_stats;
+  f.pairs += job->stats.pairs;
+  f.pairs_hashed += job->stats.pairs_hashed;
+  f.pairs_mid += job->stats.pairs_mid;
+  f.pairs_partial += job->stats.pairs_partial;
+  f.words_combined += job->stats.words_combined;
+  f.flushes += job->stats.flushes;
+  XSource xs;
+  xs.nranks = 1;
+  xs.mode = kXSegs;
+  xs.n = job->nseg;
+  xs.keys = job->keys_out.p;
+  xs.key_off = job->key_off.p;
+  xs.counts = job->counts.p;
+  CK(job->xcounts.ensure(2), "alloc counts");
+  CK(job->xcursors.ensure(2), "alloc cursors");
+  CK(job->xheapbase.ensure(1), "alloc heap base");
+  CK(job->xcounts_h.ensure(4), "alloc host counts");
+  CK(launch_x_count(xs, job->xcounts.p, job->nsm, s), "fold count");
+  CK(cudaMemcpyAsync(job->xcounts_h.p, job->xcounts.p, 16, cudaMemcpyDeviceToHost, s), "D2H fold counts");
+  CK(cudaStreamSynchronize(s), "sync fold counts");
+  const uint64_t ne = job->xcounts_h.p[0], nh = job->xcounts_h.p[1];
+  CK(grow_keep(job->acc_e, job->acc_ne * sizeof(XEntry), (job->acc_ne + ne) * sizeof(XEntry) + 64, s), "grow arena");
+  CK(grow_keep(job->acc_h, job->acc_nh, job->acc_nh + nh + 64, s), "grow arena");
+  unsigned long long* cur = job->xcounts_h.p + 2;   // entries / heap cursors at the arena's ends
+  cur[0] = job->acc_ne;
+  cur[1] = job->acc_nh;
+  CK(cudaMemcpyAsync(job->xcursors.p, cur, 16, cudaMemcpyHostToDevice, s), "H2D cursors");
+  CK(cudaMemsetAsync(job->xheapbase.p, 0, 8, s), "heap base");   // entry key offsets = arena offsets
+  xs.heap_base = job->xheapbase.p;
+  CK(launch_x_scatter(xs, job->xcursors.p, job->acc_e.p, job->acc_h.p, s), "fold scatter");
+  CK(cudaStreamSynchronize(s), "sync fold");
+  job->acc_ne += ne;
+  job->acc_nh += nh;
+  ++job->nfolds;
+  // a fresh Map state for the next batch (buffers kept; the folded batches may be released)
+  job->batches.clear();
+  CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), s), "reset state");
+  job->state = kCreated;
+  return MR_OK;
+}
+
+// mr_group of a folded job: fold the pending batches, then ingest every batch's partials (one
+// source) as the pairs to group (u64 counts, keys by reference into the arena)
+mr_status fold_finish(mr_job* job) {
+  if (!job->batches.empty()) {
+    mr_status st = fold(job);
+    if (st != MR_OK) return st;
+  }
+  const uint64_t rc[2] = {job->acc_ne, job->acc_nh};
+  mr_status st = ingest_impl(job, job->acc_e.p, job->acc_h.p, rc, 1);
+  job->nfolds = 0;   // (the arena stays referenced until mr_reduce; reset clears it)
+  return st;
 }
 
 }  // namespace
@@ -711,6 +807,10 @@ mr_status mr_job_reset(mr_job* job) {
   job->owned.clear();
   job->host_batches = 0;
   job->ingested = false;
+  job->exchanged = false;
+  job->nfolds = 0;
+  job->acc_ne = job->acc_nh = 0;
+  job->fold_stats = mr_stats{};
   job->km_partial = false;
   job->km_combined = false;
   job->key_bits = (job->cfg.workload == MR_WORDCOUNT || job->cfg.workload == MR_INVINDEX) ? 48u : 64u;
@@ -766,6 +866,11 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
     nbytes = job->tmp_h.p[0];
   }
   if (nbytes && !records) return fail(job, MR_ERR_INVALID, "records is NULL");
+  if ((job->cfg.flags & MR_FLAG_BATCH_COMBINE) && job->cfg.workload == MR_WORDCOUNT && !job->ingested &&
+      !job->batches.empty()) {
+    mr_status fs = fold(job);   // WC batch combine: the previous batches become (key, count) partials
+    if (fs != MR_OK) return fs;
+  }
   if (job->cap == 0) {
     // WC: ~1 word per 6 bytes, a few % of them longer than 7 bytes (hashed stream)
     const bool wc = job->cfg.workload == MR_WORDCOUNT;
@@ -913,7 +1018,11 @@ mr_status mr_group(mr_job* job) {
   if (!job) return MR_ERR_INVALID;
   if (job->state != kMapped && job->state != kCreated) return fail(job, MR_ERR_STATE, "mr_group out of order");
   CK(cudaSetDevice(job->cfg.device), "set device");
-  if (job->cfg.nranks > 1 && job->cfg.nccl_comm && !job->in_exchange && !job->ingested && !job->km_partial &&
+  if (job->nfolds && !job->in_fold) {   // WC batch combine: fold the last batch, ingest all partials
+    mr_status fs = fold_finish(job);
+    if (fs != MR_OK) return fs;
+  }
+  if (job->cfg.nranks > 1 && job->cfg.nccl_comm && !job->in_exchange && !job->in_fold && !job->exchanged &&
       job->cfg.workload != MR_STRINGMATCH) {
     mr_status xs = exchange(job);   // -> ingested pairs (or KM partials) of the keys this rank owns
     if (xs != MR_OK) return xs;
@@ -1102,6 +1211,15 @@ mr_status mr_group(mr_job* job) {
     job->key_bytes = job->tmp_h.p[0];
   }
   if (job->prof.on) { job->prof.end(job->stream, sp3, &job->stats.seg_ms); CK(cudaStreamSynchronize(job->stream), "sync"); job->prof.collect(); }
+  if (!job->in_fold && !job->in_exchange) {   // the folded batches' own group-by counters
+    const mr_stats& f = job->fold_stats;
+    job->stats.pairs += f.pairs;
+    job->stats.pairs_hashed += f.pairs_hashed;
+    job->stats.pairs_mid += f.pairs_mid;
+    job->stats.pairs_partial += f.pairs_partial;
+    job->stats.words_combined += f.words_combined;
+    job->stats.flushes += f.flushes;
+  }
   job->state = kGrouped;
   return MR_OK;
 }
@@ -1344,7 +1462,16 @@ mr_status mr_ingest(mr_job* job, const void* entries, const void* heap, const ui
   if (!job || !recv_counts) return MR_ERR_INVALID;
   if (job->state != kPartitioned) return fail(job, MR_ERR_STATE, "mr_ingest before mr_partition_write");
   CK(cudaSetDevice(job->cfg.device), "set device");
-  const uint32_t R = static_cast<uint32_t>(job->cfg.nranks);
+  job->exchanged = true;
+  return ingest_impl(job, entries, heap, recv_counts, static_cast<uint32_t>(job->cfg.nranks));
+}
+
+}  // extern "C"
+
+namespace {
+// received entries of R sources (recv_counts[2r], [2r+1]) -> the job's ingested pair stream (or,
+// for KM, the owner's partial sums)
+mr_status ingest_impl(mr_job* job, const void* entries, const void* heap, const uint64_t* recv_counts, uint32_t R) {
   std::vector<uint64_t> se(R + 1, 0), sh(R + 1, 0);
   for (uint32_t r = 0; r < R; ++r) {
     se[r + 1] = se[r] + recv_counts[2 * r];
@@ -1363,7 +1490,7 @@ mr_status mr_ingest(mr_job* job, const void* entries, const void* heap, const ui
     CK(launch_x_ingest_km(entries, n, job->sums.p, job->cnts.p, k, s), "ingest km");
     std::vector<uint32_t> own;
     for (uint32_t j = 0; j < k; ++j)
-      if (km_owner(j, R) == static_cast<uint32_t>(job->cfg.rank)) own.push_back(j);
+      if (km_owner(j, static_cast<uint32_t>(job->cfg.nranks)) == static_cast<uint32_t>(job->cfg.rank)) own.push_back(j);
     CK(job->km_list.ensure(own.size() + 1), "alloc owner list");
     if (!own.empty())
       CK(cudaMemcpyAsync(job->km_list.p, own.data(), own.size() * 4, cudaMemcpyHostToDevice, s), "H2D owners");
@@ -1396,6 +1523,9 @@ mr_status mr_ingest(mr_job* job, const void* entries, const void* heap, const ui
   job->state = kMapped;
   return MR_OK;
 }
+}  // namespace
+
+extern "C" {
 
 mr_status mr_set_xwindows(mr_job* job, uint32_t nranks, void* const* entries, void* const* heaps,
                           uint64_t* const* cursors, uint64_t entry_cap, uint64_t heap_cap) {
@@ -1515,7 +1645,7 @@ mr_status mr_job_destroy(mr_job* job) {
   job->xcounts.release(); job->xcursors.release(); job->xheapbase.release(); job->xcounts_h.release();
   job->src_e.release(); job->src_h.release(); job->km_list.release(); job->xwin.release();
   job->xsend_e.release(); job->xsend_h.release(); job->xrecv_e.release(); job->xrecv_h.release();
-  job->xrecv_counts.release();
+  job->xrecv_counts.release(); job->acc_e.release(); job->acc_h.release();
   job->cent.release(); release_pairs(job); job->tb.release();
   job->swp.release(); job->seg_startp.release(); job->psum.release(); job->pxcounts.release();
   job->midx.release(); job->xkeys.release();

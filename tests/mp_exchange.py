@@ -23,7 +23,7 @@ def shard(workload, r, R, units):
     return pygen.host_text(spec, b - a, page0=a)
 
 
-def worker(rank, world, port, mode, workload, flags, units, outdir):
+def worker(rank, world, port, mode, workload, flags, units, outdir, nbatch=1):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), NCCL_HOSTID=f"bmrtest{rank}",
                       NCCL_SOCKET_IFNAME="lo", NCCL_IB_DISABLE="1")
     if ROOT not in sys.path:
@@ -43,13 +43,22 @@ def worker(rank, world, port, mode, workload, flags, units, outdir):
             kw["centroids"] = pygen.km_centres(pygen.KMSpec())[1]
         if workload == "ii":
             kw["input_base"] = g["base"]
-        d = torch.from_numpy(g["data"]).cuda()
-        o = torch.from_numpy(g["offsets"].view(np.int64)).cuda() if g["offsets"] is not None else None
+        # nbatch > 1 (text): the shard is mapped as consecutive record batches
+        cuts = [g["n"] * i // nbatch for i in range(nbatch + 1)]
+        batches = []
+        for a, c in zip(cuts, cuts[1:]):
+            if g["offsets"] is None:
+                batches.append((torch.from_numpy(g["data"][a * 32:c * 32]).cuda(), None, c - a))
+            else:
+                off = g["offsets"]
+                batches.append((torch.from_numpy(g["data"][int(off[a]):int(off[c])]).cuda(),
+                                torch.from_numpy((off[a:c + 1] - off[a]).view(np.int64)).cuda(), c - a))
         outs, stats = [], []
         with bmr.Job(workload, **kw) as job:
             for _ in range(2):
                 job.reset()
-                job.map(d, o, g["n"])
+                for d, o, n in batches:
+                    job.map(d, o, n)
                 if mode == "shuffle":
                     job.shuffle()
                 job.group()

@@ -32,10 +32,10 @@ def _free_port():
     return p
 
 
-def run_ranks(mode, workload, R, flags, units, tmp_path, timeout=240):
+def run_ranks(mode, workload, R, flags, units, tmp_path, timeout=240, nbatch=1):
     ctx = torch.multiprocessing.get_context("spawn")
     port = _free_port()
-    ps = [ctx.Process(target=mp_exchange.worker, args=(r, R, port, mode, workload, flags, units, str(tmp_path)))
+    ps = [ctx.Process(target=mp_exchange.worker, args=(r, R, port, mode, workload, flags, units, str(tmp_path), nbatch))
           for r in range(R)]
     for p in ps:
         p.start()
@@ -82,6 +82,15 @@ def test_exchange_text(mode, workload, flags, units, tmp_path):
         assert got == exp, f"step {step}"
     if mode == "nccl":
         assert sum(r["stats"][1]["xchg_send_bytes"] for r in res) == sum(r["stats"][1]["xchg_recv_bytes"] for r in res) > 0
+
+
+def test_exchange_batch_combine(tmp_path):
+    # strong-scaling shape: every rank folds its shard batch by batch
+    # (MR_FLAG_BATCH_COMBINE), then the merged partials go through the NCCL exchange
+    res = run_ranks("nccl", "wc", 2, bmr.FLAG_BATCH_COMBINE, 6, tmp_path, nbatch=3)
+    exp = decode("wc", whole("wc", 6)[1])
+    for step in range(2):
+        assert union([r["outs"][step] for r in res], "wc") == exp
 
 
 @pytest.mark.parametrize("mode", ["nccl", "shuffle"])

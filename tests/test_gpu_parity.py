@@ -264,6 +264,33 @@ def test_wc_multibatch():
     assert got == decode("wc", ora("wc", [(data, off, g["n"])]))
 
 
+@pytest.mark.parametrize("flags", [0, bmr.FLAG_NO_MAP_COMBINE], ids=["map-combiner", "no-map-combiner"])
+def test_wc_batch_combine(flags):
+    # MR_FLAG_BATCH_COMBINE ("batched processing at another level"): every batch is
+    # grouped + reduced when the next one is mapped; mr_group merges the (key, count) partials
+    g = pygen.host_text(pygen.spec_wc(1_000_000, 5), 10)
+    data, off = g["data"], g["offsets"]
+    cuts = [0, g["n"] // 5, g["n"] // 2, g["n"] // 2 + 1, g["n"]]
+    b = [(data[int(off[a]):int(off[c])], off[a:c + 1] - off[a], c - a) for a, c in zip(cuts, cuts[1:])]
+    exp = decode("wc", ora("wc", [(data, off, g["n"])]))
+    for f in (bmr.FLAG_BATCH_COMBINE | flags, flags):
+        r, st = gpu("wc", b, flags=f)
+        assert decode("wc", r) == exp
+        assert st["n_keys"] == len(exp)
+    # the job is reusable after a folded run (reset keeps the buffers, clears the partials)
+    keep = []
+    with bmr.Job("wc", flags=bmr.FLAG_BATCH_COMBINE | flags) as job:
+        for _ in range(2):
+            job.reset()
+            for data_b, off_b, n in b:
+                d, o = dev(data_b, off_b)
+                keep.append((d, o))
+                job.map(d, o, n)
+            job.group()
+            job.reduce()
+            assert decode("wc", job.fetch()) == exp
+
+
 # ------------------------------------------------------------------ StringMatch
 def test_sm_generator_dense_plants():
     spec = pygen.spec_sm(plant_ppm=260_000)            # paper-shaped dense variant (3.83:1)
