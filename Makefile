@@ -17,7 +17,7 @@ gen/libbmrgen.so: gen/gen_host.c gen/bmr_gen.h
 	gcc -O2 -fPIC -shared -Wall -Wextra -o $@ gen/gen_host.c -lpthread -lm
 
 oracle/liboracle.so: oracle/oracle.cpp
-	g++ -O2 -std=c++17 -fPIC -shared -ffp-contract=off -Wall -Wextra -o $@ oracle/oracle.cpp
+	g++ -O3 -std=c++17 -fPIC -shared -ffp-contract=off -Wall -Wextra -o $@ oracle/oracle.cpp
 
 gen/libbmrgen_cuda.so: gen/gen_device.cu gen/bmr_gen.h
 	$(NVCC) -O3 $(ARCH) -Xcompiler -fPIC -shared -o $@ gen/gen_device.cu

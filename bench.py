@@ -3,7 +3,8 @@
 % HBM roofline, vs the CPU oracle).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C5|C4|C3|C2|C1] [--impl reference]
-                    [--mode SIO|SO|SI|G] [--no-map-combine] [--xchg a2a|fused] [--units U]
+                    [--scaling weak|strong] [--mode SIO|SO|SI|G] [--no-map-combine]
+                    [--xchg nccl|caller|fused] [--units U]
 
 One step = one pass of the whole hot path (tile scheduling, stage-in,
 user map, emit, flush, digit histogram, onesweep passes, segment boundaries, reduce + output
@@ -12,9 +13,17 @@ assembly) over one shard of synthetic input already resident in HBM.  Default wo
 "1/2/4/8 B200" is quoted on that exercises every row (C2 StringMatch is Map-only).
 Prints ONE JSON line on rank 0.  Timing: W warm-up steps, then K steps bracketed by barrier +
 cuda.synchronize, CUDA events on the job stream, max over ranks.  Inputs (8 GiB) exceed L2
-(126 MB), so no extra flush is needed.  At N > 1 the exchange is the partition + all-to-all over
-NCCL, or with --xchg fused (InvertedIndex) the Maps store straight into the owners' receive
-windows through CUDA IPC.
+(126 MB), so no extra flush is needed.
+
+Multi-GPU: ``--gpus N`` without a torchrun environment re-launches this script under
+``torch.distributed.run`` with N ranks (one per GPU, 127.0.0.1 rendezvous); under torchrun the
+world size comes from the environment (and must equal N).  The exchange is
+libbmr's own: mr_group over an NCCL communicator the library creates (``--xchg nccl``, default);
+``--xchg caller`` moves the partition buffers with torch.distributed (Job.shuffle); ``--xchg
+fused`` (InvertedIndex) lets the Maps store straight into the owners' receive windows through
+CUDA IPC.  ``--scaling strong`` fixes the total input (C5: 64 GiB, split 64/N
+GiB per GPU and processed in 8 GiB batches with the per-batch combine, MR_FLAG_BATCH_COMBINE);
+the default ``weak`` gives every GPU the 1-GPU configuration's shard.
 """
 from __future__ import annotations
 
@@ -39,6 +48,13 @@ WORKLOADS = {
     "C4": ("ii", "InvertedIndex 8 GiB HTML-like", 8192),
     "C5": ("wc", "WordCount 8 GiB/GPU Zipf text, V=1M (weak)", 8192),
 }
+
+
+# BASELINE.json's metric (both arms print it, so the driver can divide them)
+METRIC = "Map+Group+Reduce input GB/s and % HBM roofline at 1/2/4/8 B200 vs CPU oracle"
+# strong scaling: total units of the whole job (C5: 64 GiB, configs[4]) and units per mapped batch
+STRONG_TOTAL = {"C1": 1, "C2": 4096, "C3": 64 << 20, "C4": 8192, "C5": 65536}
+BATCH_UNITS = {"C5": 8192}
 
 
 def load_peaks():
@@ -108,19 +124,27 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------ inputs
-def make_input(cfg, rank, dev):
-    """Device-resident synthetic shard of rank `rank` (weak scaling: global units r*P..)."""
+def make_batches(cfg, u0, units, dev):
+    """Device-resident synthetic input of global units [u0, u0 + units), as mapped batches of at
+    most BATCH_UNITS[cfg] units (weak scaling: u0 = rank * P; strong: the rank's slice of the
+    fixed total)."""
     from gen import pygen
-    wl, _, units = WORKLOADS[cfg]
+    wl = WORKLOADS[cfg][0]
     spec = spec_for(cfg)
-    if wl == "km":
-        pts = pygen.device_km(spec, units, i0=rank * units, device=dev)
-        _, init = pygen.km_centres(spec)
-        return {"wl": wl, "data": pts.view(-1).view(__import__("torch").uint8), "offsets": None, "n": units,
-                "nbytes": units * 32, "centroids": init, "spec": spec, "page0": rank * units}
-    g = pygen.device_text(spec, units, page0=rank * units, device=dev)
-    return {"wl": wl, "data": g["data"], "offsets": g["offsets"], "n": g["n"], "nbytes": units * spec.page_bytes,
-            "spec": spec, "page0": rank * units, "base": g["base"]}
+    step = BATCH_UNITS.get(cfg, units) or 1
+    out = []
+    for a in range(u0, u0 + units, step):
+        m = min(step, u0 + units - a)
+        if wl == "km":
+            pts = pygen.device_km(spec, m, i0=a, device=dev)
+            _, init = pygen.km_centres(spec)
+            out.append({"wl": wl, "data": pts.view(-1).view(__import__("torch").uint8), "offsets": None, "n": m,
+                        "nbytes": m * 32, "centroids": init, "spec": spec, "page0": a, "base": 0})
+        else:
+            g = pygen.device_text(spec, m, page0=a, device=dev)
+            out.append({"wl": wl, "data": g["data"], "offsets": g["offsets"], "n": g["n"],
+                        "nbytes": m * spec.page_bytes, "spec": spec, "page0": a, "base": g["base"]})
+    return out
 
 
 def job_kwargs(inp, flags=0, device=0, rank=0, world=1):
@@ -135,10 +159,23 @@ def job_kwargs(inp, flags=0, device=0, rank=0, world=1):
 
 
 # ------------------------------------------------------------------ CPU oracle (baseline / reference arm)
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    import platform
+    return platform.processor() or "unknown"
+
+
 def oracle_sample(cfg, sample_units, page0=0):
-    """Time the oracle (as it stands) on the first `sample_units` pages/points of rank 0's shard."""
+    """Time the oracle (as it stands; SURVEY §8(d) D-5 build: -O3 -march=native -ffp-contract=off,
+    compiled on this host) on the first `sample_units` pages/points of rank 0's shard."""
     from gen import pygen
     from oracle import oracle
+    oracle.use_native()
     wl = WORKLOADS[cfg][0]
     spec = spec_for(cfg)
     if wl == "km":
@@ -155,6 +192,12 @@ def oracle_sample(cfg, sample_units, page0=0):
     oracle.run(wl, [(g["data"], g["offsets"], g["n"], 0, g["base"])], **kw)
     dt = time.perf_counter() - t0
     return g["data"].size, dt, f"first {sample_units} pages ({sample_units} MiB) of the shard"
+
+
+def cpu_info():
+    from oracle import oracle
+    return {"cores": 1, "cpu_model": cpu_model(), "oracle_build": oracle.build_flags(),
+            "host_cores_available": len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()}
 
 
 ORACLE_SAMPLE = {"C1": 1, "C2": 2048, "C3": 16 << 20, "C4": 2048, "C5": 96}   # ~10-30 s of CPU work
@@ -176,12 +219,13 @@ def run_reference(args, rank, world):
         times.append(dt)
     ms = 1000.0 * sum(times) / len(times)
     val = nb / (ms / 1000.0) / 1e9
-    line = {"impl": "reference", "metric": "Map+Group+Reduce input GB/s (CPU oracle)", "value": round(val, 6),
+    line = {"impl": "reference", "metric": METRIC, "value": round(val, 6),
             "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": round(ms, 3), "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "ms_per_step": round(ms, 3), "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None,
             "dtype": "u8" if WORKLOADS[cfg][0] != "km" else "f32", "data": "synthetic",
-            "config": {"workload": cfg, "description": WORKLOADS[cfg][1], "sample": desc},
-            "cpu_baseline": {"value": round(val, 6), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": desc},
+            "config": {"workload": cfg, "description": WORKLOADS[cfg][1], "sample": desc,
+                       "parallelism": f"dp{world}"},
+            "cpu_baseline": {"value": round(val, 6), "unit": "GB/s", "kind": "oracle", "sample": desc, **cpu_info()},
             "e2e": {"value": round(val, 6), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -222,6 +266,20 @@ def algorithmic(inp, st, steps):
             "passes_keys": px}
 
 
+def relaunch(args_n):
+    """--gpus N without a torchrun environment: run this script under torch.distributed.run with
+    N ranks on this node (127.0.0.1 rendezvous); rank 0 prints the JSON line."""
+    import socket
+    import subprocess
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args_n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -229,24 +287,36 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--workload", default="C5", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="bmr", choices=["bmr", "reference"])
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="weak: the 1-GPU shard per GPU; strong: fixed total (C5 64 GiB) split over the GPUs")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--units", type=int, default=0, help="override pages (text) / points (KM) per GPU")
     ap.add_argument("--mode", default="SIO", choices=["SIO", "SO", "SI", "G"],
                     help="Map memory-usage mode (PAPER.md L129-135 ablation, SURVEY §8(f) f-2)")
     ap.add_argument("--no-map-combine", action="store_true", help="literal north-star order (no Map combiner)")
-    ap.add_argument("--xchg", default="a2a", choices=["a2a", "fused"],
-                    help="InvertedIndex exchange: partition + all-to-all (a2a) or the fused Map flush into "
-                         "receive windows (f-3; one GPU: the rank's own window, timed with its ingest)")
+    ap.add_argument("--xchg", default="nccl", choices=["nccl", "caller", "fused"],
+                    help="exchange at N > 1: libbmr's mr_group over NCCL (nccl), torch.distributed moving the "
+                         "partition buffers (caller), or the fused Map flush into receive windows (fused, II)")
     args = ap.parse_args()
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
+    env_world = os.environ.get("WORLD_SIZE")
+    if env_world is None and args.gpus > 1:
+        sys.exit(relaunch(args.gpus))
+    world = int(env_world or "1")
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus and rank == 0:
+        sys.stderr.write(f"[bench] --gpus {args.gpus} but WORLD_SIZE={world}: using the launched world\n")
     if args.impl == "reference":
         run_reference(args, rank, world)
         return
 
+    share = os.environ.get("BMR_SHARE_GPU") == "1" and world > 1
+    if share:   # plumbing test on a 1-GPU box: every rank on cuda:0, each its own NCCL "host"
+        local = 0
+        os.environ.setdefault("NCCL_HOSTID", f"bmrbench{rank}")
+        os.environ.setdefault("NCCL_SOCKET_IFNAME", "lo")
     import torch
     import torch.distributed as dist
     import paper_conf_ipps_jim11_b200 as bmr
@@ -261,27 +331,38 @@ def main():
             dist.barrier()
         torch.cuda.synchronize()
 
+    cfg = args.workload
+    wl = WORKLOADS[cfg][0]
     if args.units:
-        w = WORKLOADS[args.workload]
-        WORKLOADS[args.workload] = (w[0], w[1] + f" [reduced: {args.units} units]", args.units)
-    inp = make_input(args.workload, rank, dev)
+        w = WORKLOADS[cfg]
+        WORKLOADS[cfg] = (w[0], w[1] + f" [reduced: {args.units} units]", args.units)
+    P = WORKLOADS[cfg][2]
+    if args.scaling == "strong":
+        T = args.units or STRONG_TOTAL[cfg]
+        u0, units = rank * T // world, (rank + 1) * T // world - rank * T // world
+    else:
+        u0, units = rank * P, P
+    batches = make_batches(cfg, u0, units, dev)
+    inp = batches[0]
+    nbytes_rank = sum(b["nbytes"] for b in batches)
+    n_rank = sum(b["n"] for b in batches)
     torch.cuda.synchronize()
     mode_flags = {"SIO": 0, "SO": bmr.FLAG_NO_SMEM_IN, "SI": bmr.FLAG_NO_SMEM_OUT,
                   "G": bmr.FLAG_NO_SMEM_IN | bmr.FLAG_NO_SMEM_OUT}[args.mode]
     if args.no_map_combine:
         mode_flags |= bmr.FLAG_NO_MAP_COMBINE
-    job = bmr.Job(inp["wl"], **job_kwargs(inp, bmr.FLAG_PROFILE | mode_flags, local, rank, world))
+    if len(batches) > 1 and wl == "wc":
+        mode_flags |= bmr.FLAG_BATCH_COMBINE   # per-batch group + combine (SURVEY §8(e) strong scaling)
+    exchange = world > 1 and wl != "sm"       # SM is Map-only: no exchange
+    comm = bmr.Comm.from_torch() if exchange and args.xchg == "nccl" else None
+    job = bmr.Job(wl, comm=comm, **job_kwargs(inp, bmr.FLAG_PROFILE | mode_flags, local, rank, world))
     stream = torch.cuda.current_stream()
-    exchange = world > 1 and inp["wl"] != "sm"      # SM is Map-only: no exchange
-    xbytes = [0]
     xwin = None
-    if args.xchg == "fused":
-        if inp["wl"] != "ii":
-            raise SystemExit("--xchg fused: InvertedIndex only")
+    if args.xchg == "fused" and world >= 1 and wl == "ii":
         # every rank's receive window holds what all ranks may send it (uniform hash partition;
         # 2x headroom for skew)
-        ecap = 2 * inp["nbytes"] // 48 + 4096
-        hcap = 2 * inp["nbytes"] // 4 + 65536
+        ecap = 2 * nbytes_rank // 48 + 4096
+        hcap = 2 * nbytes_rank // 4 + 65536
         if world > 1:   # windows shared through CUDA IPC: the Maps store into peers over NVLink
             from paper_conf_ipps_jim11_b200 import dist as D
             xwin = bmr.XWindow(ecap, hcap, device=torch.device(dev), ipc=True)
@@ -290,20 +371,24 @@ def main():
             xwin = bmr.XWindow(ecap, hcap, device=torch.device(dev))
             job.set_xwindows([xwin])
         exchange = False
+    elif args.xchg == "fused":
+        raise SystemExit("--xchg fused: InvertedIndex only")
 
     def step():
         job.reset()
         if xwin is not None:   # f-3: the Maps append the records to the owners' windows, then ingest
             xwin.reset()
             barrier()          # every window is empty before any rank maps
-            job.map(inp["data"], inp["offsets"], inp["n"])
+            for b in batches:
+                job.map(b["data"], b["offsets"], b["n"])
             barrier()          # every rank's records have landed
             job.ingest_xwindow(xwin)
         else:
-            job.map(inp["data"], inp["offsets"], inp["n"])
-        if exchange:  # one hash all-to-all over NCCL
-            xbytes[0] = job.shuffle()
-        job.group()
+            for b in batches:
+                job.map(b["data"], b["offsets"], b["n"])
+        if exchange and args.xchg == "caller":   # torch.distributed moves the partition buffers
+            job.shuffle()
+        job.group()            # (--xchg nccl: the exchange happens inside mr_group)
         job.reduce()
 
     for _ in range(max(3, args.warmup)):
@@ -312,9 +397,10 @@ def main():
     barrier()
     job.reset()
     # timed region: K steps, per-phase device times from the job's CUDA events
-    acc = {k: 0.0 for k in ("map_ms", "hist_ms", "sort_ms", "seg_ms", "sort_keys_ms")}
+    acc = {k: 0.0 for k in ("map_ms", "hist_ms", "sort_ms", "seg_ms", "sort_keys_ms", "xchg_ms")}
     tot = {"pairs": 0, "sort_passes": 0, "kernel_launches": 0, "flushes": 0, "n_keys": 0, "pairs_hashed": 0,
-           "sort_passes_keys": 0, "pairs_mid": 0, "sort_passes_mid": 0, "words_combined": 0, "pairs_partial": 0}
+           "sort_passes_keys": 0, "pairs_mid": 0, "sort_passes_mid": 0, "words_combined": 0, "pairs_partial": 0,
+           "collisions": 0, "xchg_send_bytes": 0, "replays": 0}
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         barrier()
@@ -326,11 +412,11 @@ def main():
             e = torch.cuda.Event(enable_timing=True)
             e.record(stream)
             evs.append(e)
-            s = job.stats()  # map/hist/sort/seg events are collected at mr_group's synchronisation
+            st = job.stats()  # map/hist/sort/seg events are collected at mr_group's synchronisation
             for k in tot:
-                tot[k] += s[k]
+                tot[k] += st[k]
             for k in acc:
-                acc[k] += s[k]
+                acc[k] += st[k]
         ev1.record(stream)
         ev1.synchronize()
         wall = time.perf_counter() - t0
@@ -349,7 +435,7 @@ def main():
         red += job.stats()["reduce_ms"]
     per = {k: v / args.steps for k, v in acc.items()}
     per["reduce_ms"] = red / args.steps
-    alg = algorithmic(inp, tot, args.steps)
+    alg = algorithmic(dict(inp, n=n_rank, nbytes=nbytes_rank), tot, args.steps)
     hbm, peak_kind = load_peaks()
     # roofline of the dominant kernel (the larger device-time share of the step): the Map kernel
     # or the onesweep LSD passes (all sort streams together, per launch)
@@ -367,29 +453,51 @@ def main():
         tkey = "k_onesweep"
     else:
         kname, launch_ms, launch_bytes, tkey = "k_map", per["map_ms"], alg["map"], "k_map"
+    nmaps = len(batches)
+    if tkey == "k_map" and nmaps > 1:   # one Map launch per batch
+        launch_ms, launch_bytes = launch_ms / nmaps, launch_bytes / nmaps
     ach = launch_bytes / (launch_ms / 1e3) / 1e9 if launch_ms else 0.0
     roof = {"kernel": kname, "bound": "hbm", "achieved": round(ach, 1), "peak": hbm, "peak_kind": peak_kind,
             "unit": "GB/s", "frac": round(ach / hbm, 4), "traffic": None, "bytes_per_launch": int(launch_bytes),
             "ms_per_launch": round(launch_ms, 4),
             "share_of_step": round((sort_ms_all if tkey == "k_onesweep" else per["map_ms"]) / ms, 3)}
+    if wl == "km" and tkey == "k_map":
+        # KMeans Map: FP32-pipe bound: per point k centroids x 8 dims x (sub + fma)
+        # lane-ops; peak = 148 SMs x 128 FP32 lanes x the max SM clock (FFMA / FFMA2 on the fma pipe)
+        k = len(inp["centroids"])
+        ops = 16.0 * k * n_rank / nmaps
+        clk_mhz = 1965.0
+        try:
+            clk_mhz = float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["sm_max_mhz"])
+        except Exception:
+            pass
+        peak_ops = 148 * 128 * clk_mhz * 1e6
+        roof_hbm = dict(roof)
+        roof = {"kernel": "k_map (KMeans distances)", "bound": "fp32",
+                "achieved": round(ops / (launch_ms / 1e3) / 1e12, 3), "peak": round(peak_ops / 1e12, 2),
+                "peak_kind": f"derived: 148 SMs x 128 FP32 lanes x {clk_mhz:.0f} MHz (FFMA/FFMA2, fma pipe)",
+                "unit": "Tlane-op/s", "frac": round(ops / (launch_ms / 1e3) / peak_ops, 4), "traffic": None,
+                "ops_per_launch": int(ops), "ms_per_launch": round(launch_ms, 4),
+                "share_of_step": roof["share_of_step"], "hbm": {k2: roof_hbm[k2] for k2 in ("achieved", "peak", "frac")}}
     traffic_p = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(traffic_p):
-        tr = json.load(open(traffic_p)).get(args.workload, {}).get(tkey)
+        tr = json.load(open(traffic_p)).get(cfg, {}).get(tkey)
         if tr:
             roof["traffic"] = tr["bytes_per_launch"]
             roof["traffic_source"] = tr["source"]
 
-    nbytes_all = inp["nbytes"] * world
+    nbytes_all = nbytes_rank * world if args.scaling == "weak" else (args.units or STRONG_TOTAL[cfg]) * (
+        32 if wl == "km" else inp["spec"].page_bytes)
     value = nbytes_all / (ms_max / 1e3) / 1e9
 
-    # ---- end to end: host buffers through mr_map_host, H2D + D2H inside the timed region
+    # ---- end to end: host buffers through mr_map_host(_lines), H2D + D2H inside the timed region
     e2e = None
-    if args.e2e_steps > 0:
+    if args.e2e_steps > 0 and len(batches) == 1 and xwin is None:
         h_data = torch.empty(inp["data"].numel(), dtype=torch.uint8, pin_memory=True)
         h_data.copy_(inp["data"])
         h_off = inp["offsets"]   # text workloads: only a flag here (offsets are derived on the device)
         torch.cuda.synchronize()
-        job_e = bmr.Job(inp["wl"], **job_kwargs(inp, mode_flags, local, rank, world))
+        job_e = bmr.Job(wl, comm=comm, **job_kwargs(inp, mode_flags, local, rank, world))
         d2h = 0
 
         def estep():
@@ -398,7 +506,7 @@ def main():
                 job_e.map_host(h_data.numpy(), None, inp["n"])
             else:               # text: records are the lines; offsets derived on the device
                 job_e.map_host_lines(h_data.numpy())
-            if exchange:
+            if exchange and args.xchg == "caller":
                 job_e.shuffle()
             job_e.group()
             job_e.reduce()
@@ -428,36 +536,44 @@ def main():
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        su = ORACLE_SAMPLE[args.workload]
-        nb, dt, desc = oracle_sample(args.workload, su)
-        cpu = {"value": round(nb / dt / 1e9, 6), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": desc,
-               "seconds": round(dt, 2)}
+        su = ORACLE_SAMPLE[cfg]
+        nb, dt, desc = oracle_sample(cfg, su)
+        cpu = {"value": round(nb / dt / 1e9, 6), "unit": "GB/s", "kind": "oracle", "sample": desc,
+               "seconds": round(dt, 2), **cpu_info()}
 
     if rank == 0:
-        wl = inp["wl"]
         line = {
-            "metric": "Map+Group+Reduce input GB/s", "value": round(value, 3), "unit": "GB/s",
+            "metric": METRIC, "value": round(value, 3), "unit": "GB/s",
             "n_gpus": world, "steps": args.steps, "warmup": max(3, args.warmup), "ms_per_step": round(ms_max, 3),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "us_per_step": round(ms_max * 1e3, 1),
+            "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None,
             "dtype": "f32" if wl == "km" else "u8", "data": "synthetic",
-            "config": {"workload": args.workload, "description": WORKLOADS[args.workload][1],
-                       "input_bytes_per_gpu": inp["nbytes"], "records_per_gpu": inp["n"],
-                       "l2": "inputs larger than L2 (no flush needed)", "parallelism": f"dp{world}",
-                       "map_mode": args.mode, "map_combiner": not args.no_map_combine},
-            "records_per_s": round(inp["n"] * world / (ms_max / 1e3), 1),
+            "config": {"workload": cfg, "description": WORKLOADS[cfg][1],
+                       "input_bytes_per_gpu": nbytes_rank, "records_per_gpu": n_rank, "batches_per_gpu": nmaps,
+                       "input_bytes_total": nbytes_all,
+                       "l2": "inputs larger than L2 (no flush needed)" if nbytes_rank > (256 << 20) else
+                             "input smaller than L2: L2-resident (C1 is reported in us)",
+                       "parallelism": f"dp{world}", "map_mode": args.mode, "map_combiner": not args.no_map_combine,
+                       **({"shared_gpu_plumbing_test": True} if share else {})},
+            "records_per_s": round(n_rank * world / (ms_max / 1e3), 1),
             "hbm_frac_end_to_end": round((alg["map"] + alg["hist"] + alg["sort"]) / (ms_max / 1e3) / 1e9 / hbm, 4),
+            "hbm_frac_nominal_8tbs": round((alg["map"] + alg["hist"] + alg["sort"]) / (ms_max / 1e3) / 1e9 / 8000.0, 4),
             "phases_ms": {k[:-3]: round(v, 3) for k, v in per.items()},
             "map": {"achieved_gbs": round(map_ach, 1), "frac": round(map_ach / hbm, 4),
-                    "bytes_per_step": int(alg["map"])},
+                    "frac_nominal_8tbs": round(map_ach / 8000.0, 4), "bytes_per_step": int(alg["map"])},
             "pairs_per_step": int(alg["pairs"]), "sort_passes": alg["passes"],
             "wc_streams": ({"exact": int(alg["pairs_exact"]), "mid": int(tot["pairs_mid"] / args.steps),
                             "hashed": int(tot["pairs_hashed"] / args.steps),
-                            "partials": int(tot["pairs_partial"] / args.steps)} if inp["wl"] == "wc" else None),
+                            "partials": int(tot["pairs_partial"] / args.steps)} if wl == "wc" else None),
             "map_combiner": {"words_or_points_absorbed": int(tot["words_combined"] / args.steps)},
             "distinct_keys": int(tot["n_keys"] / args.steps),
+            "hash_collisions_per_step": tot["collisions"] / args.steps,
+            "replays": tot["replays"],
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
-            "exchange": ({"kind": "hash all-to-all over NCCL (torch.distributed)", "send_bytes_per_rank": xbytes[0],
-                          "combiner": inp["wl"] in ("wc", "km")} if exchange else
+            "exchange": ({"kind": ("libbmr mr_group over NCCL (" + bmr.Comm.backend() + ")") if args.xchg == "nccl"
+                          else "torch.distributed all_to_all_single (NCCL) of libbmr's partition buffers",
+                          "ranks": world, "send_bytes_per_rank": int(tot["xchg_send_bytes"] / args.steps),
+                          "xchg_ms": round(per["xchg_ms"], 3), "combiner": wl in ("wc", "km")} if exchange else
                          ({"kind": "fused Map flush into the owners' receive windows (f-3, CUDA IPC / NVLink)",
                            "window_entries_heap": list(xwin.used())} if xwin is not None else None)),
             "gpu_launches": int(tot["kernel_launches"]),
@@ -467,6 +583,8 @@ def main():
         }
         print(json.dumps(line), flush=True)
     job.close()
+    if comm is not None:
+        comm.close()
     if world > 1:
         dist.destroy_process_group()
 

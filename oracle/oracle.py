@@ -22,12 +22,42 @@ class _Result(C.Structure):
 
 
 _LIB = None
+_PATH = os.path.join(_HERE, "liboracle.so")   # the portable build (Makefile: -O3 -ffp-contract=off)
+_FLAGS = "-O3 -ffp-contract=off (portable build)"
+
+
+def use_native() -> str:
+    """Switch to an oracle build for THIS host (-O3 -march=native
+    -ffp-contract=off), compiled once into the temp directory; the arithmetic is the same source
+    (no fast-math, no contraction).  Falls back to the portable build if g++ fails.  Returns the
+    flags of the build in use."""
+    global _PATH, _FLAGS, _LIB
+    if _LIB is not None or "march=native" in _FLAGS:
+        return _FLAGS
+    import hashlib
+    import subprocess
+    import tempfile
+    src = os.path.join(_HERE, "oracle.cpp")
+    tag = hashlib.sha1(open(src, "rb").read() + os.uname().nodename.encode()).hexdigest()[:12]
+    out = os.path.join(tempfile.gettempdir(), f"bmr_oracle_native_{tag}.so")
+    flags = ["-O3", "-march=native", "-std=c++17", "-fPIC", "-shared", "-ffp-contract=off"]
+    if not os.path.exists(out):
+        r = subprocess.run(["g++", *flags, "-o", out + ".tmp", src], capture_output=True, text=True)
+        if r.returncode != 0:
+            return _FLAGS
+        os.replace(out + ".tmp", out)
+    _PATH, _FLAGS = out, " ".join(f for f in flags if f not in ("-fPIC", "-shared", "-std=c++17"))
+    return _FLAGS
+
+
+def build_flags() -> str:
+    return _FLAGS
 
 
 def lib():
     global _LIB
     if _LIB is None:
-        path = os.path.join(_HERE, "liboracle.so")
+        path = _PATH
         if not os.path.exists(path):
             raise RuntimeError(f"{path} missing: run __graft_entry__.build()")
         L = C.CDLL(path)
