@@ -14,7 +14,7 @@
  * Threading: a job is used by one host thread at a time; distinct jobs are independent.
  * Errors: every call returns an mr_status; nothing aborts, exits or throws across the ABI.
  * Asynchronous device faults surface as MR_ERR_CUDA at the next synchronising call
- * (mr_map for text batches, mr_group, mr_fetch); mr_last_error() gives the detail.
+ * (mr_group, mr_fetch); mr_last_error() gives the detail.
  */
 #ifndef BMR_H
 #define BMR_H
@@ -142,9 +142,12 @@ mr_status mr_job_create(const mr_config* cfg, mr_job** out);
  *   offsets: device, n+1 u64, offsets[0] == 0, non-decreasing, offsets[n] = batch length;
  *            NULL iff record_stride > 0 (then record i = records[i*stride, (i+1)*stride)).
  *   n:       number of records (0 allowed).
- * Text batches read offsets[n] back to the host (8 bytes, synchronising the stream) to size
- * the launch; fixed-stride batches are fully asynchronous.  Global byte offsets emitted by
- * SM/II are input_base + (sum of earlier batch lengths) + in-batch offset. */
+ * Asynchronous (§8(b): enqueue and return): a text batch's length offsets[n], its tile count
+ * and global byte base are derived on the device (never read back here), so no call but the
+ * synchronising ones (mr_group, mr_fetch) waits for the device.  Global byte offsets emitted by
+ * SM/II are input_base + (sum of earlier batch lengths) + in-batch offset.  Errors found on the
+ * device (records NULL for a non-empty batch, a key > 65535 bytes) surface at mr_group.
+ * Exception: MR_FLAG_BATCH_COMBINE folds the previous batches first (synchronising). */
 mr_status mr_map(mr_job* job, const uint8_t* records, const uint64_t* offsets, uint64_t n);
 
 /* Same as mr_map for HOST buffers: the library copies records/offsets into job-owned device

@@ -97,7 +97,8 @@ struct Prof {
 struct Batch {
   const uint8_t* rec;
   const uint64_t* off;
-  uint64_t n, nbytes, gbase;
+  uint64_t n, nbytes, gbase;   // text: nbytes / gbase live in the batch's device descriptor
+  uint32_t di;                 // descriptor index (text)
 };
 
 // Sort workspace shared by mr_group and mr_sort_u64.
@@ -286,7 +287,13 @@ struct mr_job {
   DBuf<uint8_t> v;
   uint64_t cap = 0;
   std::vector<Batch> batches;
-  uint64_t next_base = 0;
+  uint64_t next_base = 0;        // fixed-stride batches: running global byte base
+  // text batches: device descriptors (nbytes, ntiles, gbase, tile-cap overflow) written by
+  // k_tile_bounds, 4 u64 per batch since the last reset; tile-bounds capacity in tiles
+  DBuf<uint64_t> bdesc;
+  HBuf<uint64_t> bdesc_h;
+  uint32_t ndesc = 0;
+  uint64_t tb_cap = 0;
   std::vector<void*> owned;       // reserved
   std::vector<DBuf<uint8_t>> host_rec;   // device copies made by mr_map_host (reused after reset)
   std::vector<DBuf<uint64_t>> host_off;
@@ -450,13 +457,17 @@ cudaError_t launch_batch(mr_job* job, const Batch& b) {
   a.key_bits = job->key_bits;
   a.xwin = job->xranks ? job->xwin.p : nullptr;
   a.xranks = job->xranks;
-  const uint64_t nt = map_tiles(a);
-  if (a.workload != kKM) {
-    cudaError_t e = job->tb.ensure(2 * nt + 2);
+  if (a.workload != kKM) {   // text: dimensions on the device
+    cudaError_t e = job->tb.ensure(2 * job->tb_cap + 2);
     if (e) return e;
+    a.desc = job->bdesc.p + 4ULL * b.di;
+    a.prev_desc = b.di ? job->bdesc.p + 4ULL * (b.di - 1) : nullptr;
+    a.input_base = job->cfg.input_base;
+    a.tb_cap = job->tb_cap;
+  } else {
+    job->stats.map_tiles += map_tiles(a);
   }
   a.tile_bounds = job->tb.p;
-  job->stats.map_tiles += nt;
   return launch_map(a, job->nsm, job->stream);
 }
 
@@ -543,19 +554,40 @@ mr_status do_segments32(mr_job* job, const uint32_t* skeys, uint64_t m, DBuf<uin
 mr_status settle_map(mr_job* job) {
   CK(read_state(job), "map (async)");
   DevState* hs = job->st_h.p;
+  if (hs->err & kErrNullRecords) return fail(job, MR_ERR_INVALID, "records is NULL for a non-empty batch");
   if (hs->err & kErrKeyTooLong) return fail(job, MR_ERR_OVERFLOW, "an emitted key exceeds 65535 bytes");
   if (job->ingested) return MR_OK;   // ingested pairs: exact count, written into buffers sized for it
+  // text batches: the dimensions the device derived (stats; tile-bounds capacity)
+  uint64_t max_tiles = 0;
+  if (job->cfg.record_stride == 0 && job->ndesc) {
+    CK(job->bdesc_h.ensure(4ULL * job->ndesc), "alloc host descriptors");
+    CK(cudaMemcpyAsync(job->bdesc_h.p, job->bdesc.p, 32ULL * job->ndesc, cudaMemcpyDeviceToHost, job->stream),
+       "D2H descriptors");
+    CK(cudaStreamSynchronize(job->stream), "sync descriptors");
+    uint64_t bytes = 0, tiles = 0;
+    for (uint32_t i = 0; i < job->ndesc; ++i) {
+      bytes += job->bdesc_h.p[4 * i];
+      tiles += job->bdesc_h.p[4 * i + 1];
+      max_tiles = std::max(max_tiles, job->bdesc_h.p[4 * i + 1]);
+    }
+    job->stats.input_bytes = bytes;
+    job->stats.map_tiles = tiles;
+  }
+  const bool tile_over = (hs->err & kErrTileCap) != 0;
   const uint64_t m = hs->pair_cursor, mb = job->split() ? hs->pair_cursor_b : 0;
   const uint64_t mc = job->split() ? hs->pair_cursor_c : 0;
   const uint64_t mp = job->wc_comb() ? hs->pair_cursor_p : 0;
-  if (m > job->cap || mb > job->cap_b || mc > job->cap_c || mp > job->cap_p) {
+  if (tile_over || m > job->cap || mb > job->cap_b || mc > job->cap_c || mp > job->cap_p) {
+    if (tile_over) job->tb_cap = max_tiles + 1024;   // (tb itself is grown by launch_batch)
     const uint64_t ncap_p = job->wc_comb() ? std::max(job->cap_p, mp + mp / 8 + 4096) : 0;
     const uint64_t ncap = std::max(job->cap, m + m / 8 + 4096);
     const uint64_t ncap_b = job->split() ? std::max(job->cap_b, mb + mb / 8 + 4096) : 0;
     const uint64_t ncap_c = job->split() ? std::max(job->cap_c, mc + mc / 8 + 4096) : 0;
-    release_pairs(job);
-    CK(ensure_pairs(job, ncap, ncap_b, ncap_c), "grow intermediate");
-    if (ncap_p) {
+    if (ncap > job->cap || ncap_b > job->cap_b || ncap_c > job->cap_c) {
+      release_pairs(job);
+      CK(ensure_pairs(job, ncap, ncap_b, ncap_c), "grow intermediate");
+    }
+    if (ncap_p > job->cap_p) {
       CK(job->hp.ensure(ncap_p), "grow partials");
       job->cap_p = ncap_p;
     }
@@ -568,7 +600,7 @@ mr_status settle_map(mr_job* job) {
     for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
     job->stats.replays += job->batches.size();
     CK(read_state(job), "replay (async)");
-    if (hs->pair_cursor > job->cap ||
+    if ((hs->err & kErrTileCap) || hs->pair_cursor > job->cap ||
         (job->split() && (hs->pair_cursor_b > job->cap_b || hs->pair_cursor_c > job->cap_c)) ||
         (job->wc_comb() && hs->pair_cursor_p > job->cap_p))
       return fail(job, MR_ERR_OOM, "replay still overflows");
@@ -825,6 +857,7 @@ mr_status mr_job_reset(mr_job* job) {
   job->prof.collect();
   job->batches.clear();
   job->next_base = 0;
+  job->ndesc = 0;
   job->m = job->nseg = job->key_bytes = 0;
   job->skeys = nullptr;
   job->perm = nullptr;
@@ -847,25 +880,28 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
   if (fixed && (reinterpret_cast<uintptr_t>(records) & 15u))
     return fail(job, MR_ERR_INVALID, "fixed-stride records must be 16-byte aligned");
   if ((reinterpret_cast<uintptr_t>(records) >> 48) != 0) return fail(job, MR_ERR_INVALID, "records address >= 2^48");
-  uint64_t nbytes = 0;
+  // Text batches are enqueued without a host round trip: the batch length offsets[n], its tile
+  // count and global base are derived on the device (map.cu k_tile_bounds) and read back at the
+  // next synchronising call (settle_map).  known_nbytes (mr_map_host_lines) only sizes buffers.
+  uint64_t nbytes = ~0ULL;
   if (fixed) {
     nbytes = n * job->cfg.record_stride;
-  } else if (known_nbytes != ~0ULL && !(job->cfg.flags & MR_FLAG_VALIDATE)) {
+    if (nbytes && !records) return fail(job, MR_ERR_INVALID, "records is NULL");
+  } else if (job->cfg.flags & MR_FLAG_VALIDATE) {
+    std::vector<uint64_t> o(n + 1);
+    CK(cudaMemcpyAsync(o.data(), offsets, (n + 1) * 8, cudaMemcpyDeviceToHost, job->stream), "read offsets");
+    CK(cudaStreamSynchronize(job->stream), "sync");
+    if (o[0] != 0) return fail(job, MR_ERR_INVALID, "offsets[0] != 0");
+    for (uint64_t i = 0; i < n; ++i)
+      if (o[i + 1] < o[i]) return fail(job, MR_ERR_INVALID, "offsets not non-decreasing");
+    nbytes = o[n];
+    if (nbytes && !records) return fail(job, MR_ERR_INVALID, "records is NULL");
+  } else if (known_nbytes != ~0ULL) {
     nbytes = known_nbytes;
-  } else {
-    CK(cudaMemcpyAsync(job->tmp_h.p, offsets + n, sizeof(uint64_t), cudaMemcpyDeviceToHost, job->stream), "read offsets[n]");
-    if (job->cfg.flags & MR_FLAG_VALIDATE) {
-      std::vector<uint64_t> o(n + 1);
-      CK(cudaMemcpyAsync(o.data(), offsets, (n + 1) * 8, cudaMemcpyDeviceToHost, job->stream), "read offsets");
-      CK(cudaStreamSynchronize(job->stream), "sync");
-      if (o[0] != 0) return fail(job, MR_ERR_INVALID, "offsets[0] != 0");
-      for (uint64_t i = 0; i < n; ++i)
-        if (o[i + 1] < o[i]) return fail(job, MR_ERR_INVALID, "offsets not non-decreasing");
-    }
-    CK(cudaStreamSynchronize(job->stream), "sync offsets[n]");
-    nbytes = job->tmp_h.p[0];
   }
-  if (nbytes && !records) return fail(job, MR_ERR_INVALID, "records is NULL");
+  // sizing estimate for the first batch's buffers (text of unknown length: <= 32 B per record
+  // assumed; overflow is caught by the demand counters and replayed at mr_group)
+  const uint64_t est = nbytes != ~0ULL ? nbytes : 32 * n;
   if ((job->cfg.flags & MR_FLAG_BATCH_COMBINE) && job->cfg.workload == MR_WORDCOUNT && !job->ingested &&
       !job->batches.empty()) {
     mr_status fs = fold(job);   // WC batch combine: the previous batches become (key, count) partials
@@ -875,9 +911,9 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
     // WC: ~1 word per 6 bytes, a few % of them longer than 7 bytes (hashed stream)
     const bool wc = job->cfg.workload == MR_WORDCOUNT;
     const uint64_t hint = job->cfg.max_pairs_hint;
-    const uint64_t cap_b = !wc ? 0 : hint ? hint : nbytes / 48 + 4096;
-    const uint64_t cap_c = !wc ? 0 : hint ? hint : nbytes / 32 + 4096;
-    CK(ensure_pairs(job, initial_cap(job, nbytes, n), cap_b, cap_c), "alloc intermediate");
+    const uint64_t cap_b = !wc ? 0 : hint ? hint : est / 48 + 4096;
+    const uint64_t cap_c = !wc ? 0 : hint ? hint : est / 32 + 4096;
+    CK(ensure_pairs(job, initial_cap(job, est, n), cap_b, cap_c), "alloc intermediate");
     if (job->wc_comb()) {   // combiner partials: <= 2^kCombBits per CTA per batch (grown + replayed if exceeded)
       job->cap_p = job->cfg.max_pairs_hint ? job->cfg.max_pairs_hint : 2ULL * 4096 * job->nsm + 4096;
       CK(job->hp.ensure(job->cap_p), "alloc partials");
@@ -890,10 +926,25 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
     CK(cudaMemsetAsync(job->sums.p, 0, 64ULL * job->k, job->stream), "zero sums");
     CK(cudaMemsetAsync(job->cnts.p, 0, 8ULL * job->k, job->stream), "zero counts");
   }
-  Batch b{records, offsets, n, nbytes, job->cfg.input_base + job->next_base};
-  job->next_base += nbytes;
+  Batch b{records, offsets, n, fixed ? nbytes : 0, fixed ? job->cfg.input_base + job->next_base : 0, 0};
+  if (fixed) {
+    job->next_base += nbytes;
+    job->stats.input_bytes += nbytes;
+  } else {
+    if (job->tb_cap == 0) job->tb_cap = (std::max<uint64_t>(est, 128 * n) + kMapTileBytes - 1) / kMapTileBytes + 1024;
+    if (job->ndesc + 1 > job->bdesc.n / 4) {   // descriptor table (grown keeping earlier batches')
+      DBuf<uint64_t> nb;
+      CK(nb.ensure(4ULL * std::max<uint32_t>(256, 2 * job->ndesc)), "alloc batch descriptors");
+      if (job->ndesc) {
+        CK(cudaMemcpyAsync(nb.p, job->bdesc.p, 32ULL * job->ndesc, cudaMemcpyDeviceToDevice, job->stream), "copy descriptors");
+        CK(cudaStreamSynchronize(job->stream), "sync descriptors");
+      }
+      job->bdesc.release();
+      job->bdesc = nb;
+    }
+    b.di = job->ndesc++;
+  }
   job->batches.push_back(b);
-  job->stats.input_bytes += nbytes;
   Prof::Span sp{};
   if (job->prof.on) job->prof.begin(job->stream, sp);
   CK(launch_batch(job, b), "map kernel launch");
@@ -925,7 +976,7 @@ mr_status mr_map_host(mr_job* job, const uint8_t* records, const uint64_t* offse
     CK(cudaMemcpyAsync(job->host_off[i].p, offsets, (n + 1) * 8, cudaMemcpyHostToDevice, job->stream), "H2D offsets");
     doff = job->host_off[i].p;
   }
-  return map_common(job, job->host_rec[i].p, doff, n);
+  return map_common(job, job->host_rec[i].p, doff, n, fixed ? ~0ULL : nbytes);
 }
 
 // mr_map_host_lines batch size (BMR_LINE_CHUNK bytes, default 256 MiB): copies of batch b + 1

@@ -35,7 +35,7 @@ struct DevState {
   unsigned long long n_extra;        // WC: partial-only keys found by the merge (mr_group)
   unsigned long long words_comb;     // WC: words absorbed by the combiners (sum of partial counts)
 };
-constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u;
+constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u, kErrTileCap = 4u, kErrNullRecords = 8u;
 
 // Intermediate pairs, SoA in HBM (SURVEY §8(a) layout): sort key, key reference, value.
 // WordCount Map output is three streams: exact keys (hx, u32: the key is the record, value 1),
@@ -87,11 +87,17 @@ struct MapArgs {
   int grid = 0;                       // persistent CTAs (0 = one per SM)
   const XWindow* xwin = nullptr;      // f-3: InvertedIndex records go straight to these R windows
   uint32_t xranks = 0;
+  // text batches: dimensions derived on the device (map.cu k_tile_bounds)
+  uint64_t* desc = nullptr;            // this batch's descriptor: nbytes, ntiles, gbase, tile-cap overflow
+  const uint64_t* prev_desc = nullptr; // the previous batch's (nullptr: the first batch, base = input_base)
+  uint64_t input_base = 0;
+  uint64_t tb_cap = 0;                 // tiles tile_bounds can hold
 };
 
 int vbytes_of(int workload);                 // value bytes per pair (WC Map output: none, value 1)
 bool has_kref(int workload);
-uint64_t map_tiles(const MapArgs& a);        // number of tiles of a batch
+uint64_t map_tiles(const MapArgs& a);        // number of tiles of a batch (fixed stride, or nbytes known)
+constexpr uint64_t kMapTileBytes = 16384;    // owned bytes per text tile (map.cu kT)
 uint32_t map_prefetch(int w);
 uint32_t map_wait_hint();
 uint32_t map_dyn_windows(int workload);

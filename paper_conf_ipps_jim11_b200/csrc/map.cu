@@ -24,6 +24,7 @@
 //     (cp.async.bulk.global.shared::cta).  Flushes are rounded to 4 pairs (16-B alignment) with
 //     sentinel filler pairs.  The global cursor counts demand even past capacity (D7), so the
 //     host can grow the buffers and replay the batch.
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
 
@@ -85,7 +86,7 @@ template <int W>
 constexpr uint32_t nflush() { return W == kWC ? BMR_WC_NFLUSH : 1u; }
 template <int W>
 constexpr int threads_of() { return (nmap<W>() + kNProd + static_cast<int>(nflush<W>())) * 32; }
-constexpr int kT = 16384;        // owned bytes per tile (text) / bytes per tile (KM)
+constexpr int kT = static_cast<int>(kMapTileBytes);   // owned bytes per tile (text) / bytes per tile (KM)
 constexpr int kLead = 16;        // bytes staged before the tile (previous-byte context)
 constexpr int kHalo = 256;       // bytes staged after the tile (words / matches / URLs crossing it)
 constexpr int kWin = 512;        // bytes per warp window = 32 lanes x 16 B
@@ -217,6 +218,15 @@ struct PairFmt {
   static_assert(kCap >= kMaxReserve, "output half smaller than one warp result");
 };
 
+// Dimensions of the mapped batch: (byte length, tiles, global byte base).  Text batches are
+// enqueued without a host round trip (mr_map never reads offsets[n] back): k_tile_bounds derives
+// them from offsets[n] on the device into the batch's descriptor, and every CTA of k_map copies
+// them into shared memory at start-up.  Fixed-stride batches (KM) carry host values.
+__shared__ unsigned long long s_bd[4];
+__device__ __forceinline__ long long bd_nbytes() { return static_cast<long long>(s_bd[0]); }
+__device__ __forceinline__ uint64_t bd_ntiles() { return s_bd[1]; }
+__device__ __forceinline__ uint64_t bd_gbase() { return s_bd[2]; }
+
 struct Params {
   const uint8_t* rec;
   const uint64_t* off;
@@ -262,6 +272,7 @@ struct Params {
   uint32_t wc_fast;        // WordCount: wc_map_loop / wc_window (BMR_WC_FAST, default on)
   const XWindow* xwin;     // f-3: InvertedIndex records appended straight to these windows
   uint32_t xranks;         // number of windows (0: local output)
+  const uint64_t* desc;    // text: the batch descriptor (nbytes, ntiles, gbase, tile-bounds overflow)
 };
 
 // Idle wait of a role warp on an mbarrier phase (map warps on a staged tile, producers on a free
@@ -379,7 +390,7 @@ struct TileView {
 // Word length for a word at position p whose end lies beyond the 32-byte window [p0, p0+32).
 __device__ uint32_t slow_word_len(const Params& P, const TileView& tv, long long p, long long from) {
   long long q = from;
-  const long long N = static_cast<long long>(P.nbytes);
+  const long long N = bd_nbytes();
   const long long lim = min(tv.stg_hi, N);
   // inside the stage: 4 bytes per step (SWAR word classes + bitmap record starts)
   while (q < lim && ((q - tv.sbase) & 3)) {
@@ -408,7 +419,7 @@ __device__ uint32_t slow_word_len(const Params& P, const TileView& tv, long long
 // Position of the closing '"' of a URL starting at q0, or -1 if the record (or input) ends
 // first.  Scans the stage 16 bytes at a time, then global memory (slow path).
 __device__ long long find_quote(const Params& P, const TileView& tv, long long q0, long long p_marker) {
-  const long long N = static_cast<long long>(P.nbytes);
+  const long long N = bd_nbytes();
   const long long lim = min(tv.stg_hi, N);
   long long q = q0;
   while (q < lim && ((q - tv.sbase) & 3)) {               // align to a 4-byte SMEM word
@@ -753,10 +764,10 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
   const uint32_t lane = threadIdx.x & 31;
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
   uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
-  const long long N = static_cast<long long>(P.nbytes);
+  const long long N = bd_nbytes();
   const uint64_t G = gridDim.x;
   // iterations of this CTA: tiles blockIdx.x + it * G; this producer takes it == pw (mod kNProd)
-  const uint32_t T = blockIdx.x < P.ntiles ? static_cast<uint32_t>((P.ntiles - blockIdx.x + G - 1) / G) : 0u;
+  const uint32_t T = blockIdx.x < bd_ntiles() ? static_cast<uint32_t>((bd_ntiles() - blockIdx.x + G - 1) / G) : 0u;
   for (uint32_t i0 = pw; i0 < T; i0 += 32u * kNProd) {
     // lanes prefetch the bounds of this producer's next 32 tiles (one latency per 32 tiles)
     const uint32_t my_it = i0 + lane * kNProd;
@@ -1112,7 +1123,7 @@ __device__ __forceinline__ uint32_t exact_key30_bf(uint32_t lo, uint32_t b4, uin
 __device__ __forceinline__ void wc_window(const Params& P, OutCtl* oc, uint8_t* outh, const TileView& tv,
                                           long long p0w, uint32_t* xq, uint32_t* hq, uint32_t* ctab) {
   const uint32_t lane = threadIdx.x & 31;
-  const long long N = static_cast<long long>(P.nbytes);
+  const long long N = bd_nbytes();
   const long long p0 = p0w + 16 * lane;
   const uint32_t i0 = static_cast<uint32_t>(p0 - tv.sbase);   // 16-B aligned stage offset
   const uint4 c0 = *reinterpret_cast<const uint4*>(tv.sb + i0);
@@ -1290,7 +1301,7 @@ __device__ void ii_drain_xwin(const Params& P, uint32_t qn, const uint64_t* qpos
       if (ie < w.ecap && ih + hb <= w.hcap) {
         XEntry* o = reinterpret_cast<XEntry*>(w.entries) + ie;
         o->koff_len = (static_cast<uint64_t>(ih) << 16) | len;
-        o->v = P.gbase + static_cast<uint64_t>(q0);
+        o->v = bd_gbase() + static_cast<uint64_t>(q0);
         for (uint32_t k = 0; k < len; k += 8)   // heap records are 8-B aligned
           *reinterpret_cast<uint64_t*>(w.heap + ih + k) = load8(kp + k, min(8u, len - k));
       }
@@ -1323,7 +1334,7 @@ __device__ void ii_drain(const Params& P, OutCtl* oc, uint8_t* outh, uint32_t& q
     const uint32_t idx = slot.base + e;
     sh[idx] = key_at(P, gv, q0, len);
     sk[idx] = (reinterpret_cast<uint64_t>(P.rec + q0) << 16) | len;
-    sv[idx] = P.gbase + static_cast<uint64_t>(q0);
+    sv[idx] = bd_gbase() + static_cast<uint64_t>(q0);
   }
   commit(oc, slot, qn);
   qn = 0;
@@ -1333,7 +1344,7 @@ template <int W>
 __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, const TileView& tv,
                                 long long p0, long long i0, bool live, uint32_t& qn) {
   using F = PairFmt<W>;
-  const long long N = static_cast<long long>(P.nbytes);
+  const long long N = bd_nbytes();
   uint32_t x[8];
   uint32_t vm = 0, R = 0;
   if (live) {
@@ -1578,7 +1589,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
           }
           key = P.off[lo - 1];   // lo >= 1: offsets[0] = 0 <= p
         }
-        if (idx < cap) sh[idx] = P.gbase + key;
+        if (idx < cap) sh[idx] = bd_gbase() + key;
       } else if constexpr (W == kII) {
         uint32_t len = nth == 0 ? aux[0] : aux[1];
         ++nth;
@@ -1588,7 +1599,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
         if (idx < cap) {
           sh[idx] = key;
           sk[idx] = (reinterpret_cast<uint64_t>(P.rec + q0) << 16) | len;
-          reinterpret_cast<uint64_t*>(sv)[idx] = P.gbase + static_cast<uint64_t>(q0);
+          reinterpret_cast<uint64_t*>(sv)[idx] = bd_gbase() + static_cast<uint64_t>(q0);
         }
       }
     }
@@ -1615,11 +1626,11 @@ __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl
   uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
   uint8_t* outh = smem + Layout<W>::out;
   const uint32_t b0 = (P.pat[0] & 0xFFu) * 0x01010101u;
-  const long long N = static_cast<long long>(P.nbytes);
+  const long long N = bd_nbytes();
   // this CTA's iterations (as producer_loop): a warp's super-windows are nmap apart and may skip
   // whole tiles (kNSup < nmap), so it must stop at T itself rather than wait for the end marker
   const uint64_t G = gridDim.x;
-  const uint32_t T = blockIdx.x < P.ntiles ? static_cast<uint32_t>((P.ntiles - blockIdx.x + G - 1) / G) : 0u;
+  const uint32_t T = blockIdx.x < bd_ntiles() ? static_cast<uint32_t>((bd_ntiles() - blockIdx.x + G - 1) / G) : 0u;
   uint32_t have_it = ~0u;
   StageHdr hd{};
   for (uint32_t kseq = 0;; ++kseq) {
@@ -1747,7 +1758,7 @@ __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl
       const unsigned long long u = hi;               // (offsets[rb] lies beyond the halo)
       const bool ok = !(u < h.rb && P.off[u] <= p + 15);
       if (!ok) continue;
-      const uint64_t key = P.gbase + (P.sm_lines ? P.off[u - 1] : p);   // u >= 1: offsets[0] = 0 <= p
+      const uint64_t key = bd_gbase() + (P.sm_lines ? P.off[u - 1] : p);   // u >= 1: offsets[0] = 0 <= p
       if (P.si) {
         if (lane == 0) {
           const unsigned long long g = atomicAdd(&P.st->pair_cursor, 1ULL);
@@ -1934,7 +1945,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       const long long wp = hd.chunk0 + static_cast<long long>(w) * kWin;
       if (wp < hd.hi) {                               // warp-uniform
         const long long p0 = wp + lane * 16;
-        const bool live = (p0 + 16 > 0) && (p0 < static_cast<long long>(P.nbytes));
+        const bool live = (p0 + 16 > 0) && (p0 < bd_nbytes());
         emit_text_chunk<W>(P, oc, outh, tv, p0, p0 - hd.sbase, live, qn);
       }
       __syncwarp();
@@ -2001,6 +2012,14 @@ __global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
       mbar_init(&ready[s], 1);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    if (P.desc) {   // text: the dimensions k_tile_bounds derived on the device
+      for (int i = 0; i < 4; ++i) s_bd[i] = P.desc[i];
+    } else {        // fixed stride: host values
+      s_bd[0] = P.nbytes;
+      s_bd[1] = P.ntiles;
+      s_bd[2] = P.gbase;
+      s_bd[3] = 0;
+    }
   }
   if constexpr (W == kWC) {
     uint32_t* ctab = reinterpret_cast<uint32_t*>(smem + Layout<W>::comb);   // keys, then counts
@@ -2024,6 +2043,7 @@ __global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
     }
   }
   __syncthreads();
+  if (s_bd[3]) return;   // more tiles than tile-bounds capacity: nothing mapped, the host grows + replays
   const uint32_t warp = threadIdx.x >> 5;
   if (warp >= static_cast<uint32_t>(nmap<W>()) && warp < static_cast<uint32_t>(nmap<W>() + kNProd))
     producer_loop<W>(P, smem, warp - nmap<W>());
@@ -2031,25 +2051,44 @@ __global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
   else map_loop<W>(P, smem, oc);
 }
 
-// tile bounds: record starts inside the staged window [w_lo, w_hi) of each text tile
-__global__ void k_tile_bounds(const uint64_t* off, uint64_t n, uint64_t ntiles, long long a0, uint64_t* tb) {
-  const uint64_t t = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
-  if (t >= ntiles) return;
-  const long long chunk0 = static_cast<long long>(t) * kT - a0;
-  const long long w_lo = max(0LL, chunk0 - kLead), w_hi = chunk0 + kT + kHalo;
-  uint64_t res[2];
-  const long long qs[2] = {w_lo, w_hi};
-  for (int k = 0; k < 2; ++k) {  // lower_bound over offsets[0..n]
-    uint64_t lo = 0, hi = n + 1;
-    const uint64_t q = static_cast<uint64_t>(qs[k]);
-    while (lo < hi) {
-      const uint64_t mid = (lo + hi) >> 1;
-      if (off[mid] < q) lo = mid + 1; else hi = mid;
-    }
-    res[k] = lo;
+// Batch dimensions + tile bounds of a text batch, on the device (mr_map enqueues without reading
+// offsets[n] back): nbytes = offsets[n], ntiles, the batch's global byte base (the previous
+// batch's base + length, or input_base) into desc[0..2]; desc[3] = 1 (and kErrTileCap) if the
+// tile-bounds buffer is too small.  Then, grid-stride, the record starts inside the staged window
+// [w_lo, w_hi) of every tile.
+__global__ void k_tile_bounds(const uint64_t* off, uint64_t n, long long a0, uint64_t tb_cap, const uint64_t* prev,
+                              uint64_t input_base, const uint8_t* rec, uint64_t* desc, uint64_t* tb,
+                              unsigned int* err) {
+  const uint64_t nbytes = off[n];
+  const uint64_t ntiles = nbytes ? (nbytes + static_cast<uint64_t>(a0) + kT - 1) / kT : 0;
+  const bool null_rec = nbytes && !rec;
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    desc[0] = nbytes;
+    desc[1] = ntiles;
+    desc[2] = prev ? prev[2] + prev[0] : input_base;
+    desc[3] = (ntiles > tb_cap || null_rec) ? 1ULL : 0ULL;   // the Map skips the batch
+    if (ntiles > tb_cap) atomicOr(err, kErrTileCap);
+    if (null_rec) atomicOr(err, kErrNullRecords);
   }
-  tb[2 * t] = res[0];
-  tb[2 * t + 1] = res[1];
+  if (ntiles > tb_cap || null_rec) return;
+  for (uint64_t t = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; t < ntiles;
+       t += static_cast<uint64_t>(gridDim.x) * blockDim.x) {
+    const long long chunk0 = static_cast<long long>(t) * kT - a0;
+    const long long w_lo = max(0LL, chunk0 - kLead), w_hi = chunk0 + kT + kHalo;
+    uint64_t res[2];
+    const long long qs[2] = {w_lo, w_hi};
+    for (int k = 0; k < 2; ++k) {  // lower_bound over offsets[0..n]
+      uint64_t lo = 0, hi = n + 1;
+      const uint64_t q = static_cast<uint64_t>(qs[k]);
+      while (lo < hi) {
+        const uint64_t mid = (lo + hi) >> 1;
+        if (off[mid] < q) lo = mid + 1; else hi = mid;
+      }
+      res[k] = lo;
+    }
+    tb[2 * t] = res[0];
+    tb[2 * t + 1] = res[1];
+  }
 }
 
 template <int W>
@@ -2059,10 +2098,11 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.rec = a.records;
   P.off = a.offsets;
   P.n = a.n;
-  P.nbytes = a.nbytes;
+  P.nbytes = a.nbytes;   // (fixed stride; text batches: on the device, P.desc)
   P.a0 = static_cast<long long>(reinterpret_cast<uintptr_t>(a.records) & 15u);
-  P.ntiles = map_tiles(a);
+  P.ntiles = W == kKM ? map_tiles(a) : 0;
   P.gbase = a.gbase;
+  P.desc = W == kKM ? nullptr : a.desc;
   for (int i = 0; i < 4; ++i)
     P.pat[i] = a.pattern[4 * i] | (a.pattern[4 * i + 1] << 8) | (a.pattern[4 * i + 2] << 16) |
                (static_cast<uint32_t>(a.pattern[4 * i + 3]) << 24);
@@ -2108,17 +2148,18 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
     }();
     P.wc_fast = fast;
   }
-  if (P.ntiles == 0) return cudaSuccess;
+  if (W == kKM && P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
-    const unsigned blocks = static_cast<unsigned>((P.ntiles + 255) / 256);
-    k_tile_bounds<<<blocks, 256, 0, s>>>(a.offsets, a.n, P.ntiles, P.a0, a.tile_bounds);
+    const unsigned blocks = static_cast<unsigned>(std::min<uint64_t>((a.tb_cap + 255) / 256 + 1, 8ULL * num_sms));
+    k_tile_bounds<<<blocks, 256, 0, s>>>(a.offsets, a.n, P.a0, a.tb_cap, a.prev_desc, a.input_base, a.records,
+                                         a.desc, a.tile_bounds, &a.st->err);
     count_launch();
   }
   const size_t smem = Layout<W>::cent + (W == kKM ? static_cast<size_t>(a.k) * 32 : 0);
   cudaError_t e = cudaFuncSetAttribute(k_map<W>, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
   if (e != cudaSuccess) return e;
-  int grid = a.grid > 0 ? a.grid : num_sms;
-  if (static_cast<uint64_t>(grid) > P.ntiles) grid = static_cast<int>(P.ntiles);
+  int grid = a.grid > 0 ? a.grid : num_sms;   // persistent CTAs; CTAs without a tile exit at once
+  if (W == kKM && static_cast<uint64_t>(grid) > P.ntiles) grid = static_cast<int>(P.ntiles);
   k_map<W><<<grid, threads_of<W>(), smem, s>>>(P);
   count_launch();
   return cudaGetLastError();
