@@ -337,6 +337,10 @@ struct mr_job {
   // one general stream (key, kref, u64 partial count) like II
   bool split() const { return cfg.workload == MR_WORDCOUNT && !ingested; }
   bool wc_comb() const { return split() && !(cfg.flags & MR_FLAG_NO_MAP_COMBINE); }
+  // second combiner level: exact words that miss the SMEM table go to an L2-resident count table
+  bool wc_table() const { return wc_comb() && map_wc_table_ok(cfg.flags); }
+  DBuf<uint32_t> xtab;            // 2^30 u32 counts by exact key (zero between runs)
+  bool xtab_dirty = false;        // a Map fed the table since its last extraction
   // KM: the Map accumulates the cluster sums itself (k <= 64; not for ingested partials)
   bool km_comb() const {
     return cfg.workload == MR_KMEANS && k <= 64 && !km_partial && !(cfg.flags & MR_FLAG_NO_MAP_COMBINE);
@@ -441,6 +445,8 @@ cudaError_t launch_batch(mr_job* job, const Batch& b) {
   a.out.h = job->h.p;
   a.out.hx = job->hx.p;
   a.out.hp = job->wc_comb() ? job->hp.p : nullptr;
+  a.out.xtab = job->wc_table() ? job->xtab.p : nullptr;
+  if (a.out.xtab) job->xtab_dirty = true;
   a.out.km_sums = job->km_comb() ? job->sums.p : nullptr;
   a.out.km_cnts = job->km_comb() ? job->cnts.p : nullptr;
   a.out.cap_p = job->cap_p;
@@ -593,6 +599,7 @@ mr_status settle_map(mr_job* job) {
     }
     job->stats.capacity_pairs = job->cap + job->cap_b + job->cap_c;
     CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
+    if (job->xtab_dirty) CK(cudaMemsetAsync(job->xtab.p, 0, job->xtab.n * 4, job->stream), "clear count table");
     if (job->km_comb()) {
       CK(cudaMemsetAsync(job->sums.p, 0, 64ULL * job->k, job->stream), "reset sums");
       CK(cudaMemsetAsync(job->cnts.p, 0, 8ULL * job->k, job->stream), "reset counts");
@@ -617,6 +624,7 @@ namespace {
 mr_status ingest_impl(mr_job* job, const void* entries, const void* heap, const uint64_t* recv_counts, uint32_t R);
 mr_status fold(mr_job* job);
 mr_status fold_finish(mr_job* job);
+mr_status xtab_extract(mr_job* job, uint64_t* mp);
 }
 
 namespace {
@@ -673,13 +681,14 @@ mr_status exchange(mr_job* job) {
   return ingest_impl(job, job->xrecv_e.p, job->xrecv_h.p, rc.data(), static_cast<uint32_t>(R));
 }
 
-// grow a device byte arena to >= need bytes, keeping its first `used` bytes
-cudaError_t grow_keep(DBuf<uint8_t>& b, uint64_t used, uint64_t need, cudaStream_t s) {
+// grow a device array to >= need elements, keeping its first `used` elements
+template <typename T>
+cudaError_t grow_keep(DBuf<T>& b, uint64_t used, uint64_t need, cudaStream_t s) {
   if (need <= b.n && b.p) return cudaSuccess;
-  DBuf<uint8_t> nb;
+  DBuf<T> nb;
   cudaError_t e = nb.ensure(std::max<uint64_t>(need, 2 * b.n));
   if (e != cudaSuccess) return e;
-  if (used && (e = cudaMemcpyAsync(nb.p, b.p, used, cudaMemcpyDeviceToDevice, s)) != cudaSuccess) return e;
+  if (used && (e = cudaMemcpyAsync(nb.p, b.p, used * sizeof(T), cudaMemcpyDeviceToDevice, s)) != cudaSuccess) return e;
   if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return e;
   b.release();
   b = nb;
@@ -751,6 +760,33 @@ mr_status fold_finish(mr_job* job) {
   mr_status st = ingest_impl(job, job->acc_e.p, job->acc_h.p, rc, 1);
   job->nfolds = 0;   // (the arena stays referenced until mr_reduce; reset clears it)
   return st;
+}
+
+// WC two-level combiner: the L2 count table -> combiner partial entries in hp (the same format
+// the SMEM table flush writes), so the partials' group-by, the exchange and the fold treat them
+// as before.  *mp = the number of distinct exact keys.  Leaves the table zeroed.  Synchronises.
+mr_status xtab_extract(mr_job* job, uint64_t* mp) {
+  cudaStream_t s = job->stream;
+  unsigned long long* cur = &job->st->n_extra;   // (scratch: n_extra is reset before its own use)
+  CK(cudaMemsetAsync(cur, 0, sizeof(unsigned long long), s), "memset cursor");
+  CK(launch_xtab_extract(job->xtab.p, job->xtab.n, job->hp.p, job->cap_p, cur, job->nsm, s), "table extract");
+  CK(read_state(job), "sync table extract");
+  uint64_t t = job->st_h.p->n_extra;
+  if (t > job->cap_p) {   // more distinct keys than partial capacity: grow (keeping the written ones), continue
+    const uint64_t done = job->cap_p;
+    CK(grow_keep(job->hp, done, t + t / 8 + 4096, s), "grow partials");
+    job->cap_p = job->hp.n;
+    job->tmp_h.p[4] = done;
+    CK(cudaMemcpyAsync(cur, job->tmp_h.p + 4, 8, cudaMemcpyHostToDevice, s), "set cursor");
+    CK(launch_xtab_extract(job->xtab.p, job->xtab.n, job->hp.p, job->cap_p, cur, job->nsm, s), "table extract");
+    CK(read_state(job), "sync table extract");
+    t = job->st_h.p->n_extra;
+    if (t > job->cap_p) return fail(job, MR_ERR_OOM, "table extraction still overflows");
+  }
+  CK(cudaMemsetAsync(cur, 0, sizeof(unsigned long long), s), "memset cursor");
+  job->xtab_dirty = false;
+  *mp = t;
+  return MR_OK;
 }
 
 }  // namespace
@@ -866,6 +902,10 @@ mr_status mr_job_reset(mr_job* job) {
   job->stats.capacity_pairs = cap;
   job->launches0 = g_kernel_launches.load();
   CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset state");
+  if (job->xtab_dirty) {   // a Map fed the count table but no mr_group extracted it
+    CK(cudaMemsetAsync(job->xtab.p, 0, job->xtab.n * 4, job->stream), "clear count table");
+    job->xtab_dirty = false;
+  }
   job->state = kCreated;
   return MR_OK;
 }
@@ -919,6 +959,10 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
       CK(job->hp.ensure(job->cap_p), "alloc partials");
     }
     job->stats.capacity_pairs = job->cap + job->cap_b + job->cap_c;
+  }
+  if (job->wc_table() && !job->xtab.p) {   // the L2 count table, zeroed once (extraction re-zeroes it)
+    CK(job->xtab.ensure(1ULL << kExactBits), "alloc count table");
+    CK(cudaMemsetAsync(job->xtab.p, 0, job->xtab.n * 4, job->stream), "zero count table");
   }
   if (job->batches.empty() && job->km_comb()) {   // KM combiner accumulators (summed over batches)
     CK(job->sums.ensure(8ULL * job->k), "alloc sums");
@@ -1094,6 +1138,10 @@ mr_status mr_group(mr_job* job) {
   job->mb = mb;
   job->mc = mc;
   job->mp = job->wc_comb() ? hs->pair_cursor_p : 0;
+  if (job->wc_table()) {   // the partials come from the L2 count table
+    st = xtab_extract(job, &job->mp);
+    if (st != MR_OK) return st;
+  }
   job->stats.pairs_partial = job->mp;
   job->stats.pairs = m + mb + mc;
   job->stats.pairs_hashed = mb;
@@ -1459,6 +1507,12 @@ mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_byte
       xs.nc = job->mc;
       xs.hp = job->hp.p;
       xs.np = job->wc_comb() ? hs->pair_cursor_p : 0;
+      if (job->wc_table()) {
+        uint64_t mpt = 0;
+        st = xtab_extract(job, &mpt);
+        if (st != MR_OK) return st;
+        xs.np = mpt;
+      }
       xs.n = m + xs.np + job->mc + job->mb;
       xs.kref = job->krefb.p;
     } else {
@@ -1696,7 +1750,7 @@ mr_status mr_job_destroy(mr_job* job) {
   job->xcounts.release(); job->xcursors.release(); job->xheapbase.release(); job->xcounts_h.release();
   job->src_e.release(); job->src_h.release(); job->km_list.release(); job->xwin.release();
   job->xsend_e.release(); job->xsend_h.release(); job->xrecv_e.release(); job->xrecv_h.release();
-  job->xrecv_counts.release(); job->acc_e.release(); job->acc_h.release();
+  job->xrecv_counts.release(); job->acc_e.release(); job->acc_h.release(); job->xtab.release();
   job->cent.release(); release_pairs(job); job->tb.release();
   job->swp.release(); job->seg_startp.release(); job->psum.release(); job->pxcounts.release();
   job->midx.release(); job->xkeys.release();

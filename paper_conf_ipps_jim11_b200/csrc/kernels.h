@@ -55,6 +55,7 @@ struct PairBufs {
   uint64_t cap_b = 0;
   uint64_t* hc = nullptr;    // WC mid stream: keys, capacity
   uint64_t cap_c = 0;
+  uint32_t* xtab = nullptr;  // WC two-level combiner: L2 count table (2^30 u32, by exact key)
 };
 
 // f-3 fused exchange: a destination rank's receive window (device pointers valid in this
@@ -101,7 +102,8 @@ constexpr uint64_t kMapTileBytes = 16384;    // owned bytes per text tile (map.c
 uint32_t map_prefetch(int w);
 uint32_t map_wait_hint();
 uint32_t map_dyn_windows(int workload);
-uint32_t map_wc_balanced();                     // L2 prefetch distance of the Map producers (BMR_MAP_PF)
+uint32_t map_wc_balanced();
+bool map_wc_table_ok(uint32_t flags);           // the WC Map can feed the L2 count table (SIO fast path)
 cudaError_t launch_map(const MapArgs& a, int num_sms, cudaStream_t s);
 
 // ---- group-by-key (hash radix sort + segment boundaries) ----
@@ -198,6 +200,11 @@ cudaError_t launch_comb_merge(const uint64_t* segp, uint64_t nsegp, const uint64
 cudaError_t launch_comb_add(const uint32_t* midx, const uint64_t* psum, uint64_t nsegp, uint64_t* counts,
                             cudaStream_t s);
 cudaError_t launch_key_lengths_list32(const uint32_t* keys, uint64_t n, uint64_t* lens, cudaStream_t s);
+// WC two-level combiner: the nonzero counts of the L2 table -> combiner partial entries
+// (key | count << 32) at out[*cursor ...] while *cursor < cap (those entries are zeroed; the rest
+// stay for a second call after growing out); *cursor counts every nonzero entry found
+cudaError_t launch_xtab_extract(uint32_t* tab, uint64_t nent, uint64_t* out, uint64_t cap,
+                                unsigned long long* cursor, int num_sms, cudaStream_t s);
 cudaError_t launch_key_decode_list32(const uint32_t* keys, uint64_t n, const uint64_t* key_off, uint8_t* out,
                                      cudaStream_t s);
 cudaError_t launch_offsets_scaled(const uint64_t* seg_start, uint64_t nseg, uint64_t scale, uint64_t* out,

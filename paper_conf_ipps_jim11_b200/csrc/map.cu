@@ -273,6 +273,8 @@ struct Params {
   const XWindow* xwin;     // f-3: InvertedIndex records appended straight to these windows
   uint32_t xranks;         // number of windows (0: local output)
   const uint64_t* desc;    // text: the batch descriptor (nbytes, ntiles, gbase, tile-bounds overflow)
+  uint32_t* xtab;          // WC: second combiner level, the L2-resident direct-address count table
+                           // (2^30 u32 counts indexed by the exact key); nullptr: exact stream
 };
 
 // Idle wait of a role warp on an mbarrier phase (map warps on a staged tile, producers on a free
@@ -1183,6 +1185,10 @@ __device__ __forceinline__ void wc_window(const Params& P, OutCtl* oc, uint8_t* 
     const uint32_t key = exact_key30_bf(__funnelshift_r(w0, w1, sh), (w1 >> sh) & 0xFFu, max(len, 1u));
     bool miss = act;
     if (act && P.comb) miss = !comb_add(ctab, key);
+    if (P.xtab) {   // second level: one fire-and-forget L2 atomic per miss (RED.ADD), no pair
+      if (miss) atomicAdd(P.xtab + key, 1u);
+      continue;
+    }
     const uint32_t ma = __ballot_sync(kFull, miss);
     if (miss) xq[nx + __popc(ma & lanemask_lt())] = key;
     nx += __popc(ma);
@@ -1969,7 +1975,13 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   // final flush of the partially filled half (all map warps done, nothing pending)
   named_bar_sync(2, nmap<W>() * 32);
   if constexpr (W == kWC) {
-    if (P.comb) {   // combiner partials -> global (one atomic per warp step; demand counted past capacity)
+    if (P.comb && P.xtab) {   // two-level combiner: the CTA's slots are added into the L2 table
+      const uint32_t* ctab = reinterpret_cast<const uint32_t*>(smem + Layout<W>::comb);
+      for (uint32_t i = warp * 32 + lane; i < static_cast<uint32_t>(Cfg<W>::kCombSlots); i += nmap<W>() * 32) {
+        const uint32_t k = ctab[i], c = ctab[Cfg<W>::kCombSlots + i];
+        if (k != kCombEmpty32) atomicAdd(P.xtab + k, c);
+      }
+    } else if (P.comb) {   // combiner partials -> global (one atomic per warp step; demand counted past capacity)
       const uint32_t* ctab = reinterpret_cast<const uint32_t*>(smem + Layout<W>::comb);
       for (uint32_t i0 = warp * 32; i0 < static_cast<uint32_t>(Cfg<W>::kCombSlots); i0 += nmap<W>() * 32) {
         const uint32_t k = ctab[i0 + lane], c = ctab[Cfg<W>::kCombSlots + i0 + lane];
@@ -2141,13 +2153,8 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.si = (a.flags & 2u) ? 1u : 0u;   // MR_FLAG_NO_SMEM_OUT
   P.sm_lines = (W == kSM && (a.flags & 0x200u)) ? 1u : 0u;   // MR_FLAG_SM_LINES
   P.wc_bal = map_wc_balanced();
-  {
-    static uint32_t fast = [] {
-      const char* e = getenv("BMR_WC_FAST");
-      return e ? static_cast<uint32_t>(atoi(e)) : 1u;
-    }();
-    P.wc_fast = fast;
-  }
+  P.wc_fast = 1;
+  P.xtab = (W == kWC && P.comb && map_wc_table_ok(a.flags)) ? a.out.xtab : nullptr;
   if (W == kKM && P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>(std::min<uint64_t>((a.tb_cap + 255) / 256 + 1, 8ULL * num_sms));
@@ -2207,6 +2214,12 @@ uint32_t map_wc_balanced() {
     return e ? static_cast<uint32_t>(atoi(e)) : 1u;
   }();
   return v;
+}
+
+// The WordCount L2 count table is fed by the SIO fast path only (wc_window); the memory-mode
+// ablations and the lane-serial emission keep the exact stream
+bool map_wc_table_ok(uint32_t flags) {
+  return !(flags & 3u) && map_wc_balanced() && map_dyn_windows(kWC);
 }
 
 int vbytes_of(int w) { return w == kKM ? 32 : w == kII ? 8 : 0; }

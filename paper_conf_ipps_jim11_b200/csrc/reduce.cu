@@ -629,6 +629,52 @@ cudaError_t launch_comb_add(const uint32_t* midx, const uint64_t* psum, uint64_t
   count_launch();
   return cudaGetLastError();
 }
+// WordCount two-level combiner (MapCG-style grouping by table):
+// the L2-resident count table the Map fed with one RED per exact word that missed the SMEM table
+// is turned into combiner partials.  One streaming read of the table (16 B per thread step, the
+// nonzero entries are sparse: a warp ballot skips empty steps); a warp's nonzero entries take one
+// global atomic for their output slots; written entries are zeroed, so the table is clean for the
+// next Map.
+__global__ void __launch_bounds__(256) k_xtab_extract(uint32_t* __restrict__ tab, uint64_t nv4, uint64_t* out,
+                                                    uint64_t cap, unsigned long long* cursor) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
+  uint4* t4 = reinterpret_cast<uint4*>(tab);
+  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i - threadIdx.x % 32 < nv4;
+       i += stride) {
+    uint4 v = i < nv4 ? __ldcs(t4 + i) : make_uint4(0, 0, 0, 0);
+    const uint32_t nz = (v.x != 0) + (v.y != 0) + (v.z != 0) + (v.w != 0);
+    if (!__any_sync(0xffffffffu, nz != 0)) continue;
+    const uint32_t incl = warp_inclusive_add(nz);
+    const uint32_t tot = __shfl_sync(0xffffffffu, incl, 31);
+    unsigned long long base = 0;
+    if (lane == 31) base = atomicAdd(cursor, static_cast<unsigned long long>(tot));
+    base = __shfl_sync(0xffffffffu, base, 31);
+    uint64_t o = base + incl - nz;
+    uint32_t c[4] = {v.x, v.y, v.z, v.w};
+    bool wrote = false;
+    for (int q = 0; q < 4; ++q) {
+      if (!c[q]) continue;
+      if (o < cap) {
+        out[o] = (4 * i + q) | (static_cast<uint64_t>(c[q]) << 32);
+        c[q] = 0;
+        wrote = true;
+      }
+      ++o;
+    }
+    if (wrote) t4[i] = make_uint4(c[0], c[1], c[2], c[3]);   // (entries past cap stay for the next call)
+  }
+}
+
+cudaError_t launch_xtab_extract(uint32_t* tab, uint64_t nent, uint64_t* out, uint64_t cap, unsigned long long* cursor,
+                                int num_sms, cudaStream_t s) {
+  const uint64_t nv4 = nent / 4;
+  k_xtab_extract<<<static_cast<unsigned>(std::min<uint64_t>(8ULL * num_sms, (nv4 + 255) / 256)), 256, 0, s>>>(
+      tab, nv4, out, cap, cursor);
+  count_launch();
+  return cudaGetLastError();
+}
+
 cudaError_t launch_key_lengths_list32(const uint32_t* keys, uint64_t n, uint64_t* lens, cudaStream_t s) {
   if (n == 0) return cudaSuccess;
   k_key_lengths_list32<<<blocks_for(n, 256), 256, 0, s>>>(keys, n, lens);
