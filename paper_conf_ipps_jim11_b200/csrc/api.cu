@@ -1132,8 +1132,10 @@ mr_status mr_group(mr_job* job) {
   const bool split = job->split();
   const uint64_t m_total = hs->pair_cursor;            // includes the flush filler pairs (sentinel keys)
   const uint64_t m = m_total - hs->pads;
-  const uint64_t mb = split ? hs->pair_cursor_b : 0;
-  const uint64_t mc = split ? hs->pair_cursor_c : 0;
+  // WC mid / hashed streams: slots taken (incl. the sentinel-filled chunk tails) and real entries
+  const uint64_t mb_total = split ? hs->pair_cursor_b : 0, mc_total = split ? hs->pair_cursor_c : 0;
+  const uint64_t mb = split ? mb_total - hs->pads_b : 0;
+  const uint64_t mc = split ? mc_total - hs->pads_c : 0;
   job->m = m;
   job->mb = mb;
   job->mc = mc;
@@ -1230,7 +1232,7 @@ mr_status mr_group(mr_job* job) {
     }
     if (job->prof.on) job->prof.end(job->stream, sp, &job->stats.seg_ms);
     // mid stream: exact 48-bit keys, keys only (no fillers: plain stores)
-    CK(run_sort(job->swc, job->hc.p, mc, &job->skeysc, nullptr, job->st, job->nsm, job->stream, &job->prof,
+    CK(run_sort(job->swc, job->hc.p, mc_total, &job->skeysc, nullptr, job->st, job->nsm, job->stream, &job->prof,
                 &job->stats.hist_ms, &job->stats.sort_ms, kMidBits),
        "radix sort (mid)");
     job->stats.sort_passes += job->swc.passes;
@@ -1247,7 +1249,7 @@ mr_status mr_group(mr_job* job) {
   {
     uint64_t* keys = split ? job->hb.p : job->h.p;
     const uint64_t* kref = split ? job->krefb.p : (has_kref(job->cfg.workload) || job->ingested ? job->kref.p : nullptr);
-    const uint64_t n = split ? mb : m_total;
+    const uint64_t n = split ? mb_total : m_total;   // (sentinel entries sort after every real key)
     const uint64_t nreal = split ? mb : m;
     uint32_t& kbits = split ? job->key_bits_b : job->key_bits;
     SortWork& W = split ? job->swb : job->sw;
@@ -1496,15 +1498,15 @@ mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_byte
     DevState* hs = job->st_h.p;
     const uint64_t m = hs->pair_cursor;
     job->m = m - hs->pads;
-    job->mb = job->split() ? hs->pair_cursor_b : 0;
-    job->mc = job->split() ? hs->pair_cursor_c : 0;
+    job->mb = job->split() ? hs->pair_cursor_b - hs->pads_b : 0;
+    job->mc = job->split() ? hs->pair_cursor_c - hs->pads_c : 0;
     job->stats.pairs = job->m + job->mb + job->mc;
     if (job->split()) {
       xs.mode = kXSplit;
       xs.hx = job->hx.p;
       xs.nx = m;
       xs.hc = job->hc.p;
-      xs.nc = job->mc;
+      xs.nc = hs->pair_cursor_c;   // (all slots: sentinel entries are skipped)
       xs.hp = job->hp.p;
       xs.np = job->wc_comb() ? hs->pair_cursor_p : 0;
       if (job->wc_table()) {
@@ -1513,7 +1515,7 @@ mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_byte
         if (st != MR_OK) return st;
         xs.np = mpt;
       }
-      xs.n = m + xs.np + job->mc + job->mb;
+      xs.n = m + xs.np + hs->pair_cursor_c + hs->pair_cursor_b;
       xs.kref = job->krefb.p;
     } else {
       xs.mode = kXPairs;

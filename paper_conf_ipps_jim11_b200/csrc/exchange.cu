@@ -50,6 +50,7 @@ __device__ __forceinline__ Rec get_rec(const XSource& S, uint64_t i) {
         r.v = S.hp[i - S.nx] >> 32;
       } else {
         key = S.hc[i - S.nx - S.np];
+        if (key == (1ULL << kMidBits) - 1ULL) { r.dest = ~0u; return r; }   // chunk-tail sentinel
       }
       r.kin = exact_key_bytes(key, r.klen);
       r.dest = dest_of_bytes(reinterpret_cast<const uint8_t*>(&r.kin), r.klen, S.nranks);
@@ -57,6 +58,7 @@ __device__ __forceinline__ Rec get_rec(const XSource& S, uint64_t i) {
       return r;
     }
     const uint64_t kr = S.kref[i - S.nx - S.np - S.nc];
+    if (kr == 0) { r.dest = ~0u; return r; }   // chunk-tail sentinel (hashed stream)
     r.kp = reinterpret_cast<const uint8_t*>(kr >> 16);
     r.klen = static_cast<uint32_t>(kr & 0xFFFF);
   } else if (S.mode == kXPairs) {

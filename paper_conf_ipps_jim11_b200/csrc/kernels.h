@@ -34,6 +34,7 @@ struct DevState {
   unsigned long long pair_cursor_p;  // WC combiner partials: demand in entries
   unsigned long long n_extra;        // WC: partial-only keys found by the merge (mr_group)
   unsigned long long words_comb;     // WC: words absorbed by the combiners (sum of partial counts)
+  unsigned long long pads_b, pads_c; // WC hashed / mid stream: sentinel entries in unused chunk tails
 };
 constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u, kErrTileCap = 4u, kErrNullRecords = 8u;
 

@@ -42,11 +42,17 @@ constexpr int kNMap = 16;
 #define BMR_SM_NMAP 24   // StringMatch map warps
 #endif
 #ifndef BMR_WC_COMB_BITS
-#define BMR_WC_COMB_BITS 13     // WordCount combiner: 2^bits direct-mapped slots (u32 key + u32 count);
-                                // 13 (64 KB): C5 exact stream 672 M -> 599 M keys, step 47.4 -> 46.2 ms
+#define BMR_WC_COMB_BITS 13     // WordCount SMEM combiner: 2^bits direct-mapped slots (u32 key + u32 count);
+                                // 13 (64 KB): round 1, exact stream 672 M -> 599 M keys; round 2 (L2 count
+                                // table behind it): 12 bits cost the C5 Map 0.5 ms in extra REDs
+#endif
+#ifndef BMR_WC_LQ
+#define BMR_WC_LQ 32            // WordCount long-word queue entries per map warp (>= 32; 64 measured no better)
 #endif
 #ifndef BMR_WC_OUT_BYTES
-#define BMR_WC_OUT_BYTES 8192   // WordCount output buffer bytes (x kNOut; 12 KB -> 8 KB: no measurable Map cost)
+#define BMR_WC_OUT_BYTES 3072   // WordCount output buffer bytes (x kNOut).  With the L2 count table and the
+                                // warp-chunked long-word output only rare > 16-byte words pass through them
+                                // (C5 Map, round 2: 4 KB 21.2 ms, 3 KB 18.0 ms, 2.6 KB 17.9 ms)
 #endif
 #ifndef BMR_WC_OFFCAP
 #define BMR_WC_OFFCAP 640       // WordCount: record offsets staged per tile (C1/C5 lines >= 27 B: <= 617 per
@@ -131,7 +137,12 @@ struct Cfg {
   // WC: in-SMEM combiner (MapCG-style): kCombSlots u64 entries
   // (u32 exact keys + u32 counts), direct-mapped, a slot keeps the first key that claims it
   static constexpr int kCombSlots = (W == kWC) ? (1 << BMR_WC_COMB_BITS) : 0;
+  // WC: per-warp queue of long words (> kWcExact bytes, <= 16) carried ACROSS windows with their
+  // bytes, so the stage can be released: keyed 32 at a time (one reservation per 32 words)
+  static constexpr int kLQ = (W == kWC) ? BMR_WC_LQ : 0;
 };
+struct LWord { uint64_t lo, hi, meta; };   // key bytes 0..7, 8..15; (batch position << 16) | length
+constexpr uint32_t kLQMaxLen = 16;
 constexpr int kCombBits = BMR_WC_COMB_BITS;
 static_assert(Cfg<kWC>::kCombSlots == (1 << kCombBits), "combiner slots");
 constexpr uint32_t kCombEmpty32 = 0xFFFFFFFFu;   // exact keys are < 2^30
@@ -191,7 +202,8 @@ struct Layout {
   static constexpr int hq = out + kNOut * Cfg<W>::kOutHalf;       // nmap x kHashQ x 4 (WC)
   static constexpr int xq = hq + nmap<W>() * Cfg<W>::kHashQ * 4;  // nmap x kXQ x 4 (WC)
   static constexpr int comb = xq + nmap<W>() * Cfg<W>::kXQ * 4;   // kCombSlots x 8 (WC)
-  static constexpr int cent = comb + Cfg<W>::kCombSlots * 8;      // KM centroids
+  static constexpr int lq = comb + Cfg<W>::kCombSlots * 8;        // nmap x kLQ x 24 (WC)
+  static constexpr int cent = lq + nmap<W>() * Cfg<W>::kLQ * 24;  // KM centroids
   static_assert(sizeof(OutCtl) <= hdr, "OutCtl overlaps the stage headers");
 };
 static_assert(64 % kNOut == 0, "6-bit generation counter must wrap on a buffer boundary");
@@ -1121,9 +1133,106 @@ __device__ __forceinline__ uint32_t exact_key30_bf(uint32_t lo, uint32_t b4, uin
   return y | (len == 5u ? (c4 << 24) : 0u);
 }
 
+// Output of the keyed long words: warp-private chunks of kLChunk entries of the mid stream (key
+// only) and of the hashed stream (key + kref), each taken with ONE global atomic on the stream's
+// cursor (the demand counter, D7) — the same amortisation as a buffer flush (L113) without the
+// flush warp's routing pass.  A warp's unused chunk tail is filled with sentinel entries at the
+// end (they sort last and are excluded: DevState::pads_b / pads_c).
+constexpr uint32_t kLChunk = 256;
+struct LOut { unsigned long long mid_base, hb_base; uint32_t mid_left, hb_left; };
+
+// n lanes (mask m, rank r) append to a chunked stream; returns each lane's slot
+__device__ __forceinline__ unsigned long long chunk_slot(unsigned long long* cursor, unsigned long long& base,
+                                                        uint32_t& left, uint32_t m) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t n = __popc(m), r = __popc(m & lanemask_lt());
+  unsigned long long nb = 0;
+  if (n > left) {   // the rest goes into a fresh chunk
+    if (lane == 0) nb = atomicAdd(cursor, static_cast<unsigned long long>(kLChunk));
+    nb = __shfl_sync(kFull, nb, 0);
+  }
+  const unsigned long long slot = r < left ? base + r : nb + (r - left);
+  if (n > left) {
+    base = nb + (n - left);
+    left = kLChunk - (n - left);
+  } else {
+    base += n;
+    left -= n;
+  }
+  return slot;
+}
+
+// Key up to 32 queued long words (one per lane): mid words (6..8 bytes) get their exact 48-bit key
+// (mid stream, no kref), longer ones the hash of their bytes (the same words KeyHash / hash_smem
+// feed) with the batch-relative reference; stored into the warp's output chunks.
+__device__ __forceinline__ void wc_drain(const Params& P, LOut& lo, LWord* lq, uint32_t& qn) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t n = min(qn, 32u);
+  if (n == 0) return;
+  __syncwarp();
+  const bool in = lane < n;
+  LWord w{0, 0, 0};
+  if (in) w = lq[lane];
+  const uint32_t len = static_cast<uint32_t>(w.meta & 0xFFFFu);
+  const bool mid = in && len <= kMidMax;
+  uint64_t key = 0, kref = 0;
+  if (mid) {
+    key = exact_key(w.lo, len);
+  } else if (in) {
+    KeyHash hs(P.hash_seed, len);
+    const uint32_t wd[4] = {static_cast<uint32_t>(w.lo), static_cast<uint32_t>(w.lo >> 32), static_cast<uint32_t>(w.hi),
+                            static_cast<uint32_t>(w.hi >> 32)};
+#pragma unroll
+    for (uint32_t k = 0; k < 4; ++k) {
+      if (4 * k >= len) break;
+      const uint32_t rem = len - 4 * k;
+      hs.add(rem >= 4 ? wd[k] : (wd[k] & ((1u << (8 * rem)) - 1u)));
+    }
+    key = hashed_key(hs.finish(), (P.flags & 8u) != 0, P.key_bits);
+    kref = (reinterpret_cast<uint64_t>(P.rec + (w.meta >> 16)) << 16) | len;
+  }
+  const uint32_t mm = __ballot_sync(kFull, mid), mh = __ballot_sync(kFull, in && !mid);
+  if (mm) {
+    const unsigned long long o = chunk_slot(&P.st->pair_cursor_c, lo.mid_base, lo.mid_left, mm);
+    if (mid && o < P.cap_c) P.ohc[o] = key;
+  }
+  if (mh) {
+    const unsigned long long o = chunk_slot(&P.st->pair_cursor_b, lo.hb_base, lo.hb_left, mh);
+    if (in && !mid && o < P.cap_b) {
+      P.ohb[o] = key;
+      P.okrefb[o] = kref;
+    }
+  }
+  // the remaining entries (<= kLQ - 32) move to the queue's front
+  const uint32_t rest = qn - n;
+  LWord r{0, 0, 0};
+  if (lane < rest) r = lq[n + lane];
+  __syncwarp();
+  if (lane < rest) lq[lane] = r;
+  __syncwarp();
+  qn = rest;
+}
+// end of a warp's work: sentinel entries in its chunks' unused tails
+__device__ __forceinline__ void wc_chunk_pads(const Params& P, const LOut& lo) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t sent = sentinel_of(P.key_bits);
+  for (uint32_t i = lane; i < lo.mid_left; i += 32)
+    if (lo.mid_base + i < P.cap_c) P.ohc[lo.mid_base + i] = (1ULL << kMidBits) - 1ULL;
+  for (uint32_t i = lane; i < lo.hb_left; i += 32)
+    if (lo.hb_base + i < P.cap_b) {
+      P.ohb[lo.hb_base + i] = sent;
+      P.okrefb[lo.hb_base + i] = 0;
+    }
+  if (lane == 0) {
+    if (lo.mid_left) atomicAdd(&P.st->pads_c, static_cast<unsigned long long>(lo.mid_left));
+    if (lo.hb_left) atomicAdd(&P.st->pads_b, static_cast<unsigned long long>(lo.hb_left));
+  }
+}
+
 // One 512-B window [p0w, p0w + 512) of a WordCount tile (lane = 16-byte chunk).  tv: the stage.
 __device__ __forceinline__ void wc_window(const Params& P, OutCtl* oc, uint8_t* outh, const TileView& tv,
-                                          long long p0w, uint32_t* xq, uint32_t* hq, uint32_t* ctab) {
+                                          long long p0w, uint32_t* xq, uint32_t* hq, uint32_t* ctab, LWord* lq,
+                                          uint32_t& qn, LOut& lo) {
   const uint32_t lane = threadIdx.x & 31;
   const long long N = bd_nbytes();
   const long long p0 = p0w + 16 * lane;
@@ -1193,28 +1302,44 @@ __device__ __forceinline__ void wc_window(const Params& P, OutCtl* oc, uint8_t* 
     if (miss) xq[nx + __popc(ma & lanemask_lt())] = key;
     nx += __popc(ma);
   }
-  if (nx + nl == 0) return;
-  const uint32_t packed = nx | (nl << kCbShift);
-  const Slot slot = reserve<kWC>(P, oc, outh, packed, P.out_cap);
-  uint8_t* half = outh + slot.half * Cfg<kWC>::kOutHalf;
-  uint32_t* sh = reinterpret_cast<uint32_t*>(half);
-  ulonglong2* top = reinterpret_cast<ulonglong2*>(half + Cfg<kWC>::kOutHalf);   // queued entry i: top[-1 - i]
-  const uint32_t kb0 = cur_cb(slot.base), ka = cur_ca(slot.base);
-  __syncwarp();
-  for (uint32_t i = lane; i < nx; i += 32) sh[ka + i] = xq[i];
-  for (uint32_t q = lane; q < nl; q += 32) {           // lane-parallel keys of the long words
-    const uint32_t e = hq[q];
-    const long long p = tv.sbase + static_cast<long long>(e & 0x7FFFu);
-    const uint32_t len = e >> 15;
-    ulonglong2 ent;
-    if (len <= kMidMax) {                                // mid stream: exact 48-bit key, no kref
-      ent = make_ulonglong2(exact_key(bytes8_at(P, tv, p, len), len), 0ULL);
-    } else {
-      ent = make_ulonglong2(key_at(P, tv, p, len), (reinterpret_cast<uint64_t>(P.rec + p) << 16) | len);
-    }
-    top[-1 - static_cast<int>(kb0 + q)] = ent;
+  // exact keys that missed (exact-stream mode: no L2 table): one reservation, copied out
+  if (nx) {
+    const Slot slot = reserve<kWC>(P, oc, outh, nx, P.out_cap);
+    uint32_t* sh = reinterpret_cast<uint32_t*>(outh + slot.half * Cfg<kWC>::kOutHalf);
+    const uint32_t ka = cur_ca(slot.base);
+    __syncwarp();
+    for (uint32_t i = lane; i < nx; i += 32) sh[ka + i] = xq[i];
+    commit(oc, slot, nx);
   }
-  commit(oc, slot, packed);
+  // long words: their bytes into the warp's cross-window queue (keyed 32 at a time by wc_drain);
+  // words longer than kLQMaxLen bytes (rare) are keyed here, one lane each
+  for (uint32_t q0 = 0; q0 < nl; q0 += 32) {
+    const uint32_t chunk = min(32u, nl - q0);
+    if (qn + chunk > static_cast<uint32_t>(Cfg<kWC>::kLQ)) wc_drain(P, lo, lq, qn);
+    const bool in = lane < chunk;
+    const uint32_t e = in ? hq[q0 + lane] : 0u;
+    const uint32_t pos = e & 0x7FFFu, len = e >> 15;
+    const bool small = in && len <= kLQMaxLen;
+    const uint32_t ms = __ballot_sync(kFull, small), mb = __ballot_sync(kFull, in && !small);
+    if (small) {   // (a word of <= 16 bytes starting in the tile lies inside the staged window)
+      LWord* d = lq + qn + __popc(ms & lanemask_lt());
+      d->lo = static_cast<uint64_t>(smem_word_at(tv.sb, pos)) | (static_cast<uint64_t>(smem_word_at(tv.sb, pos + 4)) << 32);
+      d->hi = static_cast<uint64_t>(smem_word_at(tv.sb, pos + 8)) | (static_cast<uint64_t>(smem_word_at(tv.sb, pos + 12)) << 32);
+      d->meta = (static_cast<uint64_t>(tv.sbase + pos) << 16) | len;
+    }
+    qn += __popc(ms);
+    if (mb) {
+      const Slot slot = reserve<kWC>(P, oc, outh, __popc(mb) << kCbShift, P.out_cap);
+      ulonglong2* top = reinterpret_cast<ulonglong2*>(outh + slot.half * Cfg<kWC>::kOutHalf + Cfg<kWC>::kOutHalf);
+      if (in && !small) {
+        const long long p = tv.sbase + static_cast<long long>(pos);
+        top[-1 - static_cast<int>(cur_cb(slot.base) + __popc(mb & lanemask_lt()))] =
+            make_ulonglong2(key_at(P, tv, p, len), (reinterpret_cast<uint64_t>(P.rec + p) << 16) | len);
+      }
+      commit(oc, slot, __popc(mb) << kCbShift);
+    }
+  }
+  __syncwarp();
 }
 
 // WordCount map warps in SIO mode: windows from the shared counter (tile order), the stage
@@ -1229,6 +1354,9 @@ __device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   uint32_t* hq = reinterpret_cast<uint32_t*>(smem + Layout<kWC>::hq) + warp * Cfg<kWC>::kHashQ;
   uint32_t* xq = reinterpret_cast<uint32_t*>(smem + Layout<kWC>::xq) + warp * Cfg<kWC>::kXQ;
   uint32_t* ctab = reinterpret_cast<uint32_t*>(smem + Layout<kWC>::comb);
+  LWord* lq = reinterpret_cast<LWord*>(smem + Layout<kWC>::lq) + warp * Cfg<kWC>::kLQ;
+  uint32_t qn = 0;   // long words queued by this warp
+  LOut lo{0, 0, 0, 0};   // this warp's output chunks (none yet)
   uint32_t have_it = ~0u;
   long long t = 0, sbase = 0, hi = 0, stg_hi = 0;
   for (;;) {
@@ -1250,11 +1378,14 @@ __device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       const TileView tv{smem + Layout<W>::bytes + s * kStageBytes,
                         reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits), sbase, stg_hi, 0,
                         0};
-      wc_window(P, oc, outh, tv, wp, xq, hq, ctab);
+      wc_window(P, oc, outh, tv, wp, xq, hq, ctab, lq, qn, lo);
+      if (qn >= 32) wc_drain(P, lo, lq, qn);
     }
     __syncwarp();
     lane0_mbar_arrive(&empty[s]);
   }
+  while (qn) wc_drain(P, lo, lq, qn);   // this warp's last long words
+  wc_chunk_pads(P, lo);
 }
 
 // InvertedIndex URL queue (per map warp, in the hq region): the markers of a window are queued as
