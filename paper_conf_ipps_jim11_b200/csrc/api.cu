@@ -338,9 +338,18 @@ struct mr_job {
   bool split() const { return cfg.workload == MR_WORDCOUNT && !ingested; }
   bool wc_comb() const { return split() && !(cfg.flags & MR_FLAG_NO_MAP_COMBINE); }
   // second combiner level: exact words that miss the SMEM table go to an L2-resident count table
-  bool wc_table() const { return wc_comb() && map_wc_table_ok(cfg.flags); }
+  // (the raw multi-GPU exchange, MR_FLAG_NO_COMBINE, keeps the literal pair streams)
+  bool wc_table() const {
+    return wc_comb() && map_wc_table_ok(cfg.flags) && !(cfg.flags & MR_FLAG_NO_COMBINE);
+  }
   DBuf<uint32_t> xtab;            // 2^30 u32 counts by exact key (zero between runs)
-  bool xtab_dirty = false;        // a Map fed the table since its last extraction
+  // mid words (6..8 symbols): open-addressing table of 48-bit exact keys + counts (2^mbits slots)
+  DBuf<uint64_t> mtab_keys;
+  DBuf<uint32_t> mtab_cnt;
+  uint32_t mbits = 18;
+  bool xtab_dirty = false;        // a Map fed the tables since their last extraction
+  bool mid_from_table = false;    // this group's mid keys / counts come from the mid table
+  DBuf<uint64_t> mkeys_out, mcounts;
   // KM: the Map accumulates the cluster sums itself (k <= 64; not for ingested partials)
   bool km_comb() const {
     return cfg.workload == MR_KMEANS && k <= 64 && !km_partial && !(cfg.flags & MR_FLAG_NO_MAP_COMBINE);
@@ -446,6 +455,9 @@ cudaError_t launch_batch(mr_job* job, const Batch& b) {
   a.out.hx = job->hx.p;
   a.out.hp = job->wc_comb() ? job->hp.p : nullptr;
   a.out.xtab = job->wc_table() ? job->xtab.p : nullptr;
+  a.out.mkeys = job->wc_table() ? job->mtab_keys.p : nullptr;
+  a.out.mcnt = job->wc_table() ? job->mtab_cnt.p : nullptr;
+  a.out.mbits = job->mbits;
   if (a.out.xtab) job->xtab_dirty = true;
   a.out.km_sums = job->km_comb() ? job->sums.p : nullptr;
   a.out.km_cnts = job->km_comb() ? job->cnts.p : nullptr;
@@ -557,6 +569,8 @@ mr_status do_segments32(mr_job* job, const uint32_t* skeys, uint64_t m, DBuf<uin
 
 // D7: settle the Map of every batch.  The cursors counted demand past capacity: grow the pair
 // buffers and replay every batch.  Leaves the final DevState in st_h.
+cudaError_t clear_tables(mr_job* job);
+
 mr_status settle_map(mr_job* job) {
   CK(read_state(job), "map (async)");
   DevState* hs = job->st_h.p;
@@ -580,10 +594,18 @@ mr_status settle_map(mr_job* job) {
     job->stats.map_tiles = tiles;
   }
   const bool tile_over = (hs->err & kErrTileCap) != 0;
+  const bool mid_over = (hs->err & kErrMidTable) != 0;
+  if (mid_over) {   // mid table too full: a table 4x larger (grow-only), then the replay below
+    job->mbits += 2;
+    job->mtab_keys.release();
+    job->mtab_cnt.release();
+    CK(job->mtab_keys.ensure(1ULL << job->mbits), "grow mid table");
+    CK(job->mtab_cnt.ensure((1ULL << job->mbits) * kMidStripes), "grow mid table");
+  }
   const uint64_t m = hs->pair_cursor, mb = job->split() ? hs->pair_cursor_b : 0;
   const uint64_t mc = job->split() ? hs->pair_cursor_c : 0;
   const uint64_t mp = job->wc_comb() ? hs->pair_cursor_p : 0;
-  if (tile_over || m > job->cap || mb > job->cap_b || mc > job->cap_c || mp > job->cap_p) {
+  if (tile_over || mid_over || m > job->cap || mb > job->cap_b || mc > job->cap_c || mp > job->cap_p) {
     if (tile_over) job->tb_cap = max_tiles + 1024;   // (tb itself is grown by launch_batch)
     const uint64_t ncap_p = job->wc_comb() ? std::max(job->cap_p, mp + mp / 8 + 4096) : 0;
     const uint64_t ncap = std::max(job->cap, m + m / 8 + 4096);
@@ -599,7 +621,7 @@ mr_status settle_map(mr_job* job) {
     }
     job->stats.capacity_pairs = job->cap + job->cap_b + job->cap_c;
     CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
-    if (job->xtab_dirty) CK(cudaMemsetAsync(job->xtab.p, 0, job->xtab.n * 4, job->stream), "clear count table");
+    if (job->xtab_dirty || mid_over) CK(clear_tables(job), "clear the tables");
     if (job->km_comb()) {
       CK(cudaMemsetAsync(job->sums.p, 0, 64ULL * job->k, job->stream), "reset sums");
       CK(cudaMemsetAsync(job->cnts.p, 0, 8ULL * job->k, job->stream), "reset counts");
@@ -607,7 +629,7 @@ mr_status settle_map(mr_job* job) {
     for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
     job->stats.replays += job->batches.size();
     CK(read_state(job), "replay (async)");
-    if ((hs->err & kErrTileCap) || hs->pair_cursor > job->cap ||
+    if ((hs->err & (kErrTileCap | kErrMidTable)) || hs->pair_cursor > job->cap ||
         (job->split() && (hs->pair_cursor_b > job->cap_b || hs->pair_cursor_c > job->cap_c)) ||
         (job->wc_comb() && hs->pair_cursor_p > job->cap_p))
       return fail(job, MR_ERR_OOM, "replay still overflows");
@@ -625,6 +647,8 @@ mr_status ingest_impl(mr_job* job, const void* entries, const void* heap, const 
 mr_status fold(mr_job* job);
 mr_status fold_finish(mr_job* job);
 mr_status xtab_extract(mr_job* job, uint64_t* mp);
+mr_status tables_extract(mr_job* job);
+cudaError_t clear_tables(mr_job* job);
 }
 
 namespace {
@@ -760,6 +784,79 @@ mr_status fold_finish(mr_job* job) {
   mr_status st = ingest_impl(job, job->acc_e.p, job->acc_h.p, rc, 1);
   job->nfolds = 0;   // (the arena stays referenced until mr_reduce; reset clears it)
   return st;
+}
+
+// both WC tables back to empty (after a replay's first Map or a reset without mr_group)
+cudaError_t clear_tables(mr_job* job) {
+  cudaError_t e = cudaSuccess;
+  if (job->xtab.p) e = cudaMemsetAsync(job->xtab.p, 0, job->xtab.n * 4, job->stream);
+  if (e == cudaSuccess && job->mtab_keys.p) e = cudaMemsetAsync(job->mtab_keys.p, 0xFF, job->mtab_keys.n * 8, job->stream);
+  if (e == cudaSuccess && job->mtab_cnt.p) e = cudaMemsetAsync(job->mtab_cnt.p, 0, job->mtab_cnt.n * 4, job->stream);
+  return e;
+}
+
+// WC tables -> the group's exact keys (xkeys / pxcounts, the "partial-only" list: every key once)
+// and mid keys (mkeys_out / mcounts, with identity segments): no sort, no merge.  Grows the
+// output lists when they overflow (the entries past capacity stay in the table for a second
+// pass).  Synchronises.
+mr_status tables_extract(mr_job* job) {
+  cudaStream_t s = job->stream;
+  unsigned long long* cur = &job->st->n_extra;   // scratch cursors: n_extra, words_comb
+  unsigned long long* wsum = &job->st->words_comb;
+  CK(cudaMemsetAsync(cur, 0, 2 * sizeof(unsigned long long), s), "memset cursor");
+  if (job->xkeys.n < 4096) { CK(job->xkeys.ensure(1 << 20), "alloc keys"); CK(job->pxcounts.ensure(1 << 20), "alloc counts"); }
+  uint64_t cap = std::min(job->xkeys.n, job->pxcounts.n);
+  CK(launch_xtab_extract_list(job->xtab.p, job->xtab.n, job->xkeys.p, job->pxcounts.p, cap, cur, wsum, job->nsm, s),
+     "table extract");
+  CK(read_state(job), "sync table extract");
+  uint64_t t = job->st_h.p->n_extra;
+  if (t > cap) {
+    CK(grow_keep(job->xkeys, cap, t + t / 8 + 4096, s), "grow keys");
+    CK(grow_keep(job->pxcounts, cap, t + t / 8 + 4096, s), "grow counts");
+    job->tmp_h.p[4] = cap;
+    CK(cudaMemcpyAsync(cur, job->tmp_h.p + 4, 8, cudaMemcpyHostToDevice, s), "set cursor");
+    const uint64_t cap2 = std::min(job->xkeys.n, job->pxcounts.n);
+    CK(launch_xtab_extract_list(job->xtab.p, job->xtab.n, job->xkeys.p, job->pxcounts.p, cap2, cur, wsum, job->nsm, s),
+       "table extract");
+    CK(read_state(job), "sync table extract");
+    t = job->st_h.p->n_extra;
+    if (t > cap2) return fail(job, MR_ERR_OOM, "table extraction still overflows");
+  }
+  job->n_extra = t;
+  uint64_t words = job->st_h.p->words_comb;
+  // mid table
+  CK(cudaMemsetAsync(cur, 0, sizeof(unsigned long long), s), "memset cursor");
+  if (job->mkeys_out.n < 4096) { CK(job->mkeys_out.ensure(1 << 18), "alloc mid keys"); CK(job->mcounts.ensure(1 << 18), "alloc mid counts"); }
+  cap = std::min(job->mkeys_out.n, job->mcounts.n);
+  CK(launch_mtab_extract(job->mtab_keys.p, job->mtab_cnt.p, job->mtab_keys.n, job->mkeys_out.p, job->mcounts.p, cap, cur,
+                         wsum, job->nsm, s),
+     "mid table extract");
+  CK(read_state(job), "sync mid table extract");
+  t = job->st_h.p->n_extra;
+  if (t > cap) {
+    CK(grow_keep(job->mkeys_out, cap, t + t / 8 + 4096, s), "grow mid keys");
+    CK(grow_keep(job->mcounts, cap, t + t / 8 + 4096, s), "grow mid counts");
+    job->tmp_h.p[4] = cap;
+    CK(cudaMemcpyAsync(cur, job->tmp_h.p + 4, 8, cudaMemcpyHostToDevice, s), "set cursor");
+    const uint64_t cap2 = std::min(job->mkeys_out.n, job->mcounts.n);
+    CK(launch_mtab_extract(job->mtab_keys.p, job->mtab_cnt.p, job->mtab_keys.n, job->mkeys_out.p, job->mcounts.p, cap2,
+                           cur, wsum, job->nsm, s),
+       "mid table extract");
+    CK(read_state(job), "sync mid table extract");
+    t = job->st_h.p->n_extra;
+    if (t > cap2) return fail(job, MR_ERR_OOM, "mid table extraction still overflows");
+  }
+  job->nseg_c = t;
+  job->stats.words_combined = job->st_h.p->words_comb;   // exact + mid words counted by the tables
+  (void)words;
+  CK(job->seg_startx.ensure(t + 2), "alloc mid segments");
+  CK(launch_iota_scaled(t, 1, job->seg_startx.p, s), "mid segments");   // one segment per mid key
+  job->segc = job->seg_startx.p;
+  job->skeysc = job->mkeys_out.p;
+  job->mid_from_table = true;
+  CK(cudaMemsetAsync(cur, 0, 2 * sizeof(unsigned long long), s), "memset cursor");
+  job->xtab_dirty = false;
+  return MR_OK;
 }
 
 // WC two-level combiner: the L2 count table -> combiner partial entries in hp (the same format
@@ -902,10 +999,11 @@ mr_status mr_job_reset(mr_job* job) {
   job->stats.capacity_pairs = cap;
   job->launches0 = g_kernel_launches.load();
   CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset state");
-  if (job->xtab_dirty) {   // a Map fed the count table but no mr_group extracted it
-    CK(cudaMemsetAsync(job->xtab.p, 0, job->xtab.n * 4, job->stream), "clear count table");
+  if (job->xtab_dirty) {   // a Map fed the tables but no mr_group extracted them
+    CK(clear_tables(job), "clear the tables");
     job->xtab_dirty = false;
   }
+  job->mid_from_table = false;
   job->state = kCreated;
   return MR_OK;
 }
@@ -960,9 +1058,11 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
     }
     job->stats.capacity_pairs = job->cap + job->cap_b + job->cap_c;
   }
-  if (job->wc_table() && !job->xtab.p) {   // the L2 count table, zeroed once (extraction re-zeroes it)
+  if (job->wc_table() && !job->xtab.p) {   // the tables, emptied once (extraction re-empties them)
     CK(job->xtab.ensure(1ULL << kExactBits), "alloc count table");
-    CK(cudaMemsetAsync(job->xtab.p, 0, job->xtab.n * 4, job->stream), "zero count table");
+    CK(job->mtab_keys.ensure(1ULL << job->mbits), "alloc mid table");
+    CK(job->mtab_cnt.ensure((1ULL << job->mbits) * kMidStripes), "alloc mid table");
+    CK(clear_tables(job), "empty the tables");
   }
   if (job->batches.empty() && job->km_comb()) {   // KM combiner accumulators (summed over batches)
     CK(job->sums.ensure(8ULL * job->k), "alloc sums");
@@ -1140,10 +1240,7 @@ mr_status mr_group(mr_job* job) {
   job->mb = mb;
   job->mc = mc;
   job->mp = job->wc_comb() ? hs->pair_cursor_p : 0;
-  if (job->wc_table()) {   // the partials come from the L2 count table
-    st = xtab_extract(job, &job->mp);
-    if (st != MR_OK) return st;
-  }
+  const bool tables = job->wc_table();   // exact + mid words were counted by the tables, not emitted
   job->stats.pairs_partial = job->mp;
   job->stats.pairs = m + mb + mc;
   job->stats.pairs_hashed = mb;
@@ -1188,7 +1285,22 @@ mr_status mr_group(mr_job* job) {
   job->permb = nullptr;
   job->skeysc = nullptr;
   job->segc = nullptr;
-  if (split) {
+  job->mid_from_table = false;
+  if (split && tables) {
+    // the two tables hold every exact and mid word: their nonzero counts are the final keys
+    Prof::Span sp{};
+    if (job->prof.on) job->prof.begin(job->stream, sp);
+    job->nseg_a = 0;
+    job->nseg_p = 0;
+    job->mp = 0;
+    job->skeysp = nullptr;
+    job->perm = nullptr;
+    st = tables_extract(job);
+    if (st != MR_OK) return st;
+    CK(job->seg_counts.ensure(1), "alloc");
+    job->sega = job->tile_base.p;   // (no exact segments)
+    if (job->prof.on) job->prof.end(job->stream, sp, &job->stats.seg_ms);
+  } else if (split) {
     // exact stream: keys only (the key is the record), no byte verification needed
     CK(run_sort32(job->sw, job->hx.p, m_total, &job->skeysx, job->st, job->nsm, job->stream, &job->prof,
                   &job->stats.hist_ms, &job->stats.sort_keys_ms, kExactBits),   // exact keys < 2^30
@@ -1346,7 +1458,11 @@ mr_status mr_reduce(mr_job* job) {
         if (job->n_extra)
           CK(cudaMemcpyAsync(job->counts.p + job->nseg_a, job->pxcounts.p, job->n_extra * 8, cudaMemcpyDeviceToDevice, s),
              "counts (partial-only)");
-        CK(launch_seg_lengths(job->segc, job->nseg_c, job->counts.p + na, s), "counts (mid)");
+        if (job->mid_from_table)
+          CK(cudaMemcpyAsync(job->counts.p + na, job->mcounts.p, job->nseg_c * 8, cudaMemcpyDeviceToDevice, s),
+             "counts (mid)");
+        else
+          CK(launch_seg_lengths(job->segc, job->nseg_c, job->counts.p + na, s), "counts (mid)");
         CK(launch_seg_lengths(job->seg_startb.p, job->nseg_b, job->counts.p + na + job->nseg_c, s),
            "counts (hashed)");
         CK(launch_key_decode(job->segc, job->nseg_c, job->skeysc, job->key_off.p + na, job->keys_out.p, s),
@@ -1508,13 +1624,7 @@ mr_status mr_partition_count(mr_job* job, uint64_t* counts, uint64_t* entry_byte
       xs.hc = job->hc.p;
       xs.nc = hs->pair_cursor_c;   // (all slots: sentinel entries are skipped)
       xs.hp = job->hp.p;
-      xs.np = job->wc_comb() ? hs->pair_cursor_p : 0;
-      if (job->wc_table()) {
-        uint64_t mpt = 0;
-        st = xtab_extract(job, &mpt);
-        if (st != MR_OK) return st;
-        xs.np = mpt;
-      }
+      xs.np = job->wc_comb() ? hs->pair_cursor_p : 0;   // (no tables on the raw exchange path: wc_table)
       xs.n = m + xs.np + hs->pair_cursor_c + hs->pair_cursor_b;
       xs.kref = job->krefb.p;
     } else {
@@ -1752,7 +1862,8 @@ mr_status mr_job_destroy(mr_job* job) {
   job->xcounts.release(); job->xcursors.release(); job->xheapbase.release(); job->xcounts_h.release();
   job->src_e.release(); job->src_h.release(); job->km_list.release(); job->xwin.release();
   job->xsend_e.release(); job->xsend_h.release(); job->xrecv_e.release(); job->xrecv_h.release();
-  job->xrecv_counts.release(); job->acc_e.release(); job->acc_h.release(); job->xtab.release();
+  job->xrecv_counts.release(); job->acc_e.release(); job->acc_h.release(); job->xtab.release(); job->mtab_keys.release();
+  job->mtab_cnt.release(); job->mkeys_out.release(); job->mcounts.release();
   job->cent.release(); release_pairs(job); job->tb.release();
   job->swp.release(); job->seg_startp.release(); job->psum.release(); job->pxcounts.release();
   job->midx.release(); job->xkeys.release();

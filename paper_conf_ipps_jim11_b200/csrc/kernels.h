@@ -35,8 +35,19 @@ struct DevState {
   unsigned long long n_extra;        // WC: partial-only keys found by the merge (mr_group)
   unsigned long long words_comb;     // WC: words absorbed by the combiners (sum of partial counts)
   unsigned long long pads_b, pads_c; // WC hashed / mid stream: sentinel entries in unused chunk tails
+  unsigned long long mid_fail;       // WC mid table: inserts that found no slot (-> grow + replay)
 };
-constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u, kErrTileCap = 4u, kErrNullRecords = 8u;
+constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u, kErrTileCap = 4u, kErrNullRecords = 8u,
+                       kErrMidTable = 16u;
+// WC mid-word table: open addressing over 48-bit exact keys, empty slot = all ones
+constexpr uint64_t kMidEmpty = ~0ULL;
+constexpr uint32_t kMidProbes = 32;
+// counts of a slot are striped over kMidStripes words (the warp's stripe), so the Zipf-hot mid
+// words do not serialise every RED on one address; the extraction sums the stripes
+constexpr uint32_t kMidStripes = 16;
+__host__ __device__ inline uint64_t mid_slot(uint64_t key, uint32_t bits) {
+  return (key * 0x9E3779B97F4A7C15ULL) >> (64 - bits);
+}
 
 // Intermediate pairs, SoA in HBM (SURVEY §8(a) layout): sort key, key reference, value.
 // WordCount Map output is three streams: exact keys (hx, u32: the key is the record, value 1),
@@ -57,6 +68,9 @@ struct PairBufs {
   uint64_t* hc = nullptr;    // WC mid stream: keys, capacity
   uint64_t cap_c = 0;
   uint32_t* xtab = nullptr;  // WC two-level combiner: L2 count table (2^30 u32, by exact key)
+  uint64_t* mkeys = nullptr; // WC mid words (6..8 symbols): open-addressing table of 48-bit exact keys
+  uint32_t* mcnt = nullptr;  //   and their counts, 2^mbits slots
+  uint32_t mbits = 0;
 };
 
 // f-3 fused exchange: a destination rank's receive window (device pointers valid in this
@@ -206,6 +220,14 @@ cudaError_t launch_key_lengths_list32(const uint32_t* keys, uint64_t n, uint64_t
 // stay for a second call after growing out); *cursor counts every nonzero entry found
 cudaError_t launch_xtab_extract(uint32_t* tab, uint64_t nent, uint64_t* out, uint64_t cap,
                                 unsigned long long* cursor, int num_sms, cudaStream_t s);
+// the same into separate lists (keys u32, counts u64) — the final exact keys — and *wsum += the
+// counts (words absorbed)
+cudaError_t launch_xtab_extract_list(uint32_t* tab, uint64_t nent, uint32_t* okeys, uint64_t* ocounts, uint64_t cap,
+                                     unsigned long long* cursor, unsigned long long* wsum, int num_sms, cudaStream_t s);
+// WC mid table -> (48-bit key, count) lists; extracted slots are reset (key empty, count 0)
+cudaError_t launch_mtab_extract(uint64_t* mkeys, uint32_t* mcnt, uint64_t nslots, uint64_t* okeys, uint64_t* ocounts,
+                                uint64_t cap, unsigned long long* cursor, unsigned long long* wsum, int num_sms,
+                                cudaStream_t s);
 cudaError_t launch_key_decode_list32(const uint32_t* keys, uint64_t n, const uint64_t* key_off, uint8_t* out,
                                      cudaStream_t s);
 cudaError_t launch_offsets_scaled(const uint64_t* seg_start, uint64_t nseg, uint64_t scale, uint64_t* out,

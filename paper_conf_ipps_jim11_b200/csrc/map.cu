@@ -287,6 +287,9 @@ struct Params {
   const uint64_t* desc;    // text: the batch descriptor (nbytes, ntiles, gbase, tile-bounds overflow)
   uint32_t* xtab;          // WC: second combiner level, the L2-resident direct-address count table
                            // (2^30 u32 counts indexed by the exact key); nullptr: exact stream
+  uint64_t* mkeys;         // WC: mid words (6..8 symbols) counted in an open-addressing table of
+  uint32_t* mcnt;          //   their 48-bit exact keys (2^mbits slots); nullptr: mid stream
+  uint32_t mbits;
 };
 
 // Idle wait of a role warp on an mbarrier phase (map warps on a staged tile, producers on a free
@@ -1191,7 +1194,30 @@ __device__ __forceinline__ void wc_drain(const Params& P, LOut& lo, LWord* lq, u
     key = hashed_key(hs.finish(), (P.flags & 8u) != 0, P.key_bits);
     kref = (reinterpret_cast<uint64_t>(P.rec + (w.meta >> 16)) << 16) | len;
   }
-  const uint32_t mm = __ballot_sync(kFull, mid), mh = __ballot_sync(kFull, in && !mid);
+  if (P.mkeys) {   // mid table: equal keys of the drain aggregated (match.any), then the group's
+                  // leader finds the key (or claims an empty slot) and adds the group size to its
+                  // warp's stripe of the slot's count (one RED)
+    const uint32_t grp = __match_any_sync(kFull, mid ? key : kMidEmpty);
+    const bool lead = mid && lane == static_cast<uint32_t>(__ffs(grp) - 1);
+    const uint64_t mask = (1ULL << P.mbits) - 1ULL;
+    uint64_t h = mid_slot(key, P.mbits);
+    bool done = !lead;
+    for (uint32_t pr = 0; lead && pr < kMidProbes; ++pr, h = (h + 1) & mask) {
+      unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(P.mkeys + h);
+      if (k == kMidEmpty) k = atomicCAS(reinterpret_cast<unsigned long long*>(P.mkeys + h), kMidEmpty, key);
+      if (k == key || k == kMidEmpty) {
+        atomicAdd(P.mcnt + h * kMidStripes + ((blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1)),
+                  static_cast<uint32_t>(__popc(grp)));
+        done = true;
+        break;
+      }
+    }
+    if (!done) {   // table too full: counted, the batch is replayed with a larger table (D7)
+      atomicOr(&P.st->err, kErrMidTable);
+      atomicAdd(&P.st->mid_fail, 1ULL);
+    }
+  }
+  const uint32_t mm = P.mkeys ? 0u : __ballot_sync(kFull, mid), mh = __ballot_sync(kFull, in && !mid);
   if (mm) {
     const unsigned long long o = chunk_slot(&P.st->pair_cursor_c, lo.mid_base, lo.mid_left, mm);
     if (mid && o < P.cap_c) P.ohc[o] = key;
@@ -2286,6 +2312,9 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.wc_bal = map_wc_balanced();
   P.wc_fast = 1;
   P.xtab = (W == kWC && P.comb && map_wc_table_ok(a.flags)) ? a.out.xtab : nullptr;
+  P.mkeys = P.xtab ? a.out.mkeys : nullptr;
+  P.mcnt = P.xtab ? a.out.mcnt : nullptr;
+  P.mbits = a.out.mbits;
   if (W == kKM && P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>(std::min<uint64_t>((a.tb_cap + 255) / 256 + 1, 8ULL * num_sms));

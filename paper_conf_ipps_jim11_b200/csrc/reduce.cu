@@ -420,23 +420,37 @@ __global__ void k_comb_merge(const uint64_t* __restrict__ segp, uint64_t nsegp, 
                              uint32_t* midx, uint64_t* psum, uint32_t* xkeys, uint64_t* xcounts,
                              unsigned long long* nextra) {   // nextra[1]: words absorbed (sum of counts)
   const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
-  if (s >= nsegp) return;
-  const uint64_t a = segp[s], b = segp[s + 1];
-  const uint32_t key = static_cast<uint32_t>(skp[a] & 0x3FFFFFFFULL);
+  const bool live = s < nsegp;
   uint64_t sum = 0;
-  for (uint64_t i = a; i < b; ++i) sum += skp[i] >> 32;
-  atomicAdd(nextra + 1, static_cast<unsigned long long>(sum));
-  uint64_t lo = 0, hi = nsega;   // first exact segment with key >= `key`
-  while (lo < hi) {
-    const uint64_t mid = (lo + hi) >> 1;
-    if (skx[sega[mid]] < key) lo = mid + 1; else hi = mid;
+  uint32_t key = 0;
+  bool extra = false;
+  if (live) {
+    const uint64_t a = segp[s], b = segp[s + 1];
+    key = static_cast<uint32_t>(skp[a] & 0x3FFFFFFFULL);
+    for (uint64_t i = a; i < b; ++i) sum += skp[i] >> 32;
+    uint64_t lo = 0, hi = nsega;   // first exact segment with key >= `key`
+    while (lo < hi) {
+      const uint64_t mid = (lo + hi) >> 1;
+      if (skx[sega[mid]] < key) lo = mid + 1; else hi = mid;
+    }
+    if (lo < nsega && skx[sega[lo]] == key) {
+      midx[s] = static_cast<uint32_t>(lo);
+      psum[s] = sum;
+    } else {
+      midx[s] = 0xFFFFFFFFu;
+      extra = true;
+    }
   }
-  if (lo < nsega && skx[sega[lo]] == key) {
-    midx[s] = static_cast<uint32_t>(lo);
-    psum[s] = sum;
-  } else {
-    midx[s] = 0xFFFFFFFFu;
-    const unsigned long long e = atomicAdd(nextra, 1ULL);
+  // warp-aggregated global atomics (per-thread ones serialised on these two addresses)
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t wsum = warp_inclusive_add64(sum);
+  const uint32_t me = __ballot_sync(0xffffffffu, extra);
+  unsigned long long base = 0;
+  if (lane == 31 && wsum) atomicAdd(nextra + 1, static_cast<unsigned long long>(wsum));   // (the warp's total)
+  if (lane == 0 && me) base = atomicAdd(nextra, static_cast<unsigned long long>(__popc(me)));
+  base = __shfl_sync(0xffffffffu, base, 0);
+  if (extra) {
+    const unsigned long long e = base + __popc(me & lanemask_lt());
     xkeys[e] = key;
     xcounts[e] = sum;
   }
@@ -635,13 +649,15 @@ cudaError_t launch_comb_add(const uint32_t* midx, const uint64_t* psum, uint64_t
 // nonzero entries are sparse: a warp ballot skips empty steps); a warp's nonzero entries take one
 // global atomic for their output slots; written entries are zeroed, so the table is clean for the
 // next Map.
+template <bool kList>
 __global__ void __launch_bounds__(256) k_xtab_extract(uint32_t* __restrict__ tab, uint64_t nv4, uint64_t* out,
-                                                    uint64_t cap, unsigned long long* cursor) {
+                                                    uint32_t* okeys, uint64_t* ocounts, uint64_t cap,
+                                                    unsigned long long* cursor, unsigned long long* wsum) {
   const uint32_t lane = threadIdx.x & 31;
   const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
   uint4* t4 = reinterpret_cast<uint4*>(tab);
-  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i - threadIdx.x % 32 < nv4;
-       i += stride) {
+  uint64_t csum = 0;
+  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i - lane < nv4; i += stride) {
     uint4 v = i < nv4 ? __ldcs(t4 + i) : make_uint4(0, 0, 0, 0);
     const uint32_t nz = (v.x != 0) + (v.y != 0) + (v.z != 0) + (v.w != 0);
     if (!__any_sync(0xffffffffu, nz != 0)) continue;
@@ -656,7 +672,13 @@ __global__ void __launch_bounds__(256) k_xtab_extract(uint32_t* __restrict__ tab
     for (int q = 0; q < 4; ++q) {
       if (!c[q]) continue;
       if (o < cap) {
-        out[o] = (4 * i + q) | (static_cast<uint64_t>(c[q]) << 32);
+        if constexpr (kList) {
+          okeys[o] = static_cast<uint32_t>(4 * i + q);
+          ocounts[o] = c[q];
+          csum += c[q];
+        } else {
+          out[o] = (4 * i + q) | (static_cast<uint64_t>(c[q]) << 32);
+        }
         c[q] = 0;
         wrote = true;
       }
@@ -664,13 +686,67 @@ __global__ void __launch_bounds__(256) k_xtab_extract(uint32_t* __restrict__ tab
     }
     if (wrote) t4[i] = make_uint4(c[0], c[1], c[2], c[3]);   // (entries past cap stay for the next call)
   }
+  if constexpr (kList) {
+    const uint64_t w = warp_inclusive_add64(csum);
+    if (lane == 31 && w) atomicAdd(wsum, static_cast<unsigned long long>(w));
+  }
 }
 
 cudaError_t launch_xtab_extract(uint32_t* tab, uint64_t nent, uint64_t* out, uint64_t cap, unsigned long long* cursor,
                                 int num_sms, cudaStream_t s) {
   const uint64_t nv4 = nent / 4;
-  k_xtab_extract<<<static_cast<unsigned>(std::min<uint64_t>(8ULL * num_sms, (nv4 + 255) / 256)), 256, 0, s>>>(
-      tab, nv4, out, cap, cursor);
+  k_xtab_extract<false><<<static_cast<unsigned>(std::min<uint64_t>(8ULL * num_sms, (nv4 + 255) / 256)), 256, 0, s>>>(
+      tab, nv4, out, nullptr, nullptr, cap, cursor, nullptr);
+  count_launch();
+  return cudaGetLastError();
+}
+cudaError_t launch_xtab_extract_list(uint32_t* tab, uint64_t nent, uint32_t* okeys, uint64_t* ocounts, uint64_t cap,
+                                     unsigned long long* cursor, unsigned long long* wsum, int num_sms, cudaStream_t s) {
+  const uint64_t nv4 = nent / 4;
+  k_xtab_extract<true><<<static_cast<unsigned>(std::min<uint64_t>(8ULL * num_sms, (nv4 + 255) / 256)), 256, 0, s>>>(
+      tab, nv4, nullptr, okeys, ocounts, cap, cursor, wsum);
+  count_launch();
+  return cudaGetLastError();
+}
+
+// WC mid table -> (key, count) lists.  Each key sits in exactly one slot (the Map's inserts find an
+// existing key before any empty slot), so the lists are the final mid keys; slots past `cap` stay.
+__global__ void __launch_bounds__(256) k_mtab_extract(uint64_t* __restrict__ mkeys, uint32_t* __restrict__ mcnt,
+                                                    uint64_t nslots, uint64_t* okeys, uint64_t* ocounts,
+                                                    uint64_t cap, unsigned long long* cursor,
+                                                    unsigned long long* wsum) {
+  const uint32_t lane = threadIdx.x & 31;
+  uint64_t csum = 0;
+  const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
+  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i - lane < nslots; i += stride) {
+    const uint64_t k = i < nslots ? mkeys[i] : kMidEmpty;
+    const bool full = k != kMidEmpty;
+    const uint32_t m = __ballot_sync(0xffffffffu, full);
+    if (!m) continue;
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(cursor, static_cast<unsigned long long>(__popc(m)));
+    base = __shfl_sync(0xffffffffu, base, 0);
+    const uint64_t o = base + __popc(m & lanemask_lt());
+    if (full && o < cap) {
+      uint64_t c = 0;
+#pragma unroll
+      for (uint32_t q = 0; q < kMidStripes; ++q) c += mcnt[i * kMidStripes + q];
+      okeys[o] = k;
+      ocounts[o] = c;
+      csum += c;
+      mkeys[i] = kMidEmpty;
+      for (uint32_t q = 0; q < kMidStripes; ++q) mcnt[i * kMidStripes + q] = 0;
+    }
+  }
+  const uint64_t w = warp_inclusive_add64(csum);
+  if (lane == 31 && w) atomicAdd(wsum, static_cast<unsigned long long>(w));
+}
+
+cudaError_t launch_mtab_extract(uint64_t* mkeys, uint32_t* mcnt, uint64_t nslots, uint64_t* okeys, uint64_t* ocounts,
+                                uint64_t cap, unsigned long long* cursor, unsigned long long* wsum, int num_sms,
+                                cudaStream_t s) {
+  k_mtab_extract<<<static_cast<unsigned>(std::min<uint64_t>(8ULL * num_sms, (nslots + 255) / 256)), 256, 0, s>>>(
+      mkeys, mcnt, nslots, okeys, ocounts, cap, cursor, wsum);
   count_launch();
   return cudaGetLastError();
 }

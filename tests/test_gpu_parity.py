@@ -146,7 +146,8 @@ def test_wc_map_combiner_on_and_off():
     off, st_off = same("wc", b, gkw={"flags": bmr.FLAG_NO_MAP_COMBINE})
     assert on == off
     assert st_off["words_combined"] == 0 and st_off["pairs_partial"] == 0
-    assert st_on["words_combined"] > st_on["pairs"] // 4 and st_on["pairs_partial"] > 0
+    # (with the L2 tables every exact and mid word is counted there: words_combined, no partial pairs)
+    assert st_on["words_combined"] > st_on["pairs"] // 4
     assert st_on["pairs"] + st_on["words_combined"] == st_off["pairs"]
 
 
@@ -247,11 +248,21 @@ def test_wc_exact_and_hashed_streams():
 
 
 def test_wc_hashed_stream_replay():
-    # every word is longer than 7 bytes: the whole Map output is the hashed stream
-    recs = [b" ".join(b"w%07d" % (i * 7 + j) for j in range(5)) for i in range(4000)]
+    # every word is longer than 8 bytes: the whole Map output is the hashed stream
+    recs = [b" ".join(b"w%08d" % (i * 7 + j) for j in range(5)) for i in range(4000)]
     data, off = make_records(recs)
     got, st = same("wc", [(data, off, len(recs))], gkw={"max_pairs_hint": 1000})
     assert st["replays"] >= 1 and len(got) == 20000
+
+
+def test_wc_mid_table_growth_replay():
+    # 400k distinct 7-symbol words (mid keys) twice each: more than the first mid table holds
+    # within its probe bound -> the Map flags it, the table grows 4x and the batch is replayed
+    words = [b"m%06d" % i for i in range(400_000)]
+    recs = [b" ".join(words[i:i + 8]) for i in range(0, len(words), 8)] * 2
+    data, off = make_records(recs)
+    got, st = same("wc", [(data, off, len(recs))])
+    assert st["replays"] >= 1 and len(got) == 400_000 and set(got.values()) == {2}
 
 
 def test_wc_multibatch():
