@@ -646,7 +646,6 @@ namespace {
 mr_status ingest_impl(mr_job* job, const void* entries, const void* heap, const uint64_t* recv_counts, uint32_t R);
 mr_status fold(mr_job* job);
 mr_status fold_finish(mr_job* job);
-mr_status xtab_extract(mr_job* job, uint64_t* mp);
 mr_status tables_extract(mr_job* job);
 cudaError_t clear_tables(mr_job* job);
 }
@@ -823,7 +822,6 @@ mr_status tables_extract(mr_job* job) {
     if (t > cap2) return fail(job, MR_ERR_OOM, "table extraction still overflows");
   }
   job->n_extra = t;
-  uint64_t words = job->st_h.p->words_comb;
   // mid table
   CK(cudaMemsetAsync(cur, 0, sizeof(unsigned long long), s), "memset cursor");
   if (job->mkeys_out.n < 4096) { CK(job->mkeys_out.ensure(1 << 18), "alloc mid keys"); CK(job->mcounts.ensure(1 << 18), "alloc mid counts"); }
@@ -848,7 +846,6 @@ mr_status tables_extract(mr_job* job) {
   }
   job->nseg_c = t;
   job->stats.words_combined = job->st_h.p->words_comb;   // exact + mid words counted by the tables
-  (void)words;
   CK(job->seg_startx.ensure(t + 2), "alloc mid segments");
   CK(launch_iota_scaled(t, 1, job->seg_startx.p, s), "mid segments");   // one segment per mid key
   job->segc = job->seg_startx.p;
@@ -859,32 +856,6 @@ mr_status tables_extract(mr_job* job) {
   return MR_OK;
 }
 
-// WC two-level combiner: the L2 count table -> combiner partial entries in hp (the same format
-// the SMEM table flush writes), so the partials' group-by, the exchange and the fold treat them
-// as before.  *mp = the number of distinct exact keys.  Leaves the table zeroed.  Synchronises.
-mr_status xtab_extract(mr_job* job, uint64_t* mp) {
-  cudaStream_t s = job->stream;
-  unsigned long long* cur = &job->st->n_extra;   // (scratch: n_extra is reset before its own use)
-  CK(cudaMemsetAsync(cur, 0, sizeof(unsigned long long), s), "memset cursor");
-  CK(launch_xtab_extract(job->xtab.p, job->xtab.n, job->hp.p, job->cap_p, cur, job->nsm, s), "table extract");
-  CK(read_state(job), "sync table extract");
-  uint64_t t = job->st_h.p->n_extra;
-  if (t > job->cap_p) {   // more distinct keys than partial capacity: grow (keeping the written ones), continue
-    const uint64_t done = job->cap_p;
-    CK(grow_keep(job->hp, done, t + t / 8 + 4096, s), "grow partials");
-    job->cap_p = job->hp.n;
-    job->tmp_h.p[4] = done;
-    CK(cudaMemcpyAsync(cur, job->tmp_h.p + 4, 8, cudaMemcpyHostToDevice, s), "set cursor");
-    CK(launch_xtab_extract(job->xtab.p, job->xtab.n, job->hp.p, job->cap_p, cur, job->nsm, s), "table extract");
-    CK(read_state(job), "sync table extract");
-    t = job->st_h.p->n_extra;
-    if (t > job->cap_p) return fail(job, MR_ERR_OOM, "table extraction still overflows");
-  }
-  CK(cudaMemsetAsync(cur, 0, sizeof(unsigned long long), s), "memset cursor");
-  job->xtab_dirty = false;
-  *mp = t;
-  return MR_OK;
-}
 
 }  // namespace
 

@@ -75,8 +75,11 @@ constexpr int kKmUnroll = BMR_KM_UNROLL;
 #define BMR_SM_SUB 4     // StringMatch 512-B windows per map-warp super-window
 #endif
 constexpr int kNMapText = 24;
+#ifndef BMR_II_NMAP
+#define BMR_II_NMAP 24   // InvertedIndex map warps
+#endif
 template <int W>
-constexpr int nmap() { return W == 3 ? kNMap : W == 2 ? BMR_SM_NMAP : kNMapText; }
+constexpr int nmap() { return W == 3 ? kNMap : W == 2 ? BMR_SM_NMAP : W == 4 ? BMR_II_NMAP : kNMapText; }
 // Producer warps kProdWarp0 .. + kNProd - 1: producer p owns the iterations it == p (mod kNProd)
 // (and so the stages s == p (mod kNProd)); one warp alone is latency-bound at ~465 instructions
 // per tile (TMA issue + bitmap), slower than HBM delivers a tile (ncu, C2 round 1).
@@ -1503,6 +1506,143 @@ __device__ void ii_drain(const Params& P, OutCtl* oc, uint8_t* outh, uint32_t& q
   qn = 0;
 }
 
+// ---------------------------------------------------------------- InvertedIndex fast path (SIO)
+// The computation of emit_text_chunk<kII> for one 512-B window, with the work done lazily: the
+// has-'<' test first (most 16-B chunks have none), the '<' positions and marker checks only in
+// lanes that have one, the '"' / record-start stop masks only when the warp found a marker, the
+// range masks only in the input's first / last window; predicated lane-0 atomics.
+__device__ __forceinline__ void ii_window(const Params& P, OutCtl* oc, uint8_t* outh, const TileView& tv,
+                                          long long p0w, uint32_t& qn) {
+  const uint32_t lane = threadIdx.x & 31;
+  const long long N = bd_nbytes();
+  const long long p0 = p0w + 16 * lane;
+  const uint32_t i0 = static_cast<uint32_t>(p0 - tv.sbase);
+  const uint4 c0 = *reinterpret_cast<const uint4*>(tv.sb + i0);
+  uint32_t a = 0;
+  {
+    const uint32_t t0 = c0.x ^ 0x3C3C3C3Cu, t1 = c0.y ^ 0x3C3C3C3Cu, t2 = c0.z ^ 0x3C3C3C3Cu, t3 = c0.w ^ 0x3C3C3C3Cu;
+    a = (((t0 - 0x01010101u) & ~t0) | ((t1 - 0x01010101u) & ~t1) | ((t2 - 0x01010101u) & ~t2) |
+         ((t3 - 0x01010101u) & ~t3)) & 0x80808080u;
+  }
+  if (!__any_sync(kFull, a != 0)) return;   // no '<' in the window: no marker (exact has-byte test)
+  const bool edge = p0w < 0 || p0w + kWin + 16 > N;   // warp-uniform
+  const uint32_t vm = edge ? range_mask32(p0, 0, N) : kFull;
+  const uint32_t R = bits32(tv.bm, i0);
+  const uint4 c1 = *reinterpret_cast<const uint4*>(tv.sb + i0 + 16);
+  const uint32_t x[8] = {c0.x, c0.y, c0.z, c0.w, c1.x, c1.y, c1.z, c1.w};
+  uint32_t mk = 0;
+  if (a) {   // markers of this lane's chunk (rare lanes)
+    uint32_t cand = (eq_mask4(x[0], 0x3C3C3C3Cu) | (eq_mask4(x[1], 0x3C3C3C3Cu) << 4) |
+                     (eq_mask4(x[2], 0x3C3C3C3Cu) << 8) | (eq_mask4(x[3], 0x3C3C3C3Cu) << 12)) & vm & 0xFFFFu;
+    while (cand) {
+      const uint32_t j = __ffs(cand) - 1;
+      cand &= cand - 1;
+      if (p0 + j + 9 > N) continue;
+      if ((R >> (j + 1)) & 0xFFu) continue;               // marker inside one record
+      uint32_t w[4];
+      window16(x, j, w);
+      // "<a href=\"" little-endian: 3C 61 20 68 | 72 65 66 3D | 22
+      if (w[0] != 0x6820613Cu || w[1] != 0x3D666572u || (w[2] & 0xFFu) != 0x22u) continue;
+      mk |= 1u << j;
+    }
+  }
+  if (!__any_sync(kFull, mk != 0)) return;
+  // the URL of a marker ends at the first '"' unless a record starts first (C-3 #9): every lane
+  // publishes its 16-bit stop mask and a marker finds the first stop after its URL start with two
+  // shuffles; only URLs leaving the window scan onwards
+  const uint32_t qm = eq_mask4(x[0], 0x22222222u) | (eq_mask4(x[1], 0x22222222u) << 4) |
+                      (eq_mask4(x[2], 0x22222222u) << 8) | (eq_mask4(x[3], 0x22222222u) << 12);
+  const uint32_t st16 = ((qm & vm) | R) & 0xFFFFu;
+  const uint32_t lanes_st = __ballot_sync(kFull, st16 != 0);
+  const uint32_t r16 = R & 0xFFFFu;
+  uint32_t emit_mask = 0, aux[2] = {0, 0};
+  int nm = 0;
+  for (int mi = 0; mi < 2; ++mi) {          // a 9-byte marker: at most two start in 16 bytes
+    if (!__any_sync(kFull, mk != 0)) break;
+    const bool has = mk != 0;
+    const uint32_t j = has ? static_cast<uint32_t>(__ffs(mk) - 1) : 0u;
+    if (has) mk &= mk - 1;
+    const uint32_t au = lane * 16 + j + 9;   // window offset of the URL start
+    const uint32_t T = min(au >> 4, 31u);
+    const uint32_t sT = __shfl_sync(kFull, st16, T), rT = __shfl_sync(kFull, r16, T);
+    const uint32_t cT = au < static_cast<uint32_t>(kWin) ? (sT >> (au & 15u)) << (au & 15u) : 0u;
+    const uint32_t later = T < 31 ? (lanes_st & ~((2u << T) - 1u)) : 0u;
+    const uint32_t F = later ? static_cast<uint32_t>(__ffs(later) - 1) : 31u;
+    const uint32_t sF = __shfl_sync(kFull, st16, F), rF = __shfl_sync(kFull, r16, F);
+    if (!has) continue;
+    const long long q0 = p0 + j + 9;
+    long long q;
+    if (cT) {
+      const uint32_t b = __ffs(cT) - 1;
+      q = ((rT >> b) & 1u) ? -1 : p0w + T * 16 + b;     // record ends first -> unclosed
+    } else if (later && au < static_cast<uint32_t>(kWin)) {
+      const uint32_t b = __ffs(sF) - 1;
+      q = ((rF >> b) & 1u) ? -1 : p0w + F * 16 + b;
+    } else {                                           // no stop in the window: scan onwards
+      q = find_quote(P, tv, max(q0, p0w + kWin), p0 + j);
+    }
+    if (q > q0 && nm < 2) {
+      aux[nm++] = static_cast<uint32_t>(q - q0);
+      emit_mask |= 1u << j;
+    }
+  }
+  // queue the URLs (drained lane-parallel by ii_drain)
+  const uint32_t cnt = __popc(emit_mask);   // <= 2 markers start in 16 bytes
+  const uint32_t incl = warp_inclusive_add(cnt);
+  const uint32_t tot = __shfl_sync(kFull, incl, 31);
+  if (tot == 0) return;
+  if (qn + tot > 64) ii_drain(P, oc, outh, qn);
+  uint64_t* qpos = ii_qpos(outh);
+  uint32_t* qlen = reinterpret_cast<uint32_t*>(qpos + 64);
+  uint32_t k = qn + incl - cnt;
+  int nth = 0;
+  for (uint32_t m = emit_mask; m; m &= m - 1) {
+    const uint32_t j = __ffs(m) - 1;
+    uint32_t len = nth == 0 ? aux[0] : aux[1];
+    ++nth;
+    if (len > 0xFFFFu) { atomicOr(&P.st->err, kErrKeyTooLong); len = 0xFFFFu; }
+    qpos[k] = static_cast<uint64_t>(p0 + j + 9);
+    qlen[k] = len;
+    ++k;
+  }
+  qn += tot;
+  if (qn >= 32) ii_drain(P, oc, outh, qn);
+}
+
+__device__ __forceinline__ void ii_map_loop(const Params& P, uint8_t* smem, OutCtl* oc, uint32_t& qn) {
+  constexpr int W = kII;
+  constexpr int kStages = Cfg<W>::kStages;
+  uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
+  uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout<W>::ready);
+  uint8_t* outh = smem + Layout<W>::out;
+  uint32_t have_it = ~0u;
+  long long t = 0, sbase = 0, hi = 0, stg_hi = 0;
+  for (;;) {
+    const uint32_t g = lane0_atom_add_shared(&oc->win_next, 1u);
+    const uint32_t it = g / kNWin, w = g % kNWin;
+    const uint32_t s = it % kStages;
+    if (it != have_it) {
+      map_wait(P, ready + s, (it / kStages) & 1u, kReadyWaitNs);
+      const StageHdr* hd = reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
+      t = hd->t;
+      sbase = hd->sbase;
+      hi = hd->hi;
+      stg_hi = hd->stg_hi;
+      have_it = it;
+    }
+    if (t < 0) break;
+    const long long wp = sbase + kLead + static_cast<long long>(w) * kWin;
+    if (wp < hi) {   // warp-uniform
+      const TileView tv{smem + Layout<W>::bytes + s * kStageBytes,
+                        reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits), sbase, stg_hi, 0,
+                        0};
+      ii_window(P, oc, outh, tv, wp, qn);
+    }
+    __syncwarp();
+    lane0_mbar_arrive(&empty[s]);
+  }
+}
+
 template <int W>
 __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, const TileView& tv,
                                 long long p0, long long i0, bool live, uint32_t& qn) {
@@ -1975,6 +2115,10 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
     fast = !P.so && !P.si && P.wc_bal && P.dyn && P.wc_fast;
     if (fast) wc_map_loop(P, smem, oc);
   }
+  if constexpr (W == kII) {
+    fast = !P.so && !P.si && P.dyn && P.wc_fast;
+    if (fast) ii_map_loop(P, smem, oc, qn);
+  }
   for (uint32_t it = 0; !fast; ++it) {
     uint32_t w = 0;
     if constexpr (W != kKM) {
@@ -2319,7 +2463,7 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.si = (a.flags & 2u) ? 1u : 0u;   // MR_FLAG_NO_SMEM_OUT
   P.sm_lines = (W == kSM && (a.flags & 0x200u)) ? 1u : 0u;   // MR_FLAG_SM_LINES
   P.wc_bal = map_wc_balanced();
-  P.wc_fast = 1;
+  P.wc_fast = map_fast_path() ? 1u : 0u;
   P.xtab = (W == kWC && P.comb && map_wc_table_ok(a.flags)) ? a.out.xtab : nullptr;
   P.mkeys = P.xtab ? a.out.mkeys : nullptr;
   P.mcnt = P.xtab ? a.out.mcnt : nullptr;
@@ -2388,7 +2532,17 @@ uint32_t map_wc_balanced() {
 // The WordCount L2 count table is fed by the SIO fast path only (wc_window); the memory-mode
 // ablations and the lane-serial emission keep the exact stream
 bool map_wc_table_ok(uint32_t flags) {
-  return !(flags & 3u) && map_wc_balanced() && map_dyn_windows(kWC);
+  return !(flags & 3u) && map_wc_balanced() && map_dyn_windows(kWC) && map_fast_path();
+}
+
+// WordCount / InvertedIndex SIO fast paths (wc_window / ii_window); BMR_MAP_FAST=0 selects the
+// generic per-window path for A/B measurements (same results)
+bool map_fast_path() {
+  static const bool v = [] {
+    const char* e = getenv("BMR_MAP_FAST");
+    return e ? atoi(e) != 0 : true;
+  }();
+  return v;
 }
 
 int vbytes_of(int w) { return w == kKM ? 32 : w == kII ? 8 : 0; }
