@@ -400,7 +400,7 @@ def main():
     acc = {k: 0.0 for k in ("map_ms", "hist_ms", "sort_ms", "seg_ms", "sort_keys_ms", "xchg_ms")}
     tot = {"pairs": 0, "sort_passes": 0, "kernel_launches": 0, "flushes": 0, "n_keys": 0, "pairs_hashed": 0,
            "sort_passes_keys": 0, "pairs_mid": 0, "sort_passes_mid": 0, "words_combined": 0, "pairs_partial": 0,
-           "collisions": 0, "xchg_send_bytes": 0, "replays": 0}
+           "collisions": 0, "xchg_send_bytes": 0, "replays": 0, "map_seal_waits": 0, "map_spills": 0}
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         barrier()
@@ -569,6 +569,8 @@ def main():
             "distinct_keys": int(tot["n_keys"] / args.steps),
             "hash_collisions_per_step": tot["collisions"] / args.steps,
             "replays": tot["replays"],
+            "map_output_ring": {"seal_waits_per_step": tot["map_seal_waits"] / args.steps,
+                                "spills_per_step": tot["map_spills"] / args.steps},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
             "exchange": ({"kind": ("libbmr mr_group over NCCL (" + bmr.Comm.backend() + ")") if args.xchg == "nccl"
                           else "torch.distributed all_to_all_single (NCCL) of libbmr's partition buffers",

@@ -56,6 +56,9 @@ typedef enum { MR_WORDCOUNT = 1, MR_STRINGMATCH = 2, MR_KMEANS = 3, MR_INVINDEX 
 #define MR_FLAG_NO_MAP_COMBINE  0x100u /* WC: no in-SMEM combiner in the Map (every word is emitted as a pair) */
 #define MR_FLAG_SM_LINES        0x200u /* SM: the paper's per-line output (L125): the global offset of every
                                           record containing the pattern, once (grouped by key) */
+#define MR_FLAG_FORCE_SPILL     0x800u /* test hook: every warp result that overflows the output buffer is
+                                          written straight to HBM (the a5 spill path), not only while the
+                                          buffer ring is congested */
 #define MR_FLAG_BATCH_COMBINE   0x400u /* WC: each mapped batch is grouped + reduced (combined) when the next
                                           one is mapped — mr_map then synchronises — and its (key, count)
                                           partials kept; mr_group merges the partials (exact sums).  For
@@ -126,6 +129,10 @@ typedef struct {
   uint64_t xchg_send_bytes;
   uint64_t xchg_recv_bytes;
   double xchg_ms;
+  /* Map output ring (L113, §8(a) a5): seals that found every buffer still flushing, and the warp
+   * results written straight to HBM (the overflow spill) while the sealer waited */
+  uint64_t map_seal_waits;
+  uint64_t map_spills;
 } mr_stats;
 
 /* State machine: CREATED -> mr_map x k (batches append) -> mr_group -> mr_reduce -> mr_fetch

@@ -36,6 +36,8 @@ struct DevState {
   unsigned long long words_comb;     // WC: words absorbed by the combiners (sum of partial counts)
   unsigned long long pads_b, pads_c; // WC hashed / mid stream: sentinel entries in unused chunk tails
   unsigned long long mid_fail;       // WC mid table: inserts that found no slot (-> grow + replay)
+  unsigned long long seal_waits;     // Map: seals that waited for a buffer still flushing (ring full)
+  unsigned long long spills;         // Map: warp results written straight to HBM while the ring was full
 };
 constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u, kErrTileCap = 4u, kErrNullRecords = 8u,
                        kErrMidTable = 16u;

@@ -75,6 +75,13 @@ constexpr int kKmUnroll = BMR_KM_UNROLL;
 #define BMR_SM_SUB 4     // StringMatch 512-B windows per map-warp super-window
 #endif
 constexpr int kNMapText = 24;
+#ifndef BMR_II_STAGES
+#define BMR_II_STAGES 6    // InvertedIndex stages in flight per SM (round 2: 4 -> 6 with 8 KB output
+                           // buffers, C4 Map 7.81 -> 7.66 ms)
+#endif
+#ifndef BMR_II_OUT_BYTES
+#define BMR_II_OUT_BYTES 8192   // InvertedIndex output buffer bytes (x kNOut; 24-B pairs, ~1 per 500 B)
+#endif
 #ifndef BMR_II_NMAP
 #define BMR_II_NMAP 24   // InvertedIndex map warps
 #endif
@@ -115,7 +122,7 @@ template <int W>
 struct Cfg {
   // StringMatch (read-bound, almost no output, lazy record directory below: no offsets or bitmap
   // regions): 8 stages of bytes in flight
-  static constexpr int kStages = (W == kSM) ? BMR_SM_STAGES : 4;
+  static constexpr int kStages = (W == kSM) ? BMR_SM_STAGES : (W == kII) ? BMR_II_STAGES : 4;
   static constexpr int kOffCap = (W == kSM) ? 0 : (W == kWC) ? BMR_WC_OFFCAP : 1024;   // record offsets staged per tile (more: read from global)
   // StringMatch reads the record directory lazily: record boundaries matter only where the
   // pattern's first byte matches (planted, rare), so no offsets are staged and no bitmap is built;
@@ -124,7 +131,7 @@ struct Cfg {
   static constexpr bool kLazyDir = (W == kSM);
   static constexpr int kOffBytes = (W == kSM) ? 0 : ((kOffCap + 2) * 8 + 127) / 128 * 128;
   static constexpr int kBits = (W == kSM) ? 0 : kBitBytes;   // record-start bitmap bytes per stage
-  static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? BMR_WC_OUT_BYTES : 20480;   // bytes per output buffer
+  static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? BMR_WC_OUT_BYTES : (W == kII) ? BMR_II_OUT_BYTES : 20480;   // bytes per output buffer
   // the producer builds the bitmap of tile it - kLag right after issuing tile it: kLag stages of
   // TMA traffic stay in flight per SM while one stage is being consumed
   static constexpr int kLag = kStages - 2;
@@ -186,6 +193,7 @@ struct OutCtl {
   unsigned long long fbase[kNOut];   // global base reserved for the sealed buffer (one atomic per flush)
   unsigned int nsealed, is_final;  // sealed generations so far (full count); final flush flag
   unsigned int win_next;         // text: next window (tile * kNWin + window) to hand to a map warp
+  unsigned int congested;        // the sealing warp waits for a flushing buffer: overflowing warps spill
   uint64_t req[kNOut];           // mbarrier: buffer sealed -> flush warp
   uint64_t done[kNOut];          // mbarrier: buffer flushed -> free
 };
@@ -558,7 +566,12 @@ __device__ void seal(const Params& P, OutCtl* oc, uint32_t gen8, uint32_t h, uin
   if (!last) {
     if (full_gen + 1 >= kNOut) {                               // next buffer last used by gen q
       const uint32_t q = full_gen + 1 - kNOut;
-      mbar_wait(&oc->done[q % kNOut], (q / kNOut) & 1u);
+      if (!mbar_try_wait(&oc->done[q % kNOut], (q / kNOut) & 1u)) {   // every buffer still flushing
+        atomicAdd(&P.st->seal_waits, 1ULL);
+        st_release_cta_shared_u32(&oc->congested, 1u);         // overflowing warps spill meanwhile
+        mbar_wait(&oc->done[q % kNOut], (q / kNOut) & 1u);
+        st_release_cta_shared_u32(&oc->congested, 0u);
+      }
     }
     oc->committed[(h + 1) % kNOut] = 0;
     oc->nsealed = full_gen + 1;
@@ -572,9 +585,14 @@ __device__ void seal(const Params& P, OutCtl* oc, uint32_t gen8, uint32_t h, uin
   __threadfence_block();
   mbar_arrive(&oc->req[h]);
 }
-// cnt: packed counts (cb << 14 | ca); cap: buffer capacity in units
+// cnt: packed counts (cb << 14 | ca); cap: buffer capacity in units.  spill_ok: the caller can
+// write its result straight to HBM (§8(a) a5 overflow spill): an overflowing warp that is not the
+// sealer then returns kSpill instead of waiting while the ring is congested (the sealer waits for
+// a flushing buffer).
+constexpr uint32_t kSpill = 0xFFFFFFFFu;
 template <int W>
-__device__ __forceinline__ Slot reserve(const Params& P, OutCtl* oc, uint8_t* outh, uint32_t cnt, uint32_t cap) {
+__device__ __forceinline__ Slot reserve(const Params& P, OutCtl* oc, uint8_t* outh, uint32_t cnt, uint32_t cap,
+                                        bool spill_ok = false) {
   const uint32_t lane = threadIdx.x & 31;
   for (;;) {
     uint32_t old = 0;
@@ -584,15 +602,29 @@ __device__ __forceinline__ Slot reserve(const Params& P, OutCtl* oc, uint8_t* ou
     const uint32_t h = gen % kNOut;
     const uint32_t u0 = units<W>(base);
     if (u0 + units<W>(cnt) <= cap) return {h, base};
+    uint32_t spill = 0;
+    const bool force = spill_ok && (P.flags & 0x800u);   // MR_FLAG_FORCE_SPILL (tests)
     if (lane == 0) {
       if (u0 <= cap) {
         // This warp crossed the capacity first (units grow monotonically within a generation):
         // it seals half h (L113 "overflow handling").
         seal<W>(P, oc, gen, h, base, false);
+        if (force) {
+          spill = 1;
+          atomicAdd(&P.st->spills, 1ULL);
+        }
       } else {
-        while (cur_gen(ld_acquire_cta_shared_u32(&oc->cur)) == gen) __nanosleep(128);
+        while (cur_gen(ld_acquire_cta_shared_u32(&oc->cur)) == gen) {
+          if (spill_ok && (force || ld_acquire_cta_shared_u32(&oc->congested))) {
+            spill = 1;
+            atomicAdd(&P.st->spills, 1ULL);
+            break;
+          }
+          __nanosleep(128);
+        }
       }
     }
+    if (__shfl_sync(kFull, spill, 0)) return {kSpill, 0};
     __syncwarp();
   }
 }
@@ -1333,12 +1365,24 @@ __device__ __forceinline__ void wc_window(const Params& P, OutCtl* oc, uint8_t* 
   }
   // exact keys that missed (exact-stream mode: no L2 table): one reservation, copied out
   if (nx) {
-    const Slot slot = reserve<kWC>(P, oc, outh, nx, P.out_cap);
-    uint32_t* sh = reinterpret_cast<uint32_t*>(outh + slot.half * Cfg<kWC>::kOutHalf);
-    const uint32_t ka = cur_ca(slot.base);
+    const Slot slot = reserve<kWC>(P, oc, outh, nx, P.out_cap, true);
     __syncwarp();
-    for (uint32_t i = lane; i < nx; i += 32) sh[ka + i] = xq[i];
-    commit(oc, slot, nx);
+    if (slot.half == kSpill) {   // ring congested: straight to HBM, padded to 4 keys like a flush
+      const uint32_t r = (nx + 3u) & ~3u;
+      unsigned long long gb = 0;
+      if (lane == 0) {
+        gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(r));
+        if (r > nx) atomicAdd(&P.st->pads, static_cast<unsigned long long>(r - nx));
+      }
+      gb = __shfl_sync(kFull, gb, 0);
+      for (uint32_t i = lane; i < r; i += 32)
+        if (gb + i < P.cap_pairs) P.ohx[gb + i] = i < nx ? xq[i] : 0xFFFFFFFFu;
+    } else {
+      uint32_t* sh = reinterpret_cast<uint32_t*>(outh + slot.half * Cfg<kWC>::kOutHalf);
+      const uint32_t ka = cur_ca(slot.base);
+      for (uint32_t i = lane; i < nx; i += 32) sh[ka + i] = xq[i];
+      commit(oc, slot, nx);
+    }
   }
   // long words: their bytes into the warp's cross-window queue (keyed 32 at a time by wc_drain);
   // words longer than kLQMaxLen bytes (rare) are keyed here, one lane each
@@ -1488,12 +1532,38 @@ __device__ void ii_drain(const Params& P, OutCtl* oc, uint8_t* outh, uint32_t& q
     qn = 0;
     return;
   }
-  const Slot slot = reserve<kII>(P, oc, outh, qn, P.out_cap);
+  const Slot slot = reserve<kII>(P, oc, outh, qn, P.out_cap, true);
+  const TileView gv{nullptr, nullptr, 0, LLONG_MIN, 0, 0};   // key bytes from global memory
+  if (slot.half == kSpill) {   // ring congested: straight to HBM, padded to 4 pairs like a flush
+    const uint32_t r = (qn + 3u) & ~3u;
+    unsigned long long gb = 0;
+    if (lane == 0) {
+      gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(r));
+      if (r > qn) atomicAdd(&P.st->pads, static_cast<unsigned long long>(r - qn));
+    }
+    gb = __shfl_sync(kFull, gb, 0);
+    for (uint32_t e = lane; e < r; e += 32) {
+      if (gb + e >= P.cap_pairs) continue;
+      if (e < qn) {
+        const long long q0 = static_cast<long long>(qpos[e]);
+        const uint32_t len = qlen[e];
+        P.oh[gb + e] = key_at(P, gv, q0, len);
+        P.okref[gb + e] = (reinterpret_cast<uint64_t>(P.rec + q0) << 16) | len;
+        reinterpret_cast<uint64_t*>(P.ov)[gb + e] = bd_gbase() + static_cast<uint64_t>(q0);
+      } else {
+        P.oh[gb + e] = sentinel_key<kII>(P);
+        P.okref[gb + e] = 0;
+        reinterpret_cast<uint64_t*>(P.ov)[gb + e] = 0;
+      }
+    }
+    __syncwarp();
+    qn = 0;
+    return;
+  }
   uint8_t* half = outh + slot.half * Cfg<kII>::kOutHalf;
   uint64_t* sh = reinterpret_cast<uint64_t*>(half);
   uint64_t* sk = sh + F::kCap;
   uint64_t* sv = reinterpret_cast<uint64_t*>(half + F::kCap * 16);
-  const TileView gv{nullptr, nullptr, 0, LLONG_MIN, 0, 0};   // key bytes from global memory
   for (uint32_t e = lane; e < qn; e += 32) {
     const long long q0 = static_cast<long long>(qpos[e]);
     const uint32_t len = qlen[e];
@@ -2068,7 +2138,14 @@ __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl
           if (g < P.cap_pairs) P.oh[g] = key;
         }
       } else {
-        const Slot slot = reserve<W>(P, oc, outh, 1u, P.out_cap);
+        const Slot slot = reserve<W>(P, oc, outh, 1u, P.out_cap, true);
+        if (slot.half == kSpill) {   // ring congested: straight to HBM (SM flushes need no alignment)
+          if (lane == 0) {
+            const unsigned long long g = atomicAdd(&P.st->pair_cursor, 1ULL);
+            if (g < P.cap_pairs) P.oh[g] = key;
+          }
+          continue;
+        }
         if (lane == 0) reinterpret_cast<uint64_t*>(outh + slot.half * Cfg<W>::kOutHalf)[slot.base] = key;
         commit(oc, slot, 1u);
       }
@@ -2243,16 +2320,34 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         }
       } else if (m) {
         const uint32_t total = __popc(m);
-        const Slot slot = reserve<W>(P, oc, outh, total, P.out_cap);
-        if (valid) {
-          const uint32_t idx = slot.base + __popc(m & lanemask_lt());
-          uint8_t* half = outh + slot.half * Cfg<W>::kOutHalf;
-          reinterpret_cast<uint64_t*>(half)[idx] = best;
-          float4* sv = reinterpret_cast<float4*>(half + F::kCap * 8 + static_cast<size_t>(idx) * 32);
-          sv[0] = make_float4(x[0], x[1], x[2], x[3]);
-          sv[1] = make_float4(x[4], x[5], x[6], x[7]);
+        const Slot slot = reserve<W>(P, oc, outh, total, P.out_cap, true);
+        if (slot.half == kSpill) {   // ring congested: straight to HBM, padded to 4 pairs like a flush
+          const uint32_t r = (total + 3u) & ~3u;
+          unsigned long long gb = 0;
+          if (lane == 0) {
+            gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(r));
+            if (r > total) atomicAdd(&P.st->pads, static_cast<unsigned long long>(r - total));
+          }
+          gb = __shfl_sync(kFull, gb, 0);
+          const uint32_t rk = __popc(m & lanemask_lt());
+          if (valid && gb + rk < P.cap_pairs) {
+            P.oh[gb + rk] = best;
+            float4* gv = reinterpret_cast<float4*>(P.ov + (gb + rk) * 32);
+            gv[0] = make_float4(x[0], x[1], x[2], x[3]);
+            gv[1] = make_float4(x[4], x[5], x[6], x[7]);
+          }
+          if (lane < r - total && gb + total + lane < P.cap_pairs) P.oh[gb + total + lane] = sentinel_key<W>(P);
+        } else {
+          if (valid) {
+            const uint32_t idx = slot.base + __popc(m & lanemask_lt());
+            uint8_t* half = outh + slot.half * Cfg<W>::kOutHalf;
+            reinterpret_cast<uint64_t*>(half)[idx] = best;
+            float4* sv = reinterpret_cast<float4*>(half + F::kCap * 8 + static_cast<size_t>(idx) * 32);
+            sv[0] = make_float4(x[0], x[1], x[2], x[3]);
+            sv[1] = make_float4(x[4], x[5], x[6], x[7]);
+          }
+          commit(oc, slot, total);
         }
-        commit(oc, slot, total);
       }
     } else {
       const uint32_t* bm = reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits);
@@ -2324,6 +2419,7 @@ __global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
     oc->nsealed = 0;
     oc->is_final = 0;
     oc->win_next = 0;
+    oc->congested = 0;
     for (int b = 0; b < kNOut; ++b) { mbar_init(&oc->req[b], 1); mbar_init(&oc->done[b], 1); }
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
     uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);

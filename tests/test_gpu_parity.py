@@ -302,6 +302,36 @@ def test_wc_batch_combine(flags):
             assert decode("wc", job.fetch()) == exp
 
 
+@pytest.mark.parametrize("workload", ["ii", "km", "sm"])
+def test_overflow_spill_under_forced_congestion(workload):
+    # MR_FLAG_FORCE_TINY_OUT: every warp result fills an output buffer; with MR_FLAG_FORCE_SPILL
+    # every overflowing warp result is written straight to HBM (map_spills, §8(a) a5) instead of
+    # waiting for the next buffer (the default spills only while the ring is congested) — the
+    # output must not change
+    if workload == "ii":
+        g = pygen.host_text(pygen.spec_ii(4), 6)
+        b, kw = [(g["data"], g["offsets"], g["n"])], {}
+    elif workload == "sm":
+        spec = pygen.spec_sm(260_000, 2)                 # dense plants: > 512 matches per CTA
+        g = pygen.host_text(spec, 24)
+        b, kw = [(g["data"], g["offsets"], g["n"])], {"pattern": spec.pattern}
+    else:
+        spec = pygen.KMSpec()
+        n = 32 * 20_000
+        pts = pygen.host_km(spec, n)
+        b, kw = [(pts.view(np.uint8).reshape(-1), None, n)], {"centroids": pygen.km_centres(spec)[1]}
+    okw = dict(kw)
+    flags = bmr.FLAG_FORCE_TINY_OUT | bmr.FLAG_FORCE_SPILL | (bmr.FLAG_NO_MAP_COMBINE if workload == "km" else 0)
+    if workload == "km":
+        r, st = gpu("km", b, flags=flags, **kw)
+        cen, cnt = decode("km", r)
+        co, no = decode("km", ora("km", b, **okw))
+        assert np.array_equal(cnt, no)
+    else:
+        _, st = same(workload, b, gkw=dict(flags=flags, **kw), okw=okw)
+    assert st["map_spills"] > 0, st
+
+
 # ------------------------------------------------------------------ StringMatch
 def test_sm_generator_dense_plants():
     spec = pygen.spec_sm(plant_ppm=260_000)            # paper-shaped dense variant (3.83:1)
