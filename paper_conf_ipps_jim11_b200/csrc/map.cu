@@ -95,6 +95,15 @@ constexpr int kNProd = 2;
 // warp removed the map warps' spinning on sealed buffers but cost the Map more than it saved
 // (C5 Map 20.4 -> 21.3 ms, round 2: a 28th warp lowers the register budget of every warp).
 // Warps: map 0 .. nmap-1, producers nmap .. nmap+kNProd-1, then the flush warps.
+#ifndef BMR_MID_MATCH
+#define BMR_MID_MATCH 1
+#endif
+#ifndef BMR_MID_LDCA
+#define BMR_MID_LDCA 0
+#endif
+#ifndef BMR_FLUSH_SLEEP_NS
+#define BMR_FLUSH_SLEEP_NS 0
+#endif
 #ifndef BMR_WC_NFLUSH
 #define BMR_WC_NFLUSH 1u
 #endif
@@ -667,6 +676,8 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc, uint32_t 
         past = true;
         break;
       }
+      if (BMR_FLUSH_SLEEP_NS) __nanosleep(BMR_FLUSH_SLEEP_NS);   // the flush warp has the highest scheduling
+                                                                  // priority: polling would take the map warps' slots
     }
     if (past) break;
     // (the sealing warp wrote these before its release-arrive on req[h]; the wait above acquires)
@@ -1232,13 +1243,16 @@ __device__ __forceinline__ void wc_drain(const Params& P, LOut& lo, LWord* lq, u
   if (P.mkeys) {   // mid table: equal keys of the drain aggregated (match.any), then the group's
                   // leader finds the key (or claims an empty slot) and adds the group size to its
                   // warp's stripe of the slot's count (one RED)
-    const uint32_t grp = __match_any_sync(kFull, mid ? key : kMidEmpty);
+    const uint32_t grp = BMR_MID_MATCH ? __match_any_sync(kFull, mid ? key : kMidEmpty) : (1u << lane);
     const bool lead = mid && lane == static_cast<uint32_t>(__ffs(grp) - 1);
     const uint64_t mask = (1ULL << P.mbits) - 1ULL;
     uint64_t h = mid_slot(key, P.mbits);
     bool done = !lead;
     for (uint32_t pr = 0; lead && pr < kMidProbes; ++pr, h = (h + 1) & mask) {
-      unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(P.mkeys + h);
+      // (an L1-cached read: a claimed slot never changes during the Map, and a stale empty only
+      // sends the lane to the CAS, which returns the slot's real key)
+      unsigned long long k = BMR_MID_LDCA ? __ldca(reinterpret_cast<const unsigned long long*>(P.mkeys + h))
+                                          : *reinterpret_cast<volatile unsigned long long*>(P.mkeys + h);
       if (k == kMidEmpty) k = atomicCAS(reinterpret_cast<unsigned long long*>(P.mkeys + h), kMidEmpty, key);
       if (k == key || k == kMidEmpty) {
         atomicAdd(P.mcnt + h * kMidStripes + ((blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1)),
