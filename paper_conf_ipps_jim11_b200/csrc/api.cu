@@ -340,8 +340,11 @@ struct mr_job {
   // second combiner level: exact words that miss the SMEM table go to an L2-resident count table
   // (the raw multi-GPU exchange, MR_FLAG_NO_COMBINE, keeps the literal pair streams)
   bool wc_table() const {
-    return wc_comb() && map_wc_table_ok(cfg.flags) && !(cfg.flags & MR_FLAG_NO_COMBINE);
+    return tables_on && wc_comb() && map_wc_table_ok(cfg.flags) && !(cfg.flags & MR_FLAG_NO_COMBINE);
   }
+  // per run, from the first batch's size: extracting the tables streams the 4 GiB count table
+  // (~0.7 ms), more than sorting the exact keys of a small input costs (C1: 1 MiB)
+  bool tables_on = true;
   DBuf<uint32_t> xtab;            // 2^30 u32 counts by exact key (zero between runs)
   // mid words (6..8 symbols): open-addressing table of 48-bit exact keys + counts (2^mbits slots)
   DBuf<uint64_t> mtab_keys;
@@ -1011,6 +1014,10 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
   // sizing estimate for the first batch's buffers (text of unknown length: <= 32 B per record
   // assumed; overflow is caught by the demand counters and replayed at mr_group)
   const uint64_t est = nbytes != ~0ULL ? nbytes : 32 * n;
+  if (job->batches.empty() && job->nfolds == 0 && !job->ingested) {
+    const char* tm = getenv("BMR_TABLE_MIN_BYTES");   // (tests: 0 = always the tables)
+    job->tables_on = est >= (tm ? strtoull(tm, nullptr, 10) : (64ULL << 20));
+  }
   if ((job->cfg.flags & MR_FLAG_BATCH_COMBINE) && job->cfg.workload == MR_WORDCOUNT && !job->ingested &&
       !job->batches.empty()) {
     mr_status fs = fold(job);   // WC batch combine: the previous batches become (key, count) partials

@@ -20,6 +20,10 @@
 
 #include "common.cuh"
 
+#ifndef BMR_XTAB_UNROLL
+#define BMR_XTAB_UNROLL 1   // (2 and 4 in-flight loads per thread measured no better: 1.0 vs 1.0 / 1.34 ms)
+#endif
+
 namespace bmr {
 namespace {
 
@@ -301,11 +305,24 @@ __global__ void k_reduce_km_small(const uint64_t* __restrict__ seg, uint64_t nse
   }
 }
 
+// Large cluster segments in 8192-position work items (block reduce, BR — PAPER.md L181, L286:
+// KM-BR gains from staging its input in shared memory): the block stages the item's points in
+// SMEM, kKmStage at a time, with asynchronous 16-B gathers (cp.async: the whole sub-tile's random
+// reads are in flight together instead of one dependent load chain per thread), then every thread
+// adds its points from SMEM (<= 32 fp32 adds per thread and item, reading 5) and the
+// block combines in fp64.
+constexpr int kKmStage = 1024;   // points per staged sub-tile (32 KB)
+__device__ __forceinline__ void cp_async16(void* sdst, const void* gsrc) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(sdst))),
+               "l"(gsrc)
+               : "memory");
+}
 __global__ void __launch_bounds__(256) k_reduce_km_large(const uint64_t* __restrict__ seg,
                                                        const uint64_t* __restrict__ sk,
                                                        const uint32_t* __restrict__ perm,
                                                        const uint8_t* __restrict__ v, double* sums,
                                                        const uint64_t* __restrict__ worklist, DevState* st) {
+  extern __shared__ __align__(16) float4 stg[];   // kKmStage x 2 float4
   __shared__ unsigned long long item;
   __shared__ double red[8][8];
   const unsigned long long nitems = st->large_items;
@@ -319,11 +336,22 @@ __global__ void __launch_bounds__(256) k_reduce_km_large(const uint64_t* __restr
     const uint64_t a = seg[s] + t * kLargeTile, b = min(seg[s + 1], a + kLargeTile);
     const uint64_t cid = sk[seg[s]];
     float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};           // kLargeTile / 256 = 32 fp32 adds per thread
-    for (uint64_t i = a + threadIdx.x; i < b; i += blockDim.x) {
-      float x[8];
-      load_point(v, perm[i], x);
-#pragma unroll
-      for (int q = 0; q < 8; ++q) acc[q] = __fadd_rn(acc[q], x[q]);
+    for (uint64_t sub = a; sub < b; sub += kKmStage) {
+      const uint32_t n = static_cast<uint32_t>(min(static_cast<uint64_t>(kKmStage), b - sub));
+      for (uint32_t i = threadIdx.x; i < 2 * n; i += blockDim.x) {   // two 16-B halves per point
+        const uint8_t* src = v + static_cast<uint64_t>(perm[sub + (i >> 1)]) * 32 + (i & 1u) * 16;
+        cp_async16(&stg[i], src);
+      }
+      asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+      __syncthreads();
+      for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
+        const float4 p0 = stg[2 * i], p1 = stg[2 * i + 1];
+        acc[0] = __fadd_rn(acc[0], p0.x); acc[1] = __fadd_rn(acc[1], p0.y);
+        acc[2] = __fadd_rn(acc[2], p0.z); acc[3] = __fadd_rn(acc[3], p0.w);
+        acc[4] = __fadd_rn(acc[4], p1.x); acc[5] = __fadd_rn(acc[5], p1.y);
+        acc[6] = __fadd_rn(acc[6], p1.z); acc[7] = __fadd_rn(acc[7], p1.w);
+      }
+      __syncthreads();   // the next sub-tile overwrites the stage
     }
 #pragma unroll
     for (int q = 0; q < 8; ++q) {
@@ -580,7 +608,7 @@ cudaError_t launch_reduce_km(const uint64_t* seg_start, uint64_t nseg, const uin
   const unsigned g1 = static_cast<unsigned>(std::min<uint64_t>(blocks_for(nseg * 32, 256), 148ULL * 64));
   k_reduce_km_small<<<g1, 256, 0, s>>>(seg_start, nseg, skeys, perm, v, sums, cnts, k, worklist, st);
   count_launch();
-  k_reduce_km_large<<<num_sms * 4, 256, 0, s>>>(seg_start, skeys, perm, v, sums, worklist, st);
+  k_reduce_km_large<<<num_sms * 4, 256, kKmStage * 32, s>>>(seg_start, skeys, perm, v, sums, worklist, st);
   count_launch();
   return cudaGetLastError();
 }
@@ -657,8 +685,24 @@ __global__ void __launch_bounds__(256) k_xtab_extract(uint32_t* __restrict__ tab
   const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
   uint4* t4 = reinterpret_cast<uint4*>(tab);
   uint64_t csum = 0;
-  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i - lane < nv4; i += stride) {
-    uint4 v = i < nv4 ? __ldcs(t4 + i) : make_uint4(0, 0, 0, 0);
+  // (kXU 16-B loads in flight per thread: one load per step left the stream at ~4.5 TB/s)
+  constexpr int kXU = BMR_XTAB_UNROLL;
+  for (uint64_t i0 = blockIdx.x * static_cast<uint64_t>(blockDim.x) * kXU + threadIdx.x; i0 - lane < nv4;
+       i0 += stride * kXU) {
+    uint4 vv[kXU];
+#pragma unroll
+    for (int u = 0; u < kXU; ++u) {
+      const uint64_t i = i0 + static_cast<uint64_t>(u) * blockDim.x;
+      vv[u] = i < nv4 ? __ldcs(t4 + i) : make_uint4(0, 0, 0, 0);
+    }
+    uint32_t any = 0;
+#pragma unroll
+    for (int u = 0; u < kXU; ++u) any |= vv[u].x | vv[u].y | vv[u].z | vv[u].w;
+    if (!__any_sync(0xffffffffu, any != 0)) continue;
+#pragma unroll 1
+    for (int u = 0; u < kXU; ++u) {
+    const uint64_t i = i0 + static_cast<uint64_t>(u) * blockDim.x;
+    const uint4 v = vv[u];
     const uint32_t nz = (v.x != 0) + (v.y != 0) + (v.z != 0) + (v.w != 0);
     if (!__any_sync(0xffffffffu, nz != 0)) continue;
     const uint32_t incl = warp_inclusive_add(nz);
@@ -685,6 +729,7 @@ __global__ void __launch_bounds__(256) k_xtab_extract(uint32_t* __restrict__ tab
       ++o;
     }
     if (wrote) t4[i] = make_uint4(c[0], c[1], c[2], c[3]);   // (entries past cap stay for the next call)
+    }
   }
   if constexpr (kList) {
     const uint64_t w = warp_inclusive_add64(csum);
@@ -695,7 +740,7 @@ __global__ void __launch_bounds__(256) k_xtab_extract(uint32_t* __restrict__ tab
 cudaError_t launch_xtab_extract(uint32_t* tab, uint64_t nent, uint64_t* out, uint64_t cap, unsigned long long* cursor,
                                 int num_sms, cudaStream_t s) {
   const uint64_t nv4 = nent / 4;
-  k_xtab_extract<false><<<static_cast<unsigned>(std::min<uint64_t>(8ULL * num_sms, (nv4 + 255) / 256)), 256, 0, s>>>(
+  k_xtab_extract<false><<<static_cast<unsigned>(std::min<uint64_t>(8ULL * num_sms, (nv4 + 256 * BMR_XTAB_UNROLL - 1) / (256 * BMR_XTAB_UNROLL))), 256, 0, s>>>(
       tab, nv4, out, nullptr, nullptr, cap, cursor, nullptr);
   count_launch();
   return cudaGetLastError();
@@ -703,7 +748,7 @@ cudaError_t launch_xtab_extract(uint32_t* tab, uint64_t nent, uint64_t* out, uin
 cudaError_t launch_xtab_extract_list(uint32_t* tab, uint64_t nent, uint32_t* okeys, uint64_t* ocounts, uint64_t cap,
                                      unsigned long long* cursor, unsigned long long* wsum, int num_sms, cudaStream_t s) {
   const uint64_t nv4 = nent / 4;
-  k_xtab_extract<true><<<static_cast<unsigned>(std::min<uint64_t>(8ULL * num_sms, (nv4 + 255) / 256)), 256, 0, s>>>(
+  k_xtab_extract<true><<<static_cast<unsigned>(std::min<uint64_t>(8ULL * num_sms, (nv4 + 256 * BMR_XTAB_UNROLL - 1) / (256 * BMR_XTAB_UNROLL))), 256, 0, s>>>(
       tab, nv4, nullptr, okeys, ocounts, cap, cursor, wsum);
   count_launch();
   return cudaGetLastError();

@@ -151,6 +151,18 @@ def test_wc_map_combiner_on_and_off():
     assert st_on["pairs"] + st_on["words_combined"] == st_off["pairs"]
 
 
+def test_wc_small_input_sort_path(monkeypatch):
+    # below BMR_TABLE_MIN_BYTES the exact words take the sorted exact stream + SMEM-combiner
+    # partials (no L2 tables): same result, and the partials are pairs this time
+    g = pygen.host_text(pygen.spec_wc(1_000_000, 5), 24)
+    b = [(g["data"], g["offsets"], g["n"])]
+    monkeypatch.setenv("BMR_TABLE_MIN_BYTES", str(1 << 40))
+    small, st = same("wc", b)
+    monkeypatch.setenv("BMR_TABLE_MIN_BYTES", "0")
+    big, st2 = same("wc", b)
+    assert small == big and st["pairs_partial"] > 0 and st2["pairs_partial"] == 0
+
+
 def test_wc_combiner_partials_replay_and_multibatch():
     # tiny capacities: the exact, partial and hashed streams all overflow and the batches replay
     g = pygen.host_text(pygen.spec_wc(10_000, 3), 3)

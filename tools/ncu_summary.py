@@ -22,6 +22,16 @@ METRICS = [
     ("smsp__inst_executed.sum", "warp instructions"),
     ("l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum", "smem bank conflicts"),
     ("smsp__issue_active.avg.pct_of_peak_sustained_active", "issue active %"),
+    ("sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active", "ALU pipe %"),
+    ("sm__inst_executed_pipe_fma.avg.pct_of_peak_sustained_active", "FMA pipe %"),
+    ("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active", "FMA pipe cycles %"),
+    ("sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active", "LSU pipe %"),
+    ("smsp__thread_inst_executed_per_inst_executed.ratio", "threads / instruction"),
+    ("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum", "smem wavefronts"),
+    ("l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_atom.sum", "smem bank conflicts (atomics)"),
+    ("smsp__inst_executed_op_shared_atom.sum", "shared atomics (warp inst)"),
+    ("l1tex__m_xbar2l1tex_read_sectors_mem_global_op_atom.sum", "global atomic sectors"),
+    ("l1tex__m_l1tex2xbar_write_sectors_mem_global_op_red.sum", "global RED sectors"),
 ]
 
 
