@@ -353,6 +353,12 @@ struct mr_job {
   bool xtab_dirty = false;        // a Map fed the tables since their last extraction
   bool mid_from_table = false;    // this group's mid keys / counts come from the mid table
   DBuf<uint64_t> mkeys_out, mcounts;
+  // long words (9..16 symbols): open-addressing table of their 16 zero-padded key bytes + counts
+  DBuf<uint64_t> ltab_keys;
+  DBuf<uint32_t> ltab_cnt;
+  uint32_t lbits = 18;
+  DBuf<uint64_t> lkeys_out, lkref_out, lcounts;
+  uint64_t nseg_l = 0;            // long-table keys of this group (the output's last list)
   // KM: the Map accumulates the cluster sums itself (k <= 64; not for ingested partials)
   bool km_comb() const {
     return cfg.workload == MR_KMEANS && k <= 64 && !km_partial && !(cfg.flags & MR_FLAG_NO_MAP_COMBINE);
@@ -461,6 +467,9 @@ cudaError_t launch_batch(mr_job* job, const Batch& b) {
   a.out.mkeys = job->wc_table() ? job->mtab_keys.p : nullptr;
   a.out.mcnt = job->wc_table() ? job->mtab_cnt.p : nullptr;
   a.out.mbits = job->mbits;
+  a.out.lkeys = job->wc_table() ? job->ltab_keys.p : nullptr;
+  a.out.lcnt = job->wc_table() ? job->ltab_cnt.p : nullptr;
+  a.out.lbits = job->lbits;
   if (a.out.xtab) job->xtab_dirty = true;
   a.out.km_sums = job->km_comb() ? job->sums.p : nullptr;
   a.out.km_cnts = job->km_comb() ? job->cnts.p : nullptr;
@@ -598,6 +607,14 @@ mr_status settle_map(mr_job* job) {
   }
   const bool tile_over = (hs->err & kErrTileCap) != 0;
   const bool mid_over = (hs->err & kErrMidTable) != 0;
+  const bool long_over = (hs->err & kErrLongTable) != 0;
+  if (long_over) {   // long-word table too full: 4x larger, then the replay below
+    job->lbits += 2;
+    job->ltab_keys.release();
+    job->ltab_cnt.release();
+    CK(job->ltab_keys.ensure(2ULL << job->lbits), "grow long table");
+    CK(job->ltab_cnt.ensure((1ULL << job->lbits) * kMidStripes), "grow long table");
+  }
   if (mid_over) {   // mid table too full: a table 4x larger (grow-only), then the replay below
     job->mbits += 2;
     job->mtab_keys.release();
@@ -608,7 +625,7 @@ mr_status settle_map(mr_job* job) {
   const uint64_t m = hs->pair_cursor, mb = job->split() ? hs->pair_cursor_b : 0;
   const uint64_t mc = job->split() ? hs->pair_cursor_c : 0;
   const uint64_t mp = job->wc_comb() ? hs->pair_cursor_p : 0;
-  if (tile_over || mid_over || m > job->cap || mb > job->cap_b || mc > job->cap_c || mp > job->cap_p) {
+  if (tile_over || mid_over || long_over || m > job->cap || mb > job->cap_b || mc > job->cap_c || mp > job->cap_p) {
     if (tile_over) job->tb_cap = max_tiles + 1024;   // (tb itself is grown by launch_batch)
     const uint64_t ncap_p = job->wc_comb() ? std::max(job->cap_p, mp + mp / 8 + 4096) : 0;
     const uint64_t ncap = std::max(job->cap, m + m / 8 + 4096);
@@ -624,7 +641,7 @@ mr_status settle_map(mr_job* job) {
     }
     job->stats.capacity_pairs = job->cap + job->cap_b + job->cap_c;
     CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
-    if (job->xtab_dirty || mid_over) CK(clear_tables(job), "clear the tables");
+    if (job->xtab_dirty || mid_over || long_over) CK(clear_tables(job), "clear the tables");
     if (job->km_comb()) {
       CK(cudaMemsetAsync(job->sums.p, 0, 64ULL * job->k, job->stream), "reset sums");
       CK(cudaMemsetAsync(job->cnts.p, 0, 8ULL * job->k, job->stream), "reset counts");
@@ -632,7 +649,7 @@ mr_status settle_map(mr_job* job) {
     for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
     job->stats.replays += job->batches.size();
     CK(read_state(job), "replay (async)");
-    if ((hs->err & (kErrTileCap | kErrMidTable)) || hs->pair_cursor > job->cap ||
+    if ((hs->err & (kErrTileCap | kErrMidTable | kErrLongTable)) || hs->pair_cursor > job->cap ||
         (job->split() && (hs->pair_cursor_b > job->cap_b || hs->pair_cursor_c > job->cap_c)) ||
         (job->wc_comb() && hs->pair_cursor_p > job->cap_p))
       return fail(job, MR_ERR_OOM, "replay still overflows");
@@ -794,6 +811,8 @@ cudaError_t clear_tables(mr_job* job) {
   if (job->xtab.p) e = cudaMemsetAsync(job->xtab.p, 0, job->xtab.n * 4, job->stream);
   if (e == cudaSuccess && job->mtab_keys.p) e = cudaMemsetAsync(job->mtab_keys.p, 0xFF, job->mtab_keys.n * 8, job->stream);
   if (e == cudaSuccess && job->mtab_cnt.p) e = cudaMemsetAsync(job->mtab_cnt.p, 0, job->mtab_cnt.n * 4, job->stream);
+  if (e == cudaSuccess && job->ltab_keys.p) e = cudaMemsetAsync(job->ltab_keys.p, 0, job->ltab_keys.n * 8, job->stream);
+  if (e == cudaSuccess && job->ltab_cnt.p) e = cudaMemsetAsync(job->ltab_cnt.p, 0, job->ltab_cnt.n * 4, job->stream);
   return e;
 }
 
@@ -848,7 +867,25 @@ mr_status tables_extract(mr_job* job) {
     if (t > cap2) return fail(job, MR_ERR_OOM, "mid table extraction still overflows");
   }
   job->nseg_c = t;
-  job->stats.words_combined = job->st_h.p->words_comb;   // exact + mid words counted by the tables
+  // long-word table
+  CK(cudaMemsetAsync(cur, 0, sizeof(unsigned long long), s), "memset cursor");
+  {   // (the table holds at most one key per slot: output lists of the slot count never overflow)
+    const uint64_t slots = job->ltab_keys.n / 2;
+    CK(job->lkeys_out.ensure(2 * slots), "alloc long keys");
+    CK(job->lkref_out.ensure(slots), "alloc long keys");
+    CK(job->lcounts.ensure(slots), "alloc long counts");
+  }
+  uint64_t lcap = std::min({job->lkeys_out.n / 2, job->lkref_out.n, job->lcounts.n});
+  CK(launch_ltab_extract(job->ltab_keys.p, job->ltab_cnt.p, job->ltab_keys.n / 2, job->lkeys_out.p, job->lkref_out.p,
+                         job->lcounts.p, lcap, cur, wsum, job->nsm, s),
+     "long table extract");
+  CK(read_state(job), "sync long table extract");
+  uint64_t tl = job->st_h.p->n_extra;
+  if (tl > lcap) {   // (the references point into lkeys_out: grow it first, then re-extract everything)
+    return fail(job, MR_ERR_OOM, "long table extraction overflow");
+  }
+  job->nseg_l = tl;
+  job->stats.words_combined = job->st_h.p->words_comb;   // exact + mid + long words counted by the tables
   CK(job->seg_startx.ensure(t + 2), "alloc mid segments");
   CK(launch_iota_scaled(t, 1, job->seg_startx.p, s), "mid segments");   // one segment per mid key
   job->segc = job->seg_startx.p;
@@ -1040,6 +1077,8 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
     CK(job->xtab.ensure(1ULL << kExactBits), "alloc count table");
     CK(job->mtab_keys.ensure(1ULL << job->mbits), "alloc mid table");
     CK(job->mtab_cnt.ensure((1ULL << job->mbits) * kMidStripes), "alloc mid table");
+    CK(job->ltab_keys.ensure(2ULL << job->lbits), "alloc long table");
+    CK(job->ltab_cnt.ensure((1ULL << job->lbits) * kMidStripes), "alloc long table");
     CK(clear_tables(job), "empty the tables");
   }
   if (job->batches.empty() && job->km_comb()) {   // KM combiner accumulators (summed over batches)
@@ -1266,6 +1305,7 @@ mr_status mr_group(mr_job* job) {
   job->skeysc = nullptr;
   job->segc = nullptr;
   job->mid_from_table = false;
+  job->nseg_l = 0;
   if (split && tables) {
     // the two tables hold every exact and mid word: their nonzero counts are the final keys
     Prof::Span sp{};
@@ -1370,7 +1410,7 @@ mr_status mr_group(mr_job* job) {
     }
     if (!split) { job->nseg_a = ns; }
   }
-  job->nseg = job->nseg_a + job->n_extra + job->nseg_c + job->nseg_b;
+  job->nseg = job->nseg_a + job->n_extra + job->nseg_c + job->nseg_b + (job->mid_from_table ? job->nseg_l : 0);
   job->stats.n_keys = job->nseg;
   Prof::Span sp3{};
   if (job->prof.on) job->prof.begin(job->stream, sp3);
@@ -1388,6 +1428,10 @@ mr_status mr_group(mr_job* job) {
                             job->key_off.p + na + job->nseg_c,
                             job->stream),
          "key lengths (hashed)");
+      if (job->mid_from_table && job->nseg_l)   // the long-word table's keys (a reference list)
+        CK(launch_key_lengths(nullptr, job->nseg_l, nullptr, job->lkref_out.p,
+                              job->key_off.p + na + job->nseg_c + job->nseg_b, job->stream),
+           "key lengths (long table)");
     } else {
       CK(launch_key_lengths(job->seg_start.p, job->nseg, job->perm, job->kref.p, job->key_off.p, job->stream),
          "key lengths");
@@ -1455,6 +1499,13 @@ mr_status mr_reduce(mr_job* job) {
                            job->key_off.p + na + job->nseg_c,
                            job->keys_out.p, s),
            "key copy");
+        if (job->mid_from_table && job->nseg_l) {   // the long-word table's keys and counts
+          const uint64_t nl0 = na + job->nseg_c + job->nseg_b;
+          CK(launch_key_copy(nullptr, job->nseg_l, nullptr, job->lkref_out.p, job->key_off.p + nl0, job->keys_out.p, s),
+             "key copy (long table)");
+          CK(cudaMemcpyAsync(job->counts.p + nl0, job->lcounts.p, job->nseg_l * 8, cudaMemcpyDeviceToDevice, s),
+             "counts (long table)");
+        }
       } else {
         CK(job->worklist.ensure(m / 1024 + 64), "alloc worklist");
         CK(launch_reduce_wc(job->seg_start.p, S, job->skeys, job->perm, job->v.p, 1, job->counts.p, job->worklist.p,
@@ -1844,6 +1895,8 @@ mr_status mr_job_destroy(mr_job* job) {
   job->xsend_e.release(); job->xsend_h.release(); job->xrecv_e.release(); job->xrecv_h.release();
   job->xrecv_counts.release(); job->acc_e.release(); job->acc_h.release(); job->xtab.release(); job->mtab_keys.release();
   job->mtab_cnt.release(); job->mkeys_out.release(); job->mcounts.release();
+  job->ltab_keys.release(); job->ltab_cnt.release(); job->lkeys_out.release(); job->lkref_out.release();
+  job->lcounts.release();
   job->cent.release(); release_pairs(job); job->tb.release();
   job->swp.release(); job->seg_startp.release(); job->psum.release(); job->pxcounts.release();
   job->midx.release(); job->xkeys.release();

@@ -36,11 +36,12 @@ struct DevState {
   unsigned long long words_comb;     // WC: words absorbed by the combiners (sum of partial counts)
   unsigned long long pads_b, pads_c; // WC hashed / mid stream: sentinel entries in unused chunk tails
   unsigned long long mid_fail;       // WC mid table: inserts that found no slot (-> grow + replay)
+  unsigned long long long_fail;      // WC long-word table: inserts that found no slot (-> grow + replay)
   unsigned long long seal_waits;     // Map: seals that waited for a buffer still flushing (ring full)
   unsigned long long spills;         // Map: warp results written straight to HBM while the ring was full
 };
 constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u, kErrTileCap = 4u, kErrNullRecords = 8u,
-                       kErrMidTable = 16u;
+                       kErrMidTable = 16u, kErrLongTable = 32u;
 // WC mid-word table: open addressing over 48-bit exact keys, empty slot = all ones
 constexpr uint64_t kMidEmpty = ~0ULL;
 constexpr uint32_t kMidProbes = 32;
@@ -49,6 +50,9 @@ constexpr uint32_t kMidProbes = 32;
 constexpr uint32_t kMidStripes = 16;
 __host__ __device__ inline uint64_t mid_slot(uint64_t key, uint32_t bits) {
   return (key * 0x9E3779B97F4A7C15ULL) >> (64 - bits);
+}
+__host__ __device__ inline uint64_t long_slot(uint64_t lo, uint64_t hi, uint32_t bits) {
+  return ((lo * 0x9E3779B97F4A7C15ULL) ^ (hi * 0xC2B2AE3D27D4EB4FULL) ^ (lo >> 29)) * 0x94D049BB133111EBULL >> (64 - bits);
 }
 
 // Intermediate pairs, SoA in HBM (SURVEY §8(a) layout): sort key, key reference, value.
@@ -73,6 +77,9 @@ struct PairBufs {
   uint64_t* mkeys = nullptr; // WC mid words (6..8 symbols): open-addressing table of 48-bit exact keys
   uint32_t* mcnt = nullptr;  //   and their counts, 2^mbits slots
   uint32_t mbits = 0;
+  uint64_t* lkeys = nullptr; // WC long words (9..16 symbols): open-addressing table of their 16 key bytes
+  uint32_t* lcnt = nullptr;  //   (zero-padded; 2 x u64 per slot, all-zero = empty) and counts, 2^lbits slots
+  uint32_t lbits = 0;
 };
 
 // f-3 fused exchange: a destination rank's receive window (device pointers valid in this
@@ -227,6 +234,11 @@ cudaError_t launch_xtab_extract(uint32_t* tab, uint64_t nent, uint64_t* out, uin
 // counts (words absorbed)
 cudaError_t launch_xtab_extract_list(uint32_t* tab, uint64_t nent, uint32_t* okeys, uint64_t* ocounts, uint64_t cap,
                                      unsigned long long* cursor, unsigned long long* wsum, int num_sms, cudaStream_t s);
+// WC long-word table -> the final long keys: 16 zero-padded key bytes per key (okeys, 2 x u64),
+// their references (okref = (address of the bytes << 16) | length) and counts; slots reset
+cudaError_t launch_ltab_extract(uint64_t* lkeys, uint32_t* lcnt, uint64_t nslots, uint64_t* okeys, uint64_t* okref,
+                                uint64_t* ocounts, uint64_t cap, unsigned long long* cursor, unsigned long long* wsum,
+                                int num_sms, cudaStream_t s);
 // WC mid table -> (48-bit key, count) lists; extracted slots are reset (key empty, count 0)
 cudaError_t launch_mtab_extract(uint64_t* mkeys, uint32_t* mcnt, uint64_t nslots, uint64_t* okeys, uint64_t* ocounts,
                                 uint64_t cap, unsigned long long* cursor, unsigned long long* wsum, int num_sms,

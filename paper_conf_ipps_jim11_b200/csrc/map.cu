@@ -95,6 +95,9 @@ constexpr int kNProd = 2;
 // warp removed the map warps' spinning on sealed buffers but cost the Map more than it saved
 // (C5 Map 20.4 -> 21.3 ms, round 2: a 28th warp lowers the register budget of every warp).
 // Warps: map 0 .. nmap-1, producers nmap .. nmap+kNProd-1, then the flush warps.
+#ifndef BMR_LTAB
+#define BMR_LTAB 1
+#endif
 #ifndef BMR_STREAM_HINT
 #define BMR_STREAM_HINT 1   // WC Map input TMA loads L2 evict-first (C5 Map 21.4 -> 20.5 ms, DRAM 15.8 -> 14.4 GB)
 #endif
@@ -313,6 +316,9 @@ struct Params {
   uint64_t* mkeys;         // WC: mid words (6..8 symbols) counted in an open-addressing table of
   uint32_t* mcnt;          //   their 48-bit exact keys (2^mbits slots); nullptr: mid stream
   uint32_t mbits;
+  uint64_t* lkeys;         // WC: words of 9..16 symbols counted in an open-addressing table of their
+  uint32_t* lcnt;          //   16 zero-padded key bytes (2^lbits slots); nullptr: hashed stream
+  uint32_t lbits;
 };
 
 // Idle wait of a role warp on an mbarrier phase (map warps on a staged tile, producers on a free
@@ -1191,6 +1197,24 @@ __device__ __forceinline__ uint32_t exact_key30_bf(uint32_t lo, uint32_t b4, uin
   return y | (len == 5u ? (c4 << 24) : 0u);
 }
 
+// 128-bit compare-and-swap on global memory (sm_90+ ATOMG.CAS.128): returns the old low half,
+// the old high half in *ohi
+__device__ __forceinline__ unsigned long long cas128(unsigned long long* p, unsigned long long clo,
+                                                     unsigned long long chi, unsigned long long nlo,
+                                                     unsigned long long nhi, unsigned long long& ohi) {
+  unsigned long long olo;
+  asm volatile(
+      "{\n\t.reg .b128 c, n, r;\n\t"
+      "mov.b128 c, {%2, %3};\n\t"
+      "mov.b128 n, {%4, %5};\n\t"
+      "atom.global.cas.b128 r, [%6], c, n;\n\t"
+      "mov.b128 {%0, %1}, r;\n\t}"
+      : "=l"(olo), "=l"(ohi)
+      : "l"(clo), "l"(chi), "l"(nlo), "l"(nhi), "l"(p)
+      : "memory");
+  return olo;
+}
+
 // Output of the keyed long words: warp-private chunks of kLChunk entries of the mid stream (key
 // only) and of the hashed stream (key + kref), each taken with ONE global atomic on the stream's
 // cursor (the demand counter, D7) — the same amortisation as a buffer flush (L113) without the
@@ -1275,7 +1299,40 @@ __device__ __forceinline__ void wc_drain(const Params& P, LOut& lo, LWord* lq, u
       atomicAdd(&P.st->mid_fail, 1ULL);
     }
   }
-  const uint32_t mm = P.mkeys ? 0u : __ballot_sync(kFull, mid), mh = __ballot_sync(kFull, in && !mid);
+  if (P.lkeys) {   // long-word table (9..16 symbols): the same, keyed by the zero-padded key bytes
+                  // (exact: words have no zero byte), slots claimed with a 128-bit CAS
+    const bool lng = in && !mid;
+    const uint64_t klo = lng ? w.lo : ~0ULL;
+    const uint64_t khi = lng ? (len >= 16 ? w.hi : (w.hi & ((1ULL << (8 * (len - 8))) - 1ULL))) : ~0ULL;
+    const uint32_t grp = __match_any_sync(kFull, klo) & __match_any_sync(kFull, khi);
+    const bool lead = lng && lane == static_cast<uint32_t>(__ffs(grp) - 1);
+    const uint64_t mask = (1ULL << P.lbits) - 1ULL;
+    uint64_t h = long_slot(klo, khi, P.lbits);
+    bool done = !lead;
+    for (uint32_t pr = 0; lead && pr < kMidProbes; ++pr, h = (h + 1) & mask) {
+      unsigned long long* slot = reinterpret_cast<unsigned long long*>(P.lkeys + 2 * h);
+      unsigned long long olo, ohi;   // one 16-B access: the slot as the 128-bit CAS wrote it
+      asm volatile("ld.volatile.global.v2.u64 {%0, %1}, [%2];" : "=l"(olo), "=l"(ohi) : "l"(slot) : "memory");
+      // (two separate 8-B reads were measured to see claims half-done; should a 16-B read ever
+      // do so — a key of 9+ bytes has hi != 0 — an atomic read settles it: CAS of zero by zero)
+      if (olo != 0 && ohi == 0) olo = cas128(slot, 0ULL, 0ULL, 0ULL, 0ULL, ohi);
+      if (olo == 0) {   // empty: claim it (128-bit CAS from all-zero)
+        olo = cas128(slot, 0ULL, 0ULL, klo, khi, ohi);
+        if (olo == 0) { olo = klo; ohi = khi; }   // claimed by this lane
+      }
+      if (olo == klo && ohi == khi) {
+        atomicAdd(P.lcnt + h * kMidStripes + ((blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1)),
+                  static_cast<uint32_t>(__popc(grp)));
+        done = true;
+        break;
+      }
+    }
+    if (!done) {
+      atomicOr(&P.st->err, kErrLongTable);
+      atomicAdd(&P.st->long_fail, 1ULL);
+    }
+  }
+  const uint32_t mm = P.mkeys ? 0u : __ballot_sync(kFull, mid), mh = P.lkeys ? 0u : __ballot_sync(kFull, in && !mid);
   if (mm) {
     const unsigned long long o = chunk_slot(&P.st->pair_cursor_c, lo.mid_base, lo.mid_left, mm);
     if (mid && o < P.cap_c) P.ohc[o] = key;
@@ -2587,6 +2644,9 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.mkeys = P.xtab ? a.out.mkeys : nullptr;
   P.mcnt = P.xtab ? a.out.mcnt : nullptr;
   P.mbits = a.out.mbits;
+  P.lkeys = (BMR_LTAB && P.xtab) ? a.out.lkeys : nullptr;
+  P.lcnt = (BMR_LTAB && P.xtab) ? a.out.lcnt : nullptr;
+  P.lbits = a.out.lbits;
   if (W == kKM && P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>(std::min<uint64_t>((a.tb_cap + 255) / 256 + 1, 8ULL * num_sms));

@@ -392,7 +392,7 @@ __global__ void k_km_finalize(const double* sums, const unsigned long long* cnts
 __global__ void k_key_lengths(const uint64_t* seg, uint64_t nseg, const uint32_t* perm, const uint64_t* kref,
                               uint64_t* lens) {
   const uint64_t s = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x;
-  if (s < nseg) lens[s] = kref[perm[seg[s]]] & 0xFFFF;
+  if (s < nseg) lens[s] = kref[seg ? perm[seg[s]] : s] & 0xFFFF;   // (seg == nullptr: kref is the key list)
 }
 __global__ void k_key_copy(const uint64_t* seg, uint64_t nseg, const uint32_t* perm, const uint64_t* kref,
                            const uint64_t* key_off, uint8_t* keys) {
@@ -404,7 +404,7 @@ __global__ void k_key_copy(const uint64_t* seg, uint64_t nseg, const uint32_t* p
   const uint32_t lane = threadIdx.x & 31;
   uint64_t kr = 0, d = 0;
   if (s < nseg) {
-    kr = kref[perm[seg[s]]];
+    kr = kref[seg ? perm[seg[s]] : s];   // (seg == nullptr: kref is the key list)
     d = key_off[s];
   }
 #pragma unroll 4
@@ -785,6 +785,51 @@ __global__ void __launch_bounds__(256) k_mtab_extract(uint64_t* __restrict__ mke
   }
   const uint64_t w = warp_inclusive_add64(csum);
   if (lane == 31 && w) atomicAdd(wsum, static_cast<unsigned long long>(w));
+}
+
+__global__ void __launch_bounds__(256) k_ltab_extract(uint64_t* __restrict__ lkeys, uint32_t* __restrict__ lcnt,
+                                                    uint64_t nslots, uint64_t* okeys, uint64_t* okref,
+                                                    uint64_t* ocounts, uint64_t cap, unsigned long long* cursor,
+                                                    unsigned long long* wsum) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
+  uint64_t csum = 0;
+  for (uint64_t i = blockIdx.x * static_cast<uint64_t>(blockDim.x) + threadIdx.x; i - lane < nslots; i += stride) {
+    const uint64_t lo = i < nslots ? lkeys[2 * i] : 0, hi = i < nslots ? lkeys[2 * i + 1] : 0;
+    const bool full = lo != 0;   // (a word's first byte is never 0)
+    const uint32_t m = __ballot_sync(0xffffffffu, full);
+    if (!m) continue;
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(cursor, static_cast<unsigned long long>(__popc(m)));
+    base = __shfl_sync(0xffffffffu, base, 0);
+    const uint64_t o = base + __popc(m & lanemask_lt());
+    if (full && o < cap) {
+      uint64_t c = 0;
+#pragma unroll
+      for (uint32_t q = 0; q < kMidStripes; ++q) c += lcnt[i * kMidStripes + q];
+      okeys[2 * o] = lo;
+      okeys[2 * o + 1] = hi;
+      // length = the number of nonzero (word) bytes of the zero-padded key
+      const uint32_t len = 8u + (hi ? (64u - static_cast<uint32_t>(__clzll(static_cast<long long>(hi))) + 7u) / 8u : 0u);
+      okref[o] = (reinterpret_cast<uint64_t>(okeys + 2 * o) << 16) | len;
+      ocounts[o] = c;
+      csum += c;
+      lkeys[2 * i] = 0;
+      lkeys[2 * i + 1] = 0;
+      for (uint32_t q = 0; q < kMidStripes; ++q) lcnt[i * kMidStripes + q] = 0;
+    }
+  }
+  const uint64_t w = warp_inclusive_add64(csum);
+  if (lane == 31 && w) atomicAdd(wsum, static_cast<unsigned long long>(w));
+}
+
+cudaError_t launch_ltab_extract(uint64_t* lkeys, uint32_t* lcnt, uint64_t nslots, uint64_t* okeys, uint64_t* okref,
+                                uint64_t* ocounts, uint64_t cap, unsigned long long* cursor, unsigned long long* wsum,
+                                int num_sms, cudaStream_t s) {
+  k_ltab_extract<<<static_cast<unsigned>(std::min<uint64_t>(8ULL * num_sms, (nslots + 255) / 256)), 256, 0, s>>>(
+      lkeys, lcnt, nslots, okeys, okref, ocounts, cap, cursor, wsum);
+  count_launch();
+  return cudaGetLastError();
 }
 
 cudaError_t launch_mtab_extract(uint64_t* mkeys, uint32_t* mcnt, uint64_t nslots, uint64_t* okeys, uint64_t* ocounts,

@@ -125,7 +125,7 @@ def test_wc_single_words_and_record_boundaries():
     same("wc", [(data, off, len(recs))])
 
 
-def test_wc_force_tiny_out_and_weak_hash():
+def test_wc_force_tiny_out_and_weak_hash(monkeypatch):
     g = pygen.host_text(pygen.spec_wc(1_000_000, 5), 2)
     b = [(g["data"], g["offsets"], g["n"])]
     base, _ = same("wc", b)
@@ -133,6 +133,9 @@ def test_wc_force_tiny_out_and_weak_hash():
     assert st["flushes"] > 500            # 641-unit buffers instead of 3068
     tiny2, _ = same("wc", b, gkw={"flags": bmr.FLAG_FORCE_TINY_OUT})
     assert tiny2 == tiny
+    # the hashed stream (words > 8 symbols without the L2 tables, which count words of <= 16
+    # symbols exactly): a 4-bit hash forces collisions, the byte verification must split them
+    monkeypatch.setenv("BMR_TABLE_MIN_BYTES", str(1 << 40))
     weak, st2 = same("wc", b, gkw={"flags": bmr.FLAG_WEAK_HASH_DEBUG})
     assert st2["collisions"] > 0          # verification found the forced collisions
     assert base == tiny == weak
@@ -163,8 +166,10 @@ def test_wc_small_input_sort_path(monkeypatch):
     assert small == big and st["pairs_partial"] > 0 and st2["pairs_partial"] == 0
 
 
-def test_wc_combiner_partials_replay_and_multibatch():
+def test_wc_combiner_partials_replay_and_multibatch(monkeypatch):
     # tiny capacities: the exact, partial and hashed streams all overflow and the batches replay
+    # (the streams: no L2 tables)
+    monkeypatch.setenv("BMR_TABLE_MIN_BYTES", str(1 << 40))
     g = pygen.host_text(pygen.spec_wc(10_000, 3), 3)
     data, off = g["data"], g["offsets"]
     cuts = [0, g["n"] // 4, g["n"] // 2, g["n"]]
@@ -232,7 +237,8 @@ def test_map_host_lines_equals_offsets(chunk, monkeypatch):
         assert st["input_bytes"] == len(text)
 
 
-def test_wc_replay_on_overflow():
+def test_wc_replay_on_overflow(monkeypatch):
+    monkeypatch.setenv("BMR_TABLE_MIN_BYTES", str(1 << 40))   # (pair streams, no L2 tables)
     g = pygen.host_text(pygen.spec_wc(10_000, 1), 1)
     got, st = same("wc", [(g["data"], g["offsets"], g["n"])], gkw={"max_pairs_hint": 1000})
     assert st["replays"] >= 1
@@ -259,12 +265,29 @@ def test_wc_exact_and_hashed_streams():
     assert min(lens) == 1 and max(lens) >= 12 and {6, 7} <= lens
 
 
-def test_wc_hashed_stream_replay():
-    # every word is longer than 8 bytes: the whole Map output is the hashed stream
+def test_wc_hashed_stream_replay(monkeypatch):
+    # every word is longer than 8 bytes: without the L2 tables the whole Map output is the hashed
+    # stream
+    monkeypatch.setenv("BMR_TABLE_MIN_BYTES", str(1 << 40))
     recs = [b" ".join(b"w%08d" % (i * 7 + j) for j in range(5)) for i in range(4000)]
     data, off = make_records(recs)
     got, st = same("wc", [(data, off, len(recs))], gkw={"max_pairs_hint": 1000})
     assert st["replays"] >= 1 and len(got) == 20000
+
+
+@pytest.mark.parametrize("fmt", [b"L%011d", b"x%016d"], ids=["12-symbol", "17-symbol"])
+def test_wc_long_words_table_and_stream(fmt):
+    # 300k distinct words of 12 symbols (long-word table: more than its first 2^18 slots hold ->
+    # grow + replay) or of 17 symbols (> 16: the hashed stream), twice each
+    words = [fmt % i for i in range(300_000)]
+    recs = [b" ".join(words[i:i + 6]) for i in range(0, len(words), 6)] * 2
+    data, off = make_records(recs)
+    got, st = same("wc", [(data, off, len(recs))])
+    assert len(got) == 300_000 and set(got.values()) == {2}
+    if len(words[0]) <= 16:
+        assert st["replays"] >= 1 and st["pairs_hashed"] == 0
+    else:
+        assert st["pairs_hashed"] == 600_000
 
 
 def test_wc_mid_table_growth_replay():
