@@ -91,6 +91,13 @@ __device__ __forceinline__ void fence_proxy_async_shared() {
 __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
+// Fire-and-forget global add (REDG).  A plain atomicAdd whose result is unused was compiled to
+// ATOMG with an RZ destination inside the Map's divergent loops, and the loop's next write to the
+// address registers then waited on the atomic's long scoreboard (ncu C5 round 2: 22% of the
+// WordCount Map's stall samples at one branch).
+__device__ __forceinline__ void red_add_u32(uint32_t* p, uint32_t v) {
+  asm volatile("red.relaxed.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
 __device__ __forceinline__ uint32_t lanemask_lt() {
   uint32_t m;
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
@@ -245,16 +252,14 @@ __device__ __forceinline__ uint64_t inline_key(uint64_t bytes_le, uint32_t len, 
 // code: '0'-'9' -> 1..10, 'A'-'Z' -> 11..36, 'a'-'z' -> 37..62.  A word of L <= 8 symbols packs
 // injectively into 6L bits (symbol i at bits 6i; the highest nonzero code gives the length):
 // <= 5 symbols -> 30 bits (four 8-bit LSD digits), 6..8 symbols -> 48 bits (six digits).  Codes
-// of 4 bytes at once: code = low nibble + base[high nibble], the 5-entry base table looked up
-// with one byte permute (PRMT) indexed by the high nibbles.
+// of 4 bytes at once, arithmetically: code = c - 47 - 7 [c >= 0x40] - 6 [c >= 0x60] (bits 6 and
+// 5 of a word byte give its class; two of the five operations run on the FMA pipe).  Bytes past a
+// word's end may borrow into the bytes above them, never below, and are masked off by the callers.
 __device__ __forceinline__ uint32_t exact_codes4(uint32_t w) {
-  const uint32_t hi = (w >> 4) & 0x0F0F0F0Fu;                  // 3 digit, 4-5 upper, 6-7 lower
-  const uint32_t h2 = hi | (hi >> 4);
-  const uint32_t sel = (h2 & 0xFFu) | ((h2 >> 8) & 0xFF00u);   // four selector nibbles
-  // table bytes 3..7 = {1, 10, 26, 36, 52}: '0' (low 0) -> 1, 'A' (low 1) -> 11, 'P' (low 0) -> 26,
-  // 'a' (low 1) -> 37, 'p' (low 0) -> 52
-  const uint32_t base = __byte_perm(0x01000000u, 0x34241A0Au, sel);
-  return (w & 0x0F0F0F0Fu) + base;                             // <= 62 per byte: no carries
+  const uint32_t s6 = w >> 6, s5 = w >> 5;
+  const uint32_t t6 = s6 & 0x01010101u;                 // [c >= 0x40] per byte
+  const uint32_t t65 = s6 & s5 & 0x01010101u;           // [c >= 0x60]
+  return (w - 0x2F2F2F2Fu) - 7u * t6 - 6u * t65;        // <= 62 per byte for word bytes
 }
 __device__ __forceinline__ uint64_t exact_key(uint64_t bytes_le, uint32_t len) {   // len 1..8
   uint64_t x = (static_cast<uint64_t>(exact_codes4(static_cast<uint32_t>(bytes_le >> 32))) << 32) |
@@ -272,10 +277,7 @@ __device__ __forceinline__ uint32_t exact_key30(uint64_t bytes_le, uint32_t len)
   if (len < 4) c &= (1u << (8 * len)) - 1u;
   uint32_t y = (c & 0x003F003Fu) | ((c >> 2) & 0x0FC00FC0u);   // byte pairs -> 12 bits
   y = (y & 0x00000FFFu) | ((y >> 4) & 0x00FFF000u);            // -> 24 bits
-  if (len == 5) {
-    const uint32_t b4 = static_cast<uint32_t>(bytes_le >> 32) & 0xFFu;
-    y |= ((b4 & 0xFu) + (__byte_perm(0x01000000u, 0x34241A0Au, b4 >> 4) & 0xFFu)) << 24;
-  }
+  if (len == 5) y |= (exact_codes4(static_cast<uint32_t>(bytes_le >> 32)) & 0xFFu) << 24;
   return y;
 }
 // Inverse: key bytes little-endian and the length.

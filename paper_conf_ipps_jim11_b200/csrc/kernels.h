@@ -129,6 +129,7 @@ uint32_t map_dyn_windows(int workload);
 uint32_t map_wc_balanced();
 bool map_wc_table_ok(uint32_t flags);           // the WC Map can feed the L2 count table (SIO fast path)
 bool map_fast_path();                           // the WC / II SIO fast paths are on (BMR_MAP_FAST)
+bool map_wc_tab();                              // WordCount table mode uses wc_window_tab (BMR_WC_TAB)
 cudaError_t launch_map(const MapArgs& a, int num_sms, cudaStream_t s);
 
 // ---- group-by-key (hash radix sort + segment boundaries) ----

@@ -107,8 +107,8 @@ constexpr int kNProd = 2;
 #ifndef BMR_MID_LDCA
 #define BMR_MID_LDCA 0
 #endif
-#ifndef BMR_FLUSH_SLEEP_NS
-#define BMR_FLUSH_SLEEP_NS 0
+#ifndef BMR_WC_TAB
+#define BMR_WC_TAB 1   // WordCount table mode: per-lane start loop (wc_window_tab); 0: the queued rounds of wc_window
 #endif
 #ifndef BMR_WC_NFLUSH
 #define BMR_WC_NFLUSH 1u
@@ -668,6 +668,10 @@ __device__ __forceinline__ void tma_store_1d(void* gdst, const void* ssrc, uint3
 // (one lane per stream: all three reservations in flight together), the TMA bulk store of the
 // buffer's SoA runs, the routed stores of the queued entries while the TMA reads SMEM, and only
 // then the wait for the TMA's reads before the buffer is handed back.
+#ifndef BMR_FLUSH_BACKOFF_NS
+#define BMR_FLUSH_BACKOFF_NS 2048
+#endif
+constexpr uint32_t kFlushBackoffNs = BMR_FLUSH_BACKOFF_NS;
 template <int W>
 __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc, uint32_t fw) {
   using F = PairFmt<W>;
@@ -679,14 +683,18 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc, uint32_t 
     // wait for generation f to be sealed; with several flush warps the one waiting past the
     // final generation sees the final flag instead (no arrival ever comes for it)
     bool past = false;
-    // (suspended try_wait: a polling flush warp would take issue slots from the map warps)
+    // (suspended try_wait: a polling flush warp would take issue slots from the map warps; the
+    // suspend hint is an upper bound the hardware often cuts short, so an idle flush warp also
+    // backs off with __nanosleep up to kFlushBackoffNs — in WordCount table mode buffers seal
+    // rarely and the polls were 3% of the Map's instructions, ncu C5 round 2)
+    uint32_t backoff = 0;
     while (!mbar_try_wait_hint(&oc->req[h], (f / kNOut) & 1u, 2000)) {
+      if (backoff) __nanosleep(backoff);
+      backoff = min(backoff ? 2 * backoff : 64u, kFlushBackoffNs);
       if (NF > 1 && ld_acquire_cta_shared_u32(&oc->is_final) && ld_acquire_cta_shared_u32(&oc->final_seq) < f) {
         past = true;
         break;
       }
-      if (BMR_FLUSH_SLEEP_NS) __nanosleep(BMR_FLUSH_SLEEP_NS);   // the flush warp has the highest scheduling
-                                                                  // priority: polling would take the map warps' slots
     }
     if (past) break;
     // (the sealing warp wrote these before its release-arrive on req[h]; the wait above acquires)
@@ -1190,10 +1198,10 @@ __device__ __forceinline__ void lane0_mbar_arrive(uint64_t* bar) {
 }
 // exact_key30 (common.cuh) without branches: lo = word bytes 0..3, b4 = byte 4, len 1..5
 __device__ __forceinline__ uint32_t exact_key30_bf(uint32_t lo, uint32_t b4, uint32_t len) {
-  uint32_t c = exact_codes4(lo) & (0xFFFFFFFFu >> (32u - 8u * min(len, 4u)));
+  const uint32_t c = exact_codes4(lo) & __funnelshift_lc(0xFFFFFFFFu, 0u, 8u * len);   // bytes < len
   uint32_t y = (c & 0x003F003Fu) | ((c >> 2) & 0x0FC00FC0u);   // byte pairs -> 12 bits
   y = (y & 0x00000FFFu) | ((y >> 4) & 0x00FFF000u);            // -> 24 bits
-  const uint32_t c4 = (b4 & 0xFu) + __byte_perm(0x01000000u, 0x34241A0Au, (b4 >> 4) & 0xFu);
+  const uint32_t c4 = exact_codes4(b4) & 0x3Fu;
   return y | (len == 5u ? (c4 << 24) : 0u);
 }
 
@@ -1288,8 +1296,8 @@ __device__ __forceinline__ void wc_drain(const Params& P, LOut& lo, LWord* lq, u
                                           : *reinterpret_cast<volatile unsigned long long*>(P.mkeys + h);
       if (k == kMidEmpty) k = atomicCAS(reinterpret_cast<unsigned long long*>(P.mkeys + h), kMidEmpty, key);
       if (k == key || k == kMidEmpty) {
-        atomicAdd(P.mcnt + h * kMidStripes + ((blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1)),
-                  static_cast<uint32_t>(__popc(grp)));
+        red_add_u32(P.mcnt + h * kMidStripes + ((blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1)),
+                    static_cast<uint32_t>(__popc(grp)));
         done = true;
         break;
       }
@@ -1321,8 +1329,8 @@ __device__ __forceinline__ void wc_drain(const Params& P, LOut& lo, LWord* lq, u
         if (olo == 0) { olo = klo; ohi = khi; }   // claimed by this lane
       }
       if (olo == klo && ohi == khi) {
-        atomicAdd(P.lcnt + h * kMidStripes + ((blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1)),
-                  static_cast<uint32_t>(__popc(grp)));
+        red_add_u32(P.lcnt + h * kMidStripes + ((blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1)),
+                    static_cast<uint32_t>(__popc(grp)));
         done = true;
         break;
       }
@@ -1353,6 +1361,67 @@ __device__ __forceinline__ void wc_drain(const Params& P, LOut& lo, LWord* lq, u
   __syncwarp();
   qn = rest;
 }
+// Table mode (mid AND long tables present): the same counts as wc_drain with one probe pass.
+// Mid words (6..8) and long words (9..16) share the match groups — a lane's (klo, khi) is
+// (48-bit exact key, 0) for a mid word and its zero-padded key bytes for a long word; the two
+// never collide (a long word's first 8 bytes are all non-zero: klo >= 2^56 > any 48-bit key) —
+// and each group leader issues its table load (8-B mid slot or 16-B long slot) in the same
+// round, so the two L2 round trips overlap.  No hash is computed (the tables are exact).
+__device__ __forceinline__ void wc_drain_tab(const Params& P, LWord* lq, uint32_t& qn) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t n = min(qn, 32u);
+  if (n == 0) return;
+  __syncwarp();
+  const bool in = lane < n;
+  LWord w{0, 0, 0};
+  if (in) w = lq[lane];
+  const uint32_t len = static_cast<uint32_t>(w.meta & 0xFFFFu);
+  const bool mid = in && len <= kMidMax, lng = in && !mid;
+  const uint64_t klo = mid ? exact_key(w.lo, len) : lng ? w.lo : ~0ULL;
+  const uint64_t khi = mid ? 0ULL : lng ? (len >= 16 ? w.hi : (w.hi & ((1ULL << (8 * (len - 8))) - 1ULL))) : ~0ULL;
+  const uint32_t grp = __match_any_sync(kFull, klo) & __match_any_sync(kFull, khi);
+  bool todo = in && lane == static_cast<uint32_t>(__ffs(grp) - 1);
+  const uint32_t stripe = (blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1);
+  const uint64_t mmask = (1ULL << P.mbits) - 1ULL, lmask = (1ULL << P.lbits) - 1ULL;
+  uint64_t h = mid ? mid_slot(klo, P.mbits) : long_slot(klo, khi, P.lbits);
+  for (uint32_t pr = 0; todo && pr < kMidProbes; ++pr) {
+    if (mid) {
+      unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(P.mkeys + h);
+      if (k == kMidEmpty) k = atomicCAS(reinterpret_cast<unsigned long long*>(P.mkeys + h), kMidEmpty, klo);
+      if (k == klo || k == kMidEmpty) {
+        red_add_u32(P.mcnt + h * kMidStripes + stripe, static_cast<uint32_t>(__popc(grp)));
+        todo = false;
+      }
+      h = (h + 1) & mmask;
+    } else {
+      unsigned long long* slot = reinterpret_cast<unsigned long long*>(P.lkeys + 2 * h);
+      unsigned long long olo, ohi;   // one 16-B access: the slot as the 128-bit CAS wrote it
+      asm volatile("ld.volatile.global.v2.u64 {%0, %1}, [%2];" : "=l"(olo), "=l"(ohi) : "l"(slot) : "memory");
+      if (olo != 0 && ohi == 0) olo = cas128(slot, 0ULL, 0ULL, 0ULL, 0ULL, ohi);   // (see wc_drain)
+      if (olo == 0) {
+        olo = cas128(slot, 0ULL, 0ULL, klo, khi, ohi);
+        if (olo == 0) { olo = klo; ohi = khi; }
+      }
+      if (olo == klo && ohi == khi) {
+        red_add_u32(P.lcnt + h * kMidStripes + stripe, static_cast<uint32_t>(__popc(grp)));
+        todo = false;
+      }
+      h = (h + 1) & lmask;
+    }
+  }
+  if (todo) {   // table too full: counted, the batch is replayed with a larger table (D7)
+    atomicOr(&P.st->err, mid ? kErrMidTable : kErrLongTable);
+    atomicAdd(mid ? &P.st->mid_fail : &P.st->long_fail, 1ULL);
+  }
+  const uint32_t rest = qn - n;
+  LWord r{0, 0, 0};
+  if (lane < rest) r = lq[n + lane];
+  __syncwarp();
+  if (lane < rest) lq[lane] = r;
+  __syncwarp();
+  qn = rest;
+}
+
 // end of a warp's work: sentinel entries in its chunks' unused tails
 __device__ __forceinline__ void wc_chunk_pads(const Params& P, const LOut& lo) {
   const uint32_t lane = threadIdx.x & 31;
@@ -1436,7 +1505,7 @@ __device__ __forceinline__ void wc_window(const Params& P, OutCtl* oc, uint8_t* 
     bool miss = act;
     if (act && P.comb) miss = !comb_add(ctab, key);
     if (P.xtab) {   // second level: one fire-and-forget L2 atomic per miss (RED.ADD), no pair
-      if (miss) atomicAdd(P.xtab + key, 1u);
+      if (miss) red_add_u32(P.xtab + key, 1u);
       continue;
     }
     const uint32_t ma = __ballot_sync(kFull, miss);
@@ -1495,8 +1564,113 @@ __device__ __forceinline__ void wc_window(const Params& P, OutCtl* oc, uint8_t* 
   __syncwarp();
 }
 
+// Combiner update of one exact word without branches (predicated PTX): the slot's key is read;
+// an empty slot is claimed by CAS; a slot holding the key (or just claimed) counts the word in
+// SMEM, any other slot sends it to the L2 count table (RED).  Same semantics as comb_add + RED.
+__device__ __forceinline__ void comb_or_table(uint32_t* slot_key, uint32_t* slot_cnt, uint32_t* tab, uint32_t key) {
+  asm volatile(
+      "{\n\t.reg .pred pe, ph;\n\t.reg .b32 v;\n\t"
+      "ld.volatile.shared.u32 v, [%0];\n\t"
+      "setp.eq.u32 pe, v, -1;\n\t"
+      "@pe atom.shared.cas.b32 v, [%0], -1, %3;\n\t"
+      "setp.eq.u32 ph, v, %3;\n\t"
+      "@!ph setp.eq.u32 ph, v, -1;\n\t"
+      "@ph red.shared.add.u32 [%1], 1;\n\t"
+      "@!ph red.relaxed.gpu.global.add.u32 [%2], 1;\n\t}" ::"r"(smem_u32(slot_key)),
+      "r"(smem_u32(slot_cnt)), "l"(tab), "r"(key)
+      : "memory");
+}
+
+// One 512-B window in table mode (the default for large batches: exact words counted in the
+// SMEM combiner + the L2 count table, longer words in the L2 mid / long tables, so the window
+// emits nothing): no descriptor queues, no warp scan.  Each lane walks the exact-word starts of
+// its own 16 bytes (a loop of max-over-lanes iterations; ~2.7 starts per lane at C5) and counts
+// each word where it finds it; the starts of longer words are then moved into the warp's
+// long-word queue one per lane per round.  The same words, keys and tables as wc_window.
+__device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8_t* outh, const TileView& tv,
+                                              long long p0w, uint32_t* ctab, LWord* lq, uint32_t& qn) {
+  const uint32_t lane = threadIdx.x & 31;
+  const long long N = bd_nbytes();
+  const long long p0 = p0w + 16 * lane;
+  const uint32_t i0 = static_cast<uint32_t>(p0 - tv.sbase);   // 16-B aligned stage offset
+  const uint4 c0 = *reinterpret_cast<const uint4*>(tv.sb + i0);
+  const uint4 c1 = *reinterpret_cast<const uint4*>(tv.sb + i0 + 16);   // next chunk (lane 31: the halo)
+  const uint32_t pb = tv.sb[i0 - 1];                                    // byte before the chunk (lead bytes)
+  uint32_t wm = word_mask4(c0.x) | (word_mask4(c0.y) << 4) | (word_mask4(c0.z) << 8) | (word_mask4(c0.w) << 12) |
+                (word_mask4(c1.x) << 16) | (word_mask4(c1.y) << 20) | (word_mask4(c1.z) << 24) |
+                (word_mask4(c1.w) << 28);
+  const bool edge = p0w < 0 || p0w + kWin + 16 > N;   // warp-uniform: only the input's first / last window
+  if (edge) wm &= range_mask32(p0, 0, N);
+  const uint32_t R = bits32(tv.bm, i0);                // record starts at p0 .. p0 + 31
+  const uint32_t prevw = (p0 > 0 && is_word_byte(pb)) ? 1u : 0u;
+  const uint32_t nb = ~wm | R;                          // a word cannot continue here
+  const uint32_t S = wm & 0xFFFFu & ~(((wm << 1) | prevw) & ~R);   // word starts (C-2 WC)
+  const uint32_t near = (nb >> 1) | (nb >> 2) | (nb >> 3) | (nb >> 4) | (nb >> 5);   // ends within 5 bytes
+  uint32_t* ccnt = ctab + Cfg<kWC>::kCombSlots;
+  // exact words (<= 5 bytes): key from the stage, combiner slot or L2 count table
+  for (uint32_t E = S & near; E; E &= E - 1) {
+    const uint32_t j = __ffs(E) - 1;
+    const uint32_t len = __ffs(nb >> (j + 1));         // 1..5: a stop within 5 bytes
+    const uint32_t pos = i0 + j;
+    const uint32_t a = pos & ~3u, sh = (pos & 3u) * 8;
+    const uint32_t w0 = *reinterpret_cast<const uint32_t*>(tv.sb + a);
+    const uint32_t w1 = *reinterpret_cast<const uint32_t*>(tv.sb + a + 4);
+    const uint32_t key = exact_key30_bf(__funnelshift_r(w0, w1, sh), (w1 >> sh) & 0xFFu, len);
+    const uint32_t home = (key * 0x9E3779B1u) >> (32 - kCombBits);
+    comb_or_table(ctab + home, ccnt + home, P.xtab + key, key);
+  }
+  // longer words: only the lane's highest start can lack a visible end (no stop in the 31 - j
+  // bytes after it)
+  uint32_t L = S & ~near;
+  if (!__any_sync(kFull, L)) return;
+  uint32_t len_slow = 0;
+  if (L) {
+    const uint32_t jh = 31 - __clz(S);
+    if ((nb >> (jh + 1)) == 0) len_slow = slow_word_len(P, tv, p0 + jh, p0 + 32);
+  }
+  for (;;) {   // one long word per lane per round, appended to the warp's queue
+    const uint32_t m = __ballot_sync(kFull, L != 0);
+    if (!m) break;
+    if (qn + __popc(m) > static_cast<uint32_t>(Cfg<kWC>::kLQ)) wc_drain_tab(P, lq, qn);
+    uint32_t j = 0, len = 0;
+    if (L) {
+      j = __ffs(L) - 1;
+      L &= L - 1;
+      const uint32_t rest = nb >> (j + 1);
+      len = rest ? static_cast<uint32_t>(__ffs(rest)) : len_slow;
+      if (len > 0xFFFFu) atomicOr(&P.st->err, kErrKeyTooLong);
+    }
+    const bool in = (m >> lane) & 1u;
+    const bool small = in && len <= kLQMaxLen;
+    const uint32_t ms = __ballot_sync(kFull, small), mb = m & ~ms;
+    const uint32_t pos = i0 + j;
+    if (small) {   // (a word of <= 16 bytes starting in the tile lies inside the staged window)
+      LWord* d = lq + qn + __popc(ms & lanemask_lt());
+      const uint32_t* src = reinterpret_cast<const uint32_t*>(tv.sb + (pos & ~3u));
+      const uint32_t sh = (pos & 3u) * 8;   // 5 aligned words, funnel-shifted
+      const uint32_t y0 = src[0], y1 = src[1], y2 = src[2], y3 = src[3], y4 = src[4];
+      d->lo = static_cast<uint64_t>(__funnelshift_r(y0, y1, sh)) | (static_cast<uint64_t>(__funnelshift_r(y1, y2, sh)) << 32);
+      d->hi = static_cast<uint64_t>(__funnelshift_r(y2, y3, sh)) | (static_cast<uint64_t>(__funnelshift_r(y3, y4, sh)) << 32);
+      d->meta = (static_cast<uint64_t>(tv.sbase + pos) << 16) | len;
+    }
+    qn += __popc(ms);
+    if (mb) {   // words of > 16 bytes (rare): hashed-stream entries through the output ring
+      const Slot slot = reserve<kWC>(P, oc, outh, __popc(mb) << kCbShift, P.out_cap);
+      ulonglong2* top = reinterpret_cast<ulonglong2*>(outh + slot.half * Cfg<kWC>::kOutHalf + Cfg<kWC>::kOutHalf);
+      if (in && !small) {
+        const long long p = tv.sbase + static_cast<long long>(pos);
+        top[-1 - static_cast<int>(cur_cb(slot.base) + __popc(mb & lanemask_lt()))] =
+            make_ulonglong2(key_at(P, tv, p, len), (reinterpret_cast<uint64_t>(P.rec + p) << 16) | len);
+      }
+      commit(oc, slot, __popc(mb) << kCbShift);
+    }
+  }
+  __syncwarp();
+}
+
 // WordCount map warps in SIO mode: windows from the shared counter (tile order), the stage
-// header read once per tile change, the window loop of wc_window.
+// header read once per tile change, the window loop of wc_window (wc_window_tab in table mode).
+template <bool kTab>
 __device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   constexpr int W = kWC;
   constexpr int kStages = Cfg<W>::kStages;
@@ -1531,13 +1705,20 @@ __device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       const TileView tv{smem + Layout<W>::bytes + s * kStageBytes,
                         reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits), sbase, stg_hi, 0,
                         0};
-      wc_window(P, oc, outh, tv, wp, xq, hq, ctab, lq, qn, lo);
-      if (qn >= 32) wc_drain(P, lo, lq, qn);
+      if constexpr (kTab) wc_window_tab(P, oc, outh, tv, wp, ctab, lq, qn);
+      else wc_window(P, oc, outh, tv, wp, xq, hq, ctab, lq, qn, lo);
+      if (qn >= 32) {
+        if constexpr (kTab) wc_drain_tab(P, lq, qn);
+        else wc_drain(P, lo, lq, qn);
+      }
     }
     __syncwarp();
     lane0_mbar_arrive(&empty[s]);
   }
-  while (qn) wc_drain(P, lo, lq, qn);   // this warp's last long words
+  while (qn) {   // this warp's last long words
+    if constexpr (kTab) wc_drain_tab(P, lq, qn);
+    else wc_drain(P, lo, lq, qn);
+  }
   wc_chunk_pads(P, lo);
 }
 
@@ -2233,7 +2414,9 @@ __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl
   }
 }
 
-template <int W>
+// V: 1 = the WordCount table-mode instantiation (wc_window_tab), a kernel of its own so that the
+// two window paths do not share one register allocation
+template <int W, int V>
 __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   constexpr int kStages = Cfg<W>::kStages;
   using F = PairFmt<W>;
@@ -2270,7 +2453,10 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   }
   if constexpr (W == kWC) {
     fast = !P.so && !P.si && P.wc_bal && P.dyn && P.wc_fast;
-    if (fast) wc_map_loop(P, smem, oc);
+    if (fast) {
+      if constexpr (V == 1) wc_map_loop<true>(P, smem, oc);
+      else wc_map_loop<false>(P, smem, oc);
+    }
   }
   if constexpr (W == kII) {
     fast = !P.so && !P.si && P.dyn && P.wc_fast;
@@ -2464,7 +2650,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       const uint32_t* ctab = reinterpret_cast<const uint32_t*>(smem + Layout<W>::comb);
       for (uint32_t i = warp * 32 + lane; i < static_cast<uint32_t>(Cfg<W>::kCombSlots); i += nmap<W>() * 32) {
         const uint32_t k = ctab[i], c = ctab[Cfg<W>::kCombSlots + i];
-        if (k != kCombEmpty32) atomicAdd(P.xtab + k, c);
+        if (k != kCombEmpty32) red_add_u32(P.xtab + k, c);
       }
     } else if (P.comb) {   // combiner partials -> global (one atomic per warp step; demand counted past capacity)
       const uint32_t* ctab = reinterpret_cast<const uint32_t*>(smem + Layout<W>::comb);
@@ -2487,7 +2673,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   }
 }
 
-template <int W>
+template <int W, int V = 0>
 __global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
   constexpr int kStages = Cfg<W>::kStages;
   extern __shared__ __align__(128) uint8_t smem[];
@@ -2546,7 +2732,7 @@ __global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
   if (warp >= static_cast<uint32_t>(nmap<W>()) && warp < static_cast<uint32_t>(nmap<W>() + kNProd))
     producer_loop<W>(P, smem, warp - nmap<W>());
   else if (warp >= static_cast<uint32_t>(nmap<W>() + kNProd)) flush_loop<W>(P, smem, oc, warp - nmap<W>() - kNProd);
-  else map_loop<W>(P, smem, oc);
+  else map_loop<W, V>(P, smem, oc);
 }
 
 // Batch dimensions + tile bounds of a text batch, on the device (mr_map enqueues without reading
@@ -2655,11 +2841,17 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
     count_launch();
   }
   const size_t smem = Layout<W>::cent + (W == kKM ? static_cast<size_t>(a.k) * 32 : 0);
-  cudaError_t e = cudaFuncSetAttribute(k_map<W>, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
+  // WordCount table mode (the fast SIO path with the L2 tables): its own instantiation
+  const bool tab = W == kWC && map_wc_tab() && P.xtab && P.mkeys && P.lkeys && P.comb && !P.so && !P.si && P.wc_bal && P.dyn && P.wc_fast;
+  auto kern = k_map<W, 0>;
+  if constexpr (W == kWC) {
+    if (tab) kern = k_map<W, 1>;
+  }
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
   if (e != cudaSuccess) return e;
   int grid = a.grid > 0 ? a.grid : num_sms;   // persistent CTAs; CTAs without a tile exit at once
   if (W == kKM && static_cast<uint64_t>(grid) > P.ntiles) grid = static_cast<int>(P.ntiles);
-  k_map<W><<<grid, threads_of<W>(), smem, s>>>(P);
+  kern<<<grid, threads_of<W>(), smem, s>>>(P);
   count_launch();
   return cudaGetLastError();
 }
@@ -2681,6 +2873,16 @@ uint32_t map_prefetch(int w) {
 
 // idle-wait flavour of the Map role warps (BMR_MAP_WAIT: 0 = plain try_wait, 1 = suspend-time
 // hint, 2 = plain for the map warps and __nanosleep polling for the producers / flush warp)
+// WordCount table-mode window path (BMR_WC_TAB env, default BMR_WC_TAB = 1: wc_window_tab; 0: the
+// queued rounds of wc_window)
+bool map_wc_tab() {
+  static bool v = [] {
+    const char* e = getenv("BMR_WC_TAB");
+    return e ? atoi(e) != 0 : BMR_WC_TAB != 0;
+  }();
+  return v;
+}
+
 uint32_t map_wait_hint() {
   static uint32_t v = [] {
     const char* e = getenv("BMR_MAP_WAIT");

@@ -1,8 +1,10 @@
 """Aggregate ncu source-page metrics per CUDA source line (needs -lineinfo builds).
 usage: python tools/ncu_lines.py report.ncu-rep [topN]"""
-import csv, io, subprocess, sys
+import csv, io, os, sys
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+from ncu_csv import page
 rep = sys.argv[1]; top = int(sys.argv[2]) if len(sys.argv) > 2 else 30
-out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"], capture_output=True, text=True).stdout
+out = page(rep, "src")
 rows = list(csv.reader(io.StringIO(out)))
 agg = []
 cur_file = None; hdr = None; cur = None

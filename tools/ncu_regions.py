@@ -1,8 +1,9 @@
 """Share of warp instructions / stall samples per source region of the Map kernel.
 usage: python tools/ncu_regions.py report.ncu-rep"""
-import collections, csv, io, subprocess, sys
-out = subprocess.run(["ncu", "-i", sys.argv[1], "--page", "source", "--csv", "--print-source", "cuda,sass"],
-                     capture_output=True, text=True).stdout
+import collections, csv, io, os, sys
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+from ncu_csv import page
+out = page(sys.argv[1], "src")
 cur = hdr = None; data = []
 for r in csv.reader(io.StringIO(out)):
     if not r: continue

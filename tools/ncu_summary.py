@@ -5,8 +5,12 @@ usage: python tools/ncu_summary.py OUT.md report1.ncu-rep [report2 ...]
 """
 import csv
 import io
+import os
 import subprocess
 import sys
+
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+from ncu_csv import page  # noqa: E402
 from collections import defaultdict
 
 METRICS = [
@@ -36,15 +40,13 @@ METRICS = [
 
 
 def raw(rep):
-    out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
-    rows = list(csv.reader(io.StringIO(out)))
-    return rows[0], rows[1], rows[2:]
+    rows = list(csv.reader(io.StringIO(page(rep, "raw"))))
+    hi = next(i for i, r in enumerate(rows) if "Kernel Name" in r)
+    return rows[hi], rows[hi + 1], rows[hi + 2:]
 
 
 def top_stalls(rep, idx=0, n=6):
-    out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass",
-                          "--launch-skip", str(idx), "--launch-count", "1"],
-                         capture_output=True, text=True).stdout
+    out = page(rep, "sass", ["--launch-skip", str(idx), "--launch-count", "1"])
     rows = list(csv.reader(io.StringIO(out)))
     if len(rows) < 3:
         return []
