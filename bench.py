@@ -3,7 +3,7 @@
 % HBM roofline, vs the CPU oracle).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C5|C4|C3|C2|C1] [--impl reference]
-                    [--scaling weak|strong] [--mode SIO|SO|SI|G] [--no-map-combine]
+                    [--scaling weak|strong] [--mode SIO|SO|SI|G] [--no-map-combine] [--km-full-scan]
                     [--xchg nccl|caller|fused] [--units U]
 
 One step = one pass of the whole hot path (tile scheduling, stage-in,
@@ -295,6 +295,8 @@ def main():
     ap.add_argument("--mode", default="SIO", choices=["SIO", "SO", "SI", "G"],
                     help="Map memory-usage mode (PAPER.md L129-135 ablation, SURVEY §8(f) f-2)")
     ap.add_argument("--no-map-combine", action="store_true", help="literal north-star order (no Map combiner)")
+    ap.add_argument("--km-full-scan", action="store_true",
+                    help="KMeans: every point scans all k centroids (no bound test; the paper's literal Map)")
     ap.add_argument("--xchg", default="nccl", choices=["nccl", "caller", "fused"],
                     help="exchange at N > 1: libbmr's mr_group over NCCL (nccl), torch.distributed moving the "
                          "partition buffers (caller), or the fused Map flush into receive windows (fused, II)")
@@ -351,6 +353,8 @@ def main():
                   "G": bmr.FLAG_NO_SMEM_IN | bmr.FLAG_NO_SMEM_OUT}[args.mode]
     if args.no_map_combine:
         mode_flags |= bmr.FLAG_NO_MAP_COMBINE
+    if args.km_full_scan:
+        mode_flags |= bmr.FLAG_KM_FULL_SCAN
     if len(batches) > 1 and wl == "wc":
         mode_flags |= bmr.FLAG_BATCH_COMBINE   # per-batch group + combine (SURVEY §8(e) strong scaling)
     exchange = world > 1 and wl != "sm"       # SM is Map-only: no exchange
@@ -400,7 +404,8 @@ def main():
     acc = {k: 0.0 for k in ("map_ms", "hist_ms", "sort_ms", "seg_ms", "sort_keys_ms", "xchg_ms")}
     tot = {"pairs": 0, "sort_passes": 0, "kernel_launches": 0, "flushes": 0, "n_keys": 0, "pairs_hashed": 0,
            "sort_passes_keys": 0, "pairs_mid": 0, "sort_passes_mid": 0, "words_combined": 0, "pairs_partial": 0,
-           "collisions": 0, "xchg_send_bytes": 0, "replays": 0, "map_seal_waits": 0, "map_spills": 0}
+           "collisions": 0, "xchg_send_bytes": 0, "replays": 0, "map_seal_waits": 0, "map_spills": 0,
+           "km_points_scanned": 0}
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         barrier()
@@ -461,24 +466,41 @@ def main():
             "unit": "GB/s", "frac": round(ach / hbm, 4), "traffic": None, "bytes_per_launch": int(launch_bytes),
             "ms_per_launch": round(launch_ms, 4),
             "share_of_step": round((sort_ms_all if tkey == "k_onesweep" else per["map_ms"]) / ms, 3)}
+    km_stats = None
     if wl == "km" and tkey == "k_map":
-        # KMeans Map: FP32-pipe bound: per point k centroids x 8 dims x (sub + fma)
-        # lane-ops; peak = 148 SMs x 128 FP32 lanes x the max SM clock (FFMA / FFMA2 on the fma pipe)
+        # KMeans Map.  Full scan (--km-full-scan): FP32-pipe bound, per point k
+        # centroids x 8 dims x (sub + fma) lane-ops against 148 SMs x 128 FP32 lanes x the max SM
+        # clock.  Default (bound test): a shortcut point costs one centroid (16
+        # lane-ops), so the Map is bound by its HBM read; the FP32 figure is then reported on the
+        # lane-ops actually executed.
         k = len(inp["centroids"])
-        ops = 16.0 * k * n_rank / nmaps
+        scanned = tot["km_points_scanned"] / args.steps / nmaps
+        pts_launch = n_rank / nmaps
+        full = bool(args.km_full_scan) or scanned >= pts_launch
+        ops_exec = 16.0 * k * scanned + 16.0 * (pts_launch - scanned)
+        ops = 16.0 * k * pts_launch if full else ops_exec
         clk_mhz = 1965.0
         try:
             clk_mhz = float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["sm_max_mhz"])
         except Exception:
             pass
         peak_ops = 148 * 128 * clk_mhz * 1e6
-        roof_hbm = dict(roof)
-        roof = {"kernel": "k_map (KMeans distances)", "bound": "fp32",
-                "achieved": round(ops / (launch_ms / 1e3) / 1e12, 3), "peak": round(peak_ops / 1e12, 2),
+        fp32 = {"achieved": round(ops / (launch_ms / 1e3) / 1e12, 3), "peak": round(peak_ops / 1e12, 2),
                 "peak_kind": f"derived: 148 SMs x 128 FP32 lanes x {clk_mhz:.0f} MHz (FFMA/FFMA2, fma pipe)",
-                "unit": "Tlane-op/s", "frac": round(ops / (launch_ms / 1e3) / peak_ops, 4), "traffic": None,
-                "ops_per_launch": int(ops), "ms_per_launch": round(launch_ms, 4),
-                "share_of_step": roof["share_of_step"], "hbm": {k2: roof_hbm[k2] for k2 in ("achieved", "peak", "frac")}}
+                "unit": "Tlane-op/s", "frac": round(ops / (launch_ms / 1e3) / peak_ops, 4),
+                "ops_per_launch": int(ops), "ops_basis": "all k centroids per point" if full else
+                "executed: k centroids per scanned point, 1 per bound-test point"}
+        km_stats = {"full_scan": bool(args.km_full_scan), "points_scanned_per_launch": int(scanned),
+                    "bound_test_frac": round(1.0 - scanned / pts_launch, 6) if pts_launch else None}
+        if full:
+            roof_hbm = dict(roof)
+            roof = {"kernel": "k_map (KMeans distances)", "bound": "fp32", **{k2: fp32[k2] for k2 in (
+                "achieved", "peak", "peak_kind", "unit", "frac", "ops_per_launch")}, "traffic": None,
+                    "ms_per_launch": round(launch_ms, 4), "share_of_step": roof["share_of_step"],
+                    "hbm": {k2: roof_hbm[k2] for k2 in ("achieved", "peak", "frac")}}
+        else:
+            roof["kernel"] = "k_map (KMeans, bound test)"
+            roof["fp32"] = fp32
     traffic_p = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(traffic_p):
         tr = json.load(open(traffic_p)).get(cfg, {}).get(tkey)
@@ -571,7 +593,7 @@ def main():
             "replays": tot["replays"],
             "map_output_ring": {"seal_waits_per_step": tot["map_seal_waits"] / args.steps,
                                 "spills_per_step": tot["map_spills"] / args.steps},
-            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "kmeans": km_stats,
             "exchange": ({"kind": ("libbmr mr_group over NCCL (" + bmr.Comm.backend() + ")") if args.xchg == "nccl"
                           else "torch.distributed all_to_all_single (NCCL) of libbmr's partition buffers",
                           "ranks": world, "send_bytes_per_rank": int(tot["xchg_send_bytes"] / args.steps),

@@ -59,6 +59,12 @@ typedef enum { MR_WORDCOUNT = 1, MR_STRINGMATCH = 2, MR_KMEANS = 3, MR_INVINDEX 
 #define MR_FLAG_FORCE_SPILL     0x800u /* test hook: every warp result that overflows the output buffer is
                                           written straight to HBM (the a5 spill path), not only while the
                                           buffer ring is congested */
+#define MR_FLAG_KM_FULL_SCAN    0x1000u /* KM: every point scans all k centroids (the paper's literal Map); by
+                                          default a point whose distance to its lane's previous winner g is
+                                          below a quarter of the squared distance from g to its nearest other
+                                          centroid (with an fp32 rounding margin) is assigned g directly: the
+                                          triangle inequality makes every other centroid strictly farther, so
+                                          the assignment is the one the full scan computes */
 #define MR_FLAG_BATCH_COMBINE   0x400u /* WC: each mapped batch is grouped + reduced (combined) when the next
                                           one is mapped — mr_map then synchronises — and its (key, count)
                                           partials kept; mr_group merges the partials (exact sums).  For
@@ -133,6 +139,9 @@ typedef struct {
    * results written straight to HBM (the overflow spill) while the sealer waited */
   uint64_t map_seal_waits;
   uint64_t map_spills;
+  /* KMeans Map: points that scanned all k centroids (the rest were assigned by the bound test,
+   * MR_FLAG_KM_FULL_SCAN off) */
+  uint64_t km_points_scanned;
 } mr_stats;
 
 /* State machine: CREATED -> mr_map x k (batches append) -> mr_group -> mr_reduce -> mr_fetch

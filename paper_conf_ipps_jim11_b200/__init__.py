@@ -24,7 +24,7 @@ WORKLOADS = {"wc": WORDCOUNT, "sm": STRINGMATCH, "km": KMEANS, "ii": INVINDEX}
 FLAG_NO_SMEM_IN, FLAG_NO_SMEM_OUT, FLAG_FORCE_TINY_OUT = 0x01, 0x02, 0x04
 FLAG_WEAK_HASH_DEBUG, FLAG_VALIDATE, FLAG_NO_COMBINE = 0x08, 0x10, 0x20
 FLAG_PROFILE, FLAG_OWN_STREAM, FLAG_NO_MAP_COMBINE, FLAG_SM_LINES = 0x40, 0x80, 0x100, 0x200
-FLAG_BATCH_COMBINE, FLAG_FORCE_SPILL = 0x400, 0x800
+FLAG_BATCH_COMBINE, FLAG_FORCE_SPILL, FLAG_KM_FULL_SCAN = 0x400, 0x800, 0x1000
 
 STATUS = {0: "MR_OK", 1: "MR_ERR_INVALID", 2: "MR_ERR_STATE", 3: "MR_ERR_OOM", 4: "MR_ERR_OVERFLOW",
           5: "MR_ERR_CUDA", 6: "MR_ERR_NCCL", 7: "MR_ERR_UNSUPPORTED"}
@@ -151,7 +151,8 @@ class Stats(C.Structure):
                 ("pairs_mid", C.c_uint64), ("sort_passes_mid", C.c_uint64),
                 ("pairs_partial", C.c_uint64), ("words_combined", C.c_uint64),
                 ("xchg_send_bytes", C.c_uint64), ("xchg_recv_bytes", C.c_uint64), ("xchg_ms", C.c_double),
-                ("map_seal_waits", C.c_uint64), ("map_spills", C.c_uint64)]
+                ("map_seal_waits", C.c_uint64), ("map_spills", C.c_uint64),
+                ("km_points_scanned", C.c_uint64)]
 
 
 _LIB = None

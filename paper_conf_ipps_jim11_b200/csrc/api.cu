@@ -1265,6 +1265,7 @@ mr_status mr_group(mr_job* job) {
   job->stats.flushes = hs->flushes;
   job->stats.map_seal_waits = hs->seal_waits;
   job->stats.map_spills = hs->spills;
+  job->stats.km_points_scanned = hs->km_scanned;
   if (m_total >= (1ULL << 32) - 1 || mb >= (1ULL << 32) - 1 || mc >= (1ULL << 32) - 1)
     return fail(job, MR_ERR_UNSUPPORTED, ">= 2^32 intermediate pairs in one group");
   if (job->km_comb()) {   // KM combiner: the Map produced the cluster sums; nothing to group

@@ -39,6 +39,7 @@ struct DevState {
   unsigned long long long_fail;      // WC long-word table: inserts that found no slot (-> grow + replay)
   unsigned long long seal_waits;     // Map: seals that waited for a buffer still flushing (ring full)
   unsigned long long spills;         // Map: warp results written straight to HBM while the ring was full
+  unsigned long long km_scanned;     // KMeans Map: points that scanned every centroid (bound test failed / off)
 };
 constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u, kErrTileCap = 4u, kErrNullRecords = 8u,
                        kErrMidTable = 16u, kErrLongTable = 32u;

@@ -82,6 +82,13 @@ constexpr int kNMapText = 24;
 #ifndef BMR_II_OUT_BYTES
 #define BMR_II_OUT_BYTES 8192   // InvertedIndex output buffer bytes (x kNOut; 24-B pairs, ~1 per 500 B)
 #endif
+#ifndef BMR_KM_STAGES
+#define BMR_KM_STAGES 8      // KMeans stages in flight per SM (round 3: with the bound test the KM Map is
+                             // read-bound, 4 x 16 KiB in flight per SM capped it at ~1/3 of HBM)
+#endif
+#ifndef BMR_KM_OUT_BYTES
+#define BMR_KM_OUT_BYTES 4096   // KMeans output buffer bytes (x kNOut; only the sorted path, NO_MAP_COMBINE, emits)
+#endif
 #ifndef BMR_II_NMAP
 #define BMR_II_NMAP 24   // InvertedIndex map warps
 #endif
@@ -137,16 +144,17 @@ template <int W>
 struct Cfg {
   // StringMatch (read-bound, almost no output, lazy record directory below: no offsets or bitmap
   // regions): 8 stages of bytes in flight
-  static constexpr int kStages = (W == kSM) ? BMR_SM_STAGES : (W == kII) ? BMR_II_STAGES : 4;
-  static constexpr int kOffCap = (W == kSM) ? 0 : (W == kWC) ? BMR_WC_OFFCAP : 1024;   // record offsets staged per tile (more: read from global)
+  static constexpr int kStages = (W == kSM) ? BMR_SM_STAGES : (W == kII) ? BMR_II_STAGES : (W == kKM) ? BMR_KM_STAGES : 4;
+  // record offsets staged per tile (more: read from global); KM has fixed-stride records
+  static constexpr int kOffCap = (W == kSM || W == kKM) ? 0 : (W == kWC) ? BMR_WC_OFFCAP : 1024;
   // StringMatch reads the record directory lazily: record boundaries matter only where the
   // pattern's first byte matches (planted, rare), so no offsets are staged and no bitmap is built;
   // a candidate checks for a record start inside its 16 bytes by a binary search over the tile's
   // offsets slice in global memory.  The producers only issue the byte TMA.
   static constexpr bool kLazyDir = (W == kSM);
-  static constexpr int kOffBytes = (W == kSM) ? 0 : ((kOffCap + 2) * 8 + 127) / 128 * 128;
-  static constexpr int kBits = (W == kSM) ? 0 : kBitBytes;   // record-start bitmap bytes per stage
-  static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? BMR_WC_OUT_BYTES : (W == kII) ? BMR_II_OUT_BYTES : 20480;   // bytes per output buffer
+  static constexpr int kOffBytes = (W == kSM || W == kKM) ? 0 : ((kOffCap + 2) * 8 + 127) / 128 * 128;
+  static constexpr int kBits = (W == kSM || W == kKM) ? 0 : kBitBytes;   // record-start bitmap bytes per stage
+  static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? BMR_WC_OUT_BYTES : (W == kII) ? BMR_II_OUT_BYTES : BMR_KM_OUT_BYTES;   // bytes per output buffer
   // the producer builds the bitmap of tile it - kLag right after issuing tile it: kLag stages of
   // TMA traffic stay in flight per SM while one stage is being consumed
   static constexpr int kLag = kStages - 2;
@@ -183,6 +191,15 @@ constexpr int kKmPts = kT / 32;                // 512 points per KM tile
 // KM combiner (k <= kKmCombMax): per-warp fp32 accumulators [kNMap][64][8] + counts [kNMap][64]
 // in the (otherwise unused for KM) offsets + bitmap stage regions
 constexpr int kKmCombMax = 64;
+// KM bound test (MR_FLAG_KM_FULL_SCAN off): for k <= kKmBoundMax the CTA keeps a row-layout copy of
+// the centroids and s2[g] = (squared distance from centroid g to its nearest other centroid,
+// rounded down) after the paired copy.  A point whose fp32 distance d_g to its lane's previous
+// winner g satisfies 4 d_g (1 + 1e-5) < s2[g] is assigned g: exactly, ||x - c_g|| < s/2 gives
+// ||x - c_j|| >= s - ||x - c_g|| > ||x - c_g|| for every j != g (triangle inequality), and the
+// 1e-5 margin exceeds the relative error of the two fp32 distance chains (<= ~10 ulp each), so
+// the fp32 d_j the full scan would compute are all strictly greater than d_g.
+constexpr int kKmBoundMax = 128;
+constexpr float kKmBoundFactor = 4.00004f;
 constexpr int kKmWaccBytes = kNMap * kKmCombMax * 8 * 4;
 
 static_assert(kLead + kT + kHalo + 32 <= kStageBytes, "stage too small");
@@ -229,15 +246,15 @@ struct Layout {
   static constexpr int xq = hq + nmap<W>() * Cfg<W>::kHashQ * 4;  // nmap x kXQ x 4 (WC)
   static constexpr int comb = xq + nmap<W>() * Cfg<W>::kXQ * 4;   // kCombSlots x 8 (WC)
   static constexpr int lq = comb + Cfg<W>::kCombSlots * 8;        // nmap x kLQ x 24 (WC)
-  static constexpr int cent = lq + nmap<W>() * Cfg<W>::kLQ * 24;  // KM centroids
+  static constexpr int kmacc = lq + nmap<W>() * Cfg<W>::kLQ * 24;  // KM combiner: per-warp fp32 sums + counts
+  static constexpr int cent = kmacc + ((W == kKM) ? kKmWaccBytes + kNMap * kKmCombMax * 4 : 0);   // KM centroids
   static_assert(sizeof(OutCtl) <= hdr, "OutCtl overlaps the stage headers");
 };
 static_assert(64 % kNOut == 0, "6-bit generation counter must wrap on a buffer boundary");
 static_assert(Layout<kWC>::cent <= 232448 && Layout<kSM>::cent <= 232448 && Layout<kII>::cent <= 232448 &&
                   Layout<kKM>::cent + 1024 * 32 <= 232448,
               "SMEM layout exceeds 227 KB per CTA");
-static_assert(kKmWaccBytes + kNMap * kKmCombMax * 4 <= Layout<kKM>::out - Layout<kKM>::offs,
-              "KM combiner accumulators exceed the offsets + bitmap regions");
+
 
 // Output-buffer formats.  SM / KM / II: SoA runs [keys | krefs | values] of kCap entries.
 // WC: exact-key entries (u32 key) fill the buffer from the bottom, queued long-word entries (u64
@@ -319,6 +336,7 @@ struct Params {
   uint64_t* lkeys;         // WC: words of 9..16 symbols counted in an open-addressing table of their
   uint32_t* lcnt;          //   16 zero-padded key bytes (2^lbits slots); nullptr: hashed stream
   uint32_t lbits;
+  uint32_t km_bound;       // KM: the exact bound test before the full centroid scan (kKmBoundMax)
 };
 
 // Idle wait of a role warp on an mbarrier phase (map warps on a staged tile, producers on a free
@@ -2414,8 +2432,8 @@ __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl
   }
 }
 
-// V: 1 = the WordCount table-mode instantiation (wc_window_tab), a kernel of its own so that the
-// two window paths do not share one register allocation
+// V: 1 = the WordCount table-mode instantiation (wc_window_tab) / the KMeans bound-test
+// instantiation, kernels of their own so that the two paths do not share one register allocation
 template <int W, int V>
 __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   constexpr int kStages = Cfg<W>::kStages;
@@ -2442,6 +2460,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   // (P.dyn == 0: static order, map warp w takes windows w, w + nmap, w + 2 nmap, ... of the CTA's
   // window sequence)
   uint32_t kseq = 0, have_it = ~0u;
+  uint32_t km_guess = W == kKM && P.k ? lane % P.k : 0u;   // KM: this lane's previous winner (bound test)
   uint32_t qn = 0;   // II: queued URLs of this warp (ii_drain)
   StageHdr hd{};
   bool fast = W == kSM && !P.dyn;
@@ -2493,7 +2512,28 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
                           static_cast<uint64_t>(tid) * 32;
       float x[8];
       uint32_t best = 0;
-      if (valid) {
+      bool scan = valid;
+      if (V == 1 && valid) {   // the lane's previous winner first: bound test (kKmBoundMax)
+        const float4* cg = reinterpret_cast<const float4*>(cent + P.k * 8 + km_guess * 8);
+        const float4 a = P.so ? __ldg(reinterpret_cast<const float4*>(P.rec + i * 32)) : reinterpret_cast<const float4*>(pt)[0];
+        const float4 b = P.so ? __ldg(reinterpret_cast<const float4*>(P.rec + i * 32) + 1) : reinterpret_cast<const float4*>(pt)[1];
+        const float4 g0 = cg[0], g1 = cg[1];
+        float d = 0.0f, e;
+        e = __fsub_rn(a.x, g0.x); d = __fmaf_rn(e, e, d);
+        e = __fsub_rn(a.y, g0.y); d = __fmaf_rn(e, e, d);
+        e = __fsub_rn(a.z, g0.z); d = __fmaf_rn(e, e, d);
+        e = __fsub_rn(a.w, g0.w); d = __fmaf_rn(e, e, d);
+        e = __fsub_rn(b.x, g1.x); d = __fmaf_rn(e, e, d);
+        e = __fsub_rn(b.y, g1.y); d = __fmaf_rn(e, e, d);
+        e = __fsub_rn(b.z, g1.z); d = __fmaf_rn(e, e, d);
+        e = __fsub_rn(b.w, g1.w); d = __fmaf_rn(e, e, d);
+        if (d * kKmBoundFactor < cent[P.k * 16 + km_guess]) {
+          best = km_guess;
+          scan = false;
+          x[0] = a.x; x[1] = a.y; x[2] = a.z; x[3] = a.w; x[4] = b.x; x[5] = b.y; x[6] = b.z; x[7] = b.w;
+        }
+      }
+      if (scan) {
         const float4* src = P.so ? reinterpret_cast<const float4*>(P.rec + i * 32) : reinterpret_cast<const float4*>(pt);
         const float4 a = P.so ? __ldg(src) : src[0];
         const float4 b = P.so ? __ldg(src + 1) : src[1];
@@ -2533,23 +2573,45 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
           if (first || d < bd) { bd = d; best = j; }
         }
       }
+      if (valid) km_guess = best;   // the next point of this lane starts from this winner
       const uint32_t m = __ballot_sync(kFull, valid);
+      {
+        const uint32_t ms = __ballot_sync(kFull, scan);
+        if (lane == 0 && ms) atomicAdd(&P.st->km_scanned, static_cast<unsigned long long>(__popc(ms)));
+      }
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[s]);   // stage no longer read by this warp
       if (P.comb) {
         // f-1 combiner: fp32 per-warp cluster sums of this tile (<= 32 points per partial, as
         // in the sorted Reduce, reading 5), folded into lane-owned fp64 registers
-        float* wacc = reinterpret_cast<float*>(smem + Layout<W>::offs) + warp * (kKmCombMax * 8);
-        uint32_t* wcnt = reinterpret_cast<uint32_t*>(smem + Layout<W>::offs + kKmWaccBytes) + warp * kKmCombMax;
+        float* wacc = reinterpret_cast<float*>(smem + Layout<W>::kmacc) + warp * (kKmCombMax * 8);
+        uint32_t* wcnt = reinterpret_cast<uint32_t*>(smem + Layout<W>::kmacc + kKmWaccBytes) + warp * kKmCombMax;
         // lanes with the same cluster form a match group; the group's members add their point
         // in rank order, one member per round (plain read-modify-write: no two lanes of a round
         // share a cluster) — shared-memory fp32 atomics are CAS loops on sm_100a (ATOMS.CAST.SPIN,
         // ncu round 2: 19% of the KM Map's instructions, 38% of its stall samples)
-        const uint32_t grp = __match_any_sync(kFull, valid ? best : 0xFFFFFFFFu);
+        // A point of one of the lane's own clusters (lane, lane + 32: the clusters whose fp64
+        // accumulators it holds) is added straight into those registers (fp64: at least as exact
+        // as the fp32 partials of reading 5); only the other points take the SMEM match rounds.
+        const bool own = valid && (best & 31u) == lane && best < static_cast<uint32_t>(kKmCombMax);
+        if (own) {
+          if (best < 32u) {
+            kcnt[0] += 1;
+#pragma unroll
+            for (int t = 0; t < 8; ++t) kacc[0][t] += static_cast<double>(x[t]);
+          } else {
+            kcnt[1] += 1;
+#pragma unroll
+            for (int t = 0; t < 8; ++t) kacc[1][t] += static_cast<double>(x[t]);
+          }
+        }
+        const bool other = valid && !own;
+        if (__any_sync(kFull, other)) {
+        const uint32_t grp = __match_any_sync(kFull, other ? best : 0xFFFFFFFFu);
         const uint32_t rank = __popc(grp & lanemask_lt());
-        const uint32_t rounds = __reduce_max_sync(kFull, valid ? static_cast<uint32_t>(__popc(grp)) : 0u);
+        const uint32_t rounds = __reduce_max_sync(kFull, other ? static_cast<uint32_t>(__popc(grp)) : 0u);
         for (uint32_t r = 0; r < rounds; ++r) {
-          if (valid && rank == r) {
+          if (other && rank == r) {
 #pragma unroll
             for (int t = 0; t < 8; ++t) wacc[t * kKmCombMax + best] += x[t];   // [dim][cluster]: no bank conflicts
             wcnt[best] += 1u;
@@ -2573,6 +2635,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
           }
         }
         __syncwarp();
+        }
       } else if (m && P.si) {   // SI / G ablation: global append per warp result
         unsigned long long gb = 0;
         if (lane == 0) gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(__popc(m)));
@@ -2714,7 +2777,7 @@ __global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
   }
   if constexpr (W == kKM) {
     if (P.comb) {
-      uint32_t* z = reinterpret_cast<uint32_t*>(smem + Layout<W>::offs);
+      uint32_t* z = reinterpret_cast<uint32_t*>(smem + Layout<W>::kmacc);
       for (uint32_t i = threadIdx.x; i < static_cast<uint32_t>(kKmWaccBytes / 4 + kNMap * kKmCombMax); i += blockDim.x)
         z[i] = 0;
     }
@@ -2724,6 +2787,24 @@ __global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
       const uint32_t j = i / 8, t = i % 8;
       const uint32_t kp = P.k & ~1u;
       cent[j < kp ? ((j & ~1u) * 8 + t * 2 + (j & 1u)) : i] = P.cent[i];
+      if (P.km_bound) cent[P.k * 8 + i] = P.cent[i];   // row-layout copy (the bound test's centroid g)
+    }
+    if (P.km_bound) {   // s2[g]: squared distance to the nearest other centroid, fp64, rounded down
+      float* s2 = cent + P.k * 16;
+      for (uint32_t g = threadIdx.x; g < P.k; g += blockDim.x) {
+        double m = 1.0 / 0.0;
+        for (uint32_t j = 0; j < P.k; ++j) {
+          if (j == g) continue;
+          double d = 0.0;
+          for (int t = 0; t < 8; ++t) {
+            const double e = static_cast<double>(P.cent[g * 8 + t]) - static_cast<double>(P.cent[j * 8 + t]);
+            d += e * e;
+          }
+          m = d < m ? d : m;
+        }
+        const float f = __double2float_rd(m * (1.0 - 1e-12));
+        s2[g] = f < 1e-30f ? 0.0f : f;   // coincident / nearly coincident centroids: never take the shortcut
+      }
     }
   }
   __syncthreads();
@@ -2833,6 +2914,7 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.lkeys = (BMR_LTAB && P.xtab) ? a.out.lkeys : nullptr;
   P.lcnt = (BMR_LTAB && P.xtab) ? a.out.lcnt : nullptr;
   P.lbits = a.out.lbits;
+  P.km_bound = (W == kKM && !(a.flags & 0x1000u) && a.k <= static_cast<uint32_t>(kKmBoundMax)) ? 1u : 0u;   // MR_FLAG_KM_FULL_SCAN
   if (W == kKM && P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>(std::min<uint64_t>((a.tb_cap + 255) / 256 + 1, 8ULL * num_sms));
@@ -2840,12 +2922,15 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
                                          a.desc, a.tile_bounds, &a.st->err);
     count_launch();
   }
-  const size_t smem = Layout<W>::cent + (W == kKM ? static_cast<size_t>(a.k) * 32 : 0);
+  const size_t smem = Layout<W>::cent + (W == kKM ? static_cast<size_t>(a.k) * (P.km_bound ? 68 : 32) : 0);
   // WordCount table mode (the fast SIO path with the L2 tables): its own instantiation
   const bool tab = W == kWC && map_wc_tab() && P.xtab && P.mkeys && P.lkeys && P.comb && !P.so && !P.si && P.wc_bal && P.dyn && P.wc_fast;
   auto kern = k_map<W, 0>;
   if constexpr (W == kWC) {
     if (tab) kern = k_map<W, 1>;
+  }
+  if constexpr (W == kKM) {   // the bound-test instantiation (the full scan keeps its own registers)
+    if (P.km_bound) kern = k_map<W, 1>;
   }
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
   if (e != cudaSuccess) return e;

@@ -477,6 +477,52 @@ def test_km_combiner_multibatch():
     assert np.all(np.abs(cg.astype(np.float64) - co) <= KM_RTOL * np.maximum(np.abs(co), floor[None, :]))
 
 
+def km_pair(pts, cen, flags=0):
+    data = pts.view(np.uint8).reshape(-1)
+    r, _ = gpu("km", [(data, None, len(pts))], centroids=cen, flags=flags)
+    return decode("km", r)
+
+
+def _near_bisector_points(rng, cen, n):
+    # points on / just off the bisector of random centroid pairs (the bound test must fail there
+    # or decide exactly as the full scan): m + t (c_b - c_a) for t in a few ulps-to-1e-4 around 0
+    a = rng.integers(0, len(cen), n)
+    b = (a + 1 + rng.integers(0, len(cen) - 1, n)) % len(cen)
+    m = (cen[a].astype(np.float64) + cen[b]) / 2
+    t = rng.choice([0.0, 1e-7, -1e-7, 1e-6, -1e-6, 1e-5, -1e-5, 1e-4, -1e-4, 0.3, -0.3], n)
+    return (m + t[:, None] * (cen[b].astype(np.float64) - cen[a])).astype(np.float32)
+
+
+@pytest.mark.parametrize("case", ["blobs", "bisectors", "duplicates", "k1"])
+def test_km_bound_test_equals_full_scan(case):
+    # the default Map assigns a point to its lane's previous winner when the triangle-inequality
+    # bound holds; MR_FLAG_KM_FULL_SCAN scans every centroid.  Same assignments ->
+    # bit-identical output, and both equal the oracle (counts exact).
+    rng = np.random.default_rng(7)
+    spec = pygen.KMSpec()
+    if case == "blobs":
+        pts = pygen.host_km(spec, 32 * 2000 + 9)
+        cen = pygen.km_centres(spec)[1]
+    elif case == "bisectors":
+        cen = (rng.integers(-4096, 4096, size=(32, 8)) / 64.0).astype(np.float32)
+        pts = _near_bisector_points(rng, cen, 40_000)
+        pts[::7] = cen[rng.integers(0, 32, len(pts[::7]))]   # exactly on a centroid
+    elif case == "duplicates":
+        cen = (rng.integers(-64, 64, size=(16, 8))).astype(np.float32)
+        cen[5] = cen[3]
+        cen[9] = cen[3]                                      # coincident centroids: ties -> lowest id
+        pts = np.concatenate([cen[rng.integers(0, 16, 5000)] + rng.normal(0, 2, (5000, 8)),
+                              _near_bisector_points(rng, cen, 5000)]).astype(np.float32)
+    else:
+        cen = np.array([[1.5] * 8], np.float32)
+        pts = rng.normal(0, 10, (10_000, 8)).astype(np.float32)
+    cb, nb = km_pair(pts, cen)
+    cf, nf = km_pair(pts, cen, bmr.FLAG_KM_FULL_SCAN)
+    assert np.array_equal(nb, nf)
+    assert np.array_equal(cb.view(np.uint32), cf.view(np.uint32))
+    km_check(pts, cen)
+
+
 def test_km_empty_and_tiny():
     cen = np.array([[0] * 8, [100] * 8], np.float32)
     km_check(np.zeros((0, 8), np.float32), cen)
