@@ -542,22 +542,23 @@ __device__ __forceinline__ uint64_t bytes8_at(const Params& P, const TileView& t
   return b;
 }
 
+// Sort key of key bytes in global memory (8-byte aligned loads): out of line, so that the
+// register allocation of the Map loops does not carry it (II keys every URL from global memory in
+// its drain; WC only words that leave the stage).
+__device__ __noinline__ uint64_t key_global(const uint8_t* p, uint32_t len, uint64_t seed, bool weak, uint32_t bits) {
+  if (len <= inline_max(bits)) return inline_key(load8(p, len), len, bits);
+  return hashed_key(hash_bytes_g(p, len, seed), weak, bits);
+}
 // Sort key of the key bytes [q, q + len): inline when short, else the hash (common.cuh).
 __device__ __forceinline__ uint64_t key_at(const Params& P, const TileView& tv, long long q, uint32_t len) {
   const bool in_stage = (q + static_cast<long long>(len) <= tv.stg_hi) && (q - tv.sbase + len + 12 <= kStageBytes);
+  if (!in_stage) return key_global(P.rec + q, len, P.hash_seed, (P.flags & 8u) != 0, P.key_bits);
+  const uint32_t i = static_cast<uint32_t>(q - tv.sbase);
   if (len <= inline_max(P.key_bits)) {
-    uint64_t b = 0;
-    if (in_stage) {
-      const uint32_t i = static_cast<uint32_t>(q - tv.sbase);
-      b = static_cast<uint64_t>(smem_word_at(tv.sb, i)) | (static_cast<uint64_t>(smem_word_at(tv.sb, i + 4)) << 32);
-    } else {
-      for (uint32_t k = 0; k < len; ++k) b |= static_cast<uint64_t>(P.rec[q + k]) << (8 * k);
-    }
+    const uint64_t b = static_cast<uint64_t>(smem_word_at(tv.sb, i)) | (static_cast<uint64_t>(smem_word_at(tv.sb, i + 4)) << 32);
     return inline_key(b, len, P.key_bits);
   }
-  const uint64_t h = in_stage ? hash_smem(tv.sb, static_cast<uint32_t>(q - tv.sbase), len, P.hash_seed)
-                              : hash_bytes(P.rec + q, len, P.hash_seed);
-  return hashed_key(h, (P.flags & 8u) != 0, P.key_bits);
+  return hashed_key(hash_smem(tv.sb, i, len, P.hash_seed), (P.flags & 8u) != 0, P.key_bits);
 }
 
 // ---------------------------------------------------------------- emit allocator
@@ -707,8 +708,10 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc, uint32_t 
     // rarely and the polls were 3% of the Map's instructions, ncu C5 round 2)
     uint32_t backoff = 0;
     while (!mbar_try_wait_hint(&oc->req[h], (f / kNOut) & 1u, 2000)) {
-      if (backoff) __nanosleep(backoff);
-      backoff = min(backoff ? 2 * backoff : 64u, kFlushBackoffNs);
+      if (W == kWC && P.xtab) {   // (table mode only: the other workloads flush continuously)
+        if (backoff) __nanosleep(backoff);
+        backoff = min(backoff ? 2 * backoff : 64u, kFlushBackoffNs);
+      }
       if (NF > 1 && ld_acquire_cta_shared_u32(&oc->is_final) && ld_acquire_cta_shared_u32(&oc->final_seq) < f) {
         past = true;
         break;
@@ -1931,7 +1934,9 @@ __device__ __forceinline__ void ii_window(const Params& P, OutCtl* oc, uint8_t* 
       q = find_quote(P, tv, max(q0, p0w + kWin), p0 + j);
     }
     if (q > q0 && nm < 2) {
-      aux[nm++] = static_cast<uint32_t>(q - q0);
+      if (nm == 0) aux[0] = static_cast<uint32_t>(q - q0);   // (no dynamic index: registers, not local memory)
+      else aux[1] = static_cast<uint32_t>(q - q0);
+      ++nm;
       emit_mask |= 1u << j;
     }
   }
@@ -2163,7 +2168,9 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
         q = find_quote(P, tv, max(q0, wp + kWin), p0 + j);
       }
       if (q > q0 && nm < 2) {
-        aux[nm++] = static_cast<uint32_t>(q - q0);
+        if (nm == 0) aux[0] = static_cast<uint32_t>(q - q0);   // (no dynamic index: registers, not local memory)
+      else aux[1] = static_cast<uint32_t>(q - q0);
+      ++nm;
         emit_mask |= 1u << j;
       }
     }
@@ -2432,6 +2439,164 @@ __device__ __noinline__ void sm_fast_loop(const Params& P, uint8_t* smem, OutCtl
   }
 }
 
+// KMeans f-1 combiner step of one warp (one point per valid lane, cluster `best`): a point of the
+// lane's own cluster (cluster == lane; the lane holds the fp64 accumulators kacc of clusters lane
+// and lane + 32) is added to the lane's fp32 partial of it, folded into kacc every 32 points
+// (<= 32 values per fp32 partial, as in the sorted Reduce: DESIGN.md reading 5); the other points
+// are summed into per-warp fp32 SMEM partials of this tile, which are folded into their owner
+// lanes' kacc right away.  Lanes with the same cluster form a match group and add in rank order,
+// one member per round (plain read-modify-write: no two lanes of a round share a cluster) —
+// shared-memory fp32 atomics are CAS loops on sm_100a (ATOMS.CAST.SPIN, ncu round 2: 19% of the
+// KM Map's instructions, 38% of its stall samples).
+__device__ __forceinline__ void km_flush_partial(double (&acc)[8], unsigned long long& cnt, float (&pa)[8],
+                                                 uint32_t& pn) {
+  cnt += pn;
+#pragma unroll
+  for (int t = 0; t < 8; ++t) {
+    acc[t] += static_cast<double>(pa[t]);
+    pa[t] = 0.0f;
+  }
+  pn = 0;
+}
+__device__ __forceinline__ void km_combine(uint8_t* smem, uint32_t warp, uint32_t lane, bool valid, uint32_t best,
+                                           const float (&x)[8], uint32_t k, double (&kacc)[kKmCombMax / 32][8],
+                                           unsigned long long (&kcnt)[kKmCombMax / 32], float (&pacc)[8],
+                                           uint32_t& pn) {
+  const bool own = valid && best == lane;
+  if (own) {
+#pragma unroll
+    for (int t = 0; t < 8; ++t) pacc[t] += x[t];
+    if (++pn == 32u) km_flush_partial(kacc[0], kcnt[0], pacc, pn);
+  }
+  const bool other = valid && !own;
+  if (!__any_sync(kFull, other)) return;
+  float* wacc = reinterpret_cast<float*>(smem + Layout<kKM>::kmacc) + warp * (kKmCombMax * 8);
+  uint32_t* wcnt = reinterpret_cast<uint32_t*>(smem + Layout<kKM>::kmacc + kKmWaccBytes) + warp * kKmCombMax;
+  const uint32_t grp = __match_any_sync(kFull, other ? best : 0xFFFFFFFFu);
+  const uint32_t rank = __popc(grp & lanemask_lt());
+  const uint32_t rounds = __reduce_max_sync(kFull, other ? static_cast<uint32_t>(__popc(grp)) : 0u);
+  for (uint32_t r = 0; r < rounds; ++r) {
+    if (other && rank == r) {
+#pragma unroll
+      for (int t = 0; t < 8; ++t) wacc[t * kKmCombMax + best] += x[t];   // [dim][cluster]: no bank conflicts
+      wcnt[best] += 1u;
+    }
+    __syncwarp();
+  }
+#pragma unroll
+  for (int q = 0; q < kKmCombMax / 32; ++q) {
+    const uint32_t c = lane + 32 * q;
+    if (c < k) {
+      const uint32_t nc = wcnt[c];
+      if (nc) {
+        wcnt[c] = 0;
+        kcnt[q] += nc;
+#pragma unroll
+        for (int t = 0; t < 8; ++t) {
+          kacc[q][t] += static_cast<double>(wacc[t * kKmCombMax + c]);
+          wacc[t * kKmCombMax + c] = 0.0f;
+        }
+      }
+    }
+  }
+  __syncwarp();
+}
+
+// KMeans full scan of one point (reading 4): fp32 RN chain d = fma(x_t - c_t, x_t - c_t, d) over
+// t = 0..7, ties -> lowest j.  Two centroids per instruction with packed FADD2/FFMA2 (each lane of
+// the pair performs exactly the scalar RN operations, so the result is bit-identical); cent is
+// the pair layout (centroids 2p, 2p+1 interleaved per coordinate), an odd last centroid unpaired.
+__device__ __forceinline__ uint32_t km_scan(const float (&x)[8], const float* cent, uint32_t k) {
+  uint32_t best = 0;
+  float bd = 0.0f;
+  uint64_t X[8];
+#pragma unroll
+  for (int t = 0; t < 8; ++t) X[t] = f2pack(x[t], x[t]);
+  const uint32_t kp = k & ~1u;
+  bool first = true;
+#pragma unroll kKmUnroll
+  for (uint32_t j = 0; j < kp; j += 2) {
+    const ulonglong2* cp = reinterpret_cast<const ulonglong2*>(cent + j * 8);   // pair layout
+    const ulonglong2 q0 = cp[0], q1 = cp[1], q2 = cp[2], q3 = cp[3];
+    const uint64_t C[8] = {q0.x, q0.y, q1.x, q1.y, q2.x, q2.y, q3.x, q3.y};
+    uint64_t D = 0;
+#pragma unroll
+    for (int t = 0; t < 8; ++t) {
+      const uint64_t E = f2sub(X[t], C[t]);
+      D = f2fma(E, E, D);
+    }
+    float d0, d1;
+    f2unpack(D, d0, d1);
+    if (first || d0 < bd) { bd = d0; best = j; }
+    first = false;
+    if (d1 < bd) { bd = d1; best = j + 1; }
+  }
+  if (k & 1u) {
+    const uint32_t j = k - 1;
+    const float* c = cent + j * 8;   // last centroid stored unpaired
+    float d = 0.0f, e;
+#pragma unroll
+    for (int t = 0; t < 8; ++t) { e = __fsub_rn(x[t], c[t]); d = __fmaf_rn(e, e, d); }
+    if (first || d < bd) { bd = d; best = j; }
+  }
+  return best;
+}
+
+// KMeans Map, bound-test instantiation with the combiner in SIO mode (the default C3 path): one
+// point per map lane per tile; the lane's previous winner g first — if 4 d_g (1 + 1e-5) < s2[g]
+// the point is g's (reading 12), else the full scan.  No ablation branches in the loop.
+__device__ void km_bound_loop(const Params& P, uint8_t* smem, double (&kacc)[kKmCombMax / 32][8],
+                              unsigned long long (&kcnt)[kKmCombMax / 32], float (&pacc)[8], uint32_t& pn,
+                              uint32_t guess) {
+  constexpr int W = kKM;
+  constexpr int kStages = Cfg<W>::kStages;
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31, tid = threadIdx.x;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
+  uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
+  const float* cent = reinterpret_cast<const float*>(smem + Layout<W>::cent);
+  const uint32_t k = P.k;
+  const float* crow = cent + k * 8;
+  const float* s2 = cent + k * 16;
+  const uint32_t phase16 = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(P.rec) & 15u);
+  unsigned long long scanned = 0;
+  for (uint32_t it = 0;; ++it) {
+    const uint32_t s = it % kStages;
+    mbar_wait(&full[s], (it / kStages) & 1u);
+    const StageHdr* hd = reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
+    const long long t = hd->t;
+    if (t < 0) break;
+    const long long lo = hd->lo, hi = hd->hi;
+    const bool valid = lo + static_cast<long long>(tid) < hi;
+    // stage byte offset of the first point: the source's 16-B phase (points are 32 B)
+    const float4* pt = reinterpret_cast<const float4*>(smem + Layout<W>::bytes + s * kStageBytes +
+                                                       ((phase16 + static_cast<uint32_t>(lo) * 32u) & 15u) + tid * 32u);
+    float x[8];
+    uint32_t best = guess;
+    bool scan = false;
+    if (valid) {
+      const float4 a = pt[0], b = pt[1];
+      x[0] = a.x; x[1] = a.y; x[2] = a.z; x[3] = a.w; x[4] = b.x; x[5] = b.y; x[6] = b.z; x[7] = b.w;
+      const float4* cg = reinterpret_cast<const float4*>(crow + guess * 8);
+      const float4 g0 = cg[0], g1 = cg[1];
+      const float c[8] = {g0.x, g0.y, g0.z, g0.w, g1.x, g1.y, g1.z, g1.w};
+      float d = 0.0f;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const float e = __fsub_rn(x[q], c[q]);
+        d = __fmaf_rn(e, e, d);
+      }
+      scan = !(d * kKmBoundFactor < s2[guess]);
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[s]);   // x is in registers: the stage can go
+    if (scan) best = km_scan(x, cent, k);
+    scanned += __popc(__ballot_sync(kFull, scan));
+    if (valid) guess = best;
+    km_combine(smem, warp, lane, valid, best, x, k, kacc, kcnt, pacc, pn);
+  }
+  if (lane == 0 && scanned) atomicAdd(&P.st->km_scanned, scanned);
+}
+
 // V: 1 = the WordCount table-mode instantiation (wc_window_tab) / the KMeans bound-test
 // instantiation, kernels of their own so that the two paths do not share one register allocation
 template <int W, int V>
@@ -2461,6 +2626,10 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   // window sequence)
   uint32_t kseq = 0, have_it = ~0u;
   uint32_t km_guess = W == kKM && P.k ? lane % P.k : 0u;   // KM: this lane's previous winner (bound test)
+  float pacc[8];   // KM: fp32 partial of the lane's own cluster (km_combine)
+  uint32_t pn = 0;
+#pragma unroll
+  for (int t = 0; t < 8; ++t) pacc[t] = 0.0f;
   uint32_t qn = 0;   // II: queued URLs of this warp (ii_drain)
   StageHdr hd{};
   bool fast = W == kSM && !P.dyn;
@@ -2480,6 +2649,10 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   if constexpr (W == kII) {
     fast = !P.so && !P.si && P.dyn && P.wc_fast;
     if (fast) ii_map_loop(P, smem, oc, qn);
+  }
+  if constexpr (W == kKM && V == 1) {
+    fast = P.comb && !P.so && !P.si;
+    if (fast) km_bound_loop(P, smem, kacc, kcnt, pacc, pn, km_guess);
   }
   for (uint32_t it = 0; !fast; ++it) {
     uint32_t w = 0;
@@ -2538,40 +2711,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         const float4 a = P.so ? __ldg(src) : src[0];
         const float4 b = P.so ? __ldg(src + 1) : src[1];
         x[0] = a.x; x[1] = a.y; x[2] = a.z; x[3] = a.w; x[4] = b.x; x[5] = b.y; x[6] = b.z; x[7] = b.w;
-        float bd = 0.0f;
-        // C-2 KM: fp32 RN, explicit chain d = fma(x_t - c_t, x_t - c_t, d) over t = 0..7, ties ->
-        // lowest j.  Two centroids per instruction with packed FADD2/FFMA2 (each lane of the pair
-        // performs exactly the scalar RN operations, so the result is bit-identical).
-        uint64_t X[8];
-#pragma unroll
-        for (int t = 0; t < 8; ++t) X[t] = f2pack(x[t], x[t]);
-        const uint32_t kp = P.k & ~1u;
-        bool first = true;
-#pragma unroll kKmUnroll
-        for (uint32_t j = 0; j < kp; j += 2) {
-          const ulonglong2* cp = reinterpret_cast<const ulonglong2*>(cent + j * 8);   // pair layout
-          const ulonglong2 q0 = cp[0], q1 = cp[1], q2 = cp[2], q3 = cp[3];
-          const uint64_t C[8] = {q0.x, q0.y, q1.x, q1.y, q2.x, q2.y, q3.x, q3.y};
-          uint64_t D = 0;
-#pragma unroll
-          for (int t = 0; t < 8; ++t) {
-            const uint64_t E = f2sub(X[t], C[t]);
-            D = f2fma(E, E, D);
-          }
-          float d0, d1;
-          f2unpack(D, d0, d1);
-          if (first || d0 < bd) { bd = d0; best = j; }
-          first = false;
-          if (d1 < bd) { bd = d1; best = j + 1; }
-        }
-        if (P.k & 1u) {
-          const uint32_t j = P.k - 1;
-          const float* c = cent + j * 8;   // last centroid stored unpaired
-          float d = 0.0f, e;
-#pragma unroll
-          for (int t = 0; t < 8; ++t) { e = __fsub_rn(x[t], c[t]); d = __fmaf_rn(e, e, d); }
-          if (first || d < bd) { bd = d; best = j; }
-        }
+        best = km_scan(x, cent, P.k);   // C-2 KM (reading 4)
       }
       if (valid) km_guess = best;   // the next point of this lane starts from this winner
       const uint32_t m = __ballot_sync(kFull, valid);
@@ -2582,60 +2722,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[s]);   // stage no longer read by this warp
       if (P.comb) {
-        // f-1 combiner: fp32 per-warp cluster sums of this tile (<= 32 points per partial, as
-        // in the sorted Reduce, reading 5), folded into lane-owned fp64 registers
-        float* wacc = reinterpret_cast<float*>(smem + Layout<W>::kmacc) + warp * (kKmCombMax * 8);
-        uint32_t* wcnt = reinterpret_cast<uint32_t*>(smem + Layout<W>::kmacc + kKmWaccBytes) + warp * kKmCombMax;
-        // lanes with the same cluster form a match group; the group's members add their point
-        // in rank order, one member per round (plain read-modify-write: no two lanes of a round
-        // share a cluster) — shared-memory fp32 atomics are CAS loops on sm_100a (ATOMS.CAST.SPIN,
-        // ncu round 2: 19% of the KM Map's instructions, 38% of its stall samples)
-        // A point of one of the lane's own clusters (lane, lane + 32: the clusters whose fp64
-        // accumulators it holds) is added straight into those registers (fp64: at least as exact
-        // as the fp32 partials of reading 5); only the other points take the SMEM match rounds.
-        const bool own = valid && (best & 31u) == lane && best < static_cast<uint32_t>(kKmCombMax);
-        if (own) {
-          if (best < 32u) {
-            kcnt[0] += 1;
-#pragma unroll
-            for (int t = 0; t < 8; ++t) kacc[0][t] += static_cast<double>(x[t]);
-          } else {
-            kcnt[1] += 1;
-#pragma unroll
-            for (int t = 0; t < 8; ++t) kacc[1][t] += static_cast<double>(x[t]);
-          }
-        }
-        const bool other = valid && !own;
-        if (__any_sync(kFull, other)) {
-        const uint32_t grp = __match_any_sync(kFull, other ? best : 0xFFFFFFFFu);
-        const uint32_t rank = __popc(grp & lanemask_lt());
-        const uint32_t rounds = __reduce_max_sync(kFull, other ? static_cast<uint32_t>(__popc(grp)) : 0u);
-        for (uint32_t r = 0; r < rounds; ++r) {
-          if (other && rank == r) {
-#pragma unroll
-            for (int t = 0; t < 8; ++t) wacc[t * kKmCombMax + best] += x[t];   // [dim][cluster]: no bank conflicts
-            wcnt[best] += 1u;
-          }
-          __syncwarp();
-        }
-#pragma unroll
-        for (int q = 0; q < kKmCombMax / 32; ++q) {
-          const uint32_t c = lane + 32 * q;
-          if (c < P.k) {
-            const uint32_t nc = wcnt[c];
-            if (nc) {
-              wcnt[c] = 0;
-              kcnt[q] += nc;
-#pragma unroll
-              for (int t = 0; t < 8; ++t) {
-                kacc[q][t] += static_cast<double>(wacc[t * kKmCombMax + c]);
-                wacc[t * kKmCombMax + c] = 0.0f;
-              }
-            }
-          }
-        }
-        __syncwarp();
-        }
+        km_combine(smem, warp, lane, valid, best, x, P.k, kacc, kcnt, pacc, pn);
       } else if (m && P.si) {   // SI / G ablation: global append per warp result
         unsigned long long gb = 0;
         if (lane == 0) gb = atomicAdd(&P.st->pair_cursor, static_cast<unsigned long long>(__popc(m)));
@@ -2694,6 +2781,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   }
   if constexpr (W == kKM) {
     if (P.comb) {   // this lane's clusters -> global fp64 sums / u64 counts (job accumulators)
+      if (pn) km_flush_partial(kacc[0], kcnt[0], pacc, pn);
 #pragma unroll
       for (int q = 0; q < kKmCombMax / 32; ++q) {
         const uint32_t c = lane + 32 * q;
