@@ -542,23 +542,22 @@ __device__ __forceinline__ uint64_t bytes8_at(const Params& P, const TileView& t
   return b;
 }
 
-// Sort key of key bytes in global memory (8-byte aligned loads): out of line, so that the
-// register allocation of the Map loops does not carry it (II keys every URL from global memory in
-// its drain; WC only words that leave the stage).
-__device__ __noinline__ uint64_t key_global(const uint8_t* p, uint32_t len, uint64_t seed, bool weak, uint32_t bits) {
-  if (len <= inline_max(bits)) return inline_key(load8(p, len), len, bits);
-  return hashed_key(hash_bytes_g(p, len, seed), weak, bits);
-}
 // Sort key of the key bytes [q, q + len): inline when short, else the hash (common.cuh).
 __device__ __forceinline__ uint64_t key_at(const Params& P, const TileView& tv, long long q, uint32_t len) {
   const bool in_stage = (q + static_cast<long long>(len) <= tv.stg_hi) && (q - tv.sbase + len + 12 <= kStageBytes);
-  if (!in_stage) return key_global(P.rec + q, len, P.hash_seed, (P.flags & 8u) != 0, P.key_bits);
-  const uint32_t i = static_cast<uint32_t>(q - tv.sbase);
   if (len <= inline_max(P.key_bits)) {
-    const uint64_t b = static_cast<uint64_t>(smem_word_at(tv.sb, i)) | (static_cast<uint64_t>(smem_word_at(tv.sb, i + 4)) << 32);
+    uint64_t b = 0;
+    if (in_stage) {
+      const uint32_t i = static_cast<uint32_t>(q - tv.sbase);
+      b = static_cast<uint64_t>(smem_word_at(tv.sb, i)) | (static_cast<uint64_t>(smem_word_at(tv.sb, i + 4)) << 32);
+    } else {
+      for (uint32_t k = 0; k < len; ++k) b |= static_cast<uint64_t>(P.rec[q + k]) << (8 * k);
+    }
     return inline_key(b, len, P.key_bits);
   }
-  return hashed_key(hash_smem(tv.sb, i, len, P.hash_seed), (P.flags & 8u) != 0, P.key_bits);
+  const uint64_t h = in_stage ? hash_smem(tv.sb, static_cast<uint32_t>(q - tv.sbase), len, P.hash_seed)
+                              : hash_bytes(P.rec + q, len, P.hash_seed);
+  return hashed_key(h, (P.flags & 8u) != 0, P.key_bits);
 }
 
 // ---------------------------------------------------------------- emit allocator
@@ -1934,9 +1933,7 @@ __device__ __forceinline__ void ii_window(const Params& P, OutCtl* oc, uint8_t* 
       q = find_quote(P, tv, max(q0, p0w + kWin), p0 + j);
     }
     if (q > q0 && nm < 2) {
-      if (nm == 0) aux[0] = static_cast<uint32_t>(q - q0);   // (no dynamic index: registers, not local memory)
-      else aux[1] = static_cast<uint32_t>(q - q0);
-      ++nm;
+      aux[nm++] = static_cast<uint32_t>(q - q0);
       emit_mask |= 1u << j;
     }
   }
@@ -2168,9 +2165,7 @@ __device__ void emit_text_chunk(const Params& P, OutCtl* oc, uint8_t* outh, cons
         q = find_quote(P, tv, max(q0, wp + kWin), p0 + j);
       }
       if (q > q0 && nm < 2) {
-        if (nm == 0) aux[0] = static_cast<uint32_t>(q - q0);   // (no dynamic index: registers, not local memory)
-      else aux[1] = static_cast<uint32_t>(q - q0);
-      ++nm;
+        aux[nm++] = static_cast<uint32_t>(q - q0);
         emit_mask |= 1u << j;
       }
     }
