@@ -117,6 +117,9 @@ constexpr int kNProd = 2;
 #ifndef BMR_WC_TAB
 #define BMR_WC_TAB 1   // WordCount table mode: per-lane start loop (wc_window_tab); 0: the queued rounds of wc_window
 #endif
+#ifndef BMR_WC_LSCAN
+#define BMR_WC_LSCAN 1   // WordCount table mode: long words of <= 16 bytes queued at their warp rank (no rounds)
+#endif
 #ifndef BMR_WC_NFLUSH
 #define BMR_WC_NFLUSH 1u
 #endif
@@ -1643,6 +1646,43 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
   // bytes after it)
   uint32_t L = S & ~near;
   if (!__any_sync(kFull, L)) return;
+#if BMR_WC_LSCAN
+  {
+    // words of <= 16 bytes (a stop within 16 bytes after the start: t16 bit j = an nb bit at
+    // j+1..j+16) go to the queue at their warp rank, each lane writing its own (no rounds); longer
+    // ones and windows with more than a queue of them take the round loop below
+    uint32_t t16 = nb >> 1;
+    t16 |= t16 >> 1;
+    t16 |= t16 >> 2;
+    t16 |= t16 >> 4;
+    t16 |= t16 >> 8;
+    const uint32_t Ls = L & t16;
+    const uint32_t cs = __popc(Ls);
+    const uint32_t incl = warp_inclusive_add(cs);
+    const uint32_t tot = __shfl_sync(kFull, incl, 31);
+    if (tot <= static_cast<uint32_t>(Cfg<kWC>::kLQ)) {
+      L &= ~t16;
+      if (tot) {
+        while (qn + tot > static_cast<uint32_t>(Cfg<kWC>::kLQ)) wc_drain_tab(P, lq, qn);
+        LWord* d = lq + qn + incl - cs;
+        for (uint32_t m = Ls; m; m &= m - 1, ++d) {
+          const uint32_t j = __ffs(m) - 1;
+          const uint32_t len = __ffs(nb >> (j + 1));   // 6..16
+          const uint32_t pos = i0 + j;
+          const uint32_t* src = reinterpret_cast<const uint32_t*>(tv.sb + (pos & ~3u));
+          const uint32_t sh = (pos & 3u) * 8;   // 5 aligned words, funnel-shifted
+          const uint32_t y0 = src[0], y1 = src[1], y2 = src[2], y3 = src[3], y4 = src[4];
+          d->lo = static_cast<uint64_t>(__funnelshift_r(y0, y1, sh)) | (static_cast<uint64_t>(__funnelshift_r(y1, y2, sh)) << 32);
+          d->hi = static_cast<uint64_t>(__funnelshift_r(y2, y3, sh)) | (static_cast<uint64_t>(__funnelshift_r(y3, y4, sh)) << 32);
+          d->meta = (static_cast<uint64_t>(tv.sbase + pos) << 16) | len;
+        }
+        qn += tot;
+        __syncwarp();
+      }
+      if (!__any_sync(kFull, L)) return;
+    }
+  }
+#endif
   uint32_t len_slow = 0;
   if (L) {
     const uint32_t jh = 31 - __clz(S);
