@@ -342,9 +342,13 @@ struct mr_job {
   bool wc_table() const {
     return tables_on && wc_comb() && map_wc_table_ok(cfg.flags) && !(cfg.flags & MR_FLAG_NO_COMBINE);
   }
-  // per run, from the first batch's size: extracting the tables streams the 4 GiB count table
-  // (~0.7 ms), more than sorting the exact keys of a small input costs (C1: 1 MiB)
+  // per run, from the first batch's size: the tables (tables_on; BMR_TABLE_MIN_BYTES, default 0)
+  // and among them the direct-address exact-key table (xtab_on; BMR_XTAB_MIN_BYTES, default
+  // 64 MiB): extracting it streams 4 GiB (~0.6 ms), so a small input (C1: 1 MiB) counts its
+  // exact words in the mid table instead ("small-table mode": the Map's exact-word combiner
+  // misses probe the open-addressing table; no sort, no 4 GiB scan)
   bool tables_on = true;
+  bool xtab_on = true;
   DBuf<uint32_t> xtab;            // 2^30 u32 counts by exact key (zero between runs)
   // mid words (6..8 symbols): open-addressing table of 48-bit exact keys + counts (2^mbits slots)
   DBuf<uint64_t> mtab_keys;
@@ -463,14 +467,14 @@ cudaError_t launch_batch(mr_job* job, const Batch& b) {
   a.out.h = job->h.p;
   a.out.hx = job->hx.p;
   a.out.hp = job->wc_comb() ? job->hp.p : nullptr;
-  a.out.xtab = job->wc_table() ? job->xtab.p : nullptr;
+  a.out.xtab = job->wc_table() && job->xtab_on ? job->xtab.p : nullptr;
   a.out.mkeys = job->wc_table() ? job->mtab_keys.p : nullptr;
   a.out.mcnt = job->wc_table() ? job->mtab_cnt.p : nullptr;
   a.out.mbits = job->mbits;
   a.out.lkeys = job->wc_table() ? job->ltab_keys.p : nullptr;
   a.out.lcnt = job->wc_table() ? job->ltab_cnt.p : nullptr;
   a.out.lbits = job->lbits;
-  if (a.out.xtab) job->xtab_dirty = true;
+  if (a.out.xtab || a.out.mkeys) job->xtab_dirty = true;
   a.out.km_sums = job->km_comb() ? job->sums.p : nullptr;
   a.out.km_cnts = job->km_comb() ? job->cnts.p : nullptr;
   a.out.cap_p = job->cap_p;
@@ -827,10 +831,13 @@ mr_status tables_extract(mr_job* job) {
   CK(cudaMemsetAsync(cur, 0, 2 * sizeof(unsigned long long), s), "memset cursor");
   if (job->xkeys.n < 4096) { CK(job->xkeys.ensure(1 << 20), "alloc keys"); CK(job->pxcounts.ensure(1 << 20), "alloc counts"); }
   uint64_t cap = std::min(job->xkeys.n, job->pxcounts.n);
+  uint64_t t = 0;
+  if (job->xtab_on) {   // (small-table mode: the exact words are in the mid table)
   CK(launch_xtab_extract_list(job->xtab.p, job->xtab.n, job->xkeys.p, job->pxcounts.p, cap, cur, wsum, job->nsm, s),
      "table extract");
   CK(read_state(job), "sync table extract");
-  uint64_t t = job->st_h.p->n_extra;
+  t = job->st_h.p->n_extra;
+  }
   if (t > cap) {
     CK(grow_keep(job->xkeys, cap, t + t / 8 + 4096, s), "grow keys");
     CK(grow_keep(job->pxcounts, cap, t + t / 8 + 4096, s), "grow counts");
@@ -1052,8 +1059,11 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
   // assumed; overflow is caught by the demand counters and replayed at mr_group)
   const uint64_t est = nbytes != ~0ULL ? nbytes : 32 * n;
   if (job->batches.empty() && job->nfolds == 0 && !job->ingested) {
-    const char* tm = getenv("BMR_TABLE_MIN_BYTES");   // (tests: 0 = always the tables)
-    job->tables_on = est >= (tm ? strtoull(tm, nullptr, 10) : (64ULL << 20));
+    const char* tm = getenv("BMR_TABLE_MIN_BYTES");   // (tests: 1 << 40 = the sorted streams)
+    job->tables_on = est >= (tm ? strtoull(tm, nullptr, 10) : 0ULL);
+    const char* xm = getenv("BMR_XTAB_MIN_BYTES");    // (tests: 0 = always the exact-key table)
+    job->xtab_on = est >= (xm ? strtoull(xm, nullptr, 10) : (64ULL << 20));
+    if (!job->xtab_on && !map_wc_tab()) job->tables_on = false;   // small-table mode needs wc_window_tab
   }
   if ((job->cfg.flags & MR_FLAG_BATCH_COMBINE) && job->cfg.workload == MR_WORDCOUNT && !job->ingested &&
       !job->batches.empty()) {
@@ -1073,8 +1083,11 @@ static mr_status map_common(mr_job* job, const uint8_t* records, const uint64_t*
     }
     job->stats.capacity_pairs = job->cap + job->cap_b + job->cap_c;
   }
-  if (job->wc_table() && !job->xtab.p) {   // the tables, emptied once (extraction re-empties them)
+  if (job->wc_table() && job->xtab_on && !job->xtab.p) {   // emptied once (extraction re-empties it)
     CK(job->xtab.ensure(1ULL << kExactBits), "alloc count table");
+    CK(cudaMemsetAsync(job->xtab.p, 0, job->xtab.n * 4, job->stream), "empty the count table");
+  }
+  if (job->wc_table() && !job->mtab_keys.p) {   // the mid / long tables, emptied once
     CK(job->mtab_keys.ensure(1ULL << job->mbits), "alloc mid table");
     CK(job->mtab_cnt.ensure((1ULL << job->mbits) * kMidStripes), "alloc mid table");
     CK(job->ltab_keys.ensure(2ULL << job->lbits), "alloc long table");

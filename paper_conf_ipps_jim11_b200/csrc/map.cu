@@ -97,7 +97,11 @@ constexpr int nmap() { return W == 3 ? kNMap : W == 2 ? BMR_SM_NMAP : W == 4 ? B
 // Producer warps kProdWarp0 .. + kNProd - 1: producer p owns the iterations it == p (mod kNProd)
 // (and so the stages s == p (mod kNProd)); one warp alone is latency-bound at ~465 instructions
 // per tile (TMA issue + bitmap), slower than HBM delivers a tile (ncu, C2 round 1).
-constexpr int kNProd = 2;
+#ifndef BMR_II_NPROD
+#define BMR_II_NPROD 2
+#endif
+template <int W>
+constexpr int nprod() { return W == 4 ? BMR_II_NPROD : 2; }
 // Flush warps (flush_loop takes generations f == fw mod nflush).  One: a second WordCount flush
 // warp removed the map warps' spinning on sealed buffers but cost the Map more than it saved
 // (C5 Map 20.4 -> 21.3 ms, round 2: a 28th warp lowers the register budget of every warp).
@@ -126,7 +130,7 @@ constexpr int kNProd = 2;
 template <int W>
 constexpr uint32_t nflush() { return W == kWC ? BMR_WC_NFLUSH : 1u; }
 template <int W>
-constexpr int threads_of() { return (nmap<W>() + kNProd + static_cast<int>(nflush<W>())) * 32; }
+constexpr int threads_of() { return (nmap<W>() + nprod<W>() + static_cast<int>(nflush<W>())) * 32; }
 constexpr int kT = static_cast<int>(kMapTileBytes);   // owned bytes per tile (text) / bytes per tile (KM)
 constexpr int kLead = 16;        // bytes staged before the tile (previous-byte context)
 constexpr int kHalo = 256;       // bytes staged after the tile (words / matches / URLs crossing it)
@@ -161,7 +165,7 @@ struct Cfg {
   // the producer builds the bitmap of tile it - kLag right after issuing tile it: kLag stages of
   // TMA traffic stay in flight per SM while one stage is being consumed
   static constexpr int kLag = kStages - 2;
-  static_assert(kStages % kNProd == 0 && kLag % kNProd == 0, "a producer owns every kNProd-th stage");
+  static_assert(kStages % nprod<W>() == 0 && kLag % nprod<W>() == 0, "a producer owns every kNProd-th stage");
   // WC: per-warp queue of the window's long (hashed) words, hashed by all 32 lanes together
   // after the emission rounds (a lane-per-word hash inside the rounds diverges: with 10% long
   // words, most rounds would carry at least one).  A window holds at most 512 / 6 + 1 starts
@@ -869,11 +873,11 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
   uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
   const long long N = bd_nbytes();
   const uint64_t G = gridDim.x;
-  // iterations of this CTA: tiles blockIdx.x + it * G; this producer takes it == pw (mod kNProd)
+  // iterations of this CTA: tiles blockIdx.x + it * G; this producer takes it == pw (mod nprod<W>())
   const uint32_t T = blockIdx.x < bd_ntiles() ? static_cast<uint32_t>((bd_ntiles() - blockIdx.x + G - 1) / G) : 0u;
-  for (uint32_t i0 = pw; i0 < T; i0 += 32u * kNProd) {
+  for (uint32_t i0 = pw; i0 < T; i0 += 32u * nprod<W>()) {
     // lanes prefetch the bounds of this producer's next 32 tiles (one latency per 32 tiles)
-    const uint32_t my_it = i0 + lane * kNProd;
+    const uint32_t my_it = i0 + lane * nprod<W>();
     uint64_t my_ra = 0, my_rb = 0;
     if constexpr (W != kKM) {
       if (my_it < T) {
@@ -883,7 +887,7 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
       }
     }
     for (uint32_t j = 0; j < 32; ++j) {
-      const uint32_t it = i0 + j * kNProd;
+      const uint32_t it = i0 + j * nprod<W>();
       if (it >= T) break;
       const uint64_t t = blockIdx.x + static_cast<uint64_t>(it) * G;
       const uint64_t ra = __shfl_sync(kFull, my_ra, j), rb = __shfl_sync(kFull, my_rb, j);
@@ -981,7 +985,7 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
         if (P.pf) {
           const uint32_t jf = j + P.pf;
           const uint64_t raf = __shfl_sync(kFull, my_ra, jf & 31), rbf = __shfl_sync(kFull, my_rb, jf & 31);
-          const uint32_t itf = i0 + jf * kNProd;
+          const uint32_t itf = i0 + jf * nprod<W>();
           if (lane == 0 && itf < T) {
             const long long c0 = static_cast<long long>(blockIdx.x + static_cast<uint64_t>(itf) * G) * kT - P.a0;
             l2_prefetch_range(P.rec + max(0LL, c0 - kLead), P.rec + min(c0 + kT + kHalo, N));
@@ -996,10 +1000,10 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
   if constexpr (W != kKM && !Cfg<W>::kLazyDir) {   // this producer's tiles whose bitmap is still pending
     const uint32_t j0 = T > static_cast<uint32_t>(Cfg<W>::kLag) ? T - Cfg<W>::kLag : 0u;
     for (uint32_t j = j0; j < T; ++j)
-      if (j % kNProd == pw) finish_stage<W>(P, smem, j);
+      if (j % nprod<W>() == pw) finish_stage<W>(P, smem, j);
   }
   // end-of-work marker at iteration T, written by its owner
-  if (T % kNProd != pw) return;
+  if (T % nprod<W>() != pw) return;
   const uint32_t s = T % kStages, ph = (T / kStages) & 1u;
   mbar_wait(&empty[s], ph ^ 1u);
   if (lane == 0) {
@@ -1587,6 +1591,25 @@ __device__ __forceinline__ void wc_window(const Params& P, OutCtl* oc, uint8_t* 
   __syncwarp();
 }
 
+// One lane adds `cnt` occurrences of `key` (a 48-bit exact key: a word of <= 8 symbols; a word of
+// <= 5 symbols has the same key as in the exact stream) to the mid table — the small-table mode's
+// path for exact words that miss the SMEM combiner (no match-group aggregation: rare per lane).
+__device__ __forceinline__ void mid_insert(const Params& P, uint64_t key, uint32_t cnt) {
+  const uint64_t mask = (1ULL << P.mbits) - 1ULL;
+  uint64_t h = mid_slot(key, P.mbits);
+  const uint32_t stripe = (blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1);
+  for (uint32_t pr = 0; pr < kMidProbes; ++pr, h = (h + 1) & mask) {
+    unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(P.mkeys + h);
+    if (k == kMidEmpty) k = atomicCAS(reinterpret_cast<unsigned long long*>(P.mkeys + h), kMidEmpty, key);
+    if (k == key || k == kMidEmpty) {
+      red_add_u32(P.mcnt + h * kMidStripes + stripe, cnt);
+      return;
+    }
+  }
+  atomicOr(&P.st->err, kErrMidTable);   // table too full: counted, the batch is replayed with a larger table
+  atomicAdd(&P.st->mid_fail, 1ULL);
+}
+
 // Combiner update of one exact word without branches (predicated PTX): the slot's key is read;
 // an empty slot is claimed by CAS; a slot holding the key (or just claimed) counts the word in
 // SMEM, any other slot sends it to the L2 count table (RED).  Same semantics as comb_add + RED.
@@ -1610,6 +1633,7 @@ __device__ __forceinline__ void comb_or_table(uint32_t* slot_key, uint32_t* slot
 // its own 16 bytes (a loop of max-over-lanes iterations; ~2.7 starts per lane at C5) and counts
 // each word where it finds it; the starts of longer words are then moved into the warp's
 // long-word queue one per lane per round.  The same words, keys and tables as wc_window.
+template <bool kX>
 __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8_t* outh, const TileView& tv,
                                               long long p0w, uint32_t* ctab, LWord* lq, uint32_t& qn) {
   const uint32_t lane = threadIdx.x & 31;
@@ -1640,7 +1664,14 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
     const uint32_t w1 = *reinterpret_cast<const uint32_t*>(tv.sb + a + 4);
     const uint32_t key = exact_key30_bf(__funnelshift_r(w0, w1, sh), (w1 >> sh) & 0xFFu, len);
     const uint32_t home = (key * 0x9E3779B1u) >> (32 - kCombBits);
-    comb_or_table(ctab + home, ccnt + home, P.xtab + key, key);
+    if constexpr (kX) {
+      comb_or_table(ctab + home, ccnt + home, P.xtab + key, key);
+    } else {   // small-table mode: a combiner miss goes to the mid table
+      uint32_t v = *reinterpret_cast<volatile uint32_t*>(ctab + home);
+      if (v == kCombEmpty32) v = atomicCAS(ctab + home, kCombEmpty32, key);
+      if (v == key || v == kCombEmpty32) atomicAdd(ccnt + home, 1u);
+      else mid_insert(P, key, 1u);
+    }
   }
   // longer words: only the lane's highest start can lack a visible end (no stop in the 31 - j
   // bytes after it)
@@ -1730,8 +1761,11 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
 
 // WordCount map warps in SIO mode: windows from the shared counter (tile order), the stage
 // header read once per tile change, the window loop of wc_window (wc_window_tab in table mode).
-template <bool kTab>
+// kMode: 0 wc_window (streams, or tables behind the old rounds), 1 wc_window_tab with the exact-key
+// table, 2 wc_window_tab in small-table mode (no exact-key table)
+template <int kMode>
 __device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
+  constexpr bool kTab = kMode != 0;
   constexpr int W = kWC;
   constexpr int kStages = Cfg<W>::kStages;
   const uint32_t warp = threadIdx.x >> 5;
@@ -1765,7 +1799,7 @@ __device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       const TileView tv{smem + Layout<W>::bytes + s * kStageBytes,
                         reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits), sbase, stg_hi, 0,
                         0};
-      if constexpr (kTab) wc_window_tab(P, oc, outh, tv, wp, ctab, lq, qn);
+      if constexpr (kTab) wc_window_tab<kMode == 1>(P, oc, outh, tv, wp, ctab, lq, qn);
       else wc_window(P, oc, outh, tv, wp, xq, hq, ctab, lq, qn, lo);
       if (qn >= 32) {
         if constexpr (kTab) wc_drain_tab(P, lq, qn);
@@ -2677,8 +2711,9 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   if constexpr (W == kWC) {
     fast = !P.so && !P.si && P.wc_bal && P.dyn && P.wc_fast;
     if (fast) {
-      if constexpr (V == 1) wc_map_loop<true>(P, smem, oc);
-      else wc_map_loop<false>(P, smem, oc);
+      if constexpr (V == 1) wc_map_loop<1>(P, smem, oc);
+      else if constexpr (V == 2) wc_map_loop<2>(P, smem, oc);
+      else wc_map_loop<0>(P, smem, oc);
     }
   }
   if constexpr (W == kII) {
@@ -2838,6 +2873,12 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         const uint32_t k = ctab[i], c = ctab[Cfg<W>::kCombSlots + i];
         if (k != kCombEmpty32) red_add_u32(P.xtab + k, c);
       }
+    } else if (P.comb && P.mkeys) {   // small-table mode: the CTA's slots go to the mid table
+      const uint32_t* ctab = reinterpret_cast<const uint32_t*>(smem + Layout<W>::comb);
+      for (uint32_t i = warp * 32 + lane; i < static_cast<uint32_t>(Cfg<W>::kCombSlots); i += nmap<W>() * 32) {
+        const uint32_t k = ctab[i], c = ctab[Cfg<W>::kCombSlots + i];
+        if (k != kCombEmpty32 && c) mid_insert(P, k, c);
+      }
     } else if (P.comb) {   // combiner partials -> global (one atomic per warp step; demand counted past capacity)
       const uint32_t* ctab = reinterpret_cast<const uint32_t*>(smem + Layout<W>::comb);
       for (uint32_t i0 = warp * 32; i0 < static_cast<uint32_t>(Cfg<W>::kCombSlots); i0 += nmap<W>() * 32) {
@@ -2933,9 +2974,9 @@ __global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
   __syncthreads();
   if (s_bd[3]) return;   // more tiles than tile-bounds capacity: nothing mapped, the host grows + replays
   const uint32_t warp = threadIdx.x >> 5;
-  if (warp >= static_cast<uint32_t>(nmap<W>()) && warp < static_cast<uint32_t>(nmap<W>() + kNProd))
+  if (warp >= static_cast<uint32_t>(nmap<W>()) && warp < static_cast<uint32_t>(nmap<W>() + nprod<W>()))
     producer_loop<W>(P, smem, warp - nmap<W>());
-  else if (warp >= static_cast<uint32_t>(nmap<W>() + kNProd)) flush_loop<W>(P, smem, oc, warp - nmap<W>() - kNProd);
+  else if (warp >= static_cast<uint32_t>(nmap<W>() + nprod<W>())) flush_loop<W>(P, smem, oc, warp - nmap<W>() - nprod<W>());
   else map_loop<W, V>(P, smem, oc);
 }
 
@@ -3031,11 +3072,14 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.wc_bal = map_wc_balanced();
   P.wc_fast = map_fast_path() ? 1u : 0u;
   P.xtab = (W == kWC && P.comb && map_wc_table_ok(a.flags)) ? a.out.xtab : nullptr;
-  P.mkeys = P.xtab ? a.out.mkeys : nullptr;
-  P.mcnt = P.xtab ? a.out.mcnt : nullptr;
+  // the mid / long tables: with the exact-key table, or alone in small-table mode (which needs the
+  // table-mode window; the host enables it only then, map_wc_tab)
+  const bool tabs = W == kWC && P.comb && map_wc_table_ok(a.flags) && a.out.mkeys && (P.xtab || map_wc_tab());
+  P.mkeys = tabs ? a.out.mkeys : nullptr;
+  P.mcnt = tabs ? a.out.mcnt : nullptr;
   P.mbits = a.out.mbits;
-  P.lkeys = (BMR_LTAB && P.xtab) ? a.out.lkeys : nullptr;
-  P.lcnt = (BMR_LTAB && P.xtab) ? a.out.lcnt : nullptr;
+  P.lkeys = (BMR_LTAB && tabs) ? a.out.lkeys : nullptr;
+  P.lcnt = (BMR_LTAB && tabs) ? a.out.lcnt : nullptr;
   P.lbits = a.out.lbits;
   P.km_bound = (W == kKM && !(a.flags & 0x1000u) && a.k <= static_cast<uint32_t>(kKmBoundMax)) ? 1u : 0u;   // MR_FLAG_KM_FULL_SCAN
   if (W == kKM && P.ntiles == 0) return cudaSuccess;
@@ -3047,10 +3091,10 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   }
   const size_t smem = Layout<W>::cent + (W == kKM ? static_cast<size_t>(a.k) * (P.km_bound ? 68 : 32) : 0);
   // WordCount table mode (the fast SIO path with the L2 tables): its own instantiation
-  const bool tab = W == kWC && map_wc_tab() && P.xtab && P.mkeys && P.lkeys && P.comb && !P.so && !P.si && P.wc_bal && P.dyn && P.wc_fast;
+  const bool tab = W == kWC && map_wc_tab() && P.mkeys && P.lkeys && P.comb && !P.so && !P.si && P.wc_bal && P.dyn && P.wc_fast;
   auto kern = k_map<W, 0>;
   if constexpr (W == kWC) {
-    if (tab) kern = k_map<W, 1>;
+    if (tab) kern = P.xtab ? k_map<W, 1> : k_map<W, 2>;
   }
   if constexpr (W == kKM) {   // the bound-test instantiation (the full scan keeps its own registers)
     if (P.km_bound) kern = k_map<W, 1>;

@@ -4,9 +4,11 @@ import sys
 import pytest
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-# the WordCount L2 count tables are used for every input size in the tests (libbmr's default skips
-# them below 64 MiB, where sorting the exact keys is cheaper than streaming the table);
-# test_wc_small_input_sort_path covers the other side
+# WordCount tables: libbmr counts exact / mid / long words in tables for every input size; below
+# 64 MiB (BMR_XTAB_MIN_BYTES) without the 4 GiB direct-address exact-key table ("small-table mode":
+# exact words that miss the SMEM combiner go to the mid table).  The small test inputs therefore
+# run the small-table mode; tests/test_gpu_tables.py re-runs the WordCount cases with the exact-key
+# table (BMR_XTAB_MIN_BYTES=0, the C5 path), and test_wc_small_input_sort_path the sorted streams.
 os.environ.setdefault("BMR_TABLE_MIN_BYTES", "0")
 if ROOT not in sys.path:
     sys.path.insert(0, ROOT)

@@ -1,19 +1,22 @@
 """Write profiles/traffic.json: DRAM bytes (dram__bytes_read.sum + dram__bytes_write.sum) per
 launch of the dominant kernels, from `ncu --set full` captures brought back in gpurun_out/.
 
-usage: python tools/make_traffic.py OUT.json WORKLOAD=report.ncu-rep [WORKLOAD=report ...]
+usage: python tools/make_traffic.py OUT.json WORKLOAD=report.ncu-rep|export-prefix [WORKLOAD=... ...]
 (bench.py reads OUT.json for the roofline `traffic` field; the report names are recorded)."""
 import csv
 import io
 import json
 import os
-import subprocess
 import sys
+
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+from ncu_csv import page  # noqa: E402  (a report, or the CSV export prefix of tools/r03/ncu_export.sh)
 
 
 def launches(rep):
-    out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
-    rows = list(csv.reader(io.StringIO(out)))
+    rows = list(csv.reader(io.StringIO(page(rep, "raw"))))
+    hi = next(i for i, r in enumerate(rows) if "Kernel Name" in r)
+    rows = rows[hi:]
     h = rows[0]
     iname, ir, iw = h.index("Kernel Name"), h.index("dram__bytes_read.sum"), h.index("dram__bytes_write.sum")
     units = rows[1]
