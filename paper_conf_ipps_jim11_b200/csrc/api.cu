@@ -633,8 +633,12 @@ mr_status settle_map(mr_job* job) {
     if (tile_over) job->tb_cap = max_tiles + 1024;   // (tb itself is grown by launch_batch)
     const uint64_t ncap_p = job->wc_comb() ? std::max(job->cap_p, mp + mp / 8 + 4096) : 0;
     const uint64_t ncap = std::max(job->cap, m + m / 8 + 4096);
-    const uint64_t ncap_b = job->split() ? std::max(job->cap_b, mb + mb / 8 + 4096) : 0;
-    const uint64_t ncap_c = job->split() ? std::max(job->cap_c, mc + mc / 8 + 4096) : 0;
+    // the mid / hashed streams are appended in warp-private chunks (map.cu kLChunk = 256 entries):
+    // a run may leave up to a chunk unused per map warp, and which warps see long words varies
+    // between runs (dynamic windows and tiles), so the replay adds a chunk per warp of headroom
+    const uint64_t chunk_slack = static_cast<uint64_t>(job->nsm) * 24u * 256u;
+    const uint64_t ncap_b = job->split() ? std::max(job->cap_b, mb + mb / 8 + 4096 + chunk_slack) : 0;
+    const uint64_t ncap_c = job->split() ? std::max(job->cap_c, mc + mc / 8 + 4096 + chunk_slack) : 0;
     if (ncap > job->cap || ncap_b > job->cap_b || ncap_c > job->cap_c) {
       release_pairs(job);
       CK(ensure_pairs(job, ncap, ncap_b, ncap_c), "grow intermediate");

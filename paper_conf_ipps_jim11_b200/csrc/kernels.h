@@ -40,6 +40,7 @@ struct DevState {
   unsigned long long seal_waits;     // Map: seals that waited for a buffer still flushing (ring full)
   unsigned long long spills;         // Map: warp results written straight to HBM while the ring was full
   unsigned long long km_scanned;     // KMeans Map: points that scanned every centroid (bound test failed / off)
+  unsigned long long tile_next;      // text Map: dynamic tile counter of the current batch (k_tile_bounds zeroes it)
 };
 constexpr unsigned int kErrKeyTooLong = 1u, kErrCollision = 2u, kErrTileCap = 4u, kErrNullRecords = 8u,
                        kErrMidTable = 16u, kErrLongTable = 32u;

@@ -124,6 +124,18 @@ constexpr int nprod() { return W == 4 ? BMR_II_NPROD : 2; }
 #ifndef BMR_WC_LSCAN
 #define BMR_WC_LSCAN 1   // WordCount table mode: long words of <= 16 bytes queued at their warp rank (no rounds)
 #endif
+#ifndef BMR_WC_XLOOP
+#define BMR_WC_XLOOP 1   // WordCount table mode: lean exact-word loop (bfind starts, 32-bit shared addresses, unconditional shared RED)
+#endif
+#ifndef BMR_WC_CLS16
+#define BMR_WC_CLS16 1   // WordCount table mode: each lane classifies its own 16 bytes only (next chunk by shuffle)
+#endif
+#ifndef BMR_WC_ADRAIN
+#define BMR_WC_ADRAIN 1   // WordCount table mode: long-word table probes prefetched by cp.async one drain ahead
+#endif
+#ifndef BMR_DYN_TILES
+#define BMR_DYN_TILES 1   // WordCount / InvertedIndex: tiles from a global counter (producer_loop_dyn)
+#endif
 #ifndef BMR_WC_NFLUSH
 #define BMR_WC_NFLUSH 1u
 #endif
@@ -235,6 +247,8 @@ struct OutCtl {
   unsigned int congested;        // the sealing warp waits for a flushing buffer: overflowing warps spill
   uint64_t req[kNOut];           // mbarrier: buffer sealed -> flush warp
   uint64_t done[kNOut];          // mbarrier: buffer flushed -> free
+  unsigned int pout[2];          // dynamic tiles: first iteration producer p found no tile (~0: not yet)
+  unsigned int plast[2];         // dynamic tiles: last iteration producer p filled with a tile (+1; 0: none)
 };
 
 template <int W>
@@ -344,6 +358,7 @@ struct Params {
   uint32_t* lcnt;          //   16 zero-padded key bytes (2^lbits slots); nullptr: hashed stream
   uint32_t lbits;
   uint32_t km_bound;       // KM: the exact bound test before the full centroid scan (kKmBoundMax)
+  unsigned long long* tile_next;   // text (WC / II): dynamic tile counter of the batch (zeroed by k_tile_bounds)
 };
 
 // Idle wait of a role warp on an mbarrier phase (map warps on a staged tile, producers on a free
@@ -848,8 +863,9 @@ __device__ void finish_stage(const Params& P, uint8_t* smem, uint32_t it) {
   const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
   uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout<W>::ready);
-  mbar_wait(&full[s], ph);
   const StageHdr* hd = reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
+  if (hd->t < 0) return;   // a skip stage (dynamic tiles): released when it was posted
+  mbar_wait(&full[s], ph);
   uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits);
   const uint64_t* soff =
       reinterpret_cast<const uint64_t*>(smem + Layout<W>::offs + s * Cfg<W>::kOffBytes + hd->off_shift);
@@ -865,8 +881,183 @@ __device__ void finish_stage(const Params& P, uint8_t* smem, uint32_t it) {
   if (lane == 0) mbar_arrive(&ready[s]);
 }
 
+// Text tile t into stage s: bytes (+ lead / halo) and the offsets slice offsets[ra..rb) by TMA,
+// the stage header, the bitmap cleared (built by finish_stage once the bytes have landed).
+template <int W>
+__device__ __forceinline__ void issue_text_stage(const Params& P, uint8_t* smem, uint32_t s, uint64_t t, uint64_t ra,
+                                                 uint64_t rb) {
+  const uint32_t lane = threadIdx.x & 31;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
+  const long long N = bd_nbytes();
+  StageHdr* hd = reinterpret_cast<StageHdr*>(smem + Layout<W>::hdr + s * 128);
+  uint8_t* sb = smem + Layout<W>::bytes + s * kStageBytes;
+  uint32_t b_off = 0, b_len = 0, o_off = 0, o_len = 0;
+  uint8_t* so = smem + Layout<W>::offs + s * Cfg<W>::kOffBytes;
+  const long long chunk0 = static_cast<long long>(t) * kT - P.a0;
+  const long long sbase = chunk0 - kLead;
+  const long long w_lo = max(0LL, sbase);
+  const long long w_hi = chunk0 + kT + kHalo;
+  const long long stg_hi = min(w_hi, N);
+  // stage bytes [w_lo, stg_hi) at sb + (w_lo - sbase); (rec + sbase) is 16-B aligned
+  uint8_t* d = sb + (w_lo - sbase);
+  const uint8_t* g = P.rec + w_lo;
+  if (!P.so) stage_copy_edges(d, g, static_cast<uint64_t>(max(0LL, stg_hi - w_lo)), lane, b_off, b_len);
+  // clear the record-start bitmap (map warps set bits after the full barrier)
+  if constexpr (!Cfg<W>::kLazyDir) {
+    uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits);
+    for (uint32_t i = lane; i < Cfg<W>::kBits / 16; i += 32) reinterpret_cast<uint4*>(bm)[i] = make_uint4(0, 0, 0, 0);
+  }
+  // offsets slice offsets[ra..rb) (record starts in the staged window)
+  const uint64_t cnt = rb - ra;
+  const bool staged = !Cfg<W>::kLazyDir && cnt <= static_cast<uint64_t>(Cfg<W>::kOffCap);
+  uint32_t shift = 0;
+  const uint8_t* og = reinterpret_cast<const uint8_t*>(P.off + ra);
+  if (staged && cnt) {
+    shift = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(og) & 15u);
+    // Copy the 16-B aligned superset of the slice with TMA alone (no synchronous edge
+    // loads on the producer's critical path) whenever it stays inside offsets[0..n].
+    const uint8_t* a_lo = og - shift;
+    const uint8_t* a_hi = reinterpret_cast<const uint8_t*>(
+        (reinterpret_cast<uintptr_t>(og + cnt * 8) + 15u) & ~static_cast<uintptr_t>(15u));
+    if (a_lo >= reinterpret_cast<const uint8_t*>(P.off) && a_hi <= P.off_end) {
+      o_off = 0;
+      o_len = static_cast<uint32_t>(a_hi - a_lo);
+      og = a_lo;
+      // so + shift still addresses offsets[ra]; the TMA below starts at so (= a_lo)
+    } else {
+      stage_copy_edges(so + shift, og, cnt * 8, lane, o_off, o_len);
+      og = og - shift;
+      o_off += shift;
+    }
+  }
+  if (lane == 0) {
+    hd->t = static_cast<long long>(t);
+    hd->sbase = sbase;
+    hd->chunk0 = chunk0;
+    hd->lo = max(0LL, chunk0);
+    hd->hi = min(N, chunk0 + kT);
+    hd->stg_hi = stg_hi;
+    hd->ra = ra;
+    hd->rb = rb;
+    hd->off_shift = shift;
+    hd->off_staged = staged ? 1u : 0u;
+  }
+  __syncwarp();
+  if (lane == 0) {
+    mbar_arrive_expect_tx(&full[s], b_len + o_len);
+    if (BMR_STREAM_HINT && P.xtab) {   // WC with the L2 count table: the input streams past it
+      const uint64_t pol = l2_policy_evict_first();
+      if (b_len) tma_load_1d_stream(d + b_off, g + b_off, b_len, &full[s], pol);
+      if (o_len) tma_load_1d_stream(so + o_off, og + o_off, o_len, &full[s], pol);
+    } else {
+      if (b_len) tma_load_1d(d + b_off, g + b_off, b_len, &full[s]);
+      if (o_len) tma_load_1d(so + o_off, og + o_off, o_len, &full[s]);
+    }
+  }
+}
+
+// Dynamic tile scheduling (WordCount / InvertedIndex): the producers take tiles from the batch's
+// global counter, kTileChunk at a time, instead of the static blockIdx.x + it * G order — the
+// per-SM time of the text Maps varies by a quarter (ncu C5: sm__cycles_active min 30.4 M / max
+// 41.4 M cycles of 40.9 M), so static shares leave the fast SMs idle for the last sixth.
+// Producer p still owns the CTA iterations it == p (mod 2).  A producer whose fetch finds no tile
+// publishes that first empty iteration x0 (pout[p]); the batch ends at E = max(x0_0, x0_1) (every
+// tile lies at an earlier iteration): the owner of E posts the end marker there, and each of the
+// producer's empty iterations below E is posted as a skip stage (no bytes; hi = LLONG_MIN, so its
+// windows are empty).  An empty iteration x below the other producer's x0 is only known to be a
+// skip once the other has filled an iteration > x (plast) or run out itself; it can always get
+// there (its next iteration needs x - 1 consumed at most), so the wait never deadlocks.
+#ifndef BMR_TILE_CHUNK
+#define BMR_TILE_CHUNK 4
+#endif
+template <int W>
+__device__ void producer_loop_dyn(const Params& P, uint8_t* smem, uint32_t pw) {
+  constexpr int kStages = Cfg<W>::kStages;
+  constexpr uint32_t kNP = nprod<W>(), kLag = Cfg<W>::kLag, kChunk = BMR_TILE_CHUNK;
+  static_assert(kNP == 2 && kChunk <= 32, "dynamic tiles: two producers");
+  const uint32_t lane = threadIdx.x & 31;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
+  uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
+  uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout<W>::ready);
+  OutCtl* oc = reinterpret_cast<OutCtl*>(smem + Layout<W>::ctl);
+  const uint64_t ntiles = bd_ntiles();
+  uint32_t it = pw;
+  for (;;) {   // chunks of tiles
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(P.tile_next, static_cast<unsigned long long>(kChunk));
+    base = __shfl_sync(kFull, base, 0);
+    if (base >= ntiles) break;
+    const uint32_t cnt = static_cast<uint32_t>(min(static_cast<unsigned long long>(kChunk), ntiles - base));
+    uint64_t my_ra = 0, my_rb = 0;
+    if (lane < cnt) {
+      my_ra = P.tb[2 * (base + lane)];
+      my_rb = P.tb[2 * (base + lane) + 1];
+    }
+    for (uint32_t j = 0; j < cnt; ++j, it += kNP) {
+      const uint64_t ra = __shfl_sync(kFull, my_ra, j), rb = __shfl_sync(kFull, my_rb, j);
+      const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
+      if (it >= kLag) finish_stage<W>(P, smem, it - kLag);
+      helper_wait(P, &empty[s], ph ^ 1u, 128);
+      if (lane == 0) *reinterpret_cast<volatile unsigned int*>(&oc->plast[pw]) = it + 1u;
+      issue_text_stage<W>(P, smem, s, base + j, ra, rb);
+    }
+  }
+  const uint32_t x0 = it;   // this producer's first empty iteration
+  if (lane == 0) {
+    *reinterpret_cast<volatile unsigned int*>(&oc->pout[pw]) = x0;
+    __threadfence_block();
+  }
+  __syncwarp();
+  const uint32_t other = pw ^ 1u;
+  for (;; it += kNP) {
+    // E = max(x0, x0_other) once the other has run out; below it, iterations past the other's
+    // filled ones are skips
+    bool post_end = false, post_skip = false;
+    for (uint32_t spin = 0;; ++spin) {
+      const uint32_t xo = *reinterpret_cast<volatile unsigned int*>(&oc->pout[other]);
+      if (xo != ~0u) {
+        const uint32_t E = max(x0, xo);
+        post_end = it == E;
+        post_skip = it < E;
+        break;
+      }
+      if (*reinterpret_cast<volatile unsigned int*>(&oc->plast[other]) > it + 1u) { post_skip = true; break; }
+      __nanosleep(spin < 4 ? 32 : 256);
+    }
+    if (!post_end && !post_skip) break;   // E is the other producer's iteration
+    const uint32_t s = it % kStages, ph = (it / kStages) & 1u;
+    if (it >= kLag) finish_stage<W>(P, smem, it - kLag);
+    helper_wait(P, &empty[s], ph ^ 1u, 128);
+    if (lane == 0) {
+      StageHdr* hd = reinterpret_cast<StageHdr*>(smem + Layout<W>::hdr + s * 128);
+      hd->t = post_end ? -1 : -2;
+      hd->sbase = 0;
+      hd->chunk0 = 0;
+      hd->lo = 0;
+      hd->hi = LLONG_MIN;
+      hd->stg_hi = 0;
+      hd->ra = hd->rb = 0;
+      hd->off_shift = 0;
+      hd->off_staged = 0;
+      mbar_arrive(&full[s]);    // keeps the stage's full phase in step (no bytes)
+      mbar_arrive(&ready[s]);
+    }
+    __syncwarp();
+    if (post_end) { it += kNP; break; }
+  }
+  // this producer's tiles whose bitmap is still pending (skip stages return at once)
+  for (uint32_t j = it >= kLag + kNP ? it - kLag : pw; j < it; j += kNP)
+    if (j + kLag >= it) finish_stage<W>(P, smem, j);
+}
+
 template <int W>
 __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
+  if constexpr (W == kWC || W == kII) {
+    if (P.tile_next) {
+      producer_loop_dyn<W>(P, smem, pw);
+      return;
+    }
+  }
   constexpr int kStages = Cfg<W>::kStages;
   const uint32_t lane = threadIdx.x & 31;
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
@@ -919,67 +1110,7 @@ __device__ void producer_loop(const Params& P, uint8_t* smem, uint32_t pw) {
           if (b_len) tma_load_1d(d + b_off, g + b_off, b_len, &full[s]);
         }
       } else {
-        const long long chunk0 = static_cast<long long>(t) * kT - P.a0;
-        const long long sbase = chunk0 - kLead;
-        const long long w_lo = max(0LL, sbase);
-        const long long w_hi = chunk0 + kT + kHalo;
-        const long long stg_hi = min(w_hi, N);
-        // stage bytes [w_lo, stg_hi) at sb + (w_lo - sbase); (rec + sbase) is 16-B aligned
-        uint8_t* d = sb + (w_lo - sbase);
-        const uint8_t* g = P.rec + w_lo;
-        if (!P.so) stage_copy_edges(d, g, static_cast<uint64_t>(max(0LL, stg_hi - w_lo)), lane, b_off, b_len);
-        // clear the record-start bitmap (map warps set bits after the full barrier)
-        if constexpr (!Cfg<W>::kLazyDir) {
-          uint32_t* bm = reinterpret_cast<uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits);
-          for (uint32_t i = lane; i < Cfg<W>::kBits / 16; i += 32) reinterpret_cast<uint4*>(bm)[i] = make_uint4(0, 0, 0, 0);
-        }
-        // offsets slice offsets[ra..rb) (record starts in the staged window)
-        const uint64_t cnt = rb - ra;
-        const bool staged = !Cfg<W>::kLazyDir && cnt <= static_cast<uint64_t>(Cfg<W>::kOffCap);
-        uint32_t shift = 0;
-        const uint8_t* og = reinterpret_cast<const uint8_t*>(P.off + ra);
-        if (staged && cnt) {
-          shift = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(og) & 15u);
-          // Copy the 16-B aligned superset of the slice with TMA alone (no synchronous edge
-          // loads on the producer's critical path) whenever it stays inside offsets[0..n].
-          const uint8_t* a_lo = og - shift;
-          const uint8_t* a_hi = reinterpret_cast<const uint8_t*>(
-              (reinterpret_cast<uintptr_t>(og + cnt * 8) + 15u) & ~static_cast<uintptr_t>(15u));
-          if (a_lo >= reinterpret_cast<const uint8_t*>(P.off) && a_hi <= P.off_end) {
-            o_off = 0;
-            o_len = static_cast<uint32_t>(a_hi - a_lo);
-            og = a_lo;
-            // so + shift still addresses offsets[ra]; the TMA below starts at so (= a_lo)
-          } else {
-            stage_copy_edges(so + shift, og, cnt * 8, lane, o_off, o_len);
-            og = og - shift;
-            o_off += shift;
-          }
-        }
-        if (lane == 0) {
-          hd->t = static_cast<long long>(t);
-          hd->sbase = sbase;
-          hd->chunk0 = chunk0;
-          hd->lo = max(0LL, chunk0);
-          hd->hi = min(N, chunk0 + kT);
-          hd->stg_hi = stg_hi;
-          hd->ra = ra;
-          hd->rb = rb;
-          hd->off_shift = shift;
-          hd->off_staged = staged ? 1u : 0u;
-        }
-        __syncwarp();
-        if (lane == 0) {
-          mbar_arrive_expect_tx(&full[s], b_len + o_len);
-          if (BMR_STREAM_HINT && P.xtab) {   // WC with the L2 count table: the input streams past it
-            const uint64_t pol = l2_policy_evict_first();
-            if (b_len) tma_load_1d_stream(d + b_off, g + b_off, b_len, &full[s], pol);
-            if (o_len) tma_load_1d_stream(so + o_off, og + o_off, o_len, &full[s], pol);
-          } else {
-            if (b_len) tma_load_1d(d + b_off, g + b_off, b_len, &full[s]);
-            if (o_len) tma_load_1d(so + o_off, og + o_off, o_len, &full[s]);
-          }
-        }
+        issue_text_stage<W>(P, smem, s, t, ra, rb);
         // L2 prefetch of this producer's tile P.pf tiles ahead (bytes + offsets slice): the TMA of
         // that tile then hits L2, so the kLag stages in flight cover L2 latency, not HBM latency
         if (P.pf) {
@@ -1449,6 +1580,114 @@ __device__ __forceinline__ void wc_drain_tab(const Params& P, LWord* lq, uint32_
   qn = rest;
 }
 
+// Table mode with asynchronous probes (BMR_WC_ADRAIN): a drain resolves the warp's PREVIOUS batch
+// of 32 long words and only issues this one.  Issue: the same keys, match groups and first slot
+// as wc_drain_tab; each group leader stores its key in the warp's pending area and starts a
+// cp.async of its first probe slot (8-B mid slot / 16-B long slot) next to it.  Resolve (one drain
+// later, several windows of work after the issue, so the L2 round trip is long over): the
+// prefetched slot is used as the first probe.  A stale slot value is safe — a slot only ever goes
+// from empty to one key: a key seen is the slot's key for good, an empty slot is claimed by CAS
+// (which returns the real value), and a torn 16-B view (low half only) is re-read atomically.
+struct PEnt { unsigned long long klo, khi, vlo, vhi; };
+struct PendQ {
+  PEnt* e;          // 32 entries per warp (the exact-key queue region, unused in table mode)
+  uint32_t* meta;   // per lane: bit 31 pending, bit 30 mid, bits 0..5 group size
+  uint32_t* slot;   // per lane: first probe slot
+};
+__device__ __forceinline__ void wc_probe_resolve(const Params& P, const PendQ& pq) {
+  const uint32_t lane = threadIdx.x & 31;
+  cp_async_wait_all();
+  const uint32_t meta = pq.meta[lane];
+  if (meta >> 31) {
+    const PEnt e = pq.e[lane];
+    const bool mid = (meta >> 30) & 1u;
+    const uint32_t cnt = meta & 63u;
+    const uint32_t stripe = (blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1);
+    uint64_t h = pq.slot[lane];
+    bool todo = true;
+    unsigned long long vlo = e.vlo, vhi = e.vhi;   // first probe: the prefetched slot
+    if (mid) {
+      const uint64_t mmask = (1ULL << P.mbits) - 1ULL;
+      for (uint32_t pr = 0; pr < kMidProbes; ++pr) {
+        unsigned long long k = pr ? *reinterpret_cast<volatile unsigned long long*>(P.mkeys + h) : vlo;
+        if (k == kMidEmpty) k = atomicCAS(reinterpret_cast<unsigned long long*>(P.mkeys + h), kMidEmpty, e.klo);
+        if (k == e.klo || k == kMidEmpty) {
+          red_add_u32(P.mcnt + h * kMidStripes + stripe, cnt);
+          todo = false;
+          break;
+        }
+        h = (h + 1) & mmask;
+      }
+    } else {
+      const uint64_t lmask = (1ULL << P.lbits) - 1ULL;
+      for (uint32_t pr = 0; pr < kMidProbes; ++pr) {
+        unsigned long long* sl = reinterpret_cast<unsigned long long*>(P.lkeys + 2 * h);
+        unsigned long long olo = vlo, ohi = vhi;
+        if (pr) asm volatile("ld.volatile.global.v2.u64 {%0, %1}, [%2];" : "=l"(olo), "=l"(ohi) : "l"(sl) : "memory");
+        if (olo != 0 && ohi == 0) olo = cas128(sl, 0ULL, 0ULL, 0ULL, 0ULL, ohi);   // torn view: atomic re-read
+        if (olo == 0) {
+          olo = cas128(sl, 0ULL, 0ULL, e.klo, e.khi, ohi);
+          if (olo == 0) { olo = e.klo; ohi = e.khi; }
+        }
+        if (olo == e.klo && ohi == e.khi) {
+          red_add_u32(P.lcnt + h * kMidStripes + stripe, cnt);
+          todo = false;
+          break;
+        }
+        h = (h + 1) & lmask;
+      }
+    }
+    if (todo) {   // table too full: counted, the batch is replayed with a larger table (D7)
+      atomicOr(&P.st->err, mid ? kErrMidTable : kErrLongTable);
+      atomicAdd(mid ? &P.st->mid_fail : &P.st->long_fail, 1ULL);
+    }
+    pq.meta[lane] = 0;
+  }
+  __syncwarp();
+}
+__device__ __forceinline__ void wc_probe_issue(const Params& P, LWord* lq, uint32_t& qn, const PendQ& pq) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t n = min(qn, 32u);
+  if (n == 0) return;
+  __syncwarp();
+  const bool in = lane < n;
+  LWord w{0, 0, 0};
+  if (in) w = lq[lane];
+  const uint32_t len = static_cast<uint32_t>(w.meta & 0xFFFFu);
+  const bool mid = in && len <= kMidMax, lng = in && !mid;
+  const uint64_t klo = mid ? exact_key(w.lo, len) : lng ? w.lo : ~0ULL;
+  const uint64_t khi = mid ? 0ULL : lng ? (len >= 16 ? w.hi : (w.hi & ((1ULL << (8 * (len - 8))) - 1ULL))) : ~0ULL;
+  const uint32_t grp = __match_any_sync(kFull, klo) & __match_any_sync(kFull, khi);
+  const bool lead = in && lane == static_cast<uint32_t>(__ffs(grp) - 1);
+  if (lead) {
+    const uint64_t h = mid ? mid_slot(klo, P.mbits) : long_slot(klo, khi, P.lbits);
+    PEnt* e = pq.e + lane;
+    e->klo = klo;
+    e->khi = khi;
+    if (mid) cp_async_8(&e->vlo, P.mkeys + h);
+    else cp_async_16(&e->vlo, P.lkeys + 2 * h);
+    pq.slot[lane] = static_cast<uint32_t>(h);
+    pq.meta[lane] = (1u << 31) | (mid ? (1u << 30) : 0u) | static_cast<uint32_t>(__popc(grp));
+  }
+  cp_async_commit();
+  const uint32_t rest = qn - n;
+  LWord r{0, 0, 0};
+  if (lane < rest) r = lq[n + lane];
+  __syncwarp();
+  if (lane < rest) lq[lane] = r;
+  __syncwarp();
+  qn = rest;
+}
+// drain of the table mode: synchronous (wc_drain_tab) or resolve-previous + issue
+__device__ __forceinline__ void wc_drain_tq(const Params& P, LWord* lq, uint32_t& qn, const PendQ& pq) {
+#if BMR_WC_ADRAIN
+  wc_probe_resolve(P, pq);
+  wc_probe_issue(P, lq, qn, pq);
+#else
+  wc_drain_tab(P, lq, qn);
+#endif
+}
+
 // end of a warp's work: sentinel entries in its chunks' unused tails
 __device__ __forceinline__ void wc_chunk_pads(const Params& P, const LOut& lo) {
   const uint32_t lane = threadIdx.x & 31;
@@ -1635,17 +1874,28 @@ __device__ __forceinline__ void comb_or_table(uint32_t* slot_key, uint32_t* slot
 // long-word queue one per lane per round.  The same words, keys and tables as wc_window.
 template <bool kX>
 __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8_t* outh, const TileView& tv,
-                                              long long p0w, uint32_t* ctab, LWord* lq, uint32_t& qn) {
+                                              long long p0w, uint32_t* ctab, LWord* lq, uint32_t& qn,
+                                              uint32_t* dummy, const PendQ& pq) {
   const uint32_t lane = threadIdx.x & 31;
   const long long N = bd_nbytes();
   const long long p0 = p0w + 16 * lane;
   const uint32_t i0 = static_cast<uint32_t>(p0 - tv.sbase);   // 16-B aligned stage offset
   const uint4 c0 = *reinterpret_cast<const uint4*>(tv.sb + i0);
-  const uint4 c1 = *reinterpret_cast<const uint4*>(tv.sb + i0 + 16);   // next chunk (lane 31: the halo)
   const uint32_t pb = tv.sb[i0 - 1];                                    // byte before the chunk (lead bytes)
+#if BMR_WC_CLS16
+  // classes of the lane's own 16 bytes; those of the next 16 come from the next lane, and lane
+  // 31's (the 16 bytes after the window) from lanes 0..3, one 4-byte word each (OR-reduced)
+  const uint32_t own = word_mask4(c0.x) | (word_mask4(c0.y) << 4) | (word_mask4(c0.z) << 8) | (word_mask4(c0.w) << 12);
+  const uint32_t hw = *reinterpret_cast<const uint32_t*>(tv.sb + (i0 - 16u * lane) + kWin + 4u * (lane & 3u));
+  const uint32_t halo = __reduce_or_sync(kFull, lane < 4u ? word_mask4(hw) << (4u * lane) : 0u);
+  const uint32_t nxt = __shfl_down_sync(kFull, own, 1);
+  uint32_t wm = own | ((lane == 31u ? halo : nxt) << 16);
+#else
+  const uint4 c1 = *reinterpret_cast<const uint4*>(tv.sb + i0 + 16);   // next chunk (lane 31: the halo)
   uint32_t wm = word_mask4(c0.x) | (word_mask4(c0.y) << 4) | (word_mask4(c0.z) << 8) | (word_mask4(c0.w) << 12) |
                 (word_mask4(c1.x) << 16) | (word_mask4(c1.y) << 20) | (word_mask4(c1.z) << 24) |
                 (word_mask4(c1.w) << 28);
+#endif
   const bool edge = p0w < 0 || p0w + kWin + 16 > N;   // warp-uniform: only the input's first / last window
   if (edge) wm &= range_mask32(p0, 0, N);
   const uint32_t R = bits32(tv.bm, i0);                // record starts at p0 .. p0 + 31
@@ -1655,6 +1905,33 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
   const uint32_t near = (nb >> 1) | (nb >> 2) | (nb >> 3) | (nb >> 4) | (nb >> 5);   // ends within 5 bytes
   uint32_t* ccnt = ctab + Cfg<kWC>::kCombSlots;
   // exact words (<= 5 bytes): key from the stage, combiner slot or L2 count table
+#if BMR_WC_XLOOP
+  if constexpr (kX) {
+    // The same words, keys and tables as the loop below, written for fewer instructions per
+    // word: starts taken from the top (bfind), the length from the bit-reversed stop mask,
+    // 32-bit shared addresses throughout, and the combiner hit counted by an unconditional
+    // shared RED (a miss adds into this lane's dummy word) -- ptxas wraps every predicated
+    // atomic in a divergent loop in its own branch region.
+    const uint32_t sb32 = smem_u32(tv.sb) + i0;
+    const uint32_t kb32 = smem_u32(ctab);
+    const uint32_t dmy = smem_u32(dummy) + 4u * lane;
+    const uint32_t rnb = __brev(nb);
+    for (uint32_t E = S & near; E;) {
+      const uint32_t j = bfind_u32(E);
+      E &= ~(1u << j);
+      const uint32_t len = 31u - j - bfind_u32(rnb & (0x7FFFFFFFu >> j));   // first stop above j
+      const uint32_t a = sb32 + (j & ~3u);
+      const uint32_t w0 = lds_u32(a), w1 = lds_u32(a + 4u);
+      const uint32_t key = exact_key30_bf(__funnelshift_r(w0, w1, j << 3), __funnelshift_r(w1, w1, j << 3) & 0xFFu, len);
+      const uint32_t ka = kb32 + 4u * ((key * 0x9E3779B1u) >> (32 - kCombBits));
+      uint32_t v = lds_volatile_u32(ka);
+      if (v == kCombEmpty32) v = atom_cas_shared_u32(ka, kCombEmpty32, key);
+      const bool hit = v == key || v == kCombEmpty32;
+      red_shared_add_u32(hit ? ka + 4u * Cfg<kWC>::kCombSlots : dmy, 1u);
+      if (!hit) red_add_u32(P.xtab + key, 1u);
+    }
+  } else
+#endif
   for (uint32_t E = S & near; E; E &= E - 1) {
     const uint32_t j = __ffs(E) - 1;
     const uint32_t len = __ffs(nb >> (j + 1));         // 1..5: a stop within 5 bytes
@@ -1694,7 +1971,7 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
     if (tot <= static_cast<uint32_t>(Cfg<kWC>::kLQ)) {
       L &= ~t16;
       if (tot) {
-        while (qn + tot > static_cast<uint32_t>(Cfg<kWC>::kLQ)) wc_drain_tab(P, lq, qn);
+        while (qn + tot > static_cast<uint32_t>(Cfg<kWC>::kLQ)) wc_drain_tq(P, lq, qn, pq);
         LWord* d = lq + qn + incl - cs;
         for (uint32_t m = Ls; m; m &= m - 1, ++d) {
           const uint32_t j = __ffs(m) - 1;
@@ -1722,7 +1999,7 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
   for (;;) {   // one long word per lane per round, appended to the warp's queue
     const uint32_t m = __ballot_sync(kFull, L != 0);
     if (!m) break;
-    if (qn + __popc(m) > static_cast<uint32_t>(Cfg<kWC>::kLQ)) wc_drain_tab(P, lq, qn);
+    if (qn + __popc(m) > static_cast<uint32_t>(Cfg<kWC>::kLQ)) wc_drain_tq(P, lq, qn, pq);
     uint32_t j = 0, len = 0;
     if (L) {
       j = __ffs(L) - 1;
@@ -1778,6 +2055,12 @@ __device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   LWord* lq = reinterpret_cast<LWord*>(smem + Layout<kWC>::lq) + warp * Cfg<kWC>::kLQ;
   uint32_t qn = 0;   // long words queued by this warp
   LOut lo{0, 0, 0, 0};   // this warp's output chunks (none yet)
+  // table mode: the exact-key / hash queues are unused -> dummy words, pending probes
+  const PendQ pq{reinterpret_cast<PEnt*>(xq), hq + 32, hq + 64};
+  if constexpr (kTab) {
+    pq.meta[threadIdx.x & 31] = 0;
+    __syncwarp();
+  }
   uint32_t have_it = ~0u;
   long long t = 0, sbase = 0, hi = 0, stg_hi = 0;
   for (;;) {
@@ -1793,16 +2076,16 @@ __device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       stg_hi = hd->stg_hi;
       have_it = it;
     }
-    if (t < 0) break;
+    if (t == -1) break;   // (-2: a skip stage, no windows)
     const long long wp = sbase + kLead + static_cast<long long>(w) * kWin;
     if (wp < hi) {   // warp-uniform
       const TileView tv{smem + Layout<W>::bytes + s * kStageBytes,
                         reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits), sbase, stg_hi, 0,
                         0};
-      if constexpr (kTab) wc_window_tab<kMode == 1>(P, oc, outh, tv, wp, ctab, lq, qn);
+      if constexpr (kTab) wc_window_tab<kMode == 1>(P, oc, outh, tv, wp, ctab, lq, qn, hq, pq);
       else wc_window(P, oc, outh, tv, wp, xq, hq, ctab, lq, qn, lo);
       if (qn >= 32) {
-        if constexpr (kTab) wc_drain_tab(P, lq, qn);
+        if constexpr (kTab) wc_drain_tq(P, lq, qn, pq);
         else wc_drain(P, lo, lq, qn);
       }
     }
@@ -1810,9 +2093,12 @@ __device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
     lane0_mbar_arrive(&empty[s]);
   }
   while (qn) {   // this warp's last long words
-    if constexpr (kTab) wc_drain_tab(P, lq, qn);
+    if constexpr (kTab) wc_drain_tq(P, lq, qn, pq);
     else wc_drain(P, lo, lq, qn);
   }
+#if BMR_WC_ADRAIN
+  if constexpr (kTab) wc_probe_resolve(P, pq);   // the last batch issued
+#endif
   wc_chunk_pads(P, lo);
 }
 
@@ -2055,7 +2341,7 @@ __device__ __forceinline__ void ii_map_loop(const Params& P, uint8_t* smem, OutC
       stg_hi = hd->stg_hi;
       have_it = it;
     }
-    if (t < 0) break;
+    if (t == -1) break;   // (-2: a skip stage, no windows)
     const long long wp = sbase + kLead + static_cast<long long>(w) * kWin;
     if (wp < hi) {   // warp-uniform
       const TileView tv{smem + Layout<W>::bytes + s * kStageBytes,
@@ -2745,7 +3031,7 @@ __device__ void map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       hd = *reinterpret_cast<const StageHdr*>(smem + Layout<W>::hdr + s * 128);
       have_it = it;
     }
-    if (hd.t < 0) break;
+    if (hd.t == -1) break;   // (-2: a skip stage, no windows)
     const uint8_t* sb = smem + Layout<W>::bytes + s * kStageBytes;
     if constexpr (W == kKM) {
       const uint64_t i = static_cast<uint64_t>(hd.lo) + tid;
@@ -2913,6 +3199,8 @@ __global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
     oc->is_final = 0;
     oc->win_next = 0;
     oc->congested = 0;
+    oc->pout[0] = oc->pout[1] = ~0u;
+    oc->plast[0] = oc->plast[1] = 0;
     for (int b = 0; b < kNOut; ++b) { mbar_init(&oc->req[b], 1); mbar_init(&oc->done[b], 1); }
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + Layout<W>::full);
     uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Layout<W>::empty);
@@ -2987,7 +3275,7 @@ __global__ void __launch_bounds__(threads_of<W>(), 1) k_map(Params P) {
 // [w_lo, w_hi) of every tile.
 __global__ void k_tile_bounds(const uint64_t* off, uint64_t n, long long a0, uint64_t tb_cap, const uint64_t* prev,
                               uint64_t input_base, const uint8_t* rec, uint64_t* desc, uint64_t* tb,
-                              unsigned int* err) {
+                              unsigned int* err, unsigned long long* tile_next) {
   const uint64_t nbytes = off[n];
   const uint64_t ntiles = nbytes ? (nbytes + static_cast<uint64_t>(a0) + kT - 1) / kT : 0;
   const bool null_rec = nbytes && !rec;
@@ -2996,6 +3284,7 @@ __global__ void k_tile_bounds(const uint64_t* off, uint64_t n, long long a0, uin
     desc[1] = ntiles;
     desc[2] = prev ? prev[2] + prev[0] : input_base;
     desc[3] = (ntiles > tb_cap || null_rec) ? 1ULL : 0ULL;   // the Map skips the batch
+    *tile_next = 0;                                           // the Map's dynamic tile counter
     if (ntiles > tb_cap) atomicOr(err, kErrTileCap);
     if (null_rec) atomicOr(err, kErrNullRecords);
   }
@@ -3081,12 +3370,13 @@ cudaError_t launch_w(const MapArgs& a, int num_sms, cudaStream_t s) {
   P.lkeys = (BMR_LTAB && tabs) ? a.out.lkeys : nullptr;
   P.lcnt = (BMR_LTAB && tabs) ? a.out.lcnt : nullptr;
   P.lbits = a.out.lbits;
+  P.tile_next = (BMR_DYN_TILES && (W == kWC || W == kII)) ? &a.st->tile_next : nullptr;
   P.km_bound = (W == kKM && !(a.flags & 0x1000u) && a.k <= static_cast<uint32_t>(kKmBoundMax)) ? 1u : 0u;   // MR_FLAG_KM_FULL_SCAN
   if (W == kKM && P.ntiles == 0) return cudaSuccess;
   if constexpr (W != kKM) {
     const unsigned blocks = static_cast<unsigned>(std::min<uint64_t>((a.tb_cap + 255) / 256 + 1, 8ULL * num_sms));
     k_tile_bounds<<<blocks, 256, 0, s>>>(a.offsets, a.n, P.a0, a.tb_cap, a.prev_desc, a.input_base, a.records,
-                                         a.desc, a.tile_bounds, &a.st->err);
+                                         a.desc, a.tile_bounds, &a.st->err, &a.st->tile_next);
     count_launch();
   }
   const size_t smem = Layout<W>::cent + (W == kKM ? static_cast<size_t>(a.k) * (P.km_bound ? 68 : 32) : 0);
