@@ -626,16 +626,48 @@ mr_status settle_map(mr_job* job) {
     CK(job->mtab_keys.ensure(1ULL << job->mbits), "grow mid table");
     CK(job->mtab_cnt.ensure((1ULL << job->mbits) * kMidStripes), "grow mid table");
   }
-  const uint64_t m = hs->pair_cursor, mb = job->split() ? hs->pair_cursor_b : 0;
-  const uint64_t mc = job->split() ? hs->pair_cursor_c : 0;
-  const uint64_t mp = job->wc_comb() ? hs->pair_cursor_p : 0;
-  if (tile_over || mid_over || long_over || m > job->cap || mb > job->cap_b || mc > job->cap_c || mp > job->cap_p) {
-    if (tile_over) job->tb_cap = max_tiles + 1024;   // (tb itself is grown by launch_batch)
+  // Grow from the demand counted past capacity and replay every batch.  The demand of a run is
+  // not exactly that of the next: flush / spill padding and the warp-private chunks depend on
+  // which warps and CTAs took which windows and tiles (dynamic scheduling), so a replay that
+  // still overflows grows again from its own demand (up to kMaxReplays rounds).
+  constexpr int kMaxReplays = 4;
+  for (int round = 0;; ++round) {
+    const uint64_t m = hs->pair_cursor, mb = job->split() ? hs->pair_cursor_b : 0;
+    const uint64_t mc = job->split() ? hs->pair_cursor_c : 0;
+    const uint64_t mp = job->wc_comb() ? hs->pair_cursor_p : 0;
+    const bool t_over = (hs->err & kErrTileCap) != 0, m_over = (hs->err & kErrMidTable) != 0;
+    const bool l_over = (hs->err & kErrLongTable) != 0;
+    if (!(t_over || m_over || l_over || m > job->cap || mb > job->cap_b || mc > job->cap_c || mp > job->cap_p))
+      return MR_OK;
+    if (round == kMaxReplays) return fail(job, MR_ERR_OOM, "replay still overflows");
+    if (round > 0) {   // tables overflowing again after a replay: grow them again
+      if (l_over) {
+        job->lbits += 2;
+        job->ltab_keys.release();
+        job->ltab_cnt.release();
+        CK(job->ltab_keys.ensure(2ULL << job->lbits), "grow long table");
+        CK(job->ltab_cnt.ensure((1ULL << job->lbits) * kMidStripes), "grow long table");
+      }
+      if (m_over) {
+        job->mbits += 2;
+        job->mtab_keys.release();
+        job->mtab_cnt.release();
+        CK(job->mtab_keys.ensure(1ULL << job->mbits), "grow mid table");
+        CK(job->mtab_cnt.ensure((1ULL << job->mbits) * kMidStripes), "grow mid table");
+      }
+      if (t_over) {   // (the descriptors of the replay)
+        CK(job->bdesc_h.ensure(4ULL * job->ndesc), "alloc host descriptors");
+        CK(cudaMemcpyAsync(job->bdesc_h.p, job->bdesc.p, 32ULL * job->ndesc, cudaMemcpyDeviceToHost, job->stream),
+           "D2H descriptors");
+        CK(cudaStreamSynchronize(job->stream), "sync descriptors");
+        for (uint32_t i = 0; i < job->ndesc; ++i) max_tiles = std::max(max_tiles, job->bdesc_h.p[4 * i + 1]);
+      }
+    }
+    if (t_over) job->tb_cap = max_tiles + 1024;   // (tb itself is grown by launch_batch)
     const uint64_t ncap_p = job->wc_comb() ? std::max(job->cap_p, mp + mp / 8 + 4096) : 0;
     const uint64_t ncap = std::max(job->cap, m + m / 8 + 4096);
     // the mid / hashed streams are appended in warp-private chunks (map.cu kLChunk = 256 entries):
-    // a run may leave up to a chunk unused per map warp, and which warps see long words varies
-    // between runs (dynamic windows and tiles), so the replay adds a chunk per warp of headroom
+    // a run may leave up to a chunk unused per map warp
     const uint64_t chunk_slack = static_cast<uint64_t>(job->nsm) * 24u * 256u;
     const uint64_t ncap_b = job->split() ? std::max(job->cap_b, mb + mb / 8 + 4096 + chunk_slack) : 0;
     const uint64_t ncap_c = job->split() ? std::max(job->cap_c, mc + mc / 8 + 4096 + chunk_slack) : 0;
@@ -649,7 +681,7 @@ mr_status settle_map(mr_job* job) {
     }
     job->stats.capacity_pairs = job->cap + job->cap_b + job->cap_c;
     CK(cudaMemsetAsync(job->st, 0, sizeof(DevState), job->stream), "reset cursor");
-    if (job->xtab_dirty || mid_over || long_over) CK(clear_tables(job), "clear the tables");
+    if (job->xtab_dirty || m_over || l_over) CK(clear_tables(job), "clear the tables");
     if (job->km_comb()) {
       CK(cudaMemsetAsync(job->sums.p, 0, 64ULL * job->k, job->stream), "reset sums");
       CK(cudaMemsetAsync(job->cnts.p, 0, 8ULL * job->k, job->stream), "reset counts");
@@ -657,10 +689,6 @@ mr_status settle_map(mr_job* job) {
     for (const Batch& b : job->batches) CK(launch_batch(job, b), "replay");
     job->stats.replays += job->batches.size();
     CK(read_state(job), "replay (async)");
-    if ((hs->err & (kErrTileCap | kErrMidTable | kErrLongTable)) || hs->pair_cursor > job->cap ||
-        (job->split() && (hs->pair_cursor_b > job->cap_b || hs->pair_cursor_c > job->cap_c)) ||
-        (job->wc_comb() && hs->pair_cursor_p > job->cap_p))
-      return fail(job, MR_ERR_OOM, "replay still overflows");
   }
   return MR_OK;
 }
@@ -859,7 +887,7 @@ mr_status tables_extract(mr_job* job) {
   CK(cudaMemsetAsync(cur, 0, sizeof(unsigned long long), s), "memset cursor");
   if (job->mkeys_out.n < 4096) { CK(job->mkeys_out.ensure(1 << 18), "alloc mid keys"); CK(job->mcounts.ensure(1 << 18), "alloc mid counts"); }
   cap = std::min(job->mkeys_out.n, job->mcounts.n);
-  CK(launch_mtab_extract(job->mtab_keys.p, job->mtab_cnt.p, job->mtab_keys.n, job->mkeys_out.p, job->mcounts.p, cap, cur,
+  CK(launch_mtab_extract(job->mtab_keys.p, job->mtab_cnt.p, job->mtab_keys.n, job->mbits, job->mkeys_out.p, job->mcounts.p, cap, cur,
                          wsum, job->nsm, s),
      "mid table extract");
   CK(read_state(job), "sync mid table extract");
@@ -870,7 +898,7 @@ mr_status tables_extract(mr_job* job) {
     job->tmp_h.p[4] = cap;
     CK(cudaMemcpyAsync(cur, job->tmp_h.p + 4, 8, cudaMemcpyHostToDevice, s), "set cursor");
     const uint64_t cap2 = std::min(job->mkeys_out.n, job->mcounts.n);
-    CK(launch_mtab_extract(job->mtab_keys.p, job->mtab_cnt.p, job->mtab_keys.n, job->mkeys_out.p, job->mcounts.p, cap2,
+    CK(launch_mtab_extract(job->mtab_keys.p, job->mtab_cnt.p, job->mtab_keys.n, job->mbits, job->mkeys_out.p, job->mcounts.p, cap2,
                            cur, wsum, job->nsm, s),
        "mid table extract");
     CK(read_state(job), "sync mid table extract");
@@ -887,7 +915,7 @@ mr_status tables_extract(mr_job* job) {
     CK(job->lcounts.ensure(slots), "alloc long counts");
   }
   uint64_t lcap = std::min({job->lkeys_out.n / 2, job->lkref_out.n, job->lcounts.n});
-  CK(launch_ltab_extract(job->ltab_keys.p, job->ltab_cnt.p, job->ltab_keys.n / 2, job->lkeys_out.p, job->lkref_out.p,
+  CK(launch_ltab_extract(job->ltab_keys.p, job->ltab_cnt.p, job->ltab_keys.n / 2, job->lbits, job->lkeys_out.p, job->lkref_out.p,
                          job->lcounts.p, lcap, cur, wsum, job->nsm, s),
      "long table extract");
   CK(read_state(job), "sync long table extract");

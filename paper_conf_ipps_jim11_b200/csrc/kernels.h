@@ -50,6 +50,11 @@ constexpr uint32_t kMidProbes = 32;
 // counts of a slot are striped over kMidStripes words (the warp's stripe), so the Zipf-hot mid
 // words do not serialise every RED on one address; the extraction sums the stripes
 constexpr uint32_t kMidStripes = 16;
+// stripe-major: stripe q of slot h at q * 2^bits + h, so the stripes of a Zipf-hot word sit in
+// kMidStripes different L2 lines (slot-major they shared one line, and its REDs serialised there)
+__host__ __device__ inline uint64_t stripe_at(uint64_t slot, uint32_t stripe, uint32_t bits) {
+  return (static_cast<uint64_t>(stripe) << bits) | slot;
+}
 __host__ __device__ inline uint64_t mid_slot(uint64_t key, uint32_t bits) {
   return (key * 0x9E3779B97F4A7C15ULL) >> (64 - bits);
 }
@@ -239,11 +244,11 @@ cudaError_t launch_xtab_extract_list(uint32_t* tab, uint64_t nent, uint32_t* oke
                                      unsigned long long* cursor, unsigned long long* wsum, int num_sms, cudaStream_t s);
 // WC long-word table -> the final long keys: 16 zero-padded key bytes per key (okeys, 2 x u64),
 // their references (okref = (address of the bytes << 16) | length) and counts; slots reset
-cudaError_t launch_ltab_extract(uint64_t* lkeys, uint32_t* lcnt, uint64_t nslots, uint64_t* okeys, uint64_t* okref,
+cudaError_t launch_ltab_extract(uint64_t* lkeys, uint32_t* lcnt, uint64_t nslots, uint32_t bits, uint64_t* okeys, uint64_t* okref,
                                 uint64_t* ocounts, uint64_t cap, unsigned long long* cursor, unsigned long long* wsum,
                                 int num_sms, cudaStream_t s);
 // WC mid table -> (48-bit key, count) lists; extracted slots are reset (key empty, count 0)
-cudaError_t launch_mtab_extract(uint64_t* mkeys, uint32_t* mcnt, uint64_t nslots, uint64_t* okeys, uint64_t* ocounts,
+cudaError_t launch_mtab_extract(uint64_t* mkeys, uint32_t* mcnt, uint64_t nslots, uint32_t bits, uint64_t* okeys, uint64_t* ocounts,
                                 uint64_t cap, unsigned long long* cursor, unsigned long long* wsum, int num_sms,
                                 cudaStream_t s);
 cudaError_t launch_key_decode_list32(const uint32_t* keys, uint64_t n, const uint64_t* key_off, uint8_t* out,

@@ -127,6 +127,15 @@ constexpr int nprod() { return W == 4 ? BMR_II_NPROD : 2; }
 #ifndef BMR_WC_XLOOP
 #define BMR_WC_XLOOP 1   // WordCount table mode: lean exact-word loop (bfind starts, 32-bit shared addresses, unconditional shared RED)
 #endif
+#ifndef BMR_WC_XPAIR
+#define BMR_WC_XPAIR 1   // WordCount table mode: two exact words per loop iteration
+#endif
+#ifndef BMR_WC_LBALLOT
+#define BMR_WC_LBALLOT 1   // WordCount table mode: long-word queue offsets from ballots (no shuffle scan)
+#endif
+#ifndef BMR_WC_X2WAY
+#define BMR_WC_X2WAY 0   // WordCount table mode: second combiner slot (home ^ 1) for exact words
+#endif
 #ifndef BMR_WC_CLS16
 #define BMR_WC_CLS16 1   // WordCount table mode: each lane classifies its own 16 bytes only (next chunk by shuffle)
 #endif
@@ -1363,6 +1372,21 @@ __device__ __forceinline__ uint32_t exact_key30_bf(uint32_t lo, uint32_t b4, uin
   return y | (len == 5u ? (c4 << 24) : 0u);
 }
 
+// The same key from the word's first 4 bytes and the 4 bytes from byte 4 on (hiw, only its low
+// byte used): the fifth code is computed on the whole word and masked, not narrowed by the
+// compiler into byte-wise selects (8 instructions fewer per word)
+__device__ __forceinline__ uint32_t opaque_u32(uint32_t x) {
+  asm("" : "+r"(x));
+  return x;
+}
+__device__ __forceinline__ uint32_t exact_key30_w(uint32_t lo, uint32_t hiw, uint32_t len) {
+  const uint32_t c = exact_codes4(lo) & __funnelshift_lc(0xFFFFFFFFu, 0u, 8u * len);   // bytes < len
+  uint32_t y = (c & 0x003F003Fu) | ((c >> 2) & 0x0FC00FC0u);   // byte pairs -> 12 bits
+  y = (y & 0x00000FFFu) | ((y >> 4) & 0x00FFF000u);            // -> 24 bits
+  const uint32_t c4 = opaque_u32(exact_codes4(opaque_u32(hiw)));
+  return y | ((c4 << 24) & (len == 5u ? 0x3F000000u : 0u));
+}
+
 // 128-bit compare-and-swap on global memory (sm_90+ ATOMG.CAS.128): returns the old low half,
 // the old high half in *ohi
 __device__ __forceinline__ unsigned long long cas128(unsigned long long* p, unsigned long long clo,
@@ -1454,7 +1478,7 @@ __device__ __forceinline__ void wc_drain(const Params& P, LOut& lo, LWord* lq, u
                                           : *reinterpret_cast<volatile unsigned long long*>(P.mkeys + h);
       if (k == kMidEmpty) k = atomicCAS(reinterpret_cast<unsigned long long*>(P.mkeys + h), kMidEmpty, key);
       if (k == key || k == kMidEmpty) {
-        red_add_u32(P.mcnt + h * kMidStripes + ((blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1)),
+        red_add_u32(P.mcnt + stripe_at(h, (blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1), P.mbits),
                     static_cast<uint32_t>(__popc(grp)));
         done = true;
         break;
@@ -1487,7 +1511,7 @@ __device__ __forceinline__ void wc_drain(const Params& P, LOut& lo, LWord* lq, u
         if (olo == 0) { olo = klo; ohi = khi; }   // claimed by this lane
       }
       if (olo == klo && ohi == khi) {
-        red_add_u32(P.lcnt + h * kMidStripes + ((blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1)),
+        red_add_u32(P.lcnt + stripe_at(h, (blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1), P.lbits),
                     static_cast<uint32_t>(__popc(grp)));
         done = true;
         break;
@@ -1547,7 +1571,7 @@ __device__ __forceinline__ void wc_drain_tab(const Params& P, LWord* lq, uint32_
       unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(P.mkeys + h);
       if (k == kMidEmpty) k = atomicCAS(reinterpret_cast<unsigned long long*>(P.mkeys + h), kMidEmpty, klo);
       if (k == klo || k == kMidEmpty) {
-        red_add_u32(P.mcnt + h * kMidStripes + stripe, static_cast<uint32_t>(__popc(grp)));
+        red_add_u32(P.mcnt + stripe_at(h, stripe, P.mbits), static_cast<uint32_t>(__popc(grp)));
         todo = false;
       }
       h = (h + 1) & mmask;
@@ -1561,7 +1585,7 @@ __device__ __forceinline__ void wc_drain_tab(const Params& P, LWord* lq, uint32_
         if (olo == 0) { olo = klo; ohi = khi; }
       }
       if (olo == klo && ohi == khi) {
-        red_add_u32(P.lcnt + h * kMidStripes + stripe, static_cast<uint32_t>(__popc(grp)));
+        red_add_u32(P.lcnt + stripe_at(h, stripe, P.lbits), static_cast<uint32_t>(__popc(grp)));
         todo = false;
       }
       h = (h + 1) & lmask;
@@ -1612,7 +1636,9 @@ __device__ __forceinline__ void wc_probe_resolve(const Params& P, const PendQ& p
         unsigned long long k = pr ? *reinterpret_cast<volatile unsigned long long*>(P.mkeys + h) : vlo;
         if (k == kMidEmpty) k = atomicCAS(reinterpret_cast<unsigned long long*>(P.mkeys + h), kMidEmpty, e.klo);
         if (k == e.klo || k == kMidEmpty) {
-          red_add_u32(P.mcnt + h * kMidStripes + stripe, cnt);
+#if !(defined(BMR_DIAG) && BMR_DIAG == 8)
+          red_add_u32(P.mcnt + stripe_at(h, stripe, P.mbits), cnt);
+#endif
           todo = false;
           break;
         }
@@ -1630,7 +1656,9 @@ __device__ __forceinline__ void wc_probe_resolve(const Params& P, const PendQ& p
           if (olo == 0) { olo = e.klo; ohi = e.khi; }
         }
         if (olo == e.klo && ohi == e.khi) {
-          red_add_u32(P.lcnt + h * kMidStripes + stripe, cnt);
+#if !(defined(BMR_DIAG) && BMR_DIAG == 8)
+          red_add_u32(P.lcnt + stripe_at(h, stripe, P.lbits), cnt);
+#endif
           todo = false;
           break;
         }
@@ -1657,7 +1685,11 @@ __device__ __forceinline__ void wc_probe_issue(const Params& P, LWord* lq, uint3
   const bool mid = in && len <= kMidMax, lng = in && !mid;
   const uint64_t klo = mid ? exact_key(w.lo, len) : lng ? w.lo : ~0ULL;
   const uint64_t khi = mid ? 0ULL : lng ? (len >= 16 ? w.hi : (w.hi & ((1ULL << (8 * (len - 8))) - 1ULL))) : ~0ULL;
+#if defined(BMR_DIAG) && BMR_DIAG == 6
+  const uint32_t grp = 1u << lane;   // (timing diagnostic: no aggregation)
+#else
   const uint32_t grp = __match_any_sync(kFull, klo) & __match_any_sync(kFull, khi);
+#endif
   const bool lead = in && lane == static_cast<uint32_t>(__ffs(grp) - 1);
   if (lead) {
     const uint64_t h = mid ? mid_slot(klo, P.mbits) : long_slot(klo, khi, P.lbits);
@@ -1670,6 +1702,9 @@ __device__ __forceinline__ void wc_probe_issue(const Params& P, LWord* lq, uint3
     pq.meta[lane] = (1u << 31) | (mid ? (1u << 30) : 0u) | static_cast<uint32_t>(__popc(grp));
   }
   cp_async_commit();
+#if defined(BMR_DIAG) && BMR_DIAG == 9
+  pq.meta[lane] = 0;   // (timing diagnostic: keys and groups computed, never probed)
+#endif
   const uint32_t rest = qn - n;
   LWord r{0, 0, 0};
   if (lane < rest) r = lq[n + lane];
@@ -1680,6 +1715,10 @@ __device__ __forceinline__ void wc_probe_issue(const Params& P, LWord* lq, uint3
 }
 // drain of the table mode: synchronous (wc_drain_tab) or resolve-previous + issue
 __device__ __forceinline__ void wc_drain_tq(const Params& P, LWord* lq, uint32_t& qn, const PendQ& pq) {
+#if defined(BMR_DIAG) && BMR_DIAG == 5
+  qn = 0;   // (timing diagnostic: long words queued, never counted)
+  return;
+#endif
 #if BMR_WC_ADRAIN
   wc_probe_resolve(P, pq);
   wc_probe_issue(P, lq, qn, pq);
@@ -1841,7 +1880,7 @@ __device__ __forceinline__ void mid_insert(const Params& P, uint64_t key, uint32
     unsigned long long k = *reinterpret_cast<volatile unsigned long long*>(P.mkeys + h);
     if (k == kMidEmpty) k = atomicCAS(reinterpret_cast<unsigned long long*>(P.mkeys + h), kMidEmpty, key);
     if (k == key || k == kMidEmpty) {
-      red_add_u32(P.mcnt + h * kMidStripes + stripe, cnt);
+      red_add_u32(P.mcnt + stripe_at(h, stripe, P.mbits), cnt);
       return;
     }
   }
@@ -1916,13 +1955,73 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
     const uint32_t kb32 = smem_u32(ctab);
     const uint32_t dmy = smem_u32(dummy) + 4u * lane;
     const uint32_t rnb = __brev(nb);
-    for (uint32_t E = S & near; E;) {
-      const uint32_t j = bfind_u32(E);
-      E &= ~(1u << j);
+    // key of the exact word starting at chunk byte j (a stop within 5 bytes after it)
+    auto xkey = [&](uint32_t j) {
       const uint32_t len = 31u - j - bfind_u32(rnb & (0x7FFFFFFFu >> j));   // first stop above j
       const uint32_t a = sb32 + (j & ~3u);
       const uint32_t w0 = lds_u32(a), w1 = lds_u32(a + 4u);
-      const uint32_t key = exact_key30_bf(__funnelshift_r(w0, w1, j << 3), __funnelshift_r(w1, w1, j << 3) & 0xFFu, len);
+      return exact_key30_w(__funnelshift_r(w0, w1, j << 3), __funnelshift_r(w1, w1, j << 3), len);
+    };
+#if defined(BMR_DIAG) && BMR_DIAG == 3
+    if (S) return;   // (timing diagnostic: no exact words, no long words)
+#endif
+#if defined(BMR_DIAG) && (BMR_DIAG == 1 || BMR_DIAG == 4)
+    if (BMR_DIAG == 4) {   // (timing diagnostic: exact words straight to the L2 table)
+      for (uint32_t E = S & near; E;) {
+        const uint32_t j = bfind_u32(E);
+        E &= ~(1u << j);
+        red_add_u32(P.xtab + xkey(j), 1u);
+      }
+    }
+    if (false)
+#endif
+#if BMR_WC_XPAIR
+    // two words per iteration (the highest and the lowest start left): the same instructions per
+    // word, two independent dependency chains (the loop is latency-bound), half the iterations
+    for (uint32_t E = S & near; E;) {
+      const uint32_t j1 = bfind_u32(E);
+      E &= ~(1u << j1);
+      const bool two = E != 0;
+      const uint32_t j2 = two ? static_cast<uint32_t>(__ffs(E)) - 1u : j1;
+      E &= E - 1u;
+      const uint32_t k1 = xkey(j1), k2 = xkey(j2);
+      uint32_t ka1 = kb32 + 4u * ((k1 * 0x9E3779B1u) >> (32 - kCombBits));
+      uint32_t ka2 = kb32 + 4u * ((k2 * 0x9E3779B1u) >> (32 - kCombBits));
+      uint32_t v1 = lds_volatile_u32(ka1), v2 = lds_volatile_u32(ka2);
+      if (v1 == kCombEmpty32) v1 = atom_cas_shared_u32(ka1, kCombEmpty32, k1);
+      if (two && v2 == kCombEmpty32) v2 = atom_cas_shared_u32(ka2, kCombEmpty32, k2);   // (CAS: the real slot)
+      bool h1 = v1 == k1 || v1 == kCombEmpty32;
+      bool h2 = two && (v2 == k2 || v2 == kCombEmpty32);
+#if BMR_WC_X2WAY
+      // a key whose home slot belongs to another key gets a second slot (home ^ 1): fewer words
+      // left to the L2 table, whose REDs on Zipf-hot keys serialise
+      if (!h1) {
+        const uint32_t kb = ka1 ^ 4u;
+        uint32_t v = lds_volatile_u32(kb);
+        if (v == kCombEmpty32) v = atom_cas_shared_u32(kb, kCombEmpty32, k1);
+        h1 = v == k1 || v == kCombEmpty32;
+        ka1 = h1 ? kb : ka1;
+      }
+      if (two && !h2) {
+        const uint32_t kb = ka2 ^ 4u;
+        uint32_t v = lds_volatile_u32(kb);
+        if (v == kCombEmpty32) v = atom_cas_shared_u32(kb, kCombEmpty32, k2);
+        h2 = v == k2 || v == kCombEmpty32;
+        ka2 = h2 ? kb : ka2;
+      }
+#endif
+      red_shared_add_u32(h1 ? ka1 + 4u * Cfg<kWC>::kCombSlots : dmy, 1u);
+      red_shared_add_u32(h2 ? ka2 + 4u * Cfg<kWC>::kCombSlots : dmy, 1u);
+#if !(defined(BMR_DIAG) && BMR_DIAG == 10)
+      if (!h1) red_add_u32(P.xtab + k1, 1u);
+      if (two && !h2) red_add_u32(P.xtab + k2, 1u);
+#endif
+    }
+#else
+    for (uint32_t E = S & near; E;) {
+      const uint32_t j = bfind_u32(E);
+      E &= ~(1u << j);
+      const uint32_t key = xkey(j);
       const uint32_t ka = kb32 + 4u * ((key * 0x9E3779B1u) >> (32 - kCombBits));
       uint32_t v = lds_volatile_u32(ka);
       if (v == kCombEmpty32) v = atom_cas_shared_u32(ka, kCombEmpty32, key);
@@ -1930,6 +2029,7 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
       red_shared_add_u32(hit ? ka + 4u * Cfg<kWC>::kCombSlots : dmy, 1u);
       if (!hit) red_add_u32(P.xtab + key, 1u);
     }
+#endif
   } else
 #endif
   for (uint32_t E = S & near; E; E &= E - 1) {
@@ -1953,6 +2053,9 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
   // longer words: only the lane's highest start can lack a visible end (no stop in the 31 - j
   // bytes after it)
   uint32_t L = S & ~near;
+#if defined(BMR_DIAG) && BMR_DIAG == 2
+  L = 0;
+#endif
   if (!__any_sync(kFull, L)) return;
 #if BMR_WC_LSCAN
   {
@@ -1966,8 +2069,18 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
     t16 |= t16 >> 8;
     const uint32_t Ls = L & t16;
     const uint32_t cs = __popc(Ls);
+#if BMR_WC_LBALLOT
+    // a lane holds at most 3 such starts (a long word and its delimiter take >= 7 of its 16
+    // bytes): the warp prefix from three ballots instead of a 5-step shuffle scan
+    const uint32_t b1 = __ballot_sync(kFull, cs >= 1u), b2 = __ballot_sync(kFull, cs >= 2u),
+                   b3 = __ballot_sync(kFull, cs >= 3u);
+    const uint32_t lt = lanemask_lt();
+    const uint32_t incl = __popc(b1 & lt) + __popc(b2 & lt) + __popc(b3 & lt) + cs;
+    const uint32_t tot = __popc(b1) + __popc(b2) + __popc(b3);
+#else
     const uint32_t incl = warp_inclusive_add(cs);
     const uint32_t tot = __shfl_sync(kFull, incl, 31);
+#endif
     if (tot <= static_cast<uint32_t>(Cfg<kWC>::kLQ)) {
       L &= ~t16;
       if (tot) {

@@ -756,7 +756,7 @@ cudaError_t launch_xtab_extract_list(uint32_t* tab, uint64_t nent, uint32_t* oke
 
 // WC mid table -> (key, count) lists.  Each key sits in exactly one slot (the Map's inserts find an
 // existing key before any empty slot), so the lists are the final mid keys; slots past `cap` stay.
-__global__ void __launch_bounds__(256) k_mtab_extract(uint64_t* __restrict__ mkeys, uint32_t* __restrict__ mcnt,
+__global__ void __launch_bounds__(256) k_mtab_extract(uint64_t* __restrict__ mkeys, uint32_t* __restrict__ mcnt, uint32_t bits,
                                                     uint64_t nslots, uint64_t* okeys, uint64_t* ocounts,
                                                     uint64_t cap, unsigned long long* cursor,
                                                     unsigned long long* wsum) {
@@ -775,19 +775,19 @@ __global__ void __launch_bounds__(256) k_mtab_extract(uint64_t* __restrict__ mke
     if (full && o < cap) {
       uint64_t c = 0;
 #pragma unroll
-      for (uint32_t q = 0; q < kMidStripes; ++q) c += mcnt[i * kMidStripes + q];
+      for (uint32_t q = 0; q < kMidStripes; ++q) c += mcnt[stripe_at(i, q, bits)];
       okeys[o] = k;
       ocounts[o] = c;
       csum += c;
       mkeys[i] = kMidEmpty;
-      for (uint32_t q = 0; q < kMidStripes; ++q) mcnt[i * kMidStripes + q] = 0;
+      for (uint32_t q = 0; q < kMidStripes; ++q) mcnt[stripe_at(i, q, bits)] = 0;
     }
   }
   const uint64_t w = warp_inclusive_add64(csum);
   if (lane == 31 && w) atomicAdd(wsum, static_cast<unsigned long long>(w));
 }
 
-__global__ void __launch_bounds__(256) k_ltab_extract(uint64_t* __restrict__ lkeys, uint32_t* __restrict__ lcnt,
+__global__ void __launch_bounds__(256) k_ltab_extract(uint64_t* __restrict__ lkeys, uint32_t* __restrict__ lcnt, uint32_t bits,
                                                     uint64_t nslots, uint64_t* okeys, uint64_t* okref,
                                                     uint64_t* ocounts, uint64_t cap, unsigned long long* cursor,
                                                     unsigned long long* wsum) {
@@ -806,7 +806,7 @@ __global__ void __launch_bounds__(256) k_ltab_extract(uint64_t* __restrict__ lke
     if (full && o < cap) {
       uint64_t c = 0;
 #pragma unroll
-      for (uint32_t q = 0; q < kMidStripes; ++q) c += lcnt[i * kMidStripes + q];
+      for (uint32_t q = 0; q < kMidStripes; ++q) c += lcnt[stripe_at(i, q, bits)];
       okeys[2 * o] = lo;
       okeys[2 * o + 1] = hi;
       // length = the number of nonzero (word) bytes of the zero-padded key
@@ -816,27 +816,27 @@ __global__ void __launch_bounds__(256) k_ltab_extract(uint64_t* __restrict__ lke
       csum += c;
       lkeys[2 * i] = 0;
       lkeys[2 * i + 1] = 0;
-      for (uint32_t q = 0; q < kMidStripes; ++q) lcnt[i * kMidStripes + q] = 0;
+      for (uint32_t q = 0; q < kMidStripes; ++q) lcnt[stripe_at(i, q, bits)] = 0;
     }
   }
   const uint64_t w = warp_inclusive_add64(csum);
   if (lane == 31 && w) atomicAdd(wsum, static_cast<unsigned long long>(w));
 }
 
-cudaError_t launch_ltab_extract(uint64_t* lkeys, uint32_t* lcnt, uint64_t nslots, uint64_t* okeys, uint64_t* okref,
+cudaError_t launch_ltab_extract(uint64_t* lkeys, uint32_t* lcnt, uint64_t nslots, uint32_t bits, uint64_t* okeys, uint64_t* okref,
                                 uint64_t* ocounts, uint64_t cap, unsigned long long* cursor, unsigned long long* wsum,
                                 int num_sms, cudaStream_t s) {
   k_ltab_extract<<<static_cast<unsigned>(std::min<uint64_t>(8ULL * num_sms, (nslots + 255) / 256)), 256, 0, s>>>(
-      lkeys, lcnt, nslots, okeys, okref, ocounts, cap, cursor, wsum);
+      lkeys, lcnt, bits, nslots, okeys, okref, ocounts, cap, cursor, wsum);
   count_launch();
   return cudaGetLastError();
 }
 
-cudaError_t launch_mtab_extract(uint64_t* mkeys, uint32_t* mcnt, uint64_t nslots, uint64_t* okeys, uint64_t* ocounts,
+cudaError_t launch_mtab_extract(uint64_t* mkeys, uint32_t* mcnt, uint64_t nslots, uint32_t bits, uint64_t* okeys, uint64_t* ocounts,
                                 uint64_t cap, unsigned long long* cursor, unsigned long long* wsum, int num_sms,
                                 cudaStream_t s) {
   k_mtab_extract<<<static_cast<unsigned>(std::min<uint64_t>(8ULL * num_sms, (nslots + 255) / 256)), 256, 0, s>>>(
-      mkeys, mcnt, nslots, okeys, ocounts, cap, cursor, wsum);
+      mkeys, mcnt, bits, nslots, okeys, ocounts, cap, cursor, wsum);
   count_launch();
   return cudaGetLastError();
 }
