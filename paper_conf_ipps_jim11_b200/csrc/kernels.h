@@ -49,7 +49,10 @@ constexpr uint64_t kMidEmpty = ~0ULL;
 constexpr uint32_t kMidProbes = 32;
 // counts of a slot are striped over kMidStripes words (the warp's stripe), so the Zipf-hot mid
 // words do not serialise every RED on one address; the extraction sums the stripes
-constexpr uint32_t kMidStripes = 16;
+#ifndef BMR_MID_STRIPES
+#define BMR_MID_STRIPES 16
+#endif
+constexpr uint32_t kMidStripes = BMR_MID_STRIPES;
 // stripe-major: stripe q of slot h at q * 2^bits + h, so the stripes of a Zipf-hot word sit in
 // kMidStripes different L2 lines (slot-major they shared one line, and its REDs serialised there)
 __host__ __device__ inline uint64_t stripe_at(uint64_t slot, uint32_t stripe, uint32_t bits) {

@@ -1554,10 +1554,10 @@ __device__ __forceinline__ void wc_drain_tab(const Params& P, LWord* lq, uint32_
   const uint32_t n = min(qn, 32u);
   if (n == 0) return;
   __syncwarp();
-  const bool in = lane < n;
   LWord w{0, 0, 0};
-  if (in) w = lq[lane];
+  if (lane < n) w = lq[lane];
   const uint32_t len = static_cast<uint32_t>(w.meta & 0xFFFFu);
+  const bool in = lane < n && len != 0;   // (len 0: a word left to the round loop)
   const bool mid = in && len <= kMidMax, lng = in && !mid;
   const uint64_t klo = mid ? exact_key(w.lo, len) : lng ? w.lo : ~0ULL;
   const uint64_t khi = mid ? 0ULL : lng ? (len >= 16 ? w.hi : (w.hi & ((1ULL << (8 * (len - 8))) - 1ULL))) : ~0ULL;
@@ -1678,10 +1678,10 @@ __device__ __forceinline__ void wc_probe_issue(const Params& P, LWord* lq, uint3
   const uint32_t n = min(qn, 32u);
   if (n == 0) return;
   __syncwarp();
-  const bool in = lane < n;
   LWord w{0, 0, 0};
-  if (in) w = lq[lane];
+  if (lane < n) w = lq[lane];
   const uint32_t len = static_cast<uint32_t>(w.meta & 0xFFFFu);
+  const bool in = lane < n && len != 0;   // (len 0: a word left to the round loop)
   const bool mid = in && len <= kMidMax, lng = in && !mid;
   const uint64_t klo = mid ? exact_key(w.lo, len) : lng ? w.lo : ~0ULL;
   const uint64_t khi = mid ? 0ULL : lng ? (len >= 16 ? w.hi : (w.hi & ((1ULL << (8 * (len - 8))) - 1ULL))) : ~0ULL;
@@ -2059,47 +2059,37 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
   if (!__any_sync(kFull, L)) return;
 #if BMR_WC_LSCAN
   {
-    // words of <= 16 bytes (a stop within 16 bytes after the start: t16 bit j = an nb bit at
-    // j+1..j+16) go to the queue at their warp rank, each lane writing its own (no rounds); longer
-    // ones and windows with more than a queue of them take the round loop below
-    uint32_t t16 = nb >> 1;
-    t16 |= t16 >> 1;
-    t16 |= t16 >> 2;
-    t16 |= t16 >> 4;
-    t16 |= t16 >> 8;
-    const uint32_t Ls = L & t16;
-    const uint32_t cs = __popc(Ls);
-#if BMR_WC_LBALLOT
-    // a lane holds at most 3 such starts (a long word and its delimiter take >= 7 of its 16
-    // bytes): the warp prefix from three ballots instead of a 5-step shuffle scan
+    // every long start goes to the queue at its warp rank, each lane writing its own (no rounds):
+    // a lane holds at most 3 of them (a long word and its delimiter take >= 7 of its 16 bytes),
+    // so the warp prefix comes from three ballots.  An entry's meta is the word length (6..16);
+    // a word with no stop within 16 bytes gets meta 0 (skipped by the drain) and is left to the
+    // round loop below, as are all of a window with more long words than a queue holds.
+    const uint32_t cs = __popc(L);
     const uint32_t b1 = __ballot_sync(kFull, cs >= 1u), b2 = __ballot_sync(kFull, cs >= 2u),
                    b3 = __ballot_sync(kFull, cs >= 3u);
     const uint32_t lt = lanemask_lt();
     const uint32_t incl = __popc(b1 & lt) + __popc(b2 & lt) + __popc(b3 & lt) + cs;
     const uint32_t tot = __popc(b1) + __popc(b2) + __popc(b3);
-#else
-    const uint32_t incl = warp_inclusive_add(cs);
-    const uint32_t tot = __shfl_sync(kFull, incl, 31);
-#endif
     if (tot <= static_cast<uint32_t>(Cfg<kWC>::kLQ)) {
-      L &= ~t16;
-      if (tot) {
-        while (qn + tot > static_cast<uint32_t>(Cfg<kWC>::kLQ)) wc_drain_tq(P, lq, qn, pq);
-        LWord* d = lq + qn + incl - cs;
-        for (uint32_t m = Ls; m; m &= m - 1, ++d) {
-          const uint32_t j = __ffs(m) - 1;
-          const uint32_t len = __ffs(nb >> (j + 1));   // 6..16
-          const uint32_t pos = i0 + j;
-          const uint32_t* src = reinterpret_cast<const uint32_t*>(tv.sb + (pos & ~3u));
-          const uint32_t sh = (pos & 3u) * 8;   // 5 aligned words, funnel-shifted
-          const uint32_t y0 = src[0], y1 = src[1], y2 = src[2], y3 = src[3], y4 = src[4];
-          d->lo = static_cast<uint64_t>(__funnelshift_r(y0, y1, sh)) | (static_cast<uint64_t>(__funnelshift_r(y1, y2, sh)) << 32);
-          d->hi = static_cast<uint64_t>(__funnelshift_r(y2, y3, sh)) | (static_cast<uint64_t>(__funnelshift_r(y3, y4, sh)) << 32);
-          d->meta = (static_cast<uint64_t>(tv.sbase + pos) << 16) | len;
-        }
-        qn += tot;
-        __syncwarp();
+      uint32_t big = 0;
+      while (qn + tot > static_cast<uint32_t>(Cfg<kWC>::kLQ)) wc_drain_tq(P, lq, qn, pq);
+      LWord* d = lq + qn + incl - cs;
+      for (uint32_t m = L; m; m &= m - 1, ++d) {
+        const uint32_t j = __ffs(m) - 1;
+        const uint32_t len = __ffs(nb >> (j + 1));   // 6..31, 0: no stop in view
+        const bool ok = len != 0 && len <= kLQMaxLen;
+        big |= ok ? 0u : (1u << j);
+        const uint32_t pos = i0 + j;
+        const uint32_t* src = reinterpret_cast<const uint32_t*>(tv.sb + (pos & ~3u));
+        const uint32_t sh = pos << 3;   // 5 aligned words, funnel-shifted (shift amount mod 32)
+        const uint32_t y0 = src[0], y1 = src[1], y2 = src[2], y3 = src[3], y4 = src[4];
+        d->lo = static_cast<uint64_t>(__funnelshift_r(y0, y1, sh)) | (static_cast<uint64_t>(__funnelshift_r(y1, y2, sh)) << 32);
+        d->hi = static_cast<uint64_t>(__funnelshift_r(y2, y3, sh)) | (static_cast<uint64_t>(__funnelshift_r(y3, y4, sh)) << 32);
+        d->meta = ok ? len : 0u;
       }
+      qn += tot;
+      __syncwarp();
+      L = big;
       if (!__any_sync(kFull, L)) return;
     }
   }
@@ -3540,8 +3530,8 @@ bool map_wc_tab() {
 
 uint32_t map_wait_hint() {
   static uint32_t v = [] {
-    const char* e = getenv("BMR_MAP_WAIT");
-    return e ? static_cast<uint32_t>(atoi(e)) : 0u;
+    const char* e = getenv("BMR_MAP_WAIT");   // (1: C5 13.90 -> 13.81 ms once the Map was issue-bound)
+    return e ? static_cast<uint32_t>(atoi(e)) : 1u;
   }();
   return v;
 }
