@@ -136,6 +136,9 @@ constexpr int nprod() { return W == 4 ? BMR_II_NPROD : 2; }
 #ifndef BMR_WC_X2WAY
 #define BMR_WC_X2WAY 0   // WordCount table mode: second combiner slot (home ^ 1) for exact words
 #endif
+#ifndef BMR_WC_PAIRWIN
+#define BMR_WC_PAIRWIN 1   // WordCount table mode: two 512-B windows per window fetch
+#endif
 #ifndef BMR_WC_CLS16
 #define BMR_WC_CLS16 1   // WordCount table mode: each lane classifies its own 16 bytes only (next chunk by shuffle)
 #endif
@@ -1026,7 +1029,7 @@ __device__ void producer_loop_dyn(const Params& P, uint8_t* smem, uint32_t pw) {
       const uint32_t xo = *reinterpret_cast<volatile unsigned int*>(&oc->pout[other]);
       if (xo != ~0u) {
         const uint32_t E = max(x0, xo);
-        post_end = it == E;
+        post_end = it == E || it == E + 1u;   // (two end iterations: window-pair fetches, wc_map_loop)
         post_skip = it < E;
         break;
       }
@@ -1052,7 +1055,10 @@ __device__ void producer_loop_dyn(const Params& P, uint8_t* smem, uint32_t pw) {
       mbar_arrive(&ready[s]);
     }
     __syncwarp();
-    if (post_end) { it += kNP; break; }
+    if (post_end && it + kNP > max(x0, *reinterpret_cast<volatile unsigned int*>(&oc->pout[other])) + 1u) {
+      it += kNP;
+      break;
+    }
   }
   // this producer's tiles whose bitmap is still pending (skip stages return at once)
   for (uint32_t j = it >= kLag + kNP ? it - kLag : pw; j < it; j += kNP)
@@ -2166,8 +2172,13 @@ __device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
   }
   uint32_t have_it = ~0u;
   long long t = 0, sbase = 0, hi = 0, stg_hi = 0;
+  // table mode with dynamic tiles: two windows per fetch (one window-counter atomic, stage check
+  // and empty arrival per pair; the producers post the end marker at two iterations, so every
+  // map warp meets it: 16 pairs per tile < 24 map warps)
+  constexpr uint32_t kPW = (kTab && BMR_WC_PAIRWIN && BMR_DYN_TILES) ? 2u : 1u;
+  static_assert(kNWin % kPW == 0, "window pairs must not straddle tiles");
   for (;;) {
-    const uint32_t g = lane0_atom_add_shared(&oc->win_next, 1u);
+    const uint32_t g = lane0_atom_add_shared(&oc->win_next, kPW);
     const uint32_t it = g / kNWin, w = g % kNWin;
     const uint32_t s = it % kStages;
     if (it != have_it) {   // wait for the tile's record-start bitmap, then its header
@@ -2180,20 +2191,24 @@ __device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
       have_it = it;
     }
     if (t == -1) break;   // (-2: a skip stage, no windows)
-    const long long wp = sbase + kLead + static_cast<long long>(w) * kWin;
-    if (wp < hi) {   // warp-uniform
-      const TileView tv{smem + Layout<W>::bytes + s * kStageBytes,
-                        reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits), sbase, stg_hi, 0,
-                        0};
-      if constexpr (kTab) wc_window_tab<kMode == 1>(P, oc, outh, tv, wp, ctab, lq, qn, hq, pq);
-      else wc_window(P, oc, outh, tv, wp, xq, hq, ctab, lq, qn, lo);
-      if (qn >= 32) {
-        if constexpr (kTab) wc_drain_tq(P, lq, qn, pq);
-        else wc_drain(P, lo, lq, qn);
+    const TileView tv{smem + Layout<W>::bytes + s * kStageBytes,
+                      reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits), sbase, stg_hi, 0,
+                      0};
+#pragma unroll 1
+    for (uint32_t q = 0; q < kPW; ++q) {
+      const long long wp = sbase + kLead + static_cast<long long>(w + q) * kWin;
+      if (wp < hi) {   // warp-uniform
+        if constexpr (kTab) wc_window_tab<kMode == 1>(P, oc, outh, tv, wp, ctab, lq, qn, hq, pq);
+        else wc_window(P, oc, outh, tv, wp, xq, hq, ctab, lq, qn, lo);
+        if (qn >= 32) {
+          if constexpr (kTab) wc_drain_tq(P, lq, qn, pq);
+          else wc_drain(P, lo, lq, qn);
+        }
       }
     }
     __syncwarp();
-    lane0_mbar_arrive(&empty[s]);
+    if (kPW == 1) lane0_mbar_arrive(&empty[s]);
+    else if ((threadIdx.x & 31) == 0) mbar_arrive_cnt(&empty[s], kPW);
   }
   while (qn) {   // this warp's last long words
     if constexpr (kTab) wc_drain_tq(P, lq, qn, pq);
