@@ -1994,8 +1994,10 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
       uint32_t ka1 = kb32 + 4u * ((k1 * 0x9E3779B1u) >> (32 - kCombBits));
       uint32_t ka2 = kb32 + 4u * ((k2 * 0x9E3779B1u) >> (32 - kCombBits));
       uint32_t v1 = lds_volatile_u32(ka1), v2 = lds_volatile_u32(ka2);
-      if (v1 == kCombEmpty32) v1 = atom_cas_shared_u32(ka1, kCombEmpty32, k1);
-      if (two && v2 == kCombEmpty32) v2 = atom_cas_shared_u32(ka2, kCombEmpty32, k2);   // (CAS: the real slot)
+      if (v1 == kCombEmpty32 || v2 == kCombEmpty32) {   // (claims: only until the table has filled)
+        if (v1 == kCombEmpty32) v1 = atom_cas_shared_u32(ka1, kCombEmpty32, k1);
+        if (two && v2 == kCombEmpty32) v2 = atom_cas_shared_u32(ka2, kCombEmpty32, k2);   // (CAS: the real slot)
+      }
       bool h1 = v1 == k1 || v1 == kCombEmpty32;
       bool h2 = two && (v2 == k2 || v2 == kCombEmpty32);
 #if BMR_WC_X2WAY
@@ -2016,8 +2018,10 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
         ka2 = h2 ? kb : ka2;
       }
 #endif
-      red_shared_add_u32(h1 ? ka1 + 4u * Cfg<kWC>::kCombSlots : dmy, 1u);
-      red_shared_add_u32(h2 ? ka2 + 4u * Cfg<kWC>::kCombSlots : dmy, 1u);
+      // the slot's count gets 1 on a hit, 0 on a miss (a no-op on another key's count): no
+      // predicated atomic, no dummy address
+      red_shared_add_u32(ka1 + 4u * Cfg<kWC>::kCombSlots, h1 ? 1u : 0u);
+      red_shared_add_u32(ka2 + 4u * Cfg<kWC>::kCombSlots, h2 ? 1u : 0u);
 #if !(defined(BMR_DIAG) && BMR_DIAG == 10)
       if (!h1) red_add_u32(P.xtab + k1, 1u);
       if (two && !h2) red_add_u32(P.xtab + k2, 1u);
