@@ -993,13 +993,15 @@ __device__ void producer_loop_dyn(const Params& P, uint8_t* smem, uint32_t pw) {
   uint64_t* ready = reinterpret_cast<uint64_t*>(smem + Layout<W>::ready);
   OutCtl* oc = reinterpret_cast<OutCtl*>(smem + Layout<W>::ctl);
   const uint64_t ntiles = bd_ntiles();
+  // small batches take single tiles (chunks would leave most SMs without a tile: C1, 64 tiles)
+  const uint32_t chunk = ntiles >= 16ULL * kChunk * gridDim.x ? kChunk : 1u;
   uint32_t it = pw;
   for (;;) {   // chunks of tiles
     unsigned long long base = 0;
-    if (lane == 0) base = atomicAdd(P.tile_next, static_cast<unsigned long long>(kChunk));
+    if (lane == 0) base = atomicAdd(P.tile_next, static_cast<unsigned long long>(chunk));
     base = __shfl_sync(kFull, base, 0);
     if (base >= ntiles) break;
-    const uint32_t cnt = static_cast<uint32_t>(min(static_cast<unsigned long long>(kChunk), ntiles - base));
+    const uint32_t cnt = static_cast<uint32_t>(min(static_cast<unsigned long long>(chunk), ntiles - base));
     uint64_t my_ra = 0, my_rb = 0;
     if (lane < cnt) {
       my_ra = P.tb[2 * (base + lane)];
