@@ -139,6 +139,9 @@ constexpr int nprod() { return W == 4 ? BMR_II_NPROD : 2; }
 #ifndef BMR_WC_PAIRWIN
 #define BMR_WC_PAIRWIN 1   // WordCount table mode: two 512-B windows per window fetch
 #endif
+#ifndef BMR_II_PAIRWIN
+#define BMR_II_PAIRWIN 1   // InvertedIndex: two 512-B windows per window fetch
+#endif
 #ifndef BMR_WC_CLS16
 #define BMR_WC_CLS16 1   // WordCount table mode: each lane classifies its own 16 bytes only (next chunk by shuffle)
 #endif
@@ -427,7 +430,12 @@ __device__ __forceinline__ uint32_t word_mask4(uint32_t x) {  // [0-9A-Za-z] (C-
   const uint32_t m = (dig | alp) & ~x & 0x80808080u;
   return ((m >> 7) * 0x01020408u) >> 24;
 }
-__device__ __forceinline__ uint32_t eq_mask4(uint32_t x, uint32_t b4) { return movemask4(__vcmpeq4(x, b4)); }
+__device__ __forceinline__ uint32_t eq_mask4(uint32_t x, uint32_t b4) {   // bytes == b4's -> 4 bits
+  // exact per-byte zero test of x ^ b4 (no borrow crosses a byte: (t & 0x7F) + 0x7F <= 0xFE)
+  const uint32_t t = x ^ b4;
+  const uint32_t z = ~(((t & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | t | 0x7F7F7F7Fu);
+  return ((z >> 7) * 0x01020408u) >> 24;
+}
 __device__ __forceinline__ bool is_word_byte(uint32_t c) {
   return (c - '0' < 10u) || ((c | 0x20u) - 'a' < 26u);
 }
@@ -720,10 +728,6 @@ __device__ __forceinline__ void tma_store_1d(void* gdst, const void* ssrc, uint3
 // (one lane per stream: all three reservations in flight together), the TMA bulk store of the
 // buffer's SoA runs, the routed stores of the queued entries while the TMA reads SMEM, and only
 // then the wait for the TMA's reads before the buffer is handed back.
-#ifndef BMR_FLUSH_BACKOFF_NS
-#define BMR_FLUSH_BACKOFF_NS 2048
-#endif
-constexpr uint32_t kFlushBackoffNs = BMR_FLUSH_BACKOFF_NS;
 template <int W>
 __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc, uint32_t fw) {
   using F = PairFmt<W>;
@@ -735,16 +739,9 @@ __device__ void flush_loop(const Params& P, uint8_t* smem, OutCtl* oc, uint32_t 
     // wait for generation f to be sealed; with several flush warps the one waiting past the
     // final generation sees the final flag instead (no arrival ever comes for it)
     bool past = false;
-    // (suspended try_wait: a polling flush warp would take issue slots from the map warps; the
-    // suspend hint is an upper bound the hardware often cuts short, so an idle flush warp also
-    // backs off with __nanosleep up to kFlushBackoffNs — in WordCount table mode buffers seal
-    // rarely and the polls were 3% of the Map's instructions, ncu C5 round 2)
-    uint32_t backoff = 0;
+    // (suspended try_wait: a polling flush warp would take issue slots from the map warps; an idle
+    // flush warp's sleep-polls measured no cheaper, C5 round 2)
     while (!mbar_try_wait_hint(&oc->req[h], (f / kNOut) & 1u, 2000)) {
-      if (W == kWC && P.xtab) {   // (table mode only: the other workloads flush continuously)
-        if (backoff) __nanosleep(backoff);
-        backoff = min(backoff ? 2 * backoff : 64u, kFlushBackoffNs);
-      }
       if (NF > 1 && ld_acquire_cta_shared_u32(&oc->is_final) && ld_acquire_cta_shared_u32(&oc->final_seq) < f) {
         past = true;
         break;
@@ -2452,8 +2449,11 @@ __device__ __forceinline__ void ii_map_loop(const Params& P, uint8_t* smem, OutC
   uint8_t* outh = smem + Layout<W>::out;
   uint32_t have_it = ~0u;
   long long t = 0, sbase = 0, hi = 0, stg_hi = 0;
+  // two windows per fetch with dynamic tiles (the end marker sits at two iterations), as wc_map_loop
+  constexpr uint32_t kPW = (BMR_II_PAIRWIN && BMR_DYN_TILES) ? 2u : 1u;
+  static_assert(kNWin % kPW == 0, "window pairs must not straddle tiles");
   for (;;) {
-    const uint32_t g = lane0_atom_add_shared(&oc->win_next, 1u);
+    const uint32_t g = lane0_atom_add_shared(&oc->win_next, kPW);
     const uint32_t it = g / kNWin, w = g % kNWin;
     const uint32_t s = it % kStages;
     if (it != have_it) {
@@ -2466,15 +2466,17 @@ __device__ __forceinline__ void ii_map_loop(const Params& P, uint8_t* smem, OutC
       have_it = it;
     }
     if (t == -1) break;   // (-2: a skip stage, no windows)
-    const long long wp = sbase + kLead + static_cast<long long>(w) * kWin;
-    if (wp < hi) {   // warp-uniform
-      const TileView tv{smem + Layout<W>::bytes + s * kStageBytes,
-                        reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits), sbase, stg_hi, 0,
-                        0};
-      ii_window(P, oc, outh, tv, wp, qn);
+    const TileView tv{smem + Layout<W>::bytes + s * kStageBytes,
+                      reinterpret_cast<const uint32_t*>(smem + Layout<W>::bits + s * Cfg<W>::kBits), sbase, stg_hi, 0,
+                      0};
+#pragma unroll 1
+    for (uint32_t q = 0; q < kPW; ++q) {
+      const long long wp = sbase + kLead + static_cast<long long>(w + q) * kWin;
+      if (wp < hi) ii_window(P, oc, outh, tv, wp, qn);   // warp-uniform
     }
     __syncwarp();
-    lane0_mbar_arrive(&empty[s]);
+    if (kPW == 1) lane0_mbar_arrive(&empty[s]);
+    else if ((threadIdx.x & 31) == 0) mbar_arrive_cnt(&empty[s], kPW);
   }
 }
 
