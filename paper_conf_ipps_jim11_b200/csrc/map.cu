@@ -1641,9 +1641,7 @@ __device__ __forceinline__ void wc_probe_resolve(const Params& P, const PendQ& p
         unsigned long long k = pr ? *reinterpret_cast<volatile unsigned long long*>(P.mkeys + h) : vlo;
         if (k == kMidEmpty) k = atomicCAS(reinterpret_cast<unsigned long long*>(P.mkeys + h), kMidEmpty, e.klo);
         if (k == e.klo || k == kMidEmpty) {
-#if !(defined(BMR_DIAG) && BMR_DIAG == 8)
           red_add_u32(P.mcnt + stripe_at(h, stripe, P.mbits), cnt);
-#endif
           todo = false;
           break;
         }
@@ -1661,9 +1659,7 @@ __device__ __forceinline__ void wc_probe_resolve(const Params& P, const PendQ& p
           if (olo == 0) { olo = e.klo; ohi = e.khi; }
         }
         if (olo == e.klo && ohi == e.khi) {
-#if !(defined(BMR_DIAG) && BMR_DIAG == 8)
           red_add_u32(P.lcnt + stripe_at(h, stripe, P.lbits), cnt);
-#endif
           todo = false;
           break;
         }
@@ -1690,11 +1686,7 @@ __device__ __forceinline__ void wc_probe_issue(const Params& P, LWord* lq, uint3
   const bool mid = in && len <= kMidMax, lng = in && !mid;
   const uint64_t klo = mid ? exact_key(w.lo, len) : lng ? w.lo : ~0ULL;
   const uint64_t khi = mid ? 0ULL : lng ? (len >= 16 ? w.hi : (w.hi & ((1ULL << (8 * (len - 8))) - 1ULL))) : ~0ULL;
-#if defined(BMR_DIAG) && BMR_DIAG == 6
-  const uint32_t grp = 1u << lane;   // (timing diagnostic: no aggregation)
-#else
   const uint32_t grp = __match_any_sync(kFull, klo) & __match_any_sync(kFull, khi);
-#endif
   const bool lead = in && lane == static_cast<uint32_t>(__ffs(grp) - 1);
   if (lead) {
     const uint64_t h = mid ? mid_slot(klo, P.mbits) : long_slot(klo, khi, P.lbits);
@@ -1707,9 +1699,6 @@ __device__ __forceinline__ void wc_probe_issue(const Params& P, LWord* lq, uint3
     pq.meta[lane] = (1u << 31) | (mid ? (1u << 30) : 0u) | static_cast<uint32_t>(__popc(grp));
   }
   cp_async_commit();
-#if defined(BMR_DIAG) && BMR_DIAG == 9
-  pq.meta[lane] = 0;   // (timing diagnostic: keys and groups computed, never probed)
-#endif
   const uint32_t rest = qn - n;
   LWord r{0, 0, 0};
   if (lane < rest) r = lq[n + lane];
@@ -1720,10 +1709,6 @@ __device__ __forceinline__ void wc_probe_issue(const Params& P, LWord* lq, uint3
 }
 // drain of the table mode: synchronous (wc_drain_tab) or resolve-previous + issue
 __device__ __forceinline__ void wc_drain_tq(const Params& P, LWord* lq, uint32_t& qn, const PendQ& pq) {
-#if defined(BMR_DIAG) && BMR_DIAG == 5
-  qn = 0;   // (timing diagnostic: long words queued, never counted)
-  return;
-#endif
 #if BMR_WC_ADRAIN
   wc_probe_resolve(P, pq);
   wc_probe_issue(P, lq, qn, pq);
@@ -1967,19 +1952,6 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
       const uint32_t w0 = lds_u32(a), w1 = lds_u32(a + 4u);
       return exact_key30_w(__funnelshift_r(w0, w1, j << 3), __funnelshift_r(w1, w1, j << 3), len);
     };
-#if defined(BMR_DIAG) && BMR_DIAG == 3
-    if (S) return;   // (timing diagnostic: no exact words, no long words)
-#endif
-#if defined(BMR_DIAG) && (BMR_DIAG == 1 || BMR_DIAG == 4)
-    if (BMR_DIAG == 4) {   // (timing diagnostic: exact words straight to the L2 table)
-      for (uint32_t E = S & near; E;) {
-        const uint32_t j = bfind_u32(E);
-        E &= ~(1u << j);
-        red_add_u32(P.xtab + xkey(j), 1u);
-      }
-    }
-    if (false)
-#endif
 #if BMR_WC_XPAIR
     // two words per iteration (the highest and the lowest start left): the same instructions per
     // word, two independent dependency chains (the loop is latency-bound), half the iterations
@@ -2021,10 +1993,8 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
       // predicated atomic, no dummy address
       red_shared_add_u32(ka1 + 4u * Cfg<kWC>::kCombSlots, h1 ? 1u : 0u);
       red_shared_add_u32(ka2 + 4u * Cfg<kWC>::kCombSlots, h2 ? 1u : 0u);
-#if !(defined(BMR_DIAG) && BMR_DIAG == 10)
       if (!h1) red_add_u32(P.xtab + k1, 1u);
       if (two && !h2) red_add_u32(P.xtab + k2, 1u);
-#endif
     }
 #else
     for (uint32_t E = S & near; E;) {
@@ -2062,9 +2032,6 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
   // longer words: only the lane's highest start can lack a visible end (no stop in the 31 - j
   // bytes after it)
   uint32_t L = S & ~near;
-#if defined(BMR_DIAG) && BMR_DIAG == 2
-  L = 0;
-#endif
   if (!__any_sync(kFull, L)) return;
 #if BMR_WC_LSCAN
   {
