@@ -20,6 +20,9 @@
 
 #include "common.cuh"
 
+#ifndef BMR_XTAB_BPS
+#define BMR_XTAB_BPS 256   // table extraction: blocks per SM (C5: 8 -> 1.21 ms, 64 -> 0.98, 512 -> 0.94; short-lived blocks keep more loads in flight)
+#endif
 #ifndef BMR_XTAB_UNROLL
 #define BMR_XTAB_UNROLL 1   // (2 and 4 in-flight loads per thread measured no better: 1.0 vs 1.0 / 1.34 ms)
 #endif
@@ -748,7 +751,7 @@ cudaError_t launch_xtab_extract(uint32_t* tab, uint64_t nent, uint64_t* out, uin
 cudaError_t launch_xtab_extract_list(uint32_t* tab, uint64_t nent, uint32_t* okeys, uint64_t* ocounts, uint64_t cap,
                                      unsigned long long* cursor, unsigned long long* wsum, int num_sms, cudaStream_t s) {
   const uint64_t nv4 = nent / 4;
-  k_xtab_extract<true><<<static_cast<unsigned>(std::min<uint64_t>(8ULL * num_sms, (nv4 + 256 * BMR_XTAB_UNROLL - 1) / (256 * BMR_XTAB_UNROLL))), 256, 0, s>>>(
+  k_xtab_extract<true><<<static_cast<unsigned>(std::min<uint64_t>(static_cast<uint64_t>(BMR_XTAB_BPS) * num_sms, (nv4 + 256 * BMR_XTAB_UNROLL - 1) / (256 * BMR_XTAB_UNROLL))), 256, 0, s>>>(
       tab, nv4, nullptr, okeys, ocounts, cap, cursor, wsum);
   count_launch();
   return cudaGetLastError();
