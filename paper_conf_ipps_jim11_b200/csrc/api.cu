@@ -360,7 +360,7 @@ struct mr_job {
   // long words (9..16 symbols): open-addressing table of their 16 zero-padded key bytes + counts
   DBuf<uint64_t> ltab_keys;
   DBuf<uint32_t> ltab_cnt;
-  uint32_t lbits = 18;
+  uint32_t lbits = 19;   // (table mode: also the words of 6..8 symbols, BMR_WC_UNITAB)
   DBuf<uint64_t> lkeys_out, lkref_out, lcounts;
   uint64_t nseg_l = 0;            // long-table keys of this group (the output's last list)
   // KM: the Map accumulates the cluster sums itself (k <= 64; not for ingested partials)

@@ -61,6 +61,9 @@ __host__ __device__ inline uint64_t stripe_at(uint64_t slot, uint32_t stripe, ui
 __host__ __device__ inline uint64_t mid_slot(uint64_t key, uint32_t bits) {
   return (key * 0x9E3779B97F4A7C15ULL) >> (64 - bits);
 }
+// long-table key of a word of <= 8 bytes: the zero-padded bytes in lo, this marker in hi (byte 15
+// = 0x80, never a word byte; nonzero, so a slot whose hi reads 0 is still a torn view)
+constexpr uint64_t kShortHi = 0x8000000000000000ULL;
 __host__ __device__ inline uint64_t long_slot(uint64_t lo, uint64_t hi, uint32_t bits) {
   return ((lo * 0x9E3779B97F4A7C15ULL) ^ (hi * 0xC2B2AE3D27D4EB4FULL) ^ (lo >> 29)) * 0x94D049BB133111EBULL >> (64 - bits);
 }

@@ -142,6 +142,9 @@ constexpr int nprod() { return W == 4 ? BMR_II_NPROD : 2; }
 #ifndef BMR_II_PAIRWIN
 #define BMR_II_PAIRWIN 1   // InvertedIndex: two 512-B windows per window fetch
 #endif
+#ifndef BMR_WC_UNITAB
+#define BMR_WC_UNITAB 1   // WordCount table mode: words of 6..16 symbols in one 16-byte-key table
+#endif
 #ifndef BMR_WC_CLS16
 #define BMR_WC_CLS16 1   // WordCount table mode: each lane classifies its own 16 bytes only (next chunk by shuffle)
 #endif
@@ -1563,9 +1566,14 @@ __device__ __forceinline__ void wc_drain_tab(const Params& P, LWord* lq, uint32_
   if (lane < n) w = lq[lane];
   const uint32_t len = static_cast<uint32_t>(w.meta & 0xFFFFu);
   const bool in = lane < n && len != 0;   // (len 0: a word left to the round loop)
-  const bool mid = in && len <= kMidMax, lng = in && !mid;
-  const uint64_t klo = mid ? exact_key(w.lo, len) : lng ? w.lo : ~0ULL;
-  const uint64_t khi = mid ? 0ULL : lng ? (len >= 16 ? w.hi : (w.hi & ((1ULL << (8 * (len - 8))) - 1ULL))) : ~0ULL;
+  // with the exact-key table (kMode 1) the words of 6..8 symbols share the long table: key = the
+  // zero-padded bytes, hi = kShortHi (no 48-bit key, no mid / long divergence in the drains)
+  const bool uni = BMR_WC_UNITAB && P.xtab != nullptr;
+  const bool mid = in && !uni && len <= kMidMax, lng = in && !mid;
+  const uint64_t klo = mid ? exact_key(w.lo, len) : lng ? (len >= 8 ? w.lo : (w.lo & ((1ULL << (8 * len)) - 1ULL))) : ~0ULL;
+  const uint64_t khi = mid ? 0ULL
+                       : lng ? (len >= 16 ? w.hi : len > 8 ? (w.hi & ((1ULL << (8 * (len - 8))) - 1ULL)) : kShortHi)
+                             : ~0ULL;
   const uint32_t grp = __match_any_sync(kFull, klo) & __match_any_sync(kFull, khi);
   bool todo = in && lane == static_cast<uint32_t>(__ffs(grp) - 1);
   const uint32_t stripe = (blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1);
@@ -1683,9 +1691,14 @@ __device__ __forceinline__ void wc_probe_issue(const Params& P, LWord* lq, uint3
   if (lane < n) w = lq[lane];
   const uint32_t len = static_cast<uint32_t>(w.meta & 0xFFFFu);
   const bool in = lane < n && len != 0;   // (len 0: a word left to the round loop)
-  const bool mid = in && len <= kMidMax, lng = in && !mid;
-  const uint64_t klo = mid ? exact_key(w.lo, len) : lng ? w.lo : ~0ULL;
-  const uint64_t khi = mid ? 0ULL : lng ? (len >= 16 ? w.hi : (w.hi & ((1ULL << (8 * (len - 8))) - 1ULL))) : ~0ULL;
+  // with the exact-key table (kMode 1) the words of 6..8 symbols share the long table: key = the
+  // zero-padded bytes, hi = kShortHi (no 48-bit key, no mid / long divergence in the drains)
+  const bool uni = BMR_WC_UNITAB && P.xtab != nullptr;
+  const bool mid = in && !uni && len <= kMidMax, lng = in && !mid;
+  const uint64_t klo = mid ? exact_key(w.lo, len) : lng ? (len >= 8 ? w.lo : (w.lo & ((1ULL << (8 * len)) - 1ULL))) : ~0ULL;
+  const uint64_t khi = mid ? 0ULL
+                       : lng ? (len >= 16 ? w.hi : len > 8 ? (w.hi & ((1ULL << (8 * (len - 8))) - 1ULL)) : kShortHi)
+                             : ~0ULL;
   const uint32_t grp = __match_any_sync(kFull, klo) & __match_any_sync(kFull, khi);
   const bool lead = in && lane == static_cast<uint32_t>(__ffs(grp) - 1);
   if (lead) {

@@ -813,7 +813,9 @@ __global__ void __launch_bounds__(256) k_ltab_extract(uint64_t* __restrict__ lke
       okeys[2 * o] = lo;
       okeys[2 * o + 1] = hi;
       // length = the number of nonzero (word) bytes of the zero-padded key
-      const uint32_t len = 8u + (hi ? (64u - static_cast<uint32_t>(__clzll(static_cast<long long>(hi))) + 7u) / 8u : 0u);
+      // (hi == kShortHi: a word of <= 8 bytes, its length from lo)
+      const uint32_t len = hi == kShortHi ? (64u - static_cast<uint32_t>(__clzll(static_cast<long long>(lo))) + 7u) / 8u
+                           : 8u + (hi ? (64u - static_cast<uint32_t>(__clzll(static_cast<long long>(hi))) + 7u) / 8u : 0u);
       okref[o] = (reinterpret_cast<uint64_t>(okeys + 2 * o) << 16) | len;
       ocounts[o] = c;
       csum += c;
