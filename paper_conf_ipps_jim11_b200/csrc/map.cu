@@ -1557,6 +1557,7 @@ __device__ __forceinline__ void wc_drain(const Params& P, LOut& lo, LWord* lq, u
 // never collide (a long word's first 8 bytes are all non-zero: klo >= 2^56 > any 48-bit key) —
 // and each group leader issues its table load (8-B mid slot or 16-B long slot) in the same
 // round, so the two L2 round trips overlap.  No hash is computed (the tables are exact).
+template <bool kUni>
 __device__ __forceinline__ void wc_drain_tab(const Params& P, LWord* lq, uint32_t& qn) {
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t n = min(qn, 32u);
@@ -1568,7 +1569,7 @@ __device__ __forceinline__ void wc_drain_tab(const Params& P, LWord* lq, uint32_
   const bool in = lane < n && len != 0;   // (len 0: a word left to the round loop)
   // with the exact-key table (kMode 1) the words of 6..8 symbols share the long table: key = the
   // zero-padded bytes, hi = kShortHi (no 48-bit key, no mid / long divergence in the drains)
-  const bool uni = BMR_WC_UNITAB && P.xtab != nullptr;
+  constexpr bool uni = kUni;
   const bool mid = in && !uni && len <= kMidMax, lng = in && !mid;
   const uint64_t klo = mid ? exact_key(w.lo, len) : lng ? (len >= 8 ? w.lo : (w.lo & ((1ULL << (8 * len)) - 1ULL))) : ~0ULL;
   const uint64_t khi = mid ? 0ULL
@@ -1631,13 +1632,14 @@ struct PendQ {
   uint32_t* meta;   // per lane: bit 31 pending, bit 30 mid, bits 0..5 group size
   uint32_t* slot;   // per lane: first probe slot
 };
+template <bool kUni>
 __device__ __forceinline__ void wc_probe_resolve(const Params& P, const PendQ& pq) {
   const uint32_t lane = threadIdx.x & 31;
   cp_async_wait_all();
   const uint32_t meta = pq.meta[lane];
   if (meta >> 31) {
     const PEnt e = pq.e[lane];
-    const bool mid = (meta >> 30) & 1u;
+    const bool mid = !kUni && ((meta >> 30) & 1u);
     const uint32_t cnt = meta & 63u;
     const uint32_t stripe = (blockIdx.x * 7u + (threadIdx.x >> 5)) & (kMidStripes - 1);
     uint64_t h = pq.slot[lane];
@@ -1682,6 +1684,7 @@ __device__ __forceinline__ void wc_probe_resolve(const Params& P, const PendQ& p
   }
   __syncwarp();
 }
+template <bool kUni>
 __device__ __forceinline__ void wc_probe_issue(const Params& P, LWord* lq, uint32_t& qn, const PendQ& pq) {
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t n = min(qn, 32u);
@@ -1721,12 +1724,14 @@ __device__ __forceinline__ void wc_probe_issue(const Params& P, LWord* lq, uint3
   qn = rest;
 }
 // drain of the table mode: synchronous (wc_drain_tab) or resolve-previous + issue
+// kUni: the exact-key table mode (kMode 1) with the unified 6..16-symbol table, decided at compile time
+template <bool kUni>
 __device__ __forceinline__ void wc_drain_tq(const Params& P, LWord* lq, uint32_t& qn, const PendQ& pq) {
 #if BMR_WC_ADRAIN
-  wc_probe_resolve(P, pq);
-  wc_probe_issue(P, lq, qn, pq);
+  wc_probe_resolve<kUni>(P, pq);
+  wc_probe_issue<kUni>(P, lq, qn, pq);
 #else
-  wc_drain_tab(P, lq, qn);
+  wc_drain_tab<kUni>(P, lq, qn);
 #endif
 }
 
@@ -2061,7 +2066,7 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
     const uint32_t tot = __popc(b1) + __popc(b2) + __popc(b3);
     if (tot <= static_cast<uint32_t>(Cfg<kWC>::kLQ)) {
       uint32_t big = 0;
-      while (qn + tot > static_cast<uint32_t>(Cfg<kWC>::kLQ)) wc_drain_tq(P, lq, qn, pq);
+      while (qn + tot > static_cast<uint32_t>(Cfg<kWC>::kLQ)) wc_drain_tq<kX && BMR_WC_UNITAB>(P, lq, qn, pq);
       LWord* d = lq + qn + incl - cs;
       for (uint32_t m = L; m; m &= m - 1, ++d) {
         const uint32_t j = __ffs(m) - 1;
@@ -2091,7 +2096,7 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
   for (;;) {   // one long word per lane per round, appended to the warp's queue
     const uint32_t m = __ballot_sync(kFull, L != 0);
     if (!m) break;
-    if (qn + __popc(m) > static_cast<uint32_t>(Cfg<kWC>::kLQ)) wc_drain_tq(P, lq, qn, pq);
+    if (qn + __popc(m) > static_cast<uint32_t>(Cfg<kWC>::kLQ)) wc_drain_tq<kX && BMR_WC_UNITAB>(P, lq, qn, pq);
     uint32_t j = 0, len = 0;
     if (L) {
       j = __ffs(L) - 1;
@@ -2184,7 +2189,7 @@ __device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
         if constexpr (kTab) wc_window_tab<kMode == 1>(P, oc, outh, tv, wp, ctab, lq, qn, hq, pq);
         else wc_window(P, oc, outh, tv, wp, xq, hq, ctab, lq, qn, lo);
         if (qn >= 32) {
-          if constexpr (kTab) wc_drain_tq(P, lq, qn, pq);
+          if constexpr (kTab) wc_drain_tq<kMode == 1 && BMR_WC_UNITAB>(P, lq, qn, pq);
           else wc_drain(P, lo, lq, qn);
         }
       }
@@ -2194,11 +2199,11 @@ __device__ void wc_map_loop(const Params& P, uint8_t* smem, OutCtl* oc) {
     else if ((threadIdx.x & 31) == 0) mbar_arrive_cnt(&empty[s], kPW);
   }
   while (qn) {   // this warp's last long words
-    if constexpr (kTab) wc_drain_tq(P, lq, qn, pq);
+    if constexpr (kTab) wc_drain_tq<kMode == 1 && BMR_WC_UNITAB>(P, lq, qn, pq);
     else wc_drain(P, lo, lq, qn);
   }
 #if BMR_WC_ADRAIN
-  if constexpr (kTab) wc_probe_resolve(P, pq);   // the last batch issued
+  if constexpr (kTab) wc_probe_resolve<kMode == 1 && BMR_WC_UNITAB>(P, pq);   // the last batch issued
 #endif
   wc_chunk_pads(P, lo);
 }
