@@ -1716,10 +1716,12 @@ __device__ __forceinline__ void wc_probe_issue(const Params& P, LWord* lq, uint3
   }
   cp_async_commit();
   const uint32_t rest = qn - n;
-  LWord r{0, 0, 0};
-  if (lane < rest) r = lq[n + lane];
-  __syncwarp();
-  if (lane < rest) lq[lane] = r;
+  if (rest) {   // (warp-uniform; a queue of <= 32 entries drains whole)
+    LWord r{0, 0, 0};
+    if (lane < rest) r = lq[n + lane];
+    __syncwarp();
+    if (lane < rest) lq[lane] = r;
+  }
   __syncwarp();
   qn = rest;
 }
@@ -1974,11 +1976,10 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
     // two words per iteration (the highest and the lowest start left): the same instructions per
     // word, two independent dependency chains (the loop is latency-bound), half the iterations
     for (uint32_t E = S & near; E;) {
-      const uint32_t j1 = bfind_u32(E);
-      E &= ~(1u << j1);
-      const bool two = E != 0;
-      const uint32_t j2 = two ? static_cast<uint32_t>(__ffs(E)) - 1u : j1;
-      E &= E - 1u;
+      const uint32_t j1 = bfind_u32(E);                          // highest start left
+      const uint32_t j2 = static_cast<uint32_t>(__ffs(E)) - 1u;   // lowest (== j1: one left)
+      const bool two = j2 != j1;
+      E &= (E - 1u) & ~(1u << j1);
       const uint32_t k1 = xkey(j1), k2 = xkey(j2);
       uint32_t ka1 = kb32 + 4u * ((k1 * 0x9E3779B1u) >> (32 - kCombBits));
       uint32_t ka2 = kb32 + 4u * ((k2 * 0x9E3779B1u) >> (32 - kCombBits));
