@@ -145,6 +145,9 @@ constexpr int nprod() { return W == 4 ? BMR_II_NPROD : 2; }
 #ifndef BMR_WC_UNITAB
 #define BMR_WC_UNITAB 1   // WordCount table mode: words of 6..16 symbols in one 16-byte-key table
 #endif
+#ifndef BMR_II_LAG
+#define BMR_II_LAG 2   // InvertedIndex: tiles between a stage's TMA issue and its bitmap (4 = stages - 2: C4 Map 7.72 ms; 2: 6.55 ms)
+#endif
 #ifndef BMR_WC_CLS16
 #define BMR_WC_CLS16 1   // WordCount table mode: each lane classifies its own 16 bytes only (next chunk by shuffle)
 #endif
@@ -194,7 +197,7 @@ struct Cfg {
   static constexpr int kOutHalf = (W == kSM) ? 4096 : (W == kWC) ? BMR_WC_OUT_BYTES : (W == kII) ? BMR_II_OUT_BYTES : BMR_KM_OUT_BYTES;   // bytes per output buffer
   // the producer builds the bitmap of tile it - kLag right after issuing tile it: kLag stages of
   // TMA traffic stay in flight per SM while one stage is being consumed
-  static constexpr int kLag = kStages - 2;
+  static constexpr int kLag = (W == kII) ? BMR_II_LAG : kStages - 2;
   static_assert(kStages % nprod<W>() == 0 && kLag % nprod<W>() == 0, "a producer owns every kNProd-th stage");
   // WC: per-warp queue of the window's long (hashed) words, hashed by all 32 lanes together
   // after the emission rounds (a lane-per-word hash inside the rounds diverges: with 10% long
