@@ -1967,10 +1967,12 @@ __device__ __forceinline__ void wc_window_tab(const Params& P, OutCtl* oc, uint8
     const uint32_t sb32 = smem_u32(tv.sb) + i0;
     const uint32_t kb32 = smem_u32(ctab);
     const uint32_t dmy = smem_u32(dummy) + 4u * lane;
-    const uint32_t rnb = __brev(nb);
+    // stops above byte j, bit-reversed and shifted so that the first one is the highest set bit:
+    // len = 32 - bfind(rnb1 << j)
+    const uint32_t rnb1 = __brev(nb) << 1;
     // key of the exact word starting at chunk byte j (a stop within 5 bytes after it)
     auto xkey = [&](uint32_t j) {
-      const uint32_t len = 31u - j - bfind_u32(rnb & (0x7FFFFFFFu >> j));   // first stop above j
+      const uint32_t len = 32u - bfind_u32(rnb1 << j);   // first stop above j
       const uint32_t a = sb32 + (j & ~3u);
       const uint32_t w0 = lds_u32(a), w1 = lds_u32(a + 4u);
       return exact_key30_w(__funnelshift_r(w0, w1, j << 3), __funnelshift_r(w1, w1, j << 3), len);
