@@ -2411,9 +2411,12 @@ __device__ __forceinline__ void ii_window(const Params& P, OutCtl* oc, uint8_t* 
   }
   // queue the URLs (drained lane-parallel by ii_drain)
   const uint32_t cnt = __popc(emit_mask);   // <= 2 markers start in 16 bytes
-  const uint32_t incl = warp_inclusive_add(cnt);
-  const uint32_t tot = __shfl_sync(kFull, incl, 31);
+  // the warp prefix from two ballots (cnt <= 2) instead of a 5-step shuffle scan
+  const uint32_t b1 = __ballot_sync(kFull, cnt >= 1u), b2 = __ballot_sync(kFull, cnt >= 2u);
+  const uint32_t tot = __popc(b1) + __popc(b2);
   if (tot == 0) return;
+  const uint32_t lt = lanemask_lt();
+  const uint32_t incl = __popc(b1 & lt) + __popc(b2 & lt) + cnt;
   if (qn + tot > 64) ii_drain(P, oc, outh, qn);
   uint64_t* qpos = ii_qpos(outh);
   uint32_t* qlen = reinterpret_cast<uint32_t*>(qpos + 64);
