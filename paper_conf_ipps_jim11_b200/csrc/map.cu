@@ -75,6 +75,9 @@ constexpr int kKmUnroll = BMR_KM_UNROLL;
 #define BMR_SM_SUB 4     // StringMatch 512-B windows per map-warp super-window
 #endif
 constexpr int kNMapText = 24;
+#ifndef BMR_WC_NMAP
+#define BMR_WC_NMAP 25   // WordCount map warps (24 -> 25: C5 Map 11.79 -> 11.68 ms; 28 warps x 72 registers fill the register file)
+#endif
 #ifndef BMR_II_STAGES
 #define BMR_II_STAGES 6    // InvertedIndex stages in flight per SM (round 2: 4 -> 6 with 8 KB output
                            // buffers, C4 Map 7.81 -> 7.66 ms)
@@ -93,7 +96,7 @@ constexpr int kNMapText = 24;
 #define BMR_II_NMAP 24   // InvertedIndex map warps
 #endif
 template <int W>
-constexpr int nmap() { return W == 3 ? kNMap : W == 2 ? BMR_SM_NMAP : W == 4 ? BMR_II_NMAP : kNMapText; }
+constexpr int nmap() { return W == 3 ? kNMap : W == 2 ? BMR_SM_NMAP : W == 4 ? BMR_II_NMAP : BMR_WC_NMAP; }
 // Producer warps kProdWarp0 .. + kNProd - 1: producer p owns the iterations it == p (mod kNProd)
 // (and so the stages s == p (mod kNProd)); one warp alone is latency-bound at ~465 instructions
 // per tile (TMA issue + bitmap), slower than HBM delivers a tile (ncu, C2 round 1).
@@ -630,8 +633,8 @@ __device__ __forceinline__ uint32_t units(uint32_t c) {   // buffer space of pac
   else return cur_ca(c);
 }
 // WC: a reservation carries <= kWin / 2 + 1 exact entries (ca) and <= kHashQ queued ones (cb)
-static_assert(PairFmt<kWC>::kCap + kNMapText * (kWin / 2 + 1) <= kCaMask, "ca field overflow");
-static_assert(PairFmt<kWC>::kCap / 4 + kNMapText * Cfg<kWC>::kHashQ <= kCbMask, "cb field overflow");
+static_assert(PairFmt<kWC>::kCap + nmap<kWC>() * (kWin / 2 + 1) <= kCaMask, "ca field overflow");
+static_assert(PairFmt<kWC>::kCap / 4 + nmap<kWC>() * Cfg<kWC>::kHashQ <= kCbMask, "cb field overflow");
 static_assert(PairFmt<kSM>::kCap + kNMapText * PairFmt<kSM>::kMaxReserve <= kCaMask, "ca field overflow");
 static_assert(PairFmt<kII>::kCap + kNMapText * PairFmt<kII>::kMaxReserve <= kCaMask, "ca field overflow");
 
