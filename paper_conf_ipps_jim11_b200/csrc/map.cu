@@ -6,11 +6,12 @@
 // stage-in / compute / stage-out, software wait-signal flags, yield by dummy global reads) are
 // prior art; the B200 re-derivation here (one persistent CTA per SM):
 //   * two producer warps (A1/A2): an elected lane issues TMA bulk copies (cp.async.bulk) of the
-//     tile bytes and of the tile's record-offset slice into an SMEM ring (4 stages; StringMatch
-//     12 stages of bytes only) guarded by mbarrier full/empty pairs; kLag tiles later the
+//     tile bytes and of the tile's record-offset slice into an SMEM ring (WordCount 4 stages,
+//     InvertedIndex 6, KMeans 8, StringMatch 12 of bytes only) guarded by mbarrier full/empty
+//     pairs; WordCount / InvertedIndex take tiles from a global counter; kLag tiles later the
 //     producer turns the staged offsets into a record-start bitmap and releases the stage
 //     (ready mbarrier) — replaces the barrier-separated staging loop (L68, L85);
-//   * map warps (A3; 24 for the text workloads, 16 for KMeans): byte-parallel, record-agnostic
+//   * map warps (A3; 24 for StringMatch / InvertedIndex, 25 for WordCount, 16 for KMeans): byte-parallel, record-agnostic
 //     scanning — each lane owns a 16-byte chunk of a 512-B window, record boundaries come from
 //     the bitmap; no map-warp barrier at all, so the per-record imbalance the paper blames for
 //     SO overhead (L273) disappears;
